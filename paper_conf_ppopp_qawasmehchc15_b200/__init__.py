@@ -1,0 +1,313 @@
+"""B200-native seismic modeling and RTM hot path (Qawasmeh et al., PMAM'15).
+
+Thin ctypes binding over the C ABI in ``include/seis.h`` (``libseis.so``, built
+in-tree for sm_100a by ``build.py``).  Argument marshalling only: every step of
+the path runs in the library's CUDA kernels.  There is no CPU fallback: if
+the library or a CUDA device is missing the calls raise.
+
+torch is used only for device memory (tensors whose ``data_ptr()`` is passed),
+streams (``torch.cuda.current_stream().cuda_stream``) and process groups (the
+NCCL unique id broadcast in ``Comm.from_torch_distributed``).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+from dataclasses import dataclass
+from typing import Optional
+
+import numpy as np
+
+__all__ = ["Grid", "Shot", "Model", "Comm", "SeisError", "lib", "slab_bounds", "ISO", "ACOUSTIC",
+           "ELASTIC", "KINDS"]
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIBPATH = os.path.join(_HERE, "libseis.so")
+
+ISO, ACOUSTIC, ELASTIC = 0, 1, 2
+KINDS = {"iso": ISO, "acoustic": ACOUSTIC, "elastic": ELASTIC}
+STATUS = {0: "SEIS_OK", 1: "SEIS_EINVAL", 2: "SEIS_ECFL", 3: "SEIS_ENOMEM", 4: "SEIS_ECUDA",
+          5: "SEIS_ENCCL", 6: "SEIS_EUNSUPPORTED"}
+
+# every symbol include/seis.h declares
+SYMBOLS = ["seis_comm_unique_id", "seis_comm_create", "seis_comm_destroy", "seis_model_create",
+           "seis_slab_bounds", "seis_model_slab", "seis_model_destroy", "seis_forward_model",
+           "seis_migrate", "seis_get_field", "seis_memory_required", "seis_profile",
+           "seis_profile_read", "seis_last_launch_count",
+           "seis_version", "seis_last_error"]
+
+
+class SeisError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        self.status = status
+        self.name = STATUS.get(status, str(status))
+        super().__init__(f"{self.name}: {msg}")
+
+
+class _CGrid(C.Structure):
+    _fields_ = [("nx", C.c_int32), ("ny", C.c_int32), ("nz", C.c_int32), ("h", C.c_float),
+                ("dt", C.c_float), ("nb", C.c_int32), ("free_surface", C.c_int32),
+                ("pml_R", C.c_float), ("pml_f", C.c_float), ("slabs", C.c_int32)]
+
+
+class _CShot(C.Structure):
+    _fields_ = [("sx", C.c_int32), ("sy", C.c_int32), ("sz", C.c_int32),
+                ("wavelet", C.POINTER(C.c_float)), ("nt", C.c_int32), ("nrec", C.c_int32),
+                ("rec", C.POINTER(C.c_int32)), ("rec_component", C.c_int32),
+                ("snap_period", C.c_int32)]
+
+
+_lib = None
+
+
+def lib():
+    """Load libseis.so (raises if it was not built: there is no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(_LIBPATH):
+            raise RuntimeError(f"{_LIBPATH} is missing: run `python -m "
+                               "paper_conf_ppopp_qawasmehchc15_b200.build` (no CPU fallback)")
+        L = C.CDLL(_LIBPATH)
+        vp = C.c_void_p
+        L.seis_comm_unique_id.argtypes = [C.POINTER(C.c_uint8)]
+        L.seis_comm_create.argtypes = [C.c_int32, C.c_int32, C.POINTER(C.c_uint8), C.c_int32,
+                                       C.POINTER(vp)]
+        L.seis_comm_destroy.argtypes = [vp]
+        L.seis_model_create.argtypes = [C.POINTER(_CGrid), C.c_int, vp, vp, vp, vp, C.c_int32,
+                                        C.POINTER(vp)]
+        L.seis_slab_bounds.argtypes = [C.c_int32, C.c_int32, C.c_int32, C.POINTER(C.c_int32),
+                                       C.POINTER(C.c_int32)]
+        L.seis_model_slab.argtypes = [vp, C.POINTER(C.c_int32), C.POINTER(C.c_int32)]
+        L.seis_model_destroy.argtypes = [vp]
+        L.seis_forward_model.argtypes = [vp, C.POINTER(_CShot), vp, vp]
+        L.seis_migrate.argtypes = [vp, C.POINTER(_CShot), vp, vp, vp]
+        L.seis_get_field.argtypes = [vp, C.c_int32, vp, vp]
+        L.seis_memory_required.argtypes = [C.POINTER(_CGrid), C.c_int, C.POINTER(_CShot),
+                                           C.c_int32, C.POINTER(C.c_uint64)]
+        L.seis_profile.argtypes = [C.c_int32]
+        L.seis_profile_read.argtypes = [C.c_int32, C.POINTER(C.c_double), C.POINTER(C.c_int64)]
+        L.seis_last_launch_count.restype = C.c_int64
+        L.seis_version.restype = C.c_char_p
+        L.seis_last_error.restype = C.c_char_p
+        for name in SYMBOLS:
+            if name not in ("seis_last_launch_count", "seis_version", "seis_last_error"):
+                getattr(L, name).restype = C.c_int
+        _lib = L
+    return _lib
+
+
+def _check(rc: int):
+    if rc != 0:
+        raise SeisError(rc, lib().seis_last_error().decode(errors="replace"))
+
+
+@dataclass
+class Grid:
+    nx: int
+    ny: int
+    nz: int
+    h: float
+    dt: float
+    nb: int = 0
+    free_surface: int = 0
+    pml_R: float = 1e-3
+    pml_f: float = 10.0
+    slabs: int = 1
+
+    def c(self) -> _CGrid:
+        return _CGrid(self.nx, self.ny, self.nz, self.h, self.dt, self.nb, self.free_surface,
+                      self.pml_R, self.pml_f, self.slabs)
+
+
+@dataclass
+class Shot:
+    src: tuple
+    wavelet: np.ndarray          # host fp32 [nt] (injected samples s[n], O11)
+    rec: np.ndarray              # host int32 [nrec][3] (x, y, z)
+    rec_component: int = 2
+    snap_period: int = 1
+
+    def c(self):
+        w = np.ascontiguousarray(self.wavelet, dtype=np.float32)
+        r = np.ascontiguousarray(np.asarray(self.rec, dtype=np.int32).reshape(-1, 3))
+        cs = _CShot(int(self.src[0]), int(self.src[1]), int(self.src[2]),
+                    w.ctypes.data_as(C.POINTER(C.c_float)), w.shape[0], r.shape[0],
+                    r.ctypes.data_as(C.POINTER(C.c_int32)), self.rec_component, self.snap_period)
+        return cs, (w, r)
+
+    @property
+    def nt(self):
+        return int(np.asarray(self.wavelet).shape[0])
+
+    @property
+    def nrec(self):
+        return int(np.asarray(self.rec).reshape(-1, 3).shape[0])
+
+
+def _ptr(a):
+    """Raw pointer of a torch tensor (device or host) or numpy array (host)."""
+    if a is None:
+        return None
+    if isinstance(a, np.ndarray):
+        assert a.flags.c_contiguous and a.dtype == np.float32, "need C-contiguous float32"
+        return a.ctypes.data
+    assert a.is_contiguous() and str(a.dtype) == "torch.float32", "need contiguous float32"
+    return a.data_ptr()
+
+
+def _stream(stream):
+    if stream is None:
+        try:
+            import torch
+
+            if torch.cuda.is_available():
+                return torch.cuda.current_stream().cuda_stream
+        except Exception:
+            pass
+        return None
+    if isinstance(stream, int):
+        return stream
+    return stream.cuda_stream
+
+
+def slab_bounds(nz: int, nranks: int, rank: int):
+    z0, n = C.c_int32(), C.c_int32()
+    _check(lib().seis_slab_bounds(nz, nranks, rank, C.byref(z0), C.byref(n)))
+    return z0.value, n.value
+
+
+class Comm:
+    """NCCL communicator for the z-slab decomposition (one process per GPU)."""
+
+    def __init__(self, nranks: int, rank: int, uid: bytes, device: int):
+        buf = (C.c_uint8 * 128).from_buffer_copy(uid)
+        h = C.c_void_p()
+        _check(lib().seis_comm_create(nranks, rank, buf, device, C.byref(h)))
+        self.h, self.nranks, self.rank, self.device = h, nranks, rank, device
+
+    @staticmethod
+    def unique_id() -> bytes:
+        buf = (C.c_uint8 * 128)()
+        _check(lib().seis_comm_unique_id(buf))
+        return bytes(buf)
+
+    @classmethod
+    def from_torch_distributed(cls, device: int):
+        """Create from an initialised torch.distributed group (broadcasts the NCCL id)."""
+        import torch
+        import torch.distributed as dist
+
+        rank, world = dist.get_rank(), dist.get_world_size()
+        uid = cls.unique_id() if rank == 0 else bytes(128)
+        t = torch.tensor(list(uid), dtype=torch.uint8,
+                         device=f"cuda:{device}" if dist.get_backend() == "nccl" else "cpu")
+        dist.broadcast(t, 0)
+        return cls(world, rank, bytes(t.cpu().tolist()), device)
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().seis_comm_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class Model:
+    """A velocity model resident on one GPU (this process's z-slab)."""
+
+    def __init__(self, grid: Grid, kind, vp, vs=None, rho=None, comm: Optional[Comm] = None,
+                 device: int = 0):
+        self.grid = grid
+        self.kind = KINDS[kind] if isinstance(kind, str) else int(kind)
+        arrs = [None if a is None else np.ascontiguousarray(a, dtype=np.float32)
+                for a in (vp, vs, rho)]
+        g = grid.c()
+        h = C.c_void_p()
+        _check(lib().seis_model_create(C.byref(g), self.kind, *[_ptr(a) for a in arrs],
+                                       comm.h if comm is not None else None, device, C.byref(h)))
+        self.h = h
+        self.device = device
+        self.comm = comm
+        z0, n = C.c_int32(), C.c_int32()
+        _check(lib().seis_model_slab(h, C.byref(z0), C.byref(n)))
+        self.z0, self.nz_local = z0.value, n.value
+
+    @property
+    def local_shape(self):
+        return (self.nz_local, self.grid.ny, self.grid.nx)
+
+    def forward_model(self, shot: Shot, seis=None, stream=None):
+        """Seismic modeling of one shot; returns seis [nt][nrec] (the given buffer, or a new
+        device tensor)."""
+        if seis is None:
+            import torch
+
+            seis = torch.empty((shot.nt, shot.nrec), dtype=torch.float32,
+                               device=f"cuda:{self.device}")
+        cs, keep = shot.c()
+        _check(lib().seis_forward_model(self.h, C.byref(cs), _ptr(seis), _stream(stream)))
+        return seis
+
+    def migrate(self, shot: Shot, data, image, stream=None):
+        """RTM of one shot; image [nz_local][ny][nx] is accumulated (+=)."""
+        cs, keep = shot.c()
+        _check(lib().seis_migrate(self.h, C.byref(cs), _ptr(data), _ptr(image), _stream(stream)))
+        return image
+
+    def get_field(self, which: int, out=None, stream=None):
+        if out is None:
+            out = np.empty(self.local_shape, dtype=np.float32)
+        _check(lib().seis_get_field(self.h, which, _ptr(out), _stream(stream)))
+        return out
+
+    @staticmethod
+    def launches() -> int:
+        return int(lib().seis_last_launch_count())
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib().seis_model_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+KERNEL_IDS = {"iso_step": 0, "ac_v": 1, "ac_p": 2, "el_v": 3, "el_s": 4, "inject": 5,
+              "gather": 6, "exchange": 7, "fs_mirror": 8}
+
+
+def profile(enable: bool):
+    """Start (resetting the counters) / stop per-kernel CUDA-event timing in the library."""
+    _check(lib().seis_profile(1 if enable else 0))
+
+
+def profile_read():
+    """{kernel: (total_ms, launches)} for every kernel id with launches since profile(True)."""
+    out = {}
+    for name, k in KERNEL_IDS.items():
+        ms, n = C.c_double(), C.c_int64()
+        _check(lib().seis_profile_read(k, C.byref(ms), C.byref(n)))
+        if n.value:
+            out[name] = (ms.value, n.value)
+    return out
+
+
+def memory_required(grid: Grid, kind, shot: Optional[Shot] = None, nranks: int = 1) -> int:
+    g = grid.c()
+    out = C.c_uint64()
+    if shot is not None:
+        cs, keep = shot.c()
+        _check(lib().seis_memory_required(C.byref(g), KINDS.get(kind, kind), C.byref(cs), nranks,
+                                          C.byref(out)))
+    else:
+        _check(lib().seis_memory_required(C.byref(g), KINDS.get(kind, kind), None, nranks,
+                                          C.byref(out)))
+    return out.value

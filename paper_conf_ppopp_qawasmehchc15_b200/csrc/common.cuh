@@ -1,0 +1,80 @@
+// common.cuh — layout, indexing and coefficients shared by the sm_100a kernels.
+//
+// Product path only (never includes or calls oracle/).  Paper: Qawasmeh et al.,
+// PMAM'15; "P:<line>" cites /root/reference/PAPER.md, O1..O19 the readings in
+// DESIGN.md §3.
+//
+// HBM layout.  Every state field and per-point coefficient of a
+// z-slab is one fp32 array with G = 4 zero ghost cells on each side of every axis
+// ("Ghost node thickness is determined by the stencil"):
+//   padded dims  PX = roundup(roundup(nx, 32) + 2G, 32),  PY = roundup(ny, TY) + 2G,
+//                PZ = nz_local + 2G,  plane stride PS = PX * PY
+//   element (i, j, k) of the slab (interior coordinates) lives at
+//                ((k + G) * PY + (j + G)) * PX + (i + G)
+// The base pointer of each array is offset so that x = 0 of every row is
+// 128-byte aligned (PX is a multiple of 32 floats).  Ghosts are never written, so
+// "values outside the grid are 0" (O1) costs no branch; the 4 z-ghost planes on a
+// slab face that touches a neighbour slab are the halo planes the exchange fills.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace seis {
+
+constexpr int G = 4;     // ghost width = stencil half-width (radius 4)
+constexpr int TXW = 32;  // tile width in x = one warp
+
+struct Dims {
+  int nx, ny, nzl;  // interior points of the slab
+  int nz;           // global nz
+  int z0;           // global z of local k = 0
+  int PX, PY;       // padded pitches
+  long long PS;     // plane stride
+  __host__ __device__ __forceinline__ long long at(int i, int j, int k) const {
+    return ((long long)(k + G) * PY + (j + G)) * PX + (i + G);
+  }
+};
+
+// 8th-order coefficients (O1): fp32 roundings of the exact rationals
+//   centred 2nd derivative c = [-205/72, 8/5, -1/5, 8/315, -1/560]
+//   staggered 1st derivative d = [1225/1024, -245/3072, 49/5120, -5/7168]
+// (each is a correctly rounded fp32 quotient of two exact fp32 integers).
+#define SEIS_C0 (-205.0f / 72.0f)
+#define SEIS_C1 (8.0f / 5.0f)
+#define SEIS_C2 (-1.0f / 5.0f)
+#define SEIS_C3 (8.0f / 315.0f)
+#define SEIS_C4 (-1.0f / 560.0f)
+#define SEIS_D1 (1225.0f / 1024.0f)
+#define SEIS_D2 (-245.0f / 3072.0f)
+#define SEIS_D3 (49.0f / 5120.0f)
+#define SEIS_D4 (-5.0f / 7168.0f)
+
+// Cooperative load of one plane tile of a padded field into shared memory:
+// (BY + 2HY) rows x (32 + 2HX) columns starting at (i0 - HX, j0 - HY).
+template <int BY, int HX, int HY>
+__device__ __forceinline__ void load_tile(float* __restrict__ s, const float* __restrict__ f,
+                                          long long o /* padded index of (i0, j0, k) */, int PX) {
+  constexpr int W = TXW + 2 * HX;
+  constexpr int H = BY + 2 * HY;
+  constexpr int N = W * H;
+  const int tid = threadIdx.y * TXW + threadIdx.x;
+#pragma unroll
+  for (int t = tid; t < N; t += TXW * BY) {
+    const int r = t / W;
+    const int c = t - r * W;
+    s[t] = __ldg(f + o + (long long)(r - HY) * PX + (c - HX));
+  }
+}
+
+// Compact C-PML memory-variable slabs (O7): psi is stored only where the
+// layer can be non-zero.  W = nb + 1 points per face (the half-node layer on the
+// high face is one point wider than the integer-node one).
+struct CpmlIdx {
+  int W;
+  __device__ __forceinline__ static bool in(int i, int n, int W, bool lo) {
+    return (lo && i < W) || i >= n - W;
+  }
+  __device__ __forceinline__ static int slot(int i, int n, int W) { return i < W ? i : i - (n - 2 * W); }
+};
+
+}  // namespace seis

@@ -1,0 +1,72 @@
+// kernels_aux.cuh — receiver sampling, receiver injection (P:206,
+// P:330) and small helpers.
+//
+// Receiver injection is ONE launch per step over all receivers (the paper's
+// per-receiver launches took 26.2% of GPU time; its suggested fix).
+// Duplicate receiver positions are merged on the host into groups (CSR): each
+// distinct node is updated by exactly one thread, summing its receivers'
+// samples in receiver-index order (O12), so there are no atomics and no races.
+#pragma once
+#include "common.cuh"
+
+namespace seis {
+
+// seis_row[r] = f[off[r]] for the receivers this slab owns (off[r] >= 0).
+// Elastic pressure (component 3): -(f0 + f1 + f2)/3 at the node.
+__global__ void gather_kernel(float* __restrict__ seis_row, const float* __restrict__ f0,
+                              const float* __restrict__ f1, const float* __restrict__ f2,
+                              const long long* __restrict__ off, const int* __restrict__ rid, int n,
+                              int pressure) {
+  const int t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= n) return;
+  const long long o = off[t];
+  float v;
+  if (pressure) {
+    v = -(f0[o] + f1[o] + f2[o]) / 3.0f;
+  } else {
+    v = f0[o];
+  }
+  seis_row[rid[t]] = v;
+}
+
+// Backward-phase receiver injection (O15): for each distinct node u of this slab,
+//   f[off[u]] += scale[u] * sum_{r in group u, index order} data_row[r]
+// (ELASTIC is not migrated in this version.)
+__global__ void inject_kernel(float* __restrict__ f, const long long* __restrict__ off,
+                              const float* __restrict__ scale, const int* __restrict__ gstart,
+                              const int* __restrict__ members, const float* __restrict__ data_row,
+                              int ngroups) {
+  const int u = blockIdx.x * blockDim.x + threadIdx.x;
+  if (u >= ngroups) return;
+  float s = 0.0f;
+  for (int t = gstart[u]; t < gstart[u + 1]; ++t) s += data_row[members[t]];
+  f[off[u]] = fmaf(scale[u], s, f[off[u]]);
+}
+
+// Copy the interior of a padded slab field to a compact [nzl][ny][nx] array.
+__global__ void unpad_kernel(float* __restrict__ dst, const float* __restrict__ src, Dims d) {
+  const long long n = (long long)d.nzl * d.ny * d.nx;
+  for (long long t = blockIdx.x * (long long)blockDim.x + threadIdx.x; t < n;
+       t += (long long)gridDim.x * blockDim.x) {
+    const int i = (int)(t % d.nx);
+    const long long r = t / d.nx;
+    const int j = (int)(r % d.ny);
+    const int k = (int)(r / d.ny);
+    dst[t] = src[d.at(i, j, k)];
+  }
+}
+
+// Scatter a compact [nzl][ny][nx] fp32 array into the interior of a padded array.
+__global__ void pad_kernel(float* __restrict__ dst, const float* __restrict__ src, Dims d) {
+  const long long n = (long long)d.nzl * d.ny * d.nx;
+  for (long long t = blockIdx.x * (long long)blockDim.x + threadIdx.x; t < n;
+       t += (long long)gridDim.x * blockDim.x) {
+    const int i = (int)(t % d.nx);
+    const long long r = t / d.nx;
+    const int j = (int)(r % d.ny);
+    const int k = (int)(r / d.ny);
+    dst[d.at(i, j, k)] = src[t];
+  }
+}
+
+}  // namespace seis

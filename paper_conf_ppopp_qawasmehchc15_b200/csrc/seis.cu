@@ -1,0 +1,1245 @@
+// seis.cu — runtime + C ABI (include/seis.h) of the B200-native hot path.
+//
+// Product path only: no oracle code, no CPU fallback.  The runtime owns the
+// device memory plan (padded z-slab fields, per-point coefficients, compact
+// C-PML slabs, the HBM snapshot pool), drives Algorithm 1 on the
+// caller's stream, and exchanges the 4 ghost planes between z-slabs:
+// cudaMemcpyAsync between slabs of one process, NCCL send/recv between ranks.
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <string>
+#include <vector>
+
+#include "../../include/seis.h"
+#include "common.cuh"
+#include "kernels_acoustic.cuh"
+#include "kernels_aux.cuh"
+#include "kernels_elastic.cuh"
+#include "kernels_iso.cuh"
+
+using namespace seis;
+
+// ------------------------------------------------------------------ errors
+static thread_local std::string g_err;
+static thread_local long long g_launches = 0;
+
+static seis_status fail(seis_status st, const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return st;
+}
+
+#define CK(call)                                                                          \
+  do {                                                                                    \
+    cudaError_t e_ = (call);                                                              \
+    if (e_ != cudaSuccess)                                                                \
+      return fail(e_ == cudaErrorMemoryAllocation ? SEIS_ENOMEM : SEIS_ECUDA, "%s: %s (%s:%d)", \
+                  #call, cudaGetErrorString(e_), __FILE__, __LINE__);                     \
+  } while (0)
+#define CKL()                                                                             \
+  do {                                                                                    \
+    ++g_launches;                                                                         \
+    cudaError_t e_ = cudaGetLastError();                                                  \
+    if (e_ != cudaSuccess)                                                                \
+      return fail(SEIS_ECUDA, "kernel launch: %s (%s:%d)", cudaGetErrorString(e_), __FILE__, \
+                  __LINE__);                                                              \
+  } while (0)
+#define NK(call)                                                                          \
+  do {                                                                                    \
+    ncclResult_t r_ = (call);                                                             \
+    if (r_ != ncclSuccess)                                                                \
+      return fail(SEIS_ENCCL, "%s: %s (%s:%d)", #call, ncclGetErrorString(r_), __FILE__, __LINE__); \
+  } while (0)
+#define TRY(expr)                      \
+  do {                                 \
+    seis_status s_ = (expr);           \
+    if (s_ != SEIS_OK) return s_;      \
+  } while (0)
+
+// ------------------------------------------------------------ profiling
+// Per-kernel CUDA-event timing (seis_profile / seis_profile_read): an event pair
+// recorded on the launching stream around every launch of a stencil / aux kernel.
+namespace prof {
+constexpr int NK = 9;
+static bool on = false;
+static std::vector<cudaEvent_t> ev[NK];  // start, stop, start, stop, ...
+static size_t used[NK] = {};
+static cudaEvent_t get(int k) {
+  if (used[k] == ev[k].size()) {
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    ev[k].push_back(e);
+  }
+  return ev[k][used[k]++];
+}
+struct Scope {
+  int k;
+  cudaStream_t st;
+  Scope(int k_, cudaStream_t s) : k(k_), st(s) {
+    if (on) cudaEventRecord(get(k), st);
+  }
+  ~Scope() {
+    if (on) cudaEventRecord(get(k), st);
+  }
+};
+}  // namespace prof
+#define PROF(id, st) prof::Scope prof_scope_(id, st)
+
+// ------------------------------------------------------------------ types
+struct seis_comm {
+  ncclComm_t nccl = nullptr;
+  int nranks = 1, rank = 0, device = 0;
+};
+
+namespace {
+
+constexpr int BY = 16;       // tile rows (block = 32 x BY threads)
+constexpr int NPSI = 18;
+
+struct Slab {
+  Dims d{};
+  std::vector<float*> fld;   // padded state fields
+  float* m = nullptr;        // ISO
+  float* kdt = nullptr;      // ACOUSTIC
+  float *bx = nullptr, *by = nullptr, *bz = nullptr;                          // ACOUSTIC, ELASTIC
+  float *l2m = nullptr, *lam = nullptr, *mxy = nullptr, *mxz = nullptr, *myz = nullptr;  // ELASTIC
+  float* psi[NPSI] = {};
+  int cur = 0;               // ISO: fld[cur] = u^n
+  int zc = 1, nzch = 1;      // z-chunking of the stencil launches
+  // shot tables
+  long long src_o = -1;
+  float src_scale = 0.f;
+  int nrec_own = 0;
+  long long* d_rec_off = nullptr;
+  int* d_rec_id = nullptr;
+  int ngroups = 0;
+  long long* d_g_off = nullptr;
+  float* d_g_scale = nullptr;
+  int* d_g_start = nullptr;
+  int* d_g_mem = nullptr;
+  float* snap = nullptr;     // nsnap * nzl*ny*nx (points into the model's pool)
+};
+
+template <class T>
+cudaError_t dmalloc(T** p, size_t n) {
+  return cudaMalloc((void**)p, std::max<size_t>(n, 1) * sizeof(T));
+}
+
+}  // namespace
+
+struct seis_model {
+  seis_grid g{};
+  seis_kind kind = SEIS_ISO;
+  int device = 0;
+  seis_comm* comm = nullptr;
+  int rank = 0, nranks = 1;
+  int pz0 = 0, pnzl = 0;       // this process's z-range
+  double vmax = 0.0;           // global max vp
+  std::vector<Slab> slabs;
+  std::vector<void*> allocs;   // every cudaMalloc of the model
+  // 1D coefficient arrays (global index)
+  float *edx = nullptr, *edy = nullptr, *edz = nullptr;      // ISO eta*dt
+  CpmlAxis cp[3] = {};                                       // C-PML
+  int W = 0;                   // C-PML slab width per face
+  // host copies of this process's model slab (point scales for sources/receivers)
+  std::vector<float> hvp, hvs, hrho;
+  std::vector<double> eta1[3];  // ISO eta per axis (double, host)
+  // snapshot pool
+  float* pool = nullptr;
+  size_t pool_elems = 0;
+  // staging buffers
+  float* stage = nullptr;
+  size_t stage_elems = 0;
+  const float* hwav = nullptr;  // host wavelet of the current call
+  int last_nt = 0;
+};
+
+namespace {
+
+// ------------------------------------------------------------ helpers
+seis_status alloc_track(seis_model* M, void** p, size_t bytes) {
+  cudaError_t e = cudaMalloc(p, std::max<size_t>(bytes, 4));
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(SEIS_ENOMEM, "cudaMalloc(%zu bytes): %s", bytes, cudaGetErrorString(e));
+  }
+  M->allocs.push_back(*p);
+  return SEIS_OK;
+}
+
+// Padded field: ghosts zero, x = 0 of each row 128-byte aligned.
+seis_status alloc_padded(seis_model* M, const Dims& d, float** out, cudaStream_t st) {
+  size_t elems = (size_t)d.PS * (size_t)(d.nzl + 2 * G);
+  void* base = nullptr;
+  TRY(alloc_track(M, &base, elems * sizeof(float) + 128));
+  CK(cudaMemsetAsync(base, 0, elems * sizeof(float) + 128, st));
+  *out = (float*)((char*)base + 112);  // (base + 112 + 4*G) % 128 == 0
+  return SEIS_OK;
+}
+
+int roundup(int a, int b) { return (a + b - 1) / b * b; }
+
+Dims make_dims(const seis_grid& g, int z0, int nzl) {
+  Dims d;
+  d.nx = g.nx;
+  d.ny = g.ny;
+  d.nzl = nzl;
+  d.nz = g.nz;
+  d.z0 = z0;
+  d.PX = roundup(roundup(g.nx, TXW) + 2 * G, 32);
+  d.PY = roundup(g.ny, BY) + 2 * G;
+  d.PS = (long long)d.PX * d.PY;
+  return d;
+}
+
+bool is_device_ptr(const void* p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+// Courant bounds of the 8th-order schemes in 3D (O5):
+//   ISO leapfrog: v dt/h <= 2/sqrt(3 * sum|c|),  sum|c| over one axis = |c0| + 2 sum|c_m|
+//   staggered:    v dt/h <= 1/(sqrt(3) * sum|d_m|)
+double courant_limit(seis_kind k) {
+  const double c[5] = {205.0 / 72.0, 8.0 / 5.0, 1.0 / 5.0, 8.0 / 315.0, 1.0 / 560.0};
+  const double d[4] = {1225.0 / 1024.0, 245.0 / 3072.0, 49.0 / 5120.0, 5.0 / 7168.0};
+  if (k == SEIS_ISO) {
+    // max of -symbol at k h = pi per axis: c0 + 2 sum c_m cos(m pi) -> |c0| + 2 sum |c_m| (alternating)
+    double s = c[0] + 2.0 * (c[1] + c[2] + c[3] + c[4]);
+    return 2.0 / std::sqrt(3.0 * s);
+  }
+  return 1.0 / (std::sqrt(3.0) * (d[0] + d[1] + d[2] + d[3]));
+}
+
+// O6: eta_d(xi) = eta_max xi^2, eta_max = 3 vmax ln(1/R) / (2 nb h), xi = layer depth / nb.
+double layer_xi(double x, int N, int nb, bool lo, bool hi) {
+  double xi = 0.0;
+  if (lo && nb - x > xi) xi = nb - x;
+  if (hi && x - (N - 1 - nb) > xi) xi = x - (N - 1 - nb);
+  xi /= (double)nb;
+  return xi > 1.0 ? 1.0 : xi;
+}
+
+// O7 (K&M 2007, kappa = 1): d = d0 xi^2, alpha = pi f (1 - xi), b = exp(-(d+alpha) dt),
+// a = d (b - 1)/(d + alpha) (0 where d = 0).
+void cpml_coef(double xi, double d0, double f, double dt, float* a, float* b) {
+  double dd = d0 * xi * xi;
+  double al = M_PI * f * (1.0 - xi);
+  double bb = std::exp(-(dd + al) * dt);
+  *b = (float)bb;
+  *a = (float)(dd > 0.0 ? dd * (bb - 1.0) / (dd + al) : 0.0);
+}
+
+seis_status upload_padded_from_host(seis_model* M, const Dims& d, const std::vector<float>& host,
+                                    float** out, cudaStream_t st) {
+  TRY(alloc_padded(M, d, out, st));
+  size_t n = (size_t)d.nzl * d.ny * d.nx;
+  float* tmp = nullptr;
+  CK(cudaMalloc(&tmp, n * sizeof(float)));
+  CK(cudaMemcpyAsync(tmp, host.data(), n * sizeof(float), cudaMemcpyHostToDevice, st));
+  pad_kernel<<<1024, 256, 0, st>>>(*out, tmp, d);
+  CKL();
+  CK(cudaStreamSynchronize(st));
+  CK(cudaFree(tmp));
+  return SEIS_OK;
+}
+
+// Choose the z-chunk so the launch fills the machine in whole waves.
+void choose_chunks(Slab& s, int resident_per_sm, int nsm) {
+  const int bxy = ((s.d.nx + TXW - 1) / TXW) * ((s.d.ny + BY - 1) / BY);
+  const long long slots = (long long)std::max(1, resident_per_sm) * nsm;
+  double best = 1e300;
+  int bestc = 1;
+  for (int c = 1; c <= 64 && c <= s.d.nzl; ++c) {
+    const int zc = (s.d.nzl + c - 1) / c;
+    const long long blocks = (long long)bxy * c;
+    const long long waves = (blocks + slots - 1) / slots;
+    const double t = (double)waves * (zc + 8);  // 8 warm-up planes per chunk
+    if (t < best - 1e-9) {
+      best = t;
+      bestc = c;
+    }
+  }
+  s.nzch = bestc;
+  s.zc = (s.d.nzl + bestc - 1) / bestc;
+  s.nzch = (s.d.nzl + s.zc - 1) / s.zc;
+}
+
+int nfields(seis_kind k) { return k == SEIS_ISO ? 2 : (k == SEIS_ACOUSTIC ? 4 : 9); }
+
+// Ghost-plane exchange of `fields` between the slabs of this process and, with a
+// communicator, with the neighbouring ranks (4 contiguous planes per face).
+seis_status exchange(seis_model* M, const std::vector<int>& fields, cudaStream_t st,
+                     const std::vector<int>* iso_cur = nullptr) {
+  if (M->slabs.size() < 2 && !(M->comm && M->nranks > 1)) return SEIS_OK;
+  PROF(7, st);
+  const size_t plane4 = 0;
+  (void)plane4;
+  for (size_t s = 0; s + 1 < M->slabs.size(); ++s) {
+    Slab& A = M->slabs[s];
+    Slab& B = M->slabs[s + 1];
+    const size_t n4 = (size_t)4 * A.d.PS;
+    for (int f : fields) {
+      float* fa = A.fld[f];
+      float* fb = B.fld[f];
+      // A's bottom ghosts (k = nzl .. nzl+3) <- B's planes 0..3
+      CK(cudaMemcpyAsync(fa + (size_t)(A.d.nzl + G) * A.d.PS, fb + (size_t)G * B.d.PS,
+                         n4 * sizeof(float), cudaMemcpyDeviceToDevice, st));
+      // B's top ghosts (k = -4 .. -1) <- A's planes nzl-4 .. nzl-1
+      CK(cudaMemcpyAsync(fb, fa + (size_t)(A.d.nzl) * A.d.PS, n4 * sizeof(float),
+                         cudaMemcpyDeviceToDevice, st));
+    }
+  }
+  if (M->comm && M->nranks > 1) {
+    Slab& top = M->slabs.front();
+    Slab& bot = M->slabs.back();
+    const size_t n4 = (size_t)4 * top.d.PS;
+    NK(ncclGroupStart());
+    for (int f : fields) {
+      if (M->rank > 0) {
+        NK(ncclSend(top.fld[f] + (size_t)G * top.d.PS, n4, ncclFloat, M->rank - 1, M->comm->nccl, st));
+        NK(ncclRecv(top.fld[f], n4, ncclFloat, M->rank - 1, M->comm->nccl, st));
+      }
+      if (M->rank < M->nranks - 1) {
+        NK(ncclSend(bot.fld[f] + (size_t)bot.d.nzl * bot.d.PS, n4, ncclFloat, M->rank + 1,
+                    M->comm->nccl, st));
+        NK(ncclRecv(bot.fld[f] + (size_t)(bot.d.nzl + G) * bot.d.PS, n4, ncclFloat, M->rank + 1,
+                    M->comm->nccl, st));
+      }
+    }
+    NK(ncclGroupEnd());
+  }
+  (void)iso_cur;
+  return SEIS_OK;
+}
+
+}  // namespace
+
+// ================================================================== C ABI
+extern "C" {
+
+const char* seis_version(void) { return "seis-b200 0.1 (sm_100a)"; }
+
+seis_status seis_profile(int32_t enable) {
+  if (enable) {
+    for (int k = 0; k < prof::NK; ++k) prof::used[k] = 0;
+  }
+  prof::on = enable != 0;
+  return SEIS_OK;
+}
+
+seis_status seis_profile_read(int32_t kernel, double* total_ms, int64_t* launches) {
+  if (kernel < 0 || kernel >= prof::NK || !total_ms || !launches)
+    return fail(SEIS_EINVAL, "seis_profile_read: bad arguments");
+  double t = 0.0;
+  const size_t n = prof::used[kernel] / 2;
+  for (size_t p = 0; p < n; ++p) {
+    float ms = 0.f;
+    CK(cudaEventSynchronize(prof::ev[kernel][2 * p + 1]));
+    CK(cudaEventElapsedTime(&ms, prof::ev[kernel][2 * p], prof::ev[kernel][2 * p + 1]));
+    t += ms;
+  }
+  *total_ms = t;
+  *launches = (int64_t)n;
+  return SEIS_OK;
+}
+const char* seis_last_error(void) { return g_err.c_str(); }
+int64_t seis_last_launch_count(void) { return (int64_t)g_launches; }
+
+seis_status seis_slab_bounds(int32_t nz, int32_t nranks, int32_t rank, int32_t* z0,
+                             int32_t* nz_local) {
+  if (!z0 || !nz_local || nranks < 1 || rank < 0 || rank >= nranks || nz < 1)
+    return fail(SEIS_EINVAL, "seis_slab_bounds: bad arguments");
+  const int base = nz / nranks, rem = nz % nranks;
+  *nz_local = base + (rank < rem ? 1 : 0);
+  *z0 = rank * base + std::min<int>(rank, rem);
+  return SEIS_OK;
+}
+
+seis_status seis_comm_unique_id(uint8_t id[128]) {
+  if (!id) return fail(SEIS_EINVAL, "null id");
+  ncclUniqueId u;
+  NK(ncclGetUniqueId(&u));
+  std::memcpy(id, u.internal, 128);
+  return SEIS_OK;
+}
+
+seis_status seis_comm_create(int32_t nranks, int32_t rank, const uint8_t id[128], int32_t device,
+                             seis_comm** out) {
+  if (!out || !id || nranks < 1 || rank < 0 || rank >= nranks)
+    return fail(SEIS_EINVAL, "seis_comm_create: bad arguments");
+  CK(cudaSetDevice(device));
+  ncclUniqueId u;
+  std::memcpy(u.internal, id, 128);
+  seis_comm* c = new seis_comm();
+  c->nranks = nranks;
+  c->rank = rank;
+  c->device = device;
+  ncclResult_t r = ncclCommInitRank(&c->nccl, nranks, u, rank);
+  if (r != ncclSuccess) {
+    delete c;
+    return fail(SEIS_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
+  }
+  *out = c;
+  return SEIS_OK;
+}
+
+seis_status seis_comm_destroy(seis_comm* c) {
+  if (!c) return SEIS_OK;
+  if (c->nccl) ncclCommDestroy(c->nccl);
+  delete c;
+  return SEIS_OK;
+}
+
+static seis_status validate_grid(const seis_grid* g, seis_kind kind) {
+  if (!g) return fail(SEIS_EINVAL, "null grid");
+  if (g->nx < 1 || g->ny < 1 || g->nz < 1) return fail(SEIS_EINVAL, "grid dims must be >= 1");
+  if (!(g->h > 0.f) || !(g->dt > 0.f)) return fail(SEIS_EINVAL, "h and dt must be > 0");
+  if (g->nb < 0 || 3 * g->nb > std::min(g->nx, std::min(g->ny, g->nz)))
+    return fail(SEIS_EINVAL, "nb=%d must satisfy 0 <= 3 nb <= min(nx, ny, nz)", g->nb);
+  if (g->nb > 0 && !(g->pml_R > 0.f && g->pml_R < 1.f)) return fail(SEIS_EINVAL, "pml_R in (0,1)");
+  if (g->pml_f < 0.f) return fail(SEIS_EINVAL, "pml_f must be >= 0");
+  if (kind != SEIS_ISO && kind != SEIS_ACOUSTIC && kind != SEIS_ELASTIC)
+    return fail(SEIS_EINVAL, "unknown kind %d", (int)kind);
+  if (g->free_surface && kind != SEIS_ELASTIC)
+    return fail(SEIS_EUNSUPPORTED, "free_surface is implemented for ELASTIC only");
+  if (g->slabs < 1) return fail(SEIS_EINVAL, "slabs must be >= 1");
+  return SEIS_OK;
+}
+
+seis_status seis_model_destroy(seis_model* M) {
+  if (!M) return SEIS_OK;
+  cudaSetDevice(M->device);
+  for (void* p : M->allocs) cudaFree(p);
+  delete M;
+  return SEIS_OK;
+}
+
+static seis_status model_create_impl(seis_model* M, const float* vp, const float* vs,
+                                     const float* rho) {
+  const seis_grid& g = M->g;
+  const seis_kind kind = M->kind;
+  cudaStream_t st = 0;
+  const size_t plane = (size_t)g.nx * g.ny;
+  const size_t npts = plane * M->pnzl;
+  // host copies of this process's model slab
+  M->hvp.assign(vp, vp + npts);
+  if (rho) M->hrho.assign(rho, rho + npts);
+  if (vs) M->hvs.assign(vs, vs + npts);
+  double vmax = 0.0;
+  for (size_t t = 0; t < npts; ++t) {
+    if (!(vp[t] > 0.f)) return fail(SEIS_EINVAL, "vp must be > 0 (index %zu)", t);
+    vmax = std::max(vmax, (double)vp[t]);
+    if (rho && !(rho[t] > 0.f)) return fail(SEIS_EINVAL, "rho must be > 0 (index %zu)", t);
+    if (vs && (!(vs[t] >= 0.f) || 2.0 * (double)vs[t] * vs[t] > (double)vp[t] * vp[t]))
+      return fail(SEIS_EINVAL, "vs must satisfy 0 <= vs <= vp/sqrt(2) (index %zu)", t);
+  }
+  // the next rank's first plane (z-face coefficients need rho / mu at k+1)
+  std::vector<float> nvp, nvs, nrho;
+  if (M->comm && M->nranks > 1) {
+    float* dv = nullptr;
+    CK(cudaMalloc(&dv, sizeof(double)));
+    CK(cudaMemcpy(dv, &vmax, sizeof(double), cudaMemcpyHostToDevice));
+    NK(ncclAllReduce(dv, dv, 1, ncclFloat64, ncclMax, M->comm->nccl, st));
+    CK(cudaMemcpy(&vmax, dv, sizeof(double), cudaMemcpyDeviceToHost));
+    CK(cudaFree(dv));
+    float* send = nullptr;
+    float* recv = nullptr;
+    CK(cudaMalloc(&send, 3 * plane * sizeof(float)));
+    CK(cudaMalloc(&recv, 3 * plane * sizeof(float)));
+    CK(cudaMemcpy(send, vp, plane * sizeof(float), cudaMemcpyHostToDevice));
+    if (rho) CK(cudaMemcpy(send + plane, rho, plane * sizeof(float), cudaMemcpyHostToDevice));
+    if (vs) CK(cudaMemcpy(send + 2 * plane, vs, plane * sizeof(float), cudaMemcpyHostToDevice));
+    NK(ncclGroupStart());
+    if (M->rank > 0) NK(ncclSend(send, 3 * plane, ncclFloat, M->rank - 1, M->comm->nccl, st));
+    if (M->rank < M->nranks - 1) NK(ncclRecv(recv, 3 * plane, ncclFloat, M->rank + 1, M->comm->nccl, st));
+    NK(ncclGroupEnd());
+    CK(cudaStreamSynchronize(st));
+    if (M->rank < M->nranks - 1) {
+      nvp.resize(plane);
+      CK(cudaMemcpy(nvp.data(), recv, plane * sizeof(float), cudaMemcpyDeviceToHost));
+      if (rho) {
+        nrho.resize(plane);
+        CK(cudaMemcpy(nrho.data(), recv + plane, plane * sizeof(float), cudaMemcpyDeviceToHost));
+      }
+      if (vs) {
+        nvs.resize(plane);
+        CK(cudaMemcpy(nvs.data(), recv + 2 * plane, plane * sizeof(float), cudaMemcpyDeviceToHost));
+      }
+    }
+    CK(cudaFree(send));
+    CK(cudaFree(recv));
+  }
+  M->vmax = vmax;
+  const double vdt_h = vmax * (double)g.dt / (double)g.h;
+  if (vdt_h > courant_limit(kind))
+    return fail(SEIS_ECFL, "Courant number vmax dt/h = %.6f exceeds the 8th-order 3D limit %.6f",
+                vdt_h, courant_limit(kind));
+
+  const double h = g.h, dt = g.dt;
+  const int N3[3] = {g.nx, g.ny, g.nz};
+  // 1D absorbing-layer profiles (host, double -> fp32)
+  if (kind == SEIS_ISO) {
+    float* e1[3];
+    for (int ax = 0; ax < 3; ++ax) {
+      const int N = N3[ax];
+      M->eta1[ax].assign(N, 0.0);
+      std::vector<float> hf(N, 0.f);
+      if (g.nb > 0) {
+        const double emax = 3.0 * vmax * std::log(1.0 / (double)g.pml_R) / (2.0 * g.nb * h);
+        for (int i = 0; i < N; ++i) {
+          const double xi = layer_xi(i, N, g.nb, true, true);
+          M->eta1[ax][i] = emax * xi * xi;
+          hf[i] = (float)(M->eta1[ax][i] * dt);
+        }
+      }
+      TRY(alloc_track(M, (void**)&e1[ax], N * sizeof(float)));
+      CK(cudaMemcpy(e1[ax], hf.data(), N * sizeof(float), cudaMemcpyHostToDevice));
+    }
+    if (g.nb > 0) {
+      M->edx = e1[0];
+      M->edy = e1[1];
+      M->edz = e1[2];
+    }
+  } else if (g.nb > 0) {
+    M->W = g.nb + 1;
+    const double d0 = 3.0 * vmax * std::log(1.0 / (double)g.pml_R) / (2.0 * g.nb * h);
+    for (int ax = 0; ax < 3; ++ax) {
+      const int N = N3[ax];
+      const bool lo = !(ax == 2 && g.free_surface);
+      std::vector<float> a(N), b(N), ah(N), bh(N);
+      for (int i = 0; i < N; ++i) {
+        cpml_coef(layer_xi(i, N, g.nb, lo, true), d0, g.pml_f, dt, &a[i], &b[i]);
+        cpml_coef(layer_xi(i + 0.5, N, g.nb, lo, true), d0, g.pml_f, dt, &ah[i], &bh[i]);
+      }
+      float* dv[4];
+      const std::vector<float>* hv[4] = {&a, &b, &ah, &bh};
+      for (int t = 0; t < 4; ++t) {
+        TRY(alloc_track(M, (void**)&dv[t], N * sizeof(float)));
+        CK(cudaMemcpy(dv[t], hv[t]->data(), N * sizeof(float), cudaMemcpyHostToDevice));
+      }
+      M->cp[ax] = CpmlAxis{dv[0], dv[1], dv[2], dv[3]};
+    }
+  }
+
+  // slabs of this process
+  const int ns = g.slabs;
+  if (M->pnzl < 4 * ns && (ns > 1 || M->nranks > 1))
+    return fail(SEIS_EINVAL, "each z-slab needs >= 4 planes (nz_local=%d, slabs=%d)", M->pnzl, ns);
+  int dev_sms = 148;
+  CK(cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, M->device));
+  M->slabs.resize(ns);
+  for (int s = 0; s < ns; ++s) {
+    int lz0, lnz;
+    seis_slab_bounds(M->pnzl, ns, s, &lz0, &lnz);
+    Slab& S = M->slabs[s];
+    S.d = make_dims(g, M->pz0 + lz0, lnz);
+    const Dims& d = S.d;
+    const size_t sp = (size_t)lnz * plane;  // slab points
+    const size_t off = (size_t)lz0 * plane;
+    S.fld.resize(nfields(kind));
+    for (auto& f : S.fld) TRY(alloc_padded(M, d, &f, st));
+    // per-point coefficients (double -> fp32), compact then padded on device
+    auto val = [&](const std::vector<float>& v, const std::vector<float>& nextp, size_t li, int i,
+                   int j, int k /*local to slab*/) -> double {
+      // value at slab-local (i, j, k) with the grid-edge clamp; k may be lnz (next plane)
+      const int gk = d.z0 + k;
+      if (gk >= g.nz) return v[off + ((size_t)(k - 1) * g.ny + j) * g.nx + i];
+      const int pk = lz0 + k;  // process-local plane
+      if (pk < M->pnzl) return v[((size_t)pk * g.ny + j) * g.nx + i];
+      return nextp[(size_t)j * g.nx + i];
+      (void)li;
+    };
+    std::vector<float> hc(sp);
+    if (kind == SEIS_ISO) {
+      for (size_t t = 0; t < sp; ++t) {
+        const double v = M->hvp[off + t];
+        hc[t] = (float)(v * v * dt * dt / (h * h));
+      }
+      TRY(upload_padded_from_host(M, d, hc, &S.m, st));
+    } else {
+      // buoyancy on faces (O8): dt * 2/(rho_i + rho_{i+1}) / h, last face clamps
+      for (int ax = 0; ax < 3; ++ax) {
+        for (int k = 0; k < lnz; ++k)
+          for (int j = 0; j < g.ny; ++j)
+            for (int i = 0; i < g.nx; ++i) {
+              const double r0 = val(M->hrho, nrho, 0, i, j, k);
+              int i1 = i, j1 = j, k1 = k;
+              if (ax == 0) i1 = std::min(i + 1, g.nx - 1);
+              if (ax == 1) j1 = std::min(j + 1, g.ny - 1);
+              if (ax == 2) k1 = k + 1;
+              const double r1 = val(M->hrho, nrho, 0, i1, j1, k1);
+              hc[((size_t)k * g.ny + j) * g.nx + i] = (float)(dt * (2.0 / (r0 + r1)) / h);
+            }
+        float** dst = ax == 0 ? &S.bx : (ax == 1 ? &S.by : &S.bz);
+        TRY(upload_padded_from_host(M, d, hc, dst, st));
+      }
+      if (kind == SEIS_ACOUSTIC) {
+        for (size_t t = 0; t < sp; ++t) {
+          const double v = M->hvp[off + t], r = M->hrho[off + t];
+          hc[t] = (float)(dt * r * v * v / h);
+        }
+        TRY(upload_padded_from_host(M, d, hc, &S.kdt, st));
+      } else {
+        auto mu_at = [&](int i, int j, int k) {
+          const double s_ = val(M->hvs, nvs, 0, i, j, k), r_ = val(M->hrho, nrho, 0, i, j, k);
+          return r_ * s_ * s_;
+        };
+        for (size_t t = 0; t < sp; ++t) {
+          const double v = M->hvp[off + t], s_ = M->hvs[off + t], r = M->hrho[off + t];
+          hc[t] = (float)(dt * r * v * v / h);  // lambda + 2 mu = rho vp^2
+        }
+        TRY(upload_padded_from_host(M, d, hc, &S.l2m, st));
+        for (size_t t = 0; t < sp; ++t) {
+          const double v = M->hvp[off + t], s_ = M->hvs[off + t], r = M->hrho[off + t];
+          hc[t] = (float)(dt * r * (v * v - 2.0 * s_ * s_) / h);
+        }
+        TRY(upload_padded_from_host(M, d, hc, &S.lam, st));
+        // edge mu: harmonic mean of the 4 adjacent node values, 0 if any is 0 (O9)
+        const int pairs[3][2] = {{0, 1}, {0, 2}, {1, 2}};
+        for (int e = 0; e < 3; ++e) {
+          for (int k = 0; k < lnz; ++k)
+            for (int j = 0; j < g.ny; ++j)
+              for (int i = 0; i < g.nx; ++i) {
+                int di[3] = {0, 0, 0}, dj[3] = {0, 0, 0};
+                di[pairs[e][0]] = 1;
+                dj[pairs[e][1]] = 1;
+                auto cl = [&](int ii, int jj, int kk) {
+                  ii = std::min(ii, g.nx - 1);
+                  jj = std::min(jj, g.ny - 1);
+                  return mu_at(ii, jj, kk);
+                };
+                const double m0 = cl(i, j, k);
+                const double m1 = cl(i + di[0], j + di[1], k + di[2]);
+                const double m2 = cl(i + dj[0], j + dj[1], k + dj[2]);
+                const double m3 = cl(i + di[0] + dj[0], j + di[1] + dj[1], k + di[2] + dj[2]);
+                double me = 0.0;
+                if (m0 > 0 && m1 > 0 && m2 > 0 && m3 > 0) me = 4.0 / (1 / m0 + 1 / m1 + 1 / m2 + 1 / m3);
+                hc[((size_t)k * g.ny + j) * g.nx + i] = (float)(dt * me / h);
+              }
+          float** dst = e == 0 ? &S.mxy : (e == 1 ? &S.mxz : &S.myz);
+          TRY(upload_padded_from_host(M, d, hc, dst, st));
+        }
+      }
+      // compact C-PML memory slabs
+      if (M->W > 0) {
+        const int W = M->W;
+        const int npsi = kind == SEIS_ACOUSTIC ? 6 : 18;
+        // axis of each psi: acoustic 0,1,2,0,1,2; elastic per the oracle's order
+        static const int el_axis[18] = {0, 1, 2, 0, 1, 2, 0, 1, 2, 0, 1, 2, 1, 0, 2, 0, 2, 1};
+        for (int t = 0; t < npsi; ++t) {
+          const int ax = kind == SEIS_ACOUSTIC ? t % 3 : el_axis[t];
+          size_t n;
+          if (ax == 0) n = (size_t)lnz * g.ny * 2 * W;
+          else if (ax == 1) n = (size_t)lnz * 2 * W * g.nx;
+          else n = (size_t)2 * W * g.ny * g.nx;
+          TRY(alloc_track(M, (void**)&S.psi[t], n * sizeof(float)));
+        }
+      }
+    }
+    int occ = 1;
+    if (kind == SEIS_ISO)
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, iso_step_kernel<BY, false, false>, TXW * BY, 0);
+    else if (kind == SEIS_ACOUSTIC)
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_v_kernel<BY, false>, TXW * BY, 0);
+    else
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BY, false>, TXW * BY, 0);
+    choose_chunks(S, occ, dev_sms);
+  }
+  CK(cudaStreamSynchronize(st));
+  return SEIS_OK;
+}
+
+seis_status seis_model_create(const seis_grid* grid, seis_kind kind, const float* vp,
+                              const float* vs, const float* rho, seis_comm* comm, int32_t device,
+                              seis_model** out) {
+  if (!out) return fail(SEIS_EINVAL, "null out");
+  *out = nullptr;
+  TRY(validate_grid(grid, kind));
+  if (!vp) return fail(SEIS_EINVAL, "vp is required");
+  if ((kind == SEIS_ACOUSTIC || kind == SEIS_ELASTIC) && !rho)
+    return fail(SEIS_EINVAL, "rho is required for ACOUSTIC and ELASTIC");
+  if (kind == SEIS_ELASTIC && !vs) return fail(SEIS_EINVAL, "vs is required for ELASTIC");
+  if (comm && grid->slabs != 1)
+    return fail(SEIS_EUNSUPPORTED, "slabs > 1 is the single-process decomposition mode");
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    return fail(SEIS_ECUDA, "no CUDA device: %s", cudaGetErrorString(e));
+  }
+  if (device < 0 || device >= ndev) return fail(SEIS_EINVAL, "device %d out of range", device);
+  CK(cudaSetDevice(device));
+  seis_model* M = new seis_model();
+  M->g = *grid;
+  M->kind = kind;
+  M->device = device;
+  M->comm = comm;
+  M->nranks = comm ? comm->nranks : 1;
+  M->rank = comm ? comm->rank : 0;
+  int32_t z0, nzl;
+  seis_slab_bounds(grid->nz, M->nranks, M->rank, &z0, &nzl);
+  M->pz0 = z0;
+  M->pnzl = nzl;
+  seis_status s = model_create_impl(M, vp, kind == SEIS_ELASTIC ? vs : nullptr,
+                                    kind == SEIS_ISO ? nullptr : rho);
+  if (s != SEIS_OK) {
+    std::string keep = g_err;
+    seis_model_destroy(M);
+    g_err = keep;
+    return s;
+  }
+  *out = M;
+  return SEIS_OK;
+}
+
+seis_status seis_model_slab(const seis_model* M, int32_t* z0, int32_t* nz_local) {
+  if (!M || !z0 || !nz_local) return fail(SEIS_EINVAL, "null argument");
+  *z0 = M->pz0;
+  *nz_local = M->pnzl;
+  return SEIS_OK;
+}
+
+seis_status seis_memory_required(const seis_grid* g, seis_kind kind, const seis_shot* shot,
+                                 int32_t nranks, uint64_t* bytes) {
+  if (!bytes || nranks < 1) return fail(SEIS_EINVAL, "bad arguments");
+  TRY(validate_grid(g, kind));
+  int32_t z0, nzl;
+  seis_slab_bounds(g->nz, nranks, 0, &z0, &nzl);
+  const Dims d = make_dims(*g, 0, nzl);
+  const double padded = (double)d.PS * (nzl + 2 * G) * 4.0;
+  int nf = nfields(kind), np = kind == SEIS_ISO ? 1 : (kind == SEIS_ACOUSTIC ? 4 : 8);
+  double b = (nf + np) * padded;
+  if (kind != SEIS_ISO && g->nb > 0) {
+    const double W = g->nb + 1;
+    const double per = (2 * W * g->ny * (double)nzl + 2 * W * g->nx * (double)nzl + 2 * W * g->nx * (double)g->ny) * 4.0;
+    b += per * (kind == SEIS_ACOUSTIC ? 2 : 6);
+  }
+  if (shot && shot->snap_period >= 1 && shot->nt >= 1)
+    b += (double)((shot->nt - 1) / shot->snap_period) * nzl * (double)g->ny * g->nx * 4.0;
+  *bytes = (uint64_t)b;
+  return SEIS_OK;
+}
+
+}  // extern "C"
+
+// ================================================================== shots
+namespace {
+
+struct ShotTables {
+  std::vector<float*> owned;  // device allocations to free
+};
+
+seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injection,
+                       cudaStream_t st) {
+  const seis_grid& g = M->g;
+  if (!sh) return fail(SEIS_EINVAL, "null shot");
+  if (sh->nt < 1) return fail(SEIS_EINVAL, "nt must be >= 1");
+  if (!sh->wavelet) return fail(SEIS_EINVAL, "null wavelet");
+  if (sh->nrec < 0 || (sh->nrec > 0 && !sh->rec)) return fail(SEIS_EINVAL, "bad receiver list");
+  if (sh->sx < 0 || sh->sy < 0 || sh->sz < 0 || sh->sx >= g.nx || sh->sy >= g.ny || sh->sz >= g.nz)
+    return fail(SEIS_EINVAL, "source (%d,%d,%d) outside the grid", sh->sx, sh->sy, sh->sz);
+  for (int r = 0; r < sh->nrec; ++r) {
+    const int* p = sh->rec + 3 * r;
+    if (p[0] < 0 || p[1] < 0 || p[2] < 0 || p[0] >= g.nx || p[1] >= g.ny || p[2] >= g.nz)
+      return fail(SEIS_EINVAL, "receiver %d (%d,%d,%d) outside the grid", r, p[0], p[1], p[2]);
+  }
+  if (M->kind == SEIS_ELASTIC && (sh->rec_component < 0 || sh->rec_component > 3))
+    return fail(SEIS_EINVAL, "rec_component must be 0..3");
+  M->hwav = sh->wavelet;  // source amplitudes are kernel arguments (one fused add per step)
+  const double h = g.h, dt = g.dt;
+  auto point_scale = [&](int x, int y, int z) -> double {
+    const size_t li = ((size_t)(z - M->pz0) * g.ny + y) * g.nx + x;
+    const double v = M->hvp[li];
+    if (M->kind == SEIS_ISO) {
+      double eta = 0.0;
+      if (g.nb > 0) eta = M->eta1[0][x] + M->eta1[1][y] + M->eta1[2][z];
+      return v * v * dt * dt / (h * h * h) / (1.0 + eta * dt);  // O3
+    }
+    const double r = M->hrho[li];
+    if (M->kind == SEIS_ACOUSTIC) return dt * r * v * v / (h * h * h);  // O8/O11
+    const double s = M->hvs[li];
+    const double mu = r * s * s, lam = r * (v * v - 2.0 * s * s);
+    return dt * (lam + 2.0 / 3.0 * mu) / (h * h * h);  // O11 explosive
+  };
+  for (Slab& S : M->slabs) {
+    const int z0 = S.d.z0, z1 = S.d.z0 + S.d.nzl;
+    S.src_o = -1;
+    if (!backward_injection && sh->sz >= z0 && sh->sz < z1) {
+      S.src_o = S.d.at(sh->sx, sh->sy, sh->sz - z0);
+      S.src_scale = (float)point_scale(sh->sx, sh->sy, sh->sz);
+    }
+    // receivers owned by this slab
+    std::vector<long long> off;
+    std::vector<int> rid;
+    for (int r = 0; r < sh->nrec; ++r) {
+      const int* p = sh->rec + 3 * r;
+      if (p[2] >= z0 && p[2] < z1) {
+        off.push_back(S.d.at(p[0], p[1], p[2] - z0));
+        rid.push_back(r);
+      }
+    }
+    S.nrec_own = (int)off.size();
+    if (S.nrec_own > 0) {
+      if (S.d_rec_off) { cudaFree(S.d_rec_off); cudaFree(S.d_rec_id); }
+      CK(dmalloc(&S.d_rec_off, off.size()));
+      CK(dmalloc(&S.d_rec_id, rid.size()));
+      CK(cudaMemcpy(S.d_rec_off, off.data(), off.size() * sizeof(long long), cudaMemcpyHostToDevice));
+      CK(cudaMemcpy(S.d_rec_id, rid.data(), rid.size() * sizeof(int), cudaMemcpyHostToDevice));
+    }
+    S.ngroups = 0;
+    if (backward_injection && S.nrec_own > 0) {
+      // merge duplicates: group receivers by node, members in receiver-index order (O12)
+      std::map<long long, std::vector<int>> groups;
+      for (size_t t = 0; t < off.size(); ++t) groups[off[t]].push_back(rid[t]);
+      std::vector<long long> goff;
+      std::vector<float> gsc;
+      std::vector<int> gstart{0}, gmem;
+      for (auto& kv : groups) {
+        goff.push_back(kv.first);
+        const int r0 = kv.second.front();
+        const int* p = sh->rec + 3 * r0;
+        gsc.push_back((float)point_scale(p[0], p[1], p[2]));
+        for (int r : kv.second) gmem.push_back(r);
+        gstart.push_back((int)gmem.size());
+      }
+      S.ngroups = (int)goff.size();
+      if (S.d_g_off) { cudaFree(S.d_g_off); cudaFree(S.d_g_scale); cudaFree(S.d_g_start); cudaFree(S.d_g_mem); }
+      CK(dmalloc(&S.d_g_off, goff.size()));
+      CK(dmalloc(&S.d_g_scale, gsc.size()));
+      CK(dmalloc(&S.d_g_start, gstart.size()));
+      CK(dmalloc(&S.d_g_mem, gmem.size()));
+      CK(cudaMemcpy(S.d_g_off, goff.data(), goff.size() * sizeof(long long), cudaMemcpyHostToDevice));
+      CK(cudaMemcpy(S.d_g_scale, gsc.data(), gsc.size() * sizeof(float), cudaMemcpyHostToDevice));
+      CK(cudaMemcpy(S.d_g_start, gstart.data(), gstart.size() * sizeof(int), cudaMemcpyHostToDevice));
+      CK(cudaMemcpy(S.d_g_mem, gmem.data(), gmem.size() * sizeof(int), cudaMemcpyHostToDevice));
+    }
+  }
+  return SEIS_OK;
+}
+
+// Zero the state of every slab (fields incl. ghosts, C-PML slabs).
+seis_status zero_state(seis_model* M, cudaStream_t st) {
+  for (Slab& S : M->slabs) {
+    const size_t elems = (size_t)S.d.PS * (S.d.nzl + 2 * G);
+    for (float* f : S.fld) CK(cudaMemsetAsync(f, 0, elems * sizeof(float), st));
+    if (M->W > 0) {
+      const int W = M->W;
+      const int npsi = M->kind == SEIS_ACOUSTIC ? 6 : (M->kind == SEIS_ELASTIC ? 18 : 0);
+      static const int el_axis[18] = {0, 1, 2, 0, 1, 2, 0, 1, 2, 0, 1, 2, 1, 0, 2, 0, 2, 1};
+      for (int t = 0; t < npsi; ++t) {
+        const int ax = M->kind == SEIS_ACOUSTIC ? t % 3 : el_axis[t];
+        size_t n;
+        if (ax == 0) n = (size_t)S.d.nzl * S.d.ny * 2 * W;
+        else if (ax == 1) n = (size_t)S.d.nzl * 2 * W * S.d.nx;
+        else n = (size_t)2 * W * S.d.ny * S.d.nx;
+        CK(cudaMemsetAsync(S.psi[t], 0, n * sizeof(float), st));
+      }
+    }
+    S.cur = 0;
+  }
+  return SEIS_OK;
+}
+
+// Free-surface ghost planes (O16) of the slab that holds the global top.
+seis_status fs_mirror(seis_model* M, std::initializer_list<int> fields, cudaStream_t st) {
+  if (!M->g.free_surface) return SEIS_OK;
+  Slab& S = M->slabs.front();
+  if (S.d.z0 != 0) return SEIS_OK;
+  for (int f : fields) {
+    // parity / staggering per field: v even, sigma_zz/xz/yz odd; vz, sxz, syz on half z nodes
+    const int odd = (f == ESZZ || f == ESXZ || f == ESYZ) ? 1 : 0;
+    const int half = (f == EVZ || f == ESXZ || f == ESYZ) ? 1 : 0;
+    {
+      PROF(8, st);
+      fs_mirror_kernel<<<dim3((S.d.nx + 127) / 128, S.d.ny), 128, 0, st>>>(S.fld[f], S.d, odd, half);
+    }
+    CKL();
+  }
+  return SEIS_OK;
+}
+
+dim3 grid_of(const Slab& S) {
+  return dim3((S.d.nx + TXW - 1) / TXW, (S.d.ny + BY - 1) / BY, S.nzch);
+}
+
+// Backward-phase receiver injection into the field just produced (before its
+// ghost planes are exchanged, so neighbouring slabs see the injected values).
+seis_status inject_rows(seis_model* M, const float* row, cudaStream_t st) {
+  for (Slab& S : M->slabs) {
+    if (S.ngroups == 0) continue;
+    float* f = M->kind == SEIS_ISO ? S.fld[S.cur] : S.fld[0];
+    PROF(5, st);
+    inject_kernel<<<(S.ngroups + 127) / 128, 128, 0, st>>>(f, S.d_g_off, S.d_g_scale, S.d_g_start,
+                                                           S.d_g_mem, row, S.ngroups);
+    CKL();
+  }
+  return SEIS_OK;
+}
+
+// One forward time step of every slab of the process, incl. exchanges.
+//   snap: compact snapshot target per slab (or null), imgS/img: imaging of the INPUT level,
+//   inj_row: receiver samples injected into the produced field (backward phase) or null
+seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
+                 std::vector<const float*>* imgS, std::vector<float*>* img, cudaStream_t st,
+                 const float* inj_row = nullptr) {
+  const dim3 blk(TXW, BY);
+  if (M->kind == SEIS_ISO) {
+    for (size_t s = 0; s < M->slabs.size(); ++s) {
+      Slab& S = M->slabs[s];
+      IsoArgs a;
+      a.un = S.fld[S.cur];
+      a.up = S.fld[1 - S.cur];
+      a.m = S.m;
+      a.edx = M->edx;
+      a.edy = M->edy;
+      a.edz = M->edz;
+      a.d = S.d;
+      a.zc = S.zc;
+      a.src_o = with_src ? S.src_o : -1;
+      a.src_amp = 0.f;
+      if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
+      a.snap = snap ? (*snap)[s] : nullptr;
+      a.imgS = imgS ? (*imgS)[s] : nullptr;
+      a.img = img ? (*img)[s] : nullptr;
+      const dim3 gr = grid_of(S);
+      {
+        PROF(0, st);
+        if (a.snap) iso_step_kernel<BY, true, false><<<gr, blk, 0, st>>>(a);
+        else if (a.img) iso_step_kernel<BY, false, true><<<gr, blk, 0, st>>>(a);
+        else iso_step_kernel<BY, false, false><<<gr, blk, 0, st>>>(a);
+      }
+      CKL();
+    }
+    for (Slab& S : M->slabs) S.cur = 1 - S.cur;
+    if (inj_row) TRY(inject_rows(M, inj_row, st));
+    // exchange the new level (fld[cur] after the swap)
+    const int f = M->slabs[0].cur;
+    TRY(exchange(M, {f}, st));
+    return SEIS_OK;
+  }
+  if (M->kind == SEIS_ACOUSTIC) {
+    for (size_t s = 0; s < M->slabs.size(); ++s) {
+      Slab& S = M->slabs[s];
+      AcVArgs a;
+      a.p = S.fld[0];
+      a.qx = S.fld[1];
+      a.qy = S.fld[2];
+      a.qz = S.fld[3];
+      a.bx = S.bx;
+      a.by = S.by;
+      a.bz = S.bz;
+      a.W = M->W;
+      a.zlo = 1;
+      a.cx = M->cp[0];
+      a.cy = M->cp[1];
+      a.cz = M->cp[2];
+      a.psx = S.psi[0];
+      a.psy = S.psi[1];
+      a.psz = S.psi[2];
+      a.d = S.d;
+      a.zc = S.zc;
+      a.imgS = imgS ? (*imgS)[s] : nullptr;
+      a.img = img ? (*img)[s] : nullptr;
+      const dim3 gr = grid_of(S);
+      {
+        PROF(1, st);
+        if (a.img) ac_v_kernel<BY, true><<<gr, blk, 0, st>>>(a);
+        else ac_v_kernel<BY, false><<<gr, blk, 0, st>>>(a);
+      }
+      CKL();
+    }
+    TRY(exchange(M, {3}, st));  // q_z has the only z-derivative in P
+    for (size_t s = 0; s < M->slabs.size(); ++s) {
+      Slab& S = M->slabs[s];
+      AcPArgs a;
+      a.p = S.fld[0];
+      a.qx = S.fld[1];
+      a.qy = S.fld[2];
+      a.qz = S.fld[3];
+      a.kdt = S.kdt;
+      a.W = M->W;
+      a.zlo = 1;
+      a.cx = M->cp[0];
+      a.cy = M->cp[1];
+      a.cz = M->cp[2];
+      a.pqx = S.psi[3];
+      a.pqy = S.psi[4];
+      a.pqz = S.psi[5];
+      a.d = S.d;
+      a.zc = S.zc;
+      a.src_o = with_src ? S.src_o : -1;
+      a.src_amp = 0.f;
+      if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
+      a.snap = snap ? (*snap)[s] : nullptr;
+      const dim3 gr = grid_of(S);
+      {
+        PROF(2, st);
+        if (a.snap) ac_p_kernel<BY, true><<<gr, blk, 0, st>>>(a);
+        else ac_p_kernel<BY, false><<<gr, blk, 0, st>>>(a);
+      }
+      CKL();
+    }
+    if (inj_row) TRY(inject_rows(M, inj_row, st));
+    TRY(exchange(M, {0}, st));  // p for the next V
+    return SEIS_OK;
+  }
+  // ELASTIC
+  for (size_t s = 0; s < M->slabs.size(); ++s) {
+    Slab& S = M->slabs[s];
+    ElVArgs a;
+    for (int t = 0; t < 9; ++t) a.f[t] = S.fld[t];
+    a.bx = S.bx;
+    a.by = S.by;
+    a.bz = S.bz;
+    a.W = M->W;
+    a.zlo = M->g.free_surface ? 0 : 1;
+    a.fs = M->g.free_surface;
+    a.cx = M->cp[0];
+    a.cy = M->cp[1];
+    a.cz = M->cp[2];
+    for (int t = 0; t < 9; ++t) a.psi[t] = S.psi[t];
+    a.d = S.d;
+    a.zc = S.zc;
+    const dim3 gr = grid_of(S);
+    {
+      PROF(3, st);
+      el_v_kernel<BY><<<gr, blk, 0, st>>>(a);
+    }
+    CKL();
+  }
+  TRY(exchange(M, {0, 1, 2}, st));
+  TRY(fs_mirror(M, {EVX, EVY, EVZ}, st));
+  for (size_t s = 0; s < M->slabs.size(); ++s) {
+    Slab& S = M->slabs[s];
+    ElSArgs a;
+    for (int t = 0; t < 9; ++t) a.f[t] = S.fld[t];
+    a.l2m = S.l2m;
+    a.lam = S.lam;
+    a.mxy = S.mxy;
+    a.mxz = S.mxz;
+    a.myz = S.myz;
+    a.W = M->W;
+    a.zlo = M->g.free_surface ? 0 : 1;
+    a.fs = M->g.free_surface;
+    a.cx = M->cp[0];
+    a.cy = M->cp[1];
+    a.cz = M->cp[2];
+    for (int t = 0; t < 9; ++t) a.psi[t] = S.psi[9 + t];
+    a.d = S.d;
+    a.zc = S.zc;
+    a.src_o = with_src ? S.src_o : -1;
+    a.src_amp = 0.f;
+    if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
+    const dim3 gr = grid_of(S);
+    {
+      PROF(4, st);
+      el_s_kernel<BY, false><<<gr, blk, 0, st>>>(a);
+    }
+    CKL();
+  }
+  TRY(exchange(M, {5, 7, 8}, st));
+  TRY(fs_mirror(M, {ESZZ, ESXZ, ESYZ}, st));
+  return SEIS_OK;
+}
+
+// Field holding the recorded / imaged quantity
+const float* out_field(seis_model* M, Slab& S, int comp) {
+  if (M->kind == SEIS_ISO) return S.fld[S.cur];
+  if (M->kind == SEIS_ACOUSTIC) return S.fld[0];
+  if (comp == 3) return S.fld[3];
+  return S.fld[comp];
+}
+
+seis_status gather(seis_model* M, const seis_shot* sh, float* seis_dev, int n, cudaStream_t st) {
+  for (Slab& S : M->slabs) {
+    if (S.nrec_own == 0) continue;
+    const int comp = M->kind == SEIS_ELASTIC ? sh->rec_component : 0;
+    const float* f0 = out_field(M, S, comp);
+    const int pres = (M->kind == SEIS_ELASTIC && comp == 3);
+    PROF(6, st);
+    gather_kernel<<<(S.nrec_own + 127) / 128, 128, 0, st>>>(
+        seis_dev + (size_t)n * sh->nrec, f0, pres ? S.fld[4] : f0, pres ? S.fld[5] : f0,
+        S.d_rec_off, S.d_rec_id, S.nrec_own, pres);
+    CKL();
+  }
+  return SEIS_OK;
+}
+
+seis_status ensure_stage(seis_model* M, size_t elems) {
+  if (M->stage_elems >= elems) return SEIS_OK;
+  void* p = nullptr;
+  TRY(alloc_track(M, &p, elems * sizeof(float)));
+  M->stage = (float*)p;
+  M->stage_elems = elems;
+  return SEIS_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+seis_status seis_forward_model(seis_model* M, const seis_shot* sh, float* seis, void* stream) {
+  g_launches = 0;
+  if (!M) return fail(SEIS_EINVAL, "null model");
+  if (!seis && sh && sh->nrec > 0) return fail(SEIS_EINVAL, "null seis");
+  CK(cudaSetDevice(M->device));
+  cudaStream_t st = (cudaStream_t)stream;
+  TRY(setup_shot(M, sh, false, st));
+  TRY(zero_state(M, st));
+  const size_t ns = (size_t)sh->nt * sh->nrec;
+  const bool dev = ns == 0 || is_device_ptr(seis);
+  float* sd = seis;
+  if (!dev) {
+    TRY(ensure_stage(M, ns));
+    sd = M->stage;
+  }
+  if (ns) CK(cudaMemsetAsync(sd, 0, ns * sizeof(float), st));
+  for (int n = 0; n < sh->nt; ++n) {
+    TRY(step(M, n, true, nullptr, nullptr, nullptr, st));
+    if (sh->nrec) TRY(gather(M, sh, sd, n, st));
+  }
+  if (M->comm && M->nranks > 1 && ns) NK(ncclAllReduce(sd, sd, ns, ncclFloat, ncclSum, M->comm->nccl, st));
+  if (!dev && ns) CK(cudaMemcpyAsync(seis, sd, ns * sizeof(float), cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  M->last_nt = sh->nt;
+  return SEIS_OK;
+}
+
+seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, float* image,
+                         void* stream) {
+  g_launches = 0;
+  if (!M) return fail(SEIS_EINVAL, "null model");
+  if (!sh) return fail(SEIS_EINVAL, "null shot");
+  if (!image) return fail(SEIS_EINVAL, "null image");
+  if (sh->nrec > 0 && !data) return fail(SEIS_EINVAL, "null data");
+  if (M->kind == SEIS_ELASTIC) return fail(SEIS_EUNSUPPORTED, "elastic RTM is not implemented in this version");
+  if (sh->snap_period < 1) return fail(SEIS_EINVAL, "snap_period must be >= 1");
+  CK(cudaSetDevice(M->device));
+  cudaStream_t st = (cudaStream_t)stream;
+  const seis_grid& g = M->g;
+  const int nt = sh->nt, snap = sh->snap_period;
+  TRY(setup_shot(M, sh, false, st));
+  // snapshot pool (O14): nsnap fields of the process slab
+  const int nsnap = nt >= 1 ? (nt - 1) / snap : 0;
+  const size_t slab_pts = (size_t)M->pnzl * g.ny * g.nx;
+  const size_t need = (size_t)nsnap * slab_pts;
+  if (need > M->pool_elems) {
+    size_t freeb = 0, totb = 0;
+    cudaMemGetInfo(&freeb, &totb);
+    if (M->pool) {
+      cudaFree(M->pool);
+      M->allocs.erase(std::find(M->allocs.begin(), M->allocs.end(), (void*)M->pool));
+      M->pool = nullptr;
+      M->pool_elems = 0;
+    }
+    void* p = nullptr;
+    cudaError_t e = cudaMalloc(&p, need * sizeof(float));
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      return fail(SEIS_ENOMEM, "snapshot pool needs %zu bytes (%d snapshots), %zu free", need * 4,
+                  nsnap, freeb);
+    }
+    M->allocs.push_back(p);
+    M->pool = (float*)p;
+    M->pool_elems = need;
+  }
+  // image / data staging
+  const bool img_dev = is_device_ptr(image);
+  const size_t nd = (size_t)nt * sh->nrec;
+  const bool data_dev = nd == 0 || is_device_ptr(data);
+  float* img_d = image;
+  const float* data_d = data;
+  TRY(ensure_stage(M, (img_dev ? 0 : slab_pts) + (data_dev ? 0 : nd)));
+  if (!img_dev) {
+    img_d = M->stage;
+    CK(cudaMemcpyAsync(img_d, image, slab_pts * sizeof(float), cudaMemcpyHostToDevice, st));
+  }
+  if (!data_dev) {
+    float* dd = M->stage + (img_dev ? 0 : slab_pts);
+    CK(cudaMemcpyAsync(dd, data, nd * sizeof(float), cudaMemcpyHostToDevice, st));
+    data_d = dd;
+  }
+  // ---- forward phase: source wavefield, snapshots S_j (j = snap .. nt-1) in HBM
+  TRY(zero_state(M, st));
+  std::vector<float*> snapp(M->slabs.size());
+  for (int n = 0; n < nt; ++n) {
+    const int j = n + 1;
+    const bool take = (j % snap == 0) && j <= nt - 1;
+    if (take) {
+      size_t off = (size_t)(j / snap - 1) * slab_pts;
+      for (size_t s = 0; s < M->slabs.size(); ++s) {
+        const size_t so = (size_t)(M->slabs[s].d.z0 - M->pz0) * g.ny * g.nx;
+        snapp[s] = M->pool + off + so;
+      }
+    }
+    TRY(step(M, n, true, take ? &snapp : nullptr, nullptr, nullptr, st));
+  }
+  // ---- backward phase: receiver wavefield from zero, same operator
+  TRY(setup_shot(M, sh, true, st));
+  TRY(zero_state(M, st));
+  std::vector<const float*> Sp(M->slabs.size());
+  std::vector<float*> Ip(M->slabs.size());
+  for (size_t s = 0; s < M->slabs.size(); ++s)
+    Ip[s] = img_d + (size_t)(M->slabs[s].d.z0 - M->pz0) * g.ny * g.nx;
+  for (int m = 0; m < nt; ++m) {
+    // imaging of level j = nt - m (the INPUT of this step, R^m) fused into the step kernel
+    const int j = nt - m;
+    const bool im = (j % snap == 0) && j >= snap && j <= nt - 1;
+    if (im) {
+      const size_t off = (size_t)(j / snap - 1) * slab_pts;
+      for (size_t s = 0; s < M->slabs.size(); ++s)
+        Sp[s] = M->pool + off + (size_t)(M->slabs[s].d.z0 - M->pz0) * g.ny * g.nx;
+    }
+    // step + receiver injection of data[nt-1-m] (all receivers, one launch per slab)
+    TRY(step(M, m, false, nullptr, im ? &Sp : nullptr, im ? &Ip : nullptr, st,
+             sh->nrec ? data_d + (size_t)(nt - 1 - m) * sh->nrec : nullptr));
+  }
+  if (!img_dev) CK(cudaMemcpyAsync(image, img_d, slab_pts * sizeof(float), cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  M->last_nt = nt;
+  return SEIS_OK;
+}
+
+seis_status seis_get_field(const seis_model* Mc, int32_t which, float* dst, void* stream) {
+  seis_model* M = const_cast<seis_model*>(Mc);
+  if (!M || !dst) return fail(SEIS_EINVAL, "null argument");
+  const int nf = nfields(M->kind);
+  if (which < 0 || which >= nf) return fail(SEIS_EINVAL, "field index %d out of range", which);
+  CK(cudaSetDevice(M->device));
+  cudaStream_t st = (cudaStream_t)stream;
+  const seis_grid& g = M->g;
+  const size_t slab_pts = (size_t)M->pnzl * g.ny * g.nx;
+  const bool dev = is_device_ptr(dst);
+  float* out = dst;
+  if (!dev) {
+    TRY(ensure_stage(M, slab_pts));
+    out = M->stage;
+  }
+  for (Slab& S : M->slabs) {
+    int f = which;
+    if (M->kind == SEIS_ISO) f = which == 0 ? S.cur : 1 - S.cur;
+    unpad_kernel<<<1024, 256, 0, st>>>(out + (size_t)(S.d.z0 - M->pz0) * g.ny * g.nx, S.fld[f], S.d);
+    CKL();
+  }
+  if (!dev) CK(cudaMemcpyAsync(dst, out, slab_pts * sizeof(float), cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  return SEIS_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,92 @@
+"""C-ABI checks that need no GPU: the library loads, exports every symbol that
+include/seis.h declares, and its pure host logic (slab bounds, validation order,
+memory estimate) behaves; compute calls are not made here."""
+import ctypes as C
+import os
+import re
+
+import pytest
+
+import paper_conf_ppopp_qawasmehchc15_b200 as seis
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _declared():
+    src = open(os.path.join(ROOT, "include", "seis.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(seis_[a-z_]+)\s*\(", src)))
+
+
+def test_header_symbols_match_binding_list():
+    assert _declared() == sorted(seis.SYMBOLS)
+
+
+def test_library_exports_every_declared_symbol():
+    L = seis.lib()
+    for name in _declared():
+        assert hasattr(L, name), name
+    out = os.popen(f"nm -D --defined-only {seis._LIBPATH}").read()
+    for name in _declared():
+        assert re.search(rf"\bT {name}\b", out), name
+
+
+def test_version_and_error_strings():
+    assert b"sm_100a" in seis.lib().seis_version()
+    assert isinstance(seis.lib().seis_last_error(), bytes)
+
+
+@pytest.mark.parametrize("nz,P", [(512, 1), (512, 3), (1024, 8), (10, 4), (7, 7)])
+def test_slab_bounds_partition(nz, P):
+    prev = 0
+    sizes = []
+    for r in range(P):
+        z0, n = seis.slab_bounds(nz, P, r)
+        assert z0 == prev
+        prev = z0 + n
+        sizes.append(n)
+    assert prev == nz
+    assert max(sizes) - min(sizes) <= 1
+
+
+def test_slab_bounds_rejects_bad_rank():
+    with pytest.raises(seis.SeisError) as e:
+        seis.slab_bounds(64, 2, 2)
+    assert e.value.name == "SEIS_EINVAL"
+
+
+def test_memory_required_counts_snapshots():
+    g = seis.Grid(128, 96, 64, 10.0, 8e-4, nb=10)
+    import numpy as np
+
+    sh = seis.Shot((1, 1, 1), np.zeros(201, np.float32), np.zeros((1, 3), np.int32), snap_period=20)
+    m0 = seis.memory_required(g, "acoustic")
+    m1 = seis.memory_required(g, "acoustic", sh)
+    assert m1 - m0 == 10 * 128 * 96 * 64 * 4
+
+
+def test_invalid_grid_is_rejected_before_touching_the_device():
+    import numpy as np
+
+    g = seis.Grid(16, 16, 16, 10.0, 1e-3, nb=7)  # 3 nb > 16
+    with pytest.raises(seis.SeisError) as e:
+        seis.Model(g, "iso", np.full((16, 16, 16), 2000.0, np.float32))
+    assert e.value.name == "SEIS_EINVAL"
+    g = seis.Grid(16, 16, 16, 10.0, 1e-3, free_surface=1)
+    with pytest.raises(seis.SeisError) as e:
+        seis.Model(g, "acoustic", np.full((16, 16, 16), 2000.0, np.float32),
+                   rho=np.ones((16, 16, 16), np.float32))
+    assert e.value.name == "SEIS_EUNSUPPORTED"
+
+
+def test_no_cpu_fallback_without_a_device():
+    """On a GPU-less host the product path must fail loudly, never compute on the CPU."""
+    import numpy as np
+    import torch
+
+    if torch.cuda.is_available():
+        pytest.skip("a CUDA device is present")
+    g = seis.Grid(16, 16, 16, 10.0, 1e-3)
+    with pytest.raises(seis.SeisError) as e:
+        seis.Model(g, "iso", np.full((16, 16, 16), 2000.0, np.float32))
+    assert e.value.name == "SEIS_ECUDA"
