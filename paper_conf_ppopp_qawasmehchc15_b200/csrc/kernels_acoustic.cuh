@@ -6,11 +6,13 @@
 // with h D+ f_{i+1/2} = sum_m d_m (f_{i+m} - f_{i-m+1}), h D- g_i = sum_m d_m (g_{i+m-1} - g_{i-m})
 // (psi is stored multiplied by h, so both updates work on the unscaled differences).
 //
-// Two z-marching kernels per step: V reads p (x/y halos from a
-// shared-memory tile, z from an 8-deep register queue), rho-derived dt b/h and
-// RMWs q_x, q_y, q_z; P reads q_x (x halo tile), q_y (y halo tile), q_z (z queue),
-// dt K / h and RMWs p.  Fused epilogues: P adds the source and stores the
-// snapshot; V applies the imaging condition to its input p (O15).
+// Two z-marching kernels per step.  V: p plane tile (x/y halo 4)
+// by TMA through an NS-stage mbarrier ring, p's z-neighbours from a register
+// queue, q_x, q_y, q_z and the face buoyancies dt b/h as coalesced streams
+// prefetched one plane ahead.  P: q_x (x halo) and q_y (y halo) tiles by TMA,
+// q_z from a register queue, p and dt K/h streamed.  Fused epilogues: P adds the
+// source and stores the snapshot; V applies the imaging
+// condition to its input p (O15).
 #pragma once
 #include "common.cuh"
 
@@ -23,7 +25,10 @@ struct CpmlAxis {
   const float* __restrict__ bh;
 };
 
+constexpr int AC_NS = 4;
+
 struct AcVArgs {
+  CUtensorMap mp;                 // p, box (32+8) x (BY+8) x 1
   const float* __restrict__ p;
   float* __restrict__ qx;
   float* __restrict__ qy;
@@ -44,24 +49,38 @@ struct AcVArgs {
 };
 
 template <int BY, bool IMG>
-__global__ void __launch_bounds__(TXW * BY) ac_v_kernel(const AcVArgs a) {
+__global__ void __launch_bounds__(TXW * BY) ac_v_kernel(const __grid_constant__ AcVArgs a) {
   constexpr int W = TXW + 8;
-  __shared__ float s[(BY + 8) * W];
+  constexpr int TILE = (BY + 8) * W;
+  constexpr uint32_t TX_BYTES = TILE * 4;
+  __shared__ __align__(128) float sm[AC_NS * TILE];
+  __shared__ __align__(8) uint64_t bar[AC_NS];
   const Dims& d = a.d;
-  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
   const int i0 = blockIdx.x * TXW, j0 = blockIdx.y * BY;
   const int i = i0 + tx, j = j0 + ty;
   const int k0 = blockIdx.z * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
+  const int np = k1 - k0;
   const bool own = (i < d.nx) && (j < d.ny);
   const long long PS = d.PS;
   const long long oc = (long long)(j + G) * d.PX + (i + G);
-  const long long ot = (long long)(j0 + G) * d.PX + (i0 + G);
   const float* __restrict__ p = a.p;
   const int Wl = a.W;
   const bool lx = Wl > 0 && CpmlIdx::in(i, d.nx, Wl, true);
   const bool ly = Wl > 0 && CpmlIdx::in(j, d.ny, Wl, true);
 
+  if (tid == 0) {
+    for (int s = 0; s < AC_NS; ++s) mbar_init(&bar[s], 1);
+    mbar_fence_init();
+  }
+  __syncthreads();
+  if (tid == 0) {
+    for (int s = 0; s < AC_NS && s < np; ++s) {
+      mbar_expect_tx(&bar[s], TX_BYTES);
+      tma_load_3d(sm + s * TILE, &a.mp, &bar[s], i0, j0, k0 + s + G);
+    }
+  }
   float r0, r1, r2, r3, r4, r5, r6, r7;  // p at k-3 .. k+4
   r0 = __ldg(p + (long long)(k0 - 3 + G) * PS + oc);
   r1 = __ldg(p + (long long)(k0 - 2 + G) * PS + oc);
@@ -70,18 +89,29 @@ __global__ void __launch_bounds__(TXW * BY) ac_v_kernel(const AcVArgs a) {
   r4 = __ldg(p + (long long)(k0 + 1 + G) * PS + oc);
   r5 = __ldg(p + (long long)(k0 + 2 + G) * PS + oc);
   r6 = __ldg(p + (long long)(k0 + 3 + G) * PS + oc);
+  float r7n = __ldg(p + (long long)(k0 + 4 + G) * PS + oc);
+  float qxn = 0.f, qyn = 0.f, qzn = 0.f, bxn = 0.f, byn = 0.f, bzn = 0.f;
+  if (own && np > 0) {
+    const long long o = (long long)(k0 + G) * PS + oc;
+    qxn = a.qx[o]; qyn = a.qy[o]; qzn = a.qz[o];
+    bxn = __ldg(a.bx + o); byn = __ldg(a.by + o); bzn = __ldg(a.bz + o);
+  }
 
-  for (int k = k0; k < k1; ++k) {
+  for (int it = 0; it < np; ++it) {
+    const int k = k0 + it;
+    const int s = it % AC_NS;
     const long long o = (long long)(k + G) * PS + oc;
-    r7 = __ldg(p + o + 4 * PS);
-    float qxv = 0.f, qyv = 0.f, qzv = 0.f, bxv = 0.f, byv = 0.f, bzv = 0.f;
-    if (own) {
-      qxv = a.qx[o]; qyv = a.qy[o]; qzv = a.qz[o];
-      bxv = __ldg(a.bx + o); byv = __ldg(a.by + o); bzv = __ldg(a.bz + o);
+    r7 = r7n;
+    const float qxv = qxn, qyv = qyn, qzv = qzn, bxv = bxn, byv = byn, bzv = bzn;
+    if (it + 1 < np) {
+      r7n = __ldg(p + o + 5 * PS);
+      if (own) {
+        qxn = a.qx[o + PS]; qyn = a.qy[o + PS]; qzn = a.qz[o + PS];
+        bxn = __ldg(a.bx + o + PS); byn = __ldg(a.by + o + PS); bzn = __ldg(a.bz + o + PS);
+      }
     }
-    load_tile<BY, 4, 4>(s, p, (long long)(k + G) * PS + ot, d.PX);
-    __syncthreads();
-    const float* c = s + (ty + 4) * W + tx + 4;
+    mbar_wait(&bar[s], (it / AC_NS) & 1);
+    const float* c = sm + s * TILE + (ty + 4) * W + tx + 4;
     float dx = SEIS_D1 * (c[1] - c[0]);
     dx = fmaf(SEIS_D2, c[2] - c[-1], dx);
     dx = fmaf(SEIS_D3, c[3] - c[-2], dx);
@@ -125,14 +155,19 @@ __global__ void __launch_bounds__(TXW * BY) ac_v_kernel(const AcVArgs a) {
       }
     }
     __syncthreads();
+    if (tid == 0 && it + AC_NS < np) {
+      fence_proxy_async();
+      mbar_expect_tx(&bar[s], TX_BYTES);
+      tma_load_3d(sm + s * TILE, &a.mp, &bar[s], i0, j0, k + AC_NS + G);
+    }
     r0 = r1; r1 = r2; r2 = r3; r3 = r4; r4 = r5; r5 = r6; r6 = r7;
   }
 }
 
 struct AcPArgs {
+  CUtensorMap mqx;                // q_x, box (32+8) x BY x 1
+  CUtensorMap mqy;                // q_y, box 32 x (BY+8) x 1
   float* __restrict__ p;
-  const float* __restrict__ qx;
-  const float* __restrict__ qy;
   const float* __restrict__ qz;
   const float* __restrict__ kdt;  // dt * rho v^2 / h (padded)
   int W;
@@ -149,25 +184,41 @@ struct AcPArgs {
 };
 
 template <int BY, bool SNAP>
-__global__ void __launch_bounds__(TXW * BY) ac_p_kernel(const AcPArgs a) {
-  constexpr int WX = TXW + 8;  // q_x tile: x halo only
-  __shared__ float sx[BY * WX];
-  __shared__ float sy[(BY + 8) * TXW];  // q_y tile: y halo only
+__global__ void __launch_bounds__(TXW * BY) ac_p_kernel(const __grid_constant__ AcPArgs a) {
+  constexpr int WX = TXW + 8;
+  constexpr int TQX = BY * WX;           // q_x tile (x halo)
+  constexpr int TQY = (BY + 8) * TXW;    // q_y tile (y halo)
+  constexpr int STAGE = TQX + TQY;       // both multiples of 32 floats (128 B)
+  constexpr uint32_t TX_BYTES = STAGE * 4;
+  __shared__ __align__(128) float sm[AC_NS * STAGE];
+  __shared__ __align__(8) uint64_t bar[AC_NS];
   const Dims& d = a.d;
-  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
   const int i0 = blockIdx.x * TXW, j0 = blockIdx.y * BY;
   const int i = i0 + tx, j = j0 + ty;
   const int k0 = blockIdx.z * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
+  const int np = k1 - k0;
   const bool own = (i < d.nx) && (j < d.ny);
   const long long PS = d.PS;
   const long long oc = (long long)(j + G) * d.PX + (i + G);
-  const long long ot = (long long)(j0 + G) * d.PX + (i0 + G);
   const float* __restrict__ qz = a.qz;
   const int Wl = a.W;
   const bool lx = Wl > 0 && CpmlIdx::in(i, d.nx, Wl, true);
   const bool ly = Wl > 0 && CpmlIdx::in(j, d.ny, Wl, true);
 
+  if (tid == 0) {
+    for (int s = 0; s < AC_NS; ++s) mbar_init(&bar[s], 1);
+    mbar_fence_init();
+  }
+  __syncthreads();
+  if (tid == 0) {
+    for (int s = 0; s < AC_NS && s < np; ++s) {
+      mbar_expect_tx(&bar[s], TX_BYTES);
+      tma_load_3d(sm + s * STAGE, &a.mqx, &bar[s], i0, j0 + G, k0 + s + G);
+      tma_load_3d(sm + s * STAGE + TQX, &a.mqy, &bar[s], i0 + G, j0, k0 + s + G);
+    }
+  }
   float s0, s1, s2, s3, s4, s5, s6, s7;  // q_z at k-4 .. k+3
   s0 = __ldg(qz + (long long)(k0 - 4 + G) * PS + oc);
   s1 = __ldg(qz + (long long)(k0 - 3 + G) * PS + oc);
@@ -176,21 +227,30 @@ __global__ void __launch_bounds__(TXW * BY) ac_p_kernel(const AcPArgs a) {
   s4 = __ldg(qz + (long long)(k0 + G) * PS + oc);
   s5 = __ldg(qz + (long long)(k0 + 1 + G) * PS + oc);
   s6 = __ldg(qz + (long long)(k0 + 2 + G) * PS + oc);
+  float s7n = __ldg(qz + (long long)(k0 + 3 + G) * PS + oc);
+  float pn = 0.f, kn = 0.f;
+  if (own && np > 0) {
+    const long long o = (long long)(k0 + G) * PS + oc;
+    pn = a.p[o];
+    kn = __ldg(a.kdt + o);
+  }
 
-  for (int k = k0; k < k1; ++k) {
+  for (int it = 0; it < np; ++it) {
+    const int k = k0 + it;
+    const int s = it % AC_NS;
     const long long o = (long long)(k + G) * PS + oc;
-    s7 = __ldg(qz + o + 3 * PS);
-    float pv = 0.f, kv = 0.f;
-    if (own) {
-      pv = a.p[o];
-      kv = __ldg(a.kdt + o);
+    s7 = s7n;
+    const float pv = pn, kv = kn;
+    if (it + 1 < np) {
+      s7n = __ldg(qz + o + 4 * PS);
+      if (own) {
+        pn = a.p[o + PS];
+        kn = __ldg(a.kdt + o + PS);
+      }
     }
-    const long long op = (long long)(k + G) * PS + ot;
-    load_tile<BY, 4, 0>(sx, a.qx, op, d.PX);
-    load_tile<BY, 0, 4>(sy, a.qy, op, d.PX);
-    __syncthreads();
-    const float* cx = sx + ty * WX + tx + 4;
-    const float* cy = sy + (ty + 4) * TXW + tx;
+    mbar_wait(&bar[s], (it / AC_NS) & 1);
+    const float* cx = sm + s * STAGE + ty * WX + tx + 4;
+    const float* cy = sm + s * STAGE + TQX + (ty + 4) * TXW + tx;
     float dx = SEIS_D1 * (cx[0] - cx[-1]);
     dx = fmaf(SEIS_D2, cx[1] - cx[-2], dx);
     dx = fmaf(SEIS_D3, cx[2] - cx[-3], dx);
@@ -231,6 +291,12 @@ __global__ void __launch_bounds__(TXW * BY) ac_p_kernel(const AcPArgs a) {
       if (SNAP) a.snap[((long long)k * d.ny + j) * d.nx + i] = out;
     }
     __syncthreads();
+    if (tid == 0 && it + AC_NS < np) {
+      fence_proxy_async();
+      mbar_expect_tx(&bar[s], TX_BYTES);
+      tma_load_3d(sm + s * STAGE, &a.mqx, &bar[s], i0, j0 + G, k + AC_NS + G);
+      tma_load_3d(sm + s * STAGE + TQX, &a.mqy, &bar[s], i0 + G, j0, k + AC_NS + G);
+    }
     s0 = s1; s1 = s2; s2 = s3; s3 = s4; s4 = s5; s5 = s6; s6 = s7;
   }
 }

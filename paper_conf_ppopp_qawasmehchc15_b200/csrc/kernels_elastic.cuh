@@ -79,7 +79,14 @@ __device__ __forceinline__ float zminus(const float* q) {
   return fmaf(SEIS_D4, q[7] - q[0], r);
 }
 
+constexpr int EL_NS = 3;
+
 struct ElVArgs {
+  CUtensorMap msxx;  // box 40 x BY      (x halo)
+  CUtensorMap msxy;  // box 40 x (BY+8)  (x and y halos)
+  CUtensorMap msxz;  // box 40 x BY
+  CUtensorMap msyy;  // box 32 x (BY+8)  (y halo)
+  CUtensorMap msyz;  // box 32 x (BY+8)
   float* f[9];
   const float* __restrict__ bx;
   const float* __restrict__ by;
@@ -92,29 +99,48 @@ struct ElVArgs {
 };
 
 template <int BY>
-__global__ void __launch_bounds__(TXW * BY) el_v_kernel(const ElVArgs a) {
+__global__ void __launch_bounds__(TXW * BY) el_v_kernel(const __grid_constant__ ElVArgs a) {
   constexpr int WX = TXW + 8;
-  __shared__ float t_sxx[BY * WX];          // x halo
-  __shared__ float t_sxy[(BY + 8) * WX];    // x and y halos
-  __shared__ float t_sxz[BY * WX];          // x halo
-  __shared__ float t_syy[(BY + 8) * TXW];   // y halo
-  __shared__ float t_syz[(BY + 8) * TXW];   // y halo
+  constexpr int T_XX = BY * WX, T_XY = (BY + 8) * WX, T_XZ = BY * WX, T_YY = (BY + 8) * TXW,
+                T_YZ = (BY + 8) * TXW;
+  constexpr int O_XY = T_XX, O_XZ = O_XY + T_XY, O_YY = O_XZ + T_XZ, O_YZ = O_YY + T_YY;
+  constexpr int STAGE = O_YZ + T_YZ;
+  constexpr uint32_t TX_BYTES = STAGE * 4;
+  static_assert((T_XX % 32) == 0 && (T_XY % 32) == 0 && (T_YY % 32) == 0, "128-byte tiles");
+  __shared__ __align__(128) float sm[EL_NS * STAGE];
+  __shared__ __align__(8) uint64_t bar[EL_NS];
   const Dims& d = a.d;
-  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
   const int i0 = blockIdx.x * TXW, j0 = blockIdx.y * BY;
   const int i = i0 + tx, j = j0 + ty;
   const int k0 = blockIdx.z * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
+  const int np = k1 - k0;
   const bool own = (i < d.nx) && (j < d.ny);
   const long long PS = d.PS;
   const long long oc = (long long)(j + G) * d.PX + (i + G);
-  const long long ot = (long long)(j0 + G) * d.PX + (i0 + G);
   const int W = a.W;
   const bool lx = W > 0 && CpmlIdx::in(i, d.nx, W, true);
   const bool ly = W > 0 && CpmlIdx::in(j, d.ny, W, true);
   const float* __restrict__ sxz = a.f[ESXZ];
   const float* __restrict__ syz = a.f[ESYZ];
   const float* __restrict__ szz = a.f[ESZZ];
+  auto issue = [&](int s, int k) {
+    float* st = sm + s * STAGE;
+    mbar_expect_tx(&bar[s], TX_BYTES);
+    tma_load_3d(st, &a.msxx, &bar[s], i0, j0 + G, k + G);
+    tma_load_3d(st + O_XY, &a.msxy, &bar[s], i0, j0, k + G);
+    tma_load_3d(st + O_XZ, &a.msxz, &bar[s], i0, j0 + G, k + G);
+    tma_load_3d(st + O_YY, &a.msyy, &bar[s], i0 + G, j0, k + G);
+    tma_load_3d(st + O_YZ, &a.msyz, &bar[s], i0 + G, j0, k + G);
+  };
+  if (tid == 0) {
+    for (int s = 0; s < EL_NS; ++s) mbar_init(&bar[s], 1);
+    mbar_fence_init();
+  }
+  __syncthreads();
+  if (tid == 0)
+    for (int s = 0; s < EL_NS && s < np; ++s) issue(s, k0 + s);
   float qxz[8], qyz[8], qzz[8];  // sxz, syz at k-4..k+3 (D-); szz at k-3..k+4 (D+)
 #pragma unroll
   for (int t = 0; t < 7; ++t) {
@@ -122,24 +148,38 @@ __global__ void __launch_bounds__(TXW * BY) el_v_kernel(const ElVArgs a) {
     qyz[t] = __ldg(syz + (long long)(k0 - 4 + t + G) * PS + oc);
     qzz[t] = __ldg(szz + (long long)(k0 - 3 + t + G) * PS + oc);
   }
-  for (int k = k0; k < k1; ++k) {
+  float nxz = __ldg(sxz + (long long)(k0 + 3 + G) * PS + oc);
+  float nyz = __ldg(syz + (long long)(k0 + 3 + G) * PS + oc);
+  float nzz = __ldg(szz + (long long)(k0 + 4 + G) * PS + oc);
+  float nv[3] = {0.f, 0.f, 0.f}, nb[3] = {0.f, 0.f, 0.f};
+  if (own && np > 0) {
+    const long long o = (long long)(k0 + G) * PS + oc;
+    nv[0] = a.f[EVX][o]; nv[1] = a.f[EVY][o]; nv[2] = a.f[EVZ][o];
+    nb[0] = __ldg(a.bx + o); nb[1] = __ldg(a.by + o); nb[2] = __ldg(a.bz + o);
+  }
+  for (int it = 0; it < np; ++it) {
+    const int k = k0 + it;
+    const int s = it % EL_NS;
     const long long o = (long long)(k + G) * PS + oc;
-    qxz[7] = __ldg(sxz + o + 3 * PS);
-    qyz[7] = __ldg(syz + o + 3 * PS);
-    qzz[7] = __ldg(szz + o + 4 * PS);
-    const long long op = (long long)(k + G) * PS + ot;
-    load_tile<BY, 4, 0>(t_sxx, a.f[ESXX], op, d.PX);
-    load_tile<BY, 4, 4>(t_sxy, a.f[ESXY], op, d.PX);
-    load_tile<BY, 4, 0>(t_sxz, a.f[ESXZ], op, d.PX);
-    load_tile<BY, 0, 4>(t_syy, a.f[ESYY], op, d.PX);
-    load_tile<BY, 0, 4>(t_syz, a.f[ESYZ], op, d.PX);
-    __syncthreads();
+    qxz[7] = nxz; qyz[7] = nyz; qzz[7] = nzz;
+    const float v0 = nv[0], v1 = nv[1], v2 = nv[2], b0 = nb[0], b1 = nb[1], b2 = nb[2];
+    if (it + 1 < np) {
+      nxz = __ldg(sxz + o + 4 * PS);
+      nyz = __ldg(syz + o + 4 * PS);
+      nzz = __ldg(szz + o + 5 * PS);
+      if (own) {
+        nv[0] = a.f[EVX][o + PS]; nv[1] = a.f[EVY][o + PS]; nv[2] = a.f[EVZ][o + PS];
+        nb[0] = __ldg(a.bx + o + PS); nb[1] = __ldg(a.by + o + PS); nb[2] = __ldg(a.bz + o + PS);
+      }
+    }
+    mbar_wait(&bar[s], (it / EL_NS) & 1);
     if (own) {
-      const float* cxx = t_sxx + ty * WX + tx + 4;
-      const float* cxy = t_sxy + (ty + 4) * WX + tx + 4;
-      const float* cxz = t_sxz + ty * WX + tx + 4;
-      const float* cyy = t_syy + (ty + 4) * TXW + tx;
-      const float* cyz = t_syz + (ty + 4) * TXW + tx;
+      const float* st = sm + s * STAGE;
+      const float* cxx = st + ty * WX + tx + 4;
+      const float* cxy = st + O_XY + (ty + 4) * WX + tx + 4;
+      const float* cxz = st + O_XZ + ty * WX + tx + 4;
+      const float* cyy = st + O_YY + (ty + 4) * TXW + tx;
+      const float* cyz = st + O_YZ + (ty + 4) * TXW + tx;
       float d0 = dplus<1>(cxx), d1 = dminus<WX>(cxy), d2 = zminus(qxz);
       float d3 = dminus<1>(cxy), d4 = dplus<TXW>(cyy), d5 = zminus(qyz);
       float d6 = dminus<1>(cxz), d7 = dminus<TXW>(cyz), d8 = zplus(qzz);
@@ -161,11 +201,15 @@ __global__ void __launch_bounds__(TXW * BY) el_v_kernel(const ElVArgs a) {
           cpml_z(d8, a.psi[8], d, W, i, j, gz, a.cz.ah, a.cz.bh);
         }
       }
-      a.f[EVX][o] = fmaf(__ldg(a.bx + o), (d0 + d1) + d2, a.f[EVX][o]);
-      a.f[EVY][o] = fmaf(__ldg(a.by + o), (d3 + d4) + d5, a.f[EVY][o]);
-      a.f[EVZ][o] = fmaf(__ldg(a.bz + o), (d6 + d7) + d8, a.f[EVZ][o]);
+      a.f[EVX][o] = fmaf(b0, (d0 + d1) + d2, v0);
+      a.f[EVY][o] = fmaf(b1, (d3 + d4) + d5, v1);
+      a.f[EVZ][o] = fmaf(b2, (d6 + d7) + d8, v2);
     }
     __syncthreads();
+    if (tid == 0 && it + EL_NS < np) {
+      fence_proxy_async();
+      issue(s, k + EL_NS);
+    }
 #pragma unroll
     for (int t = 0; t < 7; ++t) {
       qxz[t] = qxz[t + 1];
@@ -176,6 +220,9 @@ __global__ void __launch_bounds__(TXW * BY) el_v_kernel(const ElVArgs a) {
 }
 
 struct ElSArgs {
+  CUtensorMap mvx;  // box 40 x (BY+8)
+  CUtensorMap mvy;
+  CUtensorMap mvz;
   float* f[9];
   const float* __restrict__ l2m;  // dt (lam + 2 mu) / h
   const float* __restrict__ lam;  // dt lam / h
@@ -192,27 +239,43 @@ struct ElSArgs {
 };
 
 template <int BY, bool UNUSED>
-__global__ void __launch_bounds__(TXW * BY) el_s_kernel(const ElSArgs a) {
+__global__ void __launch_bounds__(TXW * BY) el_s_kernel(const __grid_constant__ ElSArgs a) {
   constexpr int WX = TXW + 8;
-  __shared__ float t_vx[(BY + 8) * WX];
-  __shared__ float t_vy[(BY + 8) * WX];
-  __shared__ float t_vz[(BY + 8) * WX];
+  constexpr int TV = (BY + 8) * WX;
+  constexpr int STAGE = 3 * TV;
+  constexpr uint32_t TX_BYTES = STAGE * 4;
+  __shared__ __align__(128) float sm[EL_NS * STAGE];
+  __shared__ __align__(8) uint64_t bar[EL_NS];
   const Dims& d = a.d;
-  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
   const int i0 = blockIdx.x * TXW, j0 = blockIdx.y * BY;
   const int i = i0 + tx, j = j0 + ty;
   const int k0 = blockIdx.z * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
+  const int np = k1 - k0;
   const bool own = (i < d.nx) && (j < d.ny);
   const long long PS = d.PS;
   const long long oc = (long long)(j + G) * d.PX + (i + G);
-  const long long ot = (long long)(j0 + G) * d.PX + (i0 + G);
   const int W = a.W;
   const bool lx = W > 0 && CpmlIdx::in(i, d.nx, W, true);
   const bool ly = W > 0 && CpmlIdx::in(j, d.ny, W, true);
   const float* __restrict__ vx = a.f[EVX];
   const float* __restrict__ vy = a.f[EVY];
   const float* __restrict__ vz = a.f[EVZ];
+  auto issue = [&](int s, int k) {
+    float* st = sm + s * STAGE;
+    mbar_expect_tx(&bar[s], TX_BYTES);
+    tma_load_3d(st, &a.mvx, &bar[s], i0, j0, k + G);
+    tma_load_3d(st + TV, &a.mvy, &bar[s], i0, j0, k + G);
+    tma_load_3d(st + 2 * TV, &a.mvz, &bar[s], i0, j0, k + G);
+  };
+  if (tid == 0) {
+    for (int s = 0; s < EL_NS; ++s) mbar_init(&bar[s], 1);
+    mbar_fence_init();
+  }
+  __syncthreads();
+  if (tid == 0)
+    for (int s = 0; s < EL_NS && s < np; ++s) issue(s, k0 + s);
   float qx[8], qy[8], qz[8];  // vx, vy at k-3..k+4 (D+); vz at k-4..k+3 (D-)
 #pragma unroll
   for (int t = 0; t < 7; ++t) {
@@ -220,21 +283,34 @@ __global__ void __launch_bounds__(TXW * BY) el_s_kernel(const ElSArgs a) {
     qy[t] = __ldg(vy + (long long)(k0 - 3 + t + G) * PS + oc);
     qz[t] = __ldg(vz + (long long)(k0 - 4 + t + G) * PS + oc);
   }
-  for (int k = k0; k < k1; ++k) {
+  float nqx = __ldg(vx + (long long)(k0 + 4 + G) * PS + oc);
+  float nqy = __ldg(vy + (long long)(k0 + 4 + G) * PS + oc);
+  float nqz = __ldg(vz + (long long)(k0 + 3 + G) * PS + oc);
+  for (int it = 0; it < np; ++it) {
+    const int k = k0 + it;
+    const int s = it % EL_NS;
     const long long o = (long long)(k + G) * PS + oc;
-    qx[7] = __ldg(vx + o + 4 * PS);
-    qy[7] = __ldg(vy + o + 4 * PS);
-    qz[7] = __ldg(vz + o + 3 * PS);
-    const long long op = (long long)(k + G) * PS + ot;
-    load_tile<BY, 4, 4>(t_vx, vx, op, d.PX);
-    load_tile<BY, 4, 4>(t_vy, vy, op, d.PX);
-    load_tile<BY, 4, 4>(t_vz, vz, op, d.PX);
-    __syncthreads();
+    qx[7] = nqx; qy[7] = nqy; qz[7] = nqz;
+    if (it + 1 < np) {
+      nqx = __ldg(vx + o + 5 * PS);
+      nqy = __ldg(vy + o + 5 * PS);
+      nqz = __ldg(vz + o + 4 * PS);
+    }
+    float sxx = 0.f, syy = 0.f, szz = 0.f, sxy = 0.f, sxz = 0.f, syz = 0.f;
+    float l2m = 0.f, lam = 0.f, mxy = 0.f, mxz = 0.f, myz = 0.f;
+    if (own) {
+      sxx = a.f[ESXX][o]; syy = a.f[ESYY][o]; szz = a.f[ESZZ][o];
+      sxy = a.f[ESXY][o]; sxz = a.f[ESXZ][o]; syz = a.f[ESYZ][o];
+      l2m = __ldg(a.l2m + o); lam = __ldg(a.lam + o);
+      mxy = __ldg(a.mxy + o); mxz = __ldg(a.mxz + o); myz = __ldg(a.myz + o);
+    }
+    mbar_wait(&bar[s], (it / EL_NS) & 1);
     if (own) {
       const int gz = k + d.z0;
-      const float* cvx = t_vx + (ty + 4) * WX + tx + 4;
-      const float* cvy = t_vy + (ty + 4) * WX + tx + 4;
-      const float* cvz = t_vz + (ty + 4) * WX + tx + 4;
+      const float* st = sm + s * STAGE;
+      const float* cvx = st + (ty + 4) * WX + tx + 4;
+      const float* cvy = st + TV + (ty + 4) * WX + tx + 4;
+      const float* cvz = st + 2 * TV + (ty + 4) * WX + tx + 4;
       float exx = dminus<1>(cvx), eyy = dminus<WX>(cvy), ezz = zminus(qz);
       float dyvx = dplus<WX>(cvx), dxvy = dplus<1>(cvy);
       float dzvx = zplus(qx), dxvz = dplus<1>(cvz);
@@ -256,10 +332,8 @@ __global__ void __launch_bounds__(TXW * BY) el_s_kernel(const ElSArgs a) {
           cpml_z(dzvy, a.psi[7], d, W, i, j, gz, a.cz.ah, a.cz.bh);
         }
       }
-      const float l2m = __ldg(a.l2m + o), lam = __ldg(a.lam + o);
       const bool surf = a.fs && gz == 0;
       if (surf) ezz = -(lam / l2m) * (exx + eyy);  // O16 surface row
-      float sxx = a.f[ESXX][o], syy = a.f[ESYY][o], szz = a.f[ESZZ][o];
       sxx += fmaf(l2m, exx, lam * (eyy + ezz));
       syy += fmaf(l2m, eyy, lam * (exx + ezz));
       szz += fmaf(l2m, ezz, lam * (exx + eyy));
@@ -272,11 +346,15 @@ __global__ void __launch_bounds__(TXW * BY) el_s_kernel(const ElSArgs a) {
       a.f[ESXX][o] = sxx;
       a.f[ESYY][o] = syy;
       a.f[ESZZ][o] = szz;
-      a.f[ESXY][o] = fmaf(__ldg(a.mxy + o), dyvx + dxvy, a.f[ESXY][o]);
-      a.f[ESXZ][o] = fmaf(__ldg(a.mxz + o), dzvx + dxvz, a.f[ESXZ][o]);
-      a.f[ESYZ][o] = fmaf(__ldg(a.myz + o), dzvy + dyvz, a.f[ESYZ][o]);
+      a.f[ESXY][o] = fmaf(mxy, dyvx + dxvy, sxy);
+      a.f[ESXZ][o] = fmaf(mxz, dzvx + dxvz, sxz);
+      a.f[ESYZ][o] = fmaf(myz, dzvy + dyvz, syz);
     }
     __syncthreads();
+    if (tid == 0 && it + EL_NS < np) {
+      fence_proxy_async();
+      issue(s, k + EL_NS);
+    }
 #pragma unroll
     for (int t = 0; t < 7; ++t) {
       qx[t] = qx[t + 1];

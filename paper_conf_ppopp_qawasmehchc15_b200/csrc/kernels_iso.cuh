@@ -4,19 +4,22 @@
 //   m = v^2 dt^2 / h^2 (per point, precomputed),  eta dt = edx[i] + edy[j] + edz[k]
 //   Lambda u = 3 c0 u + sum_m c_m sum_axes (u_{+m} + u_{-m})         (O1, O3, O6)
 //
-// One thread per (x, y) column marching down a z-chunk (2.5D blocking): the
-// x/y neighbours of plane k come from a shared-memory tile (halo 4), the
-// z neighbours from a 9-deep register queue.  u^{n+1} overwrites u^{n-1} in
-// place ("logically swapping t_n and t_{n+1} arrays").  HBM traffic per
-// point: read u^n, u^{n-1}, m; write u^{n+1} = 16 B (+4 B snapshot, +12 B imaging).
-// Fused epilogues: source injection, snapshot store (O14),
-// imaging I += S_j * u^n on the input level (O15).
+// One thread per (x, y) column marching down a z-chunk (2.5D blocking).  The
+// x/y neighbours of plane k come from a shared-memory tile (halo 4) brought in
+// by TMA through an NS-stage mbarrier ring; the z neighbours from a 9-deep
+// register queue fed by a coalesced stream prefetched one plane ahead, like
+// u^{n-1} and m.  u^{n+1} overwrites u^{n-1} in place ("logically
+// swapping t_n and t_{n+1} arrays").  HBM traffic per point: read u^n, u^{n-1},
+// m; write u^{n+1} = 16 B (+4 B snapshot, +12 B imaging).  Fused epilogues:
+// source injection, snapshot store (O14), imaging
+// I += S_j * u^n on the input level (O15).
 #pragma once
 #include "common.cuh"
 
 namespace seis {
 
 struct IsoArgs {
+  CUtensorMap mun;               // u^n, box (32+8) x (BY+8) x 1
   const float* __restrict__ un;  // u^n (padded)
   float* __restrict__ up;        // in: u^{n-1}; out: u^{n+1}
   const float* __restrict__ m;   // v^2 dt^2 / h^2 (padded)
@@ -32,23 +35,40 @@ struct IsoArgs {
   float* __restrict__ img;       // compact image (+=), or nullptr
 };
 
+constexpr int ISO_NS = 4;
+
 template <int BY, bool SNAP, bool IMG>
-__global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const IsoArgs a) {
+__global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const __grid_constant__ IsoArgs a) {
   constexpr int W = TXW + 8;
-  __shared__ float s[(BY + 8) * W];
+  constexpr int TILE = (BY + 8) * W;  // floats per stage (multiple of 32)
+  constexpr uint32_t TX_BYTES = TILE * 4;
+  __shared__ __align__(128) float sm[ISO_NS * TILE];
+  __shared__ __align__(8) uint64_t bar[ISO_NS];
   const Dims& d = a.d;
-  const int tx = threadIdx.x, ty = threadIdx.y;
+  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
   const int i0 = blockIdx.x * TXW, j0 = blockIdx.y * BY;
   const int i = i0 + tx, j = j0 + ty;
   const int k0 = blockIdx.z * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
+  const int np = k1 - k0;
   const bool own = (i < d.nx) && (j < d.ny);
   const long long PS = d.PS;
   const long long oc = (long long)(j + G) * d.PX + (i + G);
-  const long long ot = (long long)(j0 + G) * d.PX + (i0 + G);
   const float* __restrict__ un = a.un;
 
-  float q0, q1, q2, q3, q4, q5, q6, q7, q8;  // u^n at k-4 .. k+4
+  if (tid == 0) {
+    for (int s = 0; s < ISO_NS; ++s) mbar_init(&bar[s], 1);
+    mbar_fence_init();
+  }
+  __syncthreads();
+  if (tid == 0) {
+    for (int s = 0; s < ISO_NS && s < np; ++s) {
+      mbar_expect_tx(&bar[s], TX_BYTES);
+      tma_load_3d(sm + s * TILE, &a.mun, &bar[s], i0, j0, k0 + s + G);
+    }
+  }
+  // z-queue u^n(k-4 .. k+4) and the one-plane-ahead streams
+  float q0, q1, q2, q3, q4, q5, q6, q7, q8;
   q0 = __ldg(un + (long long)(k0 - 4 + G) * PS + oc);
   q1 = __ldg(un + (long long)(k0 - 3 + G) * PS + oc);
   q2 = __ldg(un + (long long)(k0 - 2 + G) * PS + oc);
@@ -57,26 +77,39 @@ __global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const IsoArgs a) {
   q5 = __ldg(un + (long long)(k0 + 1 + G) * PS + oc);
   q6 = __ldg(un + (long long)(k0 + 2 + G) * PS + oc);
   q7 = __ldg(un + (long long)(k0 + 3 + G) * PS + oc);
-  const float ex = (a.edx && own) ? a.edx[i] + a.edy[j] : 0.0f;
-
-  for (int k = k0; k < k1; ++k) {
-    const long long o = (long long)(k + G) * PS + oc;
-    q8 = __ldg(un + o + 4 * PS);
-    float upv = 0.0f, mv = 0.0f;
-    if (own) {
-      upv = a.up[o];
-      mv = __ldg(a.m + o);
+  float q8n = __ldg(un + (long long)(k0 + 4 + G) * PS + oc);
+  float upn = 0.f, mn = 0.f;
+  {
+    const long long o = (long long)(k0 + G) * PS + oc;
+    if (own && np > 0) {
+      upn = a.up[o];
+      mn = __ldg(a.m + o);
     }
-    load_tile<BY, 4, 4>(s, un, (long long)(k + G) * PS + ot, d.PX);
-    __syncthreads();
-    const float* c = s + (ty + 4) * W + tx + 4;
+  }
+  const float exy = (a.edx && own) ? a.edx[i] + a.edy[j] : 0.0f;
+
+  for (int it = 0; it < np; ++it) {
+    const int k = k0 + it;
+    const int s = it % ISO_NS;
+    const long long o = (long long)(k + G) * PS + oc;
+    q8 = q8n;
+    const float upv = upn, mv = mn;
+    if (it + 1 < np) {
+      q8n = __ldg(un + o + 5 * PS);
+      if (own) {
+        upn = a.up[o + PS];
+        mn = __ldg(a.m + o + PS);
+      }
+    }
+    mbar_wait(&bar[s], (it / ISO_NS) & 1);
+    const float* c = sm + s * TILE + (ty + 4) * W + tx + 4;
     float lap = (3.0f * SEIS_C0) * q4;
     lap = fmaf(SEIS_C1, (c[-1] + c[1]) + (c[-W] + c[W]) + (q3 + q5), lap);
     lap = fmaf(SEIS_C2, (c[-2] + c[2]) + (c[-2 * W] + c[2 * W]) + (q2 + q6), lap);
     lap = fmaf(SEIS_C3, (c[-3] + c[3]) + (c[-3 * W] + c[3 * W]) + (q1 + q7), lap);
     lap = fmaf(SEIS_C4, (c[-4] + c[4]) + (c[-4 * W] + c[4 * W]) + (q0 + q8), lap);
     if (own) {
-      const float e = a.edx ? ex + a.edz[k + d.z0] : 0.0f;
+      const float e = a.edx ? exy + a.edz[k + d.z0] : 0.0f;
       float out;
       if (e != 0.0f) {
         out = (2.0f * q4 - (1.0f - e) * upv + mv * lap) / (1.0f + e);
@@ -91,7 +124,12 @@ __global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const IsoArgs a) {
         if (IMG) a.img[cix] = fmaf(__ldg(a.imgS + cix), q4, a.img[cix]);
       }
     }
-    __syncthreads();
+    __syncthreads();  // every thread is done with stage s
+    if (tid == 0 && it + ISO_NS < np) {
+      fence_proxy_async();
+      mbar_expect_tx(&bar[s], TX_BYTES);
+      tma_load_3d(sm + s * TILE, &a.mun, &bar[s], i0, j0, k + ISO_NS + G);
+    }
     q0 = q1; q1 = q2; q2 = q3; q3 = q4; q4 = q5; q5 = q6; q6 = q7; q7 = q8;
   }
 }

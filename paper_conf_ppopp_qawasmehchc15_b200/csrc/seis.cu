@@ -5,6 +5,8 @@
 // C-PML slabs, the HBM snapshot pool), drives Algorithm 1 on the
 // caller's stream, and exchanges the 4 ghost planes between z-slabs:
 // cudaMemcpyAsync between slabs of one process, NCCL send/recv between ranks.
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 #include <nccl.h>
 
@@ -104,7 +106,8 @@ struct seis_comm {
 
 namespace {
 
-constexpr int BY = 16;       // tile rows (block = 32 x BY threads)
+constexpr int BY = 16;       // tile rows (block = 32 x BY threads), ISO and ACOUSTIC
+constexpr int BYE = 8;       // tile rows of the ELASTIC kernels (more registers per thread)
 constexpr int NPSI = 18;
 
 struct Slab {
@@ -115,6 +118,10 @@ struct Slab {
   float *bx = nullptr, *by = nullptr, *bz = nullptr;                          // ACOUSTIC, ELASTIC
   float *l2m = nullptr, *lam = nullptr, *mxy = nullptr, *mxz = nullptr, *myz = nullptr;  // ELASTIC
   float* psi[NPSI] = {};
+  // TMA descriptors of the plane tiles each kernel stages
+  CUtensorMap mu[2];                                   // ISO u (both time levels)
+  CUtensorMap mp, mqx, mqy;                            // ACOUSTIC
+  CUtensorMap msxx, msxy, msxz, msyy, msyz, mvx, mvy, mvz;  // ELASTIC
   int cur = 0;               // ISO: fld[cur] = u^n
   int zc = 1, nzch = 1;      // z-chunking of the stencil launches
   // shot tables
@@ -190,6 +197,28 @@ seis_status alloc_padded(seis_model* M, const Dims& d, float** out, cudaStream_t
 
 int roundup(int a, int b) { return (a + b - 1) / b * b; }
 
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda link).
+PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
+
+seis_status make_map(CUtensorMap* m, float* base, const Dims& d, int bw, int bh) {
+  if (!g_encode) {
+    cudaDriverEntryPointQueryResult q;
+    void* fn = nullptr;
+    CK(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q));
+    if (q != cudaDriverEntryPointSuccess || !fn) return fail(SEIS_ECUDA, "cuTensorMapEncodeTiled unavailable");
+    g_encode = (PFN_cuTensorMapEncodeTiled_v12000)fn;
+  }
+  cuuint64_t dims[3] = {(cuuint64_t)d.PX, (cuuint64_t)d.PY, (cuuint64_t)(d.nzl + 2 * G)};
+  cuuint64_t str[2] = {(cuuint64_t)d.PX * 4, (cuuint64_t)d.PS * 4};
+  cuuint32_t box[3] = {(cuuint32_t)bw, (cuuint32_t)bh, 1};
+  cuuint32_t es[3] = {1, 1, 1};
+  CUresult r = g_encode(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, base, dims, str, box, es,
+                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                        CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(SEIS_ECUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+  return SEIS_OK;
+}
+
 Dims make_dims(const seis_grid& g, int z0, int nzl) {
   Dims d;
   d.nx = g.nx;
@@ -260,8 +289,8 @@ seis_status upload_padded_from_host(seis_model* M, const Dims& d, const std::vec
 }
 
 // Choose the z-chunk so the launch fills the machine in whole waves.
-void choose_chunks(Slab& s, int resident_per_sm, int nsm) {
-  const int bxy = ((s.d.nx + TXW - 1) / TXW) * ((s.d.ny + BY - 1) / BY);
+void choose_chunks(Slab& s, int resident_per_sm, int nsm, int by) {
+  const int bxy = ((s.d.nx + TXW - 1) / TXW) * ((s.d.ny + by - 1) / by);
   const long long slots = (long long)std::max(1, resident_per_sm) * nsm;
   double best = 1e300;
   int bestc = 1;
@@ -652,14 +681,32 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
         }
       }
     }
+    // TMA descriptors
+    if (kind == SEIS_ISO) {
+      TRY(make_map(&S.mu[0], S.fld[0], d, TXW + 8, BY + 8));
+      TRY(make_map(&S.mu[1], S.fld[1], d, TXW + 8, BY + 8));
+    } else if (kind == SEIS_ACOUSTIC) {
+      TRY(make_map(&S.mp, S.fld[0], d, TXW + 8, BY + 8));
+      TRY(make_map(&S.mqx, S.fld[1], d, TXW + 8, BY));
+      TRY(make_map(&S.mqy, S.fld[2], d, TXW, BY + 8));
+    } else {
+      TRY(make_map(&S.mvx, S.fld[EVX], d, TXW + 8, BYE + 8));
+      TRY(make_map(&S.mvy, S.fld[EVY], d, TXW + 8, BYE + 8));
+      TRY(make_map(&S.mvz, S.fld[EVZ], d, TXW + 8, BYE + 8));
+      TRY(make_map(&S.msxx, S.fld[ESXX], d, TXW + 8, BYE));
+      TRY(make_map(&S.msxy, S.fld[ESXY], d, TXW + 8, BYE + 8));
+      TRY(make_map(&S.msxz, S.fld[ESXZ], d, TXW + 8, BYE));
+      TRY(make_map(&S.msyy, S.fld[ESYY], d, TXW, BYE + 8));
+      TRY(make_map(&S.msyz, S.fld[ESYZ], d, TXW, BYE + 8));
+    }
     int occ = 1;
     if (kind == SEIS_ISO)
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, iso_step_kernel<BY, false, false>, TXW * BY, 0);
     else if (kind == SEIS_ACOUSTIC)
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_v_kernel<BY, false>, TXW * BY, 0);
     else
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BY, false>, TXW * BY, 0);
-    choose_chunks(S, occ, dev_sms);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, TXW * BYE, 0);
+    choose_chunks(S, occ, dev_sms, kind == SEIS_ELASTIC ? BYE : BY);
   }
   CK(cudaStreamSynchronize(st));
   return SEIS_OK;
@@ -874,8 +921,8 @@ seis_status fs_mirror(seis_model* M, std::initializer_list<int> fields, cudaStre
   return SEIS_OK;
 }
 
-dim3 grid_of(const Slab& S) {
-  return dim3((S.d.nx + TXW - 1) / TXW, (S.d.ny + BY - 1) / BY, S.nzch);
+dim3 grid_of(const Slab& S, int by = BY) {
+  return dim3((S.d.nx + TXW - 1) / TXW, (S.d.ny + by - 1) / by, S.nzch);
 }
 
 // Backward-phase receiver injection into the field just produced (before its
@@ -903,6 +950,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (size_t s = 0; s < M->slabs.size(); ++s) {
       Slab& S = M->slabs[s];
       IsoArgs a;
+      a.mun = S.mu[S.cur];
       a.un = S.fld[S.cur];
       a.up = S.fld[1 - S.cur];
       a.m = S.m;
@@ -937,6 +985,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (size_t s = 0; s < M->slabs.size(); ++s) {
       Slab& S = M->slabs[s];
       AcVArgs a;
+      a.mp = S.mp;
       a.p = S.fld[0];
       a.qx = S.fld[1];
       a.qy = S.fld[2];
@@ -968,9 +1017,9 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (size_t s = 0; s < M->slabs.size(); ++s) {
       Slab& S = M->slabs[s];
       AcPArgs a;
+      a.mqx = S.mqx;
+      a.mqy = S.mqy;
       a.p = S.fld[0];
-      a.qx = S.fld[1];
-      a.qy = S.fld[2];
       a.qz = S.fld[3];
       a.kdt = S.kdt;
       a.W = M->W;
@@ -1003,6 +1052,11 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
   for (size_t s = 0; s < M->slabs.size(); ++s) {
     Slab& S = M->slabs[s];
     ElVArgs a;
+    a.msxx = S.msxx;
+    a.msxy = S.msxy;
+    a.msxz = S.msxz;
+    a.msyy = S.msyy;
+    a.msyz = S.msyz;
     for (int t = 0; t < 9; ++t) a.f[t] = S.fld[t];
     a.bx = S.bx;
     a.by = S.by;
@@ -1016,10 +1070,10 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (int t = 0; t < 9; ++t) a.psi[t] = S.psi[t];
     a.d = S.d;
     a.zc = S.zc;
-    const dim3 gr = grid_of(S);
+    const dim3 gr = grid_of(S, BYE);
     {
       PROF(3, st);
-      el_v_kernel<BY><<<gr, blk, 0, st>>>(a);
+      el_v_kernel<BYE><<<gr, dim3(TXW, BYE), 0, st>>>(a);
     }
     CKL();
   }
@@ -1028,6 +1082,9 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
   for (size_t s = 0; s < M->slabs.size(); ++s) {
     Slab& S = M->slabs[s];
     ElSArgs a;
+    a.mvx = S.mvx;
+    a.mvy = S.mvy;
+    a.mvz = S.mvz;
     for (int t = 0; t < 9; ++t) a.f[t] = S.fld[t];
     a.l2m = S.l2m;
     a.lam = S.lam;
@@ -1046,10 +1103,10 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     a.src_o = with_src ? S.src_o : -1;
     a.src_amp = 0.f;
     if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
-    const dim3 gr = grid_of(S);
+    const dim3 gr = grid_of(S, BYE);
     {
       PROF(4, st);
-      el_s_kernel<BY, false><<<gr, blk, 0, st>>>(a);
+      el_s_kernel<BYE, false><<<gr, dim3(TXW, BYE), 0, st>>>(a);
     }
     CKL();
   }
