@@ -88,6 +88,9 @@ struct CpmlIdx {
 
 namespace seis {
 
+__device__ __forceinline__ float* align128(float* p) {
+  return reinterpret_cast<float*>((reinterpret_cast<uintptr_t>(p) + 127) & ~uintptr_t(127));
+}
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }

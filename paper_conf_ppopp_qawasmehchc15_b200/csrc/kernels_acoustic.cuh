@@ -28,14 +28,13 @@ struct CpmlAxis {
 constexpr int AC_NS = 4;
 
 struct AcVArgs {
-  CUtensorMap mp;                 // p, box (32+8) x (BY+8) x 1
+  CUtensorMap mp;                 // p tile, box (32+8) x (BY+8) x 1
+  CUtensorMap mqx, mqy, mqz;      // q, box 32 x BY x 1
+  CUtensorMap mbx, mby, mbz;      // face buoyancy, box 32 x BY x 1
   const float* __restrict__ p;
   float* __restrict__ qx;
   float* __restrict__ qy;
   float* __restrict__ qz;
-  const float* __restrict__ bx;  // dt * 2/(rho_i + rho_{i+1}) / h on x faces (padded)
-  const float* __restrict__ by;
-  const float* __restrict__ bz;
   int W;                          // C-PML slab width per face (nb + 1), 0 = no layer
   int zlo;                        // 1 if the top z face has a layer
   CpmlAxis cx, cy, cz;
@@ -48,12 +47,21 @@ struct AcVArgs {
   float* __restrict__ img;
 };
 
+template <int BY>
+struct AcVStage {
+  static constexpr int W = TXW + 8, T = TXW * BY;
+  static constexpr int P = 0, QX = (BY + 8) * W, QY = QX + T, QZ = QY + T, BX = QZ + T, BYo = BX + T,
+                       BZ = BYo + T, SIZE = BZ + T;
+  static constexpr size_t smem_bytes() { return (size_t)AC_NS * SIZE * 4 + 128; }
+};
+
 template <int BY, bool IMG>
 __global__ void __launch_bounds__(TXW * BY) ac_v_kernel(const __grid_constant__ AcVArgs a) {
-  constexpr int W = TXW + 8;
-  constexpr int TILE = (BY + 8) * W;
-  constexpr uint32_t TX_BYTES = TILE * 4;
-  __shared__ __align__(128) float sm[AC_NS * TILE];
+  using L = AcVStage<BY>;
+  constexpr int W = L::W;
+  constexpr uint32_t TX_BYTES = L::SIZE * 4;
+  extern __shared__ __align__(128) float sm_raw[];
+  float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[AC_NS];
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
@@ -69,19 +77,26 @@ __global__ void __launch_bounds__(TXW * BY) ac_v_kernel(const __grid_constant__ 
   const int Wl = a.W;
   const bool lx = Wl > 0 && CpmlIdx::in(i, d.nx, Wl, true);
   const bool ly = Wl > 0 && CpmlIdx::in(j, d.ny, Wl, true);
-
+  auto issue = [&](int s, int k) {
+    float* st = sm + s * L::SIZE;
+    const int z = k + G, x = i0 + G, y = j0 + G;
+    mbar_expect_tx(&bar[s], TX_BYTES);
+    tma_load_3d(st + L::P, &a.mp, &bar[s], i0, j0, z);
+    tma_load_3d(st + L::QX, &a.mqx, &bar[s], x, y, z);
+    tma_load_3d(st + L::QY, &a.mqy, &bar[s], x, y, z);
+    tma_load_3d(st + L::QZ, &a.mqz, &bar[s], x, y, z);
+    tma_load_3d(st + L::BX, &a.mbx, &bar[s], x, y, z);
+    tma_load_3d(st + L::BYo, &a.mby, &bar[s], x, y, z);
+    tma_load_3d(st + L::BZ, &a.mbz, &bar[s], x, y, z);
+  };
   if (tid == 0) {
     for (int s = 0; s < AC_NS; ++s) mbar_init(&bar[s], 1);
     mbar_fence_init();
   }
   __syncthreads();
-  if (tid == 0) {
-    for (int s = 0; s < AC_NS && s < np; ++s) {
-      mbar_expect_tx(&bar[s], TX_BYTES);
-      tma_load_3d(sm + s * TILE, &a.mp, &bar[s], i0, j0, k0 + s + G);
-    }
-  }
-  float r0, r1, r2, r3, r4, r5, r6, r7;  // p at k-3 .. k+4
+  if (tid == 0)
+    for (int s = 0; s < AC_NS && s < np; ++s) issue(s, k0 + s);
+  float r0, r1, r2, r3, r4, r5, r6, r7;  // p at k-3 .. k+4, fed two planes ahead
   r0 = __ldg(p + (long long)(k0 - 3 + G) * PS + oc);
   r1 = __ldg(p + (long long)(k0 - 2 + G) * PS + oc);
   r2 = __ldg(p + (long long)(k0 - 1 + G) * PS + oc);
@@ -89,29 +104,19 @@ __global__ void __launch_bounds__(TXW * BY) ac_v_kernel(const __grid_constant__ 
   r4 = __ldg(p + (long long)(k0 + 1 + G) * PS + oc);
   r5 = __ldg(p + (long long)(k0 + 2 + G) * PS + oc);
   r6 = __ldg(p + (long long)(k0 + 3 + G) * PS + oc);
-  float r7n = __ldg(p + (long long)(k0 + 4 + G) * PS + oc);
-  float qxn = 0.f, qyn = 0.f, qzn = 0.f, bxn = 0.f, byn = 0.f, bzn = 0.f;
-  if (own && np > 0) {
-    const long long o = (long long)(k0 + G) * PS + oc;
-    qxn = a.qx[o]; qyn = a.qy[o]; qzn = a.qz[o];
-    bxn = __ldg(a.bx + o); byn = __ldg(a.by + o); bzn = __ldg(a.bz + o);
-  }
+  float na = __ldg(p + (long long)(k0 + 4 + G) * PS + oc);
+  float nb = np > 1 ? __ldg(p + (long long)(k0 + 5 + G) * PS + oc) : 0.f;
 
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % AC_NS;
     const long long o = (long long)(k + G) * PS + oc;
-    r7 = r7n;
-    const float qxv = qxn, qyv = qyn, qzv = qzn, bxv = bxn, byv = byn, bzv = bzn;
-    if (it + 1 < np) {
-      r7n = __ldg(p + o + 5 * PS);
-      if (own) {
-        qxn = a.qx[o + PS]; qyn = a.qy[o + PS]; qzn = a.qz[o + PS];
-        bxn = __ldg(a.bx + o + PS); byn = __ldg(a.by + o + PS); bzn = __ldg(a.bz + o + PS);
-      }
-    }
+    r7 = na;
+    na = nb;
+    if (it + 2 < np) nb = __ldg(p + o + 6 * PS);
     mbar_wait(&bar[s], (it / AC_NS) & 1);
-    const float* c = sm + s * TILE + (ty + 4) * W + tx + 4;
+    const float* st = sm + s * L::SIZE;
+    const float* c = st + L::P + (ty + 4) * W + tx + 4;
     float dx = SEIS_D1 * (c[1] - c[0]);
     dx = fmaf(SEIS_D2, c[2] - c[-1], dx);
     dx = fmaf(SEIS_D3, c[3] - c[-2], dx);
@@ -146,9 +151,9 @@ __global__ void __launch_bounds__(TXW * BY) ac_v_kernel(const __grid_constant__ 
           dz += ps;
         }
       }
-      a.qx[o] = fmaf(bxv, dx, qxv);
-      a.qy[o] = fmaf(byv, dy, qyv);
-      a.qz[o] = fmaf(bzv, dz, qzv);
+      a.qx[o] = fmaf(st[L::BX + tid], dx, st[L::QX + tid]);
+      a.qy[o] = fmaf(st[L::BYo + tid], dy, st[L::QY + tid]);
+      a.qz[o] = fmaf(st[L::BZ + tid], dz, st[L::QZ + tid]);
       if (IMG) {
         const long long cix = ((long long)k * d.ny + j) * d.nx + i;
         a.img[cix] = fmaf(__ldg(a.imgS + cix), r3, a.img[cix]);
@@ -157,8 +162,7 @@ __global__ void __launch_bounds__(TXW * BY) ac_v_kernel(const __grid_constant__ 
     __syncthreads();
     if (tid == 0 && it + AC_NS < np) {
       fence_proxy_async();
-      mbar_expect_tx(&bar[s], TX_BYTES);
-      tma_load_3d(sm + s * TILE, &a.mp, &bar[s], i0, j0, k + AC_NS + G);
+      issue(s, k + AC_NS);
     }
     r0 = r1; r1 = r2; r2 = r3; r3 = r4; r4 = r5; r5 = r6; r6 = r7;
   }
@@ -167,9 +171,10 @@ __global__ void __launch_bounds__(TXW * BY) ac_v_kernel(const __grid_constant__ 
 struct AcPArgs {
   CUtensorMap mqx;                // q_x, box (32+8) x BY x 1
   CUtensorMap mqy;                // q_y, box 32 x (BY+8) x 1
+  CUtensorMap mpp;                // p, box 32 x BY x 1
+  CUtensorMap mk;                 // dt K / h, box 32 x BY x 1
   float* __restrict__ p;
   const float* __restrict__ qz;
-  const float* __restrict__ kdt;  // dt * rho v^2 / h (padded)
   int W;
   int zlo;
   CpmlAxis cx, cy, cz;
@@ -183,14 +188,20 @@ struct AcPArgs {
   float* __restrict__ snap;       // compact snapshot target, or nullptr
 };
 
+template <int BY>
+struct AcPStage {
+  static constexpr int WX = TXW + 8, T = TXW * BY;
+  static constexpr int QX = 0, QY = BY * WX, P = QY + (BY + 8) * TXW, K = P + T, SIZE = K + T;
+  static constexpr size_t smem_bytes() { return (size_t)AC_NS * SIZE * 4 + 128; }
+};
+
 template <int BY, bool SNAP>
 __global__ void __launch_bounds__(TXW * BY) ac_p_kernel(const __grid_constant__ AcPArgs a) {
-  constexpr int WX = TXW + 8;
-  constexpr int TQX = BY * WX;           // q_x tile (x halo)
-  constexpr int TQY = (BY + 8) * TXW;    // q_y tile (y halo)
-  constexpr int STAGE = TQX + TQY;       // both multiples of 32 floats (128 B)
-  constexpr uint32_t TX_BYTES = STAGE * 4;
-  __shared__ __align__(128) float sm[AC_NS * STAGE];
+  using L = AcPStage<BY>;
+  constexpr int WX = L::WX;
+  constexpr uint32_t TX_BYTES = L::SIZE * 4;
+  extern __shared__ __align__(128) float sm_raw[];
+  float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[AC_NS];
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
@@ -206,20 +217,23 @@ __global__ void __launch_bounds__(TXW * BY) ac_p_kernel(const __grid_constant__ 
   const int Wl = a.W;
   const bool lx = Wl > 0 && CpmlIdx::in(i, d.nx, Wl, true);
   const bool ly = Wl > 0 && CpmlIdx::in(j, d.ny, Wl, true);
-
+  auto issue = [&](int s, int k) {
+    float* st = sm + s * L::SIZE;
+    const int z = k + G;
+    mbar_expect_tx(&bar[s], TX_BYTES);
+    tma_load_3d(st + L::QX, &a.mqx, &bar[s], i0, j0 + G, z);
+    tma_load_3d(st + L::QY, &a.mqy, &bar[s], i0 + G, j0, z);
+    tma_load_3d(st + L::P, &a.mpp, &bar[s], i0 + G, j0 + G, z);
+    tma_load_3d(st + L::K, &a.mk, &bar[s], i0 + G, j0 + G, z);
+  };
   if (tid == 0) {
     for (int s = 0; s < AC_NS; ++s) mbar_init(&bar[s], 1);
     mbar_fence_init();
   }
   __syncthreads();
-  if (tid == 0) {
-    for (int s = 0; s < AC_NS && s < np; ++s) {
-      mbar_expect_tx(&bar[s], TX_BYTES);
-      tma_load_3d(sm + s * STAGE, &a.mqx, &bar[s], i0, j0 + G, k0 + s + G);
-      tma_load_3d(sm + s * STAGE + TQX, &a.mqy, &bar[s], i0 + G, j0, k0 + s + G);
-    }
-  }
-  float s0, s1, s2, s3, s4, s5, s6, s7;  // q_z at k-4 .. k+3
+  if (tid == 0)
+    for (int s = 0; s < AC_NS && s < np; ++s) issue(s, k0 + s);
+  float s0, s1, s2, s3, s4, s5, s6, s7;  // q_z at k-4 .. k+3, fed two planes ahead
   s0 = __ldg(qz + (long long)(k0 - 4 + G) * PS + oc);
   s1 = __ldg(qz + (long long)(k0 - 3 + G) * PS + oc);
   s2 = __ldg(qz + (long long)(k0 - 2 + G) * PS + oc);
@@ -227,30 +241,20 @@ __global__ void __launch_bounds__(TXW * BY) ac_p_kernel(const __grid_constant__ 
   s4 = __ldg(qz + (long long)(k0 + G) * PS + oc);
   s5 = __ldg(qz + (long long)(k0 + 1 + G) * PS + oc);
   s6 = __ldg(qz + (long long)(k0 + 2 + G) * PS + oc);
-  float s7n = __ldg(qz + (long long)(k0 + 3 + G) * PS + oc);
-  float pn = 0.f, kn = 0.f;
-  if (own && np > 0) {
-    const long long o = (long long)(k0 + G) * PS + oc;
-    pn = a.p[o];
-    kn = __ldg(a.kdt + o);
-  }
+  float na = __ldg(qz + (long long)(k0 + 3 + G) * PS + oc);
+  float nb = np > 1 ? __ldg(qz + (long long)(k0 + 4 + G) * PS + oc) : 0.f;
 
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % AC_NS;
     const long long o = (long long)(k + G) * PS + oc;
-    s7 = s7n;
-    const float pv = pn, kv = kn;
-    if (it + 1 < np) {
-      s7n = __ldg(qz + o + 4 * PS);
-      if (own) {
-        pn = a.p[o + PS];
-        kn = __ldg(a.kdt + o + PS);
-      }
-    }
+    s7 = na;
+    na = nb;
+    if (it + 2 < np) nb = __ldg(qz + o + 5 * PS);
     mbar_wait(&bar[s], (it / AC_NS) & 1);
-    const float* cx = sm + s * STAGE + ty * WX + tx + 4;
-    const float* cy = sm + s * STAGE + TQX + (ty + 4) * TXW + tx;
+    const float* st = sm + s * L::SIZE;
+    const float* cx = st + L::QX + ty * WX + tx + 4;
+    const float* cy = st + L::QY + (ty + 4) * TXW + tx;
     float dx = SEIS_D1 * (cx[0] - cx[-1]);
     dx = fmaf(SEIS_D2, cx[1] - cx[-2], dx);
     dx = fmaf(SEIS_D3, cx[2] - cx[-3], dx);
@@ -285,7 +289,7 @@ __global__ void __launch_bounds__(TXW * BY) ac_p_kernel(const __grid_constant__ 
           dz += ps;
         }
       }
-      float out = fmaf(kv, (dx + dy) + dz, pv);
+      float out = fmaf(st[L::K + tid], (dx + dy) + dz, st[L::P + tid]);
       if (o == a.src_o) out += a.src_amp;
       a.p[o] = out;
       if (SNAP) a.snap[((long long)k * d.ny + j) * d.nx + i] = out;
@@ -293,9 +297,7 @@ __global__ void __launch_bounds__(TXW * BY) ac_p_kernel(const __grid_constant__ 
     __syncthreads();
     if (tid == 0 && it + AC_NS < np) {
       fence_proxy_async();
-      mbar_expect_tx(&bar[s], TX_BYTES);
-      tma_load_3d(sm + s * STAGE, &a.mqx, &bar[s], i0, j0 + G, k + AC_NS + G);
-      tma_load_3d(sm + s * STAGE + TQX, &a.mqy, &bar[s], i0 + G, j0, k + AC_NS + G);
+      issue(s, k + AC_NS);
     }
     s0 = s1; s1 = s2; s2 = s3; s3 = s4; s4 = s5; s5 = s6; s6 = s7;
   }

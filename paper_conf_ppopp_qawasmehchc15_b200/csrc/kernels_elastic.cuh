@@ -87,10 +87,9 @@ struct ElVArgs {
   CUtensorMap msxz;  // box 40 x BY
   CUtensorMap msyy;  // box 32 x (BY+8)  (y halo)
   CUtensorMap msyz;  // box 32 x (BY+8)
+  CUtensorMap mv[3]; // vx, vy, vz, box 32 x BY
+  CUtensorMap mb[3]; // face buoyancies, box 32 x BY
   float* f[9];
-  const float* __restrict__ bx;
-  const float* __restrict__ by;
-  const float* __restrict__ bz;
   int W, zlo, fs;
   CpmlAxis cx, cy, cz;
   float* psi[9];   // psi 0..8
@@ -99,15 +98,22 @@ struct ElVArgs {
 };
 
 template <int BY>
+struct ElVStage {
+  static constexpr int WX = TXW + 8, T = TXW * BY;
+  static constexpr int XX = 0, XY = XX + BY * WX, XZ = XY + (BY + 8) * WX, YY = XZ + BY * WX,
+                       YZ = YY + (BY + 8) * TXW, V = YZ + (BY + 8) * TXW, B = V + 3 * T, SIZE = B + 3 * T;
+  static constexpr size_t smem_bytes() { return (size_t)EL_NS * SIZE * 4 + 128; }
+};
+
+template <int BY>
 __global__ void __launch_bounds__(TXW * BY) el_v_kernel(const __grid_constant__ ElVArgs a) {
-  constexpr int WX = TXW + 8;
-  constexpr int T_XX = BY * WX, T_XY = (BY + 8) * WX, T_XZ = BY * WX, T_YY = (BY + 8) * TXW,
-                T_YZ = (BY + 8) * TXW;
-  constexpr int O_XY = T_XX, O_XZ = O_XY + T_XY, O_YY = O_XZ + T_XZ, O_YZ = O_YY + T_YY;
-  constexpr int STAGE = O_YZ + T_YZ;
-  constexpr uint32_t TX_BYTES = STAGE * 4;
-  static_assert((T_XX % 32) == 0 && (T_XY % 32) == 0 && (T_YY % 32) == 0, "128-byte tiles");
-  __shared__ __align__(128) float sm[EL_NS * STAGE];
+  using L = ElVStage<BY>;
+  constexpr int WX = L::WX, T = L::T;
+  constexpr uint32_t TX_BYTES = L::SIZE * 4;
+  static_assert((L::XY % 32) == 0 && (L::XZ % 32) == 0 && (L::YY % 32) == 0 && (L::V % 32) == 0,
+                "128-byte tiles");
+  extern __shared__ __align__(128) float sm_raw[];
+  float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[EL_NS];
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
@@ -126,13 +132,19 @@ __global__ void __launch_bounds__(TXW * BY) el_v_kernel(const __grid_constant__ 
   const float* __restrict__ syz = a.f[ESYZ];
   const float* __restrict__ szz = a.f[ESZZ];
   auto issue = [&](int s, int k) {
-    float* st = sm + s * STAGE;
+    float* st = sm + s * L::SIZE;
+    const int z = k + G;
     mbar_expect_tx(&bar[s], TX_BYTES);
-    tma_load_3d(st, &a.msxx, &bar[s], i0, j0 + G, k + G);
-    tma_load_3d(st + O_XY, &a.msxy, &bar[s], i0, j0, k + G);
-    tma_load_3d(st + O_XZ, &a.msxz, &bar[s], i0, j0 + G, k + G);
-    tma_load_3d(st + O_YY, &a.msyy, &bar[s], i0 + G, j0, k + G);
-    tma_load_3d(st + O_YZ, &a.msyz, &bar[s], i0 + G, j0, k + G);
+    tma_load_3d(st + L::XX, &a.msxx, &bar[s], i0, j0 + G, z);
+    tma_load_3d(st + L::XY, &a.msxy, &bar[s], i0, j0, z);
+    tma_load_3d(st + L::XZ, &a.msxz, &bar[s], i0, j0 + G, z);
+    tma_load_3d(st + L::YY, &a.msyy, &bar[s], i0 + G, j0, z);
+    tma_load_3d(st + L::YZ, &a.msyz, &bar[s], i0 + G, j0, z);
+#pragma unroll
+    for (int c = 0; c < 3; ++c) {
+      tma_load_3d(st + L::V + c * T, &a.mv[c], &bar[s], i0 + G, j0 + G, z);
+      tma_load_3d(st + L::B + c * T, &a.mb[c], &bar[s], i0 + G, j0 + G, z);
+    }
   };
   if (tid == 0) {
     for (int s = 0; s < EL_NS; ++s) mbar_init(&bar[s], 1);
@@ -148,38 +160,34 @@ __global__ void __launch_bounds__(TXW * BY) el_v_kernel(const __grid_constant__ 
     qyz[t] = __ldg(syz + (long long)(k0 - 4 + t + G) * PS + oc);
     qzz[t] = __ldg(szz + (long long)(k0 - 3 + t + G) * PS + oc);
   }
-  float nxz = __ldg(sxz + (long long)(k0 + 3 + G) * PS + oc);
-  float nyz = __ldg(syz + (long long)(k0 + 3 + G) * PS + oc);
-  float nzz = __ldg(szz + (long long)(k0 + 4 + G) * PS + oc);
-  float nv[3] = {0.f, 0.f, 0.f}, nb[3] = {0.f, 0.f, 0.f};
-  if (own && np > 0) {
-    const long long o = (long long)(k0 + G) * PS + oc;
-    nv[0] = a.f[EVX][o]; nv[1] = a.f[EVY][o]; nv[2] = a.f[EVZ][o];
-    nb[0] = __ldg(a.bx + o); nb[1] = __ldg(a.by + o); nb[2] = __ldg(a.bz + o);
+  float axz = __ldg(sxz + (long long)(k0 + 3 + G) * PS + oc);
+  float ayz = __ldg(syz + (long long)(k0 + 3 + G) * PS + oc);
+  float azz = __ldg(szz + (long long)(k0 + 4 + G) * PS + oc);
+  float bxz = 0.f, byz = 0.f, bzz = 0.f;
+  if (np > 1) {
+    bxz = __ldg(sxz + (long long)(k0 + 4 + G) * PS + oc);
+    byz = __ldg(syz + (long long)(k0 + 4 + G) * PS + oc);
+    bzz = __ldg(szz + (long long)(k0 + 5 + G) * PS + oc);
   }
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % EL_NS;
     const long long o = (long long)(k + G) * PS + oc;
-    qxz[7] = nxz; qyz[7] = nyz; qzz[7] = nzz;
-    const float v0 = nv[0], v1 = nv[1], v2 = nv[2], b0 = nb[0], b1 = nb[1], b2 = nb[2];
-    if (it + 1 < np) {
-      nxz = __ldg(sxz + o + 4 * PS);
-      nyz = __ldg(syz + o + 4 * PS);
-      nzz = __ldg(szz + o + 5 * PS);
-      if (own) {
-        nv[0] = a.f[EVX][o + PS]; nv[1] = a.f[EVY][o + PS]; nv[2] = a.f[EVZ][o + PS];
-        nb[0] = __ldg(a.bx + o + PS); nb[1] = __ldg(a.by + o + PS); nb[2] = __ldg(a.bz + o + PS);
-      }
+    qxz[7] = axz; qyz[7] = ayz; qzz[7] = azz;
+    axz = bxz; ayz = byz; azz = bzz;
+    if (it + 2 < np) {
+      bxz = __ldg(sxz + o + 5 * PS);
+      byz = __ldg(syz + o + 5 * PS);
+      bzz = __ldg(szz + o + 6 * PS);
     }
     mbar_wait(&bar[s], (it / EL_NS) & 1);
     if (own) {
-      const float* st = sm + s * STAGE;
-      const float* cxx = st + ty * WX + tx + 4;
-      const float* cxy = st + O_XY + (ty + 4) * WX + tx + 4;
-      const float* cxz = st + O_XZ + ty * WX + tx + 4;
-      const float* cyy = st + O_YY + (ty + 4) * TXW + tx;
-      const float* cyz = st + O_YZ + (ty + 4) * TXW + tx;
+      const float* st = sm + s * L::SIZE;
+      const float* cxx = st + L::XX + ty * WX + tx + 4;
+      const float* cxy = st + L::XY + (ty + 4) * WX + tx + 4;
+      const float* cxz = st + L::XZ + ty * WX + tx + 4;
+      const float* cyy = st + L::YY + (ty + 4) * TXW + tx;
+      const float* cyz = st + L::YZ + (ty + 4) * TXW + tx;
       float d0 = dplus<1>(cxx), d1 = dminus<WX>(cxy), d2 = zminus(qxz);
       float d3 = dminus<1>(cxy), d4 = dplus<TXW>(cyy), d5 = zminus(qyz);
       float d6 = dminus<1>(cxz), d7 = dminus<TXW>(cyz), d8 = zplus(qzz);
@@ -201,9 +209,11 @@ __global__ void __launch_bounds__(TXW * BY) el_v_kernel(const __grid_constant__ 
           cpml_z(d8, a.psi[8], d, W, i, j, gz, a.cz.ah, a.cz.bh);
         }
       }
-      a.f[EVX][o] = fmaf(b0, (d0 + d1) + d2, v0);
-      a.f[EVY][o] = fmaf(b1, (d3 + d4) + d5, v1);
-      a.f[EVZ][o] = fmaf(b2, (d6 + d7) + d8, v2);
+      const float* sv = st + L::V + tid;
+      const float* sb = st + L::B + tid;
+      a.f[EVX][o] = fmaf(sb[0], (d0 + d1) + d2, sv[0]);
+      a.f[EVY][o] = fmaf(sb[T], (d3 + d4) + d5, sv[T]);
+      a.f[EVZ][o] = fmaf(sb[2 * T], (d6 + d7) + d8, sv[2 * T]);
     }
     __syncthreads();
     if (tid == 0 && it + EL_NS < np) {
@@ -220,15 +230,10 @@ __global__ void __launch_bounds__(TXW * BY) el_v_kernel(const __grid_constant__ 
 }
 
 struct ElSArgs {
-  CUtensorMap mvx;  // box 40 x (BY+8)
-  CUtensorMap mvy;
-  CUtensorMap mvz;
+  CUtensorMap mvt[3];  // vx, vy, vz tiles, box 40 x (BY+8)
+  CUtensorMap ms[6];   // sxx, syy, szz, sxy, sxz, syz, box 32 x BY
+  CUtensorMap mc[5];   // l2m, lam, mxy, mxz, myz, box 32 x BY
   float* f[9];
-  const float* __restrict__ l2m;  // dt (lam + 2 mu) / h
-  const float* __restrict__ lam;  // dt lam / h
-  const float* __restrict__ mxy;  // dt mu_xy / h (edge, harmonic mean)
-  const float* __restrict__ mxz;
-  const float* __restrict__ myz;
   int W, zlo, fs;
   CpmlAxis cx, cy, cz;
   float* psi[9];   // psi 9..17
@@ -238,13 +243,20 @@ struct ElSArgs {
   float src_amp;   // dt (lam + 2/3 mu)_s / h^3 * s[n]
 };
 
+template <int BY>
+struct ElSStage {
+  static constexpr int WX = TXW + 8, T = TXW * BY, TV = (BY + 8) * WX;
+  static constexpr int VT = 0, S = 3 * TV, C = S + 6 * T, SIZE = C + 5 * T;
+  static constexpr size_t smem_bytes() { return (size_t)EL_NS * SIZE * 4 + 128; }
+};
+
 template <int BY, bool UNUSED>
 __global__ void __launch_bounds__(TXW * BY) el_s_kernel(const __grid_constant__ ElSArgs a) {
-  constexpr int WX = TXW + 8;
-  constexpr int TV = (BY + 8) * WX;
-  constexpr int STAGE = 3 * TV;
-  constexpr uint32_t TX_BYTES = STAGE * 4;
-  __shared__ __align__(128) float sm[EL_NS * STAGE];
+  using L = ElSStage<BY>;
+  constexpr int WX = L::WX, T = L::T, TV = L::TV;
+  constexpr uint32_t TX_BYTES = L::SIZE * 4;
+  extern __shared__ __align__(128) float sm_raw[];
+  float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[EL_NS];
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
@@ -263,11 +275,15 @@ __global__ void __launch_bounds__(TXW * BY) el_s_kernel(const __grid_constant__ 
   const float* __restrict__ vy = a.f[EVY];
   const float* __restrict__ vz = a.f[EVZ];
   auto issue = [&](int s, int k) {
-    float* st = sm + s * STAGE;
+    float* st = sm + s * L::SIZE;
+    const int z = k + G;
     mbar_expect_tx(&bar[s], TX_BYTES);
-    tma_load_3d(st, &a.mvx, &bar[s], i0, j0, k + G);
-    tma_load_3d(st + TV, &a.mvy, &bar[s], i0, j0, k + G);
-    tma_load_3d(st + 2 * TV, &a.mvz, &bar[s], i0, j0, k + G);
+#pragma unroll
+    for (int c = 0; c < 3; ++c) tma_load_3d(st + L::VT + c * TV, &a.mvt[c], &bar[s], i0, j0, z);
+#pragma unroll
+    for (int c = 0; c < 6; ++c) tma_load_3d(st + L::S + c * T, &a.ms[c], &bar[s], i0 + G, j0 + G, z);
+#pragma unroll
+    for (int c = 0; c < 5; ++c) tma_load_3d(st + L::C + c * T, &a.mc[c], &bar[s], i0 + G, j0 + G, z);
   };
   if (tid == 0) {
     for (int s = 0; s < EL_NS; ++s) mbar_init(&bar[s], 1);
@@ -283,34 +299,33 @@ __global__ void __launch_bounds__(TXW * BY) el_s_kernel(const __grid_constant__ 
     qy[t] = __ldg(vy + (long long)(k0 - 3 + t + G) * PS + oc);
     qz[t] = __ldg(vz + (long long)(k0 - 4 + t + G) * PS + oc);
   }
-  float nqx = __ldg(vx + (long long)(k0 + 4 + G) * PS + oc);
-  float nqy = __ldg(vy + (long long)(k0 + 4 + G) * PS + oc);
-  float nqz = __ldg(vz + (long long)(k0 + 3 + G) * PS + oc);
+  float ax = __ldg(vx + (long long)(k0 + 4 + G) * PS + oc);
+  float ay = __ldg(vy + (long long)(k0 + 4 + G) * PS + oc);
+  float az = __ldg(vz + (long long)(k0 + 3 + G) * PS + oc);
+  float bx = 0.f, by = 0.f, bz = 0.f;
+  if (np > 1) {
+    bx = __ldg(vx + (long long)(k0 + 5 + G) * PS + oc);
+    by = __ldg(vy + (long long)(k0 + 5 + G) * PS + oc);
+    bz = __ldg(vz + (long long)(k0 + 4 + G) * PS + oc);
+  }
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % EL_NS;
     const long long o = (long long)(k + G) * PS + oc;
-    qx[7] = nqx; qy[7] = nqy; qz[7] = nqz;
-    if (it + 1 < np) {
-      nqx = __ldg(vx + o + 5 * PS);
-      nqy = __ldg(vy + o + 5 * PS);
-      nqz = __ldg(vz + o + 4 * PS);
-    }
-    float sxx = 0.f, syy = 0.f, szz = 0.f, sxy = 0.f, sxz = 0.f, syz = 0.f;
-    float l2m = 0.f, lam = 0.f, mxy = 0.f, mxz = 0.f, myz = 0.f;
-    if (own) {
-      sxx = a.f[ESXX][o]; syy = a.f[ESYY][o]; szz = a.f[ESZZ][o];
-      sxy = a.f[ESXY][o]; sxz = a.f[ESXZ][o]; syz = a.f[ESYZ][o];
-      l2m = __ldg(a.l2m + o); lam = __ldg(a.lam + o);
-      mxy = __ldg(a.mxy + o); mxz = __ldg(a.mxz + o); myz = __ldg(a.myz + o);
+    qx[7] = ax; qy[7] = ay; qz[7] = az;
+    ax = bx; ay = by; az = bz;
+    if (it + 2 < np) {
+      bx = __ldg(vx + o + 6 * PS);
+      by = __ldg(vy + o + 6 * PS);
+      bz = __ldg(vz + o + 5 * PS);
     }
     mbar_wait(&bar[s], (it / EL_NS) & 1);
     if (own) {
       const int gz = k + d.z0;
-      const float* st = sm + s * STAGE;
-      const float* cvx = st + (ty + 4) * WX + tx + 4;
-      const float* cvy = st + TV + (ty + 4) * WX + tx + 4;
-      const float* cvz = st + 2 * TV + (ty + 4) * WX + tx + 4;
+      const float* st = sm + s * L::SIZE;
+      const float* cvx = st + L::VT + (ty + 4) * WX + tx + 4;
+      const float* cvy = cvx + TV;
+      const float* cvz = cvx + 2 * TV;
       float exx = dminus<1>(cvx), eyy = dminus<WX>(cvy), ezz = zminus(qz);
       float dyvx = dplus<WX>(cvx), dxvy = dplus<1>(cvy);
       float dzvx = zplus(qx), dxvz = dplus<1>(cvz);
@@ -332,11 +347,14 @@ __global__ void __launch_bounds__(TXW * BY) el_s_kernel(const __grid_constant__ 
           cpml_z(dzvy, a.psi[7], d, W, i, j, gz, a.cz.ah, a.cz.bh);
         }
       }
+      const float* ss = st + L::S + tid;
+      const float* sc = st + L::C + tid;
+      const float l2m = sc[0], lam = sc[T];
       const bool surf = a.fs && gz == 0;
       if (surf) ezz = -(lam / l2m) * (exx + eyy);  // O16 surface row
-      sxx += fmaf(l2m, exx, lam * (eyy + ezz));
-      syy += fmaf(l2m, eyy, lam * (exx + ezz));
-      szz += fmaf(l2m, ezz, lam * (exx + eyy));
+      float sxx = ss[0] + fmaf(l2m, exx, lam * (eyy + ezz));
+      float syy = ss[T] + fmaf(l2m, eyy, lam * (exx + ezz));
+      float szz = ss[2 * T] + fmaf(l2m, ezz, lam * (exx + eyy));
       if (o == a.src_o) {
         sxx -= a.src_amp;
         syy -= a.src_amp;
@@ -346,9 +364,9 @@ __global__ void __launch_bounds__(TXW * BY) el_s_kernel(const __grid_constant__ 
       a.f[ESXX][o] = sxx;
       a.f[ESYY][o] = syy;
       a.f[ESZZ][o] = szz;
-      a.f[ESXY][o] = fmaf(mxy, dyvx + dxvy, sxy);
-      a.f[ESXZ][o] = fmaf(mxz, dzvx + dxvz, sxz);
-      a.f[ESYZ][o] = fmaf(myz, dzvy + dyvz, syz);
+      a.f[ESXY][o] = fmaf(sc[2 * T], dyvx + dxvy, ss[3 * T]);
+      a.f[ESXZ][o] = fmaf(sc[3 * T], dzvx + dxvz, ss[4 * T]);
+      a.f[ESYZ][o] = fmaf(sc[4 * T], dzvy + dyvz, ss[5 * T]);
     }
     __syncthreads();
     if (tid == 0 && it + EL_NS < np) {

@@ -4,25 +4,26 @@
 //   m = v^2 dt^2 / h^2 (per point, precomputed),  eta dt = edx[i] + edy[j] + edz[k]
 //   Lambda u = 3 c0 u + sum_m c_m sum_axes (u_{+m} + u_{-m})         (O1, O3, O6)
 //
-// One thread per (x, y) column marching down a z-chunk (2.5D blocking).  The
-// x/y neighbours of plane k come from a shared-memory tile (halo 4) brought in
-// by TMA through an NS-stage mbarrier ring; the z neighbours from a 9-deep
-// register queue fed by a coalesced stream prefetched one plane ahead, like
-// u^{n-1} and m.  u^{n+1} overwrites u^{n-1} in place ("logically
-// swapping t_n and t_{n+1} arrays").  HBM traffic per point: read u^n, u^{n-1},
-// m; write u^{n+1} = 16 B (+4 B snapshot, +12 B imaging).  Fused epilogues:
-// source injection, snapshot store (O14), imaging
-// I += S_j * u^n on the input level (O15).
+// One thread per (x, y) column marching down a z-chunk (2.5D blocking).  Every
+// operand of plane k arrives by TMA in one stage of an NS-deep mbarrier ring
+// (the u^n tile with its x/y halo of 4, and the u^{n-1} and m tiles); the z
+// neighbours come from a 9-deep register queue fed by a coalesced stream two
+// planes ahead.  u^{n+1} overwrites u^{n-1} in place ("logically swapping
+// t_n and t_{n+1} arrays").  HBM traffic per point: read u^n, u^{n-1}, m; write
+// u^{n+1} = 16 B (+4 B snapshot, +12 B imaging).  Fused epilogues: source
+// injection, snapshot store (O14), imaging I += S_j * u^n on
+// the input level (O15).
 #pragma once
 #include "common.cuh"
 
 namespace seis {
 
 struct IsoArgs {
-  CUtensorMap mun;               // u^n, box (32+8) x (BY+8) x 1
+  CUtensorMap mun;               // u^n tile, box (32+8) x (BY+8) x 1
+  CUtensorMap mup;               // u^{n-1}, box 32 x BY x 1
+  CUtensorMap mm;                // m, box 32 x BY x 1
   const float* __restrict__ un;  // u^n (padded)
-  float* __restrict__ up;        // in: u^{n-1}; out: u^{n+1}
-  const float* __restrict__ m;   // v^2 dt^2 / h^2 (padded)
+  float* __restrict__ up;        // out: u^{n+1} (in place of u^{n-1})
   const float* __restrict__ edx; // eta*dt per axis (global index), nullptr = no layer
   const float* __restrict__ edy;
   const float* __restrict__ edz;
@@ -37,12 +38,20 @@ struct IsoArgs {
 
 constexpr int ISO_NS = 4;
 
+template <int BY>
+struct IsoStage {
+  static constexpr int W = TXW + 8;
+  static constexpr int U = 0, UP = (BY + 8) * W, M = UP + TXW * BY, SIZE = M + TXW * BY;
+  static constexpr size_t smem_bytes() { return (size_t)ISO_NS * SIZE * 4 + 128; }
+};
+
 template <int BY, bool SNAP, bool IMG>
 __global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const __grid_constant__ IsoArgs a) {
-  constexpr int W = TXW + 8;
-  constexpr int TILE = (BY + 8) * W;  // floats per stage (multiple of 32)
-  constexpr uint32_t TX_BYTES = TILE * 4;
-  __shared__ __align__(128) float sm[ISO_NS * TILE];
+  using L = IsoStage<BY>;
+  constexpr int W = L::W;
+  constexpr uint32_t TX_BYTES = L::SIZE * 4;
+  extern __shared__ __align__(128) float sm_raw[];
+  float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[ISO_NS];
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
@@ -55,19 +64,22 @@ __global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const __grid_constan
   const long long PS = d.PS;
   const long long oc = (long long)(j + G) * d.PX + (i + G);
   const float* __restrict__ un = a.un;
-
+  auto issue = [&](int s, int k) {
+    float* st = sm + s * L::SIZE;
+    mbar_expect_tx(&bar[s], TX_BYTES);
+    tma_load_3d(st + L::U, &a.mun, &bar[s], i0, j0, k + G);
+    tma_load_3d(st + L::UP, &a.mup, &bar[s], i0 + G, j0 + G, k + G);
+    tma_load_3d(st + L::M, &a.mm, &bar[s], i0 + G, j0 + G, k + G);
+  };
   if (tid == 0) {
     for (int s = 0; s < ISO_NS; ++s) mbar_init(&bar[s], 1);
     mbar_fence_init();
   }
   __syncthreads();
-  if (tid == 0) {
-    for (int s = 0; s < ISO_NS && s < np; ++s) {
-      mbar_expect_tx(&bar[s], TX_BYTES);
-      tma_load_3d(sm + s * TILE, &a.mun, &bar[s], i0, j0, k0 + s + G);
-    }
-  }
-  // z-queue u^n(k-4 .. k+4) and the one-plane-ahead streams
+  if (tid == 0)
+    for (int s = 0; s < ISO_NS && s < np; ++s) issue(s, k0 + s);
+
+  // z-queue u^n(k-4 .. k+4), fed two planes ahead
   float q0, q1, q2, q3, q4, q5, q6, q7, q8;
   q0 = __ldg(un + (long long)(k0 - 4 + G) * PS + oc);
   q1 = __ldg(un + (long long)(k0 - 3 + G) * PS + oc);
@@ -77,32 +89,21 @@ __global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const __grid_constan
   q5 = __ldg(un + (long long)(k0 + 1 + G) * PS + oc);
   q6 = __ldg(un + (long long)(k0 + 2 + G) * PS + oc);
   q7 = __ldg(un + (long long)(k0 + 3 + G) * PS + oc);
-  float q8n = __ldg(un + (long long)(k0 + 4 + G) * PS + oc);
-  float upn = 0.f, mn = 0.f;
-  {
-    const long long o = (long long)(k0 + G) * PS + oc;
-    if (own && np > 0) {
-      upn = a.up[o];
-      mn = __ldg(a.m + o);
-    }
-  }
+  float na = __ldg(un + (long long)(k0 + 4 + G) * PS + oc);
+  float nb = np > 1 ? __ldg(un + (long long)(k0 + 5 + G) * PS + oc) : 0.f;
   const float exy = (a.edx && own) ? a.edx[i] + a.edy[j] : 0.0f;
 
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % ISO_NS;
     const long long o = (long long)(k + G) * PS + oc;
-    q8 = q8n;
-    const float upv = upn, mv = mn;
-    if (it + 1 < np) {
-      q8n = __ldg(un + o + 5 * PS);
-      if (own) {
-        upn = a.up[o + PS];
-        mn = __ldg(a.m + o + PS);
-      }
-    }
+    q8 = na;
+    na = nb;
+    if (it + 2 < np) nb = __ldg(un + o + 6 * PS);
     mbar_wait(&bar[s], (it / ISO_NS) & 1);
-    const float* c = sm + s * TILE + (ty + 4) * W + tx + 4;
+    const float* st = sm + s * L::SIZE;
+    const float* c = st + L::U + (ty + 4) * W + tx + 4;
+    const float upv = st[L::UP + tid], mv = st[L::M + tid];
     float lap = (3.0f * SEIS_C0) * q4;
     lap = fmaf(SEIS_C1, (c[-1] + c[1]) + (c[-W] + c[W]) + (q3 + q5), lap);
     lap = fmaf(SEIS_C2, (c[-2] + c[2]) + (c[-2 * W] + c[2 * W]) + (q2 + q6), lap);
@@ -127,8 +128,7 @@ __global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const __grid_constan
     __syncthreads();  // every thread is done with stage s
     if (tid == 0 && it + ISO_NS < np) {
       fence_proxy_async();
-      mbar_expect_tx(&bar[s], TX_BYTES);
-      tma_load_3d(sm + s * TILE, &a.mun, &bar[s], i0, j0, k + ISO_NS + G);
+      issue(s, k + ISO_NS);
     }
     q0 = q1; q1 = q2; q2 = q3; q3 = q4; q4 = q5; q5 = q6; q6 = q7; q7 = q8;
   }

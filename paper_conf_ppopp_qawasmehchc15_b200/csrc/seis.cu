@@ -118,10 +118,12 @@ struct Slab {
   float *bx = nullptr, *by = nullptr, *bz = nullptr;                          // ACOUSTIC, ELASTIC
   float *l2m = nullptr, *lam = nullptr, *mxy = nullptr, *mxz = nullptr, *myz = nullptr;  // ELASTIC
   float* psi[NPSI] = {};
-  // TMA descriptors of the plane tiles each kernel stages
-  CUtensorMap mu[2];                                   // ISO u (both time levels)
-  CUtensorMap mp, mqx, mqy;                            // ACOUSTIC
-  CUtensorMap msxx, msxy, msxz, msyy, msyz, mvx, mvy, mvz;  // ELASTIC
+  // TMA descriptors of every operand tile the kernels stage:
+  // "t" = tile with x/y halo, "c" = interior (centre) tile 32 x BY
+  CUtensorMap iso_ut[2], iso_uc[2], iso_m;                              // ISO
+  CUtensorMap ac_pt, ac_qc[3], ac_bc[3], ac_qxt, ac_qyt, ac_pc, ac_kc;   // ACOUSTIC
+  CUtensorMap el_sxxt, el_sxyt, el_sxzt, el_syyt, el_syzt, el_vc[3], el_bc[3];  // ELASTIC V
+  CUtensorMap el_vt[3], el_sc[6], el_cc[5];                             // ELASTIC S
   int cur = 0;               // ISO: fld[cur] = u^n
   int zc = 1, nzch = 1;      // z-chunking of the stencil launches
   // shot tables
@@ -285,6 +287,25 @@ seis_status upload_padded_from_host(seis_model* M, const Dims& d, const std::vec
   CKL();
   CK(cudaStreamSynchronize(st));
   CK(cudaFree(tmp));
+  return SEIS_OK;
+}
+
+// Opt every TMA-ring kernel into its dynamic shared-memory footprint (once per process).
+seis_status set_smem_attrs() {
+  static bool done = false;
+  if (done) return SEIS_OK;
+#define SMEM_ATTR(fn, bytes) CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(bytes)))
+  SMEM_ATTR((iso_step_kernel<BY, false, false>), IsoStage<BY>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BY, true, false>), IsoStage<BY>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BY, false, true>), IsoStage<BY>::smem_bytes());
+  SMEM_ATTR((ac_v_kernel<BY, false>), AcVStage<BY>::smem_bytes());
+  SMEM_ATTR((ac_v_kernel<BY, true>), AcVStage<BY>::smem_bytes());
+  SMEM_ATTR((ac_p_kernel<BY, false>), AcPStage<BY>::smem_bytes());
+  SMEM_ATTR((ac_p_kernel<BY, true>), AcPStage<BY>::smem_bytes());
+  SMEM_ATTR((el_v_kernel<BYE>), ElVStage<BYE>::smem_bytes());
+  SMEM_ATTR((el_s_kernel<BYE, false>), ElSStage<BYE>::smem_bytes());
+#undef SMEM_ATTR
+  done = true;
   return SEIS_OK;
 }
 
@@ -683,29 +704,49 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     }
     // TMA descriptors
     if (kind == SEIS_ISO) {
-      TRY(make_map(&S.mu[0], S.fld[0], d, TXW + 8, BY + 8));
-      TRY(make_map(&S.mu[1], S.fld[1], d, TXW + 8, BY + 8));
+      for (int t = 0; t < 2; ++t) {
+        TRY(make_map(&S.iso_ut[t], S.fld[t], d, TXW + 8, BY + 8));
+        TRY(make_map(&S.iso_uc[t], S.fld[t], d, TXW, BY));
+      }
+      TRY(make_map(&S.iso_m, S.m, d, TXW, BY));
     } else if (kind == SEIS_ACOUSTIC) {
-      TRY(make_map(&S.mp, S.fld[0], d, TXW + 8, BY + 8));
-      TRY(make_map(&S.mqx, S.fld[1], d, TXW + 8, BY));
-      TRY(make_map(&S.mqy, S.fld[2], d, TXW, BY + 8));
+      TRY(make_map(&S.ac_pt, S.fld[0], d, TXW + 8, BY + 8));
+      float* bb[3] = {S.bx, S.by, S.bz};
+      for (int t = 0; t < 3; ++t) {
+        TRY(make_map(&S.ac_qc[t], S.fld[1 + t], d, TXW, BY));
+        TRY(make_map(&S.ac_bc[t], bb[t], d, TXW, BY));
+      }
+      TRY(make_map(&S.ac_qxt, S.fld[1], d, TXW + 8, BY));
+      TRY(make_map(&S.ac_qyt, S.fld[2], d, TXW, BY + 8));
+      TRY(make_map(&S.ac_pc, S.fld[0], d, TXW, BY));
+      TRY(make_map(&S.ac_kc, S.kdt, d, TXW, BY));
     } else {
-      TRY(make_map(&S.mvx, S.fld[EVX], d, TXW + 8, BYE + 8));
-      TRY(make_map(&S.mvy, S.fld[EVY], d, TXW + 8, BYE + 8));
-      TRY(make_map(&S.mvz, S.fld[EVZ], d, TXW + 8, BYE + 8));
-      TRY(make_map(&S.msxx, S.fld[ESXX], d, TXW + 8, BYE));
-      TRY(make_map(&S.msxy, S.fld[ESXY], d, TXW + 8, BYE + 8));
-      TRY(make_map(&S.msxz, S.fld[ESXZ], d, TXW + 8, BYE));
-      TRY(make_map(&S.msyy, S.fld[ESYY], d, TXW, BYE + 8));
-      TRY(make_map(&S.msyz, S.fld[ESYZ], d, TXW, BYE + 8));
+      TRY(make_map(&S.el_sxxt, S.fld[ESXX], d, TXW + 8, BYE));
+      TRY(make_map(&S.el_sxyt, S.fld[ESXY], d, TXW + 8, BYE + 8));
+      TRY(make_map(&S.el_sxzt, S.fld[ESXZ], d, TXW + 8, BYE));
+      TRY(make_map(&S.el_syyt, S.fld[ESYY], d, TXW, BYE + 8));
+      TRY(make_map(&S.el_syzt, S.fld[ESYZ], d, TXW, BYE + 8));
+      float* bb[3] = {S.bx, S.by, S.bz};
+      for (int t = 0; t < 3; ++t) {
+        TRY(make_map(&S.el_vc[t], S.fld[EVX + t], d, TXW, BYE));
+        TRY(make_map(&S.el_bc[t], bb[t], d, TXW, BYE));
+        TRY(make_map(&S.el_vt[t], S.fld[EVX + t], d, TXW + 8, BYE + 8));
+      }
+      for (int t = 0; t < 6; ++t) TRY(make_map(&S.el_sc[t], S.fld[ESXX + t], d, TXW, BYE));
+      float* cc[5] = {S.l2m, S.lam, S.mxy, S.mxz, S.myz};
+      for (int t = 0; t < 5; ++t) TRY(make_map(&S.el_cc[t], cc[t], d, TXW, BYE));
     }
+    TRY(set_smem_attrs());
     int occ = 1;
     if (kind == SEIS_ISO)
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, iso_step_kernel<BY, false, false>, TXW * BY, 0);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, iso_step_kernel<BY, false, false>, TXW * BY,
+                                                    IsoStage<BY>::smem_bytes());
     else if (kind == SEIS_ACOUSTIC)
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_v_kernel<BY, false>, TXW * BY, 0);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_v_kernel<BY, false>, TXW * BY,
+                                                    AcVStage<BY>::smem_bytes());
     else
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, TXW * BYE, 0);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, TXW * BYE,
+                                                    ElSStage<BYE>::smem_bytes());
     choose_chunks(S, occ, dev_sms, kind == SEIS_ELASTIC ? BYE : BY);
   }
   CK(cudaStreamSynchronize(st));
@@ -950,10 +991,11 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (size_t s = 0; s < M->slabs.size(); ++s) {
       Slab& S = M->slabs[s];
       IsoArgs a;
-      a.mun = S.mu[S.cur];
+      a.mun = S.iso_ut[S.cur];
+      a.mup = S.iso_uc[1 - S.cur];
+      a.mm = S.iso_m;
       a.un = S.fld[S.cur];
       a.up = S.fld[1 - S.cur];
-      a.m = S.m;
       a.edx = M->edx;
       a.edy = M->edy;
       a.edz = M->edz;
@@ -968,9 +1010,10 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       const dim3 gr = grid_of(S);
       {
         PROF(0, st);
-        if (a.snap) iso_step_kernel<BY, true, false><<<gr, blk, 0, st>>>(a);
-        else if (a.img) iso_step_kernel<BY, false, true><<<gr, blk, 0, st>>>(a);
-        else iso_step_kernel<BY, false, false><<<gr, blk, 0, st>>>(a);
+        const size_t sb = IsoStage<BY>::smem_bytes();
+        if (a.snap) iso_step_kernel<BY, true, false><<<gr, blk, sb, st>>>(a);
+        else if (a.img) iso_step_kernel<BY, false, true><<<gr, blk, sb, st>>>(a);
+        else iso_step_kernel<BY, false, false><<<gr, blk, sb, st>>>(a);
       }
       CKL();
     }
@@ -985,14 +1028,17 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (size_t s = 0; s < M->slabs.size(); ++s) {
       Slab& S = M->slabs[s];
       AcVArgs a;
-      a.mp = S.mp;
+      a.mp = S.ac_pt;
+      a.mqx = S.ac_qc[0];
+      a.mqy = S.ac_qc[1];
+      a.mqz = S.ac_qc[2];
+      a.mbx = S.ac_bc[0];
+      a.mby = S.ac_bc[1];
+      a.mbz = S.ac_bc[2];
       a.p = S.fld[0];
       a.qx = S.fld[1];
       a.qy = S.fld[2];
       a.qz = S.fld[3];
-      a.bx = S.bx;
-      a.by = S.by;
-      a.bz = S.bz;
       a.W = M->W;
       a.zlo = 1;
       a.cx = M->cp[0];
@@ -1008,8 +1054,9 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       const dim3 gr = grid_of(S);
       {
         PROF(1, st);
-        if (a.img) ac_v_kernel<BY, true><<<gr, blk, 0, st>>>(a);
-        else ac_v_kernel<BY, false><<<gr, blk, 0, st>>>(a);
+        const size_t sb = AcVStage<BY>::smem_bytes();
+        if (a.img) ac_v_kernel<BY, true><<<gr, blk, sb, st>>>(a);
+        else ac_v_kernel<BY, false><<<gr, blk, sb, st>>>(a);
       }
       CKL();
     }
@@ -1017,11 +1064,12 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (size_t s = 0; s < M->slabs.size(); ++s) {
       Slab& S = M->slabs[s];
       AcPArgs a;
-      a.mqx = S.mqx;
-      a.mqy = S.mqy;
+      a.mqx = S.ac_qxt;
+      a.mqy = S.ac_qyt;
+      a.mpp = S.ac_pc;
+      a.mk = S.ac_kc;
       a.p = S.fld[0];
       a.qz = S.fld[3];
-      a.kdt = S.kdt;
       a.W = M->W;
       a.zlo = 1;
       a.cx = M->cp[0];
@@ -1039,8 +1087,9 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       const dim3 gr = grid_of(S);
       {
         PROF(2, st);
-        if (a.snap) ac_p_kernel<BY, true><<<gr, blk, 0, st>>>(a);
-        else ac_p_kernel<BY, false><<<gr, blk, 0, st>>>(a);
+        const size_t sb = AcPStage<BY>::smem_bytes();
+        if (a.snap) ac_p_kernel<BY, true><<<gr, blk, sb, st>>>(a);
+        else ac_p_kernel<BY, false><<<gr, blk, sb, st>>>(a);
       }
       CKL();
     }
@@ -1052,15 +1101,16 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
   for (size_t s = 0; s < M->slabs.size(); ++s) {
     Slab& S = M->slabs[s];
     ElVArgs a;
-    a.msxx = S.msxx;
-    a.msxy = S.msxy;
-    a.msxz = S.msxz;
-    a.msyy = S.msyy;
-    a.msyz = S.msyz;
+    a.msxx = S.el_sxxt;
+    a.msxy = S.el_sxyt;
+    a.msxz = S.el_sxzt;
+    a.msyy = S.el_syyt;
+    a.msyz = S.el_syzt;
+    for (int t = 0; t < 3; ++t) {
+      a.mv[t] = S.el_vc[t];
+      a.mb[t] = S.el_bc[t];
+    }
     for (int t = 0; t < 9; ++t) a.f[t] = S.fld[t];
-    a.bx = S.bx;
-    a.by = S.by;
-    a.bz = S.bz;
     a.W = M->W;
     a.zlo = M->g.free_surface ? 0 : 1;
     a.fs = M->g.free_surface;
@@ -1073,7 +1123,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     const dim3 gr = grid_of(S, BYE);
     {
       PROF(3, st);
-      el_v_kernel<BYE><<<gr, dim3(TXW, BYE), 0, st>>>(a);
+      el_v_kernel<BYE><<<gr, dim3(TXW, BYE), ElVStage<BYE>::smem_bytes(), st>>>(a);
     }
     CKL();
   }
@@ -1082,15 +1132,10 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
   for (size_t s = 0; s < M->slabs.size(); ++s) {
     Slab& S = M->slabs[s];
     ElSArgs a;
-    a.mvx = S.mvx;
-    a.mvy = S.mvy;
-    a.mvz = S.mvz;
+    for (int t = 0; t < 3; ++t) a.mvt[t] = S.el_vt[t];
+    for (int t = 0; t < 6; ++t) a.ms[t] = S.el_sc[t];
+    for (int t = 0; t < 5; ++t) a.mc[t] = S.el_cc[t];
     for (int t = 0; t < 9; ++t) a.f[t] = S.fld[t];
-    a.l2m = S.l2m;
-    a.lam = S.lam;
-    a.mxy = S.mxy;
-    a.mxz = S.mxz;
-    a.myz = S.myz;
     a.W = M->W;
     a.zlo = M->g.free_surface ? 0 : 1;
     a.fs = M->g.free_surface;
@@ -1106,7 +1151,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     const dim3 gr = grid_of(S, BYE);
     {
       PROF(4, st);
-      el_s_kernel<BYE, false><<<gr, dim3(TXW, BYE), 0, st>>>(a);
+      el_s_kernel<BYE, false><<<gr, dim3(TXW, BYE), ElSStage<BYE>::smem_bytes(), st>>>(a);
     }
     CKL();
   }
