@@ -8,9 +8,9 @@
 // z-slab is one fp32 array with G = 4 zero ghost cells on each side of every axis
 // ("Ghost node thickness is determined by the stencil"):
 //   padded dims  PX = roundup(roundup(nx, 32) + 2G, 32),  PY = roundup(ny, TY) + 2G,
-//                PZ = nz_local + 2G,  plane stride PS = PX * PY
+//                PZ = nz_local + 2GZ,  plane stride PS = PX * PY   (G = 4, GZ = 8)
 //   element (i, j, k) of the slab (interior coordinates) lives at
-//                ((k + G) * PY + (j + G)) * PX + (i + G)
+//                ((k + GZ) * PY + (j + G)) * PX + (i + G)
 // The base pointer of each array is offset so that x = 0 of every row is
 // 128-byte aligned (PX is a multiple of 32 floats).  Ghosts are never written, so
 // "values outside the grid are 0" (O1) costs no branch; the 4 z-ghost planes on a
@@ -21,7 +21,9 @@
 
 namespace seis {
 
-constexpr int G = 4;     // ghost width = stencil half-width (radius 4)
+constexpr int G = 4;     // x/y ghost width = stencil half-width (radius 4)
+constexpr int GZ = 8;    // z ghost depth: 4 for the stencil + 4 for the fused acoustic kernel's
+                         // recomputed q_z halo
 constexpr int TXW = 32;  // tile width in x = one warp
 
 struct Dims {
@@ -31,7 +33,7 @@ struct Dims {
   int PX, PY;       // padded pitches
   long long PS;     // plane stride
   __host__ __device__ __forceinline__ long long at(int i, int j, int k) const {
-    return ((long long)(k + G) * PY + (j + G)) * PX + (i + G);
+    return ((long long)(k + GZ) * PY + (j + G)) * PX + (i + G);
   }
 };
 
@@ -88,11 +90,15 @@ struct CpmlIdx {
 
 namespace seis {
 
-__device__ __forceinline__ float* align128(float* p) {
-  return reinterpret_cast<float*>((reinterpret_cast<uintptr_t>(p) + 127) & ~uintptr_t(127));
-}
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+// 128-byte aligned view of a dynamic shared-memory buffer.  Pointer arithmetic
+// (not an integer round trip) keeps the compiler's knowledge that the pointer is
+// shared, so accesses stay LDS/STS instead of generic LD/ST.
+__device__ __forceinline__ float* align128(float* p) {
+  const uint32_t pad = (128u - (smem_u32(p) & 127u)) & 127u;
+  return p + (pad >> 2);
 }
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
   asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");

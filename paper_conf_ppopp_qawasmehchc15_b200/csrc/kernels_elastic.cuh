@@ -133,7 +133,7 @@ __global__ void __launch_bounds__(TXW * BY) el_v_kernel(const __grid_constant__ 
   const float* __restrict__ szz = a.f[ESZZ];
   auto issue = [&](int s, int k) {
     float* st = sm + s * L::SIZE;
-    const int z = k + G;
+    const int z = k + GZ;
     mbar_expect_tx(&bar[s], TX_BYTES);
     tma_load_3d(st + L::XX, &a.msxx, &bar[s], i0, j0 + G, z);
     tma_load_3d(st + L::XY, &a.msxy, &bar[s], i0, j0, z);
@@ -156,23 +156,23 @@ __global__ void __launch_bounds__(TXW * BY) el_v_kernel(const __grid_constant__ 
   float qxz[8], qyz[8], qzz[8];  // sxz, syz at k-4..k+3 (D-); szz at k-3..k+4 (D+)
 #pragma unroll
   for (int t = 0; t < 7; ++t) {
-    qxz[t] = __ldg(sxz + (long long)(k0 - 4 + t + G) * PS + oc);
-    qyz[t] = __ldg(syz + (long long)(k0 - 4 + t + G) * PS + oc);
-    qzz[t] = __ldg(szz + (long long)(k0 - 3 + t + G) * PS + oc);
+    qxz[t] = __ldg(sxz + (long long)(k0 - 4 + t + GZ) * PS + oc);
+    qyz[t] = __ldg(syz + (long long)(k0 - 4 + t + GZ) * PS + oc);
+    qzz[t] = __ldg(szz + (long long)(k0 - 3 + t + GZ) * PS + oc);
   }
-  float axz = __ldg(sxz + (long long)(k0 + 3 + G) * PS + oc);
-  float ayz = __ldg(syz + (long long)(k0 + 3 + G) * PS + oc);
-  float azz = __ldg(szz + (long long)(k0 + 4 + G) * PS + oc);
+  float axz = __ldg(sxz + (long long)(k0 + 3 + GZ) * PS + oc);
+  float ayz = __ldg(syz + (long long)(k0 + 3 + GZ) * PS + oc);
+  float azz = __ldg(szz + (long long)(k0 + 4 + GZ) * PS + oc);
   float bxz = 0.f, byz = 0.f, bzz = 0.f;
   if (np > 1) {
-    bxz = __ldg(sxz + (long long)(k0 + 4 + G) * PS + oc);
-    byz = __ldg(syz + (long long)(k0 + 4 + G) * PS + oc);
-    bzz = __ldg(szz + (long long)(k0 + 5 + G) * PS + oc);
+    bxz = __ldg(sxz + (long long)(k0 + 4 + GZ) * PS + oc);
+    byz = __ldg(syz + (long long)(k0 + 4 + GZ) * PS + oc);
+    bzz = __ldg(szz + (long long)(k0 + 5 + GZ) * PS + oc);
   }
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % EL_NS;
-    const long long o = (long long)(k + G) * PS + oc;
+    const long long o = (long long)(k + GZ) * PS + oc;
     qxz[7] = axz; qyz[7] = ayz; qzz[7] = azz;
     axz = bxz; ayz = byz; azz = bzz;
     if (it + 2 < np) {
@@ -276,7 +276,7 @@ __global__ void __launch_bounds__(TXW * BY) el_s_kernel(const __grid_constant__ 
   const float* __restrict__ vz = a.f[EVZ];
   auto issue = [&](int s, int k) {
     float* st = sm + s * L::SIZE;
-    const int z = k + G;
+    const int z = k + GZ;
     mbar_expect_tx(&bar[s], TX_BYTES);
 #pragma unroll
     for (int c = 0; c < 3; ++c) tma_load_3d(st + L::VT + c * TV, &a.mvt[c], &bar[s], i0, j0, z);
@@ -295,23 +295,23 @@ __global__ void __launch_bounds__(TXW * BY) el_s_kernel(const __grid_constant__ 
   float qx[8], qy[8], qz[8];  // vx, vy at k-3..k+4 (D+); vz at k-4..k+3 (D-)
 #pragma unroll
   for (int t = 0; t < 7; ++t) {
-    qx[t] = __ldg(vx + (long long)(k0 - 3 + t + G) * PS + oc);
-    qy[t] = __ldg(vy + (long long)(k0 - 3 + t + G) * PS + oc);
-    qz[t] = __ldg(vz + (long long)(k0 - 4 + t + G) * PS + oc);
+    qx[t] = __ldg(vx + (long long)(k0 - 3 + t + GZ) * PS + oc);
+    qy[t] = __ldg(vy + (long long)(k0 - 3 + t + GZ) * PS + oc);
+    qz[t] = __ldg(vz + (long long)(k0 - 4 + t + GZ) * PS + oc);
   }
-  float ax = __ldg(vx + (long long)(k0 + 4 + G) * PS + oc);
-  float ay = __ldg(vy + (long long)(k0 + 4 + G) * PS + oc);
-  float az = __ldg(vz + (long long)(k0 + 3 + G) * PS + oc);
+  float ax = __ldg(vx + (long long)(k0 + 4 + GZ) * PS + oc);
+  float ay = __ldg(vy + (long long)(k0 + 4 + GZ) * PS + oc);
+  float az = __ldg(vz + (long long)(k0 + 3 + GZ) * PS + oc);
   float bx = 0.f, by = 0.f, bz = 0.f;
   if (np > 1) {
-    bx = __ldg(vx + (long long)(k0 + 5 + G) * PS + oc);
-    by = __ldg(vy + (long long)(k0 + 5 + G) * PS + oc);
-    bz = __ldg(vz + (long long)(k0 + 4 + G) * PS + oc);
+    bx = __ldg(vx + (long long)(k0 + 5 + GZ) * PS + oc);
+    by = __ldg(vy + (long long)(k0 + 5 + GZ) * PS + oc);
+    bz = __ldg(vz + (long long)(k0 + 4 + GZ) * PS + oc);
   }
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % EL_NS;
-    const long long o = (long long)(k + G) * PS + oc;
+    const long long o = (long long)(k + GZ) * PS + oc;
     qx[7] = ax; qy[7] = ay; qz[7] = az;
     ax = bx; ay = by; az = bz;
     if (it + 2 < np) {

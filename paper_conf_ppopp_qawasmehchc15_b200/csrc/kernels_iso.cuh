@@ -67,9 +67,9 @@ __global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const __grid_constan
   auto issue = [&](int s, int k) {
     float* st = sm + s * L::SIZE;
     mbar_expect_tx(&bar[s], TX_BYTES);
-    tma_load_3d(st + L::U, &a.mun, &bar[s], i0, j0, k + G);
-    tma_load_3d(st + L::UP, &a.mup, &bar[s], i0 + G, j0 + G, k + G);
-    tma_load_3d(st + L::M, &a.mm, &bar[s], i0 + G, j0 + G, k + G);
+    tma_load_3d(st + L::U, &a.mun, &bar[s], i0, j0, k + GZ);
+    tma_load_3d(st + L::UP, &a.mup, &bar[s], i0 + G, j0 + G, k + GZ);
+    tma_load_3d(st + L::M, &a.mm, &bar[s], i0 + G, j0 + G, k + GZ);
   };
   if (tid == 0) {
     for (int s = 0; s < ISO_NS; ++s) mbar_init(&bar[s], 1);
@@ -81,22 +81,22 @@ __global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const __grid_constan
 
   // z-queue u^n(k-4 .. k+4), fed two planes ahead
   float q0, q1, q2, q3, q4, q5, q6, q7, q8;
-  q0 = __ldg(un + (long long)(k0 - 4 + G) * PS + oc);
-  q1 = __ldg(un + (long long)(k0 - 3 + G) * PS + oc);
-  q2 = __ldg(un + (long long)(k0 - 2 + G) * PS + oc);
-  q3 = __ldg(un + (long long)(k0 - 1 + G) * PS + oc);
-  q4 = __ldg(un + (long long)(k0 + G) * PS + oc);
-  q5 = __ldg(un + (long long)(k0 + 1 + G) * PS + oc);
-  q6 = __ldg(un + (long long)(k0 + 2 + G) * PS + oc);
-  q7 = __ldg(un + (long long)(k0 + 3 + G) * PS + oc);
-  float na = __ldg(un + (long long)(k0 + 4 + G) * PS + oc);
-  float nb = np > 1 ? __ldg(un + (long long)(k0 + 5 + G) * PS + oc) : 0.f;
+  q0 = __ldg(un + (long long)(k0 - 4 + GZ) * PS + oc);
+  q1 = __ldg(un + (long long)(k0 - 3 + GZ) * PS + oc);
+  q2 = __ldg(un + (long long)(k0 - 2 + GZ) * PS + oc);
+  q3 = __ldg(un + (long long)(k0 - 1 + GZ) * PS + oc);
+  q4 = __ldg(un + (long long)(k0 + GZ) * PS + oc);
+  q5 = __ldg(un + (long long)(k0 + 1 + GZ) * PS + oc);
+  q6 = __ldg(un + (long long)(k0 + 2 + GZ) * PS + oc);
+  q7 = __ldg(un + (long long)(k0 + 3 + GZ) * PS + oc);
+  float na = __ldg(un + (long long)(k0 + 4 + GZ) * PS + oc);
+  float nb = np > 1 ? __ldg(un + (long long)(k0 + 5 + GZ) * PS + oc) : 0.f;
   const float exy = (a.edx && own) ? a.edx[i] + a.edy[j] : 0.0f;
 
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % ISO_NS;
-    const long long o = (long long)(k + G) * PS + oc;
+    const long long o = (long long)(k + GZ) * PS + oc;
     q8 = na;
     na = nb;
     if (it + 2 < np) nb = __ldg(un + o + 6 * PS);

@@ -15,6 +15,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
+#include <functional>
 #include <map>
 #include <string>
 #include <vector>
@@ -114,14 +115,15 @@ struct Slab {
   Dims d{};
   std::vector<float*> fld;   // padded state fields
   float* m = nullptr;        // ISO
-  float* kdt = nullptr;      // ACOUSTIC
+  float* kdt = nullptr;      // ACOUSTIC dt K / h
+  float* rho = nullptr;      // ACOUSTIC density (z ghosts filled from the neighbour slabs)
   float *bx = nullptr, *by = nullptr, *bz = nullptr;                          // ACOUSTIC, ELASTIC
   float *l2m = nullptr, *lam = nullptr, *mxy = nullptr, *mxz = nullptr, *myz = nullptr;  // ELASTIC
   float* psi[NPSI] = {};
   // TMA descriptors of every operand tile the kernels stage:
   // "t" = tile with x/y halo, "c" = interior (centre) tile 32 x BY
   CUtensorMap iso_ut[2], iso_uc[2], iso_m;                              // ISO
-  CUtensorMap ac_pt, ac_qc[3], ac_bc[3], ac_qxt, ac_qyt, ac_pc, ac_kc;   // ACOUSTIC
+  CUtensorMap ac_pt[2], ac_qxt[2], ac_qyt[2], ac_rt, ac_kc;             // ACOUSTIC (A/B buffers)
   CUtensorMap el_sxxt, el_sxyt, el_sxzt, el_syyt, el_syzt, el_vc[3], el_bc[3];  // ELASTIC V
   CUtensorMap el_vt[3], el_sc[6], el_cc[5];                             // ELASTIC S
   int cur = 0;               // ISO: fld[cur] = u^n
@@ -189,7 +191,7 @@ seis_status alloc_track(seis_model* M, void** p, size_t bytes) {
 
 // Padded field: ghosts zero, x = 0 of each row 128-byte aligned.
 seis_status alloc_padded(seis_model* M, const Dims& d, float** out, cudaStream_t st) {
-  size_t elems = (size_t)d.PS * (size_t)(d.nzl + 2 * G);
+  size_t elems = (size_t)d.PS * (size_t)(d.nzl + 2 * GZ);
   void* base = nullptr;
   TRY(alloc_track(M, &base, elems * sizeof(float) + 128));
   CK(cudaMemsetAsync(base, 0, elems * sizeof(float) + 128, st));
@@ -210,7 +212,7 @@ seis_status make_map(CUtensorMap* m, float* base, const Dims& d, int bw, int bh)
     if (q != cudaDriverEntryPointSuccess || !fn) return fail(SEIS_ECUDA, "cuTensorMapEncodeTiled unavailable");
     g_encode = (PFN_cuTensorMapEncodeTiled_v12000)fn;
   }
-  cuuint64_t dims[3] = {(cuuint64_t)d.PX, (cuuint64_t)d.PY, (cuuint64_t)(d.nzl + 2 * G)};
+  cuuint64_t dims[3] = {(cuuint64_t)d.PX, (cuuint64_t)d.PY, (cuuint64_t)(d.nzl + 2 * GZ)};
   cuuint64_t str[2] = {(cuuint64_t)d.PX * 4, (cuuint64_t)d.PS * 4};
   cuuint32_t box[3] = {(cuuint32_t)bw, (cuuint32_t)bh, 1};
   cuuint32_t es[3] = {1, 1, 1};
@@ -298,10 +300,9 @@ seis_status set_smem_attrs() {
   SMEM_ATTR((iso_step_kernel<BY, false, false>), IsoStage<BY>::smem_bytes());
   SMEM_ATTR((iso_step_kernel<BY, true, false>), IsoStage<BY>::smem_bytes());
   SMEM_ATTR((iso_step_kernel<BY, false, true>), IsoStage<BY>::smem_bytes());
-  SMEM_ATTR((ac_v_kernel<BY, false>), AcVStage<BY>::smem_bytes());
-  SMEM_ATTR((ac_v_kernel<BY, true>), AcVStage<BY>::smem_bytes());
-  SMEM_ATTR((ac_p_kernel<BY, false>), AcPStage<BY>::smem_bytes());
-  SMEM_ATTR((ac_p_kernel<BY, true>), AcPStage<BY>::smem_bytes());
+  SMEM_ATTR((ac_step_kernel<BY, false, false>), AcFStage<BY>::smem_bytes());
+  SMEM_ATTR((ac_step_kernel<BY, true, false>), AcFStage<BY>::smem_bytes());
+  SMEM_ATTR((ac_step_kernel<BY, false, true>), AcFStage<BY>::smem_bytes());
   SMEM_ATTR((el_v_kernel<BYE>), ElVStage<BYE>::smem_bytes());
   SMEM_ATTR((el_s_kernel<BYE, false>), ElSStage<BYE>::smem_bytes());
 #undef SMEM_ATTR
@@ -330,52 +331,69 @@ void choose_chunks(Slab& s, int resident_per_sm, int nsm, int by) {
   s.nzch = (s.d.nzl + s.zc - 1) / s.zc;
 }
 
-int nfields(seis_kind k) { return k == SEIS_ISO ? 2 : (k == SEIS_ACOUSTIC ? 4 : 9); }
+// ISO: u at two time levels; ACOUSTIC: (p, qx, qy, qz) x 2 buffers (fused step reads A,
+// writes B); ELASTIC: 9 fields updated in place.
+int nfields(seis_kind k) { return k == SEIS_ISO ? 2 : (k == SEIS_ACOUSTIC ? 8 : 9); }
+int npsi_of(seis_kind k) { return k == SEIS_ACOUSTIC ? 9 : (k == SEIS_ELASTIC ? 18 : 0); }
+// axis of each C-PML memory array: ACOUSTIC psi_p A (x,y,z), psi_q (x,y,z), psi_p B (x,y,z);
+// ELASTIC in the oracle's order
+int psi_axis(seis_kind k, int t) {
+  static const int el_axis[18] = {0, 1, 2, 0, 1, 2, 0, 1, 2, 0, 1, 2, 1, 0, 2, 0, 2, 1};
+  return k == SEIS_ACOUSTIC ? t % 3 : el_axis[t];
+}
 
-// Ghost-plane exchange of `fields` between the slabs of this process and, with a
-// communicator, with the neighbouring ranks (4 contiguous planes per face).
-seis_status exchange(seis_model* M, const std::vector<int>& fields, cudaStream_t st,
-                     const std::vector<int>* iso_cur = nullptr) {
+// Ghost-plane exchange between the slabs of this process and, with a
+// communicator, with the neighbouring ranks: `np` contiguous planes per face of
+// each array `arr(slab)` (a field, or a coefficient array at create time).
+using ArrFn = std::function<float*(Slab&)>;
+
+seis_status exchange_arrays(seis_model* M, const std::vector<ArrFn>& arrs, int np, cudaStream_t st) {
   if (M->slabs.size() < 2 && !(M->comm && M->nranks > 1)) return SEIS_OK;
   PROF(7, st);
-  const size_t plane4 = 0;
-  (void)plane4;
   for (size_t s = 0; s + 1 < M->slabs.size(); ++s) {
     Slab& A = M->slabs[s];
     Slab& B = M->slabs[s + 1];
-    const size_t n4 = (size_t)4 * A.d.PS;
-    for (int f : fields) {
-      float* fa = A.fld[f];
-      float* fb = B.fld[f];
-      // A's bottom ghosts (k = nzl .. nzl+3) <- B's planes 0..3
-      CK(cudaMemcpyAsync(fa + (size_t)(A.d.nzl + G) * A.d.PS, fb + (size_t)G * B.d.PS,
-                         n4 * sizeof(float), cudaMemcpyDeviceToDevice, st));
-      // B's top ghosts (k = -4 .. -1) <- A's planes nzl-4 .. nzl-1
-      CK(cudaMemcpyAsync(fb, fa + (size_t)(A.d.nzl) * A.d.PS, n4 * sizeof(float),
-                         cudaMemcpyDeviceToDevice, st));
+    const size_t n = (size_t)np * A.d.PS;
+    for (const ArrFn& arr : arrs) {
+      float* fa = arr(A);
+      float* fb = arr(B);
+      // A's bottom ghosts (k = nzl .. nzl+np-1) <- B's planes 0 .. np-1
+      CK(cudaMemcpyAsync(fa + (size_t)(A.d.nzl + GZ) * A.d.PS, fb + (size_t)GZ * B.d.PS,
+                         n * sizeof(float), cudaMemcpyDeviceToDevice, st));
+      // B's top ghosts (k = -np .. -1) <- A's planes nzl-np .. nzl-1
+      CK(cudaMemcpyAsync(fb + (size_t)(GZ - np) * B.d.PS, fa + (size_t)(A.d.nzl + GZ - np) * A.d.PS,
+                         n * sizeof(float), cudaMemcpyDeviceToDevice, st));
     }
   }
   if (M->comm && M->nranks > 1) {
     Slab& top = M->slabs.front();
     Slab& bot = M->slabs.back();
-    const size_t n4 = (size_t)4 * top.d.PS;
+    const size_t n = (size_t)np * top.d.PS;
     NK(ncclGroupStart());
-    for (int f : fields) {
+    for (const ArrFn& arr : arrs) {
+      float* ft = arr(top);
+      float* fbm = arr(bot);
       if (M->rank > 0) {
-        NK(ncclSend(top.fld[f] + (size_t)G * top.d.PS, n4, ncclFloat, M->rank - 1, M->comm->nccl, st));
-        NK(ncclRecv(top.fld[f], n4, ncclFloat, M->rank - 1, M->comm->nccl, st));
+        NK(ncclSend(ft + (size_t)GZ * top.d.PS, n, ncclFloat, M->rank - 1, M->comm->nccl, st));
+        NK(ncclRecv(ft + (size_t)(GZ - np) * top.d.PS, n, ncclFloat, M->rank - 1, M->comm->nccl, st));
       }
       if (M->rank < M->nranks - 1) {
-        NK(ncclSend(bot.fld[f] + (size_t)bot.d.nzl * bot.d.PS, n4, ncclFloat, M->rank + 1,
+        NK(ncclSend(fbm + (size_t)(bot.d.nzl + GZ - np) * bot.d.PS, n, ncclFloat, M->rank + 1,
                     M->comm->nccl, st));
-        NK(ncclRecv(bot.fld[f] + (size_t)(bot.d.nzl + G) * bot.d.PS, n4, ncclFloat, M->rank + 1,
+        NK(ncclRecv(fbm + (size_t)(bot.d.nzl + GZ) * bot.d.PS, n, ncclFloat, M->rank + 1,
                     M->comm->nccl, st));
       }
     }
     NK(ncclGroupEnd());
   }
-  (void)iso_cur;
   return SEIS_OK;
+}
+
+// 4-plane exchange of state fields by index
+seis_status exchange(seis_model* M, const std::vector<int>& fields, cudaStream_t st) {
+  std::vector<ArrFn> arrs;
+  for (int f : fields) arrs.push_back([f](Slab& S) { return S.fld[f]; });
+  return exchange_arrays(M, arrs, 4, st);
 }
 
 }  // namespace
@@ -589,10 +607,24 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
 
   // slabs of this process
   const int ns = g.slabs;
-  if (M->pnzl < 4 * ns && (ns > 1 || M->nranks > 1))
-    return fail(SEIS_EINVAL, "each z-slab needs >= 4 planes (nz_local=%d, slabs=%d)", M->pnzl, ns);
   int dev_sms = 148;
   CK(cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, M->device));
+  if (ns > 1 || M->nranks > 1) {
+    // every internal slab boundary must keep the recomputed ghost planes (8 deep) out of the
+    // absorbing layers and each slab must hold the 8 planes its neighbours read
+    const int W = g.nb > 0 ? g.nb + 1 : 0;
+    for (int r = 0; r < M->nranks; ++r)
+      for (int s = 0; s < ns; ++s) {
+        int rz0, rn, lz0, ln;
+        seis_slab_bounds(g.nz, M->nranks, r, &rz0, &rn);
+        seis_slab_bounds(rn, ns, s, &lz0, &ln);
+        const int z0 = rz0 + lz0;
+        const int need = kind == SEIS_ACOUSTIC ? GZ : 4;
+        if (ln < need) return fail(SEIS_EINVAL, "z-slab of %d planes: the decomposition needs >= %d", ln, need);
+        if (kind == SEIS_ACOUSTIC && z0 > 0 && (z0 - GZ < W || z0 + GZ > g.nz - W))
+          return fail(SEIS_EINVAL, "slab boundary z=%d lies within %d planes of an absorbing layer", z0, GZ);
+      }
+  }
   M->slabs.resize(ns);
   for (int s = 0; s < ns; ++s) {
     int lz0, lnz;
@@ -624,7 +656,8 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       TRY(upload_padded_from_host(M, d, hc, &S.m, st));
     } else {
       // buoyancy on faces (O8): dt * 2/(rho_i + rho_{i+1}) / h, last face clamps
-      for (int ax = 0; ax < 3; ++ax) {
+      // (ELASTIC only; the fused acoustic step evaluates it on the fly from rho)
+      for (int ax = 0; ax < 3 && kind == SEIS_ELASTIC; ++ax) {
         for (int k = 0; k < lnz; ++k)
           for (int j = 0; j < g.ny; ++j)
             for (int i = 0; i < g.nx; ++i) {
@@ -645,6 +678,8 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
           hc[t] = (float)(dt * r * v * v / h);
         }
         TRY(upload_padded_from_host(M, d, hc, &S.kdt, st));
+        for (size_t t = 0; t < sp; ++t) hc[t] = M->hrho[off + t];
+        TRY(upload_padded_from_host(M, d, hc, &S.rho, st));
       } else {
         auto mu_at = [&](int i, int j, int k) {
           const double s_ = val(M->hvs, nvs, 0, i, j, k), r_ = val(M->hrho, nrho, 0, i, j, k);
@@ -689,11 +724,9 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       // compact C-PML memory slabs
       if (M->W > 0) {
         const int W = M->W;
-        const int npsi = kind == SEIS_ACOUSTIC ? 6 : 18;
-        // axis of each psi: acoustic 0,1,2,0,1,2; elastic per the oracle's order
-        static const int el_axis[18] = {0, 1, 2, 0, 1, 2, 0, 1, 2, 0, 1, 2, 1, 0, 2, 0, 2, 1};
+        const int npsi = npsi_of(kind);
         for (int t = 0; t < npsi; ++t) {
-          const int ax = kind == SEIS_ACOUSTIC ? t % 3 : el_axis[t];
+          const int ax = psi_axis(kind, t);
           size_t n;
           if (ax == 0) n = (size_t)lnz * g.ny * 2 * W;
           else if (ax == 1) n = (size_t)lnz * 2 * W * g.nx;
@@ -710,15 +743,12 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       }
       TRY(make_map(&S.iso_m, S.m, d, TXW, BY));
     } else if (kind == SEIS_ACOUSTIC) {
-      TRY(make_map(&S.ac_pt, S.fld[0], d, TXW + 8, BY + 8));
-      float* bb[3] = {S.bx, S.by, S.bz};
-      for (int t = 0; t < 3; ++t) {
-        TRY(make_map(&S.ac_qc[t], S.fld[1 + t], d, TXW, BY));
-        TRY(make_map(&S.ac_bc[t], bb[t], d, TXW, BY));
+      for (int b = 0; b < 2; ++b) {
+        TRY(make_map(&S.ac_pt[b], S.fld[4 * b + 0], d, TXW + 16, BY + 16));
+        TRY(make_map(&S.ac_qxt[b], S.fld[4 * b + 1], d, TXW + 8, BY));
+        TRY(make_map(&S.ac_qyt[b], S.fld[4 * b + 2], d, TXW, BY + 8));
       }
-      TRY(make_map(&S.ac_qxt, S.fld[1], d, TXW + 8, BY));
-      TRY(make_map(&S.ac_qyt, S.fld[2], d, TXW, BY + 8));
-      TRY(make_map(&S.ac_pc, S.fld[0], d, TXW, BY));
+      TRY(make_map(&S.ac_rt, S.rho, d, TXW + 16, BY + 16));
       TRY(make_map(&S.ac_kc, S.kdt, d, TXW, BY));
     } else {
       TRY(make_map(&S.el_sxxt, S.fld[ESXX], d, TXW + 8, BYE));
@@ -742,12 +772,16 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, iso_step_kernel<BY, false, false>, TXW * BY,
                                                     IsoStage<BY>::smem_bytes());
     else if (kind == SEIS_ACOUSTIC)
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_v_kernel<BY, false>, TXW * BY,
-                                                    AcVStage<BY>::smem_bytes());
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_step_kernel<BY, false, false>, TXW * BY,
+                                                    AcFStage<BY>::smem_bytes());
     else
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, TXW * BYE,
                                                     ElSStage<BYE>::smem_bytes());
     choose_chunks(S, occ, dev_sms, kind == SEIS_ELASTIC ? BYE : BY);
+  }
+  if (kind == SEIS_ACOUSTIC) {
+    // rho z-ghosts from the neighbouring slabs / ranks (the fused step recomputes q_z on them)
+    TRY(exchange_arrays(M, {[](Slab& S) { return S.rho; }}, GZ, st));
   }
   CK(cudaStreamSynchronize(st));
   return SEIS_OK;
@@ -810,13 +844,13 @@ seis_status seis_memory_required(const seis_grid* g, seis_kind kind, const seis_
   int32_t z0, nzl;
   seis_slab_bounds(g->nz, nranks, 0, &z0, &nzl);
   const Dims d = make_dims(*g, 0, nzl);
-  const double padded = (double)d.PS * (nzl + 2 * G) * 4.0;
-  int nf = nfields(kind), np = kind == SEIS_ISO ? 1 : (kind == SEIS_ACOUSTIC ? 4 : 8);
+  const double padded = (double)d.PS * (nzl + 2 * GZ) * 4.0;
+  int nf = nfields(kind), np = kind == SEIS_ISO ? 1 : (kind == SEIS_ACOUSTIC ? 2 : 8);
   double b = (nf + np) * padded;
   if (kind != SEIS_ISO && g->nb > 0) {
     const double W = g->nb + 1;
     const double per = (2 * W * g->ny * (double)nzl + 2 * W * g->nx * (double)nzl + 2 * W * g->nx * (double)g->ny) * 4.0;
-    b += per * (kind == SEIS_ACOUSTIC ? 2 : 6);
+    b += per * (kind == SEIS_ACOUSTIC ? 3 : 6);
   }
   if (shot && shot->snap_period >= 1 && shot->nt >= 1)
     b += (double)((shot->nt - 1) / shot->snap_period) * nzl * (double)g->ny * g->nx * 4.0;
@@ -924,14 +958,13 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
 // Zero the state of every slab (fields incl. ghosts, C-PML slabs).
 seis_status zero_state(seis_model* M, cudaStream_t st) {
   for (Slab& S : M->slabs) {
-    const size_t elems = (size_t)S.d.PS * (S.d.nzl + 2 * G);
+    const size_t elems = (size_t)S.d.PS * (S.d.nzl + 2 * GZ);
     for (float* f : S.fld) CK(cudaMemsetAsync(f, 0, elems * sizeof(float), st));
     if (M->W > 0) {
       const int W = M->W;
-      const int npsi = M->kind == SEIS_ACOUSTIC ? 6 : (M->kind == SEIS_ELASTIC ? 18 : 0);
-      static const int el_axis[18] = {0, 1, 2, 0, 1, 2, 0, 1, 2, 0, 1, 2, 1, 0, 2, 0, 2, 1};
+      const int npsi = npsi_of(M->kind);
       for (int t = 0; t < npsi; ++t) {
-        const int ax = M->kind == SEIS_ACOUSTIC ? t % 3 : el_axis[t];
+        const int ax = psi_axis(M->kind, t);
         size_t n;
         if (ax == 0) n = (size_t)S.d.nzl * S.d.ny * 2 * W;
         else if (ax == 1) n = (size_t)S.d.nzl * 2 * W * S.d.nx;
@@ -971,7 +1004,7 @@ dim3 grid_of(const Slab& S, int by = BY) {
 seis_status inject_rows(seis_model* M, const float* row, cudaStream_t st) {
   for (Slab& S : M->slabs) {
     if (S.ngroups == 0) continue;
-    float* f = M->kind == SEIS_ISO ? S.fld[S.cur] : S.fld[0];
+    float* f = M->kind == SEIS_ISO ? S.fld[S.cur] : S.fld[4 * S.cur];
     PROF(5, st);
     inject_kernel<<<(S.ngroups + 127) / 128, 128, 0, st>>>(f, S.d_g_off, S.d_g_scale, S.d_g_start,
                                                            S.d_g_mem, row, S.ngroups);
@@ -1027,54 +1060,34 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
   if (M->kind == SEIS_ACOUSTIC) {
     for (size_t s = 0; s < M->slabs.size(); ++s) {
       Slab& S = M->slabs[s];
-      AcVArgs a;
-      a.mp = S.ac_pt;
-      a.mqx = S.ac_qc[0];
-      a.mqy = S.ac_qc[1];
-      a.mqz = S.ac_qc[2];
-      a.mbx = S.ac_bc[0];
-      a.mby = S.ac_bc[1];
-      a.mbz = S.ac_bc[2];
-      a.p = S.fld[0];
-      a.qx = S.fld[1];
-      a.qy = S.fld[2];
-      a.qz = S.fld[3];
-      a.W = M->W;
-      a.zlo = 1;
-      a.cx = M->cp[0];
-      a.cy = M->cp[1];
-      a.cz = M->cp[2];
-      a.psx = S.psi[0];
-      a.psy = S.psi[1];
-      a.psz = S.psi[2];
-      a.d = S.d;
-      a.zc = S.zc;
-      a.imgS = imgS ? (*imgS)[s] : nullptr;
-      a.img = img ? (*img)[s] : nullptr;
-      const dim3 gr = grid_of(S);
-      {
-        PROF(1, st);
-        const size_t sb = AcVStage<BY>::smem_bytes();
-        if (a.img) ac_v_kernel<BY, true><<<gr, blk, sb, st>>>(a);
-        else ac_v_kernel<BY, false><<<gr, blk, sb, st>>>(a);
-      }
-      CKL();
-    }
-    TRY(exchange(M, {3}, st));  // q_z has the only z-derivative in P
-    for (size_t s = 0; s < M->slabs.size(); ++s) {
-      Slab& S = M->slabs[s];
-      AcPArgs a;
-      a.mqx = S.ac_qxt;
-      a.mqy = S.ac_qyt;
-      a.mpp = S.ac_pc;
+      const int A = S.cur, B = 1 - S.cur;
+      AcFArgs a;
+      a.mp = S.ac_pt[A];
+      a.mr = S.ac_rt;
+      a.mqx = S.ac_qxt[A];
+      a.mqy = S.ac_qyt[A];
       a.mk = S.ac_kc;
-      a.p = S.fld[0];
-      a.qz = S.fld[3];
+      a.pA = S.fld[4 * A];
+      a.qzA = S.fld[4 * A + 3];
+      a.rho = S.rho;
+      a.pB = S.fld[4 * B];
+      a.qxB = S.fld[4 * B + 1];
+      a.qyB = S.fld[4 * B + 2];
+      a.qzB = S.fld[4 * B + 3];
+      a.dth = (float)((double)M->g.dt / (double)M->g.h);
       a.W = M->W;
       a.zlo = 1;
       a.cx = M->cp[0];
       a.cy = M->cp[1];
       a.cz = M->cp[2];
+      float** pin = A == 0 ? S.psi + 0 : S.psi + 6;
+      float** pout = A == 0 ? S.psi + 6 : S.psi + 0;
+      a.psxA = pin[0];
+      a.psyA = pin[1];
+      a.pszA = pin[2];
+      a.psxB = pout[0];
+      a.psyB = pout[1];
+      a.pszB = pout[2];
       a.pqx = S.psi[3];
       a.pqy = S.psi[4];
       a.pqz = S.psi[5];
@@ -1084,17 +1097,25 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.src_amp = 0.f;
       if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
       a.snap = snap ? (*snap)[s] : nullptr;
+      a.imgS = imgS ? (*imgS)[s] : nullptr;
+      a.img = img ? (*img)[s] : nullptr;
       const dim3 gr = grid_of(S);
       {
-        PROF(2, st);
-        const size_t sb = AcPStage<BY>::smem_bytes();
-        if (a.snap) ac_p_kernel<BY, true><<<gr, blk, sb, st>>>(a);
-        else ac_p_kernel<BY, false><<<gr, blk, sb, st>>>(a);
+        PROF(1, st);
+        const size_t sb = AcFStage<BY>::smem_bytes();
+        if (a.snap) ac_step_kernel<BY, true, false><<<gr, blk, sb, st>>>(a);
+        else if (a.img) ac_step_kernel<BY, false, true><<<gr, blk, sb, st>>>(a);
+        else ac_step_kernel<BY, false, false><<<gr, blk, sb, st>>>(a);
       }
       CKL();
     }
+    for (Slab& S : M->slabs) S.cur = 1 - S.cur;
     if (inj_row) TRY(inject_rows(M, inj_row, st));
-    TRY(exchange(M, {0}, st));  // p for the next V
+    // ghosts of the new level: p (8 planes, the next step recomputes q_z on ghost planes
+    // from p at k-3 .. k+4) and q_z (4 planes)
+    const int c = M->slabs[0].cur;
+    TRY(exchange_arrays(M, {[c](Slab& S) { return S.fld[4 * c]; }}, GZ, st));
+    TRY(exchange(M, {4 * c + 3}, st));
     return SEIS_OK;
   }
   // ELASTIC
@@ -1163,7 +1184,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
 // Field holding the recorded / imaged quantity
 const float* out_field(seis_model* M, Slab& S, int comp) {
   if (M->kind == SEIS_ISO) return S.fld[S.cur];
-  if (M->kind == SEIS_ACOUSTIC) return S.fld[0];
+  if (M->kind == SEIS_ACOUSTIC) return S.fld[4 * S.cur];
   if (comp == 3) return S.fld[3];
   return S.fld[comp];
 }
@@ -1321,7 +1342,7 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
 seis_status seis_get_field(const seis_model* Mc, int32_t which, float* dst, void* stream) {
   seis_model* M = const_cast<seis_model*>(Mc);
   if (!M || !dst) return fail(SEIS_EINVAL, "null argument");
-  const int nf = nfields(M->kind);
+  const int nf = M->kind == SEIS_ACOUSTIC ? 4 : nfields(M->kind);
   if (which < 0 || which >= nf) return fail(SEIS_EINVAL, "field index %d out of range", which);
   CK(cudaSetDevice(M->device));
   cudaStream_t st = (cudaStream_t)stream;
@@ -1336,6 +1357,7 @@ seis_status seis_get_field(const seis_model* Mc, int32_t which, float* dst, void
   for (Slab& S : M->slabs) {
     int f = which;
     if (M->kind == SEIS_ISO) f = which == 0 ? S.cur : 1 - S.cur;
+    if (M->kind == SEIS_ACOUSTIC) f = 4 * S.cur + which;
     unpad_kernel<<<1024, 256, 0, st>>>(out + (size_t)(S.d.z0 - M->pz0) * g.ny * g.nx, S.fld[f], S.d);
     CKL();
   }
