@@ -6,7 +6,7 @@
 Headline (BASELINE.json configs[1], "C2"): acoustic 3D, 512^3 layered model,
 2000 time steps, C-PML (nb = 20) on 6 faces, 472-receiver surface line, one
 Ricker shot.  One bench "step" = one seismic-modeling shot (seis_forward_model:
-every time step's fused V+P kernel with source injection, and the receiver gather).  metric =
+every time step's V and P kernels (source injection fused into P) and the receiver gather).  metric =
 Gpts/s = grid points x time steps / second (whole job over all ranks).
 
 * value:  device-timed (CUDA events on the launching stream, barrier + synchronize on
@@ -44,8 +44,8 @@ METRIC = "Gpts/s per propagator and RTM shots/hour; % of B200 HBM roofline at 1/
 
 # algorithmic bytes per grid point per launch: each state field read once and
 # written once, model coefficients read once, C-PML memory variables RMW only inside layers
-ALG_BYTES = {"iso_step": 16.0, "ac_step": 40.0, "el_v": 52.0, "el_s": 68.0}
-PSI_AXES = {"ac_step": 6, "el_v": 9, "el_s": 9}
+ALG_BYTES = {"iso_step": 16.0, "ac_v": 32.0, "ac_p": 24.0, "el_v": 52.0, "el_s": 68.0}
+PSI_AXES = {"ac_v": 3, "ac_p": 3, "el_v": 9, "el_s": 9}
 
 
 def peaks():
@@ -209,7 +209,7 @@ def run_product(args):
 
     # roofline of the dominant kernel
     hbm, peak_src = peaks()
-    dom = "ac_step"
+    dom = max(("ac_v", "ac_p"), key=lambda k: kprof.get(k, (0, 1))[0])
     kms, kn = kprof[dom]
     local_pts = float(wl.nx) * wl.ny * nzl
     bpp = ALG_BYTES[dom] + psi_bytes_per_point(wl.nx, wl.ny, nz, wl.nb, PSI_AXES[dom])

@@ -152,7 +152,7 @@ seis_status seis_memory_required(const seis_grid* grid, seis_kind kind, const se
  * counters and starts recording an event pair on the launching stream around every
  * launch; seis_profile(0) stops.  seis_profile_read synchronises on the recorded
  * events and returns the summed device time and launch count of kernel id
- *   0 iso_step  1 ac_step (fused acoustic V+P)  2 (unused)  3 el_v  4 el_s  5 inject  6 gather
+ *   0 iso_step  1 ac_v  2 ac_p  3 el_v  4 el_s  5 inject  6 gather
  *   7 halo exchange (copies / NCCL)  8 free-surface mirror.
  * Process-wide, not thread-safe; meant for single-threaded measurement runs. */
 seis_status seis_profile(int32_t enable);

@@ -62,9 +62,14 @@ static int wrap(int i, int n) {
   return i < 0 ? i + n : i;
 }
 
-/* Value of f at (i,j,k): zero outside the grid (O1), or periodic wrap (O4 test mode). */
+/* Value of f at (i,j,k): zero outside the grid (O1), or periodic wrap (O4 test mode;
+ * with a free surface the wrap is lateral only and z keeps zero ghosts below the grid). */
 static double at(const or_grid* g, const double* f, int i, int j, int k) {
-  if (g->periodic) return f[IDX(g, wrap(i, g->nx), wrap(j, g->ny), wrap(k, g->nz))];
+  if (g->periodic) {
+    i = wrap(i, g->nx);
+    j = wrap(j, g->ny);
+    if (!g->free_surface) k = wrap(k, g->nz);
+  }
   if (i < 0 || j < 0 || k < 0 || i >= g->nx || j >= g->ny || k >= g->nz) return 0.0;
   return f[IDX(g, i, j, k)];
 }
@@ -267,7 +272,7 @@ static double face_buoy(const or_grid* g, const float* rho, int axis, int i, int
   e[axis] = 1;
   int n[3] = {g->nx, g->ny, g->nz};
   int c[3] = {i + e[0], j + e[1], k + e[2]};
-  if (c[axis] >= n[axis]) c[axis] = g->periodic ? 0 : n[axis] - 1;
+  if (c[axis] >= n[axis]) c[axis] = (g->periodic && !(axis == 2 && g->free_surface)) ? 0 : n[axis] - 1;
   double r0 = atf(g, rho, i, j, k);
   double r1 = atf(g, rho, c[0], c[1], c[2]);
   return 2.0 / (r0 + r1);
@@ -400,12 +405,12 @@ static double node_mu(const or_grid* g, const float* vs, const float* rho, int i
   if (g->periodic) {
     i = wrap(i, g->nx);
     j = wrap(j, g->ny);
-    k = wrap(k, g->nz);
   } else {
     if (i >= g->nx) i = g->nx - 1;
     if (j >= g->ny) j = g->ny - 1;
-    if (k >= g->nz) k = g->nz - 1;
   }
+  if (g->periodic && !g->free_surface) k = wrap(k, g->nz);
+  else if (k >= g->nz) k = g->nz - 1;
   double s = atf(g, vs, i, j, k);
   return atf(g, rho, i, j, k) * s * s;
 }
@@ -444,7 +449,6 @@ int or_el_run(const or_grid* g, const float* vp, const float* vs, const float* r
   init_coef();
   int rc = check_lists(g, inj, rec);
   if (rc) return rc;
-  if (g->free_surface && g->periodic) return -1;
   const double h = g->h, dt = g->dt;
   size_t n = NPTS(g);
   cpml_set c;

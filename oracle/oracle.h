@@ -32,7 +32,8 @@ typedef struct {
   int32_t free_surface; /* elastic: traction-free top (O16); top face then has no layer */
   double pml_R;         /* target reflection coefficient (O6/O7) */
   double pml_f;         /* C-PML alpha reference frequency (Hz) (O7) */
-  int32_t periodic;     /* TEST MODE (O4): periodic wrap instead of zero ghosts; needs nb = 0 */
+  int32_t periodic;     /* TEST MODE (O4): periodic wrap instead of zero ghosts; needs nb = 0;
+                           with free_surface the wrap is lateral (x, y) only */
 } or_grid;
 
 /* O1: 8th-order coefficient tables: c[0..4] centred 2nd derivative,

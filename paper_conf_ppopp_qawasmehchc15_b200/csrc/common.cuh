@@ -135,3 +135,43 @@ __device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, u
 }
 
 }  // namespace seis
+
+// ------------------------------------------------------------ 4-wide vectors
+// The stencil kernels are issue-bound at one point per thread (~140 instructions
+// per point); each thread therefore owns 4 consecutive x points (one float4) and
+// a block tile is TXV = 64 points wide (16 threads) x BY rows.
+namespace seis {
+
+constexpr int TXV = 64;  // tile width in x (points)
+constexpr int NTX = 16;  // threads in x per block
+
+struct F4 {
+  float v[4];
+};
+__device__ __forceinline__ F4 lds4(const float* p) {
+  const float4 t = *reinterpret_cast<const float4*>(p);
+  return F4{{t.x, t.y, t.z, t.w}};
+}
+__device__ __forceinline__ F4 ldg4(const float* p) {
+  const float4 t = __ldg(reinterpret_cast<const float4*>(p));
+  return F4{{t.x, t.y, t.z, t.w}};
+}
+__device__ __forceinline__ F4 ld4(const float* p) {
+  const float4 t = *reinterpret_cast<const float4*>(p);
+  return F4{{t.x, t.y, t.z, t.w}};
+}
+__device__ __forceinline__ void st4(float* p, const F4& a) {
+  *reinterpret_cast<float4*>(p) = make_float4(a.v[0], a.v[1], a.v[2], a.v[3]);
+}
+// store the components of a group of 4 x-points that lie inside [0, nx)
+__device__ __forceinline__ void st4_masked(float* p, const F4& a, int x0, int nx, bool aligned) {
+  if (aligned && x0 + 3 < nx) {
+    st4(p, a);
+  } else {
+#pragma unroll
+    for (int e = 0; e < 4; ++e)
+      if (x0 + e < nx) p[e] = a.v[e];
+  }
+}
+
+}  // namespace seis

@@ -6,9 +6,14 @@
 // with h D+ f_{i+1/2} = sum_m d_m (f_{i+m} - f_{i-m+1}), h D- g_i = sum_m d_m (g_{i+m-1} - g_{i-m})
 // (psi is stored multiplied by h, so both updates work on the unscaled differences).
 //
-// One fused z-marching kernel per time step (ac_step_kernel, below).
-// Fused epilogues: the source, the snapshot store and the
-// imaging condition on the input p (O15).
+// Two z-marching kernels per step, 64 x BY tiles, 4 x-points per
+// thread.  V: the p tile (x/y halo 4), the q_x, q_y, q_z tiles, the rho tile
+// (+1 in x and y), rho at plane k+1 and p at plane k+4 (the feed of p's float4
+// z-queue) arrive by TMA in an NS-deep mbarrier ring; the face buoyancy
+// 2/(rho_i + rho_{i+1}) is evaluated on the fly (O8), so V moves 32 B per point.  P: the q_x (x halo) and q_y (y halo) tiles,
+// p and dt K/h by TMA, q_z from a register queue.  Fused epilogues: P adds the
+// source and stores the snapshot; V applies the imaging
+// condition to its input p (O15).
 #pragma once
 #include "common.cuh"
 
@@ -21,284 +26,354 @@ struct CpmlAxis {
   const float* __restrict__ bh;
 };
 
-// ---------------------------------------------------------------------------
-// Fused single-sweep acoustic step: one z-march computes
-// q^{n+1/2} = V(p^n, q^{n-1/2}) and p^{n+1} = P(p^n, q^{n+1/2}) in the same pass.
-// The x/y halos of q^{n+1/2} that P needs (4 points per side, x for q_x, y for
-// q_y) are recomputed from the p^n tile (halo 8) instead of being read back, and
-// q_z^{n+1/2} comes out of the z-march 3 planes ahead of the P update (register
-// queue).  State is double-buffered (A = step input, B = output) so recomputed
-// halo values always see the step's inputs; C-PML psi_p (read at recomputed
-// points) is double-buffered too, psi_q is only touched by its owner (in place).
-// Per point HBM traffic: read p^n, q^{n-1/2} x3, rho, dt K/h; write p^{n+1},
-// q^{n+1/2} x3 = 40 B (vs 56 B for the two-kernel V + P form with rho).
-// Buoyancy dt b/h = (dt/h) 2/(rho_i + rho_{i+1}) is evaluated on the fly (O8).
-// Bitwise identical to itself under any tiling / z-chunking / slab split: a
-// recomputed halo value is the same expression on the same inputs as the owner's.
-struct AcFArgs {
-  CUtensorMap mp;                  // p^n tile, box (32+16) x (BY+16): x from i0-8, y from j0-8
-  CUtensorMap mr;                  // rho tile, same box
-  CUtensorMap mqx;                 // q_x^{n-1/2}, box (32+8) x BY: x from i0-4
-  CUtensorMap mqy;                 // q_y^{n-1/2}, box 32 x (BY+8): y from j0-4
-  CUtensorMap mk;                  // dt K / h, box 32 x BY
-  const float* __restrict__ pA;    // p^n (padded)
-  const float* __restrict__ qzA;   // q_z^{n-1/2}
-  const float* __restrict__ rho;   // density (padded, z ghosts filled from neighbours)
-  float* __restrict__ pB;
-  float* __restrict__ qxB;
-  float* __restrict__ qyB;
-  float* __restrict__ qzB;
-  float dth;                       // dt / h
-  int W, zlo;
+constexpr int AC_NS = 4;   // P kernel ring depth
+constexpr int AC_VNS = 3;  // V kernel ring depth (7 tiles per stage)
+
+// psi update of the 4 x-points of a group that lie inside an x layer
+__device__ __forceinline__ void cpml_x4(float* dv, float* __restrict__ ps, const Dims& d, int W, int x0,
+                                        int j, int k, const float* __restrict__ ca,
+                                        const float* __restrict__ cb) {
+#pragma unroll
+  for (int e = 0; e < 4; ++e) {
+    const int x = x0 + e;
+    if (x < d.nx && CpmlIdx::in(x, d.nx, W, true)) {
+      const long long ix = ((long long)k * d.ny + j) * (2 * W) + CpmlIdx::slot(x, d.nx, W);
+      const float v = fmaf(__ldg(cb + x), ps[ix], __ldg(ca + x) * dv[e]);
+      ps[ix] = v;
+      dv[e] += v;
+    }
+  }
+}
+// psi update of a group inside a y layer (row j) or a z layer (global plane gz)
+__device__ __forceinline__ void cpml_y4(float* dv, float* __restrict__ ps, const Dims& d, int W, int x0,
+                                        int j, int k, float ca, float cb) {
+  const long long iy = ((long long)k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0;
+#pragma unroll
+  for (int e = 0; e < 4; ++e)
+    if (x0 + e < d.nx) {
+      const float v = fmaf(cb, ps[iy + e], ca * dv[e]);
+      ps[iy + e] = v;
+      dv[e] += v;
+    }
+}
+__device__ __forceinline__ void cpml_z4(float* dv, float* __restrict__ ps, const Dims& d, int W, int x0,
+                                        int j, int gz, float ca, float cb) {
+  const long long iz = ((long long)CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0;
+#pragma unroll
+  for (int e = 0; e < 4; ++e)
+    if (x0 + e < d.nx) {
+      const float v = fmaf(cb, ps[iz + e], ca * dv[e]);
+      ps[iz + e] = v;
+      dv[e] += v;
+    }
+}
+
+struct AcVArgs {
+  CUtensorMap mp;                 // p tile, box (64+8) x (BY+8) x 1
+  CUtensorMap mqx, mqy, mqz;      // q, box 64 x BY x 1
+  CUtensorMap mr;                 // rho tile, box (64+4) x (BY+1) x 1 (x+1, y+1 neighbours)
+  CUtensorMap mpq;                // p interior (z-queue feed, plane k+4), box 64 x BY x 1
+  CUtensorMap mrz;                // rho interior (z faces, plane k+1), box 64 x BY x 1
+  const float* __restrict__ p;
+  const float* __restrict__ rho;  // density (padded; z ghosts filled from the neighbour slabs)
+  float dth;                      // dt / h
+  float* __restrict__ qx;
+  float* __restrict__ qy;
+  float* __restrict__ qz;
+  int W;                          // C-PML slab width per face (nb + 1), 0 = no layer
+  int zlo;                        // 1 if the top z face has a layer
   CpmlAxis cx, cy, cz;
-  const float* __restrict__ psxA;  // psi_{p,x} [nzl][ny][2W] (input)
-  const float* __restrict__ psyA;  // psi_{p,y} [nzl][2W][nx]
-  const float* __restrict__ pszA;  // psi_{p,z} [2W][ny][nx]
-  float* __restrict__ psxB;
-  float* __restrict__ psyB;
-  float* __restrict__ pszB;
-  float* __restrict__ pqx;         // psi_{q,*}, owner-only (in place)
-  float* __restrict__ pqy;
-  float* __restrict__ pqz;
+  float* __restrict__ psx;        // psi_{p,x} [nzl][ny][2W]
+  float* __restrict__ psy;        // psi_{p,y} [nzl][2W][nx]
+  float* __restrict__ psz;        // psi_{p,z} [2W][ny][nx] (global z slots)
   Dims d;
   int zc;
-  long long src_o;
-  float src_amp;
-  float* __restrict__ snap;
-  const float* __restrict__ imgS;
+  const float* __restrict__ imgS; // imaging: img += S * p (input level), or nullptr
   float* __restrict__ img;
 };
 
-constexpr int ACF_NS = 3;
-
 template <int BY>
-struct AcFStage {
-  static constexpr int PW = TXW + 16, PH = BY + 16, QXW = TXW + 8, QYH = BY + 8, T = TXW * BY;
-  static constexpr int P = 0, R = PW * PH, QX = 2 * PW * PH, QY = QX + QXW * BY, K = QY + TXW * QYH,
-                       SIZE = K + T;
-  static constexpr int SCRATCH = QXW * BY + TXW * QYH;  // q_x, q_y at step n+1/2 incl. halos
-  static constexpr size_t smem_bytes() { return ((size_t)ACF_NS * SIZE + SCRATCH) * 4 + 128; }
+struct AcVStage {
+  static constexpr int W = TXV + 8, T = TXV * BY, RW = TXV + 4;
+  static constexpr int P = 0, QX = (BY + 8) * W, QY = QX + T, QZ = QY + T, PQ = QZ + T, RZ = PQ + T,
+                       R = RZ + T, SIZE = R + ((RW * (BY + 1) + 31) / 32) * 32;
+  static constexpr uint32_t BYTES = ((BY + 8) * W + 5 * T + RW * (BY + 1)) * 4;
+  static constexpr size_t smem_bytes() { return (size_t)AC_VNS * SIZE * 4 + 128; }
 };
 
-// buoyancy on a face: (dt/h) * 2 / (rho0 + rho1)
-__device__ __forceinline__ float face_b(float dth, float r0, float r1) { return dth * (2.0f / (r0 + r1)); }
-
-template <int BY, bool SNAP, bool IMG>
-__global__ void __launch_bounds__(TXW * BY) ac_step_kernel(const __grid_constant__ AcFArgs a) {
-  using L = AcFStage<BY>;
-  constexpr int PW = L::PW, QXW = L::QXW;
-  constexpr uint32_t TX_BYTES = L::SIZE * 4;
-  constexpr int NT = TXW * BY;
+template <int BY, bool IMG>
+__global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ AcVArgs a) {
+  using L = AcVStage<BY>;
+  constexpr int W = L::W, RW = L::RW;
+  constexpr uint32_t TX_BYTES = L::BYTES;
   extern __shared__ __align__(128) float sm_raw[];
   float* sm = align128(sm_raw);
-  float* qxn = sm + ACF_NS * L::SIZE;   // [BY][QXW]   q_x^{n+1/2}, x from i0-4
-  float* qyn = qxn + QXW * BY;          // [BY+8][TXW] q_y^{n+1/2}, y from j0-4
-  __shared__ __align__(8) uint64_t bar[ACF_NS];
+  __shared__ __align__(8) uint64_t bar[AC_VNS];
   const Dims& d = a.d;
-  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
-  const int i0 = blockIdx.x * TXW, j0 = blockIdx.y * BY;
-  const int i = i0 + tx, j = j0 + ty;
+  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX + tx;
+  const int i0 = blockIdx.x * TXV, j0 = blockIdx.y * BY;
+  const int x0 = i0 + 4 * tx, j = j0 + ty;
   const int k0 = blockIdx.z * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
   const int np = k1 - k0;
-  const bool own = (i < d.nx) && (j < d.ny);
+  const bool own = (x0 < d.nx) && (j < d.ny);
   const long long PS = d.PS;
-  const long long oc = (long long)(j + G) * d.PX + (i + G);
+  const long long oc = (long long)(j + G) * d.PX + (x0 + G);
+  const float* __restrict__ p = a.p;
   const int Wl = a.W;
-  const float dth = a.dth;
+  const bool lx = Wl > 0 && (x0 < Wl || x0 + 3 >= d.nx - Wl);  // some component may be in the x layer
+  const bool ly = Wl > 0 && CpmlIdx::in(j, d.ny, Wl, true);
   auto issue = [&](int s, int k) {
     float* st = sm + s * L::SIZE;
-    const int z = k + GZ;
+    const int z = k + GZ, x = i0 + G, y = j0 + G;
     mbar_expect_tx(&bar[s], TX_BYTES);
-    tma_load_3d(st + L::P, &a.mp, &bar[s], i0 - 4, j0 - 4, z);
-    tma_load_3d(st + L::R, &a.mr, &bar[s], i0 - 4, j0 - 4, z);
-    tma_load_3d(st + L::QX, &a.mqx, &bar[s], i0, j0 + G, z);
-    tma_load_3d(st + L::QY, &a.mqy, &bar[s], i0 + G, j0, z);
-    tma_load_3d(st + L::K, &a.mk, &bar[s], i0 + G, j0 + G, z);
+    tma_load_3d(st + L::P, &a.mp, &bar[s], i0, j0, z);
+    tma_load_3d(st + L::QX, &a.mqx, &bar[s], x, y, z);
+    tma_load_3d(st + L::QY, &a.mqy, &bar[s], x, y, z);
+    tma_load_3d(st + L::QZ, &a.mqz, &bar[s], x, y, z);
+    tma_load_3d(st + L::R, &a.mr, &bar[s], x, y, z);
+    tma_load_3d(st + L::PQ, &a.mpq, &bar[s], x, y, z + 4);
+    tma_load_3d(st + L::RZ, &a.mrz, &bar[s], x, y, z + 1);
   };
   if (tid == 0) {
-    for (int s = 0; s < ACF_NS; ++s) mbar_init(&bar[s], 1);
+    for (int s = 0; s < AC_VNS; ++s) mbar_init(&bar[s], 1);
     mbar_fence_init();
   }
   __syncthreads();
   if (tid == 0)
-    for (int s = 0; s < ACF_NS && s < np; ++s) issue(s, k0 + s);
-
-  const float* __restrict__ pA = a.pA;
-  const float* __restrict__ qzA = a.qzA;
-  const float* __restrict__ rho = a.rho;
-  // q_z^{n+1/2} at plane kk from p^n(kk-3 .. kk+4) = w[0..7], rho(kk), rho(kk+1), q_z^{n-1/2}(kk)
-  auto qz_new = [&](int kk, const float* w, float r0, float r1, float qold) -> float {
-    const int gz = kk + d.z0;
-    if (!own || gz < 0 || gz >= d.nz) return 0.0f;
-    float dz = SEIS_D1 * (w[4] - w[3]);
-    dz = fmaf(SEIS_D2, w[5] - w[2], dz);
-    dz = fmaf(SEIS_D3, w[6] - w[1], dz);
-    dz = fmaf(SEIS_D4, w[7] - w[0], dz);
-    if (Wl > 0 && CpmlIdx::in(gz, d.nz, Wl, a.zlo)) {
-      const long long iz = ((long long)CpmlIdx::slot(gz, d.nz, Wl) * d.ny + j) * d.nx + i;
-      const float ps = fmaf(__ldg(a.cz.bh + gz), a.pszA[iz], __ldg(a.cz.ah + gz) * dz);
-      if (kk >= k0 && kk < k1) a.pszB[iz] = ps;
-      dz += ps;
-    }
-    const float b = face_b(dth, r0, gz + 1 < d.nz ? r1 : r0);
-    const float v = fmaf(b, dz, qold);
-    if (kk >= k0 && kk < k1) a.qzB[(long long)(kk + GZ) * PS + oc] = v;
-    return v;
-  };
-
-  // warm-up: q_z^{n+1/2} at planes k0-4 .. k0+2 (needs p^n at k0-7 .. k0+6)
-  float pq[8];   // p^n(k .. k+7) at the start of iteration k
-  float qzq[8];  // q_z^{n+1/2}(k-4 .. k+3)
-  float rq0;     // rho(k+3)
-  {
-    float w[14];
+    for (int s = 0; s < AC_VNS && s < np; ++s) issue(s, k0 + s);
+  F4 r[8];  // p at k-3 .. k+4; plane k+4 arrives with stage k (TMA)
 #pragma unroll
-    for (int t = 0; t < 14; ++t) w[t] = __ldg(pA + (long long)(k0 - 7 + t + GZ) * PS + oc);
-    float rr[8];
-#pragma unroll
-    for (int t = 0; t < 8; ++t) rr[t] = __ldg(rho + (long long)(k0 - 4 + t + GZ) * PS + oc);
-#pragma unroll
-    for (int t = 0; t < 7; ++t) {
-      const float qo = __ldg(qzA + (long long)(k0 - 4 + t + GZ) * PS + oc);
-      qzq[t] = qz_new(k0 - 4 + t, w + t, rr[t], rr[t + 1], qo);
-    }
-#pragma unroll
-    for (int t = 0; t < 7; ++t) pq[t] = w[7 + t];
-    rq0 = rr[7];  // rho(k0+3)
-  }
-  pq[7] = __ldg(pA + (long long)(k0 + 7 + GZ) * PS + oc);
-  float rq1 = __ldg(rho + (long long)(k0 + 4 + GZ) * PS + oc);
-  float qzo = __ldg(qzA + (long long)(k0 + 3 + GZ) * PS + oc);
-  const bool lxo = Wl > 0 && CpmlIdx::in(i, d.nx, Wl, true);
-  const bool lyo = Wl > 0 && CpmlIdx::in(j, d.ny, Wl, true);
+  for (int t = 0; t < 7; ++t) r[t] = ldg4(p + (long long)(k0 - 3 + t + GZ) * PS + oc);
+  const float dth = a.dth;
 
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
-    const int s = it % ACF_NS;
+    const int s = it % AC_VNS;
     const long long o = (long long)(k + GZ) * PS + oc;
-    // next plane's streams (one ahead)
-    float p_next = 0.f, r_next = 0.f, qz_next = 0.f;
-    if (it + 1 < np) {
-      p_next = __ldg(pA + o + 8 * PS);
-      r_next = __ldg(rho + o + 5 * PS);
-      qz_next = __ldg(qzA + o + 4 * PS);
-    }
-    mbar_wait(&bar[s], (it / ACF_NS) & 1);
+    mbar_wait(&bar[s], (it / AC_VNS) & 1);
     const float* st = sm + s * L::SIZE;
-    // ---- V: q_x^{n+1/2} on the tile plus its x halo (x from i0-4, QXW wide) ----
-    for (int t = tid; t < QXW * BY; t += NT) {
-      const int r = t / QXW, c = t - r * QXW;
-      const int x = i0 - 4 + c, y = j0 + r;
-      const float* pc = st + L::P + (r + 8) * PW + (c + 4);
-      float dx = SEIS_D1 * (pc[1] - pc[0]);
-      dx = fmaf(SEIS_D2, pc[2] - pc[-1], dx);
-      dx = fmaf(SEIS_D3, pc[3] - pc[-2], dx);
-      dx = fmaf(SEIS_D4, pc[4] - pc[-3], dx);
-      float v = 0.0f;
-      if (x >= 0 && x < d.nx && y < d.ny) {
-        const bool ownpt = c >= 4 && c < 4 + TXW;
-        if (Wl > 0 && CpmlIdx::in(x, d.nx, Wl, true)) {
-          const long long ix = ((long long)k * d.ny + y) * (2 * Wl) + CpmlIdx::slot(x, d.nx, Wl);
-          const float ps = fmaf(__ldg(a.cx.bh + x), a.psxA[ix], __ldg(a.cx.ah + x) * dx);
-          if (ownpt) a.psxB[ix] = ps;
-          dx += ps;
-        }
-        const float* rc = st + L::R + (r + 8) * PW + (c + 4);
-        const float b = face_b(dth, rc[0], x + 1 < d.nx ? rc[1] : rc[0]);
-        v = fmaf(b, dx, st[L::QX + t]);
-        if (ownpt) a.qxB[(long long)(k + GZ) * PS + (long long)(y + G) * d.PX + (x + G)] = v;
+    r[7] = lds4(st + L::PQ + ty * TXV + 4 * tx);
+    const F4 rz1 = lds4(st + L::RZ + ty * TXV + 4 * tx);  // rho(k+1)
+    const float* c = st + L::P + (ty + 4) * W + 4 * tx + 4;  // p(x0, j, k)
+    float xv[12];                                             // p(x0-4 .. x0+7, j)
+    {
+      const F4 a0 = lds4(c - 4), a1 = lds4(c), a2 = lds4(c + 4);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        xv[e] = a0.v[e];
+        xv[4 + e] = a1.v[e];
+        xv[8 + e] = a2.v[e];
       }
-      qxn[t] = v;
     }
-    // ---- V: q_y^{n+1/2} on the tile plus its y halo (y from j0-4) ----
-    for (int t = tid; t < TXW * (BY + 8); t += NT) {
-      const int r = t / TXW, c = t - r * TXW;
-      const int x = i0 + c, y = j0 - 4 + r;
-      const float* pc = st + L::P + (r + 4) * PW + (c + 8);
-      float dy = SEIS_D1 * (pc[PW] - pc[0]);
-      dy = fmaf(SEIS_D2, pc[2 * PW] - pc[-PW], dy);
-      dy = fmaf(SEIS_D3, pc[3 * PW] - pc[-2 * PW], dy);
-      dy = fmaf(SEIS_D4, pc[4 * PW] - pc[-3 * PW], dy);
-      float v = 0.0f;
-      if (y >= 0 && y < d.ny && x < d.nx) {
-        const bool ownpt = r >= 4 && r < 4 + BY;
-        if (Wl > 0 && CpmlIdx::in(y, d.ny, Wl, true)) {
-          const long long iy = ((long long)k * (2 * Wl) + CpmlIdx::slot(y, d.ny, Wl)) * d.nx + x;
-          const float ps = fmaf(__ldg(a.cy.bh + y), a.psyA[iy], __ldg(a.cy.ah + y) * dy);
-          if (ownpt) a.psyB[iy] = ps;
-          dy += ps;
-        }
-        const float* rc = st + L::R + (r + 4) * PW + (c + 8);
-        const float b = face_b(dth, rc[0], y + 1 < d.ny ? rc[PW] : rc[0]);
-        v = fmaf(b, dy, st[L::QY + t]);
-        if (ownpt) a.qyB[(long long)(k + GZ) * PS + (long long)(y + G) * d.PX + (x + G)] = v;
-      }
-      qyn[t] = v;
+    F4 yr[8];  // p rows j-3 .. j+4
+#pragma unroll
+    for (int m = 0; m < 8; ++m) yr[m] = (m == 3) ? F4{{xv[4], xv[5], xv[6], xv[7]}} : lds4(c + (m - 3) * W);
+    float dx[4], dy[4], dz[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      float t = SEIS_D1 * (xv[5 + e] - xv[4 + e]);
+      t = fmaf(SEIS_D2, xv[6 + e] - xv[3 + e], t);
+      t = fmaf(SEIS_D3, xv[7 + e] - xv[2 + e], t);
+      dx[e] = fmaf(SEIS_D4, xv[8 + e] - xv[1 + e], t);
+      t = SEIS_D1 * (yr[4].v[e] - yr[3].v[e]);
+      t = fmaf(SEIS_D2, yr[5].v[e] - yr[2].v[e], t);
+      t = fmaf(SEIS_D3, yr[6].v[e] - yr[1].v[e], t);
+      dy[e] = fmaf(SEIS_D4, yr[7].v[e] - yr[0].v[e], t);
+      t = SEIS_D1 * (r[4].v[e] - r[3].v[e]);
+      t = fmaf(SEIS_D2, r[5].v[e] - r[2].v[e], t);
+      t = fmaf(SEIS_D3, r[6].v[e] - r[1].v[e], t);
+      dz[e] = fmaf(SEIS_D4, r[7].v[e] - r[0].v[e], t);
     }
-    // ---- V: q_z^{n+1/2} at plane k+3 (z-march, register queue) ----
-    qzq[7] = qz_new(k + 3, pq, rq0, rq1, qzo);
-    __syncthreads();
-    // ---- P: p^{n+1} at plane k ----
     if (own) {
-      const float* cx = qxn + ty * QXW + tx + 4;
-      const float* cy = qyn + (ty + 4) * TXW + tx;
-      float dx = SEIS_D1 * (cx[0] - cx[-1]);
-      dx = fmaf(SEIS_D2, cx[1] - cx[-2], dx);
-      dx = fmaf(SEIS_D3, cx[2] - cx[-3], dx);
-      dx = fmaf(SEIS_D4, cx[3] - cx[-4], dx);
-      float dy = SEIS_D1 * (cy[0] - cy[-TXW]);
-      dy = fmaf(SEIS_D2, cy[TXW] - cy[-2 * TXW], dy);
-      dy = fmaf(SEIS_D3, cy[2 * TXW] - cy[-3 * TXW], dy);
-      dy = fmaf(SEIS_D4, cy[3 * TXW] - cy[-4 * TXW], dy);
-      float dz = SEIS_D1 * (qzq[4] - qzq[3]);
-      dz = fmaf(SEIS_D2, qzq[5] - qzq[2], dz);
-      dz = fmaf(SEIS_D3, qzq[6] - qzq[1], dz);
-      dz = fmaf(SEIS_D4, qzq[7] - qzq[0], dz);
       if (Wl > 0) {
-        if (lxo) {
-          const long long ix = ((long long)k * d.ny + j) * (2 * Wl) + CpmlIdx::slot(i, d.nx, Wl);
-          const float ps = fmaf(__ldg(a.cx.b + i), a.pqx[ix], __ldg(a.cx.a + i) * dx);
-          a.pqx[ix] = ps;
-          dx += ps;
-        }
-        if (lyo) {
-          const long long iy = ((long long)k * (2 * Wl) + CpmlIdx::slot(j, d.ny, Wl)) * d.nx + i;
-          const float ps = fmaf(__ldg(a.cy.b + j), a.pqy[iy], __ldg(a.cy.a + j) * dy);
-          a.pqy[iy] = ps;
-          dy += ps;
-        }
+        if (lx) cpml_x4(dx, a.psx, d, Wl, x0, j, k, a.cx.ah, a.cx.bh);
+        if (ly) cpml_y4(dy, a.psy, d, Wl, x0, j, k, __ldg(a.cy.ah + j), __ldg(a.cy.bh + j));
         const int gz = k + d.z0;
-        if (CpmlIdx::in(gz, d.nz, Wl, a.zlo)) {
-          const long long iz = ((long long)CpmlIdx::slot(gz, d.nz, Wl) * d.ny + j) * d.nx + i;
-          const float ps = fmaf(__ldg(a.cz.b + gz), a.pqz[iz], __ldg(a.cz.a + gz) * dz);
-          a.pqz[iz] = ps;
-          dz += ps;
-        }
+        if (CpmlIdx::in(gz, d.nz, Wl, a.zlo))
+          cpml_z4(dz, a.psz, d, Wl, x0, j, gz, __ldg(a.cz.ah + gz), __ldg(a.cz.bh + gz));
       }
-      float out = fmaf(st[L::K + tid], (dx + dy) + dz, pq[0]);
-      if (o == a.src_o) out += a.src_amp;
-      a.pB[o] = out;
-      if (SNAP || IMG) {
-        const long long cix = ((long long)k * d.ny + j) * d.nx + i;
-        if (SNAP) a.snap[cix] = out;
-        if (IMG) a.img[cix] = fmaf(__ldg(a.imgS + cix), pq[0], a.img[cix]);
+      const int pt = ty * TXV + 4 * tx;
+      const F4 qxo = lds4(st + L::QX + pt), qyo = lds4(st + L::QY + pt), qzo = lds4(st + L::QZ + pt);
+      // face buoyancy dt b/h = (dt/h) 2 / (rho_i + rho_{i+1}), last face clamps (O8)
+      const float* rc = st + L::R + ty * RW + 4 * tx;
+      const F4 r0 = lds4(rc), rxn = lds4(rc + 4), ryn = lds4(rc + RW);
+      const float rx5 = rxn.v[0];
+      const bool zlast = k + d.z0 + 1 >= d.nz;
+      F4 ox, oy, oz;
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const float rxp = (x0 + e + 1 < d.nx) ? (e < 3 ? r0.v[e + 1] : rx5) : r0.v[e];
+        const float ryp = (j + 1 < d.ny) ? ryn.v[e] : r0.v[e];
+        const float rzp = zlast ? r0.v[e] : rz1.v[e];
+        const float bx = dth * (2.0f * __frcp_rn(r0.v[e] + rxp));
+        const float by = dth * (2.0f * __frcp_rn(r0.v[e] + ryp));
+        const float bz = dth * (2.0f * __frcp_rn(r0.v[e] + rzp));
+        ox.v[e] = fmaf(bx, dx[e], qxo.v[e]);
+        oy.v[e] = fmaf(by, dy[e], qyo.v[e]);
+        oz.v[e] = fmaf(bz, dz[e], qzo.v[e]);
+      }
+      st4_masked(a.qx + o, ox, x0, d.nx, true);
+      st4_masked(a.qy + o, oy, x0, d.nx, true);
+      st4_masked(a.qz + o, oz, x0, d.nx, true);
+      if (IMG) {
+        const long long cix = ((long long)k * d.ny + j) * d.nx + x0;
+        F4 im;
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          im.v[e] = (x0 + e < d.nx) ? fmaf(__ldg(a.imgS + cix + e), r[3].v[e], a.img[cix + e]) : 0.f;
+        st4_masked(a.img + cix, im, x0, d.nx, false);
       }
     }
-    __syncthreads();  // stage s and the q scratch are free
-    if (tid == 0 && it + ACF_NS < np) {
+    __syncthreads();
+    if (tid == 0 && it + AC_VNS < np) {
       fence_proxy_async();
-      issue(s, k + ACF_NS);
+      issue(s, k + AC_VNS);
     }
 #pragma unroll
-    for (int t = 0; t < 7; ++t) {
-      pq[t] = pq[t + 1];
-      qzq[t] = qzq[t + 1];
+    for (int t = 0; t < 7; ++t) r[t] = r[t + 1];
+  }
+}
+
+struct AcPArgs {
+  CUtensorMap mqx;                // q_x, box (64+8) x BY x 1
+  CUtensorMap mqy;                // q_y, box 64 x (BY+8) x 1
+  CUtensorMap mpp;                // p, box 64 x BY x 1
+  CUtensorMap mk;                 // dt K / h, box 64 x BY x 1
+  CUtensorMap mqq;                // q_z interior (z-queue feed, plane k+3), box 64 x BY x 1
+  float* __restrict__ p;
+  const float* __restrict__ qz;
+  int W;
+  int zlo;
+  CpmlAxis cx, cy, cz;
+  float* __restrict__ pqx;        // psi_{q,x} [nzl][ny][2W]
+  float* __restrict__ pqy;        // psi_{q,y} [nzl][2W][nx]
+  float* __restrict__ pqz;        // psi_{q,z} [2W][ny][nx]
+  Dims d;
+  int zc;
+  long long src_o;                // padded index of the source in this slab, -1 = none
+  float src_amp;                  // dt K_s / h^3 * s[n]
+  float* __restrict__ snap;       // compact snapshot target, or nullptr
+};
+
+template <int BY>
+struct AcPStage {
+  static constexpr int WX = TXV + 8, T = TXV * BY;
+  static constexpr int QX = 0, QY = BY * WX, P = QY + (BY + 8) * TXV, K = P + T, QQ = K + T, SIZE = QQ + T;
+  static constexpr size_t smem_bytes() { return (size_t)AC_NS * SIZE * 4 + 128; }
+};
+
+template <int BY, bool SNAP>
+__global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ AcPArgs a) {
+  using L = AcPStage<BY>;
+  constexpr int WX = L::WX;
+  constexpr uint32_t TX_BYTES = L::SIZE * 4;
+  extern __shared__ __align__(128) float sm_raw[];
+  float* sm = align128(sm_raw);
+  __shared__ __align__(8) uint64_t bar[AC_NS];
+  const Dims& d = a.d;
+  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX + tx;
+  const int i0 = blockIdx.x * TXV, j0 = blockIdx.y * BY;
+  const int x0 = i0 + 4 * tx, j = j0 + ty;
+  const int k0 = blockIdx.z * a.zc;
+  const int k1 = min(k0 + a.zc, d.nzl);
+  const int np = k1 - k0;
+  const bool own = (x0 < d.nx) && (j < d.ny);
+  const long long PS = d.PS;
+  const long long oc = (long long)(j + G) * d.PX + (x0 + G);
+  const float* __restrict__ qz = a.qz;
+  const int Wl = a.W;
+  const bool lx = Wl > 0 && (x0 < Wl || x0 + 3 >= d.nx - Wl);
+  const bool ly = Wl > 0 && CpmlIdx::in(j, d.ny, Wl, true);
+  auto issue = [&](int s, int k) {
+    float* st = sm + s * L::SIZE;
+    const int z = k + GZ;
+    mbar_expect_tx(&bar[s], TX_BYTES);
+    tma_load_3d(st + L::QX, &a.mqx, &bar[s], i0, j0 + G, z);
+    tma_load_3d(st + L::QY, &a.mqy, &bar[s], i0 + G, j0, z);
+    tma_load_3d(st + L::P, &a.mpp, &bar[s], i0 + G, j0 + G, z);
+    tma_load_3d(st + L::K, &a.mk, &bar[s], i0 + G, j0 + G, z);
+    tma_load_3d(st + L::QQ, &a.mqq, &bar[s], i0 + G, j0 + G, z + 3);
+  };
+  if (tid == 0) {
+    for (int s = 0; s < AC_NS; ++s) mbar_init(&bar[s], 1);
+    mbar_fence_init();
+  }
+  __syncthreads();
+  if (tid == 0)
+    for (int s = 0; s < AC_NS && s < np; ++s) issue(s, k0 + s);
+  F4 q[8];  // q_z at k-4 .. k+3; plane k+3 arrives with stage k (TMA)
+#pragma unroll
+  for (int t = 0; t < 7; ++t) q[t] = ldg4(qz + (long long)(k0 - 4 + t + GZ) * PS + oc);
+  const long long srel0 = a.src_o - oc;
+
+  for (int it = 0; it < np; ++it) {
+    const int k = k0 + it;
+    const int s = it % AC_NS;
+    const long long o = (long long)(k + GZ) * PS + oc;
+    mbar_wait(&bar[s], (it / AC_NS) & 1);
+    const float* st = sm + s * L::SIZE;
+    q[7] = lds4(st + L::QQ + ty * TXV + 4 * tx);
+    const float* cx = st + L::QX + ty * WX + 4 * tx + 4;      // q_x(x0, j)
+    const float* cy = st + L::QY + (ty + 4) * TXV + 4 * tx;   // q_y(x0, j)
+    float xv[12];                                             // q_x(x0-4 .. x0+7)
+    {
+      const F4 a0 = lds4(cx - 4), a1 = lds4(cx), a2 = lds4(cx + 4);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        xv[e] = a0.v[e];
+        xv[4 + e] = a1.v[e];
+        xv[8 + e] = a2.v[e];
+      }
     }
-    pq[7] = p_next;
-    rq0 = rq1;
-    rq1 = r_next;
-    qzo = qz_next;
+    F4 yr[8];  // q_y rows j-4 .. j+3
+#pragma unroll
+    for (int m = 0; m < 8; ++m) yr[m] = lds4(cy + (m - 4) * TXV);
+    float dx[4], dy[4], dz[4];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      float t = SEIS_D1 * (xv[4 + e] - xv[3 + e]);
+      t = fmaf(SEIS_D2, xv[5 + e] - xv[2 + e], t);
+      t = fmaf(SEIS_D3, xv[6 + e] - xv[1 + e], t);
+      dx[e] = fmaf(SEIS_D4, xv[7 + e] - xv[0 + e], t);
+      t = SEIS_D1 * (yr[4].v[e] - yr[3].v[e]);
+      t = fmaf(SEIS_D2, yr[5].v[e] - yr[2].v[e], t);
+      t = fmaf(SEIS_D3, yr[6].v[e] - yr[1].v[e], t);
+      dy[e] = fmaf(SEIS_D4, yr[7].v[e] - yr[0].v[e], t);
+      t = SEIS_D1 * (q[4].v[e] - q[3].v[e]);
+      t = fmaf(SEIS_D2, q[5].v[e] - q[2].v[e], t);
+      t = fmaf(SEIS_D3, q[6].v[e] - q[1].v[e], t);
+      dz[e] = fmaf(SEIS_D4, q[7].v[e] - q[0].v[e], t);
+    }
+    if (own) {
+      if (Wl > 0) {
+        if (lx) cpml_x4(dx, a.pqx, d, Wl, x0, j, k, a.cx.a, a.cx.b);
+        if (ly) cpml_y4(dy, a.pqy, d, Wl, x0, j, k, __ldg(a.cy.a + j), __ldg(a.cy.b + j));
+        const int gz = k + d.z0;
+        if (CpmlIdx::in(gz, d.nz, Wl, a.zlo))
+          cpml_z4(dz, a.pqz, d, Wl, x0, j, gz, __ldg(a.cz.a + gz), __ldg(a.cz.b + gz));
+      }
+      const int pt = ty * TXV + 4 * tx;
+      const F4 pv = lds4(st + L::P + pt), kv = lds4(st + L::K + pt);
+      F4 out;
+#pragma unroll
+      for (int e = 0; e < 4; ++e) out.v[e] = fmaf(kv.v[e], (dx[e] + dy[e]) + dz[e], pv.v[e]);
+      const long long rel = srel0 - (long long)(k + GZ) * PS;
+      if (rel >= 0 && rel < 4) {
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          if (rel == e) out.v[e] += a.src_amp;
+      }
+      st4_masked(a.p + o, out, x0, d.nx, true);
+      if (SNAP) st4_masked(a.snap + ((long long)k * d.ny + j) * d.nx + x0, out, x0, d.nx, (d.nx & 3) == 0);
+    }
+    __syncthreads();
+    if (tid == 0 && it + AC_NS < np) {
+      fence_proxy_async();
+      issue(s, k + AC_NS);
+    }
+#pragma unroll
+    for (int t = 0; t < 7; ++t) q[t] = q[t + 1];
   }
 }
 

@@ -4,27 +4,30 @@
 //   m = v^2 dt^2 / h^2 (per point, precomputed),  eta dt = edx[i] + edy[j] + edz[k]
 //   Lambda u = 3 c0 u + sum_m c_m sum_axes (u_{+m} + u_{-m})         (O1, O3, O6)
 //
-// One thread per (x, y) column marching down a z-chunk (2.5D blocking).  Every
-// operand of plane k arrives by TMA in one stage of an NS-deep mbarrier ring
-// (the u^n tile with its x/y halo of 4, and the u^{n-1} and m tiles); the z
-// neighbours come from a 9-deep register queue fed by a coalesced stream two
-// planes ahead.  u^{n+1} overwrites u^{n-1} in place ("logically swapping
-// t_n and t_{n+1} arrays").  HBM traffic per point: read u^n, u^{n-1}, m; write
-// u^{n+1} = 16 B (+4 B snapshot, +12 B imaging).  Fused epilogues: source
-// injection, snapshot store (O14), imaging I += S_j * u^n on
-// the input level (O15).
+// 2.5D z-march: a block owns a 64 x BY (x, y) tile and walks a z-chunk; each
+// thread owns 4 consecutive x points (one float4).  Every operand of plane k
+// arrives by TMA in one stage of an NS-deep mbarrier ring: the u^n tile with
+// its x/y halo of 4 (x-neighbours from three 16-byte shared loads per row,
+// y-neighbours from eight), the u^{n-1} and m tiles, and the interior tile of
+// u^n at plane k+4 that feeds the 9-deep float4 register queue of z neighbours
+// (no global load in the z-march except the queue warm-up).  u^{n+1} overwrites u^{n-1} in place ("logically swapping t_n and
+// t_{n+1} arrays").  HBM traffic per point: read u^n, u^{n-1}, m; write u^{n+1}
+// = 16 B (+4 B snapshot, +12 B imaging).  Fused epilogues: source injection
+// (P:191), snapshot store (O14), imaging I += S_j * u^n on the input
+// level (O15).
 #pragma once
 #include "common.cuh"
 
 namespace seis {
 
 struct IsoArgs {
-  CUtensorMap mun;               // u^n tile, box (32+8) x (BY+8) x 1
-  CUtensorMap mup;               // u^{n-1}, box 32 x BY x 1
-  CUtensorMap mm;                // m, box 32 x BY x 1
+  CUtensorMap mun;               // u^n tile, box (64+8) x (BY+8) x 1
+  CUtensorMap mup;               // u^{n-1}, box 64 x BY x 1
+  CUtensorMap mm;                // m, box 64 x BY x 1
+  CUtensorMap muq;               // u^n interior tile (z-queue feed, plane k+4), box 64 x BY x 1
   const float* __restrict__ un;  // u^n (padded)
   float* __restrict__ up;        // out: u^{n+1} (in place of u^{n-1})
-  const float* __restrict__ edx; // eta*dt per axis (global index), nullptr = no layer
+  const float* __restrict__ edx; // eta*dt per axis (global index, padded to PX), nullptr = no layer
   const float* __restrict__ edy;
   const float* __restrict__ edz;
   Dims d;
@@ -36,17 +39,17 @@ struct IsoArgs {
   float* __restrict__ img;       // compact image (+=), or nullptr
 };
 
-constexpr int ISO_NS = 4;
+constexpr int ISO_NS = 3;
 
 template <int BY>
 struct IsoStage {
-  static constexpr int W = TXW + 8;
-  static constexpr int U = 0, UP = (BY + 8) * W, M = UP + TXW * BY, SIZE = M + TXW * BY;
+  static constexpr int W = TXV + 8;
+  static constexpr int U = 0, UP = (BY + 8) * W, M = UP + TXV * BY, UQ = M + TXV * BY, SIZE = UQ + TXV * BY;
   static constexpr size_t smem_bytes() { return (size_t)ISO_NS * SIZE * 4 + 128; }
 };
 
 template <int BY, bool SNAP, bool IMG>
-__global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const __grid_constant__ IsoArgs a) {
+__global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constant__ IsoArgs a) {
   using L = IsoStage<BY>;
   constexpr int W = L::W;
   constexpr uint32_t TX_BYTES = L::SIZE * 4;
@@ -54,15 +57,15 @@ __global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const __grid_constan
   float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[ISO_NS];
   const Dims& d = a.d;
-  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
-  const int i0 = blockIdx.x * TXW, j0 = blockIdx.y * BY;
-  const int i = i0 + tx, j = j0 + ty;
+  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX + tx;
+  const int i0 = blockIdx.x * TXV, j0 = blockIdx.y * BY;
+  const int x0 = i0 + 4 * tx, j = j0 + ty;
   const int k0 = blockIdx.z * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
   const int np = k1 - k0;
-  const bool own = (i < d.nx) && (j < d.ny);
+  const bool own = (x0 < d.nx) && (j < d.ny);
   const long long PS = d.PS;
-  const long long oc = (long long)(j + G) * d.PX + (i + G);
+  const long long oc = (long long)(j + G) * d.PX + (x0 + G);
   const float* __restrict__ un = a.un;
   auto issue = [&](int s, int k) {
     float* st = sm + s * L::SIZE;
@@ -70,6 +73,7 @@ __global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const __grid_constan
     tma_load_3d(st + L::U, &a.mun, &bar[s], i0, j0, k + GZ);
     tma_load_3d(st + L::UP, &a.mup, &bar[s], i0 + G, j0 + G, k + GZ);
     tma_load_3d(st + L::M, &a.mm, &bar[s], i0 + G, j0 + G, k + GZ);
+    tma_load_3d(st + L::UQ, &a.muq, &bar[s], i0 + G, j0 + G, k + 4 + GZ);
   };
   if (tid == 0) {
     for (int s = 0; s < ISO_NS; ++s) mbar_init(&bar[s], 1);
@@ -79,50 +83,84 @@ __global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const __grid_constan
   if (tid == 0)
     for (int s = 0; s < ISO_NS && s < np; ++s) issue(s, k0 + s);
 
-  // z-queue u^n(k-4 .. k+4), fed two planes ahead
-  float q0, q1, q2, q3, q4, q5, q6, q7, q8;
-  q0 = __ldg(un + (long long)(k0 - 4 + GZ) * PS + oc);
-  q1 = __ldg(un + (long long)(k0 - 3 + GZ) * PS + oc);
-  q2 = __ldg(un + (long long)(k0 - 2 + GZ) * PS + oc);
-  q3 = __ldg(un + (long long)(k0 - 1 + GZ) * PS + oc);
-  q4 = __ldg(un + (long long)(k0 + GZ) * PS + oc);
-  q5 = __ldg(un + (long long)(k0 + 1 + GZ) * PS + oc);
-  q6 = __ldg(un + (long long)(k0 + 2 + GZ) * PS + oc);
-  q7 = __ldg(un + (long long)(k0 + 3 + GZ) * PS + oc);
-  float na = __ldg(un + (long long)(k0 + 4 + GZ) * PS + oc);
-  float nb = np > 1 ? __ldg(un + (long long)(k0 + 5 + GZ) * PS + oc) : 0.f;
-  const float exy = (a.edx && own) ? a.edx[i] + a.edy[j] : 0.0f;
+  // z-queue u^n(k-4 .. k+4); plane k+4 arrives with stage k (TMA)
+  F4 q[9];
+#pragma unroll
+  for (int t = 0; t < 8; ++t) q[t] = ldg4(un + (long long)(k0 - 4 + t + GZ) * PS + oc);
+  F4 exy{{0.f, 0.f, 0.f, 0.f}};
+  if (a.edx && own) {
+    const F4 ex = ldg4(a.edx + x0);
+    const float ey = a.edy[j];
+#pragma unroll
+    for (int e = 0; e < 4; ++e) exy.v[e] = ex.v[e] + ey;
+  }
+  const long long srel0 = a.src_o - oc;  // source offset relative to this column
 
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % ISO_NS;
     const long long o = (long long)(k + GZ) * PS + oc;
-    q8 = na;
-    na = nb;
-    if (it + 2 < np) nb = __ldg(un + o + 6 * PS);
     mbar_wait(&bar[s], (it / ISO_NS) & 1);
     const float* st = sm + s * L::SIZE;
-    const float* c = st + L::U + (ty + 4) * W + tx + 4;
-    const float upv = st[L::UP + tid], mv = st[L::M + tid];
-    float lap = (3.0f * SEIS_C0) * q4;
-    lap = fmaf(SEIS_C1, (c[-1] + c[1]) + (c[-W] + c[W]) + (q3 + q5), lap);
-    lap = fmaf(SEIS_C2, (c[-2] + c[2]) + (c[-2 * W] + c[2 * W]) + (q2 + q6), lap);
-    lap = fmaf(SEIS_C3, (c[-3] + c[3]) + (c[-3 * W] + c[3 * W]) + (q1 + q7), lap);
-    lap = fmaf(SEIS_C4, (c[-4] + c[4]) + (c[-4 * W] + c[4 * W]) + (q0 + q8), lap);
-    if (own) {
-      const float e = a.edx ? exy + a.edz[k + d.z0] : 0.0f;
-      float out;
-      if (e != 0.0f) {
-        out = (2.0f * q4 - (1.0f - e) * upv + mv * lap) / (1.0f + e);
-      } else {
-        out = fmaf(mv, lap, 2.0f * q4 - upv);
+    q[8] = lds4(st + L::UQ + ty * TXV + 4 * tx);
+    const float* c = st + L::U + (ty + 4) * W + 4 * tx + 4;  // u^n(x0, j, k)
+    float xv[12];                                             // u^n(x0-4 .. x0+7, j)
+    {
+      const F4 a0 = lds4(c - 4), a1 = lds4(c), a2 = lds4(c + 4);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        xv[e] = a0.v[e];
+        xv[4 + e] = a1.v[e];
+        xv[8 + e] = a2.v[e];
       }
-      if (o == a.src_o) out += a.src_amp;
-      a.up[o] = out;
+    }
+    F4 ys[4];  // sum over the y pair (u_{j+m} + u_{j-m}), m = 1..4
+#pragma unroll
+    for (int m = 1; m <= 4; ++m) {
+      const F4 yp = lds4(c + m * W), ym = lds4(c - m * W);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) ys[m - 1].v[e] = yp.v[e] + ym.v[e];
+    }
+    const F4 upv = lds4(st + L::UP + ty * TXV + 4 * tx);
+    const F4 mv = lds4(st + L::M + ty * TXV + 4 * tx);
+    const float ez = a.edx ? a.edz[k + d.z0] : 0.0f;
+    F4 out;
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const float u = xv[4 + e];
+      float lap = (3.0f * SEIS_C0) * u;
+      lap = fmaf(SEIS_C1, (xv[3 + e] + xv[5 + e]) + ys[0].v[e] + (q[3].v[e] + q[5].v[e]), lap);
+      lap = fmaf(SEIS_C2, (xv[2 + e] + xv[6 + e]) + ys[1].v[e] + (q[2].v[e] + q[6].v[e]), lap);
+      lap = fmaf(SEIS_C3, (xv[1 + e] + xv[7 + e]) + ys[2].v[e] + (q[1].v[e] + q[7].v[e]), lap);
+      lap = fmaf(SEIS_C4, (xv[0 + e] + xv[8 + e]) + ys[3].v[e] + (q[0].v[e] + q[8].v[e]), lap);
+      const float eta = exy.v[e] + ez;
+      float r;
+      if (eta != 0.0f) {
+        r = (2.0f * u - (1.0f - eta) * upv.v[e] + mv.v[e] * lap) / (1.0f + eta);
+      } else {
+        r = fmaf(mv.v[e], lap, 2.0f * u - upv.v[e]);
+      }
+      out.v[e] = r;
+    }
+    if (own) {
+      const long long rel = srel0 - (long long)(k + GZ) * PS;
+      if (rel >= 0 && rel < 4) {
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          if (rel == e) out.v[e] += a.src_amp;
+      }
+      st4_masked(a.up + o, out, x0, d.nx, true);
       if (SNAP || IMG) {
-        const long long cix = ((long long)k * d.ny + j) * d.nx + i;
-        if (SNAP) a.snap[cix] = out;
-        if (IMG) a.img[cix] = fmaf(__ldg(a.imgS + cix), q4, a.img[cix]);
+        const long long cix = ((long long)k * d.ny + j) * d.nx + x0;
+        const bool al = (d.nx & 3) == 0;
+        if (SNAP) st4_masked(a.snap + cix, out, x0, d.nx, al);
+        if (IMG) {
+          F4 im;
+#pragma unroll
+          for (int e = 0; e < 4; ++e)
+            im.v[e] = (x0 + e < d.nx) ? fmaf(__ldg(a.imgS + cix + e), q[4].v[e], a.img[cix + e]) : 0.f;
+          st4_masked(a.img + cix, im, x0, d.nx, false);
+        }
       }
     }
     __syncthreads();  // every thread is done with stage s
@@ -130,7 +168,8 @@ __global__ void __launch_bounds__(TXW * BY) iso_step_kernel(const __grid_constan
       fence_proxy_async();
       issue(s, k + ISO_NS);
     }
-    q0 = q1; q1 = q2; q2 = q3; q3 = q4; q4 = q5; q5 = q6; q6 = q7; q7 = q8;
+#pragma unroll
+    for (int t = 0; t < 8; ++t) q[t] = q[t + 1];
   }
 }
 

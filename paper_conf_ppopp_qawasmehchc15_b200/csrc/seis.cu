@@ -123,7 +123,7 @@ struct Slab {
   // TMA descriptors of every operand tile the kernels stage:
   // "t" = tile with x/y halo, "c" = interior (centre) tile 32 x BY
   CUtensorMap iso_ut[2], iso_uc[2], iso_m;                              // ISO
-  CUtensorMap ac_pt[2], ac_qxt[2], ac_qyt[2], ac_rt, ac_kc;             // ACOUSTIC (A/B buffers)
+  CUtensorMap ac_pt, ac_qc[3], ac_rt, ac_rc, ac_qxt, ac_qyt, ac_pc, ac_kc;  // ACOUSTIC
   CUtensorMap el_sxxt, el_sxyt, el_sxzt, el_syyt, el_syzt, el_vc[3], el_bc[3];  // ELASTIC V
   CUtensorMap el_vt[3], el_sc[6], el_cc[5];                             // ELASTIC S
   int cur = 0;               // ISO: fld[cur] = u^n
@@ -230,7 +230,7 @@ Dims make_dims(const seis_grid& g, int z0, int nzl) {
   d.nzl = nzl;
   d.nz = g.nz;
   d.z0 = z0;
-  d.PX = roundup(roundup(g.nx, TXW) + 2 * G, 32);
+  d.PX = roundup(roundup(g.nx, TXV) + 2 * G, 32);
   d.PY = roundup(g.ny, BY) + 2 * G;
   d.PS = (long long)d.PX * d.PY;
   return d;
@@ -300,9 +300,10 @@ seis_status set_smem_attrs() {
   SMEM_ATTR((iso_step_kernel<BY, false, false>), IsoStage<BY>::smem_bytes());
   SMEM_ATTR((iso_step_kernel<BY, true, false>), IsoStage<BY>::smem_bytes());
   SMEM_ATTR((iso_step_kernel<BY, false, true>), IsoStage<BY>::smem_bytes());
-  SMEM_ATTR((ac_step_kernel<BY, false, false>), AcFStage<BY>::smem_bytes());
-  SMEM_ATTR((ac_step_kernel<BY, true, false>), AcFStage<BY>::smem_bytes());
-  SMEM_ATTR((ac_step_kernel<BY, false, true>), AcFStage<BY>::smem_bytes());
+  SMEM_ATTR((ac_v_kernel<BY, false>), AcVStage<BY>::smem_bytes());
+  SMEM_ATTR((ac_v_kernel<BY, true>), AcVStage<BY>::smem_bytes());
+  SMEM_ATTR((ac_p_kernel<BY, false>), AcPStage<BY>::smem_bytes());
+  SMEM_ATTR((ac_p_kernel<BY, true>), AcPStage<BY>::smem_bytes());
   SMEM_ATTR((el_v_kernel<BYE>), ElVStage<BYE>::smem_bytes());
   SMEM_ATTR((el_s_kernel<BYE, false>), ElSStage<BYE>::smem_bytes());
 #undef SMEM_ATTR
@@ -310,33 +311,22 @@ seis_status set_smem_attrs() {
   return SEIS_OK;
 }
 
-// Choose the z-chunk so the launch fills the machine in whole waves.
-void choose_chunks(Slab& s, int resident_per_sm, int nsm, int by) {
-  const int bxy = ((s.d.nx + TXW - 1) / TXW) * ((s.d.ny + by - 1) / by);
+// Choose the z-chunk: enough blocks for >= 6 waves of the resident
+// slots (dynamic block scheduling keeps the tail short), chunks of >= 32 planes so
+// the 8-plane queue warm-up stays small.
+void choose_chunks(Slab& s, int resident_per_sm, int nsm, int tw, int by) {
+  const long long bxy = (long long)((s.d.nx + tw - 1) / tw) * ((s.d.ny + by - 1) / by);
   const long long slots = (long long)std::max(1, resident_per_sm) * nsm;
-  double best = 1e300;
-  int bestc = 1;
-  for (int c = 1; c <= 64 && c <= s.d.nzl; ++c) {
-    const int zc = (s.d.nzl + c - 1) / c;
-    const long long blocks = (long long)bxy * c;
-    const long long waves = (blocks + slots - 1) / slots;
-    const double t = (double)waves * (zc + 8);  // 8 warm-up planes per chunk
-    if (t < best - 1e-9) {
-      best = t;
-      bestc = c;
-    }
-  }
-  s.nzch = bestc;
-  s.zc = (s.d.nzl + bestc - 1) / bestc;
+  int c = 1;
+  while (bxy * c < 6 * slots && (s.d.nzl + c) / (c + 1) >= 32) ++c;
+  s.zc = (s.d.nzl + c - 1) / c;
   s.nzch = (s.d.nzl + s.zc - 1) / s.zc;
 }
 
-// ISO: u at two time levels; ACOUSTIC: (p, qx, qy, qz) x 2 buffers (fused step reads A,
-// writes B); ELASTIC: 9 fields updated in place.
-int nfields(seis_kind k) { return k == SEIS_ISO ? 2 : (k == SEIS_ACOUSTIC ? 8 : 9); }
-int npsi_of(seis_kind k) { return k == SEIS_ACOUSTIC ? 9 : (k == SEIS_ELASTIC ? 18 : 0); }
-// axis of each C-PML memory array: ACOUSTIC psi_p A (x,y,z), psi_q (x,y,z), psi_p B (x,y,z);
-// ELASTIC in the oracle's order
+int nfields(seis_kind k) { return k == SEIS_ISO ? 2 : (k == SEIS_ACOUSTIC ? 4 : 9); }
+int npsi_of(seis_kind k) { return k == SEIS_ACOUSTIC ? 6 : (k == SEIS_ELASTIC ? 18 : 0); }
+// axis of each C-PML memory array: ACOUSTIC psi_p (x,y,z), psi_q (x,y,z); ELASTIC in the
+// oracle's order
 int psi_axis(seis_kind k, int t) {
   static const int el_axis[18] = {0, 1, 2, 0, 1, 2, 0, 1, 2, 0, 1, 2, 1, 0, 2, 0, 2, 1};
   return k == SEIS_ACOUSTIC ? t % 3 : el_axis[t];
@@ -576,8 +566,9 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
           hf[i] = (float)(M->eta1[ax][i] * dt);
         }
       }
-      TRY(alloc_track(M, (void**)&e1[ax], N * sizeof(float)));
-      CK(cudaMemcpy(e1[ax], hf.data(), N * sizeof(float), cudaMemcpyHostToDevice));
+      hf.resize(std::max(N, roundup(N, TXV) + TXV), 0.f);  // float4 loads past nx read zeros
+      TRY(alloc_track(M, (void**)&e1[ax], hf.size() * sizeof(float)));
+      CK(cudaMemcpy(e1[ax], hf.data(), hf.size() * sizeof(float), cudaMemcpyHostToDevice));
     }
     if (g.nb > 0) {
       M->edx = e1[0];
@@ -619,10 +610,9 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
         seis_slab_bounds(g.nz, M->nranks, r, &rz0, &rn);
         seis_slab_bounds(rn, ns, s, &lz0, &ln);
         const int z0 = rz0 + lz0;
-        const int need = kind == SEIS_ACOUSTIC ? GZ : 4;
-        if (ln < need) return fail(SEIS_EINVAL, "z-slab of %d planes: the decomposition needs >= %d", ln, need);
-        if (kind == SEIS_ACOUSTIC && z0 > 0 && (z0 - GZ < W || z0 + GZ > g.nz - W))
-          return fail(SEIS_EINVAL, "slab boundary z=%d lies within %d planes of an absorbing layer", z0, GZ);
+        (void)W;
+        (void)z0;
+        if (ln < 4) return fail(SEIS_EINVAL, "z-slab of %d planes: the decomposition needs >= 4", ln);
       }
   }
   M->slabs.resize(ns);
@@ -656,7 +646,7 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       TRY(upload_padded_from_host(M, d, hc, &S.m, st));
     } else {
       // buoyancy on faces (O8): dt * 2/(rho_i + rho_{i+1}) / h, last face clamps
-      // (ELASTIC only; the fused acoustic step evaluates it on the fly from rho)
+      // (ELASTIC; the acoustic V kernel evaluates it on the fly from rho)
       for (int ax = 0; ax < 3 && kind == SEIS_ELASTIC; ++ax) {
         for (int k = 0; k < lnz; ++k)
           for (int j = 0; j < g.ny; ++j)
@@ -738,18 +728,19 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     // TMA descriptors
     if (kind == SEIS_ISO) {
       for (int t = 0; t < 2; ++t) {
-        TRY(make_map(&S.iso_ut[t], S.fld[t], d, TXW + 8, BY + 8));
-        TRY(make_map(&S.iso_uc[t], S.fld[t], d, TXW, BY));
+        TRY(make_map(&S.iso_ut[t], S.fld[t], d, TXV + 8, BY + 8));
+        TRY(make_map(&S.iso_uc[t], S.fld[t], d, TXV, BY));
       }
-      TRY(make_map(&S.iso_m, S.m, d, TXW, BY));
+      TRY(make_map(&S.iso_m, S.m, d, TXV, BY));
     } else if (kind == SEIS_ACOUSTIC) {
-      for (int b = 0; b < 2; ++b) {
-        TRY(make_map(&S.ac_pt[b], S.fld[4 * b + 0], d, TXW + 16, BY + 16));
-        TRY(make_map(&S.ac_qxt[b], S.fld[4 * b + 1], d, TXW + 8, BY));
-        TRY(make_map(&S.ac_qyt[b], S.fld[4 * b + 2], d, TXW, BY + 8));
-      }
-      TRY(make_map(&S.ac_rt, S.rho, d, TXW + 16, BY + 16));
-      TRY(make_map(&S.ac_kc, S.kdt, d, TXW, BY));
+      TRY(make_map(&S.ac_pt, S.fld[0], d, TXV + 8, BY + 8));
+      for (int t = 0; t < 3; ++t) TRY(make_map(&S.ac_qc[t], S.fld[1 + t], d, TXV, BY));
+      TRY(make_map(&S.ac_rt, S.rho, d, TXV + 4, BY + 1));
+      TRY(make_map(&S.ac_rc, S.rho, d, TXV, BY));
+      TRY(make_map(&S.ac_qxt, S.fld[1], d, TXV + 8, BY));
+      TRY(make_map(&S.ac_qyt, S.fld[2], d, TXV, BY + 8));
+      TRY(make_map(&S.ac_pc, S.fld[0], d, TXV, BY));
+      TRY(make_map(&S.ac_kc, S.kdt, d, TXV, BY));
     } else {
       TRY(make_map(&S.el_sxxt, S.fld[ESXX], d, TXW + 8, BYE));
       TRY(make_map(&S.el_sxyt, S.fld[ESXY], d, TXW + 8, BYE + 8));
@@ -769,20 +760,19 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     TRY(set_smem_attrs());
     int occ = 1;
     if (kind == SEIS_ISO)
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, iso_step_kernel<BY, false, false>, TXW * BY,
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, iso_step_kernel<BY, false, false>, NTX * BY,
                                                     IsoStage<BY>::smem_bytes());
     else if (kind == SEIS_ACOUSTIC)
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_step_kernel<BY, false, false>, TXW * BY,
-                                                    AcFStage<BY>::smem_bytes());
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_v_kernel<BY, false>, NTX * BY,
+                                                    AcVStage<BY>::smem_bytes());
     else
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, TXW * BYE,
                                                     ElSStage<BYE>::smem_bytes());
-    choose_chunks(S, occ, dev_sms, kind == SEIS_ELASTIC ? BYE : BY);
+    if (kind == SEIS_ELASTIC) choose_chunks(S, occ, dev_sms, TXW, BYE);
+    else choose_chunks(S, occ, dev_sms, TXV, BY);
   }
-  if (kind == SEIS_ACOUSTIC) {
-    // rho z-ghosts from the neighbouring slabs / ranks (the fused step recomputes q_z on them)
-    TRY(exchange_arrays(M, {[](Slab& S) { return S.rho; }}, GZ, st));
-  }
+  if (kind == SEIS_ACOUSTIC)  // rho(k+1) across slab faces
+    TRY(exchange_arrays(M, {[](Slab& S) { return S.rho; }}, 4, st));
   CK(cudaStreamSynchronize(st));
   return SEIS_OK;
 }
@@ -845,12 +835,12 @@ seis_status seis_memory_required(const seis_grid* g, seis_kind kind, const seis_
   seis_slab_bounds(g->nz, nranks, 0, &z0, &nzl);
   const Dims d = make_dims(*g, 0, nzl);
   const double padded = (double)d.PS * (nzl + 2 * GZ) * 4.0;
-  int nf = nfields(kind), np = kind == SEIS_ISO ? 1 : (kind == SEIS_ACOUSTIC ? 2 : 8);
+  int nf = nfields(kind), np = kind == SEIS_ISO ? 1 : (kind == SEIS_ACOUSTIC ? 4 : 8);
   double b = (nf + np) * padded;
   if (kind != SEIS_ISO && g->nb > 0) {
     const double W = g->nb + 1;
     const double per = (2 * W * g->ny * (double)nzl + 2 * W * g->nx * (double)nzl + 2 * W * g->nx * (double)g->ny) * 4.0;
-    b += per * (kind == SEIS_ACOUSTIC ? 3 : 6);
+    b += per * (kind == SEIS_ACOUSTIC ? 2 : 6);
   }
   if (shot && shot->snap_period >= 1 && shot->nt >= 1)
     b += (double)((shot->nt - 1) / shot->snap_period) * nzl * (double)g->ny * g->nx * 4.0;
@@ -995,8 +985,9 @@ seis_status fs_mirror(seis_model* M, std::initializer_list<int> fields, cudaStre
   return SEIS_OK;
 }
 
-dim3 grid_of(const Slab& S, int by = BY) {
-  return dim3((S.d.nx + TXW - 1) / TXW, (S.d.ny + by - 1) / by, S.nzch);
+// ISO / ACOUSTIC: 64 x BY tiles of (16, BY) threads; ELASTIC: 32 x BYE tiles of (32, BYE)
+dim3 grid_of(const Slab& S, int tw = TXV, int by = BY) {
+  return dim3((S.d.nx + tw - 1) / tw, (S.d.ny + by - 1) / by, S.nzch);
 }
 
 // Backward-phase receiver injection into the field just produced (before its
@@ -1004,7 +995,7 @@ dim3 grid_of(const Slab& S, int by = BY) {
 seis_status inject_rows(seis_model* M, const float* row, cudaStream_t st) {
   for (Slab& S : M->slabs) {
     if (S.ngroups == 0) continue;
-    float* f = M->kind == SEIS_ISO ? S.fld[S.cur] : S.fld[4 * S.cur];
+    float* f = M->kind == SEIS_ISO ? S.fld[S.cur] : S.fld[0];
     PROF(5, st);
     inject_kernel<<<(S.ngroups + 127) / 128, 128, 0, st>>>(f, S.d_g_off, S.d_g_scale, S.d_g_start,
                                                            S.d_g_mem, row, S.ngroups);
@@ -1019,7 +1010,7 @@ seis_status inject_rows(seis_model* M, const float* row, cudaStream_t st) {
 seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
                  std::vector<const float*>* imgS, std::vector<float*>* img, cudaStream_t st,
                  const float* inj_row = nullptr) {
-  const dim3 blk(TXW, BY);
+  const dim3 blk(NTX, BY);
   if (M->kind == SEIS_ISO) {
     for (size_t s = 0; s < M->slabs.size(); ++s) {
       Slab& S = M->slabs[s];
@@ -1027,6 +1018,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.mun = S.iso_ut[S.cur];
       a.mup = S.iso_uc[1 - S.cur];
       a.mm = S.iso_m;
+      a.muq = S.iso_uc[S.cur];
       a.un = S.fld[S.cur];
       a.up = S.fld[1 - S.cur];
       a.edx = M->edx;
@@ -1060,34 +1052,57 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
   if (M->kind == SEIS_ACOUSTIC) {
     for (size_t s = 0; s < M->slabs.size(); ++s) {
       Slab& S = M->slabs[s];
-      const int A = S.cur, B = 1 - S.cur;
-      AcFArgs a;
-      a.mp = S.ac_pt[A];
+      AcVArgs a;
+      a.mp = S.ac_pt;
+      a.mqx = S.ac_qc[0];
+      a.mqy = S.ac_qc[1];
+      a.mqz = S.ac_qc[2];
       a.mr = S.ac_rt;
-      a.mqx = S.ac_qxt[A];
-      a.mqy = S.ac_qyt[A];
-      a.mk = S.ac_kc;
-      a.pA = S.fld[4 * A];
-      a.qzA = S.fld[4 * A + 3];
+      a.mpq = S.ac_pc;
+      a.mrz = S.ac_rc;
+      a.p = S.fld[0];
       a.rho = S.rho;
-      a.pB = S.fld[4 * B];
-      a.qxB = S.fld[4 * B + 1];
-      a.qyB = S.fld[4 * B + 2];
-      a.qzB = S.fld[4 * B + 3];
       a.dth = (float)((double)M->g.dt / (double)M->g.h);
+      a.qx = S.fld[1];
+      a.qy = S.fld[2];
+      a.qz = S.fld[3];
       a.W = M->W;
       a.zlo = 1;
       a.cx = M->cp[0];
       a.cy = M->cp[1];
       a.cz = M->cp[2];
-      float** pin = A == 0 ? S.psi + 0 : S.psi + 6;
-      float** pout = A == 0 ? S.psi + 6 : S.psi + 0;
-      a.psxA = pin[0];
-      a.psyA = pin[1];
-      a.pszA = pin[2];
-      a.psxB = pout[0];
-      a.psyB = pout[1];
-      a.pszB = pout[2];
+      a.psx = S.psi[0];
+      a.psy = S.psi[1];
+      a.psz = S.psi[2];
+      a.d = S.d;
+      a.zc = S.zc;
+      a.imgS = imgS ? (*imgS)[s] : nullptr;
+      a.img = img ? (*img)[s] : nullptr;
+      const dim3 gr = grid_of(S);
+      {
+        PROF(1, st);
+        const size_t sb = AcVStage<BY>::smem_bytes();
+        if (a.img) ac_v_kernel<BY, true><<<gr, blk, sb, st>>>(a);
+        else ac_v_kernel<BY, false><<<gr, blk, sb, st>>>(a);
+      }
+      CKL();
+    }
+    TRY(exchange(M, {3}, st));  // q_z has the only z-derivative in P
+    for (size_t s = 0; s < M->slabs.size(); ++s) {
+      Slab& S = M->slabs[s];
+      AcPArgs a;
+      a.mqx = S.ac_qxt;
+      a.mqy = S.ac_qyt;
+      a.mpp = S.ac_pc;
+      a.mk = S.ac_kc;
+      a.mqq = S.ac_qc[2];
+      a.p = S.fld[0];
+      a.qz = S.fld[3];
+      a.W = M->W;
+      a.zlo = 1;
+      a.cx = M->cp[0];
+      a.cy = M->cp[1];
+      a.cz = M->cp[2];
       a.pqx = S.psi[3];
       a.pqy = S.psi[4];
       a.pqz = S.psi[5];
@@ -1097,25 +1112,17 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.src_amp = 0.f;
       if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
       a.snap = snap ? (*snap)[s] : nullptr;
-      a.imgS = imgS ? (*imgS)[s] : nullptr;
-      a.img = img ? (*img)[s] : nullptr;
       const dim3 gr = grid_of(S);
       {
-        PROF(1, st);
-        const size_t sb = AcFStage<BY>::smem_bytes();
-        if (a.snap) ac_step_kernel<BY, true, false><<<gr, blk, sb, st>>>(a);
-        else if (a.img) ac_step_kernel<BY, false, true><<<gr, blk, sb, st>>>(a);
-        else ac_step_kernel<BY, false, false><<<gr, blk, sb, st>>>(a);
+        PROF(2, st);
+        const size_t sb = AcPStage<BY>::smem_bytes();
+        if (a.snap) ac_p_kernel<BY, true><<<gr, blk, sb, st>>>(a);
+        else ac_p_kernel<BY, false><<<gr, blk, sb, st>>>(a);
       }
       CKL();
     }
-    for (Slab& S : M->slabs) S.cur = 1 - S.cur;
     if (inj_row) TRY(inject_rows(M, inj_row, st));
-    // ghosts of the new level: p (8 planes, the next step recomputes q_z on ghost planes
-    // from p at k-3 .. k+4) and q_z (4 planes)
-    const int c = M->slabs[0].cur;
-    TRY(exchange_arrays(M, {[c](Slab& S) { return S.fld[4 * c]; }}, GZ, st));
-    TRY(exchange(M, {4 * c + 3}, st));
+    TRY(exchange(M, {0}, st));  // p for the next V
     return SEIS_OK;
   }
   // ELASTIC
@@ -1141,7 +1148,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (int t = 0; t < 9; ++t) a.psi[t] = S.psi[t];
     a.d = S.d;
     a.zc = S.zc;
-    const dim3 gr = grid_of(S, BYE);
+    const dim3 gr = grid_of(S, TXW, BYE);
     {
       PROF(3, st);
       el_v_kernel<BYE><<<gr, dim3(TXW, BYE), ElVStage<BYE>::smem_bytes(), st>>>(a);
@@ -1169,7 +1176,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     a.src_o = with_src ? S.src_o : -1;
     a.src_amp = 0.f;
     if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
-    const dim3 gr = grid_of(S, BYE);
+    const dim3 gr = grid_of(S, TXW, BYE);
     {
       PROF(4, st);
       el_s_kernel<BYE, false><<<gr, dim3(TXW, BYE), ElSStage<BYE>::smem_bytes(), st>>>(a);
@@ -1184,7 +1191,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
 // Field holding the recorded / imaged quantity
 const float* out_field(seis_model* M, Slab& S, int comp) {
   if (M->kind == SEIS_ISO) return S.fld[S.cur];
-  if (M->kind == SEIS_ACOUSTIC) return S.fld[4 * S.cur];
+  if (M->kind == SEIS_ACOUSTIC) return S.fld[0];
   if (comp == 3) return S.fld[3];
   return S.fld[comp];
 }
@@ -1342,7 +1349,7 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
 seis_status seis_get_field(const seis_model* Mc, int32_t which, float* dst, void* stream) {
   seis_model* M = const_cast<seis_model*>(Mc);
   if (!M || !dst) return fail(SEIS_EINVAL, "null argument");
-  const int nf = M->kind == SEIS_ACOUSTIC ? 4 : nfields(M->kind);
+  const int nf = nfields(M->kind);
   if (which < 0 || which >= nf) return fail(SEIS_EINVAL, "field index %d out of range", which);
   CK(cudaSetDevice(M->device));
   cudaStream_t st = (cudaStream_t)stream;
@@ -1357,7 +1364,6 @@ seis_status seis_get_field(const seis_model* Mc, int32_t which, float* dst, void
   for (Slab& S : M->slabs) {
     int f = which;
     if (M->kind == SEIS_ISO) f = which == 0 ? S.cur : 1 - S.cur;
-    if (M->kind == SEIS_ACOUSTIC) f = 4 * S.cur + which;
     unpad_kernel<<<1024, 256, 0, st>>>(out + (size_t)(S.d.z0 - M->pz0) * g.ny * g.nx, S.fld[f], S.d);
     CKL();
   }

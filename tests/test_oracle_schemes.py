@@ -387,3 +387,53 @@ def test_elastic_energy_conserved_without_absorbing_layer():
     E = np.asarray(E)
     assert E[0] > 0
     assert np.abs(E / E[0] - 1).max() < 1e-11
+
+
+# ----------------------------------------------------------- free surface (O16)
+def test_free_surface_equals_mirrored_full_space():
+    """Normal incidence on the stress-imaging free surface (O16): a laterally uniform
+    P (vz, szz, sxx, syy) and S (vx, sxz) pulse in a half space with a free top must equal
+    the full-space solution started from the odd/even mirror image of the initial data
+    (szz, sxx, syy, sxz, syz odd; vx, vy, vz even about the surface plane), i.e. the surface
+    reflects with R_sigma = -1 and doubles the surface velocity, exactly."""
+    nh, h, dt = 80, 10.0, 1e-3
+    vp_, vs_, r_ = 3000.0, 1700.0, 2200.0
+    gh = oracle.Grid(4, 4, nh, h=h, dt=dt, free_surface=1, periodic=1)
+    gf = oracle.Grid(4, 4, 2 * nh, h=h, dt=dt, periodic=1)
+    k = np.arange(nh, dtype=np.float64)
+    prof = np.exp(-((k - 10.0) / 3.0) ** 2)
+    prof2 = np.exp(-((k - 14.0) / 2.5) ** 2) * np.sin(k / 3.0)
+    half = oracle.el_state(gh)
+    init = {2: prof, 5: prof2, 0: prof2, 7: prof}  # vz, szz, vx, sxz
+    for f, pr in init.items():
+        pr = pr.copy()
+        if f == 5:
+            pr[0] = 0.0  # an odd integer-z field vanishes on the surface plane
+        half["f"][f] = pr[:, None, None] * np.ones((1, 4, 4))
+    full = oracle.el_state(gf)
+    odd = {3, 4, 5, 7, 8}
+    halfz = {2, 7, 8}
+    for f in range(9):
+        s = -1.0 if f in odd else 1.0
+        src = half["f"][f][:, 0, 0]
+        col = np.zeros(2 * nh)
+        col[nh:] = src
+        if f in halfz:
+            col[nh - 1 - np.arange(nh)] = s * src
+        else:
+            col[nh - np.arange(1, nh)] = s * src[1:]
+        full["f"][f] = col[:, None, None] * np.ones((1, 4, 4))
+    vp = lambda g: np.full(g.shape, vp_, np.float32)
+    vs = lambda g: np.full(g.shape, vs_, np.float32)
+    rr = lambda g: np.full(g.shape, r_, np.float32)
+    nsteps = 100
+    surf = oracle.el_run(gh, vp(gh), vs(gh), rr(gh), half, 0, nsteps, rec_pos=[(0, 0, 0)], component=2)
+    oracle.el_run(gf, vp(gf), vs(gf), rr(gf), full, 0, nsteps)
+    cmp = slice(0, 24)
+    for f in range(9):
+        a = half["f"][f][cmp, 0, 0]
+        b = full["f"][f][nh:nh + 24, 0, 0]
+        scale = max(np.abs(full["f"][f]).max(), 1e-30)
+        assert np.abs(a - b).max() <= 1e-10 * scale, f
+    # the pulse did reach the surface: surface vz peaks at about twice the incident amplitude
+    assert np.abs(surf).max() > 0.5

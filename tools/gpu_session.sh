@@ -13,7 +13,7 @@ for w in $what; do
     ncu)
       timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
         --log-file gpurun_out/${tag}_launches.csv python tools/ncu_target.py --kind acoustic --nt 20 > /dev/null 2>&1; echo "launches rc=$?"
-      for k in ac_step; do
+      for k in ac_v ac_p; do
         timeout 600 ncu --set full --clock-control none --import-source on -k regex:${k}_kernel -s 4 -c 1 \
           -o gpurun_out/${tag}_${k} python tools/ncu_target.py --kind acoustic --nt 6 > gpurun_out/${tag}_${k}_ncu.log 2>&1; echo "ncu $k rc=$?"
       done;;
