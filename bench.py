@@ -214,17 +214,20 @@ def run_product(args):
     local_pts = float(wl.nx) * wl.ny * nzl
     bpp = ALG_BYTES[dom] + psi_bytes_per_point(wl.nx, wl.ny, nz, wl.nb, PSI_AXES[dom])
     achieved = local_pts * bpp / (kms / kn * 1e-3) / 1e9
-    traffic = None
+    traffic = None  # DRAM bytes per launch from the committed ncu capture (same kernel, same size)
     try:
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
             tr = json.load(f).get(f"C2_{n}_{dom}")
-            if tr:
-                traffic = tr
+            if tr and ws == 1:
+                traffic = int(tr)
     except Exception:
         pass
     roof = {"bound": "hbm", "kernel": dom, "achieved": round(achieved, 1), "peak": hbm,
             "peak_source": peak_src, "unit": "GB/s", "frac": round(achieved / hbm, 4),
-            "traffic": traffic, "alg_bytes_per_point": round(bpp, 2),
+            "traffic": traffic, "traffic_unit": "DRAM bytes per launch (ncu, profiles/traffic.json)",
+            "alg_bytes_per_launch": round(local_pts * bpp),
+            "traffic_over_alg": round(traffic / (local_pts * bpp), 3) if traffic else None,
+            "alg_bytes_per_point": round(bpp, 2),
             "kernel_ms_avg": round(kms / kn, 4),
             "kernels": {k: {"ms_avg": round(v[0] / v[1], 4), "launches": v[1],
                             "share": round(v[0] / sum(x[0] for x in kprof.values()), 4)}

@@ -22,7 +22,8 @@ __all__ = ["Grid", "Shot", "Model", "Comm", "SeisError", "lib", "slab_bounds", "
            "ELASTIC", "KINDS"]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_LIBPATH = os.path.join(_HERE, "libseis.so")
+# SEIS_LIBPATH selects an alternative build of the same library (tools/sweep.py tuning runs)
+_LIBPATH = os.environ.get("SEIS_LIBPATH", os.path.join(_HERE, "libseis.so"))
 
 ISO, ACOUSTIC, ELASTIC = 0, 1, 2
 KINDS = {"iso": ISO, "acoustic": ACOUSTIC, "elastic": ELASTIC}

@@ -39,20 +39,23 @@ def needs_build():
     return any(os.path.getmtime(s) > t for s in sources())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not needs_build():
+def build(force: bool = False, verbose: bool = False, defines=(), out: str = None) -> str:
+    """defines: extra -D macros (tile / ring-depth tuning sweeps); out: alternative .so path."""
+    target = out or LIB
+    if not force and out is None and not needs_build():
         return LIB
     inc, lib = nccl_dirs()
     cmd = (["nvcc"] + ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-shared",
                               "-Xptxas", "-v" if verbose else "-O3",
                               "-I", inc, "-I", os.path.join(ROOT, "include"),
-                              "-o", LIB + ".tmp", os.path.join(CSRC, "seis.cu"),
+                              *[f"-D{d}" for d in defines],
+                              "-o", target + ".tmp", os.path.join(CSRC, "seis.cu"),
                               "-L", lib, "-l:libnccl.so.2", "-Xlinker", "-rpath," + lib])
     if verbose:
         print(" ".join(cmd))
     subprocess.check_call(cmd)
-    os.replace(LIB + ".tmp", LIB)
-    return LIB
+    os.replace(target + ".tmp", target)
+    return target
 
 
 if __name__ == "__main__":

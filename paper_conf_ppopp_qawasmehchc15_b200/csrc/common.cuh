@@ -175,3 +175,27 @@ __device__ __forceinline__ void st4_masked(float* p, const F4& a, int x0, int nx
 }
 
 }  // namespace seis
+
+// 2-wide variant (the elastic kernels keep three z-queues per thread; float2 keeps
+// them in registers): a block tile is TXV = 64 points wide (32 threads) x BY rows.
+namespace seis {
+constexpr int NTX2 = 32;
+struct F2 {
+  float v[2];
+};
+__device__ __forceinline__ F2 lds2(const float* p) {
+  const float2 t = *reinterpret_cast<const float2*>(p);
+  return F2{{t.x, t.y}};
+}
+__device__ __forceinline__ F2 ldg2(const float* p) {
+  const float2 t = __ldg(reinterpret_cast<const float2*>(p));
+  return F2{{t.x, t.y}};
+}
+__device__ __forceinline__ void st2_masked(float* p, const F2& a, int x0, int nx) {
+  if (x0 + 1 < nx) {
+    *reinterpret_cast<float2*>(p) = make_float2(a.v[0], a.v[1]);
+  } else if (x0 < nx) {
+    p[0] = a.v[0];
+  }
+}
+}  // namespace seis

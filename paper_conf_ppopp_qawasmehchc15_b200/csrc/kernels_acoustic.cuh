@@ -26,8 +26,14 @@ struct CpmlAxis {
   const float* __restrict__ bh;
 };
 
-constexpr int AC_NS = 4;   // P kernel ring depth
-constexpr int AC_VNS = 3;  // V kernel ring depth (7 tiles per stage)
+#ifndef SEIS_AC_NS
+#define SEIS_AC_NS 2
+#endif
+#ifndef SEIS_AC_VNS
+#define SEIS_AC_VNS 3
+#endif
+constexpr int AC_NS = SEIS_AC_NS;    // P kernel ring depth
+constexpr int AC_VNS = SEIS_AC_VNS;  // V kernel ring depth
 
 // psi update of the 4 x-points of a group that lie inside an x layer
 __device__ __forceinline__ void cpml_x4(float* dv, float* __restrict__ ps, const Dims& d, int W, int x0,

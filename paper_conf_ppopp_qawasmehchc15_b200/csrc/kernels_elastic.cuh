@@ -17,6 +17,12 @@
 // planes hold the mirror images (filled by fs_mirror_kernel after every
 // exchange), the surface row uses ezz = -lam/(lam+2mu)(exx+eyy), and szz = 0 on
 // k = 0 after the source.
+//
+// Both kernels are 2.5D z-marches over 64 x BY tiles with 2 x-points per thread
+// (float2; each thread keeps three 8-deep z-queues in registers).  Every operand
+// of plane k -- the halo tiles of the fields differentiated in x/y, the
+// pointwise fields and coefficients, and the plane-(k+3|k+4) feeds of the
+// z-queues -- arrives by TMA in one stage of an mbarrier ring.
 #pragma once
 #include "common.cuh"
 #include "kernels_acoustic.cuh"  // CpmlAxis
@@ -25,70 +31,95 @@ namespace seis {
 
 enum { EVX, EVY, EVZ, ESXX, ESYY, ESZZ, ESXY, ESXZ, ESYZ };
 
-__device__ __forceinline__ void cpml_x(float& dv, float* __restrict__ ps, const Dims& d, int W, int i,
-                                       int j, int k, const float* __restrict__ ca,
-                                       const float* __restrict__ cb) {
-  const long long ix = ((long long)k * d.ny + j) * (2 * W) + CpmlIdx::slot(i, d.nx, W);
-  const float v = fmaf(__ldg(cb + i), ps[ix], __ldg(ca + i) * dv);
-  ps[ix] = v;
-  dv += v;
+// psi updates of the 2 x-points of a group (x layer: per point; y, z layers: per row/plane)
+__device__ __forceinline__ void cpml2_x(float* dv, float* __restrict__ ps, const Dims& d, int W, int x0,
+                                        int j, int k, const float* __restrict__ ca,
+                                        const float* __restrict__ cb) {
+#pragma unroll
+  for (int e = 0; e < 2; ++e) {
+    const int x = x0 + e;
+    if (x < d.nx && CpmlIdx::in(x, d.nx, W, true)) {
+      const long long ix = ((long long)k * d.ny + j) * (2 * W) + CpmlIdx::slot(x, d.nx, W);
+      const float v = fmaf(__ldg(cb + x), ps[ix], __ldg(ca + x) * dv[e]);
+      ps[ix] = v;
+      dv[e] += v;
+    }
+  }
 }
-__device__ __forceinline__ void cpml_y(float& dv, float* __restrict__ ps, const Dims& d, int W, int i,
-                                       int j, int k, const float* __restrict__ ca,
-                                       const float* __restrict__ cb) {
-  const long long iy = ((long long)k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + i;
-  const float v = fmaf(__ldg(cb + j), ps[iy], __ldg(ca + j) * dv);
-  ps[iy] = v;
-  dv += v;
+__device__ __forceinline__ void cpml2_y(float* dv, float* __restrict__ ps, const Dims& d, int W, int x0,
+                                        int j, int k, float ca, float cb) {
+  const long long iy = ((long long)k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0;
+#pragma unroll
+  for (int e = 0; e < 2; ++e)
+    if (x0 + e < d.nx) {
+      const float v = fmaf(cb, ps[iy + e], ca * dv[e]);
+      ps[iy + e] = v;
+      dv[e] += v;
+    }
 }
-__device__ __forceinline__ void cpml_z(float& dv, float* __restrict__ ps, const Dims& d, int W, int i,
-                                       int j, int gz, const float* __restrict__ ca,
-                                       const float* __restrict__ cb) {
-  const long long iz = ((long long)CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + i;
-  const float v = fmaf(__ldg(cb + gz), ps[iz], __ldg(ca + gz) * dv);
-  ps[iz] = v;
-  dv += v;
-}
-
-// staggered differences on a shared-memory row/column (stride S), times h
-template <int S>
-__device__ __forceinline__ float dplus(const float* c) {  // at i+1/2 from integer field
-  float r = SEIS_D1 * (c[S] - c[0]);
-  r = fmaf(SEIS_D2, c[2 * S] - c[-S], r);
-  r = fmaf(SEIS_D3, c[3 * S] - c[-2 * S], r);
-  return fmaf(SEIS_D4, c[4 * S] - c[-3 * S], r);
-}
-template <int S>
-__device__ __forceinline__ float dminus(const float* c) {  // at i from half field
-  float r = SEIS_D1 * (c[0] - c[-S]);
-  r = fmaf(SEIS_D2, c[S] - c[-2 * S], r);
-  r = fmaf(SEIS_D3, c[2 * S] - c[-3 * S], r);
-  return fmaf(SEIS_D4, c[3 * S] - c[-4 * S], r);
-}
-// z-queue versions: qp[0..7] = f(k-3 .. k+4) for D+, qm[0..7] = f(k-4 .. k+3) for D-
-__device__ __forceinline__ float zplus(const float* q) {
-  float r = SEIS_D1 * (q[4] - q[3]);
-  r = fmaf(SEIS_D2, q[5] - q[2], r);
-  r = fmaf(SEIS_D3, q[6] - q[1], r);
-  return fmaf(SEIS_D4, q[7] - q[0], r);
-}
-__device__ __forceinline__ float zminus(const float* q) {
-  float r = SEIS_D1 * (q[4] - q[3]);
-  r = fmaf(SEIS_D2, q[5] - q[2], r);
-  r = fmaf(SEIS_D3, q[6] - q[1], r);
-  return fmaf(SEIS_D4, q[7] - q[0], r);
+__device__ __forceinline__ void cpml2_z(float* dv, float* __restrict__ ps, const Dims& d, int W, int x0,
+                                        int j, int gz, float ca, float cb) {
+  const long long iz = ((long long)CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0;
+#pragma unroll
+  for (int e = 0; e < 2; ++e)
+    if (x0 + e < d.nx) {
+      const float v = fmaf(cb, ps[iz + e], ca * dv[e]);
+      ps[iz + e] = v;
+      dv[e] += v;
+    }
 }
 
-constexpr int EL_NS = 3;
+// staggered differences, times h, along a line of values v (index c = the point)
+__device__ __forceinline__ float dp(const float* v, int c) {  // D+ at c+1/2 from integer field
+  float r = SEIS_D1 * (v[c + 1] - v[c]);
+  r = fmaf(SEIS_D2, v[c + 2] - v[c - 1], r);
+  r = fmaf(SEIS_D3, v[c + 3] - v[c - 2], r);
+  return fmaf(SEIS_D4, v[c + 4] - v[c - 3], r);
+}
+__device__ __forceinline__ float dm(const float* v, int c) {  // D- at c from half field
+  float r = SEIS_D1 * (v[c] - v[c - 1]);
+  r = fmaf(SEIS_D2, v[c + 1] - v[c - 2], r);
+  r = fmaf(SEIS_D3, v[c + 2] - v[c - 3], r);
+  return fmaf(SEIS_D4, v[c + 3] - v[c - 4], r);
+}
+// x-row of 10 values x0-4 .. x0+5 from a shared tile row (pointer at x0)
+__device__ __forceinline__ void xrow(float* xv, const float* c) {
+#pragma unroll
+  for (int t = 0; t < 5; ++t) {
+    const F2 a = lds2(c - 4 + 2 * t);
+    xv[2 * t] = a.v[0];
+    xv[2 * t + 1] = a.v[1];
+  }
+}
+// y-column values rows j-4 .. j+4 (9) for the 2 components, from a tile (row stride S)
+template <int S>
+__device__ __forceinline__ void ycol(float (*yv)[9], const float* c) {
+#pragma unroll
+  for (int m = 0; m < 9; ++m) {
+    const F2 a = lds2(c + (m - 4) * S);
+    yv[0][m] = a.v[0];
+    yv[1][m] = a.v[1];
+  }
+}
+
+#ifndef SEIS_EL_VNS
+#define SEIS_EL_VNS 3
+#endif
+#ifndef SEIS_EL_SNS
+#define SEIS_EL_SNS 2
+#endif
+constexpr int EL_VNS = SEIS_EL_VNS;
+constexpr int EL_SNS = SEIS_EL_SNS;
 
 struct ElVArgs {
-  CUtensorMap msxx;  // box 40 x BY      (x halo)
-  CUtensorMap msxy;  // box 40 x (BY+8)  (x and y halos)
-  CUtensorMap msxz;  // box 40 x BY
-  CUtensorMap msyy;  // box 32 x (BY+8)  (y halo)
-  CUtensorMap msyz;  // box 32 x (BY+8)
-  CUtensorMap mv[3]; // vx, vy, vz, box 32 x BY
-  CUtensorMap mb[3]; // face buoyancies, box 32 x BY
+  CUtensorMap msxx;   // box 72 x BY      (x halo)
+  CUtensorMap msxy;   // box 72 x (BY+8)  (x and y halos)
+  CUtensorMap msxz;   // box 72 x BY
+  CUtensorMap msyy;   // box 64 x (BY+8)  (y halo)
+  CUtensorMap msyz;   // box 64 x (BY+8)
+  CUtensorMap mv[3];  // vx, vy, vz, box 64 x BY
+  CUtensorMap mb[3];  // face buoyancies, box 64 x BY
+  CUtensorMap mq[3];  // z-queue feeds: sxz (k+3), syz (k+3), szz (k+4), box 64 x BY
   float* f[9];
   int W, zlo, fs;
   CpmlAxis cx, cy, cz;
@@ -99,14 +130,15 @@ struct ElVArgs {
 
 template <int BY>
 struct ElVStage {
-  static constexpr int WX = TXW + 8, T = TXW * BY;
+  static constexpr int WX = TXV + 8, T = TXV * BY;
   static constexpr int XX = 0, XY = XX + BY * WX, XZ = XY + (BY + 8) * WX, YY = XZ + BY * WX,
-                       YZ = YY + (BY + 8) * TXW, V = YZ + (BY + 8) * TXW, B = V + 3 * T, SIZE = B + 3 * T;
-  static constexpr size_t smem_bytes() { return (size_t)EL_NS * SIZE * 4 + 128; }
+                       YZ = YY + (BY + 8) * TXV, V = YZ + (BY + 8) * TXV, B = V + 3 * T, Q = B + 3 * T,
+                       SIZE = Q + 3 * T;
+  static constexpr size_t smem_bytes() { return (size_t)EL_VNS * SIZE * 4 + 128; }
 };
 
 template <int BY>
-__global__ void __launch_bounds__(TXW * BY) el_v_kernel(const __grid_constant__ ElVArgs a) {
+__global__ void __launch_bounds__(NTX2 * BY) el_v_kernel(const __grid_constant__ ElVArgs a) {
   using L = ElVStage<BY>;
   constexpr int WX = L::WX, T = L::T;
   constexpr uint32_t TX_BYTES = L::SIZE * 4;
@@ -114,111 +146,127 @@ __global__ void __launch_bounds__(TXW * BY) el_v_kernel(const __grid_constant__ 
                 "128-byte tiles");
   extern __shared__ __align__(128) float sm_raw[];
   float* sm = align128(sm_raw);
-  __shared__ __align__(8) uint64_t bar[EL_NS];
+  __shared__ __align__(8) uint64_t bar[EL_VNS];
   const Dims& d = a.d;
-  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
-  const int i0 = blockIdx.x * TXW, j0 = blockIdx.y * BY;
-  const int i = i0 + tx, j = j0 + ty;
+  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX2 + tx;
+  const int i0 = blockIdx.x * TXV, j0 = blockIdx.y * BY;
+  const int x0 = i0 + 2 * tx, j = j0 + ty;
   const int k0 = blockIdx.z * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
   const int np = k1 - k0;
-  const bool own = (i < d.nx) && (j < d.ny);
+  const bool own = (x0 < d.nx) && (j < d.ny);
   const long long PS = d.PS;
-  const long long oc = (long long)(j + G) * d.PX + (i + G);
+  const long long oc = (long long)(j + G) * d.PX + (x0 + G);
   const int W = a.W;
-  const bool lx = W > 0 && CpmlIdx::in(i, d.nx, W, true);
+  const bool lx = W > 0 && (x0 < W || x0 + 1 >= d.nx - W);
   const bool ly = W > 0 && CpmlIdx::in(j, d.ny, W, true);
-  const float* __restrict__ sxz = a.f[ESXZ];
-  const float* __restrict__ syz = a.f[ESYZ];
-  const float* __restrict__ szz = a.f[ESZZ];
   auto issue = [&](int s, int k) {
     float* st = sm + s * L::SIZE;
-    const int z = k + GZ;
+    const int z = k + GZ, x = i0 + G, y = j0 + G;
     mbar_expect_tx(&bar[s], TX_BYTES);
-    tma_load_3d(st + L::XX, &a.msxx, &bar[s], i0, j0 + G, z);
+    tma_load_3d(st + L::XX, &a.msxx, &bar[s], i0, y, z);
     tma_load_3d(st + L::XY, &a.msxy, &bar[s], i0, j0, z);
-    tma_load_3d(st + L::XZ, &a.msxz, &bar[s], i0, j0 + G, z);
-    tma_load_3d(st + L::YY, &a.msyy, &bar[s], i0 + G, j0, z);
-    tma_load_3d(st + L::YZ, &a.msyz, &bar[s], i0 + G, j0, z);
+    tma_load_3d(st + L::XZ, &a.msxz, &bar[s], i0, y, z);
+    tma_load_3d(st + L::YY, &a.msyy, &bar[s], x, j0, z);
+    tma_load_3d(st + L::YZ, &a.msyz, &bar[s], x, j0, z);
 #pragma unroll
     for (int c = 0; c < 3; ++c) {
-      tma_load_3d(st + L::V + c * T, &a.mv[c], &bar[s], i0 + G, j0 + G, z);
-      tma_load_3d(st + L::B + c * T, &a.mb[c], &bar[s], i0 + G, j0 + G, z);
+      tma_load_3d(st + L::V + c * T, &a.mv[c], &bar[s], x, y, z);
+      tma_load_3d(st + L::B + c * T, &a.mb[c], &bar[s], x, y, z);
     }
+    tma_load_3d(st + L::Q, &a.mq[0], &bar[s], x, y, z + 3);
+    tma_load_3d(st + L::Q + T, &a.mq[1], &bar[s], x, y, z + 3);
+    tma_load_3d(st + L::Q + 2 * T, &a.mq[2], &bar[s], x, y, z + 4);
   };
   if (tid == 0) {
-    for (int s = 0; s < EL_NS; ++s) mbar_init(&bar[s], 1);
+    for (int s = 0; s < EL_VNS; ++s) mbar_init(&bar[s], 1);
     mbar_fence_init();
   }
   __syncthreads();
   if (tid == 0)
-    for (int s = 0; s < EL_NS && s < np; ++s) issue(s, k0 + s);
-  float qxz[8], qyz[8], qzz[8];  // sxz, syz at k-4..k+3 (D-); szz at k-3..k+4 (D+)
+    for (int s = 0; s < EL_VNS && s < np; ++s) issue(s, k0 + s);
+  const float* __restrict__ sxz = a.f[ESXZ];
+  const float* __restrict__ syz = a.f[ESYZ];
+  const float* __restrict__ szz = a.f[ESZZ];
+  F2 qxz[8], qyz[8], qzz[8];  // sxz, syz at k-4..k+3 (D-); szz at k-3..k+4 (D+)
 #pragma unroll
   for (int t = 0; t < 7; ++t) {
-    qxz[t] = __ldg(sxz + (long long)(k0 - 4 + t + GZ) * PS + oc);
-    qyz[t] = __ldg(syz + (long long)(k0 - 4 + t + GZ) * PS + oc);
-    qzz[t] = __ldg(szz + (long long)(k0 - 3 + t + GZ) * PS + oc);
-  }
-  float axz = __ldg(sxz + (long long)(k0 + 3 + GZ) * PS + oc);
-  float ayz = __ldg(syz + (long long)(k0 + 3 + GZ) * PS + oc);
-  float azz = __ldg(szz + (long long)(k0 + 4 + GZ) * PS + oc);
-  float bxz = 0.f, byz = 0.f, bzz = 0.f;
-  if (np > 1) {
-    bxz = __ldg(sxz + (long long)(k0 + 4 + GZ) * PS + oc);
-    byz = __ldg(syz + (long long)(k0 + 4 + GZ) * PS + oc);
-    bzz = __ldg(szz + (long long)(k0 + 5 + GZ) * PS + oc);
+    qxz[t] = ldg2(sxz + (long long)(k0 - 4 + t + GZ) * PS + oc);
+    qyz[t] = ldg2(syz + (long long)(k0 - 4 + t + GZ) * PS + oc);
+    qzz[t] = ldg2(szz + (long long)(k0 - 3 + t + GZ) * PS + oc);
   }
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
-    const int s = it % EL_NS;
+    const int s = it % EL_VNS;
     const long long o = (long long)(k + GZ) * PS + oc;
-    qxz[7] = axz; qyz[7] = ayz; qzz[7] = azz;
-    axz = bxz; ayz = byz; azz = bzz;
-    if (it + 2 < np) {
-      bxz = __ldg(sxz + o + 5 * PS);
-      byz = __ldg(syz + o + 5 * PS);
-      bzz = __ldg(szz + o + 6 * PS);
-    }
-    mbar_wait(&bar[s], (it / EL_NS) & 1);
+    mbar_wait(&bar[s], (it / EL_VNS) & 1);
+    const float* st = sm + s * L::SIZE;
+    const int pt = ty * TXV + 2 * tx;
+    qxz[7] = lds2(st + L::Q + pt);
+    qyz[7] = lds2(st + L::Q + T + pt);
+    qzz[7] = lds2(st + L::Q + 2 * T + pt);
     if (own) {
-      const float* st = sm + s * L::SIZE;
-      const float* cxx = st + L::XX + ty * WX + tx + 4;
-      const float* cxy = st + L::XY + (ty + 4) * WX + tx + 4;
-      const float* cxz = st + L::XZ + ty * WX + tx + 4;
-      const float* cyy = st + L::YY + (ty + 4) * TXW + tx;
-      const float* cyz = st + L::YZ + (ty + 4) * TXW + tx;
-      float d0 = dplus<1>(cxx), d1 = dminus<WX>(cxy), d2 = zminus(qxz);
-      float d3 = dminus<1>(cxy), d4 = dplus<TXW>(cyy), d5 = zminus(qyz);
-      float d6 = dminus<1>(cxz), d7 = dminus<TXW>(cyz), d8 = zplus(qzz);
+      float xs[10], xy[10], xz[10], yxy[2][9], yyy[2][9], yyz[2][9];
+      xrow(xs, st + L::XX + ty * WX + 2 * tx + 4);
+      xrow(xy, st + L::XY + (ty + 4) * WX + 2 * tx + 4);
+      xrow(xz, st + L::XZ + ty * WX + 2 * tx + 4);
+      ycol<WX>(yxy, st + L::XY + (ty + 4) * WX + 2 * tx + 4);
+      ycol<TXV>(yyy, st + L::YY + (ty + 4) * TXV + 2 * tx);
+      ycol<TXV>(yyz, st + L::YZ + (ty + 4) * TXV + 2 * tx);
+      float d0[2], d1[2], d2[2], d3[2], d4[2], d5[2], d6[2], d7[2], d8[2];
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        float zxz[8], zyz[8], zzz[8];
+#pragma unroll
+        for (int t = 0; t < 8; ++t) {
+          zxz[t] = qxz[t].v[e];
+          zyz[t] = qyz[t].v[e];
+          zzz[t] = qzz[t].v[e];
+        }
+        d0[e] = dp(xs, 4 + e);   // Dx+ sxx
+        d1[e] = dm(yxy[e], 4);   // Dy- sxy
+        d2[e] = dm(zxz, 4);      // Dz- sxz  (zxz[0..7] = k-4..k+3)
+        d3[e] = dm(xy, 4 + e);   // Dx- sxy
+        d4[e] = dp(yyy[e], 4);   // Dy+ syy
+        d5[e] = dm(zyz, 4);      // Dz- syz
+        d6[e] = dm(xz, 4 + e);   // Dx- sxz
+        d7[e] = dm(yyz[e], 4);   // Dy- syz
+        d8[e] = dp(zzz, 3);      // Dz+ szz  (zzz[0..7] = k-3..k+4)
+      }
       if (W > 0) {
         const int gz = k + d.z0;
         if (lx) {
-          cpml_x(d0, a.psi[0], d, W, i, j, k, a.cx.ah, a.cx.bh);
-          cpml_x(d3, a.psi[3], d, W, i, j, k, a.cx.a, a.cx.b);
-          cpml_x(d6, a.psi[6], d, W, i, j, k, a.cx.a, a.cx.b);
+          cpml2_x(d0, a.psi[0], d, W, x0, j, k, a.cx.ah, a.cx.bh);
+          cpml2_x(d3, a.psi[3], d, W, x0, j, k, a.cx.a, a.cx.b);
+          cpml2_x(d6, a.psi[6], d, W, x0, j, k, a.cx.a, a.cx.b);
         }
         if (ly) {
-          cpml_y(d1, a.psi[1], d, W, i, j, k, a.cy.a, a.cy.b);
-          cpml_y(d4, a.psi[4], d, W, i, j, k, a.cy.ah, a.cy.bh);
-          cpml_y(d7, a.psi[7], d, W, i, j, k, a.cy.a, a.cy.b);
+          cpml2_y(d1, a.psi[1], d, W, x0, j, k, __ldg(a.cy.a + j), __ldg(a.cy.b + j));
+          cpml2_y(d4, a.psi[4], d, W, x0, j, k, __ldg(a.cy.ah + j), __ldg(a.cy.bh + j));
+          cpml2_y(d7, a.psi[7], d, W, x0, j, k, __ldg(a.cy.a + j), __ldg(a.cy.b + j));
         }
         if (CpmlIdx::in(gz, d.nz, W, a.zlo)) {
-          cpml_z(d2, a.psi[2], d, W, i, j, gz, a.cz.a, a.cz.b);
-          cpml_z(d5, a.psi[5], d, W, i, j, gz, a.cz.a, a.cz.b);
-          cpml_z(d8, a.psi[8], d, W, i, j, gz, a.cz.ah, a.cz.bh);
+          cpml2_z(d2, a.psi[2], d, W, x0, j, gz, __ldg(a.cz.a + gz), __ldg(a.cz.b + gz));
+          cpml2_z(d5, a.psi[5], d, W, x0, j, gz, __ldg(a.cz.a + gz), __ldg(a.cz.b + gz));
+          cpml2_z(d8, a.psi[8], d, W, x0, j, gz, __ldg(a.cz.ah + gz), __ldg(a.cz.bh + gz));
         }
       }
-      const float* sv = st + L::V + tid;
-      const float* sb = st + L::B + tid;
-      a.f[EVX][o] = fmaf(sb[0], (d0 + d1) + d2, sv[0]);
-      a.f[EVY][o] = fmaf(sb[T], (d3 + d4) + d5, sv[T]);
-      a.f[EVZ][o] = fmaf(sb[2 * T], (d6 + d7) + d8, sv[2 * T]);
+      const float* sv = st + L::V + pt;
+      const float* sb = st + L::B + pt;
+      F2 ov[3];
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        ov[0].v[e] = fmaf(sb[e], (d0[e] + d1[e]) + d2[e], sv[e]);
+        ov[1].v[e] = fmaf(sb[T + e], (d3[e] + d4[e]) + d5[e], sv[T + e]);
+        ov[2].v[e] = fmaf(sb[2 * T + e], (d6[e] + d7[e]) + d8[e], sv[2 * T + e]);
+      }
+#pragma unroll
+      for (int c = 0; c < 3; ++c) st2_masked(a.f[EVX + c] + o, ov[c], x0, d.nx);
     }
     __syncthreads();
-    if (tid == 0 && it + EL_NS < np) {
+    if (tid == 0 && it + EL_VNS < np) {
       fence_proxy_async();
-      issue(s, k + EL_NS);
+      issue(s, k + EL_VNS);
     }
 #pragma unroll
     for (int t = 0; t < 7; ++t) {
@@ -230,9 +278,10 @@ __global__ void __launch_bounds__(TXW * BY) el_v_kernel(const __grid_constant__ 
 }
 
 struct ElSArgs {
-  CUtensorMap mvt[3];  // vx, vy, vz tiles, box 40 x (BY+8)
-  CUtensorMap ms[6];   // sxx, syy, szz, sxy, sxz, syz, box 32 x BY
-  CUtensorMap mc[5];   // l2m, lam, mxy, mxz, myz, box 32 x BY
+  CUtensorMap mvt[3];  // vx, vy, vz tiles, box 72 x (BY+8)
+  CUtensorMap ms[6];   // sxx, syy, szz, sxy, sxz, syz, box 64 x BY
+  CUtensorMap mc[5];   // l2m, lam, mxy, mxz, myz, box 64 x BY
+  CUtensorMap mq[3];   // z-queue feeds: vx (k+4), vy (k+4), vz (k+3), box 64 x BY
   float* f[9];
   int W, zlo, fs;
   CpmlAxis cx, cy, cz;
@@ -245,133 +294,156 @@ struct ElSArgs {
 
 template <int BY>
 struct ElSStage {
-  static constexpr int WX = TXW + 8, T = TXW * BY, TV = (BY + 8) * WX;
-  static constexpr int VT = 0, S = 3 * TV, C = S + 6 * T, SIZE = C + 5 * T;
-  static constexpr size_t smem_bytes() { return (size_t)EL_NS * SIZE * 4 + 128; }
+  static constexpr int WX = TXV + 8, T = TXV * BY, TV = (BY + 8) * WX;
+  static constexpr int VT = 0, S = 3 * TV, C = S + 6 * T, Q = C + 5 * T, SIZE = Q + 3 * T;
+  static constexpr size_t smem_bytes() { return (size_t)EL_SNS * SIZE * 4 + 128; }
 };
 
 template <int BY, bool UNUSED>
-__global__ void __launch_bounds__(TXW * BY) el_s_kernel(const __grid_constant__ ElSArgs a) {
+__global__ void __launch_bounds__(NTX2 * BY) el_s_kernel(const __grid_constant__ ElSArgs a) {
   using L = ElSStage<BY>;
   constexpr int WX = L::WX, T = L::T, TV = L::TV;
   constexpr uint32_t TX_BYTES = L::SIZE * 4;
   extern __shared__ __align__(128) float sm_raw[];
   float* sm = align128(sm_raw);
-  __shared__ __align__(8) uint64_t bar[EL_NS];
+  __shared__ __align__(8) uint64_t bar[EL_SNS];
   const Dims& d = a.d;
-  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * TXW + tx;
-  const int i0 = blockIdx.x * TXW, j0 = blockIdx.y * BY;
-  const int i = i0 + tx, j = j0 + ty;
+  const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX2 + tx;
+  const int i0 = blockIdx.x * TXV, j0 = blockIdx.y * BY;
+  const int x0 = i0 + 2 * tx, j = j0 + ty;
   const int k0 = blockIdx.z * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
   const int np = k1 - k0;
-  const bool own = (i < d.nx) && (j < d.ny);
+  const bool own = (x0 < d.nx) && (j < d.ny);
   const long long PS = d.PS;
-  const long long oc = (long long)(j + G) * d.PX + (i + G);
+  const long long oc = (long long)(j + G) * d.PX + (x0 + G);
   const int W = a.W;
-  const bool lx = W > 0 && CpmlIdx::in(i, d.nx, W, true);
+  const bool lx = W > 0 && (x0 < W || x0 + 1 >= d.nx - W);
   const bool ly = W > 0 && CpmlIdx::in(j, d.ny, W, true);
-  const float* __restrict__ vx = a.f[EVX];
-  const float* __restrict__ vy = a.f[EVY];
-  const float* __restrict__ vz = a.f[EVZ];
   auto issue = [&](int s, int k) {
     float* st = sm + s * L::SIZE;
-    const int z = k + GZ;
+    const int z = k + GZ, x = i0 + G, y = j0 + G;
     mbar_expect_tx(&bar[s], TX_BYTES);
 #pragma unroll
     for (int c = 0; c < 3; ++c) tma_load_3d(st + L::VT + c * TV, &a.mvt[c], &bar[s], i0, j0, z);
 #pragma unroll
-    for (int c = 0; c < 6; ++c) tma_load_3d(st + L::S + c * T, &a.ms[c], &bar[s], i0 + G, j0 + G, z);
+    for (int c = 0; c < 6; ++c) tma_load_3d(st + L::S + c * T, &a.ms[c], &bar[s], x, y, z);
 #pragma unroll
-    for (int c = 0; c < 5; ++c) tma_load_3d(st + L::C + c * T, &a.mc[c], &bar[s], i0 + G, j0 + G, z);
+    for (int c = 0; c < 5; ++c) tma_load_3d(st + L::C + c * T, &a.mc[c], &bar[s], x, y, z);
+    tma_load_3d(st + L::Q, &a.mq[0], &bar[s], x, y, z + 4);
+    tma_load_3d(st + L::Q + T, &a.mq[1], &bar[s], x, y, z + 4);
+    tma_load_3d(st + L::Q + 2 * T, &a.mq[2], &bar[s], x, y, z + 3);
   };
   if (tid == 0) {
-    for (int s = 0; s < EL_NS; ++s) mbar_init(&bar[s], 1);
+    for (int s = 0; s < EL_SNS; ++s) mbar_init(&bar[s], 1);
     mbar_fence_init();
   }
   __syncthreads();
   if (tid == 0)
-    for (int s = 0; s < EL_NS && s < np; ++s) issue(s, k0 + s);
-  float qx[8], qy[8], qz[8];  // vx, vy at k-3..k+4 (D+); vz at k-4..k+3 (D-)
+    for (int s = 0; s < EL_SNS && s < np; ++s) issue(s, k0 + s);
+  const float* __restrict__ vx = a.f[EVX];
+  const float* __restrict__ vy = a.f[EVY];
+  const float* __restrict__ vz = a.f[EVZ];
+  F2 qx[8], qy[8], qz[8];  // vx, vy at k-3..k+4 (D+); vz at k-4..k+3 (D-)
 #pragma unroll
   for (int t = 0; t < 7; ++t) {
-    qx[t] = __ldg(vx + (long long)(k0 - 3 + t + GZ) * PS + oc);
-    qy[t] = __ldg(vy + (long long)(k0 - 3 + t + GZ) * PS + oc);
-    qz[t] = __ldg(vz + (long long)(k0 - 4 + t + GZ) * PS + oc);
+    qx[t] = ldg2(vx + (long long)(k0 - 3 + t + GZ) * PS + oc);
+    qy[t] = ldg2(vy + (long long)(k0 - 3 + t + GZ) * PS + oc);
+    qz[t] = ldg2(vz + (long long)(k0 - 4 + t + GZ) * PS + oc);
   }
-  float ax = __ldg(vx + (long long)(k0 + 4 + GZ) * PS + oc);
-  float ay = __ldg(vy + (long long)(k0 + 4 + GZ) * PS + oc);
-  float az = __ldg(vz + (long long)(k0 + 3 + GZ) * PS + oc);
-  float bx = 0.f, by = 0.f, bz = 0.f;
-  if (np > 1) {
-    bx = __ldg(vx + (long long)(k0 + 5 + GZ) * PS + oc);
-    by = __ldg(vy + (long long)(k0 + 5 + GZ) * PS + oc);
-    bz = __ldg(vz + (long long)(k0 + 4 + GZ) * PS + oc);
-  }
+  const long long srel0 = a.src_o - oc;
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
-    const int s = it % EL_NS;
+    const int s = it % EL_SNS;
     const long long o = (long long)(k + GZ) * PS + oc;
-    qx[7] = ax; qy[7] = ay; qz[7] = az;
-    ax = bx; ay = by; az = bz;
-    if (it + 2 < np) {
-      bx = __ldg(vx + o + 6 * PS);
-      by = __ldg(vy + o + 6 * PS);
-      bz = __ldg(vz + o + 5 * PS);
-    }
-    mbar_wait(&bar[s], (it / EL_NS) & 1);
+    mbar_wait(&bar[s], (it / EL_SNS) & 1);
+    const float* st = sm + s * L::SIZE;
+    const int pt = ty * TXV + 2 * tx;
+    qx[7] = lds2(st + L::Q + pt);
+    qy[7] = lds2(st + L::Q + T + pt);
+    qz[7] = lds2(st + L::Q + 2 * T + pt);
     if (own) {
       const int gz = k + d.z0;
-      const float* st = sm + s * L::SIZE;
-      const float* cvx = st + L::VT + (ty + 4) * WX + tx + 4;
+      const float* cvx = st + L::VT + (ty + 4) * WX + 2 * tx + 4;
       const float* cvy = cvx + TV;
       const float* cvz = cvx + 2 * TV;
-      float exx = dminus<1>(cvx), eyy = dminus<WX>(cvy), ezz = zminus(qz);
-      float dyvx = dplus<WX>(cvx), dxvy = dplus<1>(cvy);
-      float dzvx = zplus(qx), dxvz = dplus<1>(cvz);
-      float dzvy = zplus(qy), dyvz = dplus<WX>(cvz);
+      float xvx[10], xvy[10], xvz[10], yvx[2][9], yvy[2][9], yvz[2][9];
+      xrow(xvx, cvx);
+      xrow(xvy, cvy);
+      xrow(xvz, cvz);
+      ycol<WX>(yvx, cvx);
+      ycol<WX>(yvy, cvy);
+      ycol<WX>(yvz, cvz);
+      float exx[2], eyy[2], ezz[2], dyvx[2], dxvy[2], dzvx[2], dxvz[2], dzvy[2], dyvz[2];
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        float zx[8], zy[8], zz[8];
+#pragma unroll
+        for (int t = 0; t < 8; ++t) {
+          zx[t] = qx[t].v[e];
+          zy[t] = qy[t].v[e];
+          zz[t] = qz[t].v[e];
+        }
+        exx[e] = dm(xvx, 4 + e);   // Dx- vx
+        eyy[e] = dm(yvy[e], 4);    // Dy- vy
+        ezz[e] = dm(zz, 4);        // Dz- vz  (zz[0..7] = k-4..k+3)
+        dyvx[e] = dp(yvx[e], 4);   // Dy+ vx
+        dxvy[e] = dp(xvy, 4 + e);  // Dx+ vy
+        dzvx[e] = dp(zx, 3);       // Dz+ vx  (zx[0..7] = k-3..k+4)
+        dxvz[e] = dp(xvz, 4 + e);  // Dx+ vz
+        dzvy[e] = dp(zy, 3);       // Dz+ vy
+        dyvz[e] = dp(yvz[e], 4);   // Dy+ vz
+      }
       if (W > 0) {
         if (lx) {
-          cpml_x(exx, a.psi[0], d, W, i, j, k, a.cx.a, a.cx.b);
-          cpml_x(dxvy, a.psi[4], d, W, i, j, k, a.cx.ah, a.cx.bh);
-          cpml_x(dxvz, a.psi[6], d, W, i, j, k, a.cx.ah, a.cx.bh);
+          cpml2_x(exx, a.psi[0], d, W, x0, j, k, a.cx.a, a.cx.b);
+          cpml2_x(dxvy, a.psi[4], d, W, x0, j, k, a.cx.ah, a.cx.bh);
+          cpml2_x(dxvz, a.psi[6], d, W, x0, j, k, a.cx.ah, a.cx.bh);
         }
         if (ly) {
-          cpml_y(eyy, a.psi[1], d, W, i, j, k, a.cy.a, a.cy.b);
-          cpml_y(dyvx, a.psi[3], d, W, i, j, k, a.cy.ah, a.cy.bh);
-          cpml_y(dyvz, a.psi[8], d, W, i, j, k, a.cy.ah, a.cy.bh);
+          cpml2_y(eyy, a.psi[1], d, W, x0, j, k, __ldg(a.cy.a + j), __ldg(a.cy.b + j));
+          cpml2_y(dyvx, a.psi[3], d, W, x0, j, k, __ldg(a.cy.ah + j), __ldg(a.cy.bh + j));
+          cpml2_y(dyvz, a.psi[8], d, W, x0, j, k, __ldg(a.cy.ah + j), __ldg(a.cy.bh + j));
         }
         if (CpmlIdx::in(gz, d.nz, W, a.zlo)) {
-          cpml_z(ezz, a.psi[2], d, W, i, j, gz, a.cz.a, a.cz.b);
-          cpml_z(dzvx, a.psi[5], d, W, i, j, gz, a.cz.ah, a.cz.bh);
-          cpml_z(dzvy, a.psi[7], d, W, i, j, gz, a.cz.ah, a.cz.bh);
+          cpml2_z(ezz, a.psi[2], d, W, x0, j, gz, __ldg(a.cz.a + gz), __ldg(a.cz.b + gz));
+          cpml2_z(dzvx, a.psi[5], d, W, x0, j, gz, __ldg(a.cz.ah + gz), __ldg(a.cz.bh + gz));
+          cpml2_z(dzvy, a.psi[7], d, W, x0, j, gz, __ldg(a.cz.ah + gz), __ldg(a.cz.bh + gz));
         }
       }
-      const float* ss = st + L::S + tid;
-      const float* sc = st + L::C + tid;
-      const float l2m = sc[0], lam = sc[T];
+      const float* ss = st + L::S + pt;
+      const float* sc = st + L::C + pt;
       const bool surf = a.fs && gz == 0;
-      if (surf) ezz = -(lam / l2m) * (exx + eyy);  // O16 surface row
-      float sxx = ss[0] + fmaf(l2m, exx, lam * (eyy + ezz));
-      float syy = ss[T] + fmaf(l2m, eyy, lam * (exx + ezz));
-      float szz = ss[2 * T] + fmaf(l2m, ezz, lam * (exx + eyy));
-      if (o == a.src_o) {
-        sxx -= a.src_amp;
-        syy -= a.src_amp;
-        szz -= a.src_amp;
+      const long long rel = srel0 - (long long)(k + GZ) * PS;
+      F2 o6[6];
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        const float l2m = sc[e], lam = sc[T + e];
+        float ez = ezz[e];
+        if (surf) ez = -(lam / l2m) * (exx[e] + eyy[e]);  // O16 surface row
+        float sxx = ss[e] + fmaf(l2m, exx[e], lam * (eyy[e] + ez));
+        float syy = ss[T + e] + fmaf(l2m, eyy[e], lam * (exx[e] + ez));
+        float szz = ss[2 * T + e] + fmaf(l2m, ez, lam * (exx[e] + eyy[e]));
+        if (rel == e) {
+          sxx -= a.src_amp;
+          syy -= a.src_amp;
+          szz -= a.src_amp;
+        }
+        if (surf) szz = 0.0f;
+        o6[0].v[e] = sxx;
+        o6[1].v[e] = syy;
+        o6[2].v[e] = szz;
+        o6[3].v[e] = fmaf(sc[2 * T + e], dyvx[e] + dxvy[e], ss[3 * T + e]);
+        o6[4].v[e] = fmaf(sc[3 * T + e], dzvx[e] + dxvz[e], ss[4 * T + e]);
+        o6[5].v[e] = fmaf(sc[4 * T + e], dzvy[e] + dyvz[e], ss[5 * T + e]);
       }
-      if (surf) szz = 0.0f;
-      a.f[ESXX][o] = sxx;
-      a.f[ESYY][o] = syy;
-      a.f[ESZZ][o] = szz;
-      a.f[ESXY][o] = fmaf(sc[2 * T], dyvx + dxvy, ss[3 * T]);
-      a.f[ESXZ][o] = fmaf(sc[3 * T], dzvx + dxvz, ss[4 * T]);
-      a.f[ESYZ][o] = fmaf(sc[4 * T], dzvy + dyvz, ss[5 * T]);
+#pragma unroll
+      for (int c = 0; c < 6; ++c) st2_masked(a.f[ESXX + c] + o, o6[c], x0, d.nx);
     }
     __syncthreads();
-    if (tid == 0 && it + EL_NS < np) {
+    if (tid == 0 && it + EL_SNS < np) {
       fence_proxy_async();
-      issue(s, k + EL_NS);
+      issue(s, k + EL_SNS);
     }
 #pragma unroll
     for (int t = 0; t < 7; ++t) {

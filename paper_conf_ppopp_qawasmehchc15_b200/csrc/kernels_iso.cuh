@@ -39,7 +39,10 @@ struct IsoArgs {
   float* __restrict__ img;       // compact image (+=), or nullptr
 };
 
-constexpr int ISO_NS = 3;
+#ifndef SEIS_ISO_NS
+#define SEIS_ISO_NS 3
+#endif
+constexpr int ISO_NS = SEIS_ISO_NS;
 
 template <int BY>
 struct IsoStage {

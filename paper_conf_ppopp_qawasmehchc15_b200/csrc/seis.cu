@@ -107,8 +107,23 @@ struct seis_comm {
 
 namespace {
 
-constexpr int BY = 16;       // tile rows (block = 32 x BY threads), ISO and ACOUSTIC
-constexpr int BYE = 8;       // tile rows of the ELASTIC kernels (more registers per thread)
+// Tile rows per kernel (tools/sweep.py measures the alternatives on a B200).
+#ifndef SEIS_BYI
+#define SEIS_BYI 8
+#endif
+#ifndef SEIS_BYV
+#define SEIS_BYV 8
+#endif
+#ifndef SEIS_BYP
+#define SEIS_BYP 16
+#endif
+#ifndef SEIS_BYE
+#define SEIS_BYE 8
+#endif
+constexpr int BYI = SEIS_BYI;  // ISO step (block 16 x BYI threads, 4 x-points each)
+constexpr int BYV = SEIS_BYV;  // acoustic V (block 16 x BYV)
+constexpr int BYP = SEIS_BYP;  // acoustic P (block 16 x BYP)
+constexpr int BYE = SEIS_BYE;  // elastic V and S (block 32 x BYE threads, 2 x-points each)
 constexpr int NPSI = 18;
 
 struct Slab {
@@ -123,7 +138,8 @@ struct Slab {
   // TMA descriptors of every operand tile the kernels stage:
   // "t" = tile with x/y halo, "c" = interior (centre) tile 32 x BY
   CUtensorMap iso_ut[2], iso_uc[2], iso_m;                              // ISO
-  CUtensorMap ac_pt, ac_qc[3], ac_rt, ac_rc, ac_qxt, ac_qyt, ac_pc, ac_kc;  // ACOUSTIC
+  CUtensorMap ac_pt, ac_qc[3], ac_rt, ac_rc, ac_pc;        // ACOUSTIC V
+  CUtensorMap ac_qxt, ac_qyt, ac_ppc, ac_qzc, ac_kc;        // ACOUSTIC P
   CUtensorMap el_sxxt, el_sxyt, el_sxzt, el_syyt, el_syzt, el_vc[3], el_bc[3];  // ELASTIC V
   CUtensorMap el_vt[3], el_sc[6], el_cc[5];                             // ELASTIC S
   int cur = 0;               // ISO: fld[cur] = u^n
@@ -174,6 +190,12 @@ struct seis_model {
   size_t stage_elems = 0;
   const float* hwav = nullptr;  // host wavelet of the current call
   int last_nt = 0;
+  // shot-table cache and the CUDA graph of the last forward_model (single process)
+  uint64_t shot_key = 0;
+  cudaStream_t cap = nullptr;       // capture stream (the legacy stream cannot be captured)
+  cudaGraphExec_t gexec = nullptr;
+  uint64_t gkey = 0;
+  long long g_launches = 0;
 };
 
 namespace {
@@ -200,6 +222,12 @@ seis_status alloc_padded(seis_model* M, const Dims& d, float** out, cudaStream_t
 }
 
 int roundup(int a, int b) { return (a + b - 1) / b * b; }
+
+uint64_t fnv1a(const void* p, size_t n, uint64_t h = 1469598103934665603ULL) {
+  const unsigned char* c = static_cast<const unsigned char*>(p);
+  for (size_t i = 0; i < n; ++i) h = (h ^ c[i]) * 1099511628211ULL;
+  return h;
+}
 
 // cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda link).
 PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
@@ -231,7 +259,7 @@ Dims make_dims(const seis_grid& g, int z0, int nzl) {
   d.nz = g.nz;
   d.z0 = z0;
   d.PX = roundup(roundup(g.nx, TXV) + 2 * G, 32);
-  d.PY = roundup(g.ny, BY) + 2 * G;
+  d.PY = roundup(g.ny, 32) + 2 * G;  // any tile height up to 32
   d.PS = (long long)d.PX * d.PY;
   return d;
 }
@@ -297,13 +325,13 @@ seis_status set_smem_attrs() {
   static bool done = false;
   if (done) return SEIS_OK;
 #define SMEM_ATTR(fn, bytes) CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(bytes)))
-  SMEM_ATTR((iso_step_kernel<BY, false, false>), IsoStage<BY>::smem_bytes());
-  SMEM_ATTR((iso_step_kernel<BY, true, false>), IsoStage<BY>::smem_bytes());
-  SMEM_ATTR((iso_step_kernel<BY, false, true>), IsoStage<BY>::smem_bytes());
-  SMEM_ATTR((ac_v_kernel<BY, false>), AcVStage<BY>::smem_bytes());
-  SMEM_ATTR((ac_v_kernel<BY, true>), AcVStage<BY>::smem_bytes());
-  SMEM_ATTR((ac_p_kernel<BY, false>), AcPStage<BY>::smem_bytes());
-  SMEM_ATTR((ac_p_kernel<BY, true>), AcPStage<BY>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, false, false>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, true, false>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, false, true>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((ac_v_kernel<BYV, false>), AcVStage<BYV>::smem_bytes());
+  SMEM_ATTR((ac_v_kernel<BYV, true>), AcVStage<BYV>::smem_bytes());
+  SMEM_ATTR((ac_p_kernel<BYP, false>), AcPStage<BYP>::smem_bytes());
+  SMEM_ATTR((ac_p_kernel<BYP, true>), AcPStage<BYP>::smem_bytes());
   SMEM_ATTR((el_v_kernel<BYE>), ElVStage<BYE>::smem_bytes());
   SMEM_ATTR((el_s_kernel<BYE, false>), ElSStage<BYE>::smem_bytes());
 #undef SMEM_ATTR
@@ -312,13 +340,13 @@ seis_status set_smem_attrs() {
 }
 
 // Choose the z-chunk: enough blocks for >= 6 waves of the resident
-// slots (dynamic block scheduling keeps the tail short), chunks of >= 32 planes so
-// the 8-plane queue warm-up stays small.
+// slots (dynamic block scheduling keeps the tail short), chunks of >= 8 planes so
+// the 8-plane queue warm-up stays bounded (large grids stop at the wave rule first).
 void choose_chunks(Slab& s, int resident_per_sm, int nsm, int tw, int by) {
   const long long bxy = (long long)((s.d.nx + tw - 1) / tw) * ((s.d.ny + by - 1) / by);
   const long long slots = (long long)std::max(1, resident_per_sm) * nsm;
   int c = 1;
-  while (bxy * c < 6 * slots && (s.d.nzl + c) / (c + 1) >= 32) ++c;
+  while (bxy * c < 6 * slots && (s.d.nzl + c) / (c + 1) >= 8) ++c;
   s.zc = (s.d.nzl + c - 1) / c;
   s.nzch = (s.d.nzl + s.zc - 1) / s.zc;
 }
@@ -483,6 +511,8 @@ static seis_status validate_grid(const seis_grid* g, seis_kind kind) {
 seis_status seis_model_destroy(seis_model* M) {
   if (!M) return SEIS_OK;
   cudaSetDevice(M->device);
+  if (M->gexec) cudaGraphExecDestroy(M->gexec);
+  if (M->cap) cudaStreamDestroy(M->cap);
   for (void* p : M->allocs) cudaFree(p);
   delete M;
   return SEIS_OK;
@@ -728,48 +758,52 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     // TMA descriptors
     if (kind == SEIS_ISO) {
       for (int t = 0; t < 2; ++t) {
-        TRY(make_map(&S.iso_ut[t], S.fld[t], d, TXV + 8, BY + 8));
-        TRY(make_map(&S.iso_uc[t], S.fld[t], d, TXV, BY));
+        TRY(make_map(&S.iso_ut[t], S.fld[t], d, TXV + 8, BYI + 8));
+        TRY(make_map(&S.iso_uc[t], S.fld[t], d, TXV, BYI));
       }
-      TRY(make_map(&S.iso_m, S.m, d, TXV, BY));
+      TRY(make_map(&S.iso_m, S.m, d, TXV, BYI));
     } else if (kind == SEIS_ACOUSTIC) {
-      TRY(make_map(&S.ac_pt, S.fld[0], d, TXV + 8, BY + 8));
-      for (int t = 0; t < 3; ++t) TRY(make_map(&S.ac_qc[t], S.fld[1 + t], d, TXV, BY));
-      TRY(make_map(&S.ac_rt, S.rho, d, TXV + 4, BY + 1));
-      TRY(make_map(&S.ac_rc, S.rho, d, TXV, BY));
-      TRY(make_map(&S.ac_qxt, S.fld[1], d, TXV + 8, BY));
-      TRY(make_map(&S.ac_qyt, S.fld[2], d, TXV, BY + 8));
-      TRY(make_map(&S.ac_pc, S.fld[0], d, TXV, BY));
-      TRY(make_map(&S.ac_kc, S.kdt, d, TXV, BY));
+      // V tiles (BYV rows)
+      TRY(make_map(&S.ac_pt, S.fld[0], d, TXV + 8, BYV + 8));
+      for (int t = 0; t < 3; ++t) TRY(make_map(&S.ac_qc[t], S.fld[1 + t], d, TXV, BYV));
+      TRY(make_map(&S.ac_rt, S.rho, d, TXV + 4, BYV + 1));
+      TRY(make_map(&S.ac_rc, S.rho, d, TXV, BYV));
+      TRY(make_map(&S.ac_pc, S.fld[0], d, TXV, BYV));
+      // P tiles (BYP rows)
+      TRY(make_map(&S.ac_qxt, S.fld[1], d, TXV + 8, BYP));
+      TRY(make_map(&S.ac_qyt, S.fld[2], d, TXV, BYP + 8));
+      TRY(make_map(&S.ac_ppc, S.fld[0], d, TXV, BYP));
+      TRY(make_map(&S.ac_qzc, S.fld[3], d, TXV, BYP));
+      TRY(make_map(&S.ac_kc, S.kdt, d, TXV, BYP));
     } else {
-      TRY(make_map(&S.el_sxxt, S.fld[ESXX], d, TXW + 8, BYE));
-      TRY(make_map(&S.el_sxyt, S.fld[ESXY], d, TXW + 8, BYE + 8));
-      TRY(make_map(&S.el_sxzt, S.fld[ESXZ], d, TXW + 8, BYE));
-      TRY(make_map(&S.el_syyt, S.fld[ESYY], d, TXW, BYE + 8));
-      TRY(make_map(&S.el_syzt, S.fld[ESYZ], d, TXW, BYE + 8));
+      TRY(make_map(&S.el_sxxt, S.fld[ESXX], d, TXV + 8, BYE));
+      TRY(make_map(&S.el_sxyt, S.fld[ESXY], d, TXV + 8, BYE + 8));
+      TRY(make_map(&S.el_sxzt, S.fld[ESXZ], d, TXV + 8, BYE));
+      TRY(make_map(&S.el_syyt, S.fld[ESYY], d, TXV, BYE + 8));
+      TRY(make_map(&S.el_syzt, S.fld[ESYZ], d, TXV, BYE + 8));
       float* bb[3] = {S.bx, S.by, S.bz};
       for (int t = 0; t < 3; ++t) {
-        TRY(make_map(&S.el_vc[t], S.fld[EVX + t], d, TXW, BYE));
-        TRY(make_map(&S.el_bc[t], bb[t], d, TXW, BYE));
-        TRY(make_map(&S.el_vt[t], S.fld[EVX + t], d, TXW + 8, BYE + 8));
+        TRY(make_map(&S.el_vc[t], S.fld[EVX + t], d, TXV, BYE));
+        TRY(make_map(&S.el_bc[t], bb[t], d, TXV, BYE));
+        TRY(make_map(&S.el_vt[t], S.fld[EVX + t], d, TXV + 8, BYE + 8));
       }
-      for (int t = 0; t < 6; ++t) TRY(make_map(&S.el_sc[t], S.fld[ESXX + t], d, TXW, BYE));
+      for (int t = 0; t < 6; ++t) TRY(make_map(&S.el_sc[t], S.fld[ESXX + t], d, TXV, BYE));
       float* cc[5] = {S.l2m, S.lam, S.mxy, S.mxz, S.myz};
-      for (int t = 0; t < 5; ++t) TRY(make_map(&S.el_cc[t], cc[t], d, TXW, BYE));
+      for (int t = 0; t < 5; ++t) TRY(make_map(&S.el_cc[t], cc[t], d, TXV, BYE));
     }
     TRY(set_smem_attrs());
     int occ = 1;
     if (kind == SEIS_ISO)
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, iso_step_kernel<BY, false, false>, NTX * BY,
-                                                    IsoStage<BY>::smem_bytes());
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, iso_step_kernel<BYI, false, false>, NTX * BYI,
+                                                    IsoStage<BYI>::smem_bytes());
     else if (kind == SEIS_ACOUSTIC)
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_v_kernel<BY, false>, NTX * BY,
-                                                    AcVStage<BY>::smem_bytes());
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_v_kernel<BYV, false>, NTX * BYV,
+                                                    AcVStage<BYV>::smem_bytes());
     else
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, TXW * BYE,
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, NTX2 * BYE,
                                                     ElSStage<BYE>::smem_bytes());
-    if (kind == SEIS_ELASTIC) choose_chunks(S, occ, dev_sms, TXW, BYE);
-    else choose_chunks(S, occ, dev_sms, TXV, BY);
+    if (kind == SEIS_ELASTIC) choose_chunks(S, occ, dev_sms, TXV, BYE);
+    else choose_chunks(S, occ, dev_sms, TXV, kind == SEIS_ISO ? BYI : BYV);
   }
   if (kind == SEIS_ACOUSTIC)  // rho(k+1) across slab faces
     TRY(exchange_arrays(M, {[](Slab& S) { return S.rho; }}, 4, st));
@@ -874,6 +908,13 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
   if (M->kind == SEIS_ELASTIC && (sh->rec_component < 0 || sh->rec_component > 3))
     return fail(SEIS_EINVAL, "rec_component must be 0..3");
   M->hwav = sh->wavelet;  // source amplitudes are kernel arguments (one fused add per step)
+  // receiver tables are rebuilt only when the geometry changes (CUDA graphs keep pointers)
+  uint64_t key = fnv1a(&sh->sx, 3 * sizeof(int32_t));
+  key = fnv1a(&sh->nrec, sizeof(int32_t), key);
+  if (sh->nrec) key = fnv1a(sh->rec, (size_t)sh->nrec * 3 * sizeof(int32_t), key);
+  key = fnv1a(&sh->rec_component, sizeof(int32_t), key);
+  key ^= backward_injection ? 0x9e3779b97f4a7c15ULL : 0;
+  const bool same = key == M->shot_key;
   const double h = g.h, dt = g.dt;
   auto point_scale = [&](int x, int y, int z) -> double {
     const size_t li = ((size_t)(z - M->pz0) * g.ny + y) * g.nx + x;
@@ -896,6 +937,7 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
       S.src_o = S.d.at(sh->sx, sh->sy, sh->sz - z0);
       S.src_scale = (float)point_scale(sh->sx, sh->sy, sh->sz);
     }
+    if (same) continue;
     // receivers owned by this slab
     std::vector<long long> off;
     std::vector<int> rid;
@@ -942,6 +984,7 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
       CK(cudaMemcpy(S.d_g_mem, gmem.data(), gmem.size() * sizeof(int), cudaMemcpyHostToDevice));
     }
   }
+  M->shot_key = key;
   return SEIS_OK;
 }
 
@@ -986,7 +1029,7 @@ seis_status fs_mirror(seis_model* M, std::initializer_list<int> fields, cudaStre
 }
 
 // ISO / ACOUSTIC: 64 x BY tiles of (16, BY) threads; ELASTIC: 32 x BYE tiles of (32, BYE)
-dim3 grid_of(const Slab& S, int tw = TXV, int by = BY) {
+dim3 grid_of(const Slab& S, int tw, int by) {
   return dim3((S.d.nx + tw - 1) / tw, (S.d.ny + by - 1) / by, S.nzch);
 }
 
@@ -1010,7 +1053,6 @@ seis_status inject_rows(seis_model* M, const float* row, cudaStream_t st) {
 seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
                  std::vector<const float*>* imgS, std::vector<float*>* img, cudaStream_t st,
                  const float* inj_row = nullptr) {
-  const dim3 blk(NTX, BY);
   if (M->kind == SEIS_ISO) {
     for (size_t s = 0; s < M->slabs.size(); ++s) {
       Slab& S = M->slabs[s];
@@ -1032,13 +1074,13 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.snap = snap ? (*snap)[s] : nullptr;
       a.imgS = imgS ? (*imgS)[s] : nullptr;
       a.img = img ? (*img)[s] : nullptr;
-      const dim3 gr = grid_of(S);
+      const dim3 gr = grid_of(S, TXV, BYI), blk(NTX, BYI);
       {
         PROF(0, st);
-        const size_t sb = IsoStage<BY>::smem_bytes();
-        if (a.snap) iso_step_kernel<BY, true, false><<<gr, blk, sb, st>>>(a);
-        else if (a.img) iso_step_kernel<BY, false, true><<<gr, blk, sb, st>>>(a);
-        else iso_step_kernel<BY, false, false><<<gr, blk, sb, st>>>(a);
+        const size_t sb = IsoStage<BYI>::smem_bytes();
+        if (a.snap) iso_step_kernel<BYI, true, false><<<gr, blk, sb, st>>>(a);
+        else if (a.img) iso_step_kernel<BYI, false, true><<<gr, blk, sb, st>>>(a);
+        else iso_step_kernel<BYI, false, false><<<gr, blk, sb, st>>>(a);
       }
       CKL();
     }
@@ -1078,12 +1120,12 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.zc = S.zc;
       a.imgS = imgS ? (*imgS)[s] : nullptr;
       a.img = img ? (*img)[s] : nullptr;
-      const dim3 gr = grid_of(S);
+      const dim3 gr = grid_of(S, TXV, BYV), blk(NTX, BYV);
       {
         PROF(1, st);
-        const size_t sb = AcVStage<BY>::smem_bytes();
-        if (a.img) ac_v_kernel<BY, true><<<gr, blk, sb, st>>>(a);
-        else ac_v_kernel<BY, false><<<gr, blk, sb, st>>>(a);
+        const size_t sb = AcVStage<BYV>::smem_bytes();
+        if (a.img) ac_v_kernel<BYV, true><<<gr, blk, sb, st>>>(a);
+        else ac_v_kernel<BYV, false><<<gr, blk, sb, st>>>(a);
       }
       CKL();
     }
@@ -1093,9 +1135,9 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       AcPArgs a;
       a.mqx = S.ac_qxt;
       a.mqy = S.ac_qyt;
-      a.mpp = S.ac_pc;
+      a.mpp = S.ac_ppc;
       a.mk = S.ac_kc;
-      a.mqq = S.ac_qc[2];
+      a.mqq = S.ac_qzc;
       a.p = S.fld[0];
       a.qz = S.fld[3];
       a.W = M->W;
@@ -1112,12 +1154,12 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.src_amp = 0.f;
       if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
       a.snap = snap ? (*snap)[s] : nullptr;
-      const dim3 gr = grid_of(S);
+      const dim3 gr = grid_of(S, TXV, BYP), blk(NTX, BYP);
       {
         PROF(2, st);
-        const size_t sb = AcPStage<BY>::smem_bytes();
-        if (a.snap) ac_p_kernel<BY, true><<<gr, blk, sb, st>>>(a);
-        else ac_p_kernel<BY, false><<<gr, blk, sb, st>>>(a);
+        const size_t sb = AcPStage<BYP>::smem_bytes();
+        if (a.snap) ac_p_kernel<BYP, true><<<gr, blk, sb, st>>>(a);
+        else ac_p_kernel<BYP, false><<<gr, blk, sb, st>>>(a);
       }
       CKL();
     }
@@ -1138,6 +1180,9 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.mv[t] = S.el_vc[t];
       a.mb[t] = S.el_bc[t];
     }
+    a.mq[0] = S.el_sc[ESXZ - ESXX];
+    a.mq[1] = S.el_sc[ESYZ - ESXX];
+    a.mq[2] = S.el_sc[ESZZ - ESXX];
     for (int t = 0; t < 9; ++t) a.f[t] = S.fld[t];
     a.W = M->W;
     a.zlo = M->g.free_surface ? 0 : 1;
@@ -1148,10 +1193,10 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (int t = 0; t < 9; ++t) a.psi[t] = S.psi[t];
     a.d = S.d;
     a.zc = S.zc;
-    const dim3 gr = grid_of(S, TXW, BYE);
+    const dim3 gr = grid_of(S, TXV, BYE);
     {
       PROF(3, st);
-      el_v_kernel<BYE><<<gr, dim3(TXW, BYE), ElVStage<BYE>::smem_bytes(), st>>>(a);
+      el_v_kernel<BYE><<<gr, dim3(NTX2, BYE), ElVStage<BYE>::smem_bytes(), st>>>(a);
     }
     CKL();
   }
@@ -1163,6 +1208,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (int t = 0; t < 3; ++t) a.mvt[t] = S.el_vt[t];
     for (int t = 0; t < 6; ++t) a.ms[t] = S.el_sc[t];
     for (int t = 0; t < 5; ++t) a.mc[t] = S.el_cc[t];
+    for (int t = 0; t < 3; ++t) a.mq[t] = S.el_vc[t];
     for (int t = 0; t < 9; ++t) a.f[t] = S.fld[t];
     a.W = M->W;
     a.zlo = M->g.free_surface ? 0 : 1;
@@ -1176,10 +1222,10 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     a.src_o = with_src ? S.src_o : -1;
     a.src_amp = 0.f;
     if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
-    const dim3 gr = grid_of(S, TXW, BYE);
+    const dim3 gr = grid_of(S, TXV, BYE);
     {
       PROF(4, st);
-      el_s_kernel<BYE, false><<<gr, dim3(TXW, BYE), ElSStage<BYE>::smem_bytes(), st>>>(a);
+      el_s_kernel<BYE, false><<<gr, dim3(NTX2, BYE), ElSStage<BYE>::smem_bytes(), st>>>(a);
     }
     CKL();
   }
@@ -1224,6 +1270,19 @@ seis_status ensure_stage(seis_model* M, size_t elems) {
 
 extern "C" {
 
+// The time loop of one modeling shot (everything between the zeroed state and the
+// filled seismogram), issued on `st`.
+static seis_status forward_loop(seis_model* M, const seis_shot* sh, float* sd, size_t ns, cudaStream_t st) {
+  TRY(zero_state(M, st));
+  if (ns) CK(cudaMemsetAsync(sd, 0, ns * sizeof(float), st));
+  for (int n = 0; n < sh->nt; ++n) {
+    TRY(step(M, n, true, nullptr, nullptr, nullptr, st));
+    if (sh->nrec) TRY(gather(M, sh, sd, n, st));
+  }
+  if (M->comm && M->nranks > 1 && ns) NK(ncclAllReduce(sd, sd, ns, ncclFloat, ncclSum, M->comm->nccl, st));
+  return SEIS_OK;
+}
+
 seis_status seis_forward_model(seis_model* M, const seis_shot* sh, float* seis, void* stream) {
   g_launches = 0;
   if (!M) return fail(SEIS_EINVAL, "null model");
@@ -1231,7 +1290,6 @@ seis_status seis_forward_model(seis_model* M, const seis_shot* sh, float* seis, 
   CK(cudaSetDevice(M->device));
   cudaStream_t st = (cudaStream_t)stream;
   TRY(setup_shot(M, sh, false, st));
-  TRY(zero_state(M, st));
   const size_t ns = (size_t)sh->nt * sh->nrec;
   const bool dev = ns == 0 || is_device_ptr(seis);
   float* sd = seis;
@@ -1239,12 +1297,43 @@ seis_status seis_forward_model(seis_model* M, const seis_shot* sh, float* seis, 
     TRY(ensure_stage(M, ns));
     sd = M->stage;
   }
-  if (ns) CK(cudaMemsetAsync(sd, 0, ns * sizeof(float), st));
-  for (int n = 0; n < sh->nt; ++n) {
-    TRY(step(M, n, true, nullptr, nullptr, nullptr, st));
-    if (sh->nrec) TRY(gather(M, sh, sd, n, st));
+  // Single process: the whole shot is one CUDA graph (captured once per shot setup and
+  // output buffer, replayed afterwards), so small grids are not launch-bound.
+  const bool use_graph = !prof::on && !(M->comm && M->nranks > 1) && !getenv("SEIS_NO_GRAPH");
+  if (use_graph) {
+    uint64_t key = fnv1a(sh->wavelet, (size_t)sh->nt * sizeof(float), M->shot_key);
+    key = fnv1a(&sd, sizeof(sd), key);
+    key = fnv1a(&sh->nt, sizeof(int32_t), key);
+    if (!M->gexec || M->gkey != key) {
+      if (M->gexec) {
+        cudaGraphExecDestroy(M->gexec);
+        M->gexec = nullptr;
+      }
+      if (!M->cap) CK(cudaStreamCreateWithFlags(&M->cap, cudaStreamNonBlocking));
+      CK(cudaStreamSynchronize(st));
+      CK(cudaStreamBeginCapture(M->cap, cudaStreamCaptureModeThreadLocal));
+      seis_status rc = forward_loop(M, sh, sd, ns, M->cap);
+      cudaGraph_t graph = nullptr;
+      cudaError_t e = cudaStreamEndCapture(M->cap, &graph);
+      if (rc != SEIS_OK) {
+        if (graph) cudaGraphDestroy(graph);
+        return rc;
+      }
+      if (e != cudaSuccess) return fail(SEIS_ECUDA, "graph capture: %s", cudaGetErrorString(e));
+      e = cudaGraphInstantiate(&M->gexec, graph, 0);
+      cudaGraphDestroy(graph);
+      if (e != cudaSuccess) {
+        M->gexec = nullptr;
+        return fail(SEIS_ECUDA, "graph instantiate: %s", cudaGetErrorString(e));
+      }
+      M->gkey = key;
+      M->g_launches = g_launches;
+    }
+    CK(cudaGraphLaunch(M->gexec, st));
+    g_launches = M->g_launches;
+  } else {
+    TRY(forward_loop(M, sh, sd, ns, st));
   }
-  if (M->comm && M->nranks > 1 && ns) NK(ncclAllReduce(sd, sd, ns, ncclFloat, ncclSum, M->comm->nccl, st));
   if (!dev && ns) CK(cudaMemcpyAsync(seis, sd, ns * sizeof(float), cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
   M->last_nt = sh->nt;

@@ -1,0 +1,58 @@
+"""Tile / ring-depth tuning sweep of the stencil kernels (not part of the product path).
+
+    python tools/sweep.py build          # here: compile the variants into sweep_out/*.so
+    python tools/sweep.py run            # on a B200 (gpurun): time every variant
+
+Each variant is the same libseis source compiled with different -D macros
+(SEIS_BY, SEIS_BYE and the TMA ring depths); the runner loads it through
+SEIS_LIBPATH in a fresh process and reports the per-kernel CUDA-event times of
+short ISO 512^3, acoustic C2 512^3 and elastic C3 384^3 runs.
+"""
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+OUT = os.path.join(ROOT, "sweep_out")
+sys.path.insert(0, ROOT)
+
+VARIANTS = {
+    "base": [],
+    "i4": ["SEIS_BYI=4", "SEIS_ISO_NS=6"],
+    "i8ns3": ["SEIS_ISO_NS=3"],
+    "i8ns6": ["SEIS_ISO_NS=6"],
+    "v8": ["SEIS_BYV=8", "SEIS_AC_VNS=3"],
+    "v8ns4": ["SEIS_BYV=8", "SEIS_AC_VNS=4"],
+    "v16ns2": ["SEIS_AC_VNS=2"],
+    "p8": ["SEIS_BYP=8", "SEIS_AC_NS=2"],
+    "p8ns3": ["SEIS_BYP=8", "SEIS_AC_NS=3"],
+    "p16ns3": ["SEIS_AC_NS=3"],
+    "e22": ["SEIS_EL_VNS=2", "SEIS_EL_SNS=2"],
+    "e4_32": ["SEIS_BYE=4", "SEIS_EL_VNS=3", "SEIS_EL_SNS=2"],
+}
+
+
+def build():
+    from paper_conf_ppopp_qawasmehchc15_b200 import build as b
+
+    os.makedirs(OUT, exist_ok=True)
+    for name, defs in VARIANTS.items():
+        path = os.path.join(OUT, f"libseis_{name}.so")
+        b.build(force=True, defines=defs, out=path)
+        print("built", path)
+
+
+def run():
+    for name in VARIANTS:
+        path = os.path.join(OUT, f"libseis_{name}.so")
+        env = dict(os.environ, SEIS_LIBPATH=path)
+        r = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "sweep_one.py"), name],
+                           env=env, capture_output=True, text=True, timeout=900)
+        line = r.stdout.strip().splitlines()[-1] if r.stdout.strip() else json.dumps(
+            {"variant": name, "error": r.stderr[-500:]})
+        print(line, flush=True)
+
+
+if __name__ == "__main__":
+    {"build": build, "run": run}[sys.argv[1]]()
