@@ -142,8 +142,12 @@ __device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, u
 // a block tile is TXV = 64 points wide (16 threads) x BY rows.
 namespace seis {
 
-constexpr int TXV = 64;  // tile width in x (points)
-constexpr int NTX = 16;  // threads in x per block
+#ifndef SEIS_TXV
+#define SEIS_TXV 64
+#endif
+constexpr int TXV = SEIS_TXV;  // ISO / acoustic tile width in x (points)
+constexpr int NTX = TXV / 4;   // threads in x per block (4 points each)
+constexpr int TXE = 64;        // elastic tile width in x (32 threads, 2 points each)
 
 struct F4 {
   float v[4];
@@ -198,4 +202,46 @@ __device__ __forceinline__ void st2_masked(float* p, const F2& a, int x0, int nx
     p[0] = a.v[0];
   }
 }
+}  // namespace seis
+
+// ------------------------------------------------ C-PML memory-variable access
+// psi values are first-touch global data inside the layers; the kernels load the old
+// values BEFORE waiting for the plane's TMA stage (so their latency overlaps the wait
+// and the derivative arithmetic) and store the updated values afterwards.
+namespace seis {
+
+// compact-slab indices of the NV points of a group (or -1 outside the layer / grid)
+template <int NV>
+__device__ __forceinline__ void psi_idx_x(long long* ix, const Dims& d, int W, int x0, int j, int k) {
+#pragma unroll
+  for (int e = 0; e < NV; ++e) {
+    const int x = x0 + e;
+    ix[e] = (x < d.nx && CpmlIdx::in(x, d.nx, W, true))
+                ? ((long long)k * d.ny + j) * (2 * W) + CpmlIdx::slot(x, d.nx, W)
+                : -1;
+  }
+}
+template <int NV>
+__device__ __forceinline__ void psi_idx_row(long long* ix, long long base, int x0, int nx) {
+#pragma unroll
+  for (int e = 0; e < NV; ++e) ix[e] = (x0 + e < nx) ? base + e : -1;
+}
+template <int NV>
+__device__ __forceinline__ void psi_ld(float* old, const float* __restrict__ ps, const long long* ix) {
+#pragma unroll
+  for (int e = 0; e < NV; ++e) old[e] = ix[e] >= 0 ? ps[ix[e]] : 0.0f;
+}
+// psi <- b psi + a dv;  dv += psi   (per point coefficients ca[e], cb[e])
+template <int NV>
+__device__ __forceinline__ void psi_upd(float* dv, float* __restrict__ ps, const long long* ix, const float* old,
+                                        const float* ca, const float* cb) {
+#pragma unroll
+  for (int e = 0; e < NV; ++e)
+    if (ix[e] >= 0) {
+      const float v = fmaf(cb[e], old[e], ca[e] * dv[e]);
+      ps[ix[e]] = v;
+      dv[e] += v;
+    }
+}
+
 }  // namespace seis

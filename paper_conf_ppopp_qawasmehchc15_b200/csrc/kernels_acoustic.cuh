@@ -35,45 +35,6 @@ struct CpmlAxis {
 constexpr int AC_NS = SEIS_AC_NS;    // P kernel ring depth
 constexpr int AC_VNS = SEIS_AC_VNS;  // V kernel ring depth
 
-// psi update of the 4 x-points of a group that lie inside an x layer
-__device__ __forceinline__ void cpml_x4(float* dv, float* __restrict__ ps, const Dims& d, int W, int x0,
-                                        int j, int k, const float* __restrict__ ca,
-                                        const float* __restrict__ cb) {
-#pragma unroll
-  for (int e = 0; e < 4; ++e) {
-    const int x = x0 + e;
-    if (x < d.nx && CpmlIdx::in(x, d.nx, W, true)) {
-      const long long ix = ((long long)k * d.ny + j) * (2 * W) + CpmlIdx::slot(x, d.nx, W);
-      const float v = fmaf(__ldg(cb + x), ps[ix], __ldg(ca + x) * dv[e]);
-      ps[ix] = v;
-      dv[e] += v;
-    }
-  }
-}
-// psi update of a group inside a y layer (row j) or a z layer (global plane gz)
-__device__ __forceinline__ void cpml_y4(float* dv, float* __restrict__ ps, const Dims& d, int W, int x0,
-                                        int j, int k, float ca, float cb) {
-  const long long iy = ((long long)k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0;
-#pragma unroll
-  for (int e = 0; e < 4; ++e)
-    if (x0 + e < d.nx) {
-      const float v = fmaf(cb, ps[iy + e], ca * dv[e]);
-      ps[iy + e] = v;
-      dv[e] += v;
-    }
-}
-__device__ __forceinline__ void cpml_z4(float* dv, float* __restrict__ ps, const Dims& d, int W, int x0,
-                                        int j, int gz, float ca, float cb) {
-  const long long iz = ((long long)CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0;
-#pragma unroll
-  for (int e = 0; e < 4; ++e)
-    if (x0 + e < d.nx) {
-      const float v = fmaf(cb, ps[iz + e], ca * dv[e]);
-      ps[iz + e] = v;
-      dv[e] += v;
-    }
-}
-
 struct AcVArgs {
   CUtensorMap mp;                 // p tile, box (64+8) x (BY+8) x 1
   CUtensorMap mqx, mqy, mqz;      // q, box 64 x BY x 1
@@ -157,6 +118,23 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
     const int k = k0 + it;
     const int s = it % AC_VNS;
     const long long o = (long long)(k + GZ) * PS + oc;
+    // C-PML: old psi values are loaded before the wait (latency overlap)
+    const int gz = k + d.z0;
+    const bool lz = Wl > 0 && CpmlIdx::in(gz, d.nz, Wl, a.zlo);
+    long long ixx[4], iyy[4], izz[4];
+    float ox[4], oy[4], oz[4];
+    if (own && lx) {
+      psi_idx_x<4>(ixx, d, Wl, x0, j, k);
+      psi_ld<4>(ox, a.psx, ixx);
+    }
+    if (own && ly) {
+      psi_idx_row<4>(iyy, ((long long)k * (2 * Wl) + CpmlIdx::slot(j, d.ny, Wl)) * d.nx + x0, x0, d.nx);
+      psi_ld<4>(oy, a.psy, iyy);
+    }
+    if (own && lz) {
+      psi_idx_row<4>(izz, ((long long)CpmlIdx::slot(gz, d.nz, Wl) * d.ny + j) * d.nx + x0, x0, d.nx);
+      psi_ld<4>(oz, a.psz, izz);
+    }
     mbar_wait(&bar[s], (it / AC_VNS) & 1);
     const float* st = sm + s * L::SIZE;
     r[7] = lds4(st + L::PQ + ty * TXV + 4 * tx);
@@ -192,12 +170,25 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
       dz[e] = fmaf(SEIS_D4, r[7].v[e] - r[0].v[e], t);
     }
     if (own) {
-      if (Wl > 0) {
-        if (lx) cpml_x4(dx, a.psx, d, Wl, x0, j, k, a.cx.ah, a.cx.bh);
-        if (ly) cpml_y4(dy, a.psy, d, Wl, x0, j, k, __ldg(a.cy.ah + j), __ldg(a.cy.bh + j));
-        const int gz = k + d.z0;
-        if (CpmlIdx::in(gz, d.nz, Wl, a.zlo))
-          cpml_z4(dz, a.psz, d, Wl, x0, j, gz, __ldg(a.cz.ah + gz), __ldg(a.cz.bh + gz));
+      if (lx) {
+        float ca[4], cb[4];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const int x = min(x0 + e, d.nx - 1);
+          ca[e] = __ldg(a.cx.ah + x);
+          cb[e] = __ldg(a.cx.bh + x);
+        }
+        psi_upd<4>(dx, a.psx, ixx, ox, ca, cb);
+      }
+      if (ly) {
+        const float ya = __ldg(a.cy.ah + j), yb = __ldg(a.cy.bh + j);
+        const float ca[4] = {ya, ya, ya, ya}, cb[4] = {yb, yb, yb, yb};
+        psi_upd<4>(dy, a.psy, iyy, oy, ca, cb);
+      }
+      if (lz) {
+        const float za = __ldg(a.cz.ah + gz), zb = __ldg(a.cz.bh + gz);
+        const float ca[4] = {za, za, za, za}, cb[4] = {zb, zb, zb, zb};
+        psi_upd<4>(dz, a.psz, izz, oz, ca, cb);
       }
       const int pt = ty * TXV + 4 * tx;
       const F4 qxo = lds4(st + L::QX + pt), qyo = lds4(st + L::QY + pt), qzo = lds4(st + L::QZ + pt);
@@ -205,7 +196,7 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
       const float* rc = st + L::R + ty * RW + 4 * tx;
       const F4 r0 = lds4(rc), rxn = lds4(rc + 4), ryn = lds4(rc + RW);
       const float rx5 = rxn.v[0];
-      const bool zlast = k + d.z0 + 1 >= d.nz;
+      const bool zlast = gz + 1 >= d.nz;
       F4 ox, oy, oz;
 #pragma unroll
       for (int e = 0; e < 4; ++e) {
@@ -317,6 +308,23 @@ __global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ 
     const int k = k0 + it;
     const int s = it % AC_NS;
     const long long o = (long long)(k + GZ) * PS + oc;
+    // C-PML: old psi values are loaded before the wait (latency overlap)
+    const int gz = k + d.z0;
+    const bool lz = Wl > 0 && CpmlIdx::in(gz, d.nz, Wl, a.zlo);
+    long long ixx[4], iyy[4], izz[4];
+    float ox[4], oy[4], oz[4];
+    if (own && lx) {
+      psi_idx_x<4>(ixx, d, Wl, x0, j, k);
+      psi_ld<4>(ox, a.pqx, ixx);
+    }
+    if (own && ly) {
+      psi_idx_row<4>(iyy, ((long long)k * (2 * Wl) + CpmlIdx::slot(j, d.ny, Wl)) * d.nx + x0, x0, d.nx);
+      psi_ld<4>(oy, a.pqy, iyy);
+    }
+    if (own && lz) {
+      psi_idx_row<4>(izz, ((long long)CpmlIdx::slot(gz, d.nz, Wl) * d.ny + j) * d.nx + x0, x0, d.nx);
+      psi_ld<4>(oz, a.pqz, izz);
+    }
     mbar_wait(&bar[s], (it / AC_NS) & 1);
     const float* st = sm + s * L::SIZE;
     q[7] = lds4(st + L::QQ + ty * TXV + 4 * tx);
@@ -352,12 +360,25 @@ __global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ 
       dz[e] = fmaf(SEIS_D4, q[7].v[e] - q[0].v[e], t);
     }
     if (own) {
-      if (Wl > 0) {
-        if (lx) cpml_x4(dx, a.pqx, d, Wl, x0, j, k, a.cx.a, a.cx.b);
-        if (ly) cpml_y4(dy, a.pqy, d, Wl, x0, j, k, __ldg(a.cy.a + j), __ldg(a.cy.b + j));
-        const int gz = k + d.z0;
-        if (CpmlIdx::in(gz, d.nz, Wl, a.zlo))
-          cpml_z4(dz, a.pqz, d, Wl, x0, j, gz, __ldg(a.cz.a + gz), __ldg(a.cz.b + gz));
+      if (lx) {
+        float ca[4], cb[4];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const int x = min(x0 + e, d.nx - 1);
+          ca[e] = __ldg(a.cx.a + x);
+          cb[e] = __ldg(a.cx.b + x);
+        }
+        psi_upd<4>(dx, a.pqx, ixx, ox, ca, cb);
+      }
+      if (ly) {
+        const float ya = __ldg(a.cy.a + j), yb = __ldg(a.cy.b + j);
+        const float ca[4] = {ya, ya, ya, ya}, cb[4] = {yb, yb, yb, yb};
+        psi_upd<4>(dy, a.pqy, iyy, oy, ca, cb);
+      }
+      if (lz) {
+        const float za = __ldg(a.cz.a + gz), zb = __ldg(a.cz.b + gz);
+        const float ca[4] = {za, za, za, za}, cb[4] = {zb, zb, zb, zb};
+        psi_upd<4>(dz, a.pqz, izz, oz, ca, cb);
       }
       const int pt = ty * TXV + 4 * tx;
       const F4 pv = lds4(st + L::P + pt), kv = lds4(st + L::K + pt);

@@ -31,44 +31,6 @@ namespace seis {
 
 enum { EVX, EVY, EVZ, ESXX, ESYY, ESZZ, ESXY, ESXZ, ESYZ };
 
-// psi updates of the 2 x-points of a group (x layer: per point; y, z layers: per row/plane)
-__device__ __forceinline__ void cpml2_x(float* dv, float* __restrict__ ps, const Dims& d, int W, int x0,
-                                        int j, int k, const float* __restrict__ ca,
-                                        const float* __restrict__ cb) {
-#pragma unroll
-  for (int e = 0; e < 2; ++e) {
-    const int x = x0 + e;
-    if (x < d.nx && CpmlIdx::in(x, d.nx, W, true)) {
-      const long long ix = ((long long)k * d.ny + j) * (2 * W) + CpmlIdx::slot(x, d.nx, W);
-      const float v = fmaf(__ldg(cb + x), ps[ix], __ldg(ca + x) * dv[e]);
-      ps[ix] = v;
-      dv[e] += v;
-    }
-  }
-}
-__device__ __forceinline__ void cpml2_y(float* dv, float* __restrict__ ps, const Dims& d, int W, int x0,
-                                        int j, int k, float ca, float cb) {
-  const long long iy = ((long long)k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0;
-#pragma unroll
-  for (int e = 0; e < 2; ++e)
-    if (x0 + e < d.nx) {
-      const float v = fmaf(cb, ps[iy + e], ca * dv[e]);
-      ps[iy + e] = v;
-      dv[e] += v;
-    }
-}
-__device__ __forceinline__ void cpml2_z(float* dv, float* __restrict__ ps, const Dims& d, int W, int x0,
-                                        int j, int gz, float ca, float cb) {
-  const long long iz = ((long long)CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0;
-#pragma unroll
-  for (int e = 0; e < 2; ++e)
-    if (x0 + e < d.nx) {
-      const float v = fmaf(cb, ps[iz + e], ca * dv[e]);
-      ps[iz + e] = v;
-      dv[e] += v;
-    }
-}
-
 // staggered differences, times h, along a line of values v (index c = the point)
 __device__ __forceinline__ float dp(const float* v, int c) {  // D+ at c+1/2 from integer field
   float r = SEIS_D1 * (v[c + 1] - v[c]);
@@ -130,15 +92,15 @@ struct ElVArgs {
 
 template <int BY>
 struct ElVStage {
-  static constexpr int WX = TXV + 8, T = TXV * BY;
+  static constexpr int WX = TXE + 8, T = TXE * BY;
   static constexpr int XX = 0, XY = XX + BY * WX, XZ = XY + (BY + 8) * WX, YY = XZ + BY * WX,
-                       YZ = YY + (BY + 8) * TXV, V = YZ + (BY + 8) * TXV, B = V + 3 * T, Q = B + 3 * T,
+                       YZ = YY + (BY + 8) * TXE, V = YZ + (BY + 8) * TXE, B = V + 3 * T, Q = B + 3 * T,
                        SIZE = Q + 3 * T;
   static constexpr size_t smem_bytes() { return (size_t)EL_VNS * SIZE * 4 + 128; }
 };
 
 template <int BY>
-__global__ void __launch_bounds__(NTX2 * BY) el_v_kernel(const __grid_constant__ ElVArgs a) {
+__global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constant__ ElVArgs a) {
   using L = ElVStage<BY>;
   constexpr int WX = L::WX, T = L::T;
   constexpr uint32_t TX_BYTES = L::SIZE * 4;
@@ -149,7 +111,7 @@ __global__ void __launch_bounds__(NTX2 * BY) el_v_kernel(const __grid_constant__
   __shared__ __align__(8) uint64_t bar[EL_VNS];
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX2 + tx;
-  const int i0 = blockIdx.x * TXV, j0 = blockIdx.y * BY;
+  const int i0 = blockIdx.x * TXE, j0 = blockIdx.y * BY;
   const int x0 = i0 + 2 * tx, j = j0 + ty;
   const int k0 = blockIdx.z * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
@@ -199,9 +161,32 @@ __global__ void __launch_bounds__(NTX2 * BY) el_v_kernel(const __grid_constant__
     const int k = k0 + it;
     const int s = it % EL_VNS;
     const long long o = (long long)(k + GZ) * PS + oc;
+    // C-PML: old psi values are loaded before the wait (latency overlap)
+    const int gz = k + d.z0;
+    const bool lz = W > 0 && CpmlIdx::in(gz, d.nz, W, a.zlo);
+    long long ixx[2], iyy[2], izz[2];
+    float ox0[2], ox3[2], ox6[2], oy1[2], oy4[2], oy7[2], oz2[2], oz5[2], oz8[2];
+    if (own && lx) {
+      psi_idx_x<2>(ixx, d, W, x0, j, k);
+      psi_ld<2>(ox0, a.psi[0], ixx);
+      psi_ld<2>(ox3, a.psi[3], ixx);
+      psi_ld<2>(ox6, a.psi[6], ixx);
+    }
+    if (own && ly) {
+      psi_idx_row<2>(iyy, ((long long)k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0, x0, d.nx);
+      psi_ld<2>(oy1, a.psi[1], iyy);
+      psi_ld<2>(oy4, a.psi[4], iyy);
+      psi_ld<2>(oy7, a.psi[7], iyy);
+    }
+    if (own && lz) {
+      psi_idx_row<2>(izz, ((long long)CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0, x0, d.nx);
+      psi_ld<2>(oz2, a.psi[2], izz);
+      psi_ld<2>(oz5, a.psi[5], izz);
+      psi_ld<2>(oz8, a.psi[8], izz);
+    }
     mbar_wait(&bar[s], (it / EL_VNS) & 1);
     const float* st = sm + s * L::SIZE;
-    const int pt = ty * TXV + 2 * tx;
+    const int pt = ty * TXE + 2 * tx;
     qxz[7] = lds2(st + L::Q + pt);
     qyz[7] = lds2(st + L::Q + T + pt);
     qzz[7] = lds2(st + L::Q + 2 * T + pt);
@@ -211,8 +196,8 @@ __global__ void __launch_bounds__(NTX2 * BY) el_v_kernel(const __grid_constant__
       xrow(xy, st + L::XY + (ty + 4) * WX + 2 * tx + 4);
       xrow(xz, st + L::XZ + ty * WX + 2 * tx + 4);
       ycol<WX>(yxy, st + L::XY + (ty + 4) * WX + 2 * tx + 4);
-      ycol<TXV>(yyy, st + L::YY + (ty + 4) * TXV + 2 * tx);
-      ycol<TXV>(yyz, st + L::YZ + (ty + 4) * TXV + 2 * tx);
+      ycol<TXE>(yyy, st + L::YY + (ty + 4) * TXE + 2 * tx);
+      ycol<TXE>(yyz, st + L::YZ + (ty + 4) * TXE + 2 * tx);
       float d0[2], d1[2], d2[2], d3[2], d4[2], d5[2], d6[2], d7[2], d8[2];
 #pragma unroll
       for (int e = 0; e < 2; ++e) {
@@ -233,32 +218,42 @@ __global__ void __launch_bounds__(NTX2 * BY) el_v_kernel(const __grid_constant__
         d7[e] = dm(yyz[e], 4);   // Dy- syz
         d8[e] = dp(zzz, 3);      // Dz+ szz  (zzz[0..7] = k-3..k+4)
       }
-      if (W > 0) {
-        const int gz = k + d.z0;
-        if (lx) {
-          cpml2_x(d0, a.psi[0], d, W, x0, j, k, a.cx.ah, a.cx.bh);
-          cpml2_x(d3, a.psi[3], d, W, x0, j, k, a.cx.a, a.cx.b);
-          cpml2_x(d6, a.psi[6], d, W, x0, j, k, a.cx.a, a.cx.b);
+      if (lx) {
+        float ca[2], cb[2], cah[2], cbh[2];
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const int x = min(x0 + e, d.nx - 1);
+          ca[e] = __ldg(a.cx.a + x); cb[e] = __ldg(a.cx.b + x);
+          cah[e] = __ldg(a.cx.ah + x); cbh[e] = __ldg(a.cx.bh + x);
         }
-        if (ly) {
-          cpml2_y(d1, a.psi[1], d, W, x0, j, k, __ldg(a.cy.a + j), __ldg(a.cy.b + j));
-          cpml2_y(d4, a.psi[4], d, W, x0, j, k, __ldg(a.cy.ah + j), __ldg(a.cy.bh + j));
-          cpml2_y(d7, a.psi[7], d, W, x0, j, k, __ldg(a.cy.a + j), __ldg(a.cy.b + j));
-        }
-        if (CpmlIdx::in(gz, d.nz, W, a.zlo)) {
-          cpml2_z(d2, a.psi[2], d, W, x0, j, gz, __ldg(a.cz.a + gz), __ldg(a.cz.b + gz));
-          cpml2_z(d5, a.psi[5], d, W, x0, j, gz, __ldg(a.cz.a + gz), __ldg(a.cz.b + gz));
-          cpml2_z(d8, a.psi[8], d, W, x0, j, gz, __ldg(a.cz.ah + gz), __ldg(a.cz.bh + gz));
-        }
+        psi_upd<2>(d0, a.psi[0], ixx, ox0, cah, cbh);
+        psi_upd<2>(d3, a.psi[3], ixx, ox3, ca, cb);
+        psi_upd<2>(d6, a.psi[6], ixx, ox6, ca, cb);
       }
-      const float* sv = st + L::V + pt;
-      const float* sb = st + L::B + pt;
+      if (ly) {
+        const float ya = __ldg(a.cy.a + j), yb = __ldg(a.cy.b + j);
+        const float yah = __ldg(a.cy.ah + j), ybh = __ldg(a.cy.bh + j);
+        const float ca[2] = {ya, ya}, cb[2] = {yb, yb}, cah[2] = {yah, yah}, cbh[2] = {ybh, ybh};
+        psi_upd<2>(d1, a.psi[1], iyy, oy1, ca, cb);
+        psi_upd<2>(d4, a.psi[4], iyy, oy4, cah, cbh);
+        psi_upd<2>(d7, a.psi[7], iyy, oy7, ca, cb);
+      }
+      if (lz) {
+        const float za = __ldg(a.cz.a + gz), zb = __ldg(a.cz.b + gz);
+        const float zah = __ldg(a.cz.ah + gz), zbh = __ldg(a.cz.bh + gz);
+        const float ca[2] = {za, za}, cb[2] = {zb, zb}, cah[2] = {zah, zah}, cbh[2] = {zbh, zbh};
+        psi_upd<2>(d2, a.psi[2], izz, oz2, ca, cb);
+        psi_upd<2>(d5, a.psi[5], izz, oz5, ca, cb);
+        psi_upd<2>(d8, a.psi[8], izz, oz8, cah, cbh);
+      }
+      const F2 v0 = lds2(st + L::V + pt), v1 = lds2(st + L::V + T + pt), v2 = lds2(st + L::V + 2 * T + pt);
+      const F2 b0 = lds2(st + L::B + pt), b1 = lds2(st + L::B + T + pt), b2 = lds2(st + L::B + 2 * T + pt);
       F2 ov[3];
 #pragma unroll
       for (int e = 0; e < 2; ++e) {
-        ov[0].v[e] = fmaf(sb[e], (d0[e] + d1[e]) + d2[e], sv[e]);
-        ov[1].v[e] = fmaf(sb[T + e], (d3[e] + d4[e]) + d5[e], sv[T + e]);
-        ov[2].v[e] = fmaf(sb[2 * T + e], (d6[e] + d7[e]) + d8[e], sv[2 * T + e]);
+        ov[0].v[e] = fmaf(b0.v[e], (d0[e] + d1[e]) + d2[e], v0.v[e]);
+        ov[1].v[e] = fmaf(b1.v[e], (d3[e] + d4[e]) + d5[e], v1.v[e]);
+        ov[2].v[e] = fmaf(b2.v[e], (d6[e] + d7[e]) + d8[e], v2.v[e]);
       }
 #pragma unroll
       for (int c = 0; c < 3; ++c) st2_masked(a.f[EVX + c] + o, ov[c], x0, d.nx);
@@ -294,13 +289,13 @@ struct ElSArgs {
 
 template <int BY>
 struct ElSStage {
-  static constexpr int WX = TXV + 8, T = TXV * BY, TV = (BY + 8) * WX;
+  static constexpr int WX = TXE + 8, T = TXE * BY, TV = (BY + 8) * WX;
   static constexpr int VT = 0, S = 3 * TV, C = S + 6 * T, Q = C + 5 * T, SIZE = Q + 3 * T;
   static constexpr size_t smem_bytes() { return (size_t)EL_SNS * SIZE * 4 + 128; }
 };
 
 template <int BY, bool UNUSED>
-__global__ void __launch_bounds__(NTX2 * BY) el_s_kernel(const __grid_constant__ ElSArgs a) {
+__global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constant__ ElSArgs a) {
   using L = ElSStage<BY>;
   constexpr int WX = L::WX, T = L::T, TV = L::TV;
   constexpr uint32_t TX_BYTES = L::SIZE * 4;
@@ -309,7 +304,7 @@ __global__ void __launch_bounds__(NTX2 * BY) el_s_kernel(const __grid_constant__
   __shared__ __align__(8) uint64_t bar[EL_SNS];
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX2 + tx;
-  const int i0 = blockIdx.x * TXV, j0 = blockIdx.y * BY;
+  const int i0 = blockIdx.x * TXE, j0 = blockIdx.y * BY;
   const int x0 = i0 + 2 * tx, j = j0 + ty;
   const int k0 = blockIdx.z * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
@@ -356,14 +351,36 @@ __global__ void __launch_bounds__(NTX2 * BY) el_s_kernel(const __grid_constant__
     const int k = k0 + it;
     const int s = it % EL_SNS;
     const long long o = (long long)(k + GZ) * PS + oc;
+    // C-PML: old psi values are loaded before the wait (latency overlap)
+    const int gz = k + d.z0;
+    const bool lz = W > 0 && CpmlIdx::in(gz, d.nz, W, a.zlo);
+    long long ixx[2], iyy[2], izz[2];
+    float ox0[2], ox4[2], ox6[2], oy1[2], oy3[2], oy8[2], oz2[2], oz5[2], oz7[2];
+    if (own && lx) {
+      psi_idx_x<2>(ixx, d, W, x0, j, k);
+      psi_ld<2>(ox0, a.psi[0], ixx);
+      psi_ld<2>(ox4, a.psi[4], ixx);
+      psi_ld<2>(ox6, a.psi[6], ixx);
+    }
+    if (own && ly) {
+      psi_idx_row<2>(iyy, ((long long)k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0, x0, d.nx);
+      psi_ld<2>(oy1, a.psi[1], iyy);
+      psi_ld<2>(oy3, a.psi[3], iyy);
+      psi_ld<2>(oy8, a.psi[8], iyy);
+    }
+    if (own && lz) {
+      psi_idx_row<2>(izz, ((long long)CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0, x0, d.nx);
+      psi_ld<2>(oz2, a.psi[2], izz);
+      psi_ld<2>(oz5, a.psi[5], izz);
+      psi_ld<2>(oz7, a.psi[7], izz);
+    }
     mbar_wait(&bar[s], (it / EL_SNS) & 1);
     const float* st = sm + s * L::SIZE;
-    const int pt = ty * TXV + 2 * tx;
+    const int pt = ty * TXE + 2 * tx;
     qx[7] = lds2(st + L::Q + pt);
     qy[7] = lds2(st + L::Q + T + pt);
     qz[7] = lds2(st + L::Q + 2 * T + pt);
     if (own) {
-      const int gz = k + d.z0;
       const float* cvx = st + L::VT + (ty + 4) * WX + 2 * tx + 4;
       const float* cvy = cvx + TV;
       const float* cvz = cvx + 2 * TV;
@@ -394,36 +411,50 @@ __global__ void __launch_bounds__(NTX2 * BY) el_s_kernel(const __grid_constant__
         dzvy[e] = dp(zy, 3);       // Dz+ vy
         dyvz[e] = dp(yvz[e], 4);   // Dy+ vz
       }
-      if (W > 0) {
-        if (lx) {
-          cpml2_x(exx, a.psi[0], d, W, x0, j, k, a.cx.a, a.cx.b);
-          cpml2_x(dxvy, a.psi[4], d, W, x0, j, k, a.cx.ah, a.cx.bh);
-          cpml2_x(dxvz, a.psi[6], d, W, x0, j, k, a.cx.ah, a.cx.bh);
+      if (lx) {
+        float ca[2], cb[2], cah[2], cbh[2];
+#pragma unroll
+        for (int e = 0; e < 2; ++e) {
+          const int x = min(x0 + e, d.nx - 1);
+          ca[e] = __ldg(a.cx.a + x); cb[e] = __ldg(a.cx.b + x);
+          cah[e] = __ldg(a.cx.ah + x); cbh[e] = __ldg(a.cx.bh + x);
         }
-        if (ly) {
-          cpml2_y(eyy, a.psi[1], d, W, x0, j, k, __ldg(a.cy.a + j), __ldg(a.cy.b + j));
-          cpml2_y(dyvx, a.psi[3], d, W, x0, j, k, __ldg(a.cy.ah + j), __ldg(a.cy.bh + j));
-          cpml2_y(dyvz, a.psi[8], d, W, x0, j, k, __ldg(a.cy.ah + j), __ldg(a.cy.bh + j));
-        }
-        if (CpmlIdx::in(gz, d.nz, W, a.zlo)) {
-          cpml2_z(ezz, a.psi[2], d, W, x0, j, gz, __ldg(a.cz.a + gz), __ldg(a.cz.b + gz));
-          cpml2_z(dzvx, a.psi[5], d, W, x0, j, gz, __ldg(a.cz.ah + gz), __ldg(a.cz.bh + gz));
-          cpml2_z(dzvy, a.psi[7], d, W, x0, j, gz, __ldg(a.cz.ah + gz), __ldg(a.cz.bh + gz));
-        }
+        psi_upd<2>(exx, a.psi[0], ixx, ox0, ca, cb);
+        psi_upd<2>(dxvy, a.psi[4], ixx, ox4, cah, cbh);
+        psi_upd<2>(dxvz, a.psi[6], ixx, ox6, cah, cbh);
       }
-      const float* ss = st + L::S + pt;
-      const float* sc = st + L::C + pt;
+      if (ly) {
+        const float ya = __ldg(a.cy.a + j), yb = __ldg(a.cy.b + j);
+        const float yah = __ldg(a.cy.ah + j), ybh = __ldg(a.cy.bh + j);
+        const float ca[2] = {ya, ya}, cb[2] = {yb, yb}, cah[2] = {yah, yah}, cbh[2] = {ybh, ybh};
+        psi_upd<2>(eyy, a.psi[1], iyy, oy1, ca, cb);
+        psi_upd<2>(dyvx, a.psi[3], iyy, oy3, cah, cbh);
+        psi_upd<2>(dyvz, a.psi[8], iyy, oy8, cah, cbh);
+      }
+      if (lz) {
+        const float za = __ldg(a.cz.a + gz), zb = __ldg(a.cz.b + gz);
+        const float zah = __ldg(a.cz.ah + gz), zbh = __ldg(a.cz.bh + gz);
+        const float ca[2] = {za, za}, cb[2] = {zb, zb}, cah[2] = {zah, zah}, cbh[2] = {zbh, zbh};
+        psi_upd<2>(ezz, a.psi[2], izz, oz2, ca, cb);
+        psi_upd<2>(dzvx, a.psi[5], izz, oz5, cah, cbh);
+        psi_upd<2>(dzvy, a.psi[7], izz, oz7, cah, cbh);
+      }
+      F2 sv[6], cv[5];
+#pragma unroll
+      for (int c = 0; c < 6; ++c) sv[c] = lds2(st + L::S + c * T + pt);
+#pragma unroll
+      for (int c = 0; c < 5; ++c) cv[c] = lds2(st + L::C + c * T + pt);
       const bool surf = a.fs && gz == 0;
       const long long rel = srel0 - (long long)(k + GZ) * PS;
       F2 o6[6];
 #pragma unroll
       for (int e = 0; e < 2; ++e) {
-        const float l2m = sc[e], lam = sc[T + e];
+        const float l2m = cv[0].v[e], lam = cv[1].v[e];
         float ez = ezz[e];
         if (surf) ez = -(lam / l2m) * (exx[e] + eyy[e]);  // O16 surface row
-        float sxx = ss[e] + fmaf(l2m, exx[e], lam * (eyy[e] + ez));
-        float syy = ss[T + e] + fmaf(l2m, eyy[e], lam * (exx[e] + ez));
-        float szz = ss[2 * T + e] + fmaf(l2m, ez, lam * (exx[e] + eyy[e]));
+        float sxx = sv[0].v[e] + fmaf(l2m, exx[e], lam * (eyy[e] + ez));
+        float syy = sv[1].v[e] + fmaf(l2m, eyy[e], lam * (exx[e] + ez));
+        float szz = sv[2].v[e] + fmaf(l2m, ez, lam * (exx[e] + eyy[e]));
         if (rel == e) {
           sxx -= a.src_amp;
           syy -= a.src_amp;
@@ -433,9 +464,9 @@ __global__ void __launch_bounds__(NTX2 * BY) el_s_kernel(const __grid_constant__
         o6[0].v[e] = sxx;
         o6[1].v[e] = syy;
         o6[2].v[e] = szz;
-        o6[3].v[e] = fmaf(sc[2 * T + e], dyvx[e] + dxvy[e], ss[3 * T + e]);
-        o6[4].v[e] = fmaf(sc[3 * T + e], dzvx[e] + dxvz[e], ss[4 * T + e]);
-        o6[5].v[e] = fmaf(sc[4 * T + e], dzvy[e] + dyvz[e], ss[5 * T + e]);
+        o6[3].v[e] = fmaf(cv[2].v[e], dyvx[e] + dxvy[e], sv[3].v[e]);
+        o6[4].v[e] = fmaf(cv[3].v[e], dzvx[e] + dxvz[e], sv[4].v[e]);
+        o6[5].v[e] = fmaf(cv[4].v[e], dzvy[e] + dyvz[e], sv[5].v[e]);
       }
 #pragma unroll
       for (int c = 0; c < 6; ++c) st2_masked(a.f[ESXX + c] + o, o6[c], x0, d.nx);

@@ -258,7 +258,7 @@ Dims make_dims(const seis_grid& g, int z0, int nzl) {
   d.nzl = nzl;
   d.nz = g.nz;
   d.z0 = z0;
-  d.PX = roundup(roundup(g.nx, TXV) + 2 * G, 32);
+  d.PX = roundup(roundup(g.nx, std::max(TXV, TXE)) + 2 * G, 32);
   d.PY = roundup(g.ny, 32) + 2 * G;  // any tile height up to 32
   d.PS = (long long)d.PX * d.PY;
   return d;
@@ -776,20 +776,20 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       TRY(make_map(&S.ac_qzc, S.fld[3], d, TXV, BYP));
       TRY(make_map(&S.ac_kc, S.kdt, d, TXV, BYP));
     } else {
-      TRY(make_map(&S.el_sxxt, S.fld[ESXX], d, TXV + 8, BYE));
-      TRY(make_map(&S.el_sxyt, S.fld[ESXY], d, TXV + 8, BYE + 8));
-      TRY(make_map(&S.el_sxzt, S.fld[ESXZ], d, TXV + 8, BYE));
-      TRY(make_map(&S.el_syyt, S.fld[ESYY], d, TXV, BYE + 8));
-      TRY(make_map(&S.el_syzt, S.fld[ESYZ], d, TXV, BYE + 8));
+      TRY(make_map(&S.el_sxxt, S.fld[ESXX], d, TXE + 8, BYE));
+      TRY(make_map(&S.el_sxyt, S.fld[ESXY], d, TXE + 8, BYE + 8));
+      TRY(make_map(&S.el_sxzt, S.fld[ESXZ], d, TXE + 8, BYE));
+      TRY(make_map(&S.el_syyt, S.fld[ESYY], d, TXE, BYE + 8));
+      TRY(make_map(&S.el_syzt, S.fld[ESYZ], d, TXE, BYE + 8));
       float* bb[3] = {S.bx, S.by, S.bz};
       for (int t = 0; t < 3; ++t) {
-        TRY(make_map(&S.el_vc[t], S.fld[EVX + t], d, TXV, BYE));
-        TRY(make_map(&S.el_bc[t], bb[t], d, TXV, BYE));
-        TRY(make_map(&S.el_vt[t], S.fld[EVX + t], d, TXV + 8, BYE + 8));
+        TRY(make_map(&S.el_vc[t], S.fld[EVX + t], d, TXE, BYE));
+        TRY(make_map(&S.el_bc[t], bb[t], d, TXE, BYE));
+        TRY(make_map(&S.el_vt[t], S.fld[EVX + t], d, TXE + 8, BYE + 8));
       }
-      for (int t = 0; t < 6; ++t) TRY(make_map(&S.el_sc[t], S.fld[ESXX + t], d, TXV, BYE));
+      for (int t = 0; t < 6; ++t) TRY(make_map(&S.el_sc[t], S.fld[ESXX + t], d, TXE, BYE));
       float* cc[5] = {S.l2m, S.lam, S.mxy, S.mxz, S.myz};
-      for (int t = 0; t < 5; ++t) TRY(make_map(&S.el_cc[t], cc[t], d, TXV, BYE));
+      for (int t = 0; t < 5; ++t) TRY(make_map(&S.el_cc[t], cc[t], d, TXE, BYE));
     }
     TRY(set_smem_attrs());
     int occ = 1;
@@ -802,7 +802,7 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     else
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, NTX2 * BYE,
                                                     ElSStage<BYE>::smem_bytes());
-    if (kind == SEIS_ELASTIC) choose_chunks(S, occ, dev_sms, TXV, BYE);
+    if (kind == SEIS_ELASTIC) choose_chunks(S, occ, dev_sms, TXE, BYE);
     else choose_chunks(S, occ, dev_sms, TXV, kind == SEIS_ISO ? BYI : BYV);
   }
   if (kind == SEIS_ACOUSTIC)  // rho(k+1) across slab faces
@@ -1193,7 +1193,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (int t = 0; t < 9; ++t) a.psi[t] = S.psi[t];
     a.d = S.d;
     a.zc = S.zc;
-    const dim3 gr = grid_of(S, TXV, BYE);
+    const dim3 gr = grid_of(S, TXE, BYE);
     {
       PROF(3, st);
       el_v_kernel<BYE><<<gr, dim3(NTX2, BYE), ElVStage<BYE>::smem_bytes(), st>>>(a);
@@ -1222,7 +1222,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     a.src_o = with_src ? S.src_o : -1;
     a.src_amp = 0.f;
     if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
-    const dim3 gr = grid_of(S, TXV, BYE);
+    const dim3 gr = grid_of(S, TXE, BYE);
     {
       PROF(4, st);
       el_s_kernel<BYE, false><<<gr, dim3(NTX2, BYE), ElSStage<BYE>::smem_bytes(), st>>>(a);

@@ -19,17 +19,11 @@ sys.path.insert(0, ROOT)
 
 VARIANTS = {
     "base": [],
-    "i4": ["SEIS_BYI=4", "SEIS_ISO_NS=6"],
-    "i8ns3": ["SEIS_ISO_NS=3"],
-    "i8ns6": ["SEIS_ISO_NS=6"],
-    "v8": ["SEIS_BYV=8", "SEIS_AC_VNS=3"],
-    "v8ns4": ["SEIS_BYV=8", "SEIS_AC_VNS=4"],
-    "v16ns2": ["SEIS_AC_VNS=2"],
-    "p8": ["SEIS_BYP=8", "SEIS_AC_NS=2"],
-    "p8ns3": ["SEIS_BYP=8", "SEIS_AC_NS=3"],
-    "p16ns3": ["SEIS_AC_NS=3"],
-    "e22": ["SEIS_EL_VNS=2", "SEIS_EL_SNS=2"],
-    "e4_32": ["SEIS_BYE=4", "SEIS_EL_VNS=3", "SEIS_EL_SNS=2"],
+    "t128_4": ["SEIS_TXV=128", "SEIS_BYI=4", "SEIS_BYV=4", "SEIS_BYP=8"],
+    "t128_8": ["SEIS_TXV=128", "SEIS_BYI=8", "SEIS_BYV=8", "SEIS_BYP=8"],
+    "t128_4ns": ["SEIS_TXV=128", "SEIS_BYI=4", "SEIS_BYV=4", "SEIS_BYP=8", "SEIS_ISO_NS=4",
+                 "SEIS_AC_VNS=4", "SEIS_AC_NS=3"],
+    "t128_p4": ["SEIS_TXV=128", "SEIS_BYI=4", "SEIS_BYV=4", "SEIS_BYP=4", "SEIS_AC_NS=3"],
 }
 
 
