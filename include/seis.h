@@ -100,6 +100,11 @@ seis_status seis_comm_unique_id(uint8_t id[128]);
 seis_status seis_comm_create(int32_t nranks, int32_t rank, const uint8_t id[128], int32_t device,
                              seis_comm** out);
 seis_status seis_comm_destroy(seis_comm* comm);
+/* Shot-parallel RTM (sum over shots of P:111 across ranks): every rank
+ * migrates its own shots on a full-grid replica (comm = NULL model) into a local image,
+ * then this all-reduces (sums) the n floats of `image` (device) over the communicator in
+ * place.  Collective; synchronous w.r.t. `stream` on return. */
+seis_status seis_image_reduce(seis_comm* comm, float* image, uint64_t n, void* stream);
 
 /* ---- model ---- */
 /* Creates a model: validates the grid (EINVAL), the Courant bound (ECFL), the
@@ -130,7 +135,8 @@ seis_status seis_model_destroy(seis_model* model);
  *         rank-owned entries; exact because exactly one rank owns each receiver). */
 seis_status seis_forward_model(seis_model* model, const seis_shot* shot, float* seis,
                                void* stream);
-/* Reverse-time migration of one shot (ISO and ACOUSTIC; ELASTIC: EUNSUPPORTED).
+/* Reverse-time migration of one shot.  ISO images u, ACOUSTIC p, ELASTIC the pressure
+ * -(sxx+syy+szz)/3 (receivers inject like the explosive source).
  *   data  host or device [nt][nrec] fp32 observed data (replicated on every rank)
  *   image host or device [nz_local][ny][nx] fp32, ACCUMULATED (+=), never zeroed
  * Snapshot pool: nsnap = (nt-1)/snap_period fields of nz_local*ny*nx floats in HBM;

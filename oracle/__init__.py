@@ -84,7 +84,7 @@ def _L():
                                    C.POINTER(_Rec), d]
         _lib.or_el_run.argtypes = [g, f, f, f, d, d, C.c_int, C.c_int, C.POINTER(_Inj),
                                    C.POINTER(_Rec), d]
-        _lib.or_migrate.argtypes = [g, C.c_int, f, f, i32, d, C.c_int, C.c_int, i32, d,
+        _lib.or_migrate.argtypes = [g, C.c_int, f, f, f, i32, d, C.c_int, C.c_int, i32, d,
                                     C.c_int, d]
         for fn in ("or_iso_run", "or_ac_run", "or_el_run", "or_migrate"):
             getattr(_lib, fn).restype = C.c_int
@@ -271,10 +271,12 @@ def forward_model(grid, kind, vp, rho=None, vs=None, src=None, wavelet=None, rec
     return seis, st
 
 
-def migrate(grid, kind, vp, rho, src, wavelet, rec, data, snap, image=None):
-    """RTM (Alg 1) of one shot; returns image (accumulated into `image` if given)."""
+def migrate(grid, kind, vp, rho, src, wavelet, rec, data, snap, image=None, vs=None):
+    """RTM (Alg 1) of one shot; returns image (accumulated into `image` if given).
+    ELASTIC images the pressure -(sxx+syy+szz)/3 with explosive receiver injection."""
     vp = np.ascontiguousarray(vp, dtype=np.float32)
     rho = np.ascontiguousarray(rho if rho is not None else np.ones_like(vp), dtype=np.float32)
+    vs = np.ascontiguousarray(vs if vs is not None else np.zeros_like(vp), dtype=np.float32)
     sp = np.ascontiguousarray(np.asarray(src, dtype=np.int32).reshape(3))
     amp = np.ascontiguousarray(np.asarray(wavelet, dtype=np.float64))
     rp = np.ascontiguousarray(np.asarray(rec, dtype=np.int32).reshape(-1, 3))
@@ -284,7 +286,7 @@ def migrate(grid, kind, vp, rho, src, wavelet, rec, data, snap, image=None):
     if image is None:
         image = np.zeros(grid.shape)
     g = grid.c()
-    rc = _L().or_migrate(C.byref(g), KIND[kind], _fp(vp), _fp(rho), _ip(sp), _dp(amp), nt,
+    rc = _L().or_migrate(C.byref(g), KIND[kind], _fp(vp), _fp(vs), _fp(rho), _ip(sp), _dp(amp), nt,
                          rp.shape[0], _ip(rp), _dp(dd), int(snap), _dp(image))
     _check(rc, "migrate")
     return image

@@ -594,12 +594,13 @@ int or_el_run(const or_grid* g, const float* vp, const float* vs, const float* r
  *  backward (the paper's order, imaging BEFORE the step):
  *           R = 0; for m = 0..nt-1: j = nt - m; if j is a snapshot level,
  *           image += S_j * R; step R with receiver injection of data[nt-1-m][r].
- * This pairs S_j with R^{m+1}, j = nt-1-m (O15).                            */
-int or_migrate(const or_grid* g, int kind, const float* vp, const float* rho,
+ * This pairs S_j with R^{m+1}, j = nt-1-m (O15).  ELASTIC (f3): snapshots and
+ * imaging use the pressure -(sxx+syy+szz)/3; receivers inject as explosive sources. */
+int or_migrate(const or_grid* g, int kind, const float* vp, const float* vs, const float* rho,
                const int32_t src_pos[3], const double* src_amp, int nt, int nrec,
                const int32_t* rec_pos, const double* data, int snap, double* image) {
   if (snap < 1 || nt < 1) return -1;
-  if (kind != 0 && kind != 1) return -4;
+  if (kind != 0 && kind != 1 && kind != 2) return -4;
   size_t n = NPTS(g);
   int nsnap = (nt - 1) / snap;
   double* S = (double*)calloc((size_t)(nsnap > 0 ? nsnap : 1) * n, sizeof(double));
@@ -611,23 +612,27 @@ int or_migrate(const or_grid* g, int kind, const float* vp, const float* rho,
   or_inj recinj = {nrec, rec_pos, back_amp};
   int rc = 0;
   double *a = (double*)calloc(n, sizeof(double)), *b = (double*)calloc(n, sizeof(double));
-  double *q = NULL, *psi = NULL;
+  double *q = NULL, *psi = NULL, *f = NULL;
   if (kind == 1) {
     q = (double*)calloc(3 * n, sizeof(double));
     psi = (double*)calloc(6 * n, sizeof(double));
   }
+  if (kind == 2) { /* elastic: 9 fields, 18 psi; imaged field = pressure -(sxx+syy+szz)/3 */
+    f = (double*)calloc(9 * n, sizeof(double));
+    psi = (double*)calloc(18 * n, sizeof(double));
+  }
   /* forward phase */
   for (int t = 0; t < nt && !rc; ++t) {
-    double* field;
     if (kind == 0) {
       rc = or_iso_run(g, vp, a, b, t, 1, &src, NULL, NULL);
-      field = b;
-    } else {
+    } else if (kind == 1) {
       rc = or_ac_run(g, vp, rho, b, q, q + n, q + 2 * n, psi, t, 1, &src, NULL, NULL);
-      field = b;
+    } else {
+      rc = or_el_run(g, vp, vs, rho, f, psi, t, 1, &src, NULL, NULL);
+      for (size_t o = 0; o < n; ++o) b[o] = -(f[3 * n + o] + f[4 * n + o] + f[5 * n + o]) / 3.0;
     }
     int j = t + 1;
-    if (j % snap == 0 && j <= nt - 1) memcpy(S + (size_t)(j / snap - 1) * n, field, sizeof(double) * n);
+    if (j % snap == 0 && j <= nt - 1) memcpy(S + (size_t)(j / snap - 1) * n, b, sizeof(double) * n);
   }
   /* backward phase: fresh zero state */
   memset(a, 0, sizeof(double) * n);
@@ -636,16 +641,25 @@ int or_migrate(const or_grid* g, int kind, const float* vp, const float* rho,
     memset(q, 0, sizeof(double) * 3 * n);
     memset(psi, 0, sizeof(double) * 6 * n);
   }
+  if (kind == 2) {
+    memset(f, 0, sizeof(double) * 9 * n);
+    memset(psi, 0, sizeof(double) * 18 * n);
+  }
   for (int m = 0; m < nt && !rc; ++m) {
     int j = nt - m;
     if (j % snap == 0 && j >= snap && j <= nt - 1) {
       const double* Sj = S + (size_t)(j / snap - 1) * n;
       for (size_t o = 0; o < n; ++o) image[o] += Sj[o] * b[o]; /* P:111 zero-lag */
     }
-    if (kind == 0)
+    if (kind == 0) {
       rc = or_iso_run(g, vp, a, b, m, 1, &recinj, NULL, NULL);
-    else
+    } else if (kind == 1) {
       rc = or_ac_run(g, vp, rho, b, q, q + n, q + 2 * n, psi, m, 1, &recinj, NULL, NULL);
+    } else {
+      /* receivers inject as explosive sources (O11 scaling), the imaged field is pressure */
+      rc = or_el_run(g, vp, vs, rho, f, psi, m, 1, &recinj, NULL, NULL);
+      for (size_t o = 0; o < n; ++o) b[o] = -(f[3 * n + o] + f[4 * n + o] + f[5 * n + o]) / 3.0;
+    }
   }
   free(S);
   free(back_amp);
@@ -653,5 +667,6 @@ int or_migrate(const or_grid* g, int kind, const float* vp, const float* rho,
   free(b);
   free(q);
   free(psi);
+  free(f);
   return rc;
 }

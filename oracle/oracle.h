@@ -89,8 +89,10 @@ int or_el_run(const or_grid* g, const float* vp, const float* vs, const float* r
 /* RTM (Alg 1; O14/O15): forward source propagation storing
  * snapshots S_j (j = snap, 2 snap, ... <= nt-1), then backward receiver
  * propagation injecting data[nt-1-m][r] at reversed step m and imaging
- * image += S_j * R.  kind 0 = ISO, 1 = ACOUSTIC.  image is accumulated. */
-int or_migrate(const or_grid* g, int kind, const float* vp, const float* rho,
+ * image += S_j * R.  kind 0 = ISO, 1 = ACOUSTIC, 2 = ELASTIC (imaged field:
+ * pressure -(sxx+syy+szz)/3; receivers inject like the explosive source).
+ * image is accumulated. */
+int or_migrate(const or_grid* g, int kind, const float* vp, const float* vs, const float* rho,
                const int32_t src_pos[3], const double* src_amp, int nt,
                int nrec, const int32_t* rec_pos, const double* data, int snap,
                double* image);

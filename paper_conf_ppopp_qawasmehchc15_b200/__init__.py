@@ -31,7 +31,8 @@ STATUS = {0: "SEIS_OK", 1: "SEIS_EINVAL", 2: "SEIS_ECFL", 3: "SEIS_ENOMEM", 4: "
           5: "SEIS_ENCCL", 6: "SEIS_EUNSUPPORTED"}
 
 # every symbol include/seis.h declares
-SYMBOLS = ["seis_comm_unique_id", "seis_comm_create", "seis_comm_destroy", "seis_model_create",
+SYMBOLS = ["seis_comm_unique_id", "seis_comm_create", "seis_comm_destroy", "seis_image_reduce",
+           "seis_model_create",
            "seis_slab_bounds", "seis_model_slab", "seis_model_destroy", "seis_forward_model",
            "seis_migrate", "seis_get_field", "seis_memory_required", "seis_profile",
            "seis_profile_read", "seis_last_launch_count",
@@ -74,6 +75,7 @@ def lib():
         L.seis_comm_create.argtypes = [C.c_int32, C.c_int32, C.POINTER(C.c_uint8), C.c_int32,
                                        C.POINTER(vp)]
         L.seis_comm_destroy.argtypes = [vp]
+        L.seis_image_reduce.argtypes = [vp, vp, C.c_uint64, vp]
         L.seis_model_create.argtypes = [C.POINTER(_CGrid), C.c_int, vp, vp, vp, vp, C.c_int32,
                                         C.POINTER(vp)]
         L.seis_slab_bounds.argtypes = [C.c_int32, C.c_int32, C.c_int32, C.POINTER(C.c_int32),
@@ -204,6 +206,11 @@ class Comm:
                          device=f"cuda:{device}" if dist.get_backend() == "nccl" else "cpu")
         dist.broadcast(t, 0)
         return cls(world, rank, bytes(t.cpu().tolist()), device)
+
+    def reduce_image(self, image, stream=None):
+        """Sum a device image over all ranks in place (shot-parallel RTM, sum_s of P:111)."""
+        _check(lib().seis_image_reduce(self.h, _ptr(image), image.numel(), _stream(stream)))
+        return image
 
     def close(self):
         if getattr(self, "h", None):

@@ -43,6 +43,25 @@ __global__ void inject_kernel(float* __restrict__ f, const long long* __restrict
   f[off[u]] = fmaf(scale[u], s, f[off[u]]);
 }
 
+// Elastic RTM receiver injection (f3): receivers act like the explosive source (O11),
+//   s_ii -= scale[u] * sum_{r in group u} data_row[r]   for ii = xx, yy, zz,
+// except s_zz on a free-surface node, which the surface condition keeps at 0 (O16).
+__global__ void inject_el_kernel(float* __restrict__ sxx, float* __restrict__ syy, float* __restrict__ szz,
+                                 const long long* __restrict__ off, const float* __restrict__ scale,
+                                 const int* __restrict__ gstart, const int* __restrict__ members,
+                                 const float* __restrict__ data_row, const int* __restrict__ surf,
+                                 int ngroups) {
+  const int u = blockIdx.x * blockDim.x + threadIdx.x;
+  if (u >= ngroups) return;
+  float s = 0.0f;
+  for (int t = gstart[u]; t < gstart[u + 1]; ++t) s += data_row[members[t]];
+  const long long o = off[u];
+  const float v = scale[u] * s;
+  sxx[o] -= v;
+  syy[o] -= v;
+  if (!surf[u]) szz[o] -= v;
+}
+
 // Copy the interior of a padded slab field to a compact [nzl][ny][nx] array.
 __global__ void unpad_kernel(float* __restrict__ dst, const float* __restrict__ src, Dims d) {
   const long long n = (long long)d.nzl * d.ny * d.nx;

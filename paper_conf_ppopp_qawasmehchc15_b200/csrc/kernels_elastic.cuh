@@ -88,6 +88,8 @@ struct ElVArgs {
   float* psi[9];   // psi 0..8
   Dims d;
   int zc;
+  const float* __restrict__ imgS;  // elastic RTM (f3): img += S * P on the input level, P = -(sxx+syy+szz)/3
+  float* __restrict__ img;
 };
 
 template <int BY>
@@ -99,7 +101,7 @@ struct ElVStage {
   static constexpr size_t smem_bytes() { return (size_t)EL_VNS * SIZE * 4 + 128; }
 };
 
-template <int BY>
+template <int BY, bool IMG>
 __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constant__ ElVArgs a) {
   using L = ElVStage<BY>;
   constexpr int WX = L::WX, T = L::T;
@@ -257,6 +259,15 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
       }
 #pragma unroll
       for (int c = 0; c < 3; ++c) st2_masked(a.f[EVX + c] + o, ov[c], x0, d.nx);
+      if (IMG) {
+        const long long cix = ((long long)k * d.ny + j) * d.nx + x0;
+#pragma unroll
+        for (int e = 0; e < 2; ++e)
+          if (x0 + e < d.nx) {
+            const float pr = -((xs[4 + e] + yyy[e][4]) + qzz[3].v[e]) / 3.0f;
+            a.img[cix + e] = fmaf(__ldg(a.imgS + cix + e), pr, a.img[cix + e]);
+          }
+      }
     }
     __syncthreads();
     if (tid == 0 && it + EL_VNS < np) {
@@ -285,6 +296,7 @@ struct ElSArgs {
   int zc;
   long long src_o;
   float src_amp;   // dt (lam + 2/3 mu)_s / h^3 * s[n]
+  float* __restrict__ snap;  // elastic RTM (f3): snapshot of P = -(sxx+syy+szz)/3, or nullptr
 };
 
 template <int BY>
@@ -294,7 +306,7 @@ struct ElSStage {
   static constexpr size_t smem_bytes() { return (size_t)EL_SNS * SIZE * 4 + 128; }
 };
 
-template <int BY, bool UNUSED>
+template <int BY, bool SNAP>
 __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constant__ ElSArgs a) {
   using L = ElSStage<BY>;
   constexpr int WX = L::WX, T = L::T, TV = L::TV;
@@ -470,6 +482,12 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
       }
 #pragma unroll
       for (int c = 0; c < 6; ++c) st2_masked(a.f[ESXX + c] + o, o6[c], x0, d.nx);
+      if (SNAP) {
+        const long long cix = ((long long)k * d.ny + j) * d.nx + x0;
+#pragma unroll
+        for (int e = 0; e < 2; ++e)
+          if (x0 + e < d.nx) a.snap[cix + e] = -((o6[0].v[e] + o6[1].v[e]) + o6[2].v[e]) / 3.0f;
+      }
     }
     __syncthreads();
     if (tid == 0 && it + EL_SNS < np) {

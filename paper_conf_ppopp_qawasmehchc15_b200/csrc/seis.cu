@@ -155,6 +155,7 @@ struct Slab {
   float* d_g_scale = nullptr;
   int* d_g_start = nullptr;
   int* d_g_mem = nullptr;
+  int* d_g_surf = nullptr;   // ELASTIC: group node on the free surface
   float* snap = nullptr;     // nsnap * nzl*ny*nx (points into the model's pool)
 };
 
@@ -332,8 +333,10 @@ seis_status set_smem_attrs() {
   SMEM_ATTR((ac_v_kernel<BYV, true>), AcVStage<BYV>::smem_bytes());
   SMEM_ATTR((ac_p_kernel<BYP, false>), AcPStage<BYP>::smem_bytes());
   SMEM_ATTR((ac_p_kernel<BYP, true>), AcPStage<BYP>::smem_bytes());
-  SMEM_ATTR((el_v_kernel<BYE>), ElVStage<BYE>::smem_bytes());
+  SMEM_ATTR((el_v_kernel<BYE, false>), ElVStage<BYE>::smem_bytes());
+  SMEM_ATTR((el_v_kernel<BYE, true>), ElVStage<BYE>::smem_bytes());
   SMEM_ATTR((el_s_kernel<BYE, false>), ElSStage<BYE>::smem_bytes());
+  SMEM_ATTR((el_s_kernel<BYE, true>), ElSStage<BYE>::smem_bytes());
 #undef SMEM_ATTR
   done = true;
   return SEIS_OK;
@@ -482,6 +485,16 @@ seis_status seis_comm_create(int32_t nranks, int32_t rank, const uint8_t id[128]
     return fail(SEIS_ENCCL, "ncclCommInitRank: %s", ncclGetErrorString(r));
   }
   *out = c;
+  return SEIS_OK;
+}
+
+seis_status seis_image_reduce(seis_comm* c, float* image, uint64_t n, void* stream) {
+  if (!c || (!image && n)) return fail(SEIS_EINVAL, "seis_image_reduce: null argument");
+  CK(cudaSetDevice(c->device));
+  if (!is_device_ptr(image)) return fail(SEIS_EINVAL, "seis_image_reduce: image must be a device buffer");
+  cudaStream_t st = (cudaStream_t)stream;
+  if (n) NK(ncclAllReduce(image, image, n, ncclFloat, ncclSum, c->nccl, st));
+  CK(cudaStreamSynchronize(st));
   return SEIS_OK;
 }
 
@@ -963,21 +976,27 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
       for (size_t t = 0; t < off.size(); ++t) groups[off[t]].push_back(rid[t]);
       std::vector<long long> goff;
       std::vector<float> gsc;
-      std::vector<int> gstart{0}, gmem;
+      std::vector<int> gstart{0}, gmem, gsurf;
       for (auto& kv : groups) {
         goff.push_back(kv.first);
         const int r0 = kv.second.front();
         const int* p = sh->rec + 3 * r0;
         gsc.push_back((float)point_scale(p[0], p[1], p[2]));
+        gsurf.push_back(M->g.free_surface && p[2] == 0 ? 1 : 0);
         for (int r : kv.second) gmem.push_back(r);
         gstart.push_back((int)gmem.size());
       }
       S.ngroups = (int)goff.size();
-      if (S.d_g_off) { cudaFree(S.d_g_off); cudaFree(S.d_g_scale); cudaFree(S.d_g_start); cudaFree(S.d_g_mem); }
+      if (S.d_g_off) {
+        cudaFree(S.d_g_off); cudaFree(S.d_g_scale); cudaFree(S.d_g_start); cudaFree(S.d_g_mem);
+        cudaFree(S.d_g_surf);
+      }
       CK(dmalloc(&S.d_g_off, goff.size()));
       CK(dmalloc(&S.d_g_scale, gsc.size()));
       CK(dmalloc(&S.d_g_start, gstart.size()));
       CK(dmalloc(&S.d_g_mem, gmem.size()));
+      CK(dmalloc(&S.d_g_surf, gsurf.size()));
+      CK(cudaMemcpy(S.d_g_surf, gsurf.data(), gsurf.size() * sizeof(int), cudaMemcpyHostToDevice));
       CK(cudaMemcpy(S.d_g_off, goff.data(), goff.size() * sizeof(long long), cudaMemcpyHostToDevice));
       CK(cudaMemcpy(S.d_g_scale, gsc.data(), gsc.size() * sizeof(float), cudaMemcpyHostToDevice));
       CK(cudaMemcpy(S.d_g_start, gstart.data(), gstart.size() * sizeof(int), cudaMemcpyHostToDevice));
@@ -1038,10 +1057,16 @@ dim3 grid_of(const Slab& S, int tw, int by) {
 seis_status inject_rows(seis_model* M, const float* row, cudaStream_t st) {
   for (Slab& S : M->slabs) {
     if (S.ngroups == 0) continue;
-    float* f = M->kind == SEIS_ISO ? S.fld[S.cur] : S.fld[0];
     PROF(5, st);
-    inject_kernel<<<(S.ngroups + 127) / 128, 128, 0, st>>>(f, S.d_g_off, S.d_g_scale, S.d_g_start,
-                                                           S.d_g_mem, row, S.ngroups);
+    if (M->kind == SEIS_ELASTIC) {
+      inject_el_kernel<<<(S.ngroups + 127) / 128, 128, 0, st>>>(
+          S.fld[ESXX], S.fld[ESYY], S.fld[ESZZ], S.d_g_off, S.d_g_scale, S.d_g_start, S.d_g_mem, row,
+          S.d_g_surf, S.ngroups);
+    } else {
+      float* f = M->kind == SEIS_ISO ? S.fld[S.cur] : S.fld[0];
+      inject_kernel<<<(S.ngroups + 127) / 128, 128, 0, st>>>(f, S.d_g_off, S.d_g_scale, S.d_g_start,
+                                                             S.d_g_mem, row, S.ngroups);
+    }
     CKL();
   }
   return SEIS_OK;
@@ -1193,10 +1218,13 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (int t = 0; t < 9; ++t) a.psi[t] = S.psi[t];
     a.d = S.d;
     a.zc = S.zc;
+    a.imgS = imgS ? (*imgS)[s] : nullptr;
+    a.img = img ? (*img)[s] : nullptr;
     const dim3 gr = grid_of(S, TXE, BYE);
     {
       PROF(3, st);
-      el_v_kernel<BYE><<<gr, dim3(NTX2, BYE), ElVStage<BYE>::smem_bytes(), st>>>(a);
+      if (a.img) el_v_kernel<BYE, true><<<gr, dim3(NTX2, BYE), ElVStage<BYE>::smem_bytes(), st>>>(a);
+      else el_v_kernel<BYE, false><<<gr, dim3(NTX2, BYE), ElVStage<BYE>::smem_bytes(), st>>>(a);
     }
     CKL();
   }
@@ -1222,13 +1250,16 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     a.src_o = with_src ? S.src_o : -1;
     a.src_amp = 0.f;
     if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
+    a.snap = snap ? (*snap)[s] : nullptr;
     const dim3 gr = grid_of(S, TXE, BYE);
     {
       PROF(4, st);
-      el_s_kernel<BYE, false><<<gr, dim3(NTX2, BYE), ElSStage<BYE>::smem_bytes(), st>>>(a);
+      if (a.snap) el_s_kernel<BYE, true><<<gr, dim3(NTX2, BYE), ElSStage<BYE>::smem_bytes(), st>>>(a);
+      else el_s_kernel<BYE, false><<<gr, dim3(NTX2, BYE), ElSStage<BYE>::smem_bytes(), st>>>(a);
     }
     CKL();
   }
+  if (inj_row) TRY(inject_rows(M, inj_row, st));
   TRY(exchange(M, {5, 7, 8}, st));
   TRY(fs_mirror(M, {ESZZ, ESXZ, ESYZ}, st));
   return SEIS_OK;
@@ -1347,7 +1378,6 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
   if (!sh) return fail(SEIS_EINVAL, "null shot");
   if (!image) return fail(SEIS_EINVAL, "null image");
   if (sh->nrec > 0 && !data) return fail(SEIS_EINVAL, "null data");
-  if (M->kind == SEIS_ELASTIC) return fail(SEIS_EUNSUPPORTED, "elastic RTM is not implemented in this version");
   if (sh->snap_period < 1) return fail(SEIS_EINVAL, "snap_period must be >= 1");
   CK(cudaSetDevice(M->device));
   cudaStream_t st = (cudaStream_t)stream;

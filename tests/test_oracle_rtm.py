@@ -164,3 +164,23 @@ def test_flat_reflector_images_at_its_depth():
     prof = np.abs(I[:, 10:n - 10, 10:n - 10]).sum(axis=(1, 2))
     prof[:12] = 0  # exclude the source/receiver depth band
     assert abs(int(np.argmax(prof)) - zr) <= 2
+
+
+def test_elastic_rtm_fluid_limit_equals_acoustic_rtm():
+    """Elastic RTM (f3; pressure imaging, explosive receiver injection) with vs = 0 reduces
+    exactly to acoustic RTM (O9 fluid limit applied to Algorithm 1)."""
+    m, g, w, src, rec, data = _setup("acoustic", n=14, nt=30, nb=3)
+    I_ac = oracle.migrate(g, "acoustic", m["vp"], m["rho"], src, w, rec, data, 3)
+    I_el = oracle.migrate(g, "elastic", m["vp"], m["rho"], src, w, rec, data, 3,
+                          vs=np.zeros_like(m["vp"]))
+    assert np.abs(I_ac).max() > 0
+    assert np.abs(I_el - I_ac).max() <= 1e-12 * np.abs(I_ac).max()
+
+
+def test_elastic_rtm_linear_and_accumulates():
+    m, g, w, src, rec, data = _setup("elastic", n=14, nt=30, nb=3)
+    me = inputs.random_media((14, 14, 14), seed=7, elastic=True)
+    I1 = oracle.migrate(g, "elastic", me["vp"], me["rho"], src, w, rec, data, 3, vs=me["vs"])
+    I2 = oracle.migrate(g, "elastic", me["vp"], me["rho"], src, w, rec, 2.0 * data, 3, vs=me["vs"])
+    assert np.abs(I1).max() > 0
+    assert np.abs(I2 - 2 * I1).max() <= 1e-12 * np.abs(I2).max()
