@@ -1,0 +1,105 @@
+"""GPU parity at BASELINE.json's full sizes, in the launch configuration bench.py times
+(same kernels, tile shapes and z-chunking, which depend only on the grid).
+
+The fp64 oracle cannot run 2000 steps of a 512^3 grid, so these tests compare
+(a) the first K time steps on the FULL grid (every output point, relative L2), and
+(b) properties that hold at any size: bitwise z-slab invariance of the 1024^3-class
+decomposition path at 256^3 ("C5 ... parity comes from bitwise
+P-invariance plus oracle parity of the same code path at 256^3").
+"""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_ppopp_qawasmehchc15_b200 as seis
+from paper_conf_ppopp_qawasmehchc15_b200 import inputs
+from gpu_common import TOL_FIELD, TOL_IMAGE, rel_l2
+
+pytestmark = pytest.mark.gpu
+
+
+def _ogrid(wl, **kw):
+    return oracle.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=wl.nb, pml_R=wl.pml_R, pml_f=wl.fp, **kw)
+
+
+def _sgrid(wl, **kw):
+    return seis.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=wl.nb, pml_R=wl.pml_R, pml_f=wl.fp, **kw)
+
+
+def test_c2_full_grid_first_steps():
+    """C2 (acoustic 512^3 layered, C-PML nb=20, 472 receivers): 6 steps, all fields."""
+    K = 6
+    wl = inputs.c2(n=512, nt=K)
+    model = seis.Model(_sgrid(wl), "acoustic", wl.model["vp"], rho=wl.model["rho"])
+    shot = seis.Shot(wl.src, wl.wavelet, wl.rec)
+    sg = np.zeros((K, shot.nrec), np.float32)
+    model.forward_model(shot, sg)
+    p_g = model.get_field(0)
+    qz_g = model.get_field(3)
+    model.close()
+    og = _ogrid(wl)
+    st = oracle.ac_state(og)
+    so = oracle.ac_run(og, wl.model["vp"], wl.model["rho"], st, 0, K, [wl.src], wl.wavelet[:, None], wl.rec)
+    assert rel_l2(p_g, st["p"]) <= TOL_FIELD
+    assert rel_l2(qz_g, st["qz"]) <= TOL_FIELD
+    nz_cols = np.abs(so).max(axis=0) > 0
+    assert nz_cols.any()
+    assert rel_l2(sg[:, nz_cols], so[:, nz_cols]) <= TOL_FIELD
+
+
+def test_c3_full_grid_first_steps():
+    """C3 (elastic 384^3, free surface, C-PML on 5 faces, surface vz line): 4 steps."""
+    K = 4
+    wl = inputs.c3(n=384, nt=K)
+    model = seis.Model(_sgrid(wl, free_surface=1), "elastic", wl.model["vp"], vs=wl.model["vs"],
+                       rho=wl.model["rho"])
+    shot = seis.Shot(wl.src, wl.wavelet, wl.rec, rec_component=2)
+    sg = np.zeros((K, shot.nrec), np.float32)
+    model.forward_model(shot, sg)
+    g_szz = model.get_field(5)
+    g_vz = model.get_field(2)
+    model.close()
+    og = _ogrid(wl, free_surface=1)
+    st = oracle.el_state(og)
+    oracle.el_run(og, wl.model["vp"], wl.model["vs"], wl.model["rho"], st, 0, K, [wl.src],
+                  wl.wavelet[:, None], wl.rec, component=2)
+    assert rel_l2(g_szz, st["f"][5]) <= TOL_FIELD
+    assert rel_l2(g_vz, st["f"][2]) <= TOL_FIELD
+
+
+def test_c4_full_grid_short_rtm():
+    """C4 (RTM 512^3 salt model, 13 924-receiver carpet): a 16-step migration with
+    snapshots every 4 steps on the full grid against the oracle."""
+    nt, snap = 16, 4
+    wl = inputs.c4(n=512, nt=nt, snap=snap)
+    rng = np.random.default_rng(9)
+    data = rng.standard_normal((nt, wl.rec.shape[0])).astype(np.float32)
+    model = seis.Model(_sgrid(wl), "acoustic", wl.model["vp"], rho=wl.model["rho"])
+    img = np.zeros((wl.nz, wl.ny, wl.nx), np.float32)
+    model.migrate(seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=snap), data, img)
+    model.close()
+    I = oracle.migrate(_ogrid(wl), "acoustic", wl.model["vp"], wl.model["rho"], wl.src, wl.wavelet,
+                       wl.rec, data.astype(np.float64), snap)
+    assert rel_l2(img, I) <= TOL_IMAGE
+
+
+def test_c5_decomposition_path_256():
+    """C5's z-slab path (halo exchange between slabs) at 256^3: P = 1, 2, 4, 8 slabs give
+    bitwise-identical seismograms and fields, and P = 1 matches the oracle (8 steps)."""
+    K = 8
+    wl = inputs.c2(n=256, nt=K)
+    outs = []
+    for P in (1, 2, 4, 8):
+        m = seis.Model(_sgrid(wl, slabs=P), "acoustic", wl.model["vp"], rho=wl.model["rho"])
+        shot = seis.Shot(wl.src, wl.wavelet, wl.rec)
+        sg = np.zeros((K, shot.nrec), np.float32)
+        m.forward_model(shot, sg)
+        outs.append((sg, m.get_field(0), m.get_field(3)))
+        m.close()
+    for o in outs[1:]:
+        for a, b in zip(o, outs[0]):
+            assert np.array_equal(a, b)
+    og = _ogrid(wl)
+    st = oracle.ac_state(og)
+    oracle.ac_run(og, wl.model["vp"], wl.model["rho"], st, 0, K, [wl.src], wl.wavelet[:, None])
+    assert rel_l2(outs[0][1], st["p"]) <= TOL_FIELD
