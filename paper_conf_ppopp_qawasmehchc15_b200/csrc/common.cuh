@@ -124,6 +124,44 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
+// Consumer release of TMA ring stage s.  With SEIS_WARP_RELEASE=1 every warp counts
+// itself out of the stage once it has finished reading it, and the LAST warp re-arms the stage
+// (expect_tx + TMA issue): no warp waits for the others (no CTA-wide barrier per plane).
+// Default (measured faster on B200, profiles/r01_sweep4_release.jsonl): __syncthreads, then
+// thread 0 re-arms.  `more` = a later plane uses stage s.
+#ifndef SEIS_WARP_RELEASE
+#define SEIS_WARP_RELEASE 0
+#endif
+template <class Refill>
+__device__ __forceinline__ void stage_release(uint32_t* cnt, int tid, bool more, Refill&& refill) {
+#if SEIS_WARP_RELEASE
+  __syncwarp();
+  if ((tid & 31) == 0) {
+    const uint32_t nwarps = (blockDim.x * blockDim.y * blockDim.z) >> 5;
+    __threadfence_block();  // this warp's reads of the stage are ordered before its count
+    if (atomicAdd(cnt, 1u) == nwarps - 1) {
+      atomicExch(cnt, 0u);
+      __threadfence_block();
+      if (more) {
+        fence_proxy_async();
+        refill();
+      }
+    }
+  }
+#else
+  __syncthreads();
+  if (tid == 0 && more) {
+    fence_proxy_async();
+    refill();
+  }
+#endif
+}
+// Fast reciprocal (MUFU.RCP, ~1 ulp; +inf -> +0) for the on-the-fly face/edge averages
+__device__ __forceinline__ float rcp_fast(float x) {
+  float r;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+  return r;
+}
 // 3D tile load: box origin (x, y, z) in padded element coordinates
 __device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, uint64_t* bar, int x, int y,
                                             int z) {

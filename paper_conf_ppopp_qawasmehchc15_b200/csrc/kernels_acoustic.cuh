@@ -27,10 +27,10 @@ struct CpmlAxis {
 };
 
 #ifndef SEIS_AC_NS
-#define SEIS_AC_NS 2
+#define SEIS_AC_NS 3
 #endif
 #ifndef SEIS_AC_VNS
-#define SEIS_AC_VNS 3
+#define SEIS_AC_VNS 2
 #endif
 constexpr int AC_NS = SEIS_AC_NS;    // P kernel ring depth
 constexpr int AC_VNS = SEIS_AC_VNS;  // V kernel ring depth
@@ -76,6 +76,7 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
   extern __shared__ __align__(128) float sm_raw[];
   float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[AC_VNS];
+  __shared__ uint32_t cnt[AC_VNS];
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX + tx;
   const int i0 = blockIdx.x * TXV, j0 = blockIdx.y * BY;
@@ -103,7 +104,10 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
     tma_load_3d(st + L::RZ, &a.mrz, &bar[s], x, y, z + 1);
   };
   if (tid == 0) {
-    for (int s = 0; s < AC_VNS; ++s) mbar_init(&bar[s], 1);
+    for (int s = 0; s < AC_VNS; ++s) {
+      mbar_init(&bar[s], 1);
+      cnt[s] = 0u;
+    }
     mbar_fence_init();
   }
   __syncthreads();
@@ -203,9 +207,9 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
         const float rxp = (x0 + e + 1 < d.nx) ? (e < 3 ? r0.v[e + 1] : rx5) : r0.v[e];
         const float ryp = (j + 1 < d.ny) ? ryn.v[e] : r0.v[e];
         const float rzp = zlast ? r0.v[e] : rz1.v[e];
-        const float bx = dth * (2.0f * __frcp_rn(r0.v[e] + rxp));
-        const float by = dth * (2.0f * __frcp_rn(r0.v[e] + ryp));
-        const float bz = dth * (2.0f * __frcp_rn(r0.v[e] + rzp));
+        const float bx = dth * (2.0f * rcp_fast(r0.v[e] + rxp));
+        const float by = dth * (2.0f * rcp_fast(r0.v[e] + ryp));
+        const float bz = dth * (2.0f * rcp_fast(r0.v[e] + rzp));
         ox.v[e] = fmaf(bx, dx[e], qxo.v[e]);
         oy.v[e] = fmaf(by, dy[e], qyo.v[e]);
         oz.v[e] = fmaf(bz, dz[e], qzo.v[e]);
@@ -222,11 +226,7 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
         st4_masked(a.img + cix, im, x0, d.nx, false);
       }
     }
-    __syncthreads();
-    if (tid == 0 && it + AC_VNS < np) {
-      fence_proxy_async();
-      issue(s, k + AC_VNS);
-    }
+    stage_release(&cnt[s], tid, it + AC_VNS < np, [&] { issue(s, k + AC_VNS); });
 #pragma unroll
     for (int t = 0; t < 7; ++t) r[t] = r[t + 1];
   }
@@ -268,6 +268,7 @@ __global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ 
   extern __shared__ __align__(128) float sm_raw[];
   float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[AC_NS];
+  __shared__ uint32_t cnt[AC_NS];
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX + tx;
   const int i0 = blockIdx.x * TXV, j0 = blockIdx.y * BY;
@@ -293,7 +294,10 @@ __global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ 
     tma_load_3d(st + L::QQ, &a.mqq, &bar[s], i0 + G, j0 + G, z + 3);
   };
   if (tid == 0) {
-    for (int s = 0; s < AC_NS; ++s) mbar_init(&bar[s], 1);
+    for (int s = 0; s < AC_NS; ++s) {
+      mbar_init(&bar[s], 1);
+      cnt[s] = 0u;
+    }
     mbar_fence_init();
   }
   __syncthreads();
@@ -394,11 +398,7 @@ __global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ 
       st4_masked(a.p + o, out, x0, d.nx, true);
       if (SNAP) st4_masked(a.snap + ((long long)k * d.ny + j) * d.nx + x0, out, x0, d.nx, (d.nx & 3) == 0);
     }
-    __syncthreads();
-    if (tid == 0 && it + AC_NS < np) {
-      fence_proxy_async();
-      issue(s, k + AC_NS);
-    }
+    stage_release(&cnt[s], tid, it + AC_NS < np, [&] { issue(s, k + AC_NS); });
 #pragma unroll
     for (int t = 0; t < 7; ++t) q[t] = q[t + 1];
   }

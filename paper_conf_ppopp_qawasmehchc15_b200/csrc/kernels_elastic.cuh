@@ -80,10 +80,12 @@ struct ElVArgs {
   CUtensorMap msyy;   // box 64 x (BY+8)  (y halo)
   CUtensorMap msyz;   // box 64 x (BY+8)
   CUtensorMap mv[3];  // vx, vy, vz, box 64 x BY
-  CUtensorMap mb[3];  // face buoyancies, box 64 x BY
+  CUtensorMap mr;     // rho tile, box (64+4) x (BY+1) (x+1, y+1 neighbours)
+  CUtensorMap mrz;    // rho interior at plane k+1, box 64 x BY
   CUtensorMap mq[3];  // z-queue feeds: sxz (k+3), syz (k+3), szz (k+4), box 64 x BY
   float* f[9];
   int W, zlo, fs;
+  float dth;       // dt / h (face buoyancy dt b/h = dth * 2/(rho_i + rho_{i+1}), O8/O9)
   CpmlAxis cx, cy, cz;
   float* psi[9];   // psi 0..8
   Dims d;
@@ -94,10 +96,11 @@ struct ElVArgs {
 
 template <int BY>
 struct ElVStage {
-  static constexpr int WX = TXE + 8, T = TXE * BY;
+  static constexpr int WX = TXE + 8, T = TXE * BY, RW = TXE + 4;
   static constexpr int XX = 0, XY = XX + BY * WX, XZ = XY + (BY + 8) * WX, YY = XZ + BY * WX,
-                       YZ = YY + (BY + 8) * TXE, V = YZ + (BY + 8) * TXE, B = V + 3 * T, Q = B + 3 * T,
-                       SIZE = Q + 3 * T;
+                       YZ = YY + (BY + 8) * TXE, V = YZ + (BY + 8) * TXE, RZ = V + 3 * T, Q = RZ + T,
+                       R = Q + 3 * T, SIZE = R + ((RW * (BY + 1) + 31) / 32) * 32;
+  static constexpr uint32_t BYTES = (R + RW * (BY + 1)) * 4;
   static constexpr size_t smem_bytes() { return (size_t)EL_VNS * SIZE * 4 + 128; }
 };
 
@@ -105,12 +108,15 @@ template <int BY, bool IMG>
 __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constant__ ElVArgs a) {
   using L = ElVStage<BY>;
   constexpr int WX = L::WX, T = L::T;
-  constexpr uint32_t TX_BYTES = L::SIZE * 4;
-  static_assert((L::XY % 32) == 0 && (L::XZ % 32) == 0 && (L::YY % 32) == 0 && (L::V % 32) == 0,
+  constexpr uint32_t TX_BYTES = L::BYTES;
+  constexpr int RW = L::RW;
+  static_assert((L::XY % 32) == 0 && (L::XZ % 32) == 0 && (L::YY % 32) == 0 && (L::V % 32) == 0 &&
+                    (L::R % 32) == 0,
                 "128-byte tiles");
   extern __shared__ __align__(128) float sm_raw[];
   float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[EL_VNS];
+  __shared__ uint32_t cnt[EL_VNS];
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX2 + tx;
   const int i0 = blockIdx.x * TXE, j0 = blockIdx.y * BY;
@@ -134,16 +140,18 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
     tma_load_3d(st + L::YY, &a.msyy, &bar[s], x, j0, z);
     tma_load_3d(st + L::YZ, &a.msyz, &bar[s], x, j0, z);
 #pragma unroll
-    for (int c = 0; c < 3; ++c) {
-      tma_load_3d(st + L::V + c * T, &a.mv[c], &bar[s], x, y, z);
-      tma_load_3d(st + L::B + c * T, &a.mb[c], &bar[s], x, y, z);
-    }
+    for (int c = 0; c < 3; ++c) tma_load_3d(st + L::V + c * T, &a.mv[c], &bar[s], x, y, z);
+    tma_load_3d(st + L::R, &a.mr, &bar[s], x, y, z);
+    tma_load_3d(st + L::RZ, &a.mrz, &bar[s], x, y, z + 1);
     tma_load_3d(st + L::Q, &a.mq[0], &bar[s], x, y, z + 3);
     tma_load_3d(st + L::Q + T, &a.mq[1], &bar[s], x, y, z + 3);
     tma_load_3d(st + L::Q + 2 * T, &a.mq[2], &bar[s], x, y, z + 4);
   };
   if (tid == 0) {
-    for (int s = 0; s < EL_VNS; ++s) mbar_init(&bar[s], 1);
+    for (int s = 0; s < EL_VNS; ++s) {
+      mbar_init(&bar[s], 1);
+      cnt[s] = 0u;
+    }
     mbar_fence_init();
   }
   __syncthreads();
@@ -249,13 +257,23 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
         psi_upd<2>(d8, a.psi[8], izz, oz8, cah, cbh);
       }
       const F2 v0 = lds2(st + L::V + pt), v1 = lds2(st + L::V + T + pt), v2 = lds2(st + L::V + 2 * T + pt);
-      const F2 b0 = lds2(st + L::B + pt), b1 = lds2(st + L::B + T + pt), b2 = lds2(st + L::B + 2 * T + pt);
+      // face buoyancy dt b/h = (dt/h) 2/(rho_i + rho_{i+1}), the last face clamps (O8, O9)
+      const float* rc = st + L::R + ty * RW + 2 * tx;
+      const F2 r0 = lds2(rc), ryn = lds2(rc + RW), rzn = lds2(st + L::RZ + pt);
+      const float rx2 = rc[2];
+      const bool zlast = k + d.z0 + 1 >= d.nz;
       F2 ov[3];
 #pragma unroll
       for (int e = 0; e < 2; ++e) {
-        ov[0].v[e] = fmaf(b0.v[e], (d0[e] + d1[e]) + d2[e], v0.v[e]);
-        ov[1].v[e] = fmaf(b1.v[e], (d3[e] + d4[e]) + d5[e], v1.v[e]);
-        ov[2].v[e] = fmaf(b2.v[e], (d6[e] + d7[e]) + d8[e], v2.v[e]);
+        const float rxp = (x0 + e + 1 < d.nx) ? (e == 0 ? r0.v[1] : rx2) : r0.v[e];
+        const float ryp = (j + 1 < d.ny) ? ryn.v[e] : r0.v[e];
+        const float rzp = zlast ? r0.v[e] : rzn.v[e];
+        const float bx = a.dth * (2.0f * rcp_fast(r0.v[e] + rxp));
+        const float by = a.dth * (2.0f * rcp_fast(r0.v[e] + ryp));
+        const float bz = a.dth * (2.0f * rcp_fast(r0.v[e] + rzp));
+        ov[0].v[e] = fmaf(bx, (d0[e] + d1[e]) + d2[e], v0.v[e]);
+        ov[1].v[e] = fmaf(by, (d3[e] + d4[e]) + d5[e], v1.v[e]);
+        ov[2].v[e] = fmaf(bz, (d6[e] + d7[e]) + d8[e], v2.v[e]);
       }
 #pragma unroll
       for (int c = 0; c < 3; ++c) st2_masked(a.f[EVX + c] + o, ov[c], x0, d.nx);
@@ -269,11 +287,7 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
           }
       }
     }
-    __syncthreads();
-    if (tid == 0 && it + EL_VNS < np) {
-      fence_proxy_async();
-      issue(s, k + EL_VNS);
-    }
+    stage_release(&cnt[s], tid, it + EL_VNS < np, [&] { issue(s, k + EL_VNS); });
 #pragma unroll
     for (int t = 0; t < 7; ++t) {
       qxz[t] = qxz[t + 1];
@@ -286,7 +300,8 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
 struct ElSArgs {
   CUtensorMap mvt[3];  // vx, vy, vz tiles, box 72 x (BY+8)
   CUtensorMap ms[6];   // sxx, syy, szz, sxy, sxz, syz, box 64 x BY
-  CUtensorMap mc[5];   // l2m, lam, mxy, mxz, myz, box 64 x BY
+  CUtensorMap ml2m;    // dt (lam + 2 mu) / h, box 64 x BY
+  CUtensorMap mw;      // w = h / (dt mu) (+inf where mu = 0), box (64+4) x (BY+1), planes k, k+1
   CUtensorMap mq[3];   // z-queue feeds: vx (k+4), vy (k+4), vz (k+3), box 64 x BY
   float* f[9];
   int W, zlo, fs;
@@ -301,19 +316,25 @@ struct ElSArgs {
 
 template <int BY>
 struct ElSStage {
-  static constexpr int WX = TXE + 8, T = TXE * BY, TV = (BY + 8) * WX;
-  static constexpr int VT = 0, S = 3 * TV, C = S + 6 * T, Q = C + 5 * T, SIZE = Q + 3 * T;
+  static constexpr int WX = TXE + 8, T = TXE * BY, TV = (BY + 8) * WX, RW = TXE + 4;
+  static constexpr int WT = ((RW * (BY + 1) + 31) / 32) * 32;
+  static constexpr int VT = 0, S = 3 * TV, C = S + 6 * T, Q = C + T, WK = Q + 3 * T, WK1 = WK + WT,
+                       SIZE = WK1 + WT;
+  static constexpr uint32_t BYTES = (WK + 2 * RW * (BY + 1)) * 4;  // bytes the TMA boxes deliver
   static constexpr size_t smem_bytes() { return (size_t)EL_SNS * SIZE * 4 + 128; }
 };
 
 template <int BY, bool SNAP>
 __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constant__ ElSArgs a) {
   using L = ElSStage<BY>;
-  constexpr int WX = L::WX, T = L::T, TV = L::TV;
-  constexpr uint32_t TX_BYTES = L::SIZE * 4;
+  constexpr int WX = L::WX, T = L::T, TV = L::TV, RW = L::RW;
+  constexpr uint32_t TX_BYTES = L::BYTES;
+  static_assert((L::S % 32) == 0 && (L::C % 32) == 0 && (L::WK % 32) == 0 && (L::WK1 % 32) == 0,
+                "128-byte tiles");
   extern __shared__ __align__(128) float sm_raw[];
   float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[EL_SNS];
+  __shared__ uint32_t cnt[EL_SNS];
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX2 + tx;
   const int i0 = blockIdx.x * TXE, j0 = blockIdx.y * BY;
@@ -335,14 +356,18 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
     for (int c = 0; c < 3; ++c) tma_load_3d(st + L::VT + c * TV, &a.mvt[c], &bar[s], i0, j0, z);
 #pragma unroll
     for (int c = 0; c < 6; ++c) tma_load_3d(st + L::S + c * T, &a.ms[c], &bar[s], x, y, z);
-#pragma unroll
-    for (int c = 0; c < 5; ++c) tma_load_3d(st + L::C + c * T, &a.mc[c], &bar[s], x, y, z);
+    tma_load_3d(st + L::C, &a.ml2m, &bar[s], x, y, z);
+    tma_load_3d(st + L::WK, &a.mw, &bar[s], x, y, z);
+    tma_load_3d(st + L::WK1, &a.mw, &bar[s], x, y, z + 1);
     tma_load_3d(st + L::Q, &a.mq[0], &bar[s], x, y, z + 4);
     tma_load_3d(st + L::Q + T, &a.mq[1], &bar[s], x, y, z + 4);
     tma_load_3d(st + L::Q + 2 * T, &a.mq[2], &bar[s], x, y, z + 3);
   };
   if (tid == 0) {
-    for (int s = 0; s < EL_SNS; ++s) mbar_init(&bar[s], 1);
+    for (int s = 0; s < EL_SNS; ++s) {
+      mbar_init(&bar[s], 1);
+      cnt[s] = 0u;
+    }
     mbar_fence_init();
   }
   __syncthreads();
@@ -451,17 +476,34 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
         psi_upd<2>(dzvx, a.psi[5], izz, oz5, cah, cbh);
         psi_upd<2>(dzvy, a.psi[7], izz, oz7, cah, cbh);
       }
-      F2 sv[6], cv[5];
+      F2 sv[6];
 #pragma unroll
       for (int c = 0; c < 6; ++c) sv[c] = lds2(st + L::S + c * T + pt);
+      const F2 cl2m = lds2(st + L::C + pt);
+      // node w = h/(dt mu) at planes k (wa) and k+1 (wb), rows j (…0) and j+1 (…1), columns
+      // x0, x0+1, x0+2; neighbours past the last node clamp to it (O9)
+      const float* pa = st + L::WK + ty * RW + 2 * tx;
+      const float* pb = st + L::WK1 + ty * RW + 2 * tx;
+      const bool ylast = j + 1 >= d.ny, zlast = gz + 1 >= d.nz;
+      float wa0[3], wa1[3], wb0[3], wb1[3];
 #pragma unroll
-      for (int c = 0; c < 5; ++c) cv[c] = lds2(st + L::C + c * T + pt);
+      for (int c = 0; c < 3; ++c) {
+        const int cx = (x0 + c < d.nx) ? c : (c > 0 ? c - 1 : 0);
+        wa0[c] = pa[cx];
+        wa1[c] = ylast ? wa0[c] : pa[RW + cx];
+        wb0[c] = zlast ? wa0[c] : pb[cx];
+        wb1[c] = zlast ? wa1[c] : (ylast ? wb0[c] : pb[RW + cx]);
+      }
       const bool surf = a.fs && gz == 0;
       const long long rel = srel0 - (long long)(k + GZ) * PS;
       F2 o6[6];
 #pragma unroll
       for (int e = 0; e < 2; ++e) {
-        const float l2m = cv[0].v[e], lam = cv[1].v[e];
+        // edge mu = harmonic mean of its 4 nodes, 0 if any is 0 (w = inf) (O9); lam = l2m - 2 mu
+        const float mxy = 4.0f * rcp_fast((wa0[e] + wa0[e + 1]) + (wa1[e] + wa1[e + 1]));
+        const float mxz = 4.0f * rcp_fast((wa0[e] + wa0[e + 1]) + (wb0[e] + wb0[e + 1]));
+        const float myz = 4.0f * rcp_fast((wa0[e] + wa1[e]) + (wb0[e] + wb1[e]));
+        const float l2m = cl2m.v[e], lam = l2m - 2.0f * rcp_fast(wa0[e]);
         float ez = ezz[e];
         if (surf) ez = -(lam / l2m) * (exx[e] + eyy[e]);  // O16 surface row
         float sxx = sv[0].v[e] + fmaf(l2m, exx[e], lam * (eyy[e] + ez));
@@ -476,9 +518,9 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
         o6[0].v[e] = sxx;
         o6[1].v[e] = syy;
         o6[2].v[e] = szz;
-        o6[3].v[e] = fmaf(cv[2].v[e], dyvx[e] + dxvy[e], sv[3].v[e]);
-        o6[4].v[e] = fmaf(cv[3].v[e], dzvx[e] + dxvz[e], sv[4].v[e]);
-        o6[5].v[e] = fmaf(cv[4].v[e], dzvy[e] + dyvz[e], sv[5].v[e]);
+        o6[3].v[e] = fmaf(mxy, dyvx[e] + dxvy[e], sv[3].v[e]);
+        o6[4].v[e] = fmaf(mxz, dzvx[e] + dxvz[e], sv[4].v[e]);
+        o6[5].v[e] = fmaf(myz, dzvy[e] + dyvz[e], sv[5].v[e]);
       }
 #pragma unroll
       for (int c = 0; c < 6; ++c) st2_masked(a.f[ESXX + c] + o, o6[c], x0, d.nx);
@@ -489,11 +531,7 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
           if (x0 + e < d.nx) a.snap[cix + e] = -((o6[0].v[e] + o6[1].v[e]) + o6[2].v[e]) / 3.0f;
       }
     }
-    __syncthreads();
-    if (tid == 0 && it + EL_SNS < np) {
-      fence_proxy_async();
-      issue(s, k + EL_SNS);
-    }
+    stage_release(&cnt[s], tid, it + EL_SNS < np, [&] { issue(s, k + EL_SNS); });
 #pragma unroll
     for (int t = 0; t < 7; ++t) {
       qx[t] = qx[t + 1];

@@ -59,6 +59,7 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
   extern __shared__ __align__(128) float sm_raw[];
   float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[ISO_NS];
+  __shared__ uint32_t cnt[ISO_NS];
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX + tx;
   const int i0 = blockIdx.x * TXV, j0 = blockIdx.y * BY;
@@ -79,7 +80,10 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
     tma_load_3d(st + L::UQ, &a.muq, &bar[s], i0 + G, j0 + G, k + 4 + GZ);
   };
   if (tid == 0) {
-    for (int s = 0; s < ISO_NS; ++s) mbar_init(&bar[s], 1);
+    for (int s = 0; s < ISO_NS; ++s) {
+      mbar_init(&bar[s], 1);
+      cnt[s] = 0u;
+    }
     mbar_fence_init();
   }
   __syncthreads();
@@ -166,11 +170,7 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
         }
       }
     }
-    __syncthreads();  // every thread is done with stage s
-    if (tid == 0 && it + ISO_NS < np) {
-      fence_proxy_async();
-      issue(s, k + ISO_NS);
-    }
+    stage_release(&cnt[s], tid, it + ISO_NS < np, [&] { issue(s, k + ISO_NS); });
 #pragma unroll
     for (int t = 0; t < 8; ++t) q[t] = q[t + 1];
   }

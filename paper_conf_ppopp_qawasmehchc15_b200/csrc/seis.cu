@@ -115,7 +115,7 @@ namespace {
 #define SEIS_BYV 8
 #endif
 #ifndef SEIS_BYP
-#define SEIS_BYP 16
+#define SEIS_BYP 8
 #endif
 #ifndef SEIS_BYE
 #define SEIS_BYE 8
@@ -132,16 +132,15 @@ struct Slab {
   float* m = nullptr;        // ISO
   float* kdt = nullptr;      // ACOUSTIC dt K / h
   float* rho = nullptr;      // ACOUSTIC density (z ghosts filled from the neighbour slabs)
-  float *bx = nullptr, *by = nullptr, *bz = nullptr;                          // ACOUSTIC, ELASTIC
-  float *l2m = nullptr, *lam = nullptr, *mxy = nullptr, *mxz = nullptr, *myz = nullptr;  // ELASTIC
+  float *l2m = nullptr, *wmu = nullptr;  // ELASTIC: dt (lam + 2 mu) / h and h / (dt mu)
   float* psi[NPSI] = {};
   // TMA descriptors of every operand tile the kernels stage:
   // "t" = tile with x/y halo, "c" = interior (centre) tile 32 x BY
   CUtensorMap iso_ut[2], iso_uc[2], iso_m;                              // ISO
   CUtensorMap ac_pt, ac_qc[3], ac_rt, ac_rc, ac_pc;        // ACOUSTIC V
   CUtensorMap ac_qxt, ac_qyt, ac_ppc, ac_qzc, ac_kc;        // ACOUSTIC P
-  CUtensorMap el_sxxt, el_sxyt, el_sxzt, el_syyt, el_syzt, el_vc[3], el_bc[3];  // ELASTIC V
-  CUtensorMap el_vt[3], el_sc[6], el_cc[5];                             // ELASTIC S
+  CUtensorMap el_sxxt, el_sxyt, el_sxzt, el_syyt, el_syzt, el_vc[3], el_rt, el_rc;  // ELASTIC V
+  CUtensorMap el_vt[3], el_sc[6], el_l2m, el_w;                           // ELASTIC S
   int cur = 0;               // ISO: fld[cur] = u^n
   int zc = 1, nzch = 1;      // z-chunking of the stencil launches
   // shot tables
@@ -550,41 +549,15 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     if (vs && (!(vs[t] >= 0.f) || 2.0 * (double)vs[t] * vs[t] > (double)vp[t] * vp[t]))
       return fail(SEIS_EINVAL, "vs must satisfy 0 <= vs <= vp/sqrt(2) (index %zu)", t);
   }
-  // the next rank's first plane (z-face coefficients need rho / mu at k+1)
-  std::vector<float> nvp, nvs, nrho;
+  // (rho / w at k+1 across rank faces come from the ghost-plane exchange after the upload)
   if (M->comm && M->nranks > 1) {
     float* dv = nullptr;
     CK(cudaMalloc(&dv, sizeof(double)));
     CK(cudaMemcpy(dv, &vmax, sizeof(double), cudaMemcpyHostToDevice));
     NK(ncclAllReduce(dv, dv, 1, ncclFloat64, ncclMax, M->comm->nccl, st));
+    CK(cudaStreamSynchronize(st));
     CK(cudaMemcpy(&vmax, dv, sizeof(double), cudaMemcpyDeviceToHost));
     CK(cudaFree(dv));
-    float* send = nullptr;
-    float* recv = nullptr;
-    CK(cudaMalloc(&send, 3 * plane * sizeof(float)));
-    CK(cudaMalloc(&recv, 3 * plane * sizeof(float)));
-    CK(cudaMemcpy(send, vp, plane * sizeof(float), cudaMemcpyHostToDevice));
-    if (rho) CK(cudaMemcpy(send + plane, rho, plane * sizeof(float), cudaMemcpyHostToDevice));
-    if (vs) CK(cudaMemcpy(send + 2 * plane, vs, plane * sizeof(float), cudaMemcpyHostToDevice));
-    NK(ncclGroupStart());
-    if (M->rank > 0) NK(ncclSend(send, 3 * plane, ncclFloat, M->rank - 1, M->comm->nccl, st));
-    if (M->rank < M->nranks - 1) NK(ncclRecv(recv, 3 * plane, ncclFloat, M->rank + 1, M->comm->nccl, st));
-    NK(ncclGroupEnd());
-    CK(cudaStreamSynchronize(st));
-    if (M->rank < M->nranks - 1) {
-      nvp.resize(plane);
-      CK(cudaMemcpy(nvp.data(), recv, plane * sizeof(float), cudaMemcpyDeviceToHost));
-      if (rho) {
-        nrho.resize(plane);
-        CK(cudaMemcpy(nrho.data(), recv + plane, plane * sizeof(float), cudaMemcpyDeviceToHost));
-      }
-      if (vs) {
-        nvs.resize(plane);
-        CK(cudaMemcpy(nvs.data(), recv + 2 * plane, plane * sizeof(float), cudaMemcpyDeviceToHost));
-      }
-    }
-    CK(cudaFree(send));
-    CK(cudaFree(recv));
   }
   M->vmax = vmax;
   const double vdt_h = vmax * (double)g.dt / (double)g.h;
@@ -670,16 +643,6 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     S.fld.resize(nfields(kind));
     for (auto& f : S.fld) TRY(alloc_padded(M, d, &f, st));
     // per-point coefficients (double -> fp32), compact then padded on device
-    auto val = [&](const std::vector<float>& v, const std::vector<float>& nextp, size_t li, int i,
-                   int j, int k /*local to slab*/) -> double {
-      // value at slab-local (i, j, k) with the grid-edge clamp; k may be lnz (next plane)
-      const int gk = d.z0 + k;
-      if (gk >= g.nz) return v[off + ((size_t)(k - 1) * g.ny + j) * g.nx + i];
-      const int pk = lz0 + k;  // process-local plane
-      if (pk < M->pnzl) return v[((size_t)pk * g.ny + j) * g.nx + i];
-      return nextp[(size_t)j * g.nx + i];
-      (void)li;
-    };
     std::vector<float> hc(sp);
     if (kind == SEIS_ISO) {
       for (size_t t = 0; t < sp; ++t) {
@@ -688,71 +651,30 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       }
       TRY(upload_padded_from_host(M, d, hc, &S.m, st));
     } else {
-      // buoyancy on faces (O8): dt * 2/(rho_i + rho_{i+1}) / h, last face clamps
-      // (ELASTIC; the acoustic V kernel evaluates it on the fly from rho)
-      for (int ax = 0; ax < 3 && kind == SEIS_ELASTIC; ++ax) {
-        for (int k = 0; k < lnz; ++k)
-          for (int j = 0; j < g.ny; ++j)
-            for (int i = 0; i < g.nx; ++i) {
-              const double r0 = val(M->hrho, nrho, 0, i, j, k);
-              int i1 = i, j1 = j, k1 = k;
-              if (ax == 0) i1 = std::min(i + 1, g.nx - 1);
-              if (ax == 1) j1 = std::min(j + 1, g.ny - 1);
-              if (ax == 2) k1 = k + 1;
-              const double r1 = val(M->hrho, nrho, 0, i1, j1, k1);
-              hc[((size_t)k * g.ny + j) * g.nx + i] = (float)(dt * (2.0 / (r0 + r1)) / h);
-            }
-        float** dst = ax == 0 ? &S.bx : (ax == 1 ? &S.by : &S.bz);
-        TRY(upload_padded_from_host(M, d, hc, dst, st));
-      }
+      // buoyancy on faces (O8): both V kernels evaluate dt 2/(rho_i + rho_{i+1}) / h on the
+      // fly from rho, whose z-ghost planes are exchanged once below
+      for (size_t q = 0; q < sp; ++q) hc[q] = M->hrho[off + q];
+      TRY(upload_padded_from_host(M, d, hc, &S.rho, st));
       if (kind == SEIS_ACOUSTIC) {
         for (size_t t = 0; t < sp; ++t) {
           const double v = M->hvp[off + t], r = M->hrho[off + t];
           hc[t] = (float)(dt * r * v * v / h);
         }
         TRY(upload_padded_from_host(M, d, hc, &S.kdt, st));
-        for (size_t t = 0; t < sp; ++t) hc[t] = M->hrho[off + t];
-        TRY(upload_padded_from_host(M, d, hc, &S.rho, st));
       } else {
-        auto mu_at = [&](int i, int j, int k) {
-          const double s_ = val(M->hvs, nvs, 0, i, j, k), r_ = val(M->hrho, nrho, 0, i, j, k);
-          return r_ * s_ * s_;
-        };
         for (size_t t = 0; t < sp; ++t) {
           const double v = M->hvp[off + t], s_ = M->hvs[off + t], r = M->hrho[off + t];
           hc[t] = (float)(dt * r * v * v / h);  // lambda + 2 mu = rho vp^2
         }
         TRY(upload_padded_from_host(M, d, hc, &S.l2m, st));
+        // w = h / (dt mu) at nodes (+inf where mu = 0): the S kernel forms the edge mu of O9
+        // (harmonic mean of 4 nodes, 0 if any is 0) as 4 / (w0 + w1 + w2 + w3) and
+        // dt lam / h = dt (lam + 2 mu) / h - 2 / w; its z-ghost planes are exchanged below
         for (size_t t = 0; t < sp; ++t) {
-          const double v = M->hvp[off + t], s_ = M->hvs[off + t], r = M->hrho[off + t];
-          hc[t] = (float)(dt * r * (v * v - 2.0 * s_ * s_) / h);
+          const double s_ = M->hvs[off + t], r = M->hrho[off + t], mu = r * s_ * s_;
+          hc[t] = mu > 0 ? (float)(h / (dt * mu)) : INFINITY;
         }
-        TRY(upload_padded_from_host(M, d, hc, &S.lam, st));
-        // edge mu: harmonic mean of the 4 adjacent node values, 0 if any is 0 (O9)
-        const int pairs[3][2] = {{0, 1}, {0, 2}, {1, 2}};
-        for (int e = 0; e < 3; ++e) {
-          for (int k = 0; k < lnz; ++k)
-            for (int j = 0; j < g.ny; ++j)
-              for (int i = 0; i < g.nx; ++i) {
-                int di[3] = {0, 0, 0}, dj[3] = {0, 0, 0};
-                di[pairs[e][0]] = 1;
-                dj[pairs[e][1]] = 1;
-                auto cl = [&](int ii, int jj, int kk) {
-                  ii = std::min(ii, g.nx - 1);
-                  jj = std::min(jj, g.ny - 1);
-                  return mu_at(ii, jj, kk);
-                };
-                const double m0 = cl(i, j, k);
-                const double m1 = cl(i + di[0], j + di[1], k + di[2]);
-                const double m2 = cl(i + dj[0], j + dj[1], k + dj[2]);
-                const double m3 = cl(i + di[0] + dj[0], j + di[1] + dj[1], k + di[2] + dj[2]);
-                double me = 0.0;
-                if (m0 > 0 && m1 > 0 && m2 > 0 && m3 > 0) me = 4.0 / (1 / m0 + 1 / m1 + 1 / m2 + 1 / m3);
-                hc[((size_t)k * g.ny + j) * g.nx + i] = (float)(dt * me / h);
-              }
-          float** dst = e == 0 ? &S.mxy : (e == 1 ? &S.mxz : &S.myz);
-          TRY(upload_padded_from_host(M, d, hc, dst, st));
-        }
+        TRY(upload_padded_from_host(M, d, hc, &S.wmu, st));
       }
       // compact C-PML memory slabs
       if (M->W > 0) {
@@ -794,15 +716,15 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       TRY(make_map(&S.el_sxzt, S.fld[ESXZ], d, TXE + 8, BYE));
       TRY(make_map(&S.el_syyt, S.fld[ESYY], d, TXE, BYE + 8));
       TRY(make_map(&S.el_syzt, S.fld[ESYZ], d, TXE, BYE + 8));
-      float* bb[3] = {S.bx, S.by, S.bz};
+      TRY(make_map(&S.el_rt, S.rho, d, TXE + 4, BYE + 1));
+      TRY(make_map(&S.el_rc, S.rho, d, TXE, BYE));
       for (int t = 0; t < 3; ++t) {
         TRY(make_map(&S.el_vc[t], S.fld[EVX + t], d, TXE, BYE));
-        TRY(make_map(&S.el_bc[t], bb[t], d, TXE, BYE));
         TRY(make_map(&S.el_vt[t], S.fld[EVX + t], d, TXE + 8, BYE + 8));
       }
       for (int t = 0; t < 6; ++t) TRY(make_map(&S.el_sc[t], S.fld[ESXX + t], d, TXE, BYE));
-      float* cc[5] = {S.l2m, S.lam, S.mxy, S.mxz, S.myz};
-      for (int t = 0; t < 5; ++t) TRY(make_map(&S.el_cc[t], cc[t], d, TXE, BYE));
+      TRY(make_map(&S.el_l2m, S.l2m, d, TXE, BYE));
+      TRY(make_map(&S.el_w, S.wmu, d, TXE + 4, BYE + 1));
     }
     TRY(set_smem_attrs());
     int occ = 1;
@@ -820,6 +742,8 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
   }
   if (kind == SEIS_ACOUSTIC)  // rho(k+1) across slab faces
     TRY(exchange_arrays(M, {[](Slab& S) { return S.rho; }}, 4, st));
+  if (kind == SEIS_ELASTIC)  // rho(k+1), w(k+1) across slab faces
+    TRY(exchange_arrays(M, {[](Slab& S) { return S.rho; }, [](Slab& S) { return S.wmu; }}, 4, st));
   CK(cudaStreamSynchronize(st));
   return SEIS_OK;
 }
@@ -882,7 +806,7 @@ seis_status seis_memory_required(const seis_grid* g, seis_kind kind, const seis_
   seis_slab_bounds(g->nz, nranks, 0, &z0, &nzl);
   const Dims d = make_dims(*g, 0, nzl);
   const double padded = (double)d.PS * (nzl + 2 * GZ) * 4.0;
-  int nf = nfields(kind), np = kind == SEIS_ISO ? 1 : (kind == SEIS_ACOUSTIC ? 4 : 8);
+  int nf = nfields(kind), np = kind == SEIS_ISO ? 1 : (kind == SEIS_ACOUSTIC ? 2 : 3);  // m | kdt,rho | l2m,w,rho
   double b = (nf + np) * padded;
   if (kind != SEIS_ISO && g->nb > 0) {
     const double W = g->nb + 1;
@@ -1201,9 +1125,11 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     a.msxz = S.el_sxzt;
     a.msyy = S.el_syyt;
     a.msyz = S.el_syzt;
+    a.mr = S.el_rt;
+    a.mrz = S.el_rc;
+    a.dth = (float)((double)M->g.dt / (double)M->g.h);
     for (int t = 0; t < 3; ++t) {
       a.mv[t] = S.el_vc[t];
-      a.mb[t] = S.el_bc[t];
     }
     a.mq[0] = S.el_sc[ESXZ - ESXX];
     a.mq[1] = S.el_sc[ESYZ - ESXX];
@@ -1235,7 +1161,8 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     ElSArgs a;
     for (int t = 0; t < 3; ++t) a.mvt[t] = S.el_vt[t];
     for (int t = 0; t < 6; ++t) a.ms[t] = S.el_sc[t];
-    for (int t = 0; t < 5; ++t) a.mc[t] = S.el_cc[t];
+    a.ml2m = S.el_l2m;
+    a.mw = S.el_w;
     for (int t = 0; t < 3; ++t) a.mq[t] = S.el_vc[t];
     for (int t = 0; t < 9; ++t) a.f[t] = S.fld[t];
     a.W = M->W;

@@ -19,11 +19,12 @@ sys.path.insert(0, ROOT)
 
 VARIANTS = {
     "base": [],
-    "t128_4": ["SEIS_TXV=128", "SEIS_BYI=4", "SEIS_BYV=4", "SEIS_BYP=8"],
-    "t128_8": ["SEIS_TXV=128", "SEIS_BYI=8", "SEIS_BYV=8", "SEIS_BYP=8"],
-    "t128_4ns": ["SEIS_TXV=128", "SEIS_BYI=4", "SEIS_BYV=4", "SEIS_BYP=8", "SEIS_ISO_NS=4",
-                 "SEIS_AC_VNS=4", "SEIS_AC_NS=3"],
-    "t128_p4": ["SEIS_TXV=128", "SEIS_BYI=4", "SEIS_BYV=4", "SEIS_BYP=4", "SEIS_AC_NS=3"],
+    "p8_4": ["SEIS_AC_NS=4"],
+    "p4_4": ["SEIS_BYP=4", "SEIS_AC_NS=4"],
+    "p4_3": ["SEIS_BYP=4"],
+    "p8_2": ["SEIS_AC_NS=2"],
+    "v4_3": ["SEIS_BYV=4", "SEIS_AC_VNS=3"],
+    "v16_1": ["SEIS_BYV=16", "SEIS_AC_VNS=1"],
 }
 
 
