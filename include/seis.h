@@ -90,6 +90,16 @@ typedef struct {
   int32_t rec_component;     /* ELASTIC: 0 vx, 1 vy, 2 vz, 3 pressure -(sxx+syy+szz)/3 (O13);
                                 ignored for ISO (records u) and ACOUSTIC (records p) */
   int32_t snap_period;       /* >= 1: snapshot + imaging cadence (RTM only, O14) */
+  int32_t ckpt_period;       /* RTM source-wavefield storage ("simulates the source
+                                wave-field in both the forward and backward phases"):
+                                0  = every snapshot S_j kept in the HBM pool (O14);
+                                c >= 1 = checkpointing: snapshots are grouped in segments of c; the
+                                forward phase keeps only the full source state (fields incl. ghost
+                                planes + C-PML memory) at the start of segments 1.., and the last
+                                segment's snapshots; the backward phase recomputes each earlier
+                                segment's snapshots from its checkpoint just before they are imaged
+                                (one extra forward pass at most).  Results are bitwise identical to
+                                c = 0 (same kernels, same order of operations). */
 } seis_shot;
 
 /* ---- multi-GPU (one process per GPU; z-slab decomposition, §8e) ---- */
@@ -139,8 +149,10 @@ seis_status seis_forward_model(seis_model* model, const seis_shot* shot, float* 
  * -(sxx+syy+szz)/3 (receivers inject like the explosive source).
  *   data  host or device [nt][nrec] fp32 observed data (replicated on every rank)
  *   image host or device [nz_local][ny][nx] fp32, ACCUMULATED (+=), never zeroed
- * Snapshot pool: nsnap = (nt-1)/snap_period fields of nz_local*ny*nx floats in HBM;
- * SEIS_ENOMEM (with the byte count in seis_last_error) if it does not fit. */
+ * Snapshot pool: nsnap = (nt-1)/snap_period fields of nz_local*ny*nx floats in HBM
+ * (ckpt_period = 0), or min(c, nsnap) snapshot fields + (ceil(nsnap/c) - 1) source-state
+ * checkpoints (ckpt_period = c); SEIS_ENOMEM (with the byte count in seis_last_error) if
+ * it does not fit. */
 seis_status seis_migrate(seis_model* model, const seis_shot* shot, const float* data,
                          float* image, void* stream);
 

@@ -56,7 +56,7 @@ class _CShot(C.Structure):
     _fields_ = [("sx", C.c_int32), ("sy", C.c_int32), ("sz", C.c_int32),
                 ("wavelet", C.POINTER(C.c_float)), ("nt", C.c_int32), ("nrec", C.c_int32),
                 ("rec", C.POINTER(C.c_int32)), ("rec_component", C.c_int32),
-                ("snap_period", C.c_int32)]
+                ("snap_period", C.c_int32), ("ckpt_period", C.c_int32)]
 
 
 _lib = None
@@ -129,13 +129,15 @@ class Shot:
     rec: np.ndarray              # host int32 [nrec][3] (x, y, z)
     rec_component: int = 2
     snap_period: int = 1
+    ckpt_period: int = 0         # RTM: 0 = all snapshots in HBM; c >= 1 = checkpointed segments of c
 
     def c(self):
         w = np.ascontiguousarray(self.wavelet, dtype=np.float32)
         r = np.ascontiguousarray(np.asarray(self.rec, dtype=np.int32).reshape(-1, 3))
         cs = _CShot(int(self.src[0]), int(self.src[1]), int(self.src[2]),
                     w.ctypes.data_as(C.POINTER(C.c_float)), w.shape[0], r.shape[0],
-                    r.ctypes.data_as(C.POINTER(C.c_int32)), self.rec_component, self.snap_period)
+                    r.ctypes.data_as(C.POINTER(C.c_int32)), self.rec_component, self.snap_period,
+                    self.ckpt_period)
         return cs, (w, r)
 
     @property

@@ -55,6 +55,7 @@ struct AcVArgs {
   float* __restrict__ psz;        // psi_{p,z} [2W][ny][nx] (global z slots)
   Dims d;
   int zc;
+  int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   const float* __restrict__ imgS; // imaging: img += S * p (input level), or nullptr
   float* __restrict__ img;
 };
@@ -81,7 +82,7 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX + tx;
   const int i0 = blockIdx.x * TXV, j0 = blockIdx.y * BY;
   const int x0 = i0 + 4 * tx, j = j0 + ty;
-  const int k0 = blockIdx.z * a.zc;
+  const int k0 = (a.ch0 + (int)blockIdx.z * a.chs) * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
   const int np = k1 - k0;
   const bool own = (x0 < d.nx) && (j < d.ny);
@@ -248,6 +249,7 @@ struct AcPArgs {
   float* __restrict__ pqz;        // psi_{q,z} [2W][ny][nx]
   Dims d;
   int zc;
+  int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   long long src_o;                // padded index of the source in this slab, -1 = none
   float src_amp;                  // dt K_s / h^3 * s[n]
   float* __restrict__ snap;       // compact snapshot target, or nullptr
@@ -273,7 +275,7 @@ __global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ 
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX + tx;
   const int i0 = blockIdx.x * TXV, j0 = blockIdx.y * BY;
   const int x0 = i0 + 4 * tx, j = j0 + ty;
-  const int k0 = blockIdx.z * a.zc;
+  const int k0 = (a.ch0 + (int)blockIdx.z * a.chs) * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
   const int np = k1 - k0;
   const bool own = (x0 < d.nx) && (j < d.ny);

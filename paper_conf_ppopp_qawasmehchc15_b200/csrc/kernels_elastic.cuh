@@ -90,6 +90,7 @@ struct ElVArgs {
   float* psi[9];   // psi 0..8
   Dims d;
   int zc;
+  int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   const float* __restrict__ imgS;  // elastic RTM (f3): img += S * P on the input level, P = -(sxx+syy+szz)/3
   float* __restrict__ img;
 };
@@ -121,7 +122,7 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX2 + tx;
   const int i0 = blockIdx.x * TXE, j0 = blockIdx.y * BY;
   const int x0 = i0 + 2 * tx, j = j0 + ty;
-  const int k0 = blockIdx.z * a.zc;
+  const int k0 = (a.ch0 + (int)blockIdx.z * a.chs) * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
   const int np = k1 - k0;
   const bool own = (x0 < d.nx) && (j < d.ny);
@@ -309,6 +310,7 @@ struct ElSArgs {
   float* psi[9];   // psi 9..17
   Dims d;
   int zc;
+  int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   long long src_o;
   float src_amp;   // dt (lam + 2/3 mu)_s / h^3 * s[n]
   float* __restrict__ snap;  // elastic RTM (f3): snapshot of P = -(sxx+syy+szz)/3, or nullptr
@@ -339,7 +341,7 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX2 + tx;
   const int i0 = blockIdx.x * TXE, j0 = blockIdx.y * BY;
   const int x0 = i0 + 2 * tx, j = j0 + ty;
-  const int k0 = blockIdx.z * a.zc;
+  const int k0 = (a.ch0 + (int)blockIdx.z * a.chs) * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
   const int np = k1 - k0;
   const bool own = (x0 < d.nx) && (j < d.ny);

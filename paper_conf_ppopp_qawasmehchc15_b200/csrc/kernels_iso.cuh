@@ -32,6 +32,7 @@ struct IsoArgs {
   const float* __restrict__ edz;
   Dims d;
   int zc;                        // z-chunk length
+  int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   long long src_o;               // padded index of the source node in this slab, -1 = none
   float src_amp;                 // scale * s[n]
   float* __restrict__ snap;      // compact [nzl][ny][nx] or nullptr
@@ -64,7 +65,7 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX + tx;
   const int i0 = blockIdx.x * TXV, j0 = blockIdx.y * BY;
   const int x0 = i0 + 4 * tx, j = j0 + ty;
-  const int k0 = blockIdx.z * a.zc;
+  const int k0 = (a.ch0 + (int)blockIdx.z * a.chs) * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
   const int np = k1 - k0;
   const bool own = (x0 < d.nx) && (j < d.ny);

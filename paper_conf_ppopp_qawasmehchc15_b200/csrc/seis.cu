@@ -149,12 +149,17 @@ struct Slab {
   int nrec_own = 0;
   long long* d_rec_off = nullptr;
   int* d_rec_id = nullptr;
-  int ngroups = 0;
-  long long* d_g_off = nullptr;
-  float* d_g_scale = nullptr;
-  int* d_g_start = nullptr;
-  int* d_g_mem = nullptr;
-  int* d_g_surf = nullptr;   // ELASTIC: group node on the free surface
+  // backward-phase injection groups (distinct receiver nodes, CSR members), split by the
+  // z-chunk that owns the node: [0] = first / last chunk (injected before the overlapped
+  // ghost exchange), [1] = interior chunks
+  struct Groups {
+    int n = 0;
+    long long* off = nullptr;
+    float* scale = nullptr;
+    int* start = nullptr;
+    int* mem = nullptr;
+    int* surf = nullptr;     // ELASTIC: group node on the free surface
+  } grp[2];
   float* snap = nullptr;     // nsnap * nzl*ny*nx (points into the model's pool)
 };
 
@@ -195,6 +200,10 @@ struct seis_model {
   cudaStream_t cap = nullptr;       // capture stream (the legacy stream cannot be captured)
   cudaGraphExec_t gexec = nullptr;
   uint64_t gkey = 0;
+  // overlapped ghost exchange: side stream + fork / join events
+  cudaStream_t xs = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  bool no_overlap = false;  // SEIS_NO_OVERLAP=1: serial exchange (A/B measurements)
   long long g_launches = 0;
 };
 
@@ -525,6 +534,9 @@ seis_status seis_model_destroy(seis_model* M) {
   cudaSetDevice(M->device);
   if (M->gexec) cudaGraphExecDestroy(M->gexec);
   if (M->cap) cudaStreamDestroy(M->cap);
+  if (M->xs) cudaStreamDestroy(M->xs);
+  if (M->ev_fork) cudaEventDestroy(M->ev_fork);
+  if (M->ev_join) cudaEventDestroy(M->ev_join);
   for (void* p : M->allocs) cudaFree(p);
   delete M;
   return SEIS_OK;
@@ -740,6 +752,13 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     if (kind == SEIS_ELASTIC) choose_chunks(S, occ, dev_sms, TXE, BYE);
     else choose_chunks(S, occ, dev_sms, TXV, kind == SEIS_ISO ? BYI : BYV);
   }
+  if (ns > 1 || M->nranks > 1) {
+    const char* e = getenv("SEIS_NO_OVERLAP");
+    M->no_overlap = e && e[0] == '1';
+    CK(cudaStreamCreateWithFlags(&M->xs, cudaStreamNonBlocking));
+    CK(cudaEventCreateWithFlags(&M->ev_fork, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&M->ev_join, cudaEventDisableTiming));
+  }
   if (kind == SEIS_ACOUSTIC)  // rho(k+1) across slab faces
     TRY(exchange_arrays(M, {[](Slab& S) { return S.rho; }}, 4, st));
   if (kind == SEIS_ELASTIC)  // rho(k+1), w(k+1) across slab faces
@@ -813,8 +832,19 @@ seis_status seis_memory_required(const seis_grid* g, seis_kind kind, const seis_
     const double per = (2 * W * g->ny * (double)nzl + 2 * W * g->nx * (double)nzl + 2 * W * g->nx * (double)g->ny) * 4.0;
     b += per * (kind == SEIS_ACOUSTIC ? 2 : 6);
   }
-  if (shot && shot->snap_period >= 1 && shot->nt >= 1)
-    b += (double)((shot->nt - 1) / shot->snap_period) * nzl * (double)g->ny * g->nx * 4.0;
+  if (shot && shot->snap_period >= 1 && shot->nt >= 1) {
+    const long long nsnap = (shot->nt - 1) / shot->snap_period;
+    const long long c = shot->ckpt_period > 0 ? std::min<long long>(shot->ckpt_period, nsnap) : nsnap;
+    const long long nckpt = nsnap > 0 && c > 0 ? (nsnap + c - 1) / c - 1 : 0;
+    // checkpoint = every padded state field + the C-PML memory slabs
+    double ck = nf * (padded + 128.0);
+    if (kind != SEIS_ISO && g->nb > 0) {
+      const double W = g->nb + 1;
+      ck += (2 * W * g->ny * (double)nzl + 2 * W * g->nx * (double)nzl + 2 * W * g->nx * (double)g->ny) * 4.0 *
+            (kind == SEIS_ACOUSTIC ? 2 : 6);
+    }
+    b += (double)c * nzl * (double)g->ny * g->nx * 4.0 + (double)nckpt * ck;
+  }
   *bytes = (uint64_t)b;
   return SEIS_OK;
 }
@@ -870,7 +900,7 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
   for (Slab& S : M->slabs) {
     const int z0 = S.d.z0, z1 = S.d.z0 + S.d.nzl;
     S.src_o = -1;
-    if (!backward_injection && sh->sz >= z0 && sh->sz < z1) {
+    if (sh->sz >= z0 && sh->sz < z1) {  // (used only by steps with with_src)
       S.src_o = S.d.at(sh->sx, sh->sy, sh->sz - z0);
       S.src_scale = (float)point_scale(sh->sx, sh->sy, sh->sz);
     }
@@ -893,38 +923,45 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
       CK(cudaMemcpy(S.d_rec_off, off.data(), off.size() * sizeof(long long), cudaMemcpyHostToDevice));
       CK(cudaMemcpy(S.d_rec_id, rid.data(), rid.size() * sizeof(int), cudaMemcpyHostToDevice));
     }
-    S.ngroups = 0;
+    for (auto& G2 : S.grp) {
+      if (G2.off) {
+        cudaFree(G2.off); cudaFree(G2.scale); cudaFree(G2.start); cudaFree(G2.mem); cudaFree(G2.surf);
+      }
+      G2 = Slab::Groups{};
+    }
     if (backward_injection && S.nrec_own > 0) {
       // merge duplicates: group receivers by node, members in receiver-index order (O12)
       std::map<long long, std::vector<int>> groups;
       for (size_t t = 0; t < off.size(); ++t) groups[off[t]].push_back(rid[t]);
-      std::vector<long long> goff;
-      std::vector<float> gsc;
-      std::vector<int> gstart{0}, gmem, gsurf;
+      std::vector<long long> goff[2];
+      std::vector<float> gsc[2];
+      std::vector<int> gstart[2] = {{0}, {0}}, gmem[2], gsurf[2];
       for (auto& kv : groups) {
-        goff.push_back(kv.first);
         const int r0 = kv.second.front();
         const int* p = sh->rec + 3 * r0;
-        gsc.push_back((float)point_scale(p[0], p[1], p[2]));
-        gsurf.push_back(M->g.free_surface && p[2] == 0 ? 1 : 0);
-        for (int r : kv.second) gmem.push_back(r);
-        gstart.push_back((int)gmem.size());
+        const int ch = (p[2] - z0) / S.zc;
+        const int part = (ch == 0 || ch == S.nzch - 1) ? 0 : 1;
+        goff[part].push_back(kv.first);
+        gsc[part].push_back((float)point_scale(p[0], p[1], p[2]));
+        gsurf[part].push_back(M->g.free_surface && p[2] == 0 ? 1 : 0);
+        for (int r : kv.second) gmem[part].push_back(r);
+        gstart[part].push_back((int)gmem[part].size());
       }
-      S.ngroups = (int)goff.size();
-      if (S.d_g_off) {
-        cudaFree(S.d_g_off); cudaFree(S.d_g_scale); cudaFree(S.d_g_start); cudaFree(S.d_g_mem);
-        cudaFree(S.d_g_surf);
+      for (int part = 0; part < 2; ++part) {
+        Slab::Groups& G2 = S.grp[part];
+        G2.n = (int)goff[part].size();
+        if (G2.n == 0) continue;
+        CK(dmalloc(&G2.off, goff[part].size()));
+        CK(dmalloc(&G2.scale, gsc[part].size()));
+        CK(dmalloc(&G2.start, gstart[part].size()));
+        CK(dmalloc(&G2.mem, gmem[part].size()));
+        CK(dmalloc(&G2.surf, gsurf[part].size()));
+        CK(cudaMemcpy(G2.surf, gsurf[part].data(), gsurf[part].size() * sizeof(int), cudaMemcpyHostToDevice));
+        CK(cudaMemcpy(G2.off, goff[part].data(), goff[part].size() * sizeof(long long), cudaMemcpyHostToDevice));
+        CK(cudaMemcpy(G2.scale, gsc[part].data(), gsc[part].size() * sizeof(float), cudaMemcpyHostToDevice));
+        CK(cudaMemcpy(G2.start, gstart[part].data(), gstart[part].size() * sizeof(int), cudaMemcpyHostToDevice));
+        CK(cudaMemcpy(G2.mem, gmem[part].data(), gmem[part].size() * sizeof(int), cudaMemcpyHostToDevice));
       }
-      CK(dmalloc(&S.d_g_off, goff.size()));
-      CK(dmalloc(&S.d_g_scale, gsc.size()));
-      CK(dmalloc(&S.d_g_start, gstart.size()));
-      CK(dmalloc(&S.d_g_mem, gmem.size()));
-      CK(dmalloc(&S.d_g_surf, gsurf.size()));
-      CK(cudaMemcpy(S.d_g_surf, gsurf.data(), gsurf.size() * sizeof(int), cudaMemcpyHostToDevice));
-      CK(cudaMemcpy(S.d_g_off, goff.data(), goff.size() * sizeof(long long), cudaMemcpyHostToDevice));
-      CK(cudaMemcpy(S.d_g_scale, gsc.data(), gsc.size() * sizeof(float), cudaMemcpyHostToDevice));
-      CK(cudaMemcpy(S.d_g_start, gstart.data(), gstart.size() * sizeof(int), cudaMemcpyHostToDevice));
-      CK(cudaMemcpy(S.d_g_mem, gmem.data(), gmem.size() * sizeof(int), cudaMemcpyHostToDevice));
     }
   }
   M->shot_key = key;
@@ -953,6 +990,44 @@ seis_status zero_state(seis_model* M, cudaStream_t st) {
   return SEIS_OK;
 }
 
+// Every array of the propagating state (padded fields incl. ghost planes, C-PML
+// memory slabs): (pointer, floats).  A checkpoint is a copy of all of them.
+std::vector<std::pair<float*, size_t>> state_arrays(seis_model* M) {
+  std::vector<std::pair<float*, size_t>> v;
+  for (Slab& S : M->slabs) {
+    const size_t elems = (size_t)S.d.PS * (S.d.nzl + 2 * GZ) + 32;  // + the 128-byte alignment pad
+    for (float* f : S.fld) v.emplace_back(f - 28, elems);             // base = f - 112 bytes
+    if (M->W > 0) {
+      const int W = M->W;
+      for (int t = 0; t < npsi_of(M->kind); ++t) {
+        const int ax = psi_axis(M->kind, t);
+        size_t n;
+        if (ax == 0) n = (size_t)S.d.nzl * S.d.ny * 2 * W;
+        else if (ax == 1) n = (size_t)S.d.nzl * 2 * W * S.d.nx;
+        else n = (size_t)2 * W * S.d.ny * S.d.nx;
+        v.emplace_back(S.psi[t], n);
+      }
+    }
+  }
+  return v;
+}
+
+// Copy the whole state to (save = true) or from a checkpoint slot of state_elems floats.
+seis_status state_copy(seis_model* M, float* slot, bool save, cudaStream_t st) {
+  size_t o = 0;
+  for (auto& a : state_arrays(M)) {
+    if (save) CK(cudaMemcpyAsync(slot + o, a.first, a.second * 4, cudaMemcpyDeviceToDevice, st));
+    else CK(cudaMemcpyAsync(a.first, slot + o, a.second * 4, cudaMemcpyDeviceToDevice, st));
+    o += (a.second + 31) / 32 * 32;
+  }
+  return SEIS_OK;
+}
+size_t state_elems(seis_model* M) {
+  size_t o = 0;
+  for (auto& a : state_arrays(M)) o += (a.second + 31) / 32 * 32;
+  return o;
+}
+
 // Free-surface ghost planes (O16) of the slab that holds the global top.
 seis_status fs_mirror(seis_model* M, std::initializer_list<int> fields, cudaStream_t st) {
   if (!M->g.free_surface) return SEIS_OK;
@@ -972,27 +1047,72 @@ seis_status fs_mirror(seis_model* M, std::initializer_list<int> fields, cudaStre
 }
 
 // ISO / ACOUSTIC: 64 x BY tiles of (16, BY) threads; ELASTIC: 32 x BYE tiles of (32, BYE)
-dim3 grid_of(const Slab& S, int tw, int by) {
-  return dim3((S.d.nx + tw - 1) / tw, (S.d.ny + by - 1) / by, S.nzch);
+dim3 grid_of(const Slab& S, int tw, int by, int nch) {
+  return dim3((S.d.nx + tw - 1) / tw, (S.d.ny + by - 1) / by, nch);
 }
 
 // Backward-phase receiver injection into the field just produced (before its
 // ghost planes are exchanged, so neighbouring slabs see the injected values).
-seis_status inject_rows(seis_model* M, const float* row, cudaStream_t st) {
+// part: 0 = groups in the first / last z-chunk, 1 = interior chunks, 2 = all.
+seis_status inject_rows(seis_model* M, const float* row, int part, cudaStream_t st) {
   for (Slab& S : M->slabs) {
-    if (S.ngroups == 0) continue;
-    PROF(5, st);
-    if (M->kind == SEIS_ELASTIC) {
-      inject_el_kernel<<<(S.ngroups + 127) / 128, 128, 0, st>>>(
-          S.fld[ESXX], S.fld[ESYY], S.fld[ESZZ], S.d_g_off, S.d_g_scale, S.d_g_start, S.d_g_mem, row,
-          S.d_g_surf, S.ngroups);
-    } else {
-      float* f = M->kind == SEIS_ISO ? S.fld[S.cur] : S.fld[0];
-      inject_kernel<<<(S.ngroups + 127) / 128, 128, 0, st>>>(f, S.d_g_off, S.d_g_scale, S.d_g_start,
-                                                             S.d_g_mem, row, S.ngroups);
+    for (int q = 0; q < 2; ++q) {
+      if (part != 2 && part != q) continue;
+      const Slab::Groups& G2 = S.grp[q];
+      if (G2.n == 0) continue;
+      PROF(5, st);
+      if (M->kind == SEIS_ELASTIC) {
+        inject_el_kernel<<<(G2.n + 127) / 128, 128, 0, st>>>(S.fld[ESXX], S.fld[ESYY], S.fld[ESZZ], G2.off,
+                                                            G2.scale, G2.start, G2.mem, row, G2.surf, G2.n);
+      } else {
+        float* f = M->kind == SEIS_ISO ? S.fld[S.cur] : S.fld[0];
+        inject_kernel<<<(G2.n + 127) / 128, 128, 0, st>>>(f, G2.off, G2.scale, G2.start, G2.mem, row, G2.n);
+      }
+      CKL();
     }
-    CKL();
   }
+  return SEIS_OK;
+}
+
+// Launch of one stencil kernel on slab s over the z-chunks ch0 + t chs, t < nch.
+using LaunchFn = std::function<seis_status(size_t s, int ch0, int chs, int nch, cudaStream_t)>;
+// Work after the kernel: part 0 = first/last chunks (injection there, then the ghost
+// exchange and free-surface mirror), part 1 = interior chunks, part 2 = everything.
+using PostFn = std::function<seis_status(int part, cudaStream_t)>;
+
+// Is the ghost exchange of this model overlapped with interior updates?
+bool overlapped(const seis_model* M) {
+  if (M->slabs.size() < 2 && !(M->comm && M->nranks > 1)) return false;  // nothing to exchange
+  return !M->no_overlap;
+}
+
+// One kernel phase of a step (8(e) pipeline).  Without decomposition: every chunk, then
+// `post(2)`.  Decomposed: the first and last z-chunk of every slab run first on the side
+// stream xs, followed there by their injection, the ghost-plane exchange (memcpy between
+// slabs, NCCL send/recv between ranks) and the mirror; meanwhile the interior chunks run on
+// the compute stream; the compute stream then joins xs.  Per-point arithmetic is the same,
+// so results are bitwise identical to the serial order.
+seis_status run_phase(seis_model* M, const LaunchFn& launch, const PostFn& post, cudaStream_t st) {
+  if (!overlapped(M)) {
+    for (size_t s = 0; s < M->slabs.size(); ++s) TRY(launch(s, 0, 1, M->slabs[s].nzch, st));
+    return post(2, st);
+  }
+  cudaStream_t xs = M->xs;
+  CK(cudaEventRecord(M->ev_fork, st));
+  CK(cudaStreamWaitEvent(xs, M->ev_fork, 0));
+  for (size_t s = 0; s < M->slabs.size(); ++s) {
+    const int nch = M->slabs[s].nzch;
+    if (nch <= 2) TRY(launch(s, 0, 1, nch, xs));
+    else TRY(launch(s, 0, nch - 1, 2, xs));
+  }
+  TRY(post(0, xs));
+  for (size_t s = 0; s < M->slabs.size(); ++s) {
+    const int nch = M->slabs[s].nzch;
+    if (nch > 2) TRY(launch(s, 1, 1, nch - 2, st));
+  }
+  TRY(post(1, st));
+  CK(cudaEventRecord(M->ev_join, xs));
+  CK(cudaStreamWaitEvent(st, M->ev_join, 0));
   return SEIS_OK;
 }
 
@@ -1002,46 +1122,55 @@ seis_status inject_rows(seis_model* M, const float* row, cudaStream_t st) {
 seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
                  std::vector<const float*>* imgS, std::vector<float*>* img, cudaStream_t st,
                  const float* inj_row = nullptr) {
+  auto inject = [&](int part, cudaStream_t s2) -> seis_status {
+    return inj_row ? inject_rows(M, inj_row, part, s2) : SEIS_OK;
+  };
   if (M->kind == SEIS_ISO) {
-    for (size_t s = 0; s < M->slabs.size(); ++s) {
+    const int cur = M->slabs[0].cur;  // u^n = fld[cur] in every slab
+    LaunchFn k_iso = [&](size_t s, int ch0, int chs, int nch, cudaStream_t ks) -> seis_status {
       Slab& S = M->slabs[s];
       IsoArgs a;
-      a.mun = S.iso_ut[S.cur];
-      a.mup = S.iso_uc[1 - S.cur];
+      a.mun = S.iso_ut[cur];
+      a.mup = S.iso_uc[1 - cur];
       a.mm = S.iso_m;
-      a.muq = S.iso_uc[S.cur];
-      a.un = S.fld[S.cur];
-      a.up = S.fld[1 - S.cur];
+      a.muq = S.iso_uc[cur];
+      a.un = S.fld[cur];
+      a.up = S.fld[1 - cur];
       a.edx = M->edx;
       a.edy = M->edy;
       a.edz = M->edz;
       a.d = S.d;
       a.zc = S.zc;
+      a.ch0 = ch0;
+      a.chs = chs;
       a.src_o = with_src ? S.src_o : -1;
       a.src_amp = 0.f;
       if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
       a.snap = snap ? (*snap)[s] : nullptr;
       a.imgS = imgS ? (*imgS)[s] : nullptr;
       a.img = img ? (*img)[s] : nullptr;
-      const dim3 gr = grid_of(S, TXV, BYI), blk(NTX, BYI);
+      const dim3 gr = grid_of(S, TXV, BYI, nch), blk(NTX, BYI);
       {
-        PROF(0, st);
+        PROF(0, ks);
         const size_t sb = IsoStage<BYI>::smem_bytes();
-        if (a.snap) iso_step_kernel<BYI, true, false><<<gr, blk, sb, st>>>(a);
-        else if (a.img) iso_step_kernel<BYI, false, true><<<gr, blk, sb, st>>>(a);
-        else iso_step_kernel<BYI, false, false><<<gr, blk, sb, st>>>(a);
+        if (a.snap) iso_step_kernel<BYI, true, false><<<gr, blk, sb, ks>>>(a);
+        else if (a.img) iso_step_kernel<BYI, false, true><<<gr, blk, sb, ks>>>(a);
+        else iso_step_kernel<BYI, false, false><<<gr, blk, sb, ks>>>(a);
       }
       CKL();
-    }
+      return SEIS_OK;
+    };
+    // the injection targets u^{n+1} = fld[1 - cur]; swap first so inject_rows sees it as cur
     for (Slab& S : M->slabs) S.cur = 1 - S.cur;
-    if (inj_row) TRY(inject_rows(M, inj_row, st));
-    // exchange the new level (fld[cur] after the swap)
-    const int f = M->slabs[0].cur;
-    TRY(exchange(M, {f}, st));
-    return SEIS_OK;
+    PostFn post = [&](int part, cudaStream_t ps) -> seis_status {
+      TRY(inject(part, ps));
+      if (part != 1) TRY(exchange(M, {1 - cur}, ps));  // the new level
+      return SEIS_OK;
+    };
+    return run_phase(M, k_iso, post, st);
   }
   if (M->kind == SEIS_ACOUSTIC) {
-    for (size_t s = 0; s < M->slabs.size(); ++s) {
+    LaunchFn k_v = [&](size_t s, int ch0, int chs, int nch, cudaStream_t ks) -> seis_status {
       Slab& S = M->slabs[s];
       AcVArgs a;
       a.mp = S.ac_pt;
@@ -1067,19 +1196,24 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.psz = S.psi[2];
       a.d = S.d;
       a.zc = S.zc;
+      a.ch0 = ch0;
+      a.chs = chs;
       a.imgS = imgS ? (*imgS)[s] : nullptr;
       a.img = img ? (*img)[s] : nullptr;
-      const dim3 gr = grid_of(S, TXV, BYV), blk(NTX, BYV);
+      const dim3 gr = grid_of(S, TXV, BYV, nch), blk(NTX, BYV);
       {
-        PROF(1, st);
+        PROF(1, ks);
         const size_t sb = AcVStage<BYV>::smem_bytes();
-        if (a.img) ac_v_kernel<BYV, true><<<gr, blk, sb, st>>>(a);
-        else ac_v_kernel<BYV, false><<<gr, blk, sb, st>>>(a);
+        if (a.img) ac_v_kernel<BYV, true><<<gr, blk, sb, ks>>>(a);
+        else ac_v_kernel<BYV, false><<<gr, blk, sb, ks>>>(a);
       }
       CKL();
-    }
-    TRY(exchange(M, {3}, st));  // q_z has the only z-derivative in P
-    for (size_t s = 0; s < M->slabs.size(); ++s) {
+      return SEIS_OK;
+    };
+    // q_z has the only z-derivative in P
+    TRY(run_phase(M, k_v, [&](int part, cudaStream_t ps) { return part != 1 ? exchange(M, {3}, ps) : SEIS_OK; },
+                  st));
+    LaunchFn k_p = [&](size_t s, int ch0, int chs, int nch, cudaStream_t ks) -> seis_status {
       Slab& S = M->slabs[s];
       AcPArgs a;
       a.mqx = S.ac_qxt;
@@ -1099,25 +1233,31 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.pqz = S.psi[5];
       a.d = S.d;
       a.zc = S.zc;
+      a.ch0 = ch0;
+      a.chs = chs;
       a.src_o = with_src ? S.src_o : -1;
       a.src_amp = 0.f;
       if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
       a.snap = snap ? (*snap)[s] : nullptr;
-      const dim3 gr = grid_of(S, TXV, BYP), blk(NTX, BYP);
+      const dim3 gr = grid_of(S, TXV, BYP, nch), blk(NTX, BYP);
       {
-        PROF(2, st);
+        PROF(2, ks);
         const size_t sb = AcPStage<BYP>::smem_bytes();
-        if (a.snap) ac_p_kernel<BYP, true><<<gr, blk, sb, st>>>(a);
-        else ac_p_kernel<BYP, false><<<gr, blk, sb, st>>>(a);
+        if (a.snap) ac_p_kernel<BYP, true><<<gr, blk, sb, ks>>>(a);
+        else ac_p_kernel<BYP, false><<<gr, blk, sb, ks>>>(a);
       }
       CKL();
-    }
-    if (inj_row) TRY(inject_rows(M, inj_row, st));
-    TRY(exchange(M, {0}, st));  // p for the next V
-    return SEIS_OK;
+      return SEIS_OK;
+    };
+    PostFn post_p = [&](int part, cudaStream_t ps) -> seis_status {
+      TRY(inject(part, ps));
+      if (part != 1) TRY(exchange(M, {0}, ps));  // p for the next V
+      return SEIS_OK;
+    };
+    return run_phase(M, k_p, post_p, st);
   }
   // ELASTIC
-  for (size_t s = 0; s < M->slabs.size(); ++s) {
+  LaunchFn k_v = [&](size_t s, int ch0, int chs, int nch, cudaStream_t ks) -> seis_status {
     Slab& S = M->slabs[s];
     ElVArgs a;
     a.msxx = S.el_sxxt;
@@ -1144,19 +1284,26 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (int t = 0; t < 9; ++t) a.psi[t] = S.psi[t];
     a.d = S.d;
     a.zc = S.zc;
+    a.ch0 = ch0;
+    a.chs = chs;
     a.imgS = imgS ? (*imgS)[s] : nullptr;
     a.img = img ? (*img)[s] : nullptr;
-    const dim3 gr = grid_of(S, TXE, BYE);
+    const dim3 gr = grid_of(S, TXE, BYE, nch);
     {
-      PROF(3, st);
-      if (a.img) el_v_kernel<BYE, true><<<gr, dim3(NTX2, BYE), ElVStage<BYE>::smem_bytes(), st>>>(a);
-      else el_v_kernel<BYE, false><<<gr, dim3(NTX2, BYE), ElVStage<BYE>::smem_bytes(), st>>>(a);
+      PROF(3, ks);
+      if (a.img) el_v_kernel<BYE, true><<<gr, dim3(NTX2, BYE), ElVStage<BYE>::smem_bytes(), ks>>>(a);
+      else el_v_kernel<BYE, false><<<gr, dim3(NTX2, BYE), ElVStage<BYE>::smem_bytes(), ks>>>(a);
     }
     CKL();
-  }
-  TRY(exchange(M, {0, 1, 2}, st));
-  TRY(fs_mirror(M, {EVX, EVY, EVZ}, st));
-  for (size_t s = 0; s < M->slabs.size(); ++s) {
+    return SEIS_OK;
+  };
+  PostFn post_v = [&](int part, cudaStream_t ps) -> seis_status {
+    if (part == 1) return SEIS_OK;
+    TRY(exchange(M, {0, 1, 2}, ps));
+    return fs_mirror(M, {EVX, EVY, EVZ}, ps);
+  };
+  TRY(run_phase(M, k_v, post_v, st));
+  LaunchFn k_s = [&](size_t s, int ch0, int chs, int nch, cudaStream_t ks) -> seis_status {
     Slab& S = M->slabs[s];
     ElSArgs a;
     for (int t = 0; t < 3; ++t) a.mvt[t] = S.el_vt[t];
@@ -1174,22 +1321,28 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     for (int t = 0; t < 9; ++t) a.psi[t] = S.psi[9 + t];
     a.d = S.d;
     a.zc = S.zc;
+    a.ch0 = ch0;
+    a.chs = chs;
     a.src_o = with_src ? S.src_o : -1;
     a.src_amp = 0.f;
     if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
     a.snap = snap ? (*snap)[s] : nullptr;
-    const dim3 gr = grid_of(S, TXE, BYE);
+    const dim3 gr = grid_of(S, TXE, BYE, nch);
     {
-      PROF(4, st);
-      if (a.snap) el_s_kernel<BYE, true><<<gr, dim3(NTX2, BYE), ElSStage<BYE>::smem_bytes(), st>>>(a);
-      else el_s_kernel<BYE, false><<<gr, dim3(NTX2, BYE), ElSStage<BYE>::smem_bytes(), st>>>(a);
+      PROF(4, ks);
+      if (a.snap) el_s_kernel<BYE, true><<<gr, dim3(NTX2, BYE), ElSStage<BYE>::smem_bytes(), ks>>>(a);
+      else el_s_kernel<BYE, false><<<gr, dim3(NTX2, BYE), ElSStage<BYE>::smem_bytes(), ks>>>(a);
     }
     CKL();
-  }
-  if (inj_row) TRY(inject_rows(M, inj_row, st));
-  TRY(exchange(M, {5, 7, 8}, st));
-  TRY(fs_mirror(M, {ESZZ, ESXZ, ESYZ}, st));
-  return SEIS_OK;
+    return SEIS_OK;
+  };
+  PostFn post_s = [&](int part, cudaStream_t ps) -> seis_status {
+    TRY(inject(part, ps));
+    if (part == 1) return SEIS_OK;
+    TRY(exchange(M, {5, 7, 8}, ps));
+    return fs_mirror(M, {ESZZ, ESXZ, ESYZ}, ps);
+  };
+  return run_phase(M, k_s, post_s, st);
 }
 
 // Field holding the recorded / imaged quantity
@@ -1311,10 +1464,16 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
   const seis_grid& g = M->g;
   const int nt = sh->nt, snap = sh->snap_period;
   TRY(setup_shot(M, sh, false, st));
-  // snapshot pool (O14): nsnap fields of the process slab
+  // snapshot pool (O14): nsnap fields of the process slab, or (checkpointing, f2) the last
+  // segment's c snapshots + nckpt source-state checkpoints
   const int nsnap = nt >= 1 ? (nt - 1) / snap : 0;
+  const int c = sh->ckpt_period > 0 ? std::min(sh->ckpt_period, std::max(nsnap, 1)) : std::max(nsnap, 1);
+  const int nseg = nsnap > 0 ? (nsnap + c - 1) / c : 0;
+  const int nckpt = nseg > 1 ? nseg - 1 : 0;
   const size_t slab_pts = (size_t)M->pnzl * g.ny * g.nx;
-  const size_t need = (size_t)nsnap * slab_pts;
+  const size_t st_elems = nckpt ? state_elems(M) : 0;
+  const size_t snap_elems = (size_t)std::min(c, nsnap) * slab_pts;
+  const size_t need = snap_elems + (size_t)nckpt * st_elems;
   if (need > M->pool_elems) {
     size_t freeb = 0, totb = 0;
     cudaMemGetInfo(&freeb, &totb);
@@ -1328,13 +1487,22 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
     cudaError_t e = cudaMalloc(&p, need * sizeof(float));
     if (e != cudaSuccess) {
       cudaGetLastError();
-      return fail(SEIS_ENOMEM, "snapshot pool needs %zu bytes (%d snapshots), %zu free", need * 4,
-                  nsnap, freeb);
+      return fail(SEIS_ENOMEM, "snapshot pool needs %zu bytes (%d snapshots, %d checkpoints), %zu free",
+                  need * 4, std::min(c, nsnap), nckpt, freeb);
     }
     M->allocs.push_back(p);
     M->pool = (float*)p;
     M->pool_elems = need;
   }
+  float* ckpt0 = M->pool + snap_elems;  // checkpoint slot q = state at level (q + 1) c snap
+  auto slot_of = [&](int q) { return ckpt0 + (size_t)q * st_elems; };
+  std::vector<int> ckpt_cur(nckpt, 0);  // ISO: which buffer holds u^n at the checkpoint
+  // pool pointers of snapshot index i (j = (i + 1) snap), which lives in segment i / c
+  auto snap_ptrs = [&](int i, std::vector<float*>& v) {
+    const size_t off = (size_t)(i % c) * slab_pts;
+    for (size_t s = 0; s < M->slabs.size(); ++s)
+      v[s] = M->pool + off + (size_t)(M->slabs[s].d.z0 - M->pz0) * g.ny * g.nx;
+  };
   // image / data staging
   const bool img_dev = is_device_ptr(image);
   const size_t nd = (size_t)nt * sh->nrec;
@@ -1351,36 +1519,63 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
     CK(cudaMemcpyAsync(dd, data, nd * sizeof(float), cudaMemcpyHostToDevice, st));
     data_d = dd;
   }
-  // ---- forward phase: source wavefield, snapshots S_j (j = snap .. nt-1) in HBM
-  TRY(zero_state(M, st));
+  // Forward source propagation over steps [n0, n1), storing the snapshots of segment `seg`
+  // (all segments when seg < 0 and there is no checkpointing) and, in the first pass,
+  // the checkpoints at the segment starts.
   std::vector<float*> snapp(M->slabs.size());
-  for (int n = 0; n < nt; ++n) {
-    const int j = n + 1;
-    const bool take = (j % snap == 0) && j <= nt - 1;
-    if (take) {
-      size_t off = (size_t)(j / snap - 1) * slab_pts;
-      for (size_t s = 0; s < M->slabs.size(); ++s) {
-        const size_t so = (size_t)(M->slabs[s].d.z0 - M->pz0) * g.ny * g.nx;
-        snapp[s] = M->pool + off + so;
+  auto forward = [&](int n0, int n1, int seg, bool first) -> seis_status {
+    for (int n = n0; n < n1; ++n) {
+      if (first && nckpt && n > 0 && n % (c * snap) == 0 && n / (c * snap) <= nckpt) {
+        const int q = n / (c * snap) - 1;
+        TRY(state_copy(M, slot_of(q), true, st));
+        ckpt_cur[q] = M->slabs[0].cur;
       }
+      const int j = n + 1;
+      bool take = (j % snap == 0) && j <= nt - 1;
+      if (take && (j / snap - 1) / c != seg) take = false;
+      if (take) snap_ptrs(j / snap - 1, snapp);
+      TRY(step(M, n, true, take ? &snapp : nullptr, nullptr, nullptr, st));
     }
-    TRY(step(M, n, true, take ? &snapp : nullptr, nullptr, nullptr, st));
-  }
+    return SEIS_OK;
+  };
+  // ---- forward phase: source wavefield, snapshots S_j of the last segment (all of them
+  // without checkpointing), checkpoints at the starts of the other segments
+  TRY(zero_state(M, st));
+  TRY(forward(0, nt, nseg - 1, true));
   // ---- backward phase: receiver wavefield from zero, same operator
   TRY(setup_shot(M, sh, true, st));
   TRY(zero_state(M, st));
   std::vector<const float*> Sp(M->slabs.size());
-  std::vector<float*> Ip(M->slabs.size());
+  std::vector<float*> Ip(M->slabs.size()), tmp(M->slabs.size());
   for (size_t s = 0; s < M->slabs.size(); ++s)
     Ip[s] = img_d + (size_t)(M->slabs[s].d.z0 - M->pz0) * g.ny * g.nx;
+  int loaded = nseg - 1;  // segment whose snapshots are in the pool
   for (int m = 0; m < nt; ++m) {
     // imaging of level j = nt - m (the INPUT of this step, R^m) fused into the step kernel
     const int j = nt - m;
     const bool im = (j % snap == 0) && j >= snap && j <= nt - 1;
     if (im) {
-      const size_t off = (size_t)(j / snap - 1) * slab_pts;
-      for (size_t s = 0; s < M->slabs.size(); ++s)
-        Sp[s] = M->pool + off + (size_t)(M->slabs[s].d.z0 - M->pz0) * g.ny * g.nx;
+      const int i = j / snap - 1, seg = i / c;
+      if (seg != loaded) {
+        // recompute segment seg from its checkpoint (zero state for seg 0).  The receiver
+        // state is parked in checkpoint slot seg (the slot of segment seg + 1, consumed or
+        // unused by now) and restored afterwards.
+        const int rcur = M->slabs[0].cur;
+        TRY(state_copy(M, slot_of(seg), true, st));
+        if (seg == 0) {
+          TRY(zero_state(M, st));
+        } else {
+          TRY(state_copy(M, slot_of(seg - 1), false, st));
+          for (Slab& S : M->slabs) S.cur = ckpt_cur[seg - 1];
+        }
+        const int last_j = std::min((seg + 1) * c, nsnap) * snap;
+        TRY(forward(seg * c * snap, last_j, seg, false));
+        TRY(state_copy(M, slot_of(seg), false, st));
+        for (Slab& S : M->slabs) S.cur = rcur;
+        loaded = seg;
+      }
+      snap_ptrs(i, tmp);
+      for (size_t s = 0; s < M->slabs.size(); ++s) Sp[s] = tmp[s];
     }
     // step + receiver injection of data[nt-1-m] (all receivers, one launch per slab)
     TRY(step(M, m, false, nullptr, im ? &Sp : nullptr, im ? &Ip : nullptr, st,

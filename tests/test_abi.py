@@ -90,3 +90,27 @@ def test_no_cpu_fallback_without_a_device():
     with pytest.raises(seis.SeisError) as e:
         seis.Model(g, "iso", np.full((16, 16, 16), 2000.0, np.float32))
     assert e.value.name == "SEIS_ECUDA"
+
+
+def test_memory_required_checkpointing():
+    """f2: checkpointed RTM keeps c snapshots + ceil(nsnap/c)-1 state checkpoints; the
+    C5 1024^3 single-GPU RTM (49 snapshots) only fits in 180 GB with checkpointing."""
+    import numpy as np
+
+    g = seis.Grid(128, 96, 64, 10.0, 8e-4, nb=10)
+    pts = 128 * 96 * 64 * 4
+    w = np.zeros(201, np.float32)
+    rec = np.zeros((1, 3), np.int32)
+    m0 = seis.memory_required(g, "acoustic")
+    full = seis.memory_required(g, "acoustic", seis.Shot((1, 1, 1), w, rec, snap_period=20))
+    c3 = seis.memory_required(g, "acoustic", seis.Shot((1, 1, 1), w, rec, snap_period=20, ckpt_period=3))
+    c10 = seis.memory_required(g, "acoustic", seis.Shot((1, 1, 1), w, rec, snap_period=20, ckpt_period=10))
+    assert c10 == full  # one segment = no checkpoint
+    # 10 snapshots in segments of 3 -> 3 snapshots in the pool + 3 checkpoints of the state
+    ck = (c3 - m0 - 3 * pts) / 3
+    assert ck > 4 * pts  # 4 padded fields + C-PML slabs
+    g5 = seis.Grid(1024, 1024, 1024, 10.0, 8e-4, nb=20)
+    w5 = np.zeros(1000, np.float32)
+    allsnap = seis.memory_required(g5, "acoustic", seis.Shot((1, 1, 1), w5, rec, snap_period=20))
+    ckpt = seis.memory_required(g5, "acoustic", seis.Shot((1, 1, 1), w5, rec, snap_period=20, ckpt_period=10))
+    assert allsnap > 180e9 > ckpt

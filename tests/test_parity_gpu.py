@@ -211,3 +211,82 @@ def test_error_codes():
         mod.migrate(seis.Shot((1, 1, 1), w, np.zeros((1, 3), np.int32), snap_period=0),
                     np.zeros((10, 1), np.float32), np.zeros((nx, nx, nx), np.float32))
     assert e.value.name == "SEIS_EINVAL"
+
+
+def _deep_recs(nx, ny, nz):
+    """Receivers at every depth band, so the injection tables of both the boundary chunks
+    and the interior chunks of every slab are exercised (a duplicate included)."""
+    pts = [[(7 * t) % nx, (5 * t) % ny, (11 * t) % nz] for t in range(40)]
+    pts.append(pts[3])
+    return np.asarray(pts, np.int32)
+
+
+@pytest.mark.parametrize("kind", ["iso", "acoustic", "elastic"])
+def test_overlapped_exchange_bitwise(kind, monkeypatch):
+    """§8(e) pipeline: with z-slabs the first / last z-chunk of every slab runs first, the
+    ghost exchange overlaps the interior chunks on a second stream.  Grids deep enough for
+    many chunks per slab; forward modeling and RTM (receivers injected in boundary and
+    interior chunks) are bitwise identical to one slab, and to the serial exchange
+    (SEIS_NO_OVERLAP=1); one slab matches the oracle."""
+    nx, ny, nz = 64, 40, 168
+    el = kind == "elastic"
+    m = inputs.random_media((nz, ny, nx), seed=21, elastic=el)
+    h, dt, nt, snap = 10.0, 5e-4, 40, 4
+    w = inputs.source_series(kind, nt, dt, 35.0)
+    src = (nx // 2, ny // 2, 84)
+    rec = _deep_recs(nx, ny, nz)
+    data = np.random.default_rng(2).standard_normal((nt, rec.shape[0])).astype(np.float32)
+    runs = []
+    for P, serial in ((1, False), (2, False), (3, False), (3, True)):
+        monkeypatch.setenv("SEIS_NO_OVERLAP", "1" if serial else "0")
+        g = seis.Grid(nx, ny, nz, h, dt, nb=6, free_surface=int(el), pml_f=35.0, slabs=P)
+        mod = seis.Model(g, kind, m["vp"], vs=m.get("vs"), rho=m.get("rho"))
+        shot = seis.Shot(src, w, rec, rec_component=2, snap_period=snap)
+        sg = np.zeros((nt, rec.shape[0]), np.float32)
+        mod.forward_model(shot, sg)
+        img = np.zeros((nz, ny, nx), np.float32)
+        mod.migrate(shot, data, img)
+        runs.append((sg, img))
+        mod.close()
+    for sg, img in runs[1:]:
+        assert np.array_equal(sg, runs[0][0])
+        assert np.array_equal(img, runs[0][1])
+    og = oracle.Grid(nx, ny, nz, h, dt, nb=6, free_surface=int(el), pml_f=35.0)
+    if kind == "iso":
+        ref = oracle.iso_run(og, m["vp"], oracle.iso_state(og), 0, nt, [src], w[:, None], rec)
+    elif kind == "acoustic":
+        ref = oracle.ac_run(og, m["vp"], m["rho"], oracle.ac_state(og), 0, nt, [src], w[:, None], rec)
+    else:
+        ref = oracle.el_run(og, m["vp"], m["vs"], m["rho"], oracle.el_state(og), 0, nt, [src],
+                            w[:, None], rec, component=2)
+    assert rel_l2(runs[0][0], ref) <= TOL_FIELD
+
+
+@pytest.mark.parametrize("kind,P", [("iso", 1), ("acoustic", 1), ("acoustic", 3), ("elastic", 1)])
+def test_checkpointed_rtm_bitwise(kind, P):
+    """f2: RTM with source-state checkpoints (segments of c snapshots recomputed in the
+    backward phase) gives the image of the all-snapshots pool bit for bit, for segment
+    lengths that divide the snapshot count, leave a ragged last segment, or are 1; and the
+    image matches the oracle."""
+    nx, ny, nz = 48, 40, 72
+    el = kind == "elastic"
+    m = inputs.random_media((nz, ny, nx), seed=23, elastic=el)
+    h, dt, nt, snap = 10.0, 5e-4, 61, 4   # 15 snapshots
+    w = inputs.source_series(kind, nt, dt, 35.0)
+    src = (nx // 2, ny // 2, 8)
+    rec = _deep_recs(nx, ny, nz)
+    data = np.random.default_rng(3).standard_normal((nt, rec.shape[0])).astype(np.float32)
+    g = seis.Grid(nx, ny, nz, h, dt, nb=6, free_surface=int(el), pml_f=35.0, slabs=P)
+    mod = seis.Model(g, kind, m["vp"], vs=m.get("vs"), rho=m.get("rho"))
+    imgs = {}
+    for c in (0, 1, 4, 5, 7, 15):
+        img = np.zeros((nz, ny, nx), np.float32)
+        mod.migrate(seis.Shot(src, w, rec, snap_period=snap, ckpt_period=c), data, img)
+        imgs[c] = img
+    mod.close()
+    for c, img in imgs.items():
+        assert np.array_equal(img, imgs[0]), c
+    og = oracle.Grid(nx, ny, nz, h, dt, nb=6, free_surface=int(el), pml_f=35.0)
+    I = oracle.migrate(og, kind, m["vp"], m.get("rho"), src, w, rec, data.astype(np.float64), snap,
+                       vs=m.get("vs"))
+    assert rel_l2(imgs[0], I) <= TOL_IMAGE
