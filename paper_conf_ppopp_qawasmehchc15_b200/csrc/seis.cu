@@ -23,6 +23,7 @@
 #include "../../include/seis.h"
 #include "common.cuh"
 #include "kernels_acoustic.cuh"
+#include "kernels_acoustic_fused.cuh"
 #include "kernels_aux.cuh"
 #include "kernels_elastic.cuh"
 #include "kernels_iso.cuh"
@@ -123,7 +124,11 @@ namespace {
 constexpr int BYI = SEIS_BYI;  // ISO step (block 16 x BYI threads, 4 x-points each)
 constexpr int BYV = SEIS_BYV;  // acoustic V (block 16 x BYV)
 constexpr int BYP = SEIS_BYP;  // acoustic P (block 16 x BYP)
-constexpr int BYE = SEIS_BYE;  // elastic V and S (block 32 x BYE threads, 2 x-points each)
+constexpr int BYE = SEIS_BYE;
+#ifndef SEIS_BYF
+#define SEIS_BYF 16
+#endif
+constexpr int BYF = SEIS_BYF;  // fused acoustic step (block 16 x BYF, 4 x-points each)  // elastic V and S (block 32 x BYE threads, 2 x-points each)
 constexpr int NPSI = 18;
 
 struct Slab {
@@ -141,7 +146,8 @@ struct Slab {
   CUtensorMap ac_qxt, ac_qyt, ac_ppc, ac_qzc, ac_kc;        // ACOUSTIC P
   CUtensorMap el_sxxt, el_sxyt, el_sxzt, el_syyt, el_syzt, el_vc[3], el_rt, el_rc;  // ELASTIC V
   CUtensorMap el_vt[3], el_sc[6], el_l2m, el_w;                           // ELASTIC S
-  int cur = 0;               // ISO: fld[cur] = u^n
+  CUtensorMap af_pt[2], af_qx[2], af_qy[2], af_qz[2], af_pz[2], af_rt, af_rz, af_k;  // ACOUSTIC fused
+  int cur = 0;               // ISO: fld[cur] = u^n; fused ACOUSTIC: fld[4 cur .. 4 cur + 3] = p, q
   int zc = 1, nzch = 1;      // z-chunking of the stencil launches
   // shot tables
   long long src_o = -1;
@@ -204,6 +210,7 @@ struct seis_model {
   cudaStream_t xs = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   bool no_overlap = false;  // SEIS_NO_OVERLAP=1: serial exchange (A/B measurements)
+  bool ac_fused = false;    // ACOUSTIC: single-sweep fused V+P step (double-buffered state)
   long long g_launches = 0;
 };
 
@@ -341,6 +348,9 @@ seis_status set_smem_attrs() {
   SMEM_ATTR((ac_v_kernel<BYV, true>), AcVStage<BYV>::smem_bytes());
   SMEM_ATTR((ac_p_kernel<BYP, false>), AcPStage<BYP>::smem_bytes());
   SMEM_ATTR((ac_p_kernel<BYP, true>), AcPStage<BYP>::smem_bytes());
+  SMEM_ATTR((ac_fused_kernel<BYF, false, false>), AcFStage<BYF>::smem_bytes());
+  SMEM_ATTR((ac_fused_kernel<BYF, true, false>), AcFStage<BYF>::smem_bytes());
+  SMEM_ATTR((ac_fused_kernel<BYF, false, true>), AcFStage<BYF>::smem_bytes());
   SMEM_ATTR((el_v_kernel<BYE, false>), ElVStage<BYE>::smem_bytes());
   SMEM_ATTR((el_v_kernel<BYE, true>), ElVStage<BYE>::smem_bytes());
   SMEM_ATTR((el_s_kernel<BYE, false>), ElSStage<BYE>::smem_bytes());
@@ -350,20 +360,27 @@ seis_status set_smem_attrs() {
   return SEIS_OK;
 }
 
-// Choose the z-chunk: enough blocks for >= 6 waves of the resident
-// slots (dynamic block scheduling keeps the tail short), chunks of >= 8 planes so
-// the 8-plane queue warm-up stays bounded (large grids stop at the wave rule first).
-void choose_chunks(Slab& s, int resident_per_sm, int nsm, int tw, int by) {
+// Choose the z-chunk: at most `zt` planes per chunk (short chunks keep the
+// blocks resident at any moment on a narrow z-band of the whole plane and shrink the tail of
+// the last wave: measured optimum 16 planes for the staggered kernels, 24 for ISO,
+// profiles/r01_sweep_zchunk.jsonl), and in any case enough blocks for >= 6 waves of the
+// resident slots; chunks of >= 8 planes (the queue warm-up re-reads 8 planes).
+// SEIS_ZCHUNK_MAX overrides zt (sweeps).
+void choose_chunks(Slab& s, int resident_per_sm, int nsm, int tw, int by, int zt) {
   const long long bxy = (long long)((s.d.nx + tw - 1) / tw) * ((s.d.ny + by - 1) / by);
   const long long slots = (long long)std::max(1, resident_per_sm) * nsm;
+  static const int zenv = getenv("SEIS_ZCHUNK_MAX") ? atoi(getenv("SEIS_ZCHUNK_MAX")) : -1;
+  const int zmax = zenv >= 0 ? zenv : zt;
   int c = 1;
   while (bxy * c < 6 * slots && (s.d.nzl + c) / (c + 1) >= 8) ++c;
+  if (zmax >= 8)
+    while ((s.d.nzl + c - 1) / c > zmax) ++c;
   s.zc = (s.d.nzl + c - 1) / c;
   s.nzch = (s.d.nzl + s.zc - 1) / s.zc;
 }
 
-int nfields(seis_kind k) { return k == SEIS_ISO ? 2 : (k == SEIS_ACOUSTIC ? 4 : 9); }
-int npsi_of(seis_kind k) { return k == SEIS_ACOUSTIC ? 6 : (k == SEIS_ELASTIC ? 18 : 0); }
+int nfields(seis_kind k, bool fused = true) { return k == SEIS_ISO ? 2 : (k == SEIS_ACOUSTIC ? (fused ? 8 : 4) : 9); }
+int npsi_of(seis_kind k, bool fused = true) { return k == SEIS_ACOUSTIC ? (fused ? 9 : 6) : (k == SEIS_ELASTIC ? 18 : 0); }
 // axis of each C-PML memory array: ACOUSTIC psi_p (x,y,z), psi_q (x,y,z); ELASTIC in the
 // oracle's order
 int psi_axis(seis_kind k, int t) {
@@ -418,11 +435,11 @@ seis_status exchange_arrays(seis_model* M, const std::vector<ArrFn>& arrs, int n
   return SEIS_OK;
 }
 
-// 4-plane exchange of state fields by index
-seis_status exchange(seis_model* M, const std::vector<int>& fields, cudaStream_t st) {
+// np-plane (default 4) exchange of state fields by index
+seis_status exchange(seis_model* M, const std::vector<int>& fields, cudaStream_t st, int np = 4) {
   std::vector<ArrFn> arrs;
   for (int f : fields) arrs.push_back([f](Slab& S) { return S.fld[f]; });
-  return exchange_arrays(M, arrs, 4, st);
+  return exchange_arrays(M, arrs, np, st);
 }
 
 }  // namespace
@@ -643,6 +660,20 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
         if (ln < 4) return fail(SEIS_EINVAL, "z-slab of %d planes: the decomposition needs >= 4", ln);
       }
   }
+  // fused acoustic step (f1) with SEIS_AC_FUSED=1 -- slower than the split pair on B200 so
+  // far, kept as the measured alternative -- unless a z-slab is thinner than
+  // the 8 ghost planes of p it exchanges
+  if (kind == SEIS_ACOUSTIC) {
+    const char* e = getenv("SEIS_AC_FUSED");
+    M->ac_fused = e && e[0] == '1';
+    for (int r = 0; r < M->nranks && (ns > 1 || M->nranks > 1); ++r)
+      for (int s = 0; s < ns; ++s) {
+        int rz0, rn, lz0, ln;
+        seis_slab_bounds(g.nz, M->nranks, r, &rz0, &rn);
+        seis_slab_bounds(rn, ns, s, &lz0, &ln);
+        if (ln < 8) M->ac_fused = false;
+      }
+  }
   M->slabs.resize(ns);
   for (int s = 0; s < ns; ++s) {
     int lz0, lnz;
@@ -652,7 +683,7 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     const Dims& d = S.d;
     const size_t sp = (size_t)lnz * plane;  // slab points
     const size_t off = (size_t)lz0 * plane;
-    S.fld.resize(nfields(kind));
+    S.fld.resize(nfields(kind, M->ac_fused));
     for (auto& f : S.fld) TRY(alloc_padded(M, d, &f, st));
     // per-point coefficients (double -> fp32), compact then padded on device
     std::vector<float> hc(sp);
@@ -691,7 +722,7 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       // compact C-PML memory slabs
       if (M->W > 0) {
         const int W = M->W;
-        const int npsi = npsi_of(kind);
+        const int npsi = npsi_of(kind, M->ac_fused);
         for (int t = 0; t < npsi; ++t) {
           const int ax = psi_axis(kind, t);
           size_t n;
@@ -722,6 +753,18 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       TRY(make_map(&S.ac_ppc, S.fld[0], d, TXV, BYP));
       TRY(make_map(&S.ac_qzc, S.fld[3], d, TXV, BYP));
       TRY(make_map(&S.ac_kc, S.kdt, d, TXV, BYP));
+      if (M->ac_fused) {
+        for (int c = 0; c < 2; ++c) {
+          TRY(make_map(&S.af_pt[c], S.fld[4 * c], d, TXV + 16, BYF + 16));
+          TRY(make_map(&S.af_qx[c], S.fld[4 * c + 1], d, TXV + 8, BYF));
+          TRY(make_map(&S.af_qy[c], S.fld[4 * c + 2], d, TXV, BYF + 8));
+          TRY(make_map(&S.af_qz[c], S.fld[4 * c + 3], d, TXV, BYF));
+          TRY(make_map(&S.af_pz[c], S.fld[4 * c], d, TXV, BYF));
+        }
+        TRY(make_map(&S.af_rt, S.rho, d, TXV + 12, BYF + 9));
+        TRY(make_map(&S.af_rz, S.rho, d, TXV, BYF));
+        TRY(make_map(&S.af_k, S.kdt, d, TXV, BYF));
+      }
     } else {
       TRY(make_map(&S.el_sxxt, S.fld[ESXX], d, TXE + 8, BYE));
       TRY(make_map(&S.el_sxyt, S.fld[ESXY], d, TXE + 8, BYE + 8));
@@ -743,14 +786,18 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     if (kind == SEIS_ISO)
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, iso_step_kernel<BYI, false, false>, NTX * BYI,
                                                     IsoStage<BYI>::smem_bytes());
+    else if (kind == SEIS_ACOUSTIC && M->ac_fused)
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_fused_kernel<BYF, false, false>, NTX * BYF,
+                                                    AcFStage<BYF>::smem_bytes());
     else if (kind == SEIS_ACOUSTIC)
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_v_kernel<BYV, false>, NTX * BYV,
                                                     AcVStage<BYV>::smem_bytes());
     else
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, NTX2 * BYE,
                                                     ElSStage<BYE>::smem_bytes());
-    if (kind == SEIS_ELASTIC) choose_chunks(S, occ, dev_sms, TXE, BYE);
-    else choose_chunks(S, occ, dev_sms, TXV, kind == SEIS_ISO ? BYI : BYV);
+    if (kind == SEIS_ELASTIC) choose_chunks(S, occ, dev_sms, TXE, BYE, 16);
+    else if (kind == SEIS_ISO) choose_chunks(S, occ, dev_sms, TXV, BYI, 24);
+    else choose_chunks(S, occ, dev_sms, TXV, M->ac_fused ? BYF : BYV, M->ac_fused ? 64 : 16);
   }
   if (ns > 1 || M->nranks > 1) {
     const char* e = getenv("SEIS_NO_OVERLAP");
@@ -830,14 +877,14 @@ seis_status seis_memory_required(const seis_grid* g, seis_kind kind, const seis_
   if (kind != SEIS_ISO && g->nb > 0) {
     const double W = g->nb + 1;
     const double per = (2 * W * g->ny * (double)nzl + 2 * W * g->nx * (double)nzl + 2 * W * g->nx * (double)g->ny) * 4.0;
-    b += per * (kind == SEIS_ACOUSTIC ? 2 : 6);
+    b += per * (kind == SEIS_ACOUSTIC ? 3 : 6);
   }
   if (shot && shot->snap_period >= 1 && shot->nt >= 1) {
     const long long nsnap = (shot->nt - 1) / shot->snap_period;
     const long long c = shot->ckpt_period > 0 ? std::min<long long>(shot->ckpt_period, nsnap) : nsnap;
     const long long nckpt = nsnap > 0 && c > 0 ? (nsnap + c - 1) / c - 1 : 0;
-    // checkpoint = every padded state field + the C-PML memory slabs
-    double ck = nf * (padded + 128.0);
+    // checkpoint = every padded state field of the current set + the C-PML memory slabs
+    double ck = (kind == SEIS_ACOUSTIC ? 4 : nf) * (padded + 128.0);
     if (kind != SEIS_ISO && g->nb > 0) {
       const double W = g->nb + 1;
       ck += (2 * W * g->ny * (double)nzl + 2 * W * g->nx * (double)nzl + 2 * W * g->nx * (double)g->ny) * 4.0 *
@@ -975,7 +1022,7 @@ seis_status zero_state(seis_model* M, cudaStream_t st) {
     for (float* f : S.fld) CK(cudaMemsetAsync(f, 0, elems * sizeof(float), st));
     if (M->W > 0) {
       const int W = M->W;
-      const int npsi = npsi_of(M->kind);
+      const int npsi = npsi_of(M->kind, M->ac_fused);
       for (int t = 0; t < npsi; ++t) {
         const int ax = psi_axis(M->kind, t);
         size_t n;
@@ -996,10 +1043,15 @@ std::vector<std::pair<float*, size_t>> state_arrays(seis_model* M) {
   std::vector<std::pair<float*, size_t>> v;
   for (Slab& S : M->slabs) {
     const size_t elems = (size_t)S.d.PS * (S.d.nzl + 2 * GZ) + 32;  // + the 128-byte alignment pad
-    for (float* f : S.fld) v.emplace_back(f - 28, elems);             // base = f - 112 bytes
+    // fused ACOUSTIC: only the current set (fields, psi_p) and psi_q hold state
+    const bool fz = M->ac_fused;
+    for (size_t f = 0; f < S.fld.size(); ++f)
+      if (!fz || (int)f / 4 == S.cur) v.emplace_back(S.fld[f] - 28, elems);  // base = f - 112 bytes
     if (M->W > 0) {
       const int W = M->W;
-      for (int t = 0; t < npsi_of(M->kind); ++t) {
+      for (int t = 0; t < npsi_of(M->kind, fz); ++t) {
+        if (fz && t < 3 && S.cur != 0) continue;
+        if (fz && t >= 6 && S.cur != 1) continue;
         const int ax = psi_axis(M->kind, t);
         size_t n;
         if (ax == 0) n = (size_t)S.d.nzl * S.d.ny * 2 * W;
@@ -1065,7 +1117,7 @@ seis_status inject_rows(seis_model* M, const float* row, int part, cudaStream_t 
         inject_el_kernel<<<(G2.n + 127) / 128, 128, 0, st>>>(S.fld[ESXX], S.fld[ESYY], S.fld[ESZZ], G2.off,
                                                             G2.scale, G2.start, G2.mem, row, G2.surf, G2.n);
       } else {
-        float* f = M->kind == SEIS_ISO ? S.fld[S.cur] : S.fld[0];
+        float* f = M->kind == SEIS_ISO ? S.fld[S.cur] : S.fld[4 * S.cur];
         inject_kernel<<<(G2.n + 127) / 128, 128, 0, st>>>(f, G2.off, G2.scale, G2.start, G2.mem, row, G2.n);
       }
       CKL();
@@ -1168,6 +1220,69 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       return SEIS_OK;
     };
     return run_phase(M, k_iso, post, st);
+  }
+  if (M->kind == SEIS_ACOUSTIC && M->ac_fused) {
+    const int c = M->slabs[0].cur;  // read set; the step writes set 1 - c
+    LaunchFn k_f = [&](size_t s, int ch0, int chs, int nch, cudaStream_t ks) -> seis_status {
+      Slab& S = M->slabs[s];
+      AcFArgs a;
+      a.mpt = S.af_pt[c];
+      a.mrt = S.af_rt;
+      a.mqx = S.af_qx[c];
+      a.mqy = S.af_qy[c];
+      a.mqz = S.af_qz[c];
+      a.mrz = S.af_rz;
+      a.mpz = S.af_pz[c];
+      a.mk = S.af_k;
+      a.p0 = S.fld[4 * c];
+      a.qz0 = S.fld[4 * c + 3];
+      a.rho = S.rho;
+      a.p1 = S.fld[4 * (1 - c)];
+      a.qx1 = S.fld[4 * (1 - c) + 1];
+      a.qy1 = S.fld[4 * (1 - c) + 2];
+      a.qz1 = S.fld[4 * (1 - c) + 3];
+      a.dth = (float)((double)M->g.dt / (double)M->g.h);
+      a.W = M->W;
+      a.zlo = 1;
+      a.cx = M->cp[0];
+      a.cy = M->cp[1];
+      a.cz = M->cp[2];
+      for (int t = 0; t < 3; ++t) {
+        a.psr[t] = S.psi[c ? 6 + t : t];
+        a.psw[t] = S.psi[c ? t : 6 + t];
+        a.pq[t] = S.psi[3 + t];
+      }
+      a.d = S.d;
+      a.zc = S.zc;
+      a.ch0 = ch0;
+      a.chs = chs;
+      a.src_o = with_src ? S.src_o : -1;
+      a.src_amp = 0.f;
+      if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
+      a.snap = snap ? (*snap)[s] : nullptr;
+      a.imgS = imgS ? (*imgS)[s] : nullptr;
+      a.img = img ? (*img)[s] : nullptr;
+      const dim3 gr = grid_of(S, TXV, BYF, nch), blk(NTX, BYF);
+      {
+        PROF(1, ks);
+        const size_t sb = AcFStage<BYF>::smem_bytes();
+        if (a.snap) ac_fused_kernel<BYF, true, false><<<gr, blk, sb, ks>>>(a);
+        else if (a.img) ac_fused_kernel<BYF, false, true><<<gr, blk, sb, ks>>>(a);
+        else ac_fused_kernel<BYF, false, false><<<gr, blk, sb, ks>>>(a);
+      }
+      CKL();
+      return SEIS_OK;
+    };
+    for (Slab& S : M->slabs) S.cur = 1 - c;  // injection / exchange act on the new set
+    PostFn post = [&](int part, cudaStream_t ps) -> seis_status {
+      TRY(inject(part, ps));
+      if (part == 1) return SEIS_OK;
+      // the next sweep recomputes q_z 4 planes into the neighbour slab: 8 ghost planes of p,
+      // 4 of q_z
+      TRY(exchange(M, {4 * (1 - c)}, ps, 8));
+      return exchange(M, {4 * (1 - c) + 3}, ps, 4);
+    };
+    return run_phase(M, k_f, post, st);
   }
   if (M->kind == SEIS_ACOUSTIC) {
     LaunchFn k_v = [&](size_t s, int ch0, int chs, int nch, cudaStream_t ks) -> seis_status {
@@ -1348,7 +1463,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
 // Field holding the recorded / imaged quantity
 const float* out_field(seis_model* M, Slab& S, int comp) {
   if (M->kind == SEIS_ISO) return S.fld[S.cur];
-  if (M->kind == SEIS_ACOUSTIC) return S.fld[0];
+  if (M->kind == SEIS_ACOUSTIC) return S.fld[4 * S.cur];
   if (comp == 3) return S.fld[3];
   return S.fld[comp];
 }
@@ -1565,13 +1680,13 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
         if (seg == 0) {
           TRY(zero_state(M, st));
         } else {
-          TRY(state_copy(M, slot_of(seg - 1), false, st));
           for (Slab& S : M->slabs) S.cur = ckpt_cur[seg - 1];
+          TRY(state_copy(M, slot_of(seg - 1), false, st));
         }
         const int last_j = std::min((seg + 1) * c, nsnap) * snap;
         TRY(forward(seg * c * snap, last_j, seg, false));
-        TRY(state_copy(M, slot_of(seg), false, st));
         for (Slab& S : M->slabs) S.cur = rcur;
+        TRY(state_copy(M, slot_of(seg), false, st));
         loaded = seg;
       }
       snap_ptrs(i, tmp);
@@ -1590,7 +1705,7 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
 seis_status seis_get_field(const seis_model* Mc, int32_t which, float* dst, void* stream) {
   seis_model* M = const_cast<seis_model*>(Mc);
   if (!M || !dst) return fail(SEIS_EINVAL, "null argument");
-  const int nf = nfields(M->kind);
+  const int nf = nfields(M->kind, false);
   if (which < 0 || which >= nf) return fail(SEIS_EINVAL, "field index %d out of range", which);
   CK(cudaSetDevice(M->device));
   cudaStream_t st = (cudaStream_t)stream;
@@ -1605,6 +1720,7 @@ seis_status seis_get_field(const seis_model* Mc, int32_t which, float* dst, void
   for (Slab& S : M->slabs) {
     int f = which;
     if (M->kind == SEIS_ISO) f = which == 0 ? S.cur : 1 - S.cur;
+    if (M->kind == SEIS_ACOUSTIC) f = 4 * S.cur + which;
     unpad_kernel<<<1024, 256, 0, st>>>(out + (size_t)(S.d.z0 - M->pz0) * g.ny * g.nx, S.fld[f], S.d);
     CKL();
   }

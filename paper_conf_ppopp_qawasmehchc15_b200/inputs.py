@@ -95,14 +95,17 @@ def layered_acoustic(nx, ny, nz, scale=None):
     iface = [40, 120, 220, 320, 420]
     vps = [1500.0, 1800.0, 2200.0, 2700.0, 3200.0, 3800.0]
     und = _undulation(nx, ny, s)  # [ny][nx]
-    z = np.arange(nz, dtype=np.float64)[:, None, None]
-    layer = np.zeros((nz, ny, nx), dtype=np.int32)
-    for zi in iface:
-        depth = zi * s + und[None, :, :]
-        layer += (z >= depth).astype(np.int32)
-    vp = np.asarray(vps, dtype=np.float32)[layer]
-    rho = gardner(vp)
-    rho[layer == 0] = 1000.0
+    vp = np.empty((nz, ny, nx), dtype=np.float32)
+    rho = np.empty((nz, ny, nx), dtype=np.float32)
+    table = np.asarray(vps, dtype=np.float32)
+    depth = [zi * s + und for zi in iface]
+    for k in range(nz):  # plane by plane (bounded host memory at 1024^3)
+        layer = np.zeros((ny, nx), dtype=np.int32)
+        for dz in depth:
+            layer += (float(k) >= dz).astype(np.int32)
+        vp[k] = table[layer]
+        rho[k] = gardner(vp[k])
+        rho[k][layer == 0] = 1000.0
     return {"vp": vp, "rho": rho}
 
 
@@ -112,15 +115,18 @@ def salt_acoustic(nx, ny, nz):
     z = 140 to 250 (all scaled by n/512)."""
     m = layered_acoustic(nx, ny, nz)
     sx, sy, sz = nx / 512.0, ny / 512.0, nz / 512.0
-    z = np.arange(nz, dtype=np.float64)[:, None, None]
-    y = np.arange(ny, dtype=np.float64)[None, :, None]
-    x = np.arange(nx, dtype=np.float64)[None, None, :]
+    y = np.arange(ny, dtype=np.float64)[:, None]
+    x = np.arange(nx, dtype=np.float64)[None, :]
     cx, cy, cz = 256 * sx, 256 * sy, 250 * sz
-    ell = ((x - cx) / (150 * sx)) ** 2 + ((y - cy) / (120 * sy)) ** 2 + ((z - cz) / (80 * sz)) ** 2 <= 1.0
-    stem = (((x - cx) / sx) ** 2 + ((y - cy) / sy) ** 2 <= 40.0 ** 2) & (z >= 140 * sz) & (z <= 250 * sz)
-    salt = ell | stem
-    m["vp"][salt] = 4500.0
-    m["rho"][salt] = 2150.0
+    exy = ((x - cx) / (150 * sx)) ** 2 + ((y - cy) / (120 * sy)) ** 2
+    disc = ((x - cx) / sx) ** 2 + ((y - cy) / sy) ** 2 <= 40.0 ** 2
+    for k in range(nz):  # plane by plane (bounded host memory at 1024^3)
+        z = float(k)
+        salt = exy + ((z - cz) / (80 * sz)) ** 2 <= 1.0
+        if 140 * sz <= z <= 250 * sz:
+            salt = salt | disc
+        m["vp"][k][salt] = 4500.0
+        m["rho"][k][salt] = 2150.0
     return m
 
 
@@ -243,3 +249,12 @@ def recommended_snap(dt, fp):
     """snap_period = floor(1 / (2 f_max dt)), f_max = 2.5 fp ("depends on the maximum
     frequency", P:177)."""
     return max(1, int(math.floor(1.0 / (2.0 * 2.5 * fp * dt))))
+
+
+def c5(n=1024, nt=1000, nb=20, snap=20):
+    """C5: acoustic RTM 1024^3 -- the C4 geometry scaled x2 in points (same h): salt model,
+    1000 steps of 0.8 ms, source at (n/2, n/2, 48), receiver carpet at z = 48, x, y in
+    40 .. n-41 step 8 (13 924 receivers), snapshots every 20 steps (49)."""
+    wl = c4(n=n, nt=nt, nb=nb, snap=snap, carpet_step=4)
+    wl.name = "C5"
+    return wl

@@ -1,0 +1,163 @@
+"""C5 on ONE B200 (BASELINE.json configs[4]): acoustic RTM 1024^3.
+
+The driver's scaling run covers N > 1 (bench.py under torchrun); on a single GPU this tool
+measures what C5 needs there:
+  1. forward modeling 1024^3 (the strong-scaling propagation base, P = 1),
+  2. one full checkpointed RTM shot 1024^3, nt = 1000, snap 20 (49 snapshots = 196 GiB do
+     not fit in 180 GB: source-state checkpoints, f2), shots/hour,
+  3. the z-slab decomposition path on one GPU (slabs = 8, halo copies between slabs) with
+     the overlapped exchange and with the serial one (SEIS_NO_OVERLAP=1), against slabs = 1.
+Prints one JSON line.  Timing: CUDA events on the launching stream after a warm-up.
+
+    python tools/c5_bench.py [--n 1024] [--nt 1000] [--short 100] [--out gpurun_out/c5.json]
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+import numpy as np
+import torch
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import paper_conf_ppopp_qawasmehchc15_b200 as seis  # noqa: E402
+from paper_conf_ppopp_qawasmehchc15_b200 import inputs  # noqa: E402
+
+
+def timed(fn, stream, reps=1, warm=1):
+    for _ in range(warm):
+        fn()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(reps):
+        fn()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / reps
+
+
+def smooth_gpu(a, sigma, dev):
+    """Migration model: separable 3D Gaussian (sigma in points, 'nearest' edges) on the GPU,
+    plane by plane so the temporaries stay small (input preparation, not the method)."""
+    r = int(4 * sigma + 0.5)
+    x = torch.arange(-r, r + 1, dtype=torch.float32, device=dev)
+    w = torch.exp(-0.5 * (x / sigma) ** 2)
+    w = (w / w.sum()).view(1, 1, -1)
+    t = torch.from_numpy(a).to(dev)
+    nz, ny, nx = t.shape
+    out = torch.empty_like(t)
+    # x and y: per z-plane
+    for k in range(nz):
+        p = t[k]
+        p = torch.nn.functional.conv1d(torch.nn.functional.pad(p.view(ny, 1, nx), (r, r), mode="replicate"), w).view(ny, nx)
+        p = torch.nn.functional.conv1d(torch.nn.functional.pad(p.t().contiguous().view(nx, 1, ny), (r, r), mode="replicate"), w).view(nx, ny).t()
+        out[k] = p
+    # z: per y-row block
+    for j0 in range(0, ny, 64):
+        blk = out[:, j0:j0 + 64, :].permute(1, 2, 0).contiguous()  # [yb][nx][nz]
+        yb = blk.shape[0]
+        b = torch.nn.functional.conv1d(torch.nn.functional.pad(blk.view(yb * nx, 1, nz), (r, r), mode="replicate"), w)
+        out[:, j0:j0 + 64, :] = b.view(yb, nx, nz).permute(2, 0, 1)
+    res = out.cpu().numpy()
+    del t, out
+    torch.cuda.empty_cache()
+    return res
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--n", type=int, default=1024)
+    ap.add_argument("--nt", type=int, default=1000)
+    ap.add_argument("--short", type=int, default=100, help="steps of the decomposition runs")
+    ap.add_argument("--out", default=None)
+    a = ap.parse_args()
+    dev = torch.device("cuda", 0)
+    stream = torch.cuda.current_stream()
+    res = {"workload": f"C5 acoustic RTM {a.n}^3 salt model, nt={a.nt}, snap 20, carpet step 8, 1 GPU"}
+    t0 = time.time()
+    wl = inputs.c5(n=a.n, nt=a.nt)
+    res["model_build_s"] = round(time.time() - t0, 1)
+    npts = float(wl.npts)
+    g = seis.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=wl.nb, pml_f=wl.fp)
+    shot = seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap)
+
+    # 1. forward modeling on the true model = the observed data of the RTM
+    m = seis.Model(g, "acoustic", wl.model["vp"], rho=wl.model["rho"], device=0)
+    data = torch.empty((wl.nt, shot.nrec), device=dev)
+    ms = timed(lambda: m.forward_model(shot, data, stream), stream, reps=1, warm=1)
+    res["forward"] = {"gpts_s": round(npts * wl.nt / (ms * 1e-3) / 1e9, 2), "ms_per_shot": round(ms, 1),
+                      "receivers": shot.nrec}
+    m.close()
+    del m
+    torch.cuda.empty_cache()
+
+    # 2. checkpointed RTM on the smoothed model
+    t0 = time.time()
+    sm = {k: smooth_gpu(v, 5.0, dev) for k, v in wl.model.items()}
+    res["smooth_s"] = round(time.time() - t0, 1)
+    del wl.model
+    free, total = torch.cuda.mem_get_info(dev)
+    nsnap = (wl.nt - 1) // wl.snap
+    need_all = seis.memory_required(g, "acoustic", shot)
+    img_bytes = npts * 4 + data.numel() * 4
+    c = 0
+    if need_all + img_bytes > 0.97 * free:
+        # smallest pool: c ~ sqrt(nsnap * checkpoint / snapshot), then the largest c that fits
+        best = None
+        for cc in range(1, nsnap + 1):
+            need = seis.memory_required(g, "acoustic", seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap,
+                                                                 ckpt_period=cc))
+            if need + img_bytes <= 0.95 * free:
+                best = cc if best is None else max(best, cc)
+        if best is None:
+            raise SystemExit("C5 RTM does not fit even with checkpointing")
+        c = best
+    rshot = seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap, ckpt_period=c)
+    mig = seis.Model(g, "acoustic", sm["vp"], rho=sm["rho"], device=0)
+    img = torch.zeros((wl.nz, wl.ny, wl.nx), device=dev)
+    ms = timed(lambda: mig.migrate(rshot, data, img, stream), stream, reps=1, warm=1)
+    nseg = (nsnap + c - 1) // c if c else 1
+    recompute_steps = 0
+    if c:
+        for s in range(nseg - 1):
+            recompute_steps += min((s + 1) * c, nsnap) * wl.snap - s * c * wl.snap
+    res["rtm"] = {"shots_per_hour": round(3600.0 / (ms * 1e-3), 1), "ms_per_shot": round(ms, 1),
+                  "gpts_s_both_phases": round(2 * npts * wl.nt / (ms * 1e-3) / 1e9, 2),
+                  "gpts_s_all_steps": round(npts * (2 * wl.nt + recompute_steps) / (ms * 1e-3) / 1e9, 2),
+                  "snapshots": nsnap, "ckpt_period": c, "segments": nseg, "recomputed_steps": recompute_steps,
+                  "pool_bytes": int(seis.memory_required(g, "acoustic", rshot) - seis.memory_required(g, "acoustic")),
+                  "all_snapshots_would_need_bytes": int(need_all), "free_bytes_before": int(free),
+                  "image_norm": float(img.norm().item())}
+    mig.close()
+    del mig, img
+    torch.cuda.empty_cache()
+
+    # 3. decomposition path on one GPU: slabs = 1 / 8 (overlapped) / 8 (serial)
+    K = a.short
+    w = wl.wavelet[:K]
+    fshot = seis.Shot(wl.src, w, wl.rec)
+    buf = torch.empty((K, fshot.nrec), device=dev)
+    dec = {}
+    for name, P, serial in (("slabs1", 1, False), ("slabs8_overlap", 8, False), ("slabs8_serial", 8, True)):
+        os.environ["SEIS_NO_OVERLAP"] = "1" if serial else "0"
+        gg = seis.Grid(g.nx, g.ny, g.nz, g.h, g.dt, nb=g.nb, pml_f=g.pml_f, slabs=P)
+        mm = seis.Model(gg, "acoustic", sm["vp"], rho=sm["rho"], device=0)
+        ms = timed(lambda: mm.forward_model(fshot, buf, stream), stream, reps=2, warm=1)
+        dec[name] = {"gpts_s": round(npts * K / (ms * 1e-3) / 1e9, 2), "ms_per_step": round(ms / K, 3)}
+        mm.close()
+        del mm
+        torch.cuda.empty_cache()
+    os.environ.pop("SEIS_NO_OVERLAP", None)
+    res["decomposition_1gpu"] = dec
+    line = json.dumps(res)
+    print(line)
+    if a.out:
+        with open(a.out, "w") as f:
+            f.write(line + "\n")
+
+
+if __name__ == "__main__":
+    main()
