@@ -248,30 +248,30 @@ __device__ __forceinline__ void st2_masked(float* p, const F2& a, int x0, int nx
 // and the derivative arithmetic) and store the updated values afterwards.
 namespace seis {
 
-// compact-slab indices of the NV points of a group (or -1 outside the layer / grid)
+// compact-slab indices of the NV points of a group (or -1 outside the layer / grid).
+// 32-bit: a compact slab holds < 2^31 points up to 1024^3 grids (checked at create).
 template <int NV>
-__device__ __forceinline__ void psi_idx_x(long long* ix, const Dims& d, int W, int x0, int j, int k) {
+__device__ __forceinline__ void psi_idx_x(int* ix, const Dims& d, int W, int x0, int j, int k) {
 #pragma unroll
   for (int e = 0; e < NV; ++e) {
     const int x = x0 + e;
-    ix[e] = (x < d.nx && CpmlIdx::in(x, d.nx, W, true))
-                ? ((long long)k * d.ny + j) * (2 * W) + CpmlIdx::slot(x, d.nx, W)
-                : -1;
+    ix[e] = (x < d.nx && CpmlIdx::in(x, d.nx, W, true)) ? (k * d.ny + j) * (2 * W) + CpmlIdx::slot(x, d.nx, W)
+                                                          : -1;
   }
 }
 template <int NV>
-__device__ __forceinline__ void psi_idx_row(long long* ix, long long base, int x0, int nx) {
+__device__ __forceinline__ void psi_idx_row(int* ix, int base, int x0, int nx) {
 #pragma unroll
   for (int e = 0; e < NV; ++e) ix[e] = (x0 + e < nx) ? base + e : -1;
 }
 template <int NV>
-__device__ __forceinline__ void psi_ld(float* old, const float* __restrict__ ps, const long long* ix) {
+__device__ __forceinline__ void psi_ld(float* old, const float* __restrict__ ps, const int* ix) {
 #pragma unroll
   for (int e = 0; e < NV; ++e) old[e] = ix[e] >= 0 ? ps[ix[e]] : 0.0f;
 }
 // psi <- b psi + a dv;  dv += psi   (per point coefficients ca[e], cb[e])
 template <int NV>
-__device__ __forceinline__ void psi_upd(float* dv, float* __restrict__ ps, const long long* ix, const float* old,
+__device__ __forceinline__ void psi_upd(float* dv, float* __restrict__ ps, const int* ix, const float* old,
                                         const float* ca, const float* cb) {
 #pragma unroll
   for (int e = 0; e < NV; ++e)

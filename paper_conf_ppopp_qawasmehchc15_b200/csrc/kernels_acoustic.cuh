@@ -30,7 +30,7 @@ struct CpmlAxis {
 #define SEIS_AC_NS 3
 #endif
 #ifndef SEIS_AC_VNS
-#define SEIS_AC_VNS 2
+#define SEIS_AC_VNS 3
 #endif
 constexpr int AC_NS = SEIS_AC_NS;    // P kernel ring depth
 constexpr int AC_VNS = SEIS_AC_VNS;  // V kernel ring depth
@@ -126,18 +126,18 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
     // C-PML: old psi values are loaded before the wait (latency overlap)
     const int gz = k + d.z0;
     const bool lz = Wl > 0 && CpmlIdx::in(gz, d.nz, Wl, a.zlo);
-    long long ixx[4], iyy[4], izz[4];
+    int ixx[4], iyy[4], izz[4];  // 32-bit compact-slab indices (fewer live registers)
     float ox[4], oy[4], oz[4];
     if (own && lx) {
       psi_idx_x<4>(ixx, d, Wl, x0, j, k);
       psi_ld<4>(ox, a.psx, ixx);
     }
     if (own && ly) {
-      psi_idx_row<4>(iyy, ((long long)k * (2 * Wl) + CpmlIdx::slot(j, d.ny, Wl)) * d.nx + x0, x0, d.nx);
+      psi_idx_row<4>(iyy, (k * (2 * Wl) + CpmlIdx::slot(j, d.ny, Wl)) * d.nx + x0, x0, d.nx);
       psi_ld<4>(oy, a.psy, iyy);
     }
     if (own && lz) {
-      psi_idx_row<4>(izz, ((long long)CpmlIdx::slot(gz, d.nz, Wl) * d.ny + j) * d.nx + x0, x0, d.nx);
+      psi_idx_row<4>(izz, (CpmlIdx::slot(gz, d.nz, Wl) * d.ny + j) * d.nx + x0, x0, d.nx);
       psi_ld<4>(oz, a.psz, izz);
     }
     mbar_wait(&bar[s], (it / AC_VNS) & 1);
@@ -317,18 +317,18 @@ __global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ 
     // C-PML: old psi values are loaded before the wait (latency overlap)
     const int gz = k + d.z0;
     const bool lz = Wl > 0 && CpmlIdx::in(gz, d.nz, Wl, a.zlo);
-    long long ixx[4], iyy[4], izz[4];
+    int ixx[4], iyy[4], izz[4];  // 32-bit compact-slab indices (fewer live registers)
     float ox[4], oy[4], oz[4];
     if (own && lx) {
       psi_idx_x<4>(ixx, d, Wl, x0, j, k);
       psi_ld<4>(ox, a.pqx, ixx);
     }
     if (own && ly) {
-      psi_idx_row<4>(iyy, ((long long)k * (2 * Wl) + CpmlIdx::slot(j, d.ny, Wl)) * d.nx + x0, x0, d.nx);
+      psi_idx_row<4>(iyy, (k * (2 * Wl) + CpmlIdx::slot(j, d.ny, Wl)) * d.nx + x0, x0, d.nx);
       psi_ld<4>(oy, a.pqy, iyy);
     }
     if (own && lz) {
-      psi_idx_row<4>(izz, ((long long)CpmlIdx::slot(gz, d.nz, Wl) * d.ny + j) * d.nx + x0, x0, d.nx);
+      psi_idx_row<4>(izz, (CpmlIdx::slot(gz, d.nz, Wl) * d.ny + j) * d.nx + x0, x0, d.nx);
       psi_ld<4>(oz, a.pqz, izz);
     }
     mbar_wait(&bar[s], (it / AC_NS) & 1);

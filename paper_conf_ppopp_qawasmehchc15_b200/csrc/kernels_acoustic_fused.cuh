@@ -293,7 +293,7 @@ __global__ void __launch_bounds__(NTX * BY, BY <= 16 ? 2 : 1) ac_fused_kernel(co
       for (int e = 0; e < 4; ++e) dx[e] = dplus12(xv, e);
       const bool in = jr < d.ny && xg >= 0 && xg < d.nx;
       if (in && Wl > 0 && (xg < Wl || xg + 3 >= d.nx - Wl)) {
-        long long ix[4];
+        int ix[4];
         psi_idx_x<4>(ix, d, Wl, xg, jr, k);
 #pragma unroll
         for (int e = 0; e < 4; ++e)

@@ -175,7 +175,7 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
     // C-PML: old psi values are loaded before the wait (latency overlap)
     const int gz = k + d.z0;
     const bool lz = W > 0 && CpmlIdx::in(gz, d.nz, W, a.zlo);
-    long long ixx[2], iyy[2], izz[2];
+    int ixx[2], iyy[2], izz[2];  // 32-bit compact-slab indices (fewer live registers)
     float ox0[2], ox3[2], ox6[2], oy1[2], oy4[2], oy7[2], oz2[2], oz5[2], oz8[2];
     if (own && lx) {
       psi_idx_x<2>(ixx, d, W, x0, j, k);
@@ -184,13 +184,13 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
       psi_ld<2>(ox6, a.psi[6], ixx);
     }
     if (own && ly) {
-      psi_idx_row<2>(iyy, ((long long)k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0, x0, d.nx);
+      psi_idx_row<2>(iyy, (k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0, x0, d.nx);
       psi_ld<2>(oy1, a.psi[1], iyy);
       psi_ld<2>(oy4, a.psi[4], iyy);
       psi_ld<2>(oy7, a.psi[7], iyy);
     }
     if (own && lz) {
-      psi_idx_row<2>(izz, ((long long)CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0, x0, d.nx);
+      psi_idx_row<2>(izz, (CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0, x0, d.nx);
       psi_ld<2>(oz2, a.psi[2], izz);
       psi_ld<2>(oz5, a.psi[5], izz);
       psi_ld<2>(oz8, a.psi[8], izz);
@@ -393,7 +393,7 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
     // C-PML: old psi values are loaded before the wait (latency overlap)
     const int gz = k + d.z0;
     const bool lz = W > 0 && CpmlIdx::in(gz, d.nz, W, a.zlo);
-    long long ixx[2], iyy[2], izz[2];
+    int ixx[2], iyy[2], izz[2];  // 32-bit compact-slab indices (fewer live registers)
     float ox0[2], ox4[2], ox6[2], oy1[2], oy3[2], oy8[2], oz2[2], oz5[2], oz7[2];
     if (own && lx) {
       psi_idx_x<2>(ixx, d, W, x0, j, k);
@@ -402,13 +402,13 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
       psi_ld<2>(ox6, a.psi[6], ixx);
     }
     if (own && ly) {
-      psi_idx_row<2>(iyy, ((long long)k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0, x0, d.nx);
+      psi_idx_row<2>(iyy, (k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0, x0, d.nx);
       psi_ld<2>(oy1, a.psi[1], iyy);
       psi_ld<2>(oy3, a.psi[3], iyy);
       psi_ld<2>(oy8, a.psi[8], iyy);
     }
     if (own && lz) {
-      psi_idx_row<2>(izz, ((long long)CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0, x0, d.nx);
+      psi_idx_row<2>(izz, (CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0, x0, d.nx);
       psi_ld<2>(oz2, a.psi[2], izz);
       psi_ld<2>(oz5, a.psi[5], izz);
       psi_ld<2>(oz7, a.psi[7], izz);

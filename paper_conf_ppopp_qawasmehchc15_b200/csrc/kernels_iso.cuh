@@ -103,6 +103,9 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
     for (int e = 0; e < 4; ++e) exy.v[e] = ex.v[e] + ey;
   }
   const long long srel0 = a.src_o - oc;  // source offset relative to this column
+  // block-uniform: does this tile touch the x / y damping layer?  Planes outside the z layer
+  // of such tiles take the undamped update without per-point branches (same arithmetic).
+  const bool dxy = __syncthreads_or(exy.v[0] != 0.f || exy.v[1] != 0.f || exy.v[2] != 0.f || exy.v[3] != 0.f);
 
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
@@ -132,23 +135,33 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
     const F4 upv = lds4(st + L::UP + ty * TXV + 4 * tx);
     const F4 mv = lds4(st + L::M + ty * TXV + 4 * tx);
     const float ez = a.edx ? a.edz[k + d.z0] : 0.0f;
-    F4 out;
+    const bool damp = dxy || ez != 0.0f;
+    float lap[4];
 #pragma unroll
     for (int e = 0; e < 4; ++e) {
-      const float u = xv[4 + e];
-      float lap = (3.0f * SEIS_C0) * u;
-      lap = fmaf(SEIS_C1, (xv[3 + e] + xv[5 + e]) + ys[0].v[e] + (q[3].v[e] + q[5].v[e]), lap);
-      lap = fmaf(SEIS_C2, (xv[2 + e] + xv[6 + e]) + ys[1].v[e] + (q[2].v[e] + q[6].v[e]), lap);
-      lap = fmaf(SEIS_C3, (xv[1 + e] + xv[7 + e]) + ys[2].v[e] + (q[1].v[e] + q[7].v[e]), lap);
-      lap = fmaf(SEIS_C4, (xv[0 + e] + xv[8 + e]) + ys[3].v[e] + (q[0].v[e] + q[8].v[e]), lap);
-      const float eta = exy.v[e] + ez;
-      float r;
-      if (eta != 0.0f) {
-        r = (2.0f * u - (1.0f - eta) * upv.v[e] + mv.v[e] * lap) / (1.0f + eta);
-      } else {
-        r = fmaf(mv.v[e], lap, 2.0f * u - upv.v[e]);
+      float l = (3.0f * SEIS_C0) * xv[4 + e];
+      l = fmaf(SEIS_C1, (xv[3 + e] + xv[5 + e]) + ys[0].v[e] + (q[3].v[e] + q[5].v[e]), l);
+      l = fmaf(SEIS_C2, (xv[2 + e] + xv[6 + e]) + ys[1].v[e] + (q[2].v[e] + q[6].v[e]), l);
+      l = fmaf(SEIS_C3, (xv[1 + e] + xv[7 + e]) + ys[2].v[e] + (q[1].v[e] + q[7].v[e]), l);
+      lap[e] = fmaf(SEIS_C4, (xv[0 + e] + xv[8 + e]) + ys[3].v[e] + (q[0].v[e] + q[8].v[e]), l);
+    }
+    F4 out;
+    if (!damp) {  // block-uniform branch
+#pragma unroll
+      for (int e = 0; e < 4; ++e) out.v[e] = fmaf(mv.v[e], lap[e], 2.0f * xv[4 + e] - upv.v[e]);
+    } else {
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const float u = xv[4 + e];
+        const float eta = exy.v[e] + ez;
+        float r;
+        if (eta != 0.0f) {
+          r = (2.0f * u - (1.0f - eta) * upv.v[e] + mv.v[e] * lap[e]) / (1.0f + eta);
+        } else {
+          r = fmaf(mv.v[e], lap[e], 2.0f * u - upv.v[e]);
+        }
+        out.v[e] = r;
       }
-      out.v[e] = r;
     }
     if (own) {
       const long long rel = srel0 - (long long)(k + GZ) * PS;

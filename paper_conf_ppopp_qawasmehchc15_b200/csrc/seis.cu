@@ -719,9 +719,11 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
         }
         TRY(upload_padded_from_host(M, d, hc, &S.wmu, st));
       }
-      // compact C-PML memory slabs
+      // compact C-PML memory slabs (32-bit indices in the kernels)
       if (M->W > 0) {
         const int W = M->W;
+        const double big = std::max((double)lnz * g.ny, std::max((double)lnz * g.nx, (double)g.ny * g.nx)) * 2.0 * W;
+        if (big >= 2147483647.0) return fail(SEIS_EUNSUPPORTED, "C-PML slab of %.0f points exceeds 32-bit indexing", big);
         const int npsi = npsi_of(kind, M->ac_fused);
         for (int t = 0; t < npsi; ++t) {
           const int ax = psi_axis(kind, t);
