@@ -125,12 +125,13 @@ def c2_workload(n=512, nt=2000, nz=None):
     return wl
 
 
-def psi_bytes_per_point(nx, ny, nz, nb, axes_per_dir):
-    """C-PML memory-variable RMW bytes per grid point (8 B per point inside a layer, per axis)."""
+def psi_bytes_per_point(nx, ny, nz, nb, axes_per_dir, free_surface=False):
+    """C-PML memory-variable RMW bytes per grid point (8 B per point inside a layer, per axis;
+    a free-surface top has no layer)."""
     if nb == 0:
         return 0.0
     W = nb + 1
-    frac = [min(1.0, 2 * W / nx), min(1.0, 2 * W / ny), min(1.0, 2 * W / nz)]
+    frac = [min(1.0, 2 * W / nx), min(1.0, 2 * W / ny), min(1.0, (W if free_surface else 2 * W) / nz)]
     return 8.0 * sum(frac) * axes_per_dir / 3.0
 
 
@@ -329,10 +330,12 @@ def run_extras(args, local):
     seis.profile(True)
     ms = _timed_shots(lambda: m.forward_model(shot, buf, stream), 1, stream)
     seis.profile(False)
+    psi_el = psi_bytes_per_point(wl.nx, wl.ny, wl.nz, wl.nb, PSI_AXES["el_v"], free_surface=True)
     res["C3_elastic_384"] = {"gpts_s": round(wl.npts * wl.nt / (ms * 1e-3) / 1e9, 3),
                              "ms_per_shot": round(ms, 3),
-                             "roofline_v": kernel_frac("el_v", float(wl.npts), 52.0),
-                             "roofline_s": kernel_frac("el_s", float(wl.npts), 68.0)}
+                             "alg_bytes_per_point": {"el_v": round(52.0 + psi_el, 2), "el_s": round(68.0 + psi_el, 2)},
+                             "roofline_v": kernel_frac("el_v", float(wl.npts), 52.0 + psi_el),
+                             "roofline_s": kernel_frac("el_s", float(wl.npts), 68.0 + psi_el)}
     m.close()
     torch.cuda.empty_cache()
     # C4: RTM 512^3 salt model: observed data on the true model, migration on the smoothed one

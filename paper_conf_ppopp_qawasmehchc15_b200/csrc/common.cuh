@@ -172,6 +172,24 @@ __device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, u
       : "memory");
 }
 
+// L2 prefetch of a 3D tile (no shared-memory destination, no mbarrier): issued a few planes
+// ahead of the ring so the ring's own TMA load of that plane hits in L2 (SEIS_L2PF planes).
+__device__ __forceinline__ void tma_prefetch_3d(const CUtensorMap* map, int x, int y, int z) {
+  asm volatile("cp.async.bulk.prefetch.tensor.3d.L2.global.tile [%0, {%1, %2, %3}];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(x), "r"(y), "r"(z)
+               : "memory");
+}
+__device__ __forceinline__ void tma_ld(bool pf, void* dst, const CUtensorMap* map, uint64_t* bar, int x, int y,
+                                       int z) {
+  if (pf) tma_prefetch_3d(map, x, y, z);
+  else tma_load_3d(dst, map, bar, x, y, z);
+}
+#ifndef SEIS_L2PF
+#define SEIS_L2PF 0
+#endif
+constexpr int L2PF = SEIS_L2PF;  // L2 prefetch distance beyond the TMA ring (planes), 0 = off
+
 }  // namespace seis
 
 // ------------------------------------------------------------ 4-wide vectors

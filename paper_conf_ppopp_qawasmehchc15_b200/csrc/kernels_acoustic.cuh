@@ -92,17 +92,17 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
   const int Wl = a.W;
   const bool lx = Wl > 0 && (x0 < Wl || x0 + 3 >= d.nx - Wl);  // some component may be in the x layer
   const bool ly = Wl > 0 && CpmlIdx::in(j, d.ny, Wl, true);
-  auto issue = [&](int s, int k) {
+  auto issue = [&](int s, int k, bool pf = false) {
     float* st = sm + s * L::SIZE;
     const int z = k + GZ, x = i0 + G, y = j0 + G;
-    mbar_expect_tx(&bar[s], TX_BYTES);
-    tma_load_3d(st + L::P, &a.mp, &bar[s], i0, j0, z);
-    tma_load_3d(st + L::QX, &a.mqx, &bar[s], x, y, z);
-    tma_load_3d(st + L::QY, &a.mqy, &bar[s], x, y, z);
-    tma_load_3d(st + L::QZ, &a.mqz, &bar[s], x, y, z);
-    tma_load_3d(st + L::R, &a.mr, &bar[s], x, y, z);
-    tma_load_3d(st + L::PQ, &a.mpq, &bar[s], x, y, z + 4);
-    tma_load_3d(st + L::RZ, &a.mrz, &bar[s], x, y, z + 1);
+    if (!pf) mbar_expect_tx(&bar[s], TX_BYTES);
+    tma_ld(pf, st + L::P, &a.mp, &bar[s], i0, j0, z);
+    tma_ld(pf, st + L::QX, &a.mqx, &bar[s], x, y, z);
+    tma_ld(pf, st + L::QY, &a.mqy, &bar[s], x, y, z);
+    tma_ld(pf, st + L::QZ, &a.mqz, &bar[s], x, y, z);
+    tma_ld(pf, st + L::R, &a.mr, &bar[s], x, y, z);
+    tma_ld(pf, st + L::PQ, &a.mpq, &bar[s], x, y, z + 4);
+    tma_ld(pf, st + L::RZ, &a.mrz, &bar[s], x, y, z + 1);
   };
   if (tid == 0) {
     for (int s = 0; s < AC_VNS; ++s) {
@@ -114,6 +114,8 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
   __syncthreads();
   if (tid == 0)
     for (int s = 0; s < AC_VNS && s < np; ++s) issue(s, k0 + s);
+  if (tid == 0)
+    for (int t = 0; t < L2PF && AC_VNS + t < np; ++t) issue(0, k0 + AC_VNS + t, true);
   F4 r[8];  // p at k-3 .. k+4; plane k+4 arrives with stage k (TMA)
 #pragma unroll
   for (int t = 0; t < 7; ++t) r[t] = ldg4(p + (long long)(k0 - 3 + t + GZ) * PS + oc);
@@ -227,7 +229,10 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
         st4_masked(a.img + cix, im, x0, d.nx, false);
       }
     }
-    stage_release(&cnt[s], tid, it + AC_VNS < np, [&] { issue(s, k + AC_VNS); });
+    stage_release(&cnt[s], tid, it + AC_VNS < np, [&] {
+      issue(s, k + AC_VNS);
+      if (L2PF && it + AC_VNS + L2PF < np) issue(s, k + AC_VNS + L2PF, true);
+    });
 #pragma unroll
     for (int t = 0; t < 7; ++t) r[t] = r[t + 1];
   }
@@ -285,15 +290,15 @@ __global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ 
   const int Wl = a.W;
   const bool lx = Wl > 0 && (x0 < Wl || x0 + 3 >= d.nx - Wl);
   const bool ly = Wl > 0 && CpmlIdx::in(j, d.ny, Wl, true);
-  auto issue = [&](int s, int k) {
+  auto issue = [&](int s, int k, bool pf = false) {
     float* st = sm + s * L::SIZE;
     const int z = k + GZ;
-    mbar_expect_tx(&bar[s], TX_BYTES);
-    tma_load_3d(st + L::QX, &a.mqx, &bar[s], i0, j0 + G, z);
-    tma_load_3d(st + L::QY, &a.mqy, &bar[s], i0 + G, j0, z);
-    tma_load_3d(st + L::P, &a.mpp, &bar[s], i0 + G, j0 + G, z);
-    tma_load_3d(st + L::K, &a.mk, &bar[s], i0 + G, j0 + G, z);
-    tma_load_3d(st + L::QQ, &a.mqq, &bar[s], i0 + G, j0 + G, z + 3);
+    if (!pf) mbar_expect_tx(&bar[s], TX_BYTES);
+    tma_ld(pf, st + L::QX, &a.mqx, &bar[s], i0, j0 + G, z);
+    tma_ld(pf, st + L::QY, &a.mqy, &bar[s], i0 + G, j0, z);
+    tma_ld(pf, st + L::P, &a.mpp, &bar[s], i0 + G, j0 + G, z);
+    tma_ld(pf, st + L::K, &a.mk, &bar[s], i0 + G, j0 + G, z);
+    tma_ld(pf, st + L::QQ, &a.mqq, &bar[s], i0 + G, j0 + G, z + 3);
   };
   if (tid == 0) {
     for (int s = 0; s < AC_NS; ++s) {
@@ -305,6 +310,8 @@ __global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ 
   __syncthreads();
   if (tid == 0)
     for (int s = 0; s < AC_NS && s < np; ++s) issue(s, k0 + s);
+  if (tid == 0)
+    for (int t = 0; t < L2PF && AC_NS + t < np; ++t) issue(0, k0 + AC_NS + t, true);
   F4 q[8];  // q_z at k-4 .. k+3; plane k+3 arrives with stage k (TMA)
 #pragma unroll
   for (int t = 0; t < 7; ++t) q[t] = ldg4(qz + (long long)(k0 - 4 + t + GZ) * PS + oc);
@@ -400,7 +407,10 @@ __global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ 
       st4_masked(a.p + o, out, x0, d.nx, true);
       if (SNAP) st4_masked(a.snap + ((long long)k * d.ny + j) * d.nx + x0, out, x0, d.nx, (d.nx & 3) == 0);
     }
-    stage_release(&cnt[s], tid, it + AC_NS < np, [&] { issue(s, k + AC_NS); });
+    stage_release(&cnt[s], tid, it + AC_NS < np, [&] {
+      issue(s, k + AC_NS);
+      if (L2PF && it + AC_NS + L2PF < np) issue(s, k + AC_NS + L2PF, true);
+    });
 #pragma unroll
     for (int t = 0; t < 7; ++t) q[t] = q[t + 1];
   }

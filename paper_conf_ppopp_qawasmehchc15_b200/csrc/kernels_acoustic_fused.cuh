@@ -132,18 +132,18 @@ __global__ void __launch_bounds__(NTX * BY, BY <= 16 ? 2 : 1) ac_fused_kernel(co
   const long long oc = (long long)(j + G) * d.PX + (x0 + G);
   const int Wl = a.W;
   const float dth = a.dth;
-  auto issue = [&](int s, int k) {
+  auto issue = [&](int s, int k, bool pf = false) {
     float* st = sm + s * L::SIZE;
     const int z = k + GZ, x = i0 + G, y = j0 + G;
-    mbar_expect_tx(&bar[s], L::BYTES);
-    tma_load_3d(st + L::PT, &a.mpt, &bar[s], x - 8, y - 8, z);
-    tma_load_3d(st + L::RT, &a.mrt, &bar[s], x - 4, y - 4, z);
-    tma_load_3d(st + L::QX, &a.mqx, &bar[s], x - 4, y, z);
-    tma_load_3d(st + L::QY, &a.mqy, &bar[s], x, y - 4, z);
-    tma_load_3d(st + L::QZ, &a.mqz, &bar[s], x, y, z + 3);
-    tma_load_3d(st + L::RZ, &a.mrz, &bar[s], x, y, z + 4);
-    tma_load_3d(st + L::PZ, &a.mpz, &bar[s], x, y, z + 7);
-    tma_load_3d(st + L::KK, &a.mk, &bar[s], x, y, z);
+    if (!pf) mbar_expect_tx(&bar[s], L::BYTES);
+    tma_ld(pf, st + L::PT, &a.mpt, &bar[s], x - 8, y - 8, z);
+    tma_ld(pf, st + L::RT, &a.mrt, &bar[s], x - 4, y - 4, z);
+    tma_ld(pf, st + L::QX, &a.mqx, &bar[s], x - 4, y, z);
+    tma_ld(pf, st + L::QY, &a.mqy, &bar[s], x, y - 4, z);
+    tma_ld(pf, st + L::QZ, &a.mqz, &bar[s], x, y, z + 3);
+    tma_ld(pf, st + L::RZ, &a.mrz, &bar[s], x, y, z + 4);
+    tma_ld(pf, st + L::PZ, &a.mpz, &bar[s], x, y, z + 7);
+    tma_ld(pf, st + L::KK, &a.mk, &bar[s], x, y, z);
   };
   if (tid == 0) {
     for (int s = 0; s < AF_NS; ++s) {
@@ -154,6 +154,8 @@ __global__ void __launch_bounds__(NTX * BY, BY <= 16 ? 2 : 1) ac_fused_kernel(co
   __syncthreads();
   if (tid == 0)
     for (int s = 0; s < AF_NS && s < np; ++s) issue(s, k0 + s);
+  if (tid == 0)
+    for (int t = 0; t < L2PF && AF_NS + t < np; ++t) issue(0, k0 + AF_NS + t, true);
 
   const bool lxo = Wl > 0 && (x0 < Wl || x0 + 3 >= d.nx - Wl);  // own group may touch the x layer
   const bool lyo = Wl > 0 && CpmlIdx::in(j, d.ny, Wl, true);
@@ -379,6 +381,7 @@ __global__ void __launch_bounds__(NTX * BY, BY <= 16 ? 2 : 1) ac_fused_kernel(co
     if (tid == 0 && it + AF_NS < np) {
       fence_proxy_async();
       issue(s, k + AF_NS);
+      if (L2PF && it + AF_NS + L2PF < np) issue(s, k + AF_NS + L2PF, true);
     }
     // ---- P at plane k
     if (own) {

@@ -131,22 +131,22 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
   const int W = a.W;
   const bool lx = W > 0 && (x0 < W || x0 + 1 >= d.nx - W);
   const bool ly = W > 0 && CpmlIdx::in(j, d.ny, W, true);
-  auto issue = [&](int s, int k) {
+  auto issue = [&](int s, int k, bool pf = false) {
     float* st = sm + s * L::SIZE;
     const int z = k + GZ, x = i0 + G, y = j0 + G;
-    mbar_expect_tx(&bar[s], TX_BYTES);
-    tma_load_3d(st + L::XX, &a.msxx, &bar[s], i0, y, z);
-    tma_load_3d(st + L::XY, &a.msxy, &bar[s], i0, j0, z);
-    tma_load_3d(st + L::XZ, &a.msxz, &bar[s], i0, y, z);
-    tma_load_3d(st + L::YY, &a.msyy, &bar[s], x, j0, z);
-    tma_load_3d(st + L::YZ, &a.msyz, &bar[s], x, j0, z);
+    if (!pf) mbar_expect_tx(&bar[s], TX_BYTES);
+    tma_ld(pf, st + L::XX, &a.msxx, &bar[s], i0, y, z);
+    tma_ld(pf, st + L::XY, &a.msxy, &bar[s], i0, j0, z);
+    tma_ld(pf, st + L::XZ, &a.msxz, &bar[s], i0, y, z);
+    tma_ld(pf, st + L::YY, &a.msyy, &bar[s], x, j0, z);
+    tma_ld(pf, st + L::YZ, &a.msyz, &bar[s], x, j0, z);
 #pragma unroll
-    for (int c = 0; c < 3; ++c) tma_load_3d(st + L::V + c * T, &a.mv[c], &bar[s], x, y, z);
-    tma_load_3d(st + L::R, &a.mr, &bar[s], x, y, z);
-    tma_load_3d(st + L::RZ, &a.mrz, &bar[s], x, y, z + 1);
-    tma_load_3d(st + L::Q, &a.mq[0], &bar[s], x, y, z + 3);
-    tma_load_3d(st + L::Q + T, &a.mq[1], &bar[s], x, y, z + 3);
-    tma_load_3d(st + L::Q + 2 * T, &a.mq[2], &bar[s], x, y, z + 4);
+    for (int c = 0; c < 3; ++c) tma_ld(pf, st + L::V + c * T, &a.mv[c], &bar[s], x, y, z);
+    tma_ld(pf, st + L::R, &a.mr, &bar[s], x, y, z);
+    tma_ld(pf, st + L::RZ, &a.mrz, &bar[s], x, y, z + 1);
+    tma_ld(pf, st + L::Q, &a.mq[0], &bar[s], x, y, z + 3);
+    tma_ld(pf, st + L::Q + T, &a.mq[1], &bar[s], x, y, z + 3);
+    tma_ld(pf, st + L::Q + 2 * T, &a.mq[2], &bar[s], x, y, z + 4);
   };
   if (tid == 0) {
     for (int s = 0; s < EL_VNS; ++s) {
@@ -158,6 +158,8 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
   __syncthreads();
   if (tid == 0)
     for (int s = 0; s < EL_VNS && s < np; ++s) issue(s, k0 + s);
+  if (tid == 0)
+    for (int t = 0; t < L2PF && EL_VNS + t < np; ++t) issue(0, k0 + EL_VNS + t, true);
   const float* __restrict__ sxz = a.f[ESXZ];
   const float* __restrict__ syz = a.f[ESYZ];
   const float* __restrict__ szz = a.f[ESZZ];
@@ -288,7 +290,10 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
           }
       }
     }
-    stage_release(&cnt[s], tid, it + EL_VNS < np, [&] { issue(s, k + EL_VNS); });
+    stage_release(&cnt[s], tid, it + EL_VNS < np, [&] {
+      issue(s, k + EL_VNS);
+      if (L2PF && it + EL_VNS + L2PF < np) issue(s, k + EL_VNS + L2PF, true);
+    });
 #pragma unroll
     for (int t = 0; t < 7; ++t) {
       qxz[t] = qxz[t + 1];
@@ -350,20 +355,20 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
   const int W = a.W;
   const bool lx = W > 0 && (x0 < W || x0 + 1 >= d.nx - W);
   const bool ly = W > 0 && CpmlIdx::in(j, d.ny, W, true);
-  auto issue = [&](int s, int k) {
+  auto issue = [&](int s, int k, bool pf = false) {
     float* st = sm + s * L::SIZE;
     const int z = k + GZ, x = i0 + G, y = j0 + G;
-    mbar_expect_tx(&bar[s], TX_BYTES);
+    if (!pf) mbar_expect_tx(&bar[s], TX_BYTES);
 #pragma unroll
-    for (int c = 0; c < 3; ++c) tma_load_3d(st + L::VT + c * TV, &a.mvt[c], &bar[s], i0, j0, z);
+    for (int c = 0; c < 3; ++c) tma_ld(pf, st + L::VT + c * TV, &a.mvt[c], &bar[s], i0, j0, z);
 #pragma unroll
-    for (int c = 0; c < 6; ++c) tma_load_3d(st + L::S + c * T, &a.ms[c], &bar[s], x, y, z);
-    tma_load_3d(st + L::C, &a.ml2m, &bar[s], x, y, z);
-    tma_load_3d(st + L::WK, &a.mw, &bar[s], x, y, z);
-    tma_load_3d(st + L::WK1, &a.mw, &bar[s], x, y, z + 1);
-    tma_load_3d(st + L::Q, &a.mq[0], &bar[s], x, y, z + 4);
-    tma_load_3d(st + L::Q + T, &a.mq[1], &bar[s], x, y, z + 4);
-    tma_load_3d(st + L::Q + 2 * T, &a.mq[2], &bar[s], x, y, z + 3);
+    for (int c = 0; c < 6; ++c) tma_ld(pf, st + L::S + c * T, &a.ms[c], &bar[s], x, y, z);
+    tma_ld(pf, st + L::C, &a.ml2m, &bar[s], x, y, z);
+    tma_ld(pf, st + L::WK, &a.mw, &bar[s], x, y, z);
+    tma_ld(pf, st + L::WK1, &a.mw, &bar[s], x, y, z + 1);
+    tma_ld(pf, st + L::Q, &a.mq[0], &bar[s], x, y, z + 4);
+    tma_ld(pf, st + L::Q + T, &a.mq[1], &bar[s], x, y, z + 4);
+    tma_ld(pf, st + L::Q + 2 * T, &a.mq[2], &bar[s], x, y, z + 3);
   };
   if (tid == 0) {
     for (int s = 0; s < EL_SNS; ++s) {
@@ -375,6 +380,8 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
   __syncthreads();
   if (tid == 0)
     for (int s = 0; s < EL_SNS && s < np; ++s) issue(s, k0 + s);
+  if (tid == 0)
+    for (int t = 0; t < L2PF && EL_SNS + t < np; ++t) issue(0, k0 + EL_SNS + t, true);
   const float* __restrict__ vx = a.f[EVX];
   const float* __restrict__ vy = a.f[EVY];
   const float* __restrict__ vz = a.f[EVZ];
@@ -533,7 +540,10 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
           if (x0 + e < d.nx) a.snap[cix + e] = -((o6[0].v[e] + o6[1].v[e]) + o6[2].v[e]) / 3.0f;
       }
     }
-    stage_release(&cnt[s], tid, it + EL_SNS < np, [&] { issue(s, k + EL_SNS); });
+    stage_release(&cnt[s], tid, it + EL_SNS < np, [&] {
+      issue(s, k + EL_SNS);
+      if (L2PF && it + EL_SNS + L2PF < np) issue(s, k + EL_SNS + L2PF, true);
+    });
 #pragma unroll
     for (int t = 0; t < 7; ++t) {
       qx[t] = qx[t + 1];

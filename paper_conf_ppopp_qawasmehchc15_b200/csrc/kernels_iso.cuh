@@ -72,13 +72,13 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
   const long long PS = d.PS;
   const long long oc = (long long)(j + G) * d.PX + (x0 + G);
   const float* __restrict__ un = a.un;
-  auto issue = [&](int s, int k) {
+  auto issue = [&](int s, int k, bool pf = false) {
     float* st = sm + s * L::SIZE;
-    mbar_expect_tx(&bar[s], TX_BYTES);
-    tma_load_3d(st + L::U, &a.mun, &bar[s], i0, j0, k + GZ);
-    tma_load_3d(st + L::UP, &a.mup, &bar[s], i0 + G, j0 + G, k + GZ);
-    tma_load_3d(st + L::M, &a.mm, &bar[s], i0 + G, j0 + G, k + GZ);
-    tma_load_3d(st + L::UQ, &a.muq, &bar[s], i0 + G, j0 + G, k + 4 + GZ);
+    if (!pf) mbar_expect_tx(&bar[s], TX_BYTES);
+    tma_ld(pf, st + L::U, &a.mun, &bar[s], i0, j0, k + GZ);
+    tma_ld(pf, st + L::UP, &a.mup, &bar[s], i0 + G, j0 + G, k + GZ);
+    tma_ld(pf, st + L::M, &a.mm, &bar[s], i0 + G, j0 + G, k + GZ);
+    tma_ld(pf, st + L::UQ, &a.muq, &bar[s], i0 + G, j0 + G, k + 4 + GZ);
   };
   if (tid == 0) {
     for (int s = 0; s < ISO_NS; ++s) {
@@ -90,6 +90,8 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
   __syncthreads();
   if (tid == 0)
     for (int s = 0; s < ISO_NS && s < np; ++s) issue(s, k0 + s);
+  if (tid == 0)
+    for (int t = 0; t < L2PF && ISO_NS + t < np; ++t) issue(0, k0 + ISO_NS + t, true);
 
   // z-queue u^n(k-4 .. k+4); plane k+4 arrives with stage k (TMA)
   F4 q[9];
@@ -184,7 +186,10 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
         }
       }
     }
-    stage_release(&cnt[s], tid, it + ISO_NS < np, [&] { issue(s, k + ISO_NS); });
+    stage_release(&cnt[s], tid, it + ISO_NS < np, [&] {
+      issue(s, k + ISO_NS);
+      if (L2PF && it + ISO_NS + L2PF < np) issue(s, k + ISO_NS + L2PF, true);
+    });
 #pragma unroll
     for (int t = 0; t < 8; ++t) q[t] = q[t + 1];
   }

@@ -19,18 +19,10 @@ sys.path.insert(0, ROOT)
 
 VARIANTS = {
     "base": [],
-    "v4_3": ["SEIS_BYV=4", "SEIS_AC_VNS=3"],
-    "v16_2": ["SEIS_BYV=16", "SEIS_AC_VNS=2"],
-    "v8_3": ["SEIS_AC_VNS=3"],
-    "p16_2": ["SEIS_BYP=16", "SEIS_AC_NS=2"],
-    "p8_2": ["SEIS_AC_NS=2"],
-    "p4_4": ["SEIS_BYP=4", "SEIS_AC_NS=4"],
-    "i16_2": ["SEIS_BYI=16", "SEIS_ISO_NS=2"],
-    "i8_2": ["SEIS_ISO_NS=2"],
-    "i4_4": ["SEIS_BYI=4", "SEIS_ISO_NS=4"],
-    "e4": ["SEIS_BYE=4", "SEIS_EL_VNS=4", "SEIS_EL_SNS=3"],
-    "e_v2": ["SEIS_EL_VNS=2"],
-    "e_s3": ["SEIS_EL_SNS=3"],
+    "pf1": ["SEIS_L2PF=1"],
+    "pf2": ["SEIS_L2PF=2"],
+    "pf4": ["SEIS_L2PF=4"],
+    "pf2_es3": ["SEIS_L2PF=2", "SEIS_EL_SNS=3", "SEIS_EL_VNS=2"],
 }
 
 
