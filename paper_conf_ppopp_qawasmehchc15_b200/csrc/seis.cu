@@ -874,12 +874,13 @@ seis_status seis_memory_required(const seis_grid* g, seis_kind kind, const seis_
   seis_slab_bounds(g->nz, nranks, 0, &z0, &nzl);
   const Dims d = make_dims(*g, 0, nzl);
   const double padded = (double)d.PS * (nzl + 2 * GZ) * 4.0;
-  int nf = nfields(kind), np = kind == SEIS_ISO ? 1 : (kind == SEIS_ACOUSTIC ? 2 : 3);  // m | kdt,rho | l2m,w,rho
+  // (the default split acoustic step: 4 fields, psi_p + psi_q; SEIS_AC_FUSED=1 doubles p, q, psi_p)
+  int nf = nfields(kind, false), np = kind == SEIS_ISO ? 1 : (kind == SEIS_ACOUSTIC ? 2 : 3);  // m | kdt,rho | l2m,w,rho
   double b = (nf + np) * padded;
   if (kind != SEIS_ISO && g->nb > 0) {
     const double W = g->nb + 1;
     const double per = (2 * W * g->ny * (double)nzl + 2 * W * g->nx * (double)nzl + 2 * W * g->nx * (double)g->ny) * 4.0;
-    b += per * (kind == SEIS_ACOUSTIC ? 3 : 6);
+    b += per * (kind == SEIS_ACOUSTIC ? 2 : 6);
   }
   if (shot && shot->snap_period >= 1 && shot->nt >= 1) {
     const long long nsnap = (shot->nt - 1) / shot->snap_period;
