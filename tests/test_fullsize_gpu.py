@@ -103,3 +103,61 @@ def test_c5_decomposition_path_256():
     st = oracle.ac_state(og)
     oracle.ac_run(og, wl.model["vp"], wl.model["rho"], st, 0, K, [wl.src], wl.wavelet[:, None])
     assert rel_l2(outs[0][1], st["p"]) <= TOL_FIELD
+
+
+def _linear(a, b, s=2.0):
+    """b == s * a up to fp32 rounding of values near the denormal range."""
+    a = np.asarray(a, np.float64)
+    b = np.asarray(b, np.float64)
+    assert np.all(np.isfinite(b)) and np.linalg.norm(a) > 0
+    return np.linalg.norm(b - s * a) / np.linalg.norm(s * a)
+
+
+@pytest.mark.parametrize("cfg", ["C2", "C3"])
+def test_full_length_shot_properties(cfg):
+    """The WHOLE benchmark shot (C2: acoustic 512^3, 2000 steps; C3: elastic 384^3 free
+    surface, 1500 steps) in the bench's launch configuration, checked by properties that hold
+    at any size: bitwise deterministic across runs (no races between tiles / z-chunks /
+    streams), finite, and linear in the source (2 w -> 2 seis; exact in fp32 except for
+    values in the denormal range)."""
+    import torch
+
+    if cfg == "C2":
+        wl = inputs.c2()
+        m = seis.Model(_sgrid(wl), "acoustic", wl.model["vp"], rho=wl.model["rho"])
+    else:
+        wl = inputs.c3()
+        m = seis.Model(_sgrid(wl, free_surface=1), "elastic", wl.model["vp"], vs=wl.model["vs"],
+                       rho=wl.model["rho"])
+    shot = seis.Shot(wl.src, wl.wavelet, wl.rec, rec_component=2)
+    a = m.forward_model(shot).cpu().numpy()
+    b = m.forward_model(shot).cpu().numpy()
+    shot2 = seis.Shot(wl.src, (2.0 * wl.wavelet).astype(np.float32), wl.rec, rec_component=2)
+    c = m.forward_model(shot2).cpu().numpy()
+    m.close()
+    torch.cuda.synchronize()
+    assert np.all(np.isfinite(a)) and np.abs(a).max() > 0
+    assert np.array_equal(a, b)
+    assert _linear(a, c) <= 1e-6
+
+
+def test_c4_full_length_rtm_properties():
+    """C4's WHOLE migration (512^3 salt model, 2000 steps, 99 snapshots in HBM, 13 924
+    receivers): deterministic, finite and linear in the data (2 d -> 2 I); the checkpointed
+    variant (segments of 33 snapshots) gives the same image bit for bit."""
+    import torch
+
+    wl = inputs.c4()
+    m = seis.Model(_sgrid(wl), "acoustic", wl.model["vp"], rho=wl.model["rho"])
+    shot = seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap)
+    data = m.forward_model(shot)
+    imgs = []
+    for scale, ck in ((1.0, 0), (1.0, 0), (2.0, 0), (1.0, 33)):
+        img = torch.zeros((wl.nz, wl.ny, wl.nx), device="cuda")
+        m.migrate(seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap, ckpt_period=ck), data * scale, img)
+        imgs.append(img.cpu().numpy())
+    m.close()
+    assert np.all(np.isfinite(imgs[0])) and np.abs(imgs[0]).max() > 0
+    assert np.array_equal(imgs[0], imgs[1])
+    assert _linear(imgs[0], imgs[2]) <= 1e-6
+    assert np.array_equal(imgs[0], imgs[3])
