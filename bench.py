@@ -156,6 +156,8 @@ def run_product(args):
     grid = seis.Grid(wl.nx, wl.ny, nz, wl.h, wl.dt, nb=wl.nb, pml_R=wl.pml_R, pml_f=wl.fp)
     model = seis.Model(grid, "acoustic", wl.model["vp"][z0:z0 + nzl], rho=wl.model["rho"][z0:z0 + nzl],
                        comm=comm, device=local)
+    if ws > 1 and args.halo == "peer":
+        model.enable_peer_halo()  # f4: rank faces by direct NVLink ghost stores (CUDA IPC)
     shot = seis.Shot(wl.src, wl.wavelet, wl.rec)
     seis_dev = torch.empty((nt, shot.nrec), dtype=torch.float32, device=dev)
     stream = torch.cuda.current_stream()
@@ -242,6 +244,7 @@ def run_product(args):
                                   f"{shot.nrec}-receiver line, 1 shot per step",
                       "grid": [wl.nx, wl.ny, nz], "nt": nt, "dt": wl.dt, "h": wl.h,
                       "parallelism": f"z-slab x{ws}" if ws > 1 else "single GPU",
+                      "halo": (args.halo if ws > 1 else None),
                       "l2": "inputs larger than L2 (each 512^3 field is 512 MiB > 126 MB)"},
            "e2e": e2e, "gpu_launches": launches, "roofline": roof}
     if rank == 0:
@@ -423,6 +426,9 @@ def main():
     ap.add_argument("--nt", type=int, default=2000, help="time steps per shot (2000 = C2)")
     ap.add_argument("--ref-steps", type=int, default=1, help="oracle time steps per reference step")
     ap.add_argument("--no-extras", action="store_true")
+    ap.add_argument("--halo", default="nccl", choices=["nccl", "peer"],
+                    help="N>1 rank-face ghost exchange: NCCL send/recv overlapped with the interior "
+                         "(default) or direct peer stores from the kernels (f4)")
     args = ap.parse_args()
     if args.warmup < 3:
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)

@@ -138,6 +138,39 @@ seis_status seis_slab_bounds(int32_t nz, int32_t nranks, int32_t rank, int32_t* 
 seis_status seis_model_slab(const seis_model* model, int32_t* z0, int32_t* nz_local);
 seis_status seis_model_destroy(seis_model* model);
 
+/* ---- direct ghost-plane stores between ranks ----
+ * The "sub-domains" of P:175 exchange their 4 boundary z-planes every half step.  By
+ * default the ranks do that with NCCL send/recv overlapped with the interior updates.  In
+ * peer mode the kernel that produces an exchanged field stores its first / last 4 planes
+ * straight into the neighbouring rank's ghost planes (NVLink peer stores through CUDA IPC
+ * mappings); the ranks order those stores with 32-bit flag words written and waited on by
+ * stream memory operations.  No NCCL call is left in the time step.
+ *
+ * Peer-only communicator: no NCCL at all (e.g. two ranks sharing one GPU, which NCCL
+ * rejects).  vmax = the maximum vp over the WHOLE grid, reduced by the caller (the absorbing
+ * profiles and the Courant check need the global value; an NCCL communicator reduces it
+ * itself).  With a peer-only communicator seis_forward_model does NOT all-reduce the
+ * seismogram: each rank's `seis` holds the columns of the receivers its slab owns and zeros
+ * elsewhere, and the caller sums them (exact: one owner per column).  EINVAL on bad args. */
+seis_status seis_comm_create_peer(int32_t nranks, int32_t rank, int32_t device, double vmax,
+                                  seis_comm** out);
+/* Step 1 of peer mode, on every rank after seis_model_create (model with a communicator,
+ * nranks >= 2, grid.slabs == 1): writes this rank's blob -- CUDA IPC handles of its state
+ * fields, coefficient arrays and flag words -- to `blob` (host, capacity `cap` bytes) and its
+ * size to *len.  blob = NULL: size query only.  EINVAL: not a multi-rank model, cap too small;
+ * EUNSUPPORTED: SEIS_AC_FUSED=1 (the fused step exchanges 8 planes of p). */
+seis_status seis_model_peer_export(seis_model* model, uint8_t* blob, uint64_t cap, uint64_t* len);
+/* Step 2, after every rank has exported and the blobs were exchanged by the caller (any
+ * transport, e.g. torch.distributed all_gather_object): maps the blobs of rank-1 (lo_blob,
+ * the slab above; NULL on rank 0) and rank+1 (hi_blob, the slab below; NULL on the last
+ * rank), fills the coefficient ghost planes from them and switches the model to peer mode
+ * for the rest of its life.  Blobs are only read during the call.  EINVAL: a needed blob is
+ * missing / short / from another decomposition, or export did not run; ECUDA: mapping failed.
+ * Subsequent forward_model / migrate calls are collective over the neighbouring ranks (every
+ * whole-state reset is fenced by a flag barrier). */
+seis_status seis_model_peer_import(seis_model* model, const uint8_t* lo_blob, uint64_t lo_len,
+                                   const uint8_t* hi_blob, uint64_t hi_len);
+
 /* ---- the hot path ---- */
 /* Seismic modeling of one shot from a zero state (Alg 1 forward phase).
  *   seis  host or device [nt][nrec] fp32, written in full: seis[n][r] = field^{n+1}(x_r) (O13).

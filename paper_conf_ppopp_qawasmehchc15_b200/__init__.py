@@ -32,6 +32,7 @@ STATUS = {0: "SEIS_OK", 1: "SEIS_EINVAL", 2: "SEIS_ECFL", 3: "SEIS_ENOMEM", 4: "
 
 # every symbol include/seis.h declares
 SYMBOLS = ["seis_comm_unique_id", "seis_comm_create", "seis_comm_destroy", "seis_image_reduce",
+           "seis_comm_create_peer", "seis_model_peer_export", "seis_model_peer_import",
            "seis_model_create",
            "seis_slab_bounds", "seis_model_slab", "seis_model_destroy", "seis_forward_model",
            "seis_migrate", "seis_get_field", "seis_memory_required", "seis_profile",
@@ -76,6 +77,9 @@ def lib():
                                        C.POINTER(vp)]
         L.seis_comm_destroy.argtypes = [vp]
         L.seis_image_reduce.argtypes = [vp, vp, C.c_uint64, vp]
+        L.seis_comm_create_peer.argtypes = [C.c_int32, C.c_int32, C.c_int32, C.c_double, C.POINTER(vp)]
+        L.seis_model_peer_export.argtypes = [vp, vp, C.c_uint64, C.POINTER(C.c_uint64)]
+        L.seis_model_peer_import.argtypes = [vp, vp, C.c_uint64, vp, C.c_uint64]
         L.seis_model_create.argtypes = [C.POINTER(_CGrid), C.c_int, vp, vp, vp, vp, C.c_int32,
                                         C.POINTER(vp)]
         L.seis_slab_bounds.argtypes = [C.c_int32, C.c_int32, C.c_int32, C.POINTER(C.c_int32),
@@ -184,11 +188,23 @@ def slab_bounds(nz: int, nranks: int, rank: int):
 class Comm:
     """NCCL communicator for the z-slab decomposition (one process per GPU)."""
 
+    peer_only = False
+
     def __init__(self, nranks: int, rank: int, uid: bytes, device: int):
         buf = (C.c_uint8 * 128).from_buffer_copy(uid)
         h = C.c_void_p()
         _check(lib().seis_comm_create(nranks, rank, buf, device, C.byref(h)))
         self.h, self.nranks, self.rank, self.device = h, nranks, rank, device
+
+    @classmethod
+    def peer(cls, nranks: int, rank: int, device: int, vmax: float):
+        """Peer-only communicator (no NCCL; seis_comm_create_peer): the halo planes travel by
+        direct peer stores once every rank's model ran enable_peer_halo().  vmax = global max vp."""
+        self = cls.__new__(cls)
+        h = C.c_void_p()
+        _check(lib().seis_comm_create_peer(nranks, rank, device, float(vmax), C.byref(h)))
+        self.h, self.nranks, self.rank, self.device, self.peer_only = h, nranks, rank, device, True
+        return self
 
     @staticmethod
     def unique_id() -> bytes:
@@ -260,7 +276,40 @@ class Model:
                                device=f"cuda:{self.device}")
         cs, keep = shot.c()
         _check(lib().seis_forward_model(self.h, C.byref(cs), _ptr(seis), _stream(stream)))
+        if self.comm is not None and self.comm.peer_only and getattr(self, "_group", None) is not None:
+            # the library leaves each rank its own receivers' columns (no NCCL): sum them here
+            import torch
+            import torch.distributed as dist
+
+            t = torch.as_tensor(seis)
+            if dist.get_backend(self._group) == "gloo" and t.is_cuda:
+                c = t.cpu()
+                dist.all_reduce(c, group=self._group)
+                t.copy_(c)
+            else:
+                dist.all_reduce(t, group=self._group)
         return seis
+
+    def enable_peer_halo(self, group=None):
+        """Switch the rank faces to direct ghost-plane stores over peer memory (f4): export
+        this rank's CUDA IPC blob, all-gather the blobs over the torch.distributed group,
+        map the neighbours'.  Collective over the group (one rank per z-slab, rank order)."""
+        import torch.distributed as dist
+
+        n = C.c_uint64()
+        _check(lib().seis_model_peer_export(self.h, None, 0, C.byref(n)))
+        buf = (C.c_uint8 * n.value)()
+        _check(lib().seis_model_peer_export(self.h, buf, n.value, C.byref(n)))
+        blobs = [None] * dist.get_world_size(group)
+        dist.all_gather_object(blobs, bytes(buf), group=group)
+        r = dist.get_rank(group)
+        lo = blobs[r - 1] if r > 0 else None
+        hi = blobs[r + 1] if r + 1 < len(blobs) else None
+        lob = (C.c_uint8 * len(lo)).from_buffer_copy(lo) if lo else None
+        hib = (C.c_uint8 * len(hi)).from_buffer_copy(hi) if hi else None
+        _check(lib().seis_model_peer_import(self.h, lob, len(lo) if lo else 0, hib, len(hi) if hi else 0))
+        self._group = group if group is not None else dist.group.WORLD
+        return self
 
     def migrate(self, shot: Shot, data, image, stream=None):
         """RTM of one shot; image [nz_local][ny][nx] is accumulated (+=)."""

@@ -260,6 +260,42 @@ __device__ __forceinline__ void st2_masked(float* p, const F2& a, int x0, int nx
 }
 }  // namespace seis
 
+// ------------------------------------------------------ direct ghost-plane stores
+// SURVEY §8f f4 / DESIGN.md §7: the kernel that produces an exchanged field also writes its
+// first / last 4 planes straight into the neighbouring slab's ghost planes (P:175 sub-domain
+// ghosts) -- another slab of this process, or another rank's slab mapped over NVLink by CUDA
+// IPC -- so no separate exchange (copy, NCCL send/recv) follows the kernel.
+//   lo: the slab ABOVE (smaller z); lo + (o + loo) is its bottom ghost plane nzl_lo + k for my
+//       plane k < 4 (loo = nzl_lo * PS);
+//   hi: the slab BELOW; hi + (o + hio) is its top ghost plane k - nzl for my plane k >= nzl - 4
+//       (hio = -nzl * PS).
+// nullptr = no neighbour on that side (or the ghosts travel by copies).  The padded pitches
+// PX, PY are the same in every slab, so one offset per side maps a whole plane.
+namespace seis {
+struct Ghost {
+  float* lo = nullptr;
+  long long loo = 0;
+  float* hi = nullptr;
+  long long hio = 0;
+};
+__device__ __forceinline__ void ghost_st4(const Ghost& g, long long o, int k, int nzl, const F4& v, int x0,
+                                          int nx) {
+  if (g.lo && k < 4) st4_masked(g.lo + (o + g.loo), v, x0, nx, true);
+  if (g.hi && k >= nzl - 4) st4_masked(g.hi + (o + g.hio), v, x0, nx, true);
+}
+__device__ __forceinline__ void ghost_st2(const Ghost& g, long long o, int k, int nzl, const F2& v, int x0,
+                                          int nx) {
+  if (g.lo && k < 4) st2_masked(g.lo + (o + g.loo), v, x0, nx);
+  if (g.hi && k >= nzl - 4) st2_masked(g.hi + (o + g.hio), v, x0, nx);
+}
+// the same for one value at padded offset o (receiver injection): the ghost copy receives the
+// value the owner stored, so both sides hold bitwise the same number
+__device__ __forceinline__ void ghost_st1(const Ghost& g, long long o, int k, int nzl, float v) {
+  if (g.lo && k < 4) g.lo[o + g.loo] = v;
+  if (g.hi && k >= nzl - 4) g.hi[o + g.hio] = v;
+}
+}  // namespace seis
+
 // ------------------------------------------------ C-PML memory-variable access
 // psi values are first-touch global data inside the layers; the kernels load the old
 // values BEFORE waiting for the plane's TMA stage (so their latency overlaps the wait

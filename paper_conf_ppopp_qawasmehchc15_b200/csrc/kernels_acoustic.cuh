@@ -58,6 +58,7 @@ struct AcVArgs {
   int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   const float* __restrict__ imgS; // imaging: img += S * p (input level), or nullptr
   float* __restrict__ img;
+  Ghost gh;                       // direct ghost stores of q_z (f4)
 };
 
 template <int BY>
@@ -220,6 +221,7 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
       st4_masked(a.qx + o, ox, x0, d.nx, true);
       st4_masked(a.qy + o, oy, x0, d.nx, true);
       st4_masked(a.qz + o, oz, x0, d.nx, true);
+      ghost_st4(a.gh, o, k, d.nzl, oz, x0, d.nx);
       if (IMG) {
         const long long cix = ((long long)k * d.ny + j) * d.nx + x0;
         F4 im;
@@ -258,6 +260,7 @@ struct AcPArgs {
   long long src_o;                // padded index of the source in this slab, -1 = none
   float src_amp;                  // dt K_s / h^3 * s[n]
   float* __restrict__ snap;       // compact snapshot target, or nullptr
+  Ghost gh;                       // direct ghost stores of p (f4)
 };
 
 template <int BY>
@@ -405,6 +408,7 @@ __global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ 
           if (rel == e) out.v[e] += a.src_amp;
       }
       st4_masked(a.p + o, out, x0, d.nx, true);
+      ghost_st4(a.gh, o, k, d.nzl, out, x0, d.nx);
       if (SNAP) st4_masked(a.snap + ((long long)k * d.ny + j) * d.nx + x0, out, x0, d.nx, (d.nx & 3) == 0);
     }
     stage_release(&cnt[s], tid, it + AC_NS < np, [&] {

@@ -35,12 +35,15 @@ __global__ void gather_kernel(float* __restrict__ seis_row, const float* __restr
 __global__ void inject_kernel(float* __restrict__ f, const long long* __restrict__ off,
                               const float* __restrict__ scale, const int* __restrict__ gstart,
                               const int* __restrict__ members, const float* __restrict__ data_row,
-                              int ngroups) {
+                              int ngroups, Ghost gh, long long PS, int nzl) {
   const int u = blockIdx.x * blockDim.x + threadIdx.x;
   if (u >= ngroups) return;
   float s = 0.0f;
   for (int t = gstart[u]; t < gstart[u + 1]; ++t) s += data_row[members[t]];
-  f[off[u]] = fmaf(scale[u], s, f[off[u]]);
+  const long long o = off[u];
+  const float v = fmaf(scale[u], s, f[o]);
+  f[o] = v;
+  ghost_st1(gh, o, (int)(o / PS) - GZ, nzl, v);  // (f4) the neighbour's ghost copy of the node
 }
 
 // Elastic RTM receiver injection (f3): receivers act like the explosive source (O11),
@@ -50,7 +53,7 @@ __global__ void inject_el_kernel(float* __restrict__ sxx, float* __restrict__ sy
                                  const long long* __restrict__ off, const float* __restrict__ scale,
                                  const int* __restrict__ gstart, const int* __restrict__ members,
                                  const float* __restrict__ data_row, const int* __restrict__ surf,
-                                 int ngroups) {
+                                 int ngroups, Ghost gh, long long PS, int nzl) {
   const int u = blockIdx.x * blockDim.x + threadIdx.x;
   if (u >= ngroups) return;
   float s = 0.0f;
@@ -59,7 +62,11 @@ __global__ void inject_el_kernel(float* __restrict__ sxx, float* __restrict__ sy
   const float v = scale[u] * s;
   sxx[o] -= v;
   syy[o] -= v;
-  if (!surf[u]) szz[o] -= v;
+  if (!surf[u]) {
+    const float z = szz[o] - v;
+    szz[o] = z;
+    ghost_st1(gh, o, (int)(o / PS) - GZ, nzl, z);  // (f4) only szz of the three is exchanged
+  }
 }
 
 // Copy the interior of a padded slab field to a compact [nzl][ny][nx] array.

@@ -93,6 +93,7 @@ struct ElVArgs {
   int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   const float* __restrict__ imgS;  // elastic RTM (f3): img += S * P on the input level, P = -(sxx+syy+szz)/3
   float* __restrict__ img;
+  Ghost gh[3];                     // direct ghost stores of vx, vy, vz (f4)
 };
 
 template <int BY>
@@ -279,7 +280,10 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
         ov[2].v[e] = fmaf(bz, (d6[e] + d7[e]) + d8[e], v2.v[e]);
       }
 #pragma unroll
-      for (int c = 0; c < 3; ++c) st2_masked(a.f[EVX + c] + o, ov[c], x0, d.nx);
+      for (int c = 0; c < 3; ++c) {
+        st2_masked(a.f[EVX + c] + o, ov[c], x0, d.nx);
+        ghost_st2(a.gh[c], o, k, d.nzl, ov[c], x0, d.nx);
+      }
       if (IMG) {
         const long long cix = ((long long)k * d.ny + j) * d.nx + x0;
 #pragma unroll
@@ -319,6 +323,7 @@ struct ElSArgs {
   long long src_o;
   float src_amp;   // dt (lam + 2/3 mu)_s / h^3 * s[n]
   float* __restrict__ snap;  // elastic RTM (f3): snapshot of P = -(sxx+syy+szz)/3, or nullptr
+  Ghost gh[3];               // direct ghost stores of szz, sxz, syz (f4)
 };
 
 template <int BY>
@@ -533,6 +538,9 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
       }
 #pragma unroll
       for (int c = 0; c < 6; ++c) st2_masked(a.f[ESXX + c] + o, o6[c], x0, d.nx);
+      ghost_st2(a.gh[0], o, k, d.nzl, o6[2], x0, d.nx);
+      ghost_st2(a.gh[1], o, k, d.nzl, o6[4], x0, d.nx);
+      ghost_st2(a.gh[2], o, k, d.nzl, o6[5], x0, d.nx);
       if (SNAP) {
         const long long cix = ((long long)k * d.ny + j) * d.nx + x0;
 #pragma unroll

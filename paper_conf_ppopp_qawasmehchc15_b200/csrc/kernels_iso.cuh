@@ -38,6 +38,7 @@ struct IsoArgs {
   float* __restrict__ snap;      // compact [nzl][ny][nx] or nullptr
   const float* __restrict__ imgS;// compact snapshot S_j for imaging, or nullptr
   float* __restrict__ img;       // compact image (+=), or nullptr
+  Ghost gh;                      // direct ghost stores of u^{n+1} (f4)
 };
 
 #ifndef SEIS_ISO_NS
@@ -173,6 +174,7 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
           if (rel == e) out.v[e] += a.src_amp;
       }
       st4_masked(a.up + o, out, x0, d.nx, true);
+      ghost_st4(a.gh, o, k, d.nzl, out, x0, d.nx);
       if (SNAP || IMG) {
         const long long cix = ((long long)k * d.ny + j) * d.nx + x0;
         const bool al = (d.nx & 3) == 0;

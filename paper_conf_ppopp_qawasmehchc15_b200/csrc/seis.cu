@@ -102,8 +102,9 @@ struct Scope {
 
 // ------------------------------------------------------------------ types
 struct seis_comm {
-  ncclComm_t nccl = nullptr;
+  ncclComm_t nccl = nullptr;  // nullptr: peer-only communicator (seis_comm_create_peer)
   int nranks = 1, rank = 0, device = 0;
+  double vmax = 0.0;          // peer-only: the caller's global max vp (NCCL reduces it itself)
 };
 
 namespace {
@@ -167,6 +168,7 @@ struct Slab {
     int* surf = nullptr;     // ELASTIC: group node on the free surface
   } grp[2];
   float* snap = nullptr;     // nsnap * nzl*ny*nx (points into the model's pool)
+  Ghost gh[9];               // direct ghost-plane stores per field index (f4)
 };
 
 template <class T>
@@ -212,6 +214,17 @@ struct seis_model {
   bool no_overlap = false;  // SEIS_NO_OVERLAP=1: serial exchange (A/B measurements)
   bool ac_fused = false;    // ACOUSTIC: single-sweep fused V+P step (double-buffered state)
   long long g_launches = 0;
+  // f4 direct ghost stores: `direct` = the faces between the slabs of this
+  // process are written by the producing kernels (no copies); `peer` = the rank faces too,
+  // through CUDA IPC mappings of the neighbours' fields, ordered by flag words written and
+  // waited on with stream memory operations (no NCCL in the step)
+  bool direct = false;
+  bool peer = false;
+  uint32_t* flags = nullptr;      // [0] written by the rank above, [1] by the rank below
+  uint32_t* rflag_lo = nullptr;   // the rank above's flags[1] (mapped)
+  uint32_t* rflag_hi = nullptr;   // the rank below's flags[0] (mapped)
+  uint32_t sig = 0;               // signals issued so far (same sequence on every rank)
+  std::vector<void*> ipc_open;    // mapped neighbour allocations
 };
 
 namespace {
@@ -393,10 +406,16 @@ int psi_axis(seis_kind k, int t) {
 // each array `arr(slab)` (a field, or a coefficient array at create time).
 using ArrFn = std::function<float*(Slab&)>;
 
-seis_status exchange_arrays(seis_model* M, const std::vector<ArrFn>& arrs, int np, cudaStream_t st) {
-  if (M->slabs.size() < 2 && !(M->comm && M->nranks > 1)) return SEIS_OK;
+// `state`: the arrays are propagating fields, whose ghost planes the producing kernels store
+// directly when M->direct (in-process faces) / M->peer (rank faces) is set (f4); coefficient
+// arrays (create time) always travel by copy / NCCL.
+seis_status exchange_arrays(seis_model* M, const std::vector<ArrFn>& arrs, int np, cudaStream_t st,
+                            bool state = false) {
+  const bool local = M->slabs.size() > 1 && !(state && M->direct);
+  const bool ranks = M->comm && M->comm->nccl && M->nranks > 1 && !(state && M->peer);
+  if (!local && !ranks) return SEIS_OK;
   PROF(7, st);
-  for (size_t s = 0; s + 1 < M->slabs.size(); ++s) {
+  for (size_t s = 0; local && s + 1 < M->slabs.size(); ++s) {
     Slab& A = M->slabs[s];
     Slab& B = M->slabs[s + 1];
     const size_t n = (size_t)np * A.d.PS;
@@ -411,7 +430,7 @@ seis_status exchange_arrays(seis_model* M, const std::vector<ArrFn>& arrs, int n
                          n * sizeof(float), cudaMemcpyDeviceToDevice, st));
     }
   }
-  if (M->comm && M->nranks > 1) {
+  if (ranks) {
     Slab& top = M->slabs.front();
     Slab& bot = M->slabs.back();
     const size_t n = (size_t)np * top.d.PS;
@@ -439,7 +458,56 @@ seis_status exchange_arrays(seis_model* M, const std::vector<ArrFn>& arrs, int n
 seis_status exchange(seis_model* M, const std::vector<int>& fields, cudaStream_t st, int np = 4) {
   std::vector<ArrFn> arrs;
   for (int f : fields) arrs.push_back([f](Slab& S) { return S.fld[f]; });
-  return exchange_arrays(M, arrs, np, st);
+  return exchange_arrays(M, arrs, np, st, true);
+}
+
+// ---------------------------------------------- f4: rank faces through peer memory
+// Stream memory operations (driver entry points, no libcuda link): a signal is a 32-bit
+// counter written into the neighbour's flag word after the producing work of a phase; a wait
+// blocks the stream until the local flag word reaches the counter (wrap-safe >=).  Every rank
+// issues the same sequence of signals, so the counters agree without any exchange.
+PFN_cuStreamWriteValue32_v11070 g_wr32 = nullptr;
+PFN_cuStreamWaitValue32_v11070 g_wt32 = nullptr;
+
+seis_status memops_init() {
+  if (g_wr32 && g_wt32) return SEIS_OK;
+  cudaDriverEntryPointQueryResult q;
+  void* fn = nullptr;
+  CK(cudaGetDriverEntryPoint("cuStreamWriteValue32", &fn, cudaEnableDefault, &q));
+  if (q != cudaDriverEntryPointSuccess || !fn) return fail(SEIS_EUNSUPPORTED, "cuStreamWriteValue32 unavailable");
+  g_wr32 = (PFN_cuStreamWriteValue32_v11070)fn;
+  CK(cudaGetDriverEntryPoint("cuStreamWaitValue32", &fn, cudaEnableDefault, &q));
+  if (q != cudaDriverEntryPointSuccess || !fn) return fail(SEIS_EUNSUPPORTED, "cuStreamWaitValue32 unavailable");
+  g_wt32 = (PFN_cuStreamWaitValue32_v11070)fn;
+  return SEIS_OK;
+}
+
+// Tell both neighbours that this rank's work issued on `st` so far (kernels that stored into
+// their ghost planes included) is complete: the write is fenced behind the preceding work.
+seis_status peer_signal(seis_model* M, cudaStream_t st) {
+  if (!M->peer) return SEIS_OK;
+  ++M->sig;
+  if (M->rflag_lo && g_wr32((CUstream)st, (CUdeviceptr)M->rflag_lo, M->sig, CU_STREAM_WRITE_VALUE_DEFAULT))
+    return fail(SEIS_ECUDA, "cuStreamWriteValue32 (rank above) failed");
+  if (M->rflag_hi && g_wr32((CUstream)st, (CUdeviceptr)M->rflag_hi, M->sig, CU_STREAM_WRITE_VALUE_DEFAULT))
+    return fail(SEIS_ECUDA, "cuStreamWriteValue32 (rank below) failed");
+  return SEIS_OK;
+}
+// Block `st` until both neighbours have issued signal number M->sig.
+seis_status peer_wait(seis_model* M, cudaStream_t st) {
+  if (!M->peer) return SEIS_OK;
+  if (M->rflag_lo && g_wt32((CUstream)st, (CUdeviceptr)(M->flags + 0), M->sig, CU_STREAM_WAIT_VALUE_GEQ))
+    return fail(SEIS_ECUDA, "cuStreamWaitValue32 (rank above) failed");
+  if (M->rflag_hi && g_wt32((CUstream)st, (CUdeviceptr)(M->flags + 1), M->sig, CU_STREAM_WAIT_VALUE_GEQ))
+    return fail(SEIS_ECUDA, "cuStreamWaitValue32 (rank below) failed");
+  return SEIS_OK;
+}
+// Both neighbours have reached the same point of the program: used around every whole-state
+// reset / copy (zero, checkpoint save / restore), which must not interleave with the
+// neighbours' stores into this rank's ghost planes.
+seis_status peer_barrier(seis_model* M, cudaStream_t st) {
+  TRY(peer_signal(M, st));
+  return peer_wait(M, st);
 }
 
 }  // namespace
@@ -530,6 +598,20 @@ seis_status seis_comm_destroy(seis_comm* c) {
   return SEIS_OK;
 }
 
+seis_status seis_comm_create_peer(int32_t nranks, int32_t rank, int32_t device, double vmax,
+                                  seis_comm** out) {
+  if (!out || nranks < 1 || rank < 0 || rank >= nranks || !(vmax > 0.0))
+    return fail(SEIS_EINVAL, "seis_comm_create_peer: bad arguments");
+  CK(cudaSetDevice(device));
+  seis_comm* c = new seis_comm();
+  c->nranks = nranks;
+  c->rank = rank;
+  c->device = device;
+  c->vmax = vmax;
+  *out = c;
+  return SEIS_OK;
+}
+
 static seis_status validate_grid(const seis_grid* g, seis_kind kind) {
   if (!g) return fail(SEIS_EINVAL, "null grid");
   if (g->nx < 1 || g->ny < 1 || g->nz < 1) return fail(SEIS_EINVAL, "grid dims must be >= 1");
@@ -554,6 +636,7 @@ seis_status seis_model_destroy(seis_model* M) {
   if (M->xs) cudaStreamDestroy(M->xs);
   if (M->ev_fork) cudaEventDestroy(M->ev_fork);
   if (M->ev_join) cudaEventDestroy(M->ev_join);
+  for (void* p : M->ipc_open) cudaIpcCloseMemHandle(p);
   for (void* p : M->allocs) cudaFree(p);
   delete M;
   return SEIS_OK;
@@ -579,7 +662,10 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       return fail(SEIS_EINVAL, "vs must satisfy 0 <= vs <= vp/sqrt(2) (index %zu)", t);
   }
   // (rho / w at k+1 across rank faces come from the ghost-plane exchange after the upload)
-  if (M->comm && M->nranks > 1) {
+  if (M->comm && M->nranks > 1 && !M->comm->nccl) {
+    if (!(M->comm->vmax >= vmax)) return fail(SEIS_EINVAL, "peer communicator vmax %.3f < local max vp %.3f", M->comm->vmax, vmax);
+    vmax = M->comm->vmax;
+  } else if (M->comm && M->nranks > 1) {
     float* dv = nullptr;
     CK(cudaMalloc(&dv, sizeof(double)));
     CK(cudaMemcpy(dv, &vmax, sizeof(double), cudaMemcpyHostToDevice));
@@ -801,6 +887,26 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     else if (kind == SEIS_ISO) choose_chunks(S, occ, dev_sms, TXV, BYI, 24);
     else choose_chunks(S, occ, dev_sms, TXV, M->ac_fused ? BYF : BYV, M->ac_fused ? 64 : 16);
   }
+  // f4: the faces between the slabs of this process by direct ghost stores of the producing
+  // kernels (SEIS_GHOST_COPY=1 keeps the copy exchange, the A/B alternative).  Not for the
+  // fused acoustic step, which exchanges 8 ghost planes of p.
+  {
+    const char* e = getenv("SEIS_GHOST_COPY");
+    M->direct = ns > 1 && !M->ac_fused && !(e && e[0] == '1');
+    for (int s = 0; M->direct && s < ns; ++s) {
+      Slab& S = M->slabs[s];
+      for (size_t f = 0; f < S.fld.size() && f < 9; ++f) {
+        if (s > 0) {
+          S.gh[f].lo = M->slabs[s - 1].fld[f];
+          S.gh[f].loo = (long long)M->slabs[s - 1].d.nzl * S.d.PS;
+        }
+        if (s + 1 < ns) {
+          S.gh[f].hi = M->slabs[s + 1].fld[f];
+          S.gh[f].hio = -(long long)S.d.nzl * S.d.PS;
+        }
+      }
+    }
+  }
   if (ns > 1 || M->nranks > 1) {
     const char* e = getenv("SEIS_NO_OVERLAP");
     M->no_overlap = e && e[0] == '1';
@@ -856,6 +962,137 @@ seis_status seis_model_create(const seis_grid* grid, seis_kind kind, const float
     return s;
   }
   *out = M;
+  return SEIS_OK;
+}
+
+}  // extern "C"
+
+namespace {
+// What a rank publishes for its neighbours' direct ghost stores (f4): CUDA IPC handles of the
+// allocation bases of its state fields (field = base + 112 bytes, alloc_padded), of the
+// coefficient arrays whose ghost planes the neighbours fill once, and of its flag words.
+struct PeerBlob {
+  uint32_t magic;
+  int32_t kind, rank, nranks, nzl, nfld, PX, PY;
+  cudaIpcMemHandle_t fld[9];
+  cudaIpcMemHandle_t coef[2];  // rho, w (ELASTIC) -- ACOUSTIC: rho only
+  cudaIpcMemHandle_t flags;
+};
+constexpr uint32_t PEER_MAGIC = 0x50494553u;  // "SEIP"
+constexpr size_t PADB = 112;                   // alloc_padded: field = base + 112 bytes
+
+int ncoef(seis_kind k) { return k == SEIS_ISO ? 0 : (k == SEIS_ACOUSTIC ? 1 : 2); }
+float* coef_of(Slab& S, int t) { return t == 0 ? S.rho : S.wmu; }
+
+seis_status peer_open(seis_model* M, const cudaIpcMemHandle_t& h, char** p) {
+  void* q = nullptr;
+  cudaError_t e = cudaIpcOpenMemHandle(&q, h, cudaIpcMemLazyEnablePeerAccess);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(SEIS_ECUDA, "cudaIpcOpenMemHandle: %s", cudaGetErrorString(e));
+  }
+  M->ipc_open.push_back(q);
+  *p = (char*)q;
+  return SEIS_OK;
+}
+
+seis_status check_blob(const seis_model* M, const uint8_t* b, uint64_t len, int want_rank) {
+  if (!b || len < sizeof(PeerBlob)) return fail(SEIS_EINVAL, "peer blob of rank %d missing or short", want_rank);
+  PeerBlob p;
+  std::memcpy(&p, b, sizeof p);
+  const Slab& S = M->slabs.front();
+  if (p.magic != PEER_MAGIC || p.kind != (int)M->kind || p.rank != want_rank || p.nranks != M->nranks ||
+      p.nfld != (int)S.fld.size() || p.PX != S.d.PX || p.PY != S.d.PY)
+    return fail(SEIS_EINVAL, "peer blob does not belong to rank %d of this decomposition", want_rank);
+  return SEIS_OK;
+}
+}  // namespace
+
+extern "C" {
+
+seis_status seis_model_peer_export(seis_model* M, uint8_t* blob, uint64_t cap, uint64_t* len) {
+  if (!M || !len) return fail(SEIS_EINVAL, "null argument");
+  *len = sizeof(PeerBlob);
+  if (!blob) return SEIS_OK;  // size query
+  if (cap < sizeof(PeerBlob)) return fail(SEIS_EINVAL, "blob capacity %llu < %zu", (unsigned long long)cap, sizeof(PeerBlob));
+  if (!M->comm || M->nranks < 2 || M->slabs.size() != 1)
+    return fail(SEIS_EINVAL, "peer halo needs a multi-rank model (one slab per rank)");
+  if (M->ac_fused) return fail(SEIS_EUNSUPPORTED, "peer halo with the fused acoustic step (SEIS_AC_FUSED=1)");
+  CK(cudaSetDevice(M->device));
+  if (!M->flags) {
+    void* f = nullptr;
+    TRY(alloc_track(M, &f, 256));
+    CK(cudaMemset(f, 0, 256));
+    M->flags = (uint32_t*)f;
+  }
+  Slab& S = M->slabs.front();
+  PeerBlob p{};
+  p.magic = PEER_MAGIC;
+  p.kind = (int)M->kind;
+  p.rank = M->rank;
+  p.nranks = M->nranks;
+  p.nzl = S.d.nzl;
+  p.nfld = (int)S.fld.size();
+  p.PX = S.d.PX;
+  p.PY = S.d.PY;
+  for (size_t f = 0; f < S.fld.size(); ++f) CK(cudaIpcGetMemHandle(&p.fld[f], (char*)S.fld[f] - PADB));
+  for (int t = 0; t < ncoef(M->kind); ++t) CK(cudaIpcGetMemHandle(&p.coef[t], (char*)coef_of(S, t) - PADB));
+  CK(cudaIpcGetMemHandle(&p.flags, M->flags));
+  std::memcpy(blob, &p, sizeof p);
+  return SEIS_OK;
+}
+
+seis_status seis_model_peer_import(seis_model* M, const uint8_t* lo_blob, uint64_t lo_len,
+                                   const uint8_t* hi_blob, uint64_t hi_len) {
+  if (!M) return fail(SEIS_EINVAL, "null model");
+  if (!M->comm || M->nranks < 2 || M->slabs.size() != 1)
+    return fail(SEIS_EINVAL, "peer halo needs a multi-rank model (one slab per rank)");
+  if (!M->flags) return fail(SEIS_EINVAL, "seis_model_peer_export must run first");
+  if (M->peer) return fail(SEIS_EINVAL, "peer halo already imported");
+  const bool has_lo = M->rank > 0, has_hi = M->rank < M->nranks - 1;
+  if (has_lo) TRY(check_blob(M, lo_blob, lo_len, M->rank - 1));
+  if (has_hi) TRY(check_blob(M, hi_blob, hi_len, M->rank + 1));
+  CK(cudaSetDevice(M->device));
+  TRY(memops_init());
+  Slab& S = M->slabs.front();
+  const size_t PS = (size_t)S.d.PS;
+  for (int side = 0; side < 2; ++side) {
+    if (side == 0 ? !has_lo : !has_hi) continue;
+    PeerBlob p;
+    std::memcpy(&p, side == 0 ? lo_blob : hi_blob, sizeof p);
+    for (size_t f = 0; f < S.fld.size(); ++f) {
+      char* q = nullptr;
+      TRY(peer_open(M, p.fld[f], &q));
+      float* rf = (float*)(q + PADB);
+      if (side == 0) {  // the rank above: my planes 0..3 -> its bottom ghosts nzl_lo + k
+        S.gh[f].lo = rf;
+        S.gh[f].loo = (long long)p.nzl * S.d.PS;
+      } else {          // the rank below: my planes nzl-4.. -> its top ghosts k - nzl
+        S.gh[f].hi = rf;
+        S.gh[f].hio = -(long long)S.d.nzl * S.d.PS;
+      }
+    }
+    // coefficient ghost planes (rho / w at k+1 across the face), once, read from the peer
+    for (int t = 0; t < ncoef(M->kind); ++t) {
+      char* q = nullptr;
+      TRY(peer_open(M, p.coef[t], &q));
+      const float* rc = (const float*)(q + PADB);
+      float* mine = coef_of(S, t);
+      if (side == 0)
+        CK(cudaMemcpy(mine + (GZ - 4) * PS, rc + (size_t)(p.nzl + GZ - 4) * PS, 4 * PS * sizeof(float),
+                      cudaMemcpyDeviceToDevice));
+      else
+        CK(cudaMemcpy(mine + (size_t)(S.d.nzl + GZ) * PS, rc + GZ * PS, 4 * PS * sizeof(float),
+                      cudaMemcpyDeviceToDevice));
+    }
+    char* q = nullptr;
+    TRY(peer_open(M, p.flags, &q));
+    if (side == 0) M->rflag_lo = (uint32_t*)q + 1;  // its "from below" word
+    else M->rflag_hi = (uint32_t*)q + 0;            // its "from above" word
+  }
+  CK(cudaDeviceSynchronize());
+  M->sig = 0;
+  M->peer = true;
   return SEIS_OK;
 }
 
@@ -1020,6 +1257,7 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
 
 // Zero the state of every slab (fields incl. ghosts, C-PML slabs).
 seis_status zero_state(seis_model* M, cudaStream_t st) {
+  TRY(peer_barrier(M, st));  // (f4) no neighbour store into these ghost planes is in flight
   for (Slab& S : M->slabs) {
     const size_t elems = (size_t)S.d.PS * (S.d.nzl + 2 * GZ);
     for (float* f : S.fld) CK(cudaMemsetAsync(f, 0, elems * sizeof(float), st));
@@ -1037,7 +1275,7 @@ seis_status zero_state(seis_model* M, cudaStream_t st) {
     }
     S.cur = 0;
   }
-  return SEIS_OK;
+  return peer_barrier(M, st);  // (f4) ... nor starts before the reset is done
 }
 
 // Every array of the propagating state (padded fields incl. ghost planes, C-PML
@@ -1069,13 +1307,14 @@ std::vector<std::pair<float*, size_t>> state_arrays(seis_model* M) {
 
 // Copy the whole state to (save = true) or from a checkpoint slot of state_elems floats.
 seis_status state_copy(seis_model* M, float* slot, bool save, cudaStream_t st) {
+  TRY(peer_barrier(M, st));  // (f4) the ghost planes are settled (see zero_state)
   size_t o = 0;
   for (auto& a : state_arrays(M)) {
     if (save) CK(cudaMemcpyAsync(slot + o, a.first, a.second * 4, cudaMemcpyDeviceToDevice, st));
     else CK(cudaMemcpyAsync(a.first, slot + o, a.second * 4, cudaMemcpyDeviceToDevice, st));
     o += (a.second + 31) / 32 * 32;
   }
-  return SEIS_OK;
+  return peer_barrier(M, st);
 }
 size_t state_elems(seis_model* M) {
   size_t o = 0;
@@ -1118,10 +1357,12 @@ seis_status inject_rows(seis_model* M, const float* row, int part, cudaStream_t 
       PROF(5, st);
       if (M->kind == SEIS_ELASTIC) {
         inject_el_kernel<<<(G2.n + 127) / 128, 128, 0, st>>>(S.fld[ESXX], S.fld[ESYY], S.fld[ESZZ], G2.off,
-                                                            G2.scale, G2.start, G2.mem, row, G2.surf, G2.n);
+                                                            G2.scale, G2.start, G2.mem, row, G2.surf, G2.n,
+                                                            S.gh[ESZZ], S.d.PS, S.d.nzl);
       } else {
-        float* f = M->kind == SEIS_ISO ? S.fld[S.cur] : S.fld[4 * S.cur];
-        inject_kernel<<<(G2.n + 127) / 128, 128, 0, st>>>(f, G2.off, G2.scale, G2.start, G2.mem, row, G2.n);
+        const int f = M->kind == SEIS_ISO ? S.cur : 4 * S.cur;
+        inject_kernel<<<(G2.n + 127) / 128, 128, 0, st>>>(S.fld[f], G2.off, G2.scale, G2.start, G2.mem, row,
+                                                         G2.n, S.gh[f], S.d.PS, S.d.nzl);
       }
       CKL();
     }
@@ -1147,20 +1388,32 @@ bool overlapped(const seis_model* M) {
 // slabs, NCCL send/recv between ranks) and the mirror; meanwhile the interior chunks run on
 // the compute stream; the compute stream then joins xs.  Per-point arithmetic is the same,
 // so results are bitwise identical to the serial order.
+//
+// f4 (M->peer): the boundary chunks read ghost planes the neighbour ranks store directly, so
+// they wait for the neighbours' signal of the previous phase; after them (and the injection
+// of their nodes) this rank signals in turn.  Interior chunks touch no ghost plane.  The
+// write-after-read order on the ghosts needs no extra signal: a neighbour stores into my
+// ghosts of field F only after waiting for my signal of the phase that READ them (every
+// boundary-chunk kernel reads the ghosts of the previous phase's field and stores those of
+// its own).
 seis_status run_phase(seis_model* M, const LaunchFn& launch, const PostFn& post, cudaStream_t st) {
   if (!overlapped(M)) {
+    TRY(peer_wait(M, st));
     for (size_t s = 0; s < M->slabs.size(); ++s) TRY(launch(s, 0, 1, M->slabs[s].nzch, st));
-    return post(2, st);
+    TRY(post(2, st));
+    return peer_signal(M, st);
   }
   cudaStream_t xs = M->xs;
   CK(cudaEventRecord(M->ev_fork, st));
   CK(cudaStreamWaitEvent(xs, M->ev_fork, 0));
+  TRY(peer_wait(M, xs));
   for (size_t s = 0; s < M->slabs.size(); ++s) {
     const int nch = M->slabs[s].nzch;
     if (nch <= 2) TRY(launch(s, 0, 1, nch, xs));
     else TRY(launch(s, 0, nch - 1, 2, xs));
   }
   TRY(post(0, xs));
+  TRY(peer_signal(M, xs));
   for (size_t s = 0; s < M->slabs.size(); ++s) {
     const int nch = M->slabs[s].nzch;
     if (nch > 2) TRY(launch(s, 1, 1, nch - 2, st));
@@ -1204,6 +1457,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.snap = snap ? (*snap)[s] : nullptr;
       a.imgS = imgS ? (*imgS)[s] : nullptr;
       a.img = img ? (*img)[s] : nullptr;
+      a.gh = S.gh[1 - cur];
       const dim3 gr = grid_of(S, TXV, BYI, nch), blk(NTX, BYI);
       {
         PROF(0, ks);
@@ -1318,6 +1572,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.chs = chs;
       a.imgS = imgS ? (*imgS)[s] : nullptr;
       a.img = img ? (*img)[s] : nullptr;
+      a.gh = S.gh[3];
       const dim3 gr = grid_of(S, TXV, BYV, nch), blk(NTX, BYV);
       {
         PROF(1, ks);
@@ -1357,6 +1612,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.src_amp = 0.f;
       if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
       a.snap = snap ? (*snap)[s] : nullptr;
+      a.gh = S.gh[0];
       const dim3 gr = grid_of(S, TXV, BYP, nch), blk(NTX, BYP);
       {
         PROF(2, ks);
@@ -1406,6 +1662,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     a.chs = chs;
     a.imgS = imgS ? (*imgS)[s] : nullptr;
     a.img = img ? (*img)[s] : nullptr;
+    for (int t = 0; t < 3; ++t) a.gh[t] = S.gh[EVX + t];
     const dim3 gr = grid_of(S, TXE, BYE, nch);
     {
       PROF(3, ks);
@@ -1445,6 +1702,9 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     a.src_amp = 0.f;
     if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
     a.snap = snap ? (*snap)[s] : nullptr;
+    a.gh[0] = S.gh[ESZZ];
+    a.gh[1] = S.gh[ESXZ];
+    a.gh[2] = S.gh[ESYZ];
     const dim3 gr = grid_of(S, TXE, BYE, nch);
     {
       PROF(4, ks);
@@ -1508,7 +1768,9 @@ static seis_status forward_loop(seis_model* M, const seis_shot* sh, float* sd, s
     TRY(step(M, n, true, nullptr, nullptr, nullptr, st));
     if (sh->nrec) TRY(gather(M, sh, sd, n, st));
   }
-  if (M->comm && M->nranks > 1 && ns) NK(ncclAllReduce(sd, sd, ns, ncclFloat, ncclSum, M->comm->nccl, st));
+  // (a peer-only communicator has no NCCL: each rank returns its own receivers' columns)
+  if (M->comm && M->comm->nccl && M->nranks > 1 && ns)
+    NK(ncclAllReduce(sd, sd, ns, ncclFloat, ncclSum, M->comm->nccl, st));
   return SEIS_OK;
 }
 

@@ -114,3 +114,17 @@ def test_memory_required_checkpointing():
     allsnap = seis.memory_required(g5, "acoustic", seis.Shot((1, 1, 1), w5, rec, snap_period=20))
     ckpt = seis.memory_required(g5, "acoustic", seis.Shot((1, 1, 1), w5, rec, snap_period=20, ckpt_period=10))
     assert allsnap > 180e9 > ckpt
+
+
+def test_peer_mode_entry_points_validate_before_touching_the_device():
+    """f4 peer halo ABI: argument errors are reported without a device; a NULL model is
+    rejected by export / import."""
+    import ctypes as C
+
+    L = seis.lib()
+    h = C.c_void_p()
+    for args in ((0, 0, 0, 3000.0), (2, 2, 0, 3000.0), (2, -1, 0, 3000.0), (2, 0, 0, 0.0), (2, 0, 0, float("nan"))):
+        assert L.seis_comm_create_peer(*args, C.byref(h)) == 1  # SEIS_EINVAL
+    n = C.c_uint64()
+    assert L.seis_model_peer_export(None, None, 0, C.byref(n)) == 1
+    assert L.seis_model_peer_import(None, None, 0, None, 0) == 1

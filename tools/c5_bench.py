@@ -141,8 +141,12 @@ def main():
     fshot = seis.Shot(wl.src, w, wl.rec)
     buf = torch.empty((K, fshot.nrec), device=dev)
     dec = {}
-    for name, P, serial in (("slabs1", 1, False), ("slabs8_overlap", 8, False), ("slabs8_serial", 8, True)):
+    for name, P, serial, copy in (("slabs1", 1, False, False), ("slabs8_overlap", 8, False, False),
+                                  ("slabs8_serial", 8, True, False), ("slabs8_overlap_copy", 8, False, True),
+                                  ("slabs8_serial_copy", 8, True, True)):
+        # direct ghost stores (f4, default) vs the copy exchange (SEIS_GHOST_COPY=1)
         os.environ["SEIS_NO_OVERLAP"] = "1" if serial else "0"
+        os.environ["SEIS_GHOST_COPY"] = "1" if copy else "0"
         gg = seis.Grid(g.nx, g.ny, g.nz, g.h, g.dt, nb=g.nb, pml_f=g.pml_f, slabs=P)
         mm = seis.Model(gg, "acoustic", sm["vp"], rho=sm["rho"], device=0)
         ms = timed(lambda: mm.forward_model(fshot, buf, stream), stream, reps=2, warm=1)
@@ -151,6 +155,7 @@ def main():
         del mm
         torch.cuda.empty_cache()
     os.environ.pop("SEIS_NO_OVERLAP", None)
+    os.environ.pop("SEIS_GHOST_COPY", None)
     res["decomposition_1gpu"] = dec
     line = json.dumps(res)
     print(line)

@@ -16,6 +16,12 @@ VARIANTS = {  # name: (defines, env)
     "split": ([], {}),
     "f16": (["SEIS_BYF=16"], {"SEIS_AC_FUSED": "1"}),
     "f32": (["SEIS_BYF=32"], {"SEIS_AC_FUSED": "1"}),
+    "f8": (["SEIS_BYF=8"], {"SEIS_AC_FUSED": "1"}),
+    "f8_z32": (["SEIS_BYF=8"], {"SEIS_AC_FUSED": "1", "SEIS_ZCHUNK_MAX": "32"}),
+    "f8_z16": (["SEIS_BYF=8"], {"SEIS_AC_FUSED": "1", "SEIS_ZCHUNK_MAX": "16"}),
+    "f8ns3": (["SEIS_BYF=8", "SEIS_AF_NS=3"], {"SEIS_AC_FUSED": "1"}),
+    "f8ns3_z32": (["SEIS_BYF=8", "SEIS_AF_NS=3"], {"SEIS_AC_FUSED": "1", "SEIS_ZCHUNK_MAX": "32"}),
+    "f16_z32": (["SEIS_BYF=16"], {"SEIS_AC_FUSED": "1", "SEIS_ZCHUNK_MAX": "32"}),
     "split_z128": ([], {"SEIS_ZCHUNK_MAX": "128"}),
     "split_z64": ([], {"SEIS_ZCHUNK_MAX": "64"}),
     "split_z32": ([], {"SEIS_ZCHUNK_MAX": "32"}),
