@@ -322,6 +322,19 @@ def run_extras(args, local):
     res["iso_512"] = {"gpts_s": round(n ** 3 * 200 / (ms * 1e-3) / 1e9, 3), "ms_per_shot": round(ms, 3),
                       "roofline": kernel_frac("iso_step", float(n) ** 3, 16.0)}
     m.close()
+    # the same with the split-field PML (O6b): layer points also read u^(d) at two levels and
+    # write the new level (36 B per layer point)
+    g = seis.Grid(n, n, n, 10.0, 1e-3, nb=20, iso_pml=1)
+    m = seis.Model(g, "iso", vp, device=local)
+    m.forward_model(shot, buf, stream)
+    seis.profile(True)
+    ms = _timed_shots(lambda: m.forward_model(shot, buf, stream), 2, stream)
+    seis.profile(False)
+    lay = 1.0 - ((n - 40) / n) ** 3
+    res["iso_512_split_pml"] = {"gpts_s": round(n ** 3 * 200 / (ms * 1e-3) / 1e9, 3), "ms_per_shot": round(ms, 3),
+                                "alg_bytes_per_point": round(16.0 + 36.0 * lay, 2),
+                                "roofline": kernel_frac("iso_step", float(n) ** 3, 16.0 + 36.0 * lay)}
+    m.close()
     del vp
     torch.cuda.empty_cache()
     # C3: elastic 384^3, 1500 steps, free surface, C-PML on 5 faces

@@ -75,8 +75,13 @@ typedef struct {
   float pml_R;          /* target reflection coefficient, 0 < R < 1 (default 1e-3) */
   float pml_f;          /* C-PML alpha reference frequency (Hz), >= 0 (default: source peak) */
   int32_t slabs;        /* z-slabs per PROCESS (>= 1).  > 1 runs the z-slab domain
-                           decomposition on one GPU with device-to-device ghost
-                           copies; results are bitwise identical for every value. */
+                           decomposition on one GPU with direct ghost-plane stores
+                           (f4); results are bitwise identical for every value. */
+  int32_t iso_pml;      /* ISO absorbing layer ("standard PML ... in our second order
+                           (isotropic) formulation"): 0 = damped wave (O6, default), 1 =
+                           split-field PML (O6b: u = u^(x) + u^(y) + u^(z) inside the layers,
+                           (d_t + eta_d)^2 u^(d) = v^2 d_d^2 u).  Must be 0 for other kinds
+                           (EUNSUPPORTED). */
 } seis_grid;
 
 /* One shot ("one shot profile"). All arrays are borrowed for the call only. */

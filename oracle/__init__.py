@@ -50,7 +50,7 @@ class _Grid(C.Structure):
     _fields_ = [("nx", C.c_int32), ("ny", C.c_int32), ("nz", C.c_int32),
                 ("h", C.c_double), ("dt", C.c_double), ("nb", C.c_int32),
                 ("free_surface", C.c_int32), ("pml_R", C.c_double), ("pml_f", C.c_double),
-                ("periodic", C.c_int32)]
+                ("periodic", C.c_int32), ("iso_pml", C.c_int32)]
 
 
 class _Inj(C.Structure):
@@ -78,7 +78,7 @@ def _L():
         _lib.or_iso_eta.argtypes = [C.c_int, C.c_int, C.c_double, C.c_double, C.c_double, d]
         _lib.or_cpml.argtypes = [C.c_int, C.c_int, C.c_int, C.c_int, C.c_double, C.c_double,
                                  C.c_double, C.c_double, C.c_double, d, d, d, d]
-        _lib.or_iso_run.argtypes = [g, f, d, d, C.c_int, C.c_int, C.POINTER(_Inj),
+        _lib.or_iso_run.argtypes = [g, f, d, d, d, C.c_int, C.c_int, C.POINTER(_Inj),
                                     C.POINTER(_Rec), d]
         _lib.or_ac_run.argtypes = [g, f, f, d, d, d, d, d, C.c_int, C.c_int, C.POINTER(_Inj),
                                    C.POINTER(_Rec), d]
@@ -104,11 +104,13 @@ class Grid:
     pml_R: float = 1e-3
     pml_f: float = 10.0
     periodic: int = 0
+    iso_pml: int = 0  # ISO layer: 0 = damped wave (O6), 1 = split-field PML (O6b)
 
     def c(self) -> _Grid:
         return _Grid(self.nx, self.ny, self.nz, float(np.float32(self.h)),
                      float(np.float32(self.dt)), self.nb, self.free_surface,
-                     float(np.float32(self.pml_R)), float(np.float32(self.pml_f)), self.periodic)
+                     float(np.float32(self.pml_R)), float(np.float32(self.pml_f)), self.periodic,
+                     self.iso_pml)
 
     @property
     def shape(self):
@@ -195,7 +197,9 @@ def _ptr(x, T):
 
 
 def iso_state(grid: Grid):
-    return {"u_prev": np.zeros(grid.shape), "u_cur": np.zeros(grid.shape)}
+    # w: split-field PML components (O6b) [level n-1, n][x, y, z], used inside the layers
+    return {"u_prev": np.zeros(grid.shape), "u_cur": np.zeros(grid.shape),
+            "w": np.zeros((2, 3) + grid.shape)}
 
 
 def ac_state(grid: Grid):
@@ -214,7 +218,10 @@ def iso_run(grid, vp, state, n0, nsteps, inj_pos=None, inj_amp=None, rec_pos=Non
     inj, rec, nrec, keep = _lists(inj_pos, inj_amp, rec_pos)
     seis = np.zeros((nsteps, max(nrec, 1)))
     g = grid.c()
-    rc = _L().or_iso_run(C.byref(g), _fp(vp), _dp(state["u_prev"]), _dp(state["u_cur"]), n0,
+    w = state.get("w")
+    if w is None:
+        w = state["w"] = np.zeros((2, 3) + grid.shape)
+    rc = _L().or_iso_run(C.byref(g), _fp(vp), _dp(state["u_prev"]), _dp(state["u_cur"]), _dp(w), n0,
                          nsteps, _ptr(inj, _Inj), _ptr(rec, _Rec), _dp(seis))
     _check(rc, "iso_run")
     return seis[:, :nrec]

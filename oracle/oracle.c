@@ -90,6 +90,18 @@ static double lap_at(const or_grid* g, const double* u, int i, int j, int k) {
   return s;
 }
 
+/* One axis of it (O6b): L_d u = c0 u_i + sum_m c_m (u_{i+m e_d} + u_{i-m e_d});
+ * Lambda = L_x + L_y + L_z. */
+static double lap_axis(const or_grid* g, const double* u, int i, int j, int k, int d) {
+  double s = C2[0] * at(g, u, i, j, k);
+  for (int m = 1; m <= 4; ++m) {
+    int e[3] = {0, 0, 0};
+    e[d] = m;
+    s += C2[m] * (at(g, u, i + e[0], j + e[1], k + e[2]) + at(g, u, i - e[0], j - e[1], k - e[2]));
+  }
+  return s;
+}
+
 void or_lap(const or_grid* g, const double* u, double* out) {
   init_coef();
 #pragma omp parallel for schedule(static)
@@ -204,8 +216,20 @@ static int check_lists(const or_grid* g, const or_inj* inj, const or_rec* rec) {
  *   m = v^2 dt^2 / h^2,  s^n = delta_{i,s} v_s^2 dt^2 w(n dt) / h^3,
  *   eta = eta_x + eta_y + eta_z.
  * With eta = 0 this is exactly Eq 1 with f^n = w(n dt) delta / h^3 (O3).
- * Step order (O2): update -> source -> gather (Alg 1).          */
-int or_iso_run(const or_grid* g, const float* vp, double* u_prev, double* u_cur, int n0,
+ * Step order (O2): update -> source -> gather (Alg 1).
+ *
+ * Split-field PML (O6b, g->iso_pml = 1; the paper's "standard PML ... in our second
+ * order (isotropic) formulation", after Berenger [4]): inside the layers
+ * (eta > 0) the field is the sum of three components, u = u^(x) + u^(y) + u^(z), each
+ * damped along its own axis only,
+ *   (d_t + eta_d)^2 u^(d) = v^2 d_d^2 u      (eta_d = eta_max xi_d^2 of O6),
+ * centred in time:
+ *   u^(d),n+1 = [(2 - (eta_d dt)^2) u^(d),n - (1 - eta_d dt) u^(d),n-1 + m L_d u^n] / (1 + eta_d dt),
+ *   u^{n+1} = sum_d u^(d),n+1.
+ * Outside the layers the update is Eq 1 as above (with eta_d = 0 the three component
+ * updates sum to it).  A point source inside the layers enters the x component:
+ * s^n / (1 + eta_x dt) is added to u^(x),n+1 and to u^{n+1}.                       */
+int or_iso_run(const or_grid* g, const float* vp, double* u_prev, double* u_cur, double* w, int n0,
                int nsteps, const or_inj* inj, const or_rec* rec, double* seis) {
   init_coef();
   int rc = check_lists(g, inj, rec);
@@ -223,6 +247,21 @@ int or_iso_run(const or_grid* g, const float* vp, double* u_prev, double* u_cur,
   double* b = (double*)malloc(sizeof(double) * n); /* u^n */
   memcpy(a, u_prev, sizeof(double) * n);
   memcpy(b, u_cur, sizeof(double) * n);
+  const int spml = g->iso_pml == 1 && g->nb > 0;
+  if (spml && !w) {
+    free(a);
+    free(b);
+    free(ex);
+    free(ey);
+    free(ez);
+    return -5;
+  }
+  double* wa[3]; /* u^(d),n-1 (overwritten by u^(d),n+1) */
+  double* wb[3]; /* u^(d),n */
+  for (int d = 0; d < 3; ++d) {
+    wa[d] = spml ? w + (size_t)d * n : NULL;
+    wb[d] = spml ? w + (size_t)(3 + d) * n : NULL;
+  }
 
   for (int s = 0; s < nsteps; ++s) {
     int t = n0 + s;
@@ -234,6 +273,17 @@ int or_iso_run(const or_grid* g, const float* vp, double* u_prev, double* u_cur,
           double v = (double)vp[p];
           double m = v * v * dt * dt / (h * h);
           double eta = ex[i] + ey[j] + ez[k];
+          if (spml && eta > 0.0) { /* O6b */
+            const double ed[3] = {ex[i] * dt, ey[j] * dt, ez[k] * dt};
+            double sum = 0.0;
+            for (int d = 0; d < 3; ++d) {
+              const double Ld = lap_axis(g, b, i, j, k, d);
+              wa[d][p] = ((2.0 - ed[d] * ed[d]) * wb[d][p] - (1.0 - ed[d]) * wa[d][p] + m * Ld) / (1.0 + ed[d]);
+              sum += wa[d][p];
+            }
+            a[p] = sum;
+            continue;
+          }
           double L = lap_at(g, b, i, j, k);
           a[p] = (2.0 * b[p] - (1.0 - eta * dt) * a[p] + m * L) / (1.0 + eta * dt);
         }
@@ -243,7 +293,14 @@ int or_iso_run(const or_grid* g, const float* vp, double* u_prev, double* u_cur,
         size_t p = IDX(g, q[0], q[1], q[2]);
         double v = (double)vp[p];
         double eta = ex[q[0]] + ey[q[1]] + ez[q[2]];
-        a[p] += v * v * dt * dt * inj->amp[(size_t)t * inj->n + r] / (h * h * h) / (1.0 + eta * dt);
+        const double amp = v * v * dt * dt * inj->amp[(size_t)t * inj->n + r] / (h * h * h);
+        if (spml && eta > 0.0) { /* O6b: into the x component */
+          const double sx = amp / (1.0 + ex[q[0]] * dt);
+          a[p] += sx;
+          wa[0][p] += sx;
+          continue;
+        }
+        a[p] += amp / (1.0 + eta * dt);
       }
     if (rec && seis)
       for (int r = 0; r < rec->n; ++r) {
@@ -253,9 +310,22 @@ int or_iso_run(const or_grid* g, const float* vp, double* u_prev, double* u_cur,
     double* tmp = a; /* logical swap of time levels */
     a = b;
     b = tmp;
+    for (int d = 0; spml && d < 3; ++d) {
+      tmp = wa[d];
+      wa[d] = wb[d];
+      wb[d] = tmp;
+    }
   }
   memcpy(u_prev, a, sizeof(double) * n);
   memcpy(u_cur, b, sizeof(double) * n);
+  if (spml && (nsteps & 1)) /* the caller's w[0] = level n-1, w[1] = level n */
+    for (int d = 0; d < 3; ++d) {
+      double* t0 = (double*)malloc(sizeof(double) * n);
+      memcpy(t0, w + (size_t)d * n, sizeof(double) * n);
+      memcpy(w + (size_t)d * n, w + (size_t)(3 + d) * n, sizeof(double) * n);
+      memcpy(w + (size_t)(3 + d) * n, t0, sizeof(double) * n);
+      free(t0);
+    }
   free(a);
   free(b);
   free(ex);
@@ -612,7 +682,8 @@ int or_migrate(const or_grid* g, int kind, const float* vp, const float* vs, con
   or_inj recinj = {nrec, rec_pos, back_amp};
   int rc = 0;
   double *a = (double*)calloc(n, sizeof(double)), *b = (double*)calloc(n, sizeof(double));
-  double *q = NULL, *psi = NULL, *f = NULL;
+  double *q = NULL, *psi = NULL, *f = NULL, *w = NULL;
+  if (kind == 0) w = (double*)calloc(6 * n, sizeof(double)); /* O6b split fields (if used) */
   if (kind == 1) {
     q = (double*)calloc(3 * n, sizeof(double));
     psi = (double*)calloc(6 * n, sizeof(double));
@@ -624,7 +695,7 @@ int or_migrate(const or_grid* g, int kind, const float* vp, const float* vs, con
   /* forward phase */
   for (int t = 0; t < nt && !rc; ++t) {
     if (kind == 0) {
-      rc = or_iso_run(g, vp, a, b, t, 1, &src, NULL, NULL);
+      rc = or_iso_run(g, vp, a, b, w, t, 1, &src, NULL, NULL);
     } else if (kind == 1) {
       rc = or_ac_run(g, vp, rho, b, q, q + n, q + 2 * n, psi, t, 1, &src, NULL, NULL);
     } else {
@@ -637,6 +708,7 @@ int or_migrate(const or_grid* g, int kind, const float* vp, const float* vs, con
   /* backward phase: fresh zero state */
   memset(a, 0, sizeof(double) * n);
   memset(b, 0, sizeof(double) * n);
+  if (kind == 0) memset(w, 0, sizeof(double) * 6 * n);
   if (kind == 1) {
     memset(q, 0, sizeof(double) * 3 * n);
     memset(psi, 0, sizeof(double) * 6 * n);
@@ -652,7 +724,7 @@ int or_migrate(const or_grid* g, int kind, const float* vp, const float* vs, con
       for (size_t o = 0; o < n; ++o) image[o] += Sj[o] * b[o]; /* P:111 zero-lag */
     }
     if (kind == 0) {
-      rc = or_iso_run(g, vp, a, b, m, 1, &recinj, NULL, NULL);
+      rc = or_iso_run(g, vp, a, b, w, m, 1, &recinj, NULL, NULL);
     } else if (kind == 1) {
       rc = or_ac_run(g, vp, rho, b, q, q + n, q + 2 * n, psi, m, 1, &recinj, NULL, NULL);
     } else {
@@ -668,5 +740,6 @@ int or_migrate(const or_grid* g, int kind, const float* vp, const float* vs, con
   free(q);
   free(psi);
   free(f);
+  free(w);
   return rc;
 }

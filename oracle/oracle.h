@@ -34,6 +34,7 @@ typedef struct {
   double pml_f;         /* C-PML alpha reference frequency (Hz) (O7) */
   int32_t periodic;     /* TEST MODE (O4): periodic wrap instead of zero ghosts; needs nb = 0;
                            with free_surface the wrap is lateral (x, y) only */
+  int32_t iso_pml;      /* ISO absorbing layer: 0 = damped wave (O6), 1 = split-field PML (O6b) */
 } or_grid;
 
 /* O1: 8th-order coefficient tables: c[0..4] centred 2nd derivative,
@@ -69,8 +70,11 @@ typedef struct {
 
 /* ISO (Eq 1 + O3/O6): advance (u_prev, u_cur) = (u^{n-1}, u^n) by nsteps
  * steps starting at absolute step n0; on return they hold the last two
- * levels.  seis[s][r] = u^{n0+s+1}(x_r) (O13).  Returns 0 on success. */
-int or_iso_run(const or_grid* g, const float* vp, double* u_prev, double* u_cur,
+ * levels.  seis[s][r] = u^{n0+s+1}(x_r) (O13).  Returns 0 on success.
+ * w: split-field PML state (O6b, g->iso_pml = 1 and nb > 0; else ignored, may be
+ * NULL): [2][3][nz][ny][nx], w[0][d] = u^{(d),n-1}, w[1][d] = u^{(d),n}, used only
+ * inside the layers; updated in place like (u_prev, u_cur). */
+int or_iso_run(const or_grid* g, const float* vp, double* u_prev, double* u_cur, double* w,
                int n0, int nsteps, const or_inj* inj, const or_rec* rec, double* seis);
 
 /* ACOUSTIC (Eq 2 in 3D, O8 + O7): state p, qx, qy, qz and psi[6][N^3]

@@ -50,7 +50,8 @@ class SeisError(RuntimeError):
 class _CGrid(C.Structure):
     _fields_ = [("nx", C.c_int32), ("ny", C.c_int32), ("nz", C.c_int32), ("h", C.c_float),
                 ("dt", C.c_float), ("nb", C.c_int32), ("free_surface", C.c_int32),
-                ("pml_R", C.c_float), ("pml_f", C.c_float), ("slabs", C.c_int32)]
+                ("pml_R", C.c_float), ("pml_f", C.c_float), ("slabs", C.c_int32),
+                ("iso_pml", C.c_int32)]
 
 
 class _CShot(C.Structure):
@@ -120,10 +121,11 @@ class Grid:
     pml_R: float = 1e-3
     pml_f: float = 10.0
     slabs: int = 1
+    iso_pml: int = 0  # ISO layer: 0 = damped wave (O6), 1 = split-field PML (O6b)
 
     def c(self) -> _CGrid:
         return _CGrid(self.nx, self.ny, self.nz, self.h, self.dt, self.nb, self.free_surface,
-                      self.pml_R, self.pml_f, self.slabs)
+                      self.pml_R, self.pml_f, self.slabs, self.iso_pml)
 
 
 @dataclass

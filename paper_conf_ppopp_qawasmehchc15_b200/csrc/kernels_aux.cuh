@@ -35,7 +35,8 @@ __global__ void gather_kernel(float* __restrict__ seis_row, const float* __restr
 __global__ void inject_kernel(float* __restrict__ f, const long long* __restrict__ off,
                               const float* __restrict__ scale, const int* __restrict__ gstart,
                               const int* __restrict__ members, const float* __restrict__ data_row,
-                              int ngroups, Ghost gh, long long PS, int nzl) {
+                              int ngroups, Ghost gh, long long PS, int nzl,
+                              const int* __restrict__ sidx, float* __restrict__ spx) {
   const int u = blockIdx.x * blockDim.x + threadIdx.x;
   if (u >= ngroups) return;
   float s = 0.0f;
@@ -43,6 +44,7 @@ __global__ void inject_kernel(float* __restrict__ f, const long long* __restrict
   const long long o = off[u];
   const float v = fmaf(scale[u], s, f[o]);
   f[o] = v;
+  if (spx && sidx[u] >= 0) spx[sidx[u]] = fmaf(scale[u], s, spx[sidx[u]]);  // ISO O6b: x component
   ghost_st1(gh, o, (int)(o / PS) - GZ, nzl, v);  // (f4) the neighbour's ghost copy of the node
 }
 

@@ -39,7 +39,23 @@ struct IsoArgs {
   const float* __restrict__ imgS;// compact snapshot S_j for imaging, or nullptr
   float* __restrict__ img;       // compact image (+=), or nullptr
   Ghost gh;                      // direct ghost stores of u^{n+1} (f4)
+  // split-field PML (O6b, SPML kernels): components u^(x), u^(y), u^(z) of the layer points,
+  // compact storage sp[(lvl * 3 + d) * spn + idx], lvl = time level (u^n: lvl, u^{n-1} and
+  // the new u^{n+1}: 1 - lvl), idx = x-slab [nzl][ny][2nb] for points in the x layer, else
+  // y-slab [nzl][2nb][nx] (offset nxs), else z-slab [2nb][ny][nx] (global z slot, offset nxs + nys)
+  float* __restrict__ sp;
+  long long spn;
+  int nbl, nxs, nys, lvl;
 };
+
+// O6b storage index of a layer point (ex / ey: eta_x dt, eta_y dt at the point)
+__device__ __forceinline__ int spml_idx(const Dims& d, int nb, int nxs, int nys, float ex, float ey, int x, int j,
+                                        int k) {
+  if (ex != 0.0f) return (k * d.ny + j) * (2 * nb) + (x < nb ? x : x - (d.nx - 2 * nb));
+  if (ey != 0.0f) return nxs + (k * (2 * nb) + (j < nb ? j : j - (d.ny - 2 * nb))) * d.nx + x;
+  const int gz = k + d.z0;
+  return nxs + nys + ((gz < nb ? gz : gz - (d.nz - 2 * nb)) * d.ny + j) * d.nx + x;
+}
 
 #ifndef SEIS_ISO_NS
 #define SEIS_ISO_NS 3
@@ -53,7 +69,7 @@ struct IsoStage {
   static constexpr size_t smem_bytes() { return (size_t)ISO_NS * SIZE * 4 + 128; }
 };
 
-template <int BY, bool SNAP, bool IMG>
+template <int BY, bool SNAP, bool IMG, bool SPML = false>
 __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constant__ IsoArgs a) {
   using L = IsoStage<BY>;
   constexpr int W = L::W;
@@ -99,11 +115,15 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
 #pragma unroll
   for (int t = 0; t < 8; ++t) q[t] = ldg4(un + (long long)(k0 - 4 + t + GZ) * PS + oc);
   F4 exy{{0.f, 0.f, 0.f, 0.f}};
+  F4 exv{{0.f, 0.f, 0.f, 0.f}};  // (SPML) eta_x dt per component
+  float eyv = 0.f;               // (SPML) eta_y dt
   if (a.edx && own) {
     const F4 ex = ldg4(a.edx + x0);
     const float ey = a.edy[j];
 #pragma unroll
     for (int e = 0; e < 4; ++e) exy.v[e] = ex.v[e] + ey;
+    exv = ex;
+    eyv = ey;
   }
   const long long srel0 = a.src_o - oc;  // source offset relative to this column
   // block-uniform: does this tile touch the x / y damping layer?  Planes outside the z layer
@@ -149,9 +169,53 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
       lap[e] = fmaf(SEIS_C4, (xv[0 + e] + xv[8 + e]) + ys[3].v[e] + (q[0].v[e] + q[8].v[e]), l);
     }
     F4 out;
+    int sidx[4] = {-1, -1, -1, -1};  // (SPML) storage index of the layer components
     if (!damp) {  // block-uniform branch
 #pragma unroll
       for (int e = 0; e < 4; ++e) out.v[e] = fmaf(mv.v[e], lap[e], 2.0f * xv[4 + e] - upv.v[e]);
+    } else if (SPML) {
+      // O6b: layer points advance u^(x), u^(y), u^(z), each damped along its own axis with the
+      // 1D part L_d of the Laplacian; u^{n+1} is their sum.  Other points: Eq 1.
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const float u = xv[4 + e];
+        const float ed[3] = {exv.v[e], eyv, ez};
+        if (own && x0 + e < d.nx && (ed[0] != 0.0f || ed[1] != 0.0f || ed[2] != 0.0f)) {
+          float Ld[3];
+          {
+            float l = SEIS_C0 * u;
+            l = fmaf(SEIS_C1, xv[3 + e] + xv[5 + e], l);
+            l = fmaf(SEIS_C2, xv[2 + e] + xv[6 + e], l);
+            l = fmaf(SEIS_C3, xv[1 + e] + xv[7 + e], l);
+            Ld[0] = fmaf(SEIS_C4, xv[0 + e] + xv[8 + e], l);
+            l = SEIS_C0 * u;
+            l = fmaf(SEIS_C1, ys[0].v[e], l);
+            l = fmaf(SEIS_C2, ys[1].v[e], l);
+            l = fmaf(SEIS_C3, ys[2].v[e], l);
+            Ld[1] = fmaf(SEIS_C4, ys[3].v[e], l);
+            l = SEIS_C0 * u;
+            l = fmaf(SEIS_C1, q[3].v[e] + q[5].v[e], l);
+            l = fmaf(SEIS_C2, q[2].v[e] + q[6].v[e], l);
+            l = fmaf(SEIS_C3, q[1].v[e] + q[7].v[e], l);
+            Ld[2] = fmaf(SEIS_C4, q[0].v[e] + q[8].v[e], l);
+          }
+          const int id = spml_idx(d, a.nbl, a.nxs, a.nys, ed[0], ed[1], x0 + e, j, k);
+          sidx[e] = id;
+          float* cur = a.sp + (long long)a.lvl * 3 * a.spn + id;
+          float* nxt = a.sp + (long long)(1 - a.lvl) * 3 * a.spn + id;
+          float sum = 0.0f;
+#pragma unroll
+          for (int c = 0; c < 3; ++c) {
+            const float w0 = cur[c * a.spn], wm = nxt[c * a.spn];
+            const float w1 = ((2.0f - ed[c] * ed[c]) * w0 - (1.0f - ed[c]) * wm + mv.v[e] * Ld[c]) / (1.0f + ed[c]);
+            nxt[c * a.spn] = w1;
+            sum += w1;
+          }
+          out.v[e] = sum;
+        } else {
+          out.v[e] = fmaf(mv.v[e], lap[e], 2.0f * u - upv.v[e]);
+        }
+      }
     } else {
 #pragma unroll
       for (int e = 0; e < 4; ++e) {
@@ -171,7 +235,10 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
       if (rel >= 0 && rel < 4) {
 #pragma unroll
         for (int e = 0; e < 4; ++e)
-          if (rel == e) out.v[e] += a.src_amp;
+          if (rel == e) {
+            out.v[e] += a.src_amp;
+            if (SPML && sidx[e] >= 0) a.sp[(long long)(1 - a.lvl) * 3 * a.spn + sidx[e]] += a.src_amp;  // x component
+          }
       }
       st4_masked(a.up + o, out, x0, d.nx, true);
       ghost_st4(a.gh, o, k, d.nzl, out, x0, d.nx);

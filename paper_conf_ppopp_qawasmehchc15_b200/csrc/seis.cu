@@ -166,9 +166,14 @@ struct Slab {
     int* start = nullptr;
     int* mem = nullptr;
     int* surf = nullptr;     // ELASTIC: group node on the free surface
+    int* sidx = nullptr;     // ISO O6b: split-storage index of the node (-1 outside the layers)
   } grp[2];
   float* snap = nullptr;     // nsnap * nzl*ny*nx (points into the model's pool)
   Ghost gh[9];               // direct ghost-plane stores per field index (f4)
+  // ISO split-field PML (O6b): 6 x spn floats, see IsoArgs::sp
+  float* sp = nullptr;
+  long long spn = 0;
+  int spx = 0, spy = 0;      // x-slab / y-slab region sizes (offsets of the y / z regions)
 };
 
 template <class T>
@@ -357,6 +362,9 @@ seis_status set_smem_attrs() {
   SMEM_ATTR((iso_step_kernel<BYI, false, false>), IsoStage<BYI>::smem_bytes());
   SMEM_ATTR((iso_step_kernel<BYI, true, false>), IsoStage<BYI>::smem_bytes());
   SMEM_ATTR((iso_step_kernel<BYI, false, true>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, false, false, true>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, true, false, true>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, false, true, true>), IsoStage<BYI>::smem_bytes());
   SMEM_ATTR((ac_v_kernel<BYV, false>), AcVStage<BYV>::smem_bytes());
   SMEM_ATTR((ac_v_kernel<BYV, true>), AcVStage<BYV>::smem_bytes());
   SMEM_ATTR((ac_p_kernel<BYP, false>), AcPStage<BYP>::smem_bytes());
@@ -625,6 +633,8 @@ static seis_status validate_grid(const seis_grid* g, seis_kind kind) {
   if (g->free_surface && kind != SEIS_ELASTIC)
     return fail(SEIS_EUNSUPPORTED, "free_surface is implemented for ELASTIC only");
   if (g->slabs < 1) return fail(SEIS_EINVAL, "slabs must be >= 1");
+  if (g->iso_pml != 0 && g->iso_pml != 1) return fail(SEIS_EINVAL, "iso_pml must be 0 or 1");
+  if (g->iso_pml && kind != SEIS_ISO) return fail(SEIS_EUNSUPPORTED, "iso_pml applies to ISO only");
   return SEIS_OK;
 }
 
@@ -779,6 +789,15 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
         hc[t] = (float)(v * v * dt * dt / (h * h));
       }
       TRY(upload_padded_from_host(M, d, hc, &S.m, st));
+      if (g.iso_pml && g.nb > 0) {  // O6b split components of the layer points
+        const long long nbl = g.nb;
+        S.spx = (int)((long long)lnz * g.ny * 2 * nbl);
+        S.spy = (int)((long long)lnz * 2 * nbl * g.nx);
+        S.spn = (long long)S.spx + S.spy + 2 * nbl * g.ny * (long long)g.nx;
+        if (S.spn >= 2147483647LL) return fail(SEIS_EUNSUPPORTED, "split-PML storage exceeds 32-bit indexing");
+        TRY(alloc_track(M, (void**)&S.sp, (size_t)S.spn * 6 * sizeof(float)));
+        CK(cudaMemsetAsync(S.sp, 0, (size_t)S.spn * 6 * sizeof(float), st));
+      }
     } else {
       // buoyancy on faces (O8): both V kernels evaluate dt 2/(rho_i + rho_{i+1}) / h on the
       // fly from rho, whose z-ghost planes are exchanged once below
@@ -1114,6 +1133,10 @@ seis_status seis_memory_required(const seis_grid* g, seis_kind kind, const seis_
   // (the default split acoustic step: 4 fields, psi_p + psi_q; SEIS_AC_FUSED=1 doubles p, q, psi_p)
   int nf = nfields(kind, false), np = kind == SEIS_ISO ? 1 : (kind == SEIS_ACOUSTIC ? 2 : 3);  // m | kdt,rho | l2m,w,rho
   double b = (nf + np) * padded;
+  double spml = 0.0;  // ISO O6b split components (6 per layer point, compact slabs)
+  if (kind == SEIS_ISO && g->iso_pml && g->nb > 0)
+    spml = 6.0 * 4.0 * 2.0 * g->nb * ((double)nzl * g->ny + (double)nzl * g->nx + (double)g->ny * g->nx);
+  b += spml;
   if (kind != SEIS_ISO && g->nb > 0) {
     const double W = g->nb + 1;
     const double per = (2 * W * g->ny * (double)nzl + 2 * W * g->nx * (double)nzl + 2 * W * g->nx * (double)g->ny) * 4.0;
@@ -1130,6 +1153,7 @@ seis_status seis_memory_required(const seis_grid* g, seis_kind kind, const seis_
       ck += (2 * W * g->ny * (double)nzl + 2 * W * g->nx * (double)nzl + 2 * W * g->nx * (double)g->ny) * 4.0 *
             (kind == SEIS_ACOUSTIC ? 2 : 6);
     }
+    ck += spml;
     b += (double)c * nzl * (double)g->ny * g->nx * 4.0 + (double)nckpt * ck;
   }
   *bytes = (uint64_t)b;
@@ -1140,6 +1164,21 @@ seis_status seis_memory_required(const seis_grid* g, seis_kind kind, const seis_
 
 // ================================================================== shots
 namespace {
+
+// O6b storage index of global node (x, y, z) in slab S (the kernels' spml_idx), -1 outside
+// the layers or without the split-field PML
+int spml_index_host(const seis_model* M, const Slab& S, int x, int y, int z) {
+  if (!S.sp) return -1;
+  const int nb = M->g.nb;
+  const float dt = M->g.dt;  // membership as the kernels test it: eta_d dt in fp32
+  const float fx = (float)(M->eta1[0][x] * dt), fy = (float)(M->eta1[1][y] * dt), fz = (float)(M->eta1[2][z] * dt);
+  if (fx == 0.0f && fy == 0.0f && fz == 0.0f) return -1;
+  const int k = z - S.d.z0;
+  const int nx = S.d.nx, ny = S.d.ny, nz = S.d.nz;
+  if (fx != 0.0f) return (k * ny + y) * (2 * nb) + (x < nb ? x : x - (nx - 2 * nb));
+  if (fy != 0.0f) return S.spx + (k * (2 * nb) + (y < nb ? y : y - (ny - 2 * nb))) * nx + x;
+  return S.spx + S.spy + ((z < nb ? z : z - (nz - 2 * nb)) * ny + y) * nx + x;
+}
 
 struct ShotTables {
   std::vector<float*> owned;  // device allocations to free
@@ -1176,6 +1215,9 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
     if (M->kind == SEIS_ISO) {
       double eta = 0.0;
       if (g.nb > 0) eta = M->eta1[0][x] + M->eta1[1][y] + M->eta1[2][z];
+      if (g.iso_pml && g.nb > 0 && ((float)(M->eta1[0][x] * dt) != 0.0f || (float)(M->eta1[1][y] * dt) != 0.0f ||
+                                    (float)(M->eta1[2][z] * dt) != 0.0f))
+        eta = M->eta1[0][x];  // O6b: the x component takes the source
       return v * v * dt * dt / (h * h * h) / (1.0 + eta * dt);  // O3
     }
     const double r = M->hrho[li];
@@ -1213,6 +1255,7 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
     for (auto& G2 : S.grp) {
       if (G2.off) {
         cudaFree(G2.off); cudaFree(G2.scale); cudaFree(G2.start); cudaFree(G2.mem); cudaFree(G2.surf);
+        cudaFree(G2.sidx);
       }
       G2 = Slab::Groups{};
     }
@@ -1222,7 +1265,7 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
       for (size_t t = 0; t < off.size(); ++t) groups[off[t]].push_back(rid[t]);
       std::vector<long long> goff[2];
       std::vector<float> gsc[2];
-      std::vector<int> gstart[2] = {{0}, {0}}, gmem[2], gsurf[2];
+      std::vector<int> gstart[2] = {{0}, {0}}, gmem[2], gsurf[2], gsidx[2];
       for (auto& kv : groups) {
         const int r0 = kv.second.front();
         const int* p = sh->rec + 3 * r0;
@@ -1231,6 +1274,7 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
         goff[part].push_back(kv.first);
         gsc[part].push_back((float)point_scale(p[0], p[1], p[2]));
         gsurf[part].push_back(M->g.free_surface && p[2] == 0 ? 1 : 0);
+        gsidx[part].push_back(spml_index_host(M, S, p[0], p[1], p[2]));
         for (int r : kv.second) gmem[part].push_back(r);
         gstart[part].push_back((int)gmem[part].size());
       }
@@ -1243,6 +1287,8 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
         CK(dmalloc(&G2.start, gstart[part].size()));
         CK(dmalloc(&G2.mem, gmem[part].size()));
         CK(dmalloc(&G2.surf, gsurf[part].size()));
+        CK(dmalloc(&G2.sidx, gsidx[part].size()));
+        CK(cudaMemcpy(G2.sidx, gsidx[part].data(), gsidx[part].size() * sizeof(int), cudaMemcpyHostToDevice));
         CK(cudaMemcpy(G2.surf, gsurf[part].data(), gsurf[part].size() * sizeof(int), cudaMemcpyHostToDevice));
         CK(cudaMemcpy(G2.off, goff[part].data(), goff[part].size() * sizeof(long long), cudaMemcpyHostToDevice));
         CK(cudaMemcpy(G2.scale, gsc[part].data(), gsc[part].size() * sizeof(float), cudaMemcpyHostToDevice));
@@ -1261,6 +1307,7 @@ seis_status zero_state(seis_model* M, cudaStream_t st) {
   for (Slab& S : M->slabs) {
     const size_t elems = (size_t)S.d.PS * (S.d.nzl + 2 * GZ);
     for (float* f : S.fld) CK(cudaMemsetAsync(f, 0, elems * sizeof(float), st));
+    if (S.sp) CK(cudaMemsetAsync(S.sp, 0, (size_t)S.spn * 6 * sizeof(float), st));
     if (M->W > 0) {
       const int W = M->W;
       const int npsi = npsi_of(M->kind, M->ac_fused);
@@ -1288,6 +1335,7 @@ std::vector<std::pair<float*, size_t>> state_arrays(seis_model* M) {
     const bool fz = M->ac_fused;
     for (size_t f = 0; f < S.fld.size(); ++f)
       if (!fz || (int)f / 4 == S.cur) v.emplace_back(S.fld[f] - 28, elems);  // base = f - 112 bytes
+    if (S.sp) v.emplace_back(S.sp, (size_t)S.spn * 6);  // ISO O6b split components
     if (M->W > 0) {
       const int W = M->W;
       for (int t = 0; t < npsi_of(M->kind, fz); ++t) {
@@ -1362,7 +1410,8 @@ seis_status inject_rows(seis_model* M, const float* row, int part, cudaStream_t 
       } else {
         const int f = M->kind == SEIS_ISO ? S.cur : 4 * S.cur;
         inject_kernel<<<(G2.n + 127) / 128, 128, 0, st>>>(S.fld[f], G2.off, G2.scale, G2.start, G2.mem, row,
-                                                         G2.n, S.gh[f], S.d.PS, S.d.nzl);
+                                                         G2.n, S.gh[f], S.d.PS, S.d.nzl, G2.sidx,
+                                                         S.sp ? S.sp + (size_t)S.cur * 3 * S.spn : nullptr);
       }
       CKL();
     }
@@ -1458,11 +1507,21 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.imgS = imgS ? (*imgS)[s] : nullptr;
       a.img = img ? (*img)[s] : nullptr;
       a.gh = S.gh[1 - cur];
+      a.sp = S.sp;
+      a.spn = S.spn;
+      a.nbl = M->g.nb;
+      a.nxs = S.spx;
+      a.nys = S.spy;
+      a.lvl = cur;
       const dim3 gr = grid_of(S, TXV, BYI, nch), blk(NTX, BYI);
       {
         PROF(0, ks);
         const size_t sb = IsoStage<BYI>::smem_bytes();
-        if (a.snap) iso_step_kernel<BYI, true, false><<<gr, blk, sb, ks>>>(a);
+        if (S.sp) {  // O6b split-field PML
+          if (a.snap) iso_step_kernel<BYI, true, false, true><<<gr, blk, sb, ks>>>(a);
+          else if (a.img) iso_step_kernel<BYI, false, true, true><<<gr, blk, sb, ks>>>(a);
+          else iso_step_kernel<BYI, false, false, true><<<gr, blk, sb, ks>>>(a);
+        } else if (a.snap) iso_step_kernel<BYI, true, false><<<gr, blk, sb, ks>>>(a);
         else if (a.img) iso_step_kernel<BYI, false, true><<<gr, blk, sb, ks>>>(a);
         else iso_step_kernel<BYI, false, false><<<gr, blk, sb, ks>>>(a);
       }

@@ -128,3 +128,12 @@ def test_peer_mode_entry_points_validate_before_touching_the_device():
     n = C.c_uint64()
     assert L.seis_model_peer_export(None, None, 0, C.byref(n)) == 1
     assert L.seis_model_peer_import(None, None, 0, None, 0) == 1
+
+
+def test_iso_split_pml_rejected_for_other_kinds():
+    import numpy as np
+
+    vp = np.full((16, 16, 16), 2000.0, np.float32)
+    with pytest.raises(seis.SeisError) as e:
+        seis.Model(seis.Grid(16, 16, 16, 10.0, 1e-3, nb=4, iso_pml=1), "acoustic", vp, rho=vp)
+    assert e.value.name == "SEIS_EUNSUPPORTED"

@@ -126,3 +126,83 @@ def test_iso_damping_layer_reflection_below_one_percent():
 def test_layers_actually_absorb():
     """Sanity of the measurement: without a layer the zero-Dirichlet walls reflect strongly."""
     assert _reflection("acoustic", 0) > 5e-2
+
+
+# ---------------------------------------------------------------- O6b split-field PML
+def _spml_case(nb, R, iso_pml, chunks=(40,)):
+    n, h, dt, v, fp = 28, 10.0, 1e-3, 2000.0, 25.0
+    g = oracle.Grid(n, n, n, h=h, dt=dt, nb=nb, pml_R=R, pml_f=fp, iso_pml=iso_pml)
+    vp = inputs.random_media(g.shape, seed=8)["vp"] * np.float32(0.6)
+    nt = sum(chunks)
+    w = inputs.source_series("iso", nt, dt, fp)
+    src = [(3, n // 2, n // 2)]  # inside the x layer: the source enters the x component
+    rec = [(n // 2, n // 2, 2), (n - 3, 4, n // 2), (n // 2, n // 2, n // 2)]
+    st = oracle.iso_state(g)
+    seis, t = [], 0
+    for c in chunks:  # odd and even chunk lengths exercise the level bookkeeping of w
+        seis.append(oracle.iso_run(g, vp, st, t, c, src, w[:, None], rec))
+        t += c
+    return np.concatenate(seis), st, g
+
+
+def test_split_pml_components_sum_to_eq1_when_undamped():
+    """O6b with eta -> 0 (R = 1 - 1e-6, an fp32 value: every layer point takes the split
+    update with eta_d dt ~ 1e-10) reproduces Eq 1 without layers: the three 1D updates must
+    add up to the 25-point update (a dropped or mis-signed term, a wrong axis, a wrong level
+    or source routing would not).  The remaining difference is the damping itself: it must be
+    linear in ln(1/R) (x10 from R = 1 - 1e-6 to 1 - 1e-5), i.e. no O(1) part."""
+    ref, st0, _ = _spml_case(0, 1e-3, 0)
+    got, st1, g = _spml_case(8, 1.0 - 1e-6, 1, chunks=(7, 3, 30))
+    got5, _, _ = _spml_case(8, 1.0 - 1e-5, 1, chunks=(7, 3, 30))
+    assert np.abs(ref).max() > 0
+    e6 = np.linalg.norm(got - ref) / np.linalg.norm(ref)
+    e5 = np.linalg.norm(got5 - ref) / np.linalg.norm(ref)
+    assert e6 < 1e-6 and e5 / e6 == pytest.approx(10.0, rel=0.05)
+    for key in ("u_prev", "u_cur"):
+        assert np.linalg.norm(st1[key] - st0[key]) / np.linalg.norm(st0[key]) < 1e-6
+    # the split state is populated inside the layers and zero outside
+    w = st1["w"]
+    inner = (slice(8, -8),) * 3
+    assert np.abs(w[1][(slice(None),) + inner]).max() == 0.0
+    assert np.abs(w[1, 0, :, :, :8]).max() > 0
+
+
+def test_split_pml_components_sum_to_the_field_in_the_layers():
+    """u = u^(x) + u^(y) + u^(z) at every layer point and both stored levels (O6b)."""
+    _, st, g = _spml_case(8, 1e-3, 1, chunks=(9, 16))
+    n = g.nx
+    lay = np.zeros(g.shape, bool)
+    idx = np.r_[0:8, n - 8:n]
+    lay[idx, :, :] = True
+    lay[:, idx, :] = True
+    lay[:, :, idx] = True
+    for lvl, key in ((0, "u_prev"), (1, "u_cur")):
+        s = st["w"][lvl].sum(axis=0)
+        assert np.abs(st[key][lay]).max() > 0
+        assert np.allclose(s[lay], st[key][lay], rtol=1e-12, atol=1e-12 * np.abs(st[key]).max())
+
+
+@pytest.mark.slow
+def test_split_pml_absorbs():
+    """The split-field layer absorbs (walls alone reflect > 5 %, see below) and improves with
+    its width.  It reflects more than the damped-wave layer of the same width (measured 1.9 %
+    vs 0.84 % at nb = 8, 1.5 % vs 0.51 % at nb = 10): the second-order split form drops the
+    profile-gradient terms of the exact PML, the "spurious reflections" of the standard PML
+    that P:179 gives as the reason to use C-PML elsewhere."""
+    r8, r10 = _reflection_spml(8), _reflection_spml(10)
+    assert r8 < 2.5e-2 and r10 < r8
+
+
+def _reflection_spml(nb):
+    h, dt, v, fp, nt = 10.0, 1e-3, 2000.0, 25.0, 260
+    small, large = 32, 64
+    out = {}
+    for n in (small, large):
+        c = n // 2
+        g = oracle.Grid(n, n, n, h=h, dt=dt, nb=(nb if n == small else 0), pml_f=fp, iso_pml=1)
+        vp = np.full(g.shape, v, np.float32)
+        rec = [(c + 5, c, c), (c, c + 5, c), (c, c, c + 5), (c + 4, c + 4, c), (c - 5, c, c - 4)]
+        w = inputs.source_series("iso", nt, dt, fp)
+        out[n] = oracle.iso_run(g, vp, oracle.iso_state(g), 0, nt, [(c, c, c)], w[:, None], rec)
+    diff = out[small] - out[large]
+    return np.sum(diff ** 2) / np.sum(out[large] ** 2)
