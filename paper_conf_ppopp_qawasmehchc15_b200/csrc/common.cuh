@@ -190,6 +190,21 @@ __device__ __forceinline__ void tma_ld(bool pf, void* dst, const CUtensorMap* ma
 #endif
 constexpr int L2PF = SEIS_L2PF;  // L2 prefetch distance beyond the TMA ring (planes), 0 = off
 
+// Unroll factor of the z-march loops, per kernel family (u: 1 = rolled).  Unrolling by u lets
+// the compiler rename the register z-queues across u planes instead of shifting them every
+// plane (u-fold fewer queue moves), at u times the loop body in the instruction cache.
+#define SEIS_PRAGMA_(x) _Pragma(#x)
+#define SEIS_UNROLL(n) SEIS_PRAGMA_(unroll n)
+#ifndef SEIS_ZU_ISO
+#define SEIS_ZU_ISO 1
+#endif
+#ifndef SEIS_ZU_AC
+#define SEIS_ZU_AC 1
+#endif
+#ifndef SEIS_ZU_EL
+#define SEIS_ZU_EL 2  // profiles/r01_sweep_zu.jsonl: el_v -4.5 %, el_s -4.7 %; ISO / acoustic: no gain
+#endif
+
 }  // namespace seis
 
 // ------------------------------------------------------------ 4-wide vectors
@@ -278,8 +293,12 @@ struct Ghost {
   float* hi = nullptr;
   long long hio = 0;
 };
+#ifndef SEIS_GHOST_ST
+#define SEIS_GHOST_ST 1  // 0: compile the ghost stores out (A/B timing of single-slab kernels only)
+#endif
 __device__ __forceinline__ void ghost_st4(const Ghost& g, long long o, int k, int nzl, const F4& v, int x0,
                                           int nx) {
+  if (!SEIS_GHOST_ST) return;
   if (g.lo && k < 4) st4_masked(g.lo + (o + g.loo), v, x0, nx, true);
   if (g.hi && k >= nzl - 4) st4_masked(g.hi + (o + g.hio), v, x0, nx, true);
 }

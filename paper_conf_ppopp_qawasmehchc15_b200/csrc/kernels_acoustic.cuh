@@ -122,6 +122,7 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
   for (int t = 0; t < 7; ++t) r[t] = ldg4(p + (long long)(k0 - 3 + t + GZ) * PS + oc);
   const float dth = a.dth;
 
+  SEIS_UNROLL(SEIS_ZU_AC)
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % AC_VNS;
@@ -320,6 +321,7 @@ __global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ 
   for (int t = 0; t < 7; ++t) q[t] = ldg4(qz + (long long)(k0 - 4 + t + GZ) * PS + oc);
   const long long srel0 = a.src_o - oc;
 
+  SEIS_UNROLL(SEIS_ZU_AC)
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % AC_NS;

@@ -171,6 +171,7 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
     qyz[t] = ldg2(syz + (long long)(k0 - 4 + t + GZ) * PS + oc);
     qzz[t] = ldg2(szz + (long long)(k0 - 3 + t + GZ) * PS + oc);
   }
+  SEIS_UNROLL(SEIS_ZU_EL)
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % EL_VNS;
@@ -398,6 +399,7 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
     qz[t] = ldg2(vz + (long long)(k0 - 4 + t + GZ) * PS + oc);
   }
   const long long srel0 = a.src_o - oc;
+  SEIS_UNROLL(SEIS_ZU_EL)
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % EL_SNS;

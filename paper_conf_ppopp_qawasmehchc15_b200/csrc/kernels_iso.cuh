@@ -46,6 +46,9 @@ struct IsoArgs {
   float* __restrict__ sp;
   long long spn;
   int nbl, nxs, nys, lvl;
+  // per-axis update coefficients [3][spnp[axis]] (A, B, C of the component update, host-rounded)
+  const float* __restrict__ spco[3];
+  int spnp[3];
 };
 
 // O6b storage index of a layer point (ex / ey: eta_x dt, eta_y dt at the point)
@@ -69,7 +72,9 @@ struct IsoStage {
   static constexpr size_t smem_bytes() { return (size_t)ISO_NS * SIZE * 4 + 128; }
 };
 
-template <int BY, bool SNAP, bool IMG, bool SPML = false>
+// GH: this slab has a neighbour slab / rank whose ghost planes it stores (f4); the single-slab
+// instantiation leaves the check out (-2.7 % iso_step time, profiles/r01_sweep_zu.jsonl)
+template <int BY, bool SNAP, bool IMG, bool SPML = false, bool GH = true>
 __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constant__ IsoArgs a) {
   using L = IsoStage<BY>;
   constexpr int W = L::W;
@@ -125,15 +130,48 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
     exv = ex;
     eyv = ey;
   }
+  // (SPML) per-axis coefficients of this thread's points: x (4 points), y (its row)
+  F4 cax{{2.f, 2.f, 2.f, 2.f}}, cbx{{1.f, 1.f, 1.f, 1.f}}, ccx{{1.f, 1.f, 1.f, 1.f}};
+  float cay = 2.f, cby = 1.f, ccy = 1.f;
+  if (SPML && a.spco[0] && own) {
+    cax = ldg4(a.spco[0] + x0);
+    cbx = ldg4(a.spco[0] + a.spnp[0] + x0);
+    ccx = ldg4(a.spco[0] + 2 * a.spnp[0] + x0);
+    cay = __ldg(a.spco[1] + j);
+    cby = __ldg(a.spco[1] + a.spnp[1] + j);
+    ccy = __ldg(a.spco[1] + 2 * a.spnp[1] + j);
+  }
   const long long srel0 = a.src_o - oc;  // source offset relative to this column
   // block-uniform: does this tile touch the x / y damping layer?  Planes outside the z layer
   // of such tiles take the undamped update without per-point branches (same arithmetic).
   const bool dxy = __syncthreads_or(exy.v[0] != 0.f || exy.v[1] != 0.f || exy.v[2] != 0.f || exy.v[3] != 0.f);
 
+  SEIS_UNROLL(SEIS_ZU_ISO)
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % ISO_NS;
     const long long o = (long long)(k + GZ) * PS + oc;
+    const float ez = a.edx ? a.edz[k + d.z0] : 0.0f;
+    // (SPML) the layer components of this group are loaded before the stage wait (latency
+    // overlap, as the C-PML memory variables): w0 = level n, wm = level n-1
+    int sidx[4] = {-1, -1, -1, -1};
+    float w0[3][4], wm[3][4];
+    if (SPML && (dxy || ez != 0.0f)) {
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        if (own && x0 + e < d.nx && (exv.v[e] != 0.0f || eyv != 0.0f || ez != 0.0f)) {
+          const int id = spml_idx(d, a.nbl, a.nxs, a.nys, exv.v[e], eyv, x0 + e, j, k);
+          sidx[e] = id;
+          const float* cur = a.sp + (long long)a.lvl * 3 * a.spn + id;
+          const float* nxt = a.sp + (long long)(1 - a.lvl) * 3 * a.spn + id;
+#pragma unroll
+          for (int c = 0; c < 3; ++c) {
+            w0[c][e] = cur[c * a.spn];
+            wm[c][e] = nxt[c * a.spn];
+          }
+        }
+      }
+    }
     mbar_wait(&bar[s], (it / ISO_NS) & 1);
     const float* st = sm + s * L::SIZE;
     q[8] = lds4(st + L::UQ + ty * TXV + 4 * tx);
@@ -157,7 +195,6 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
     }
     const F4 upv = lds4(st + L::UP + ty * TXV + 4 * tx);
     const F4 mv = lds4(st + L::M + ty * TXV + 4 * tx);
-    const float ez = a.edx ? a.edz[k + d.z0] : 0.0f;
     const bool damp = dxy || ez != 0.0f;
     float lap[4];
 #pragma unroll
@@ -169,7 +206,6 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
       lap[e] = fmaf(SEIS_C4, (xv[0 + e] + xv[8 + e]) + ys[3].v[e] + (q[0].v[e] + q[8].v[e]), l);
     }
     F4 out;
-    int sidx[4] = {-1, -1, -1, -1};  // (SPML) storage index of the layer components
     if (!damp) {  // block-uniform branch
 #pragma unroll
       for (int e = 0; e < 4; ++e) out.v[e] = fmaf(mv.v[e], lap[e], 2.0f * xv[4 + e] - upv.v[e]);
@@ -179,8 +215,11 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
 #pragma unroll
       for (int e = 0; e < 4; ++e) {
         const float u = xv[4 + e];
-        const float ed[3] = {exv.v[e], eyv, ez};
-        if (own && x0 + e < d.nx && (ed[0] != 0.0f || ed[1] != 0.0f || ed[2] != 0.0f)) {
+        if (sidx[e] >= 0) {
+          const int gz = k + d.z0;
+          const float ca[3] = {cax.v[e], cay, __ldg(a.spco[2] + gz)};
+          const float cb[3] = {cbx.v[e], cby, __ldg(a.spco[2] + a.spnp[2] + gz)};
+          const float cc[3] = {ccx.v[e], ccy, __ldg(a.spco[2] + 2 * a.spnp[2] + gz)};
           float Ld[3];
           {
             float l = SEIS_C0 * u;
@@ -199,15 +238,12 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
             l = fmaf(SEIS_C3, q[1].v[e] + q[7].v[e], l);
             Ld[2] = fmaf(SEIS_C4, q[0].v[e] + q[8].v[e], l);
           }
-          const int id = spml_idx(d, a.nbl, a.nxs, a.nys, ed[0], ed[1], x0 + e, j, k);
-          sidx[e] = id;
-          float* cur = a.sp + (long long)a.lvl * 3 * a.spn + id;
-          float* nxt = a.sp + (long long)(1 - a.lvl) * 3 * a.spn + id;
+          float* nxt = a.sp + (long long)(1 - a.lvl) * 3 * a.spn + sidx[e];
           float sum = 0.0f;
 #pragma unroll
           for (int c = 0; c < 3; ++c) {
-            const float w0 = cur[c * a.spn], wm = nxt[c * a.spn];
-            const float w1 = ((2.0f - ed[c] * ed[c]) * w0 - (1.0f - ed[c]) * wm + mv.v[e] * Ld[c]) / (1.0f + ed[c]);
+            // = [(2 - e^2) w0 - (1 - e) wm + m L_d] / (1 + e), e = eta_d dt (O6b)
+            const float w1 = fmaf(ca[c], w0[c][e], fmaf(-cb[c], wm[c][e], cc[c] * (mv.v[e] * Ld[c])));
             nxt[c * a.spn] = w1;
             sum += w1;
           }
@@ -241,7 +277,7 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
           }
       }
       st4_masked(a.up + o, out, x0, d.nx, true);
-      ghost_st4(a.gh, o, k, d.nzl, out, x0, d.nx);
+      if (GH) ghost_st4(a.gh, o, k, d.nzl, out, x0, d.nx);
       if (SNAP || IMG) {
         const long long cix = ((long long)k * d.ny + j) * d.nx + x0;
         const bool al = (d.nx & 3) == 0;

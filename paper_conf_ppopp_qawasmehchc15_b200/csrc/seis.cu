@@ -195,6 +195,8 @@ struct seis_model {
   std::vector<void*> allocs;   // every cudaMalloc of the model
   // 1D coefficient arrays (global index)
   float *edx = nullptr, *edy = nullptr, *edz = nullptr;      // ISO eta*dt
+  float* spco[3] = {};        // ISO O6b per-axis update coefficients [3][NP] (A, B, C), see IsoArgs
+  int spnp[3] = {};           // their padded lengths NP
   CpmlAxis cp[3] = {};                                       // C-PML
   int W = 0;                   // C-PML slab width per face
   // host copies of this process's model slab (point scales for sources/receivers)
@@ -365,6 +367,12 @@ seis_status set_smem_attrs() {
   SMEM_ATTR((iso_step_kernel<BYI, false, false, true>), IsoStage<BYI>::smem_bytes());
   SMEM_ATTR((iso_step_kernel<BYI, true, false, true>), IsoStage<BYI>::smem_bytes());
   SMEM_ATTR((iso_step_kernel<BYI, false, true, true>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, false, false, false, false>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, true, false, false, false>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, false, true, false, false>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, false, false, true, false>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, true, false, true, false>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, false, true, true, false>), IsoStage<BYI>::smem_bytes());
   SMEM_ATTR((ac_v_kernel<BYV, false>), AcVStage<BYV>::smem_bytes());
   SMEM_ATTR((ac_v_kernel<BYV, true>), AcVStage<BYV>::smem_bytes());
   SMEM_ATTR((ac_p_kernel<BYP, false>), AcPStage<BYP>::smem_bytes());
@@ -710,6 +718,21 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       hf.resize(std::max(N, roundup(N, TXV) + TXV), 0.f);  // float4 loads past nx read zeros
       TRY(alloc_track(M, (void**)&e1[ax], hf.size() * sizeof(float)));
       CK(cudaMemcpy(e1[ax], hf.data(), hf.size() * sizeof(float), cudaMemcpyHostToDevice));
+      if (g.iso_pml && g.nb > 0) {
+        // O6b: u^(d),n+1 = A u^(d),n - B u^(d),n-1 + C m L_d u^n with e = eta_d dt (as the
+        // kernels' fp32 e): A = (2 - e^2)/(1 + e), B = (1 - e)/(1 + e), C = 1/(1 + e), double -> fp32
+        const int NP = (int)hf.size();
+        std::vector<float> co((size_t)3 * NP, 0.f);
+        for (int i = 0; i < NP; ++i) {
+          const double e = (double)hf[i];
+          co[i] = (float)((2.0 - e * e) / (1.0 + e));
+          co[(size_t)NP + i] = (float)((1.0 - e) / (1.0 + e));
+          co[(size_t)2 * NP + i] = (float)(1.0 / (1.0 + e));
+        }
+        TRY(alloc_track(M, (void**)&M->spco[ax], co.size() * sizeof(float)));
+        CK(cudaMemcpy(M->spco[ax], co.data(), co.size() * sizeof(float), cudaMemcpyHostToDevice));
+        M->spnp[ax] = NP;
+      }
     }
     if (g.nb > 0) {
       M->edx = e1[0];
@@ -1513,17 +1536,27 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.nxs = S.spx;
       a.nys = S.spy;
       a.lvl = cur;
+      for (int t = 0; t < 3; ++t) {
+        a.spco[t] = M->spco[t];
+        a.spnp[t] = M->spnp[t];
+      }
       const dim3 gr = grid_of(S, TXV, BYI, nch), blk(NTX, BYI);
       {
         PROF(0, ks);
         const size_t sb = IsoStage<BYI>::smem_bytes();
-        if (S.sp) {  // O6b split-field PML
-          if (a.snap) iso_step_kernel<BYI, true, false, true><<<gr, blk, sb, ks>>>(a);
-          else if (a.img) iso_step_kernel<BYI, false, true, true><<<gr, blk, sb, ks>>>(a);
-          else iso_step_kernel<BYI, false, false, true><<<gr, blk, sb, ks>>>(a);
-        } else if (a.snap) iso_step_kernel<BYI, true, false><<<gr, blk, sb, ks>>>(a);
-        else if (a.img) iso_step_kernel<BYI, false, true><<<gr, blk, sb, ks>>>(a);
-        else iso_step_kernel<BYI, false, false><<<gr, blk, sb, ks>>>(a);
+        // template flags: O6b split-field PML; direct ghost stores of this slab (f4)
+        auto go = [&](auto spml, auto gh) {
+          constexpr bool SP = decltype(spml)::value, GH = decltype(gh)::value;
+          if (a.snap) iso_step_kernel<BYI, true, false, SP, GH><<<gr, blk, sb, ks>>>(a);
+          else if (a.img) iso_step_kernel<BYI, false, true, SP, GH><<<gr, blk, sb, ks>>>(a);
+          else iso_step_kernel<BYI, false, false, SP, GH><<<gr, blk, sb, ks>>>(a);
+        };
+        const bool gh = a.gh.lo || a.gh.hi;
+        if (S.sp) {
+          if (gh) go(std::true_type{}, std::true_type{});
+          else go(std::true_type{}, std::false_type{});
+        } else if (gh) go(std::false_type{}, std::true_type{});
+        else go(std::false_type{}, std::false_type{});
       }
       CKL();
       return SEIS_OK;

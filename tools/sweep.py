@@ -19,10 +19,7 @@ sys.path.insert(0, ROOT)
 
 VARIANTS = {
     "base": [],
-    "pf1": ["SEIS_L2PF=1"],
-    "pf2": ["SEIS_L2PF=2"],
-    "pf4": ["SEIS_L2PF=4"],
-    "pf2_es3": ["SEIS_L2PF=2", "SEIS_EL_SNS=3", "SEIS_EL_VNS=2"],
+    "noghost": ["SEIS_GHOST_ST=0"],
 }
 
 
@@ -31,6 +28,8 @@ def build():
 
     os.makedirs(OUT, exist_ok=True)
     for name, defs in VARIANTS.items():
+        if defs is None:
+            continue
         path = os.path.join(OUT, f"libseis_{name}.so")
         b.build(force=True, defines=defs, out=path)
         print("built", path)

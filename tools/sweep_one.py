@@ -34,6 +34,12 @@ m = seis.Model(seis.Grid(n, n, n, 10.0, 1e-3, nb=20), "iso", vp)
 w = inputs.source_series("iso", 60, 1e-3, 15.0)
 res["iso_512"] = timed(m, seis.Shot((n // 2, n // 2, 24), w, np.asarray([[10, 10, 24]], np.int32)))
 m.close()
+try:  # split-field PML (O6b) variant of the same run
+    m = seis.Model(seis.Grid(n, n, n, 10.0, 1e-3, nb=20, iso_pml=1), "iso", vp)
+    res["iso_512_spml"] = timed(m, seis.Shot((n // 2, n // 2, 24), w, np.asarray([[10, 10, 24]], np.int32)))
+    m.close()
+except Exception as e:  # older builds without iso_pml
+    res["iso_512_spml"] = str(e)[:100]
 del vp
 wl = inputs.c2(n=512, nt=60)
 m = seis.Model(seis.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=wl.nb, pml_f=wl.fp), "acoustic",
