@@ -132,9 +132,12 @@ __device__ __forceinline__ void fence_proxy_async() {
 #ifndef SEIS_WARP_RELEASE
 #define SEIS_WARP_RELEASE 0
 #endif
-template <class Refill>
+#ifndef SEIS_WR_EL
+#define SEIS_WR_EL SEIS_WARP_RELEASE  // the elastic kernels' choice
+#endif
+template <bool WR = (SEIS_WARP_RELEASE != 0), class Refill>
 __device__ __forceinline__ void stage_release(uint32_t* cnt, int tid, bool more, Refill&& refill) {
-#if SEIS_WARP_RELEASE
+  if (WR) {
   __syncwarp();
   if ((tid & 31) == 0) {
     const uint32_t nwarps = (blockDim.x * blockDim.y * blockDim.z) >> 5;
@@ -148,13 +151,13 @@ __device__ __forceinline__ void stage_release(uint32_t* cnt, int tid, bool more,
       }
     }
   }
-#else
+  } else {
   __syncthreads();
   if (tid == 0 && more) {
     fence_proxy_async();
     refill();
   }
-#endif
+  }
 }
 // Fast reciprocal (MUFU.RCP, ~1 ulp; +inf -> +0) for the on-the-fly face/edge averages
 __device__ __forceinline__ float rcp_fast(float x) {

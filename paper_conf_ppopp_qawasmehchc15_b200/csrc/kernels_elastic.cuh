@@ -295,7 +295,7 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constan
           }
       }
     }
-    stage_release(&cnt[s], tid, it + EL_VNS < np, [&] {
+    stage_release<(SEIS_WR_EL != 0)>(&cnt[s], tid, it + EL_VNS < np, [&] {
       issue(s, k + EL_VNS);
       if (L2PF && it + EL_VNS + L2PF < np) issue(s, k + EL_VNS + L2PF, true);
     });
@@ -550,7 +550,7 @@ __global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constan
           if (x0 + e < d.nx) a.snap[cix + e] = -((o6[0].v[e] + o6[1].v[e]) + o6[2].v[e]) / 3.0f;
       }
     }
-    stage_release(&cnt[s], tid, it + EL_SNS < np, [&] {
+    stage_release<(SEIS_WR_EL != 0)>(&cnt[s], tid, it + EL_SNS < np, [&] {
       issue(s, k + EL_SNS);
       if (L2PF && it + EL_SNS + L2PF < np) issue(s, k + EL_SNS + L2PF, true);
     });

@@ -19,7 +19,9 @@ sys.path.insert(0, ROOT)
 
 VARIANTS = {
     "base": [],
-    "noghost": ["SEIS_GHOST_ST=0"],
+    "wr_el": ["SEIS_WR_EL=1"],
+    "wr_all": ["SEIS_WARP_RELEASE=1"],
+    "wr_el_ens3": ["SEIS_WR_EL=1", "SEIS_EL_SNS=3", "SEIS_EL_VNS=3"],
 }
 
 
