@@ -395,17 +395,35 @@ seis_status set_smem_attrs() {
 // profiles/r01_sweep_zchunk.jsonl), and in any case enough blocks for >= 6 waves of the
 // resident slots; chunks of >= 8 planes (the queue warm-up re-reads 8 planes).
 // SEIS_ZCHUNK_MAX overrides zt (sweeps).
-void choose_chunks(Slab& s, int resident_per_sm, int nsm, int tw, int by, int zt) {
+// zex: planes per face the decomposition exchanges (0 = one slab, no exchange).  The first and
+// the last chunk of a slab must then each hold >= zex planes: the overlapped pipeline runs
+// them before the exchange (run_phase), and with direct ghost stores they are the only
+// kernels that store into a neighbour's ghost planes.
+void choose_chunks(Slab& s, int resident_per_sm, int nsm, int tw, int by, int zt, int zex) {
   const long long bxy = (long long)((s.d.nx + tw - 1) / tw) * ((s.d.ny + by - 1) / by);
   const long long slots = (long long)std::max(1, resident_per_sm) * nsm;
   static const int zenv = getenv("SEIS_ZCHUNK_MAX") ? atoi(getenv("SEIS_ZCHUNK_MAX")) : -1;
   const int zmax = zenv >= 0 ? zenv : zt;
+  // minimum chunk: 8 planes; a small (L2-resident, launch-bound) grid may go down to
+  // SEIS_ZCHUNK_MIN planes to put more blocks on the SMs (the z-queue warm-up re-reads hit L2)
+  static const int zmin_env = getenv("SEIS_ZCHUNK_MIN") ? atoi(getenv("SEIS_ZCHUNK_MIN")) : -1;
+  // (profiles/r01_c1_sweep.jsonl: C1 64^3 ISO 36.6 -> 58.4 Gpts/s with 2-plane chunks)
+  const bool small = (double)s.d.nx * s.d.ny * s.d.nzl < 16.0 * 1024 * 1024;
+  const int zmin = std::max(zmin_env > 0 ? zmin_env : (small ? 2 : 8), zex);
   int c = 1;
-  while (bxy * c < 6 * slots && (s.d.nzl + c) / (c + 1) >= 8) ++c;
+  while (bxy * c < 6 * slots && (s.d.nzl + c) / (c + 1) >= zmin) ++c;
   if (zmax >= 8)
     while ((s.d.nzl + c - 1) / c > zmax) ++c;
   s.zc = (s.d.nzl + c - 1) / c;
   s.nzch = (s.d.nzl + s.zc - 1) / s.zc;
+  if (zex > 0) {
+    s.zc = std::max(s.zc, std::min(zex, s.d.nzl));
+    s.nzch = (s.d.nzl + s.zc - 1) / s.zc;
+    while (s.nzch > 1 && s.d.nzl - (s.nzch - 1) * s.zc < zex) {  // a short last chunk
+      ++s.zc;
+      s.nzch = (s.d.nzl + s.zc - 1) / s.zc;
+    }
+  }
 }
 
 int nfields(seis_kind k, bool fused = true) { return k == SEIS_ISO ? 2 : (k == SEIS_ACOUSTIC ? (fused ? 8 : 4) : 9); }
@@ -599,6 +617,7 @@ seis_status seis_comm_create(int32_t nranks, int32_t rank, const uint8_t id[128]
 
 seis_status seis_image_reduce(seis_comm* c, float* image, uint64_t n, void* stream) {
   if (!c || (!image && n)) return fail(SEIS_EINVAL, "seis_image_reduce: null argument");
+  if (!c->nccl) return fail(SEIS_EUNSUPPORTED, "seis_image_reduce needs an NCCL communicator (peer-only given)");
   CK(cudaSetDevice(c->device));
   if (!is_device_ptr(image)) return fail(SEIS_EINVAL, "seis_image_reduce: image must be a device buffer");
   cudaStream_t st = (cudaStream_t)stream;
@@ -925,9 +944,11 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     else
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, NTX2 * BYE,
                                                     ElSStage<BYE>::smem_bytes());
-    if (kind == SEIS_ELASTIC) choose_chunks(S, occ, dev_sms, TXE, BYE, 16);
-    else if (kind == SEIS_ISO) choose_chunks(S, occ, dev_sms, TXV, BYI, 24);
-    else choose_chunks(S, occ, dev_sms, TXV, M->ac_fused ? BYF : BYV, M->ac_fused ? 64 : 16);
+    const int zex = (ns > 1 || M->nranks > 1) ? (M->ac_fused ? 8 : 4) : 0;
+    if (kind == SEIS_ELASTIC) choose_chunks(S, occ, dev_sms, TXE, BYE, 16, zex);
+    else if (kind == SEIS_ISO) choose_chunks(S, occ, dev_sms, TXV, BYI, 24, zex);
+    else choose_chunks(S, occ, dev_sms, TXV, M->ac_fused ? BYF : BYV, M->ac_fused ? 64 : 16,
+                       M->ac_fused ? 8 : zex);  // (the fused step keeps >= 8-plane chunks)
   }
   // f4: the faces between the slabs of this process by direct ghost stores of the producing
   // kernels (SEIS_GHOST_COPY=1 keeps the copy exchange, the A/B alternative).  Not for the

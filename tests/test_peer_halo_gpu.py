@@ -149,3 +149,33 @@ def test_peer_ranks_on_one_gpu_bitwise(kind, P):
                 assert np.array_equal(a, b[z0:z0 + n])
             assert np.array_equal(img, ref[2][z0:z0 + n])
             assert np.array_equal(img2, ref[3][z0:z0 + n])
+
+
+@pytest.mark.parametrize("kind", ["iso", "acoustic", "elastic"])
+def test_short_tail_chunk_decomposition_bitwise(kind, monkeypatch):
+    """Slabs of 65 planes: an even split into >= 8-plane chunks would leave a 2-plane last
+    chunk, so the planes a neighbour needs would straddle an interior chunk.  The chunking
+    keeps >= 4 planes in the first and last chunk of every slab; receivers injected right at
+    the slab face, copy exchange and direct stores, forward + RTM == one slab bitwise."""
+    nx, ny, nz = 48, 36, 130
+    el = kind == "elastic"
+    m = inputs.random_media((nz, ny, nx), seed=33, elastic=el)
+    h, dt, nt, snap = 10.0, 5e-4, 30, 3
+    w = inputs.source_series(kind, nt, dt, 35.0)
+    rec = np.asarray([[10 + t, 7 + (t % 5), 59 + t] for t in range(12)], np.int32)
+    data = np.random.default_rng(6).standard_normal((nt, rec.shape[0])).astype(np.float32)
+    runs = []
+    for P, copy in ((1, "0"), (2, "1"), (2, "0")):
+        monkeypatch.setenv("SEIS_GHOST_COPY", copy)
+        g = seis.Grid(nx, ny, nz, h, dt, nb=5, free_surface=int(el), pml_f=35.0, slabs=P)
+        mod = seis.Model(g, kind, m["vp"], vs=m.get("vs"), rho=m.get("rho"))
+        shot = seis.Shot((nx // 2, ny // 2, 64), w, rec, rec_component=2, snap_period=snap)
+        sg = np.zeros((nt, rec.shape[0]), np.float32)
+        mod.forward_model(shot, sg)
+        img = np.zeros((nz, ny, nx), np.float32)
+        mod.migrate(shot, data, img)
+        runs.append((sg, img))
+        mod.close()
+    for sg, img in runs[1:]:
+        assert np.array_equal(sg, runs[0][0])
+        assert np.array_equal(img, runs[0][1])

@@ -1,0 +1,34 @@
+"""C1 (ISO 64^3, 200 steps; L2-resident, launch-bound) under different z-chunk minimums.
+
+    python tools/c1_sweep.py        # on a B200: one line per SEIS_ZCHUNK_MIN value
+"""
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ONE = r'''
+import json, sys, torch
+sys.path.insert(0, sys.argv[1])
+import paper_conf_ppopp_qawasmehchc15_b200 as seis
+from paper_conf_ppopp_qawasmehchc15_b200 import inputs
+wl = inputs.c1()
+m = seis.Model(seis.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=wl.nb), "iso", wl.model["vp"])
+shot = seis.Shot(wl.src, wl.wavelet, wl.rec)
+buf = torch.empty((wl.nt, shot.nrec), device="cuda")
+for _ in range(3): m.forward_model(shot, buf)
+torch.cuda.synchronize()
+e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+e0.record()
+for _ in range(20): m.forward_model(shot, buf)
+e1.record(); torch.cuda.synchronize()
+ms = e0.elapsed_time(e1) / 20
+print(json.dumps({"ms_per_shot": round(ms, 4), "gpts_s": round(wl.npts * wl.nt / (ms * 1e-3) / 1e9, 2)}))
+'''
+
+for zmin in (8, 4, 2, 1):
+    env = dict(os.environ, SEIS_ZCHUNK_MIN=str(zmin))
+    r = subprocess.run([sys.executable, "-c", ONE, ROOT], env=env, capture_output=True, text=True, timeout=600)
+    out = r.stdout.strip().splitlines()[-1] if r.stdout.strip() else json.dumps({"error": r.stderr[-300:]})
+    print(json.dumps({"zchunk_min": zmin, **json.loads(out)}), flush=True)
