@@ -22,7 +22,8 @@ Gpts/s = grid points x time steps / second (whole job over all ranks).
           sweep, C3 elastic 384^3) and RTM shots/hour (C4, 512^3 salt model, 2000 steps,
           snapshots every 20 steps in HBM).
 N > 1 (torchrun): weak scaling, z-slab decomposition with NCCL halo exchange; each rank
-holds 512^3 points (global nz = 512 N).
+holds 512^3 points (global nz = 512 N).  --scaling strong splits one 512^3 grid instead;
+--halo peer replaces the NCCL send/recv by direct ghost-plane stores over NVLink (f4).
 """
 from __future__ import annotations
 
@@ -150,7 +151,8 @@ def run_product(args):
         dist.init_process_group("nccl", device_id=dev)
         comm = seis.Comm.from_torch_distributed(local)
     n, nt = args.n, args.nt
-    nz = n * ws  # weak scaling: each rank holds n^3 points
+    # weak scaling (default): each rank holds n^3 points; strong: the n^3 grid is split
+    nz = n if args.scaling == "strong" else n * ws
     wl = c2_workload(n=n, nt=nt, nz=nz)
     z0, nzl = seis.slab_bounds(nz, ws, rank)
     grid = seis.Grid(wl.nx, wl.ny, nz, wl.h, wl.dt, nb=wl.nb, pml_R=wl.pml_R, pml_f=wl.fp)
@@ -238,7 +240,7 @@ def run_product(args):
 
     out = {"metric": METRIC, "value": round(value, 3), "unit": "Gpts/s", "n_gpus": ws,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms / args.steps, 3),
-           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+           "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f32",
            "data": "synthetic (seeded layered model, Ricker source)",
            "config": {"workload": f"C2 acoustic {wl.nx}x{wl.ny}x{nz} layered, {nt} steps, C-PML nb={wl.nb}, "
                                   f"{shot.nrec}-receiver line, 1 shot per step",
@@ -439,6 +441,8 @@ def main():
     ap.add_argument("--nt", type=int, default=2000, help="time steps per shot (2000 = C2)")
     ap.add_argument("--ref-steps", type=int, default=1, help="oracle time steps per reference step")
     ap.add_argument("--no-extras", action="store_true")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="N>1: weak = n^3 per rank (default), strong = one n^3 grid split in z-slabs")
     ap.add_argument("--halo", default="nccl", choices=["nccl", "peer"],
                     help="N>1 rank-face ghost exchange: NCCL send/recv overlapped with the interior "
                          "(default) or direct peer stores from the kernels (f4)")
