@@ -107,7 +107,7 @@ struct ElVStage {
 };
 
 template <int BY, bool IMG>
-__global__ void __launch_bounds__(NTX2 * BY, 2) el_v_kernel(const __grid_constant__ ElVArgs a) {
+__global__ void __launch_bounds__(NTX2 * BY, BY <= 8 ? 2 : 1) el_v_kernel(const __grid_constant__ ElVArgs a) {
   using L = ElVStage<BY>;
   constexpr int WX = L::WX, T = L::T;
   constexpr uint32_t TX_BYTES = L::BYTES;
@@ -338,7 +338,7 @@ struct ElSStage {
 };
 
 template <int BY, bool SNAP>
-__global__ void __launch_bounds__(NTX2 * BY, 2) el_s_kernel(const __grid_constant__ ElSArgs a) {
+__global__ void __launch_bounds__(NTX2 * BY, BY <= 8 ? 2 : 1) el_s_kernel(const __grid_constant__ ElSArgs a) {
   using L = ElSStage<BY>;
   constexpr int WX = L::WX, T = L::T, TV = L::TV, RW = L::RW;
   constexpr uint32_t TX_BYTES = L::BYTES;

@@ -19,9 +19,9 @@ sys.path.insert(0, ROOT)
 
 VARIANTS = {
     "base": [],
-    "wr_el": ["SEIS_WR_EL=1"],
-    "wr_all": ["SEIS_WARP_RELEASE=1"],
-    "wr_el_ens3": ["SEIS_WR_EL=1", "SEIS_EL_SNS=3", "SEIS_EL_VNS=3"],
+    "e16": ["SEIS_BYE=16"],
+    "e16_v2": ["SEIS_BYE=16", "SEIS_EL_VNS=2"],
+    "e16_s1": ["SEIS_BYE=16", "SEIS_EL_VNS=2", "SEIS_EL_SNS=1"],
 }
 
 
