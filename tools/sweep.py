@@ -19,9 +19,7 @@ sys.path.insert(0, ROOT)
 
 VARIANTS = {
     "base": [],
-    "e16": ["SEIS_BYE=16"],
-    "e16_v2": ["SEIS_BYE=16", "SEIS_EL_VNS=2"],
-    "e16_s1": ["SEIS_BYE=16", "SEIS_EL_VNS=2", "SEIS_EL_SNS=1"],
+    "iso_rcp": ["SEIS_ISO_RCP=1"],
 }
 
 
