@@ -19,7 +19,6 @@ sys.path.insert(0, ROOT)
 
 VARIANTS = {
     "base": [],
-    "iso_rcp": ["SEIS_ISO_RCP=1"],
 }
 
 

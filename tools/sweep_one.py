@@ -51,4 +51,14 @@ m = seis.Model(seis.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=wl.nb, free_surfac
                "elastic", wl.model["vp"], vs=wl.model["vs"], rho=wl.model["rho"])
 res["c3_384"] = timed(m, seis.Shot(wl.src, wl.wavelet, wl.rec))
 m.close()
+if os.environ.get("SWEEP_NOPML"):  # the same without absorbing layers (cost of the C-PML paths)
+    m = seis.Model(seis.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=0, free_surface=1, pml_f=wl.fp),
+                   "elastic", wl.model["vp"], vs=wl.model["vs"], rho=wl.model["rho"])
+    res["c3_384_nopml"] = timed(m, seis.Shot(wl.src, wl.wavelet, wl.rec))
+    m.close()
+    wl = inputs.c2(n=512, nt=60)
+    m = seis.Model(seis.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=0, pml_f=wl.fp), "acoustic",
+                   wl.model["vp"], rho=wl.model["rho"])
+    res["c2_512_nopml"] = timed(m, seis.Shot(wl.src, wl.wavelet, wl.rec))
+    m.close()
 print(json.dumps(res))
