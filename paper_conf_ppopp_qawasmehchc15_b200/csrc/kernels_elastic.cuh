@@ -566,6 +566,24 @@ __global__ void __launch_bounds__(NTX2 * BY, BY <= 8 ? 2 : 1) el_s_kernel(const 
 // Free-surface ghost planes above k = 0 (O16): for field f with parity `odd`
 // (1: antisymmetric, 0: symmetric) and staggering `half` (1: z-half node),
 //   integer z: ghost(-m) = +-f(m), m = 1..4;   half z: ghost(-1-m) = +-f(m), m = 0..3.
+// One launch for the three fields a phase mirrors (blockIdx.z = field t; bit t of odd / half
+// gives its parity / staggering): 2 launches per elastic step instead of 6.
+__global__ void fs_mirror3_kernel(float* __restrict__ f0, float* __restrict__ f1, float* __restrict__ f2, Dims d,
+                                  int odd_bits, int half_bits) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const int j = blockIdx.y, t = blockIdx.z;
+  if (i >= d.nx) return;
+  float* __restrict__ f = t == 0 ? f0 : (t == 1 ? f1 : f2);
+  const bool half = (half_bits >> t) & 1;
+  const float sgn = ((odd_bits >> t) & 1) ? -1.0f : 1.0f;
+#pragma unroll
+  for (int m = 0; m < 4; ++m) {
+    const int src = half ? m : m + 1;
+    const int dst = half ? -1 - m : -(m + 1);
+    f[d.at(i, j, dst)] = sgn * f[d.at(i, j, src)];
+  }
+}
+
 __global__ void fs_mirror_kernel(float* __restrict__ f, Dims d, int odd, int half) {
   const int i = blockIdx.x * blockDim.x + threadIdx.x;
   const int j = blockIdx.y;

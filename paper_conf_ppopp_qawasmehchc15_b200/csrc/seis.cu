@@ -1419,16 +1419,20 @@ seis_status fs_mirror(seis_model* M, std::initializer_list<int> fields, cudaStre
   if (!M->g.free_surface) return SEIS_OK;
   Slab& S = M->slabs.front();
   if (S.d.z0 != 0) return SEIS_OK;
-  for (int f : fields) {
-    // parity / staggering per field: v even, sigma_zz/xz/yz odd; vz, sxz, syz on half z nodes
-    const int odd = (f == ESZZ || f == ESXZ || f == ESYZ) ? 1 : 0;
-    const int half = (f == EVZ || f == ESXZ || f == ESYZ) ? 1 : 0;
-    {
-      PROF(8, st);
-      fs_mirror_kernel<<<dim3((S.d.nx + 127) / 128, S.d.ny), 128, 0, st>>>(S.fld[f], S.d, odd, half);
-    }
-    CKL();
+  // parity / staggering per field: v even, sigma_zz/xz/yz odd; vz, sxz, syz on half z nodes
+  float* f[3] = {};
+  int odd = 0, half = 0, t = 0;
+  for (int fi : fields) {
+    f[t] = S.fld[fi];
+    if (fi == ESZZ || fi == ESXZ || fi == ESYZ) odd |= 1 << t;
+    if (fi == EVZ || fi == ESXZ || fi == ESYZ) half |= 1 << t;
+    ++t;
   }
+  {
+    PROF(8, st);
+    fs_mirror3_kernel<<<dim3((S.d.nx + 127) / 128, S.d.ny, t), 128, 0, st>>>(f[0], f[1], f[2], S.d, odd, half);
+  }
+  CKL();
   return SEIS_OK;
 }
 
