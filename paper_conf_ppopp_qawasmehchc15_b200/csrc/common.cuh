@@ -345,6 +345,33 @@ __device__ __forceinline__ void psi_ld(float* old, const float* __restrict__ ps,
 #pragma unroll
   for (int e = 0; e < NV; ++e) old[e] = ix[e] >= 0 ? ps[ix[e]] : 0.0f;
 }
+// The x / y C-PML coefficients (a, b, ah, bh) of a block's TW columns and BY rows, staged in
+// shared memory once per block: the z-march uses them on every plane, and a shared load has
+// a short fixed latency where the global (L1) load it replaces sat on the critical path
+// after the stage wait.
+template <int TW, int BY>
+struct CpmlTile {
+  float x[4][TW];
+  float y[4][BY];
+};
+template <int TW, int BY, class Axis>
+__device__ __forceinline__ void cpml_tile_fill(CpmlTile<TW, BY>& t, const Axis& cx, const Axis& cy, int i0,
+                                               int j0, int nx, int ny, bool on, int tid, int nthr) {
+  if (!on) return;
+  for (int q = tid; q < 4 * TW; q += nthr) {
+    const int r = q / TW, c = q - r * TW;
+    const int x = min(i0 + c, nx - 1);
+    const float* p = r == 0 ? cx.a : (r == 1 ? cx.b : (r == 2 ? cx.ah : cx.bh));
+    t.x[r][c] = __ldg(p + x);
+  }
+  for (int q = tid; q < 4 * BY; q += nthr) {
+    const int r = q / BY, c = q - r * BY;
+    const int y = min(j0 + c, ny - 1);
+    const float* p = r == 0 ? cy.a : (r == 1 ? cy.b : (r == 2 ? cy.ah : cy.bh));
+    t.y[r][c] = __ldg(p + y);
+  }
+}
+
 // psi <- b psi + a dv;  dv += psi   (per point coefficients ca[e], cb[e])
 template <int NV>
 __device__ __forceinline__ void psi_upd(float* dv, float* __restrict__ ps, const int* ix, const float* old,

@@ -119,6 +119,7 @@ __global__ void __launch_bounds__(NTX2 * BY, BY <= 8 ? 2 : 1) el_v_kernel(const 
   float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[EL_VNS];
   __shared__ uint32_t cnt[EL_VNS];
+  __shared__ CpmlTile<TXE, BY> ctile;  // x / y C-PML coefficients of this tile
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX2 + tx;
   const int i0 = blockIdx.x * TXE, j0 = blockIdx.y * BY;
@@ -156,6 +157,8 @@ __global__ void __launch_bounds__(NTX2 * BY, BY <= 8 ? 2 : 1) el_v_kernel(const 
     }
     mbar_fence_init();
   }
+  cpml_tile_fill(ctile, a.cx, a.cy, blockIdx.x * TXE, blockIdx.y * BY, a.d.nx, a.d.ny, a.W > 0, tid,
+                 NTX2 * BY);
   __syncthreads();
   if (tid == 0)
     for (int s = 0; s < EL_VNS && s < np; ++s) issue(s, k0 + s);
@@ -237,17 +240,17 @@ __global__ void __launch_bounds__(NTX2 * BY, BY <= 8 ? 2 : 1) el_v_kernel(const 
         float ca[2], cb[2], cah[2], cbh[2];
 #pragma unroll
         for (int e = 0; e < 2; ++e) {
-          const int x = min(x0 + e, d.nx - 1);
-          ca[e] = __ldg(a.cx.a + x); cb[e] = __ldg(a.cx.b + x);
-          cah[e] = __ldg(a.cx.ah + x); cbh[e] = __ldg(a.cx.bh + x);
+          const int c = min(x0 + e, d.nx - 1) - i0;
+          ca[e] = ctile.x[0][c]; cb[e] = ctile.x[1][c];
+          cah[e] = ctile.x[2][c]; cbh[e] = ctile.x[3][c];
         }
         psi_upd<2>(d0, a.psi[0], ixx, ox0, cah, cbh);
         psi_upd<2>(d3, a.psi[3], ixx, ox3, ca, cb);
         psi_upd<2>(d6, a.psi[6], ixx, ox6, ca, cb);
       }
       if (ly) {
-        const float ya = __ldg(a.cy.a + j), yb = __ldg(a.cy.b + j);
-        const float yah = __ldg(a.cy.ah + j), ybh = __ldg(a.cy.bh + j);
+        const float ya = ctile.y[0][ty], yb = ctile.y[1][ty];
+        const float yah = ctile.y[2][ty], ybh = ctile.y[3][ty];
         const float ca[2] = {ya, ya}, cb[2] = {yb, yb}, cah[2] = {yah, yah}, cbh[2] = {ybh, ybh};
         psi_upd<2>(d1, a.psi[1], iyy, oy1, ca, cb);
         psi_upd<2>(d4, a.psi[4], iyy, oy4, cah, cbh);
@@ -348,6 +351,7 @@ __global__ void __launch_bounds__(NTX2 * BY, BY <= 8 ? 2 : 1) el_s_kernel(const 
   float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[EL_SNS];
   __shared__ uint32_t cnt[EL_SNS];
+  __shared__ CpmlTile<TXE, BY> ctile;  // x / y C-PML coefficients of this tile
   const Dims& d = a.d;
   const int tx = threadIdx.x, ty = threadIdx.y, tid = ty * NTX2 + tx;
   const int i0 = blockIdx.x * TXE, j0 = blockIdx.y * BY;
@@ -383,6 +387,8 @@ __global__ void __launch_bounds__(NTX2 * BY, BY <= 8 ? 2 : 1) el_s_kernel(const 
     }
     mbar_fence_init();
   }
+  cpml_tile_fill(ctile, a.cx, a.cy, blockIdx.x * TXE, blockIdx.y * BY, a.d.nx, a.d.ny, a.W > 0, tid,
+                 NTX2 * BY);
   __syncthreads();
   if (tid == 0)
     for (int s = 0; s < EL_SNS && s < np; ++s) issue(s, k0 + s);
@@ -468,17 +474,17 @@ __global__ void __launch_bounds__(NTX2 * BY, BY <= 8 ? 2 : 1) el_s_kernel(const 
         float ca[2], cb[2], cah[2], cbh[2];
 #pragma unroll
         for (int e = 0; e < 2; ++e) {
-          const int x = min(x0 + e, d.nx - 1);
-          ca[e] = __ldg(a.cx.a + x); cb[e] = __ldg(a.cx.b + x);
-          cah[e] = __ldg(a.cx.ah + x); cbh[e] = __ldg(a.cx.bh + x);
+          const int c = min(x0 + e, d.nx - 1) - i0;
+          ca[e] = ctile.x[0][c]; cb[e] = ctile.x[1][c];
+          cah[e] = ctile.x[2][c]; cbh[e] = ctile.x[3][c];
         }
         psi_upd<2>(exx, a.psi[0], ixx, ox0, ca, cb);
         psi_upd<2>(dxvy, a.psi[4], ixx, ox4, cah, cbh);
         psi_upd<2>(dxvz, a.psi[6], ixx, ox6, cah, cbh);
       }
       if (ly) {
-        const float ya = __ldg(a.cy.a + j), yb = __ldg(a.cy.b + j);
-        const float yah = __ldg(a.cy.ah + j), ybh = __ldg(a.cy.bh + j);
+        const float ya = ctile.y[0][ty], yb = ctile.y[1][ty];
+        const float yah = ctile.y[2][ty], ybh = ctile.y[3][ty];
         const float ca[2] = {ya, ya}, cb[2] = {yb, yb}, cah[2] = {yah, yah}, cbh[2] = {ybh, ybh};
         psi_upd<2>(eyy, a.psi[1], iyy, oy1, ca, cb);
         psi_upd<2>(dyvx, a.psi[3], iyy, oy3, cah, cbh);
