@@ -105,6 +105,14 @@ typedef struct {
                                 segment's snapshots from its checkpoint just before they are imaged
                                 (one extra forward pass at most).  Results are bitwise identical to
                                 c = 0 (same kernels, same order of operations). */
+  int32_t snap_fp16;         /* RTM snapshot storage precision (SURVEY §8f f2's "compressed fp16
+                                snapshots"): 0 = fp32 (default); 1 = fp16 scaled per snapshot and
+                                slab by a power of two (max |S_j| near 2^15; relative rounding
+                                2^-11): half the pool (C5 1024^3: all 49 snapshots on one B200
+                                without checkpointing).  The image then differs from the fp32
+                                one by the snapshot rounding (well inside the 1e-3 image bar) and
+                                is no longer bitwise invariant under the z-slab decomposition
+                                (each slab has its own scale). */
 } seis_shot;
 
 /* ---- multi-GPU (one process per GPU; z-slab decomposition, §8e) ---- */

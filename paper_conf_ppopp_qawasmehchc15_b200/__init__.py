@@ -58,7 +58,7 @@ class _CShot(C.Structure):
     _fields_ = [("sx", C.c_int32), ("sy", C.c_int32), ("sz", C.c_int32),
                 ("wavelet", C.POINTER(C.c_float)), ("nt", C.c_int32), ("nrec", C.c_int32),
                 ("rec", C.POINTER(C.c_int32)), ("rec_component", C.c_int32),
-                ("snap_period", C.c_int32), ("ckpt_period", C.c_int32)]
+                ("snap_period", C.c_int32), ("ckpt_period", C.c_int32), ("snap_fp16", C.c_int32)]
 
 
 _lib = None
@@ -136,6 +136,7 @@ class Shot:
     rec_component: int = 2
     snap_period: int = 1
     ckpt_period: int = 0         # RTM: 0 = all snapshots in HBM; c >= 1 = checkpointed segments of c
+    snap_fp16: int = 0           # RTM: 1 = fp16 snapshots scaled by a power of two (half the pool)
 
     def c(self):
         w = np.ascontiguousarray(self.wavelet, dtype=np.float32)
@@ -143,7 +144,7 @@ class Shot:
         cs = _CShot(int(self.src[0]), int(self.src[1]), int(self.src[2]),
                     w.ctypes.data_as(C.POINTER(C.c_float)), w.shape[0], r.shape[0],
                     r.ctypes.data_as(C.POINTER(C.c_int32)), self.rec_component, self.snap_period,
-                    self.ckpt_period)
+                    self.ckpt_period, self.snap_fp16)
         return cs, (w, r)
 
     @property

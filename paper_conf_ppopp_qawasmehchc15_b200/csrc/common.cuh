@@ -17,6 +17,7 @@
 // slab face that touches a neighbour slab are the halo planes the exchange fills.
 #pragma once
 #include <cstdint>
+#include <cuda_fp16.h>
 #include <cuda_runtime.h>
 
 namespace seis {
@@ -276,6 +277,20 @@ __device__ __forceinline__ void st2_masked(float* p, const F2& a, int x0, int nx
     p[0] = a.v[0];
   }
 }
+}  // namespace seis
+
+// ------------------------------------------------------ fp16 snapshots (f2 alternative)
+// Imaging reads S_j either as fp32 (s32) or as fp16 scaled by a power of two (s16 * *scale,
+// the scale written by the snapshot kernel of that level, kernels_aux.cuh).
+namespace seis {
+struct SnapRef {
+  const float* __restrict__ s32 = nullptr;
+  const __half* __restrict__ s16 = nullptr;
+  const float* __restrict__ scale = nullptr;
+  __device__ __forceinline__ float at(long long i) const {
+    return s16 ? __half2float(s16[i]) * __ldg(scale) : __ldg(s32 + i);
+  }
+};
 }  // namespace seis
 
 // ------------------------------------------------------ direct ghost-plane stores

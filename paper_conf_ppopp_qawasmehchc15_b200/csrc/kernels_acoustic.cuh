@@ -57,6 +57,7 @@ struct AcVArgs {
   int zc;
   int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   const float* __restrict__ imgS; // imaging: img += S * p (input level), or nullptr
+  SnapRef imgR;                   // the same (fp32 or fp16), what the IMG kernel reads
   float* __restrict__ img;
   Ghost gh;                       // direct ghost stores of q_z (f4)
 };
@@ -228,7 +229,7 @@ __global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ 
         F4 im;
 #pragma unroll
         for (int e = 0; e < 4; ++e)
-          im.v[e] = (x0 + e < d.nx) ? fmaf(__ldg(a.imgS + cix + e), r[3].v[e], a.img[cix + e]) : 0.f;
+          im.v[e] = (x0 + e < d.nx) ? fmaf(a.imgR.at(cix + e), r[3].v[e], a.img[cix + e]) : 0.f;
         st4_masked(a.img + cix, im, x0, d.nx, false);
       }
     }

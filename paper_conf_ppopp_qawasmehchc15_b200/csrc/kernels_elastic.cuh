@@ -92,6 +92,7 @@ struct ElVArgs {
   int zc;
   int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   const float* __restrict__ imgS;  // elastic RTM (f3): img += S * P on the input level, P = -(sxx+syy+szz)/3
+  SnapRef imgR;                    // the same (fp32 or fp16), what the IMG kernel reads
   float* __restrict__ img;
   Ghost gh[3];                     // direct ghost stores of vx, vy, vz (f4)
 };
@@ -294,7 +295,7 @@ __global__ void __launch_bounds__(NTX2 * BY, BY <= 8 ? 2 : 1) el_v_kernel(const 
         for (int e = 0; e < 2; ++e)
           if (x0 + e < d.nx) {
             const float pr = -((xs[4 + e] + yyy[e][4]) + qzz[3].v[e]) / 3.0f;
-            a.img[cix + e] = fmaf(__ldg(a.imgS + cix + e), pr, a.img[cix + e]);
+            a.img[cix + e] = fmaf(a.imgR.at(cix + e), pr, a.img[cix + e]);
           }
       }
     }

@@ -37,6 +37,7 @@ struct IsoArgs {
   float src_amp;                 // scale * s[n]
   float* __restrict__ snap;      // compact [nzl][ny][nx] or nullptr
   const float* __restrict__ imgS;// compact snapshot S_j for imaging, or nullptr
+  SnapRef imgR;                  // the same (fp32 or fp16), what the IMG kernels read
   float* __restrict__ img;       // compact image (+=), or nullptr
   Ghost gh;                      // direct ghost stores of u^{n+1} (f4)
   // split-field PML (O6b, SPML kernels): components u^(x), u^(y), u^(z) of the layer points,
@@ -297,7 +298,7 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
           F4 im;
 #pragma unroll
           for (int e = 0; e < 4; ++e)
-            im.v[e] = (x0 + e < d.nx) ? fmaf(__ldg(a.imgS + cix + e), q[4].v[e], a.img[cix + e]) : 0.f;
+            im.v[e] = (x0 + e < d.nx) ? fmaf(a.imgR.at(cix + e), q[4].v[e], a.img[cix + e]) : 0.f;
           st4_masked(a.img + cix, im, x0, d.nx, false);
         }
       }

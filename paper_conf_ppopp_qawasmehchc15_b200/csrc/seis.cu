@@ -208,6 +208,8 @@ struct seis_model {
   // staging buffers
   float* stage = nullptr;
   size_t stage_elems = 0;
+  float* scales = nullptr;  // fp16 snapshot scales + max words (seis_shot.snap_fp16)
+  size_t scales_elems = 0;
   const float* hwav = nullptr;  // host wavelet of the current call
   int last_nt = 0;
   // shot-table cache and the CUDA graph of the last forward_model (single process)
@@ -1198,7 +1200,7 @@ seis_status seis_memory_required(const seis_grid* g, seis_kind kind, const seis_
             (kind == SEIS_ACOUSTIC ? 2 : 6);
     }
     ck += spml;
-    b += (double)c * nzl * (double)g->ny * g->nx * 4.0 + (double)nckpt * ck;
+    b += (double)c * nzl * (double)g->ny * g->nx * (shot->snap_fp16 == 1 ? 2.0 : 4.0) + (double)nckpt * ck;
   }
   *bytes = (uint64_t)b;
   return SEIS_OK;
@@ -1525,7 +1527,7 @@ seis_status run_phase(seis_model* M, const LaunchFn& launch, const PostFn& post,
 //   snap: compact snapshot target per slab (or null), imgS/img: imaging of the INPUT level,
 //   inj_row: receiver samples injected into the produced field (backward phase) or null
 seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
-                 std::vector<const float*>* imgS, std::vector<float*>* img, cudaStream_t st,
+                 std::vector<SnapRef>* imgS, std::vector<float*>* img, cudaStream_t st,
                  const float* inj_row = nullptr) {
   auto inject = [&](int part, cudaStream_t s2) -> seis_status {
     return inj_row ? inject_rows(M, inj_row, part, s2) : SEIS_OK;
@@ -1552,7 +1554,8 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.src_amp = 0.f;
       if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
       a.snap = snap ? (*snap)[s] : nullptr;
-      a.imgS = imgS ? (*imgS)[s] : nullptr;
+      a.imgS = imgS ? (*imgS)[s].s32 : nullptr;
+      if (imgS) a.imgR = (*imgS)[s];
       a.img = img ? (*img)[s] : nullptr;
       a.gh = S.gh[1 - cur];
       a.sp = S.sp;
@@ -1634,7 +1637,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.src_amp = 0.f;
       if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
       a.snap = snap ? (*snap)[s] : nullptr;
-      a.imgS = imgS ? (*imgS)[s] : nullptr;
+      a.imgS = imgS ? (*imgS)[s].s32 : nullptr;
       a.img = img ? (*img)[s] : nullptr;
       const dim3 gr = grid_of(S, TXV, BYF, nch), blk(NTX, BYF);
       {
@@ -1687,7 +1690,8 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.zc = S.zc;
       a.ch0 = ch0;
       a.chs = chs;
-      a.imgS = imgS ? (*imgS)[s] : nullptr;
+      a.imgS = imgS ? (*imgS)[s].s32 : nullptr;
+      if (imgS) a.imgR = (*imgS)[s];
       a.img = img ? (*img)[s] : nullptr;
       a.gh = S.gh[3];
       const dim3 gr = grid_of(S, TXV, BYV, nch), blk(NTX, BYV);
@@ -1777,7 +1781,8 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     a.zc = S.zc;
     a.ch0 = ch0;
     a.chs = chs;
-    a.imgS = imgS ? (*imgS)[s] : nullptr;
+    a.imgS = imgS ? (*imgS)[s].s32 : nullptr;
+    if (imgS) a.imgR = (*imgS)[s];
     a.img = img ? (*img)[s] : nullptr;
     for (int t = 0; t < 3; ++t) a.gh[t] = S.gh[EVX + t];
     const dim3 gr = grid_of(S, TXE, BYE, nch);
@@ -1860,6 +1865,15 @@ seis_status gather(seis_model* M, const seis_shot* sh, float* seis_dev, int n, c
         S.d_rec_off, S.d_rec_id, S.nrec_own, pres);
     CKL();
   }
+  return SEIS_OK;
+}
+
+seis_status ensure_scales(seis_model* M, size_t elems) {
+  if (M->scales_elems >= elems) return SEIS_OK;
+  void* p = nullptr;
+  TRY(alloc_track(M, &p, elems * sizeof(float)));
+  M->scales = (float*)p;
+  M->scales_elems = elems;
   return SEIS_OK;
 }
 
@@ -1969,7 +1983,12 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
   const int nckpt = nseg > 1 ? nseg - 1 : 0;
   const size_t slab_pts = (size_t)M->pnzl * g.ny * g.nx;
   const size_t st_elems = nckpt ? state_elems(M) : 0;
-  const size_t snap_elems = (size_t)std::min(c, nsnap) * slab_pts;
+  if (sh->snap_fp16 != 0 && sh->snap_fp16 != 1) return fail(SEIS_EINVAL, "snap_fp16 must be 0 or 1");
+  const bool f16 = sh->snap_fp16 == 1;
+  if (f16 && M->ac_fused) return fail(SEIS_EUNSUPPORTED, "fp16 snapshots with the fused acoustic step");
+  const size_t esz = f16 ? 2 : 4;  // bytes per snapshot value
+  // (pool floats of the snapshot region, 256-byte aligned so the checkpoints stay aligned)
+  const size_t snap_elems = ((size_t)std::min(c, nsnap) * slab_pts * esz + 255) / 256 * 64;
   const size_t need = snap_elems + (size_t)nckpt * st_elems;
   if (need > M->pool_elems) {
     size_t freeb = 0, totb = 0;
@@ -1995,10 +2014,38 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
   auto slot_of = [&](int q) { return ckpt0 + (size_t)q * st_elems; };
   std::vector<int> ckpt_cur(nckpt, 0);  // ISO: which buffer holds u^n at the checkpoint
   // pool pointers of snapshot index i (j = (i + 1) snap), which lives in segment i / c
-  auto snap_ptrs = [&](int i, std::vector<float*>& v) {
+  auto snap_ptrs = [&](int i, std::vector<float*>& v) {  // (byte addresses for fp16)
     const size_t off = (size_t)(i % c) * slab_pts;
     for (size_t s = 0; s < M->slabs.size(); ++s)
-      v[s] = M->pool + off + (size_t)(M->slabs[s].d.z0 - M->pz0) * g.ny * g.nx;
+      v[s] = (float*)((char*)M->pool + (off + (size_t)(M->slabs[s].d.z0 - M->pz0) * g.ny * g.nx) * esz);
+  };
+  // fp16: one power-of-two scale per (snapshot, slab) and one max word per slab
+  const size_t nsl = M->slabs.size();
+  float* scales = nullptr;
+  unsigned* amax = nullptr;
+  if (f16 && nsnap > 0) {
+    TRY(ensure_scales(M, (size_t)nsnap * nsl + nsl));
+    scales = M->scales;
+    amax = (unsigned*)(M->scales + (size_t)nsnap * nsl);
+  }
+  // store snapshot i (level (i + 1) snap) of the current state as fp16
+  auto snap16 = [&](int i) -> seis_status {
+    std::vector<float*> dst(nsl);
+    snap_ptrs(i, dst);
+    CK(cudaMemsetAsync(amax, 0, nsl * sizeof(unsigned), st));
+    for (size_t s = 0; s < nsl; ++s) {
+      Slab& S = M->slabs[s];
+      const float* f0 = M->kind == SEIS_ELASTIC ? S.fld[ESXX] : out_field(M, S, 0);
+      const float* f1 = M->kind == SEIS_ELASTIC ? S.fld[ESYY] : f0;
+      const float* f2 = M->kind == SEIS_ELASTIC ? S.fld[ESZZ] : f0;
+      const int nf = M->kind == SEIS_ELASTIC ? 3 : 1;
+      snap_amax_kernel<<<4 * 148, 256, 0, st>>>(amax + s, f0, f1, f2, nf, S.d);
+      CKL();
+      snap_f16_kernel<<<8 * 148, 256, 0, st>>>((__half*)dst[s], scales + (size_t)i * nsl + s, amax + s, f0, f1, f2,
+                                              nf, S.d);
+      CKL();
+    }
+    return SEIS_OK;
   };
   // image / data staging
   const bool img_dev = is_device_ptr(image);
@@ -2030,8 +2077,9 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
       const int j = n + 1;
       bool take = (j % snap == 0) && j <= nt - 1;
       if (take && (j / snap - 1) / c != seg) take = false;
-      if (take) snap_ptrs(j / snap - 1, snapp);
-      TRY(step(M, n, true, take ? &snapp : nullptr, nullptr, nullptr, st));
+      if (take && !f16) snap_ptrs(j / snap - 1, snapp);
+      TRY(step(M, n, true, take && !f16 ? &snapp : nullptr, nullptr, nullptr, st));
+      if (take && f16) TRY(snap16(j / snap - 1));
     }
     return SEIS_OK;
   };
@@ -2042,7 +2090,7 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
   // ---- backward phase: receiver wavefield from zero, same operator
   TRY(setup_shot(M, sh, true, st));
   TRY(zero_state(M, st));
-  std::vector<const float*> Sp(M->slabs.size());
+  std::vector<SnapRef> Sp(M->slabs.size());
   std::vector<float*> Ip(M->slabs.size()), tmp(M->slabs.size());
   for (size_t s = 0; s < M->slabs.size(); ++s)
     Ip[s] = img_d + (size_t)(M->slabs[s].d.z0 - M->pz0) * g.ny * g.nx;
@@ -2072,7 +2120,15 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
         loaded = seg;
       }
       snap_ptrs(i, tmp);
-      for (size_t s = 0; s < M->slabs.size(); ++s) Sp[s] = tmp[s];
+      for (size_t s = 0; s < M->slabs.size(); ++s) {
+        Sp[s] = SnapRef{};
+        if (f16) {
+          Sp[s].s16 = (const __half*)tmp[s];
+          Sp[s].scale = scales + (size_t)i * nsl + s;
+        } else {
+          Sp[s].s32 = tmp[s];
+        }
+      }
     }
     // step + receiver injection of data[nt-1-m] (all receivers, one launch per slab)
     TRY(step(M, m, false, nullptr, im ? &Sp : nullptr, im ? &Ip : nullptr, st,
