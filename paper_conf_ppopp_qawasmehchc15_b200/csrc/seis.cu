@@ -676,6 +676,18 @@ seis_status seis_model_destroy(seis_model* M) {
   if (M->ev_fork) cudaEventDestroy(M->ev_fork);
   if (M->ev_join) cudaEventDestroy(M->ev_join);
   for (void* p : M->ipc_open) cudaIpcCloseMemHandle(p);
+  for (Slab& S : M->slabs) {  // shot tables (setup_shot), not in allocs
+    cudaFree(S.d_rec_off);
+    cudaFree(S.d_rec_id);
+    for (auto& G2 : S.grp) {
+      cudaFree(G2.off);
+      cudaFree(G2.scale);
+      cudaFree(G2.start);
+      cudaFree(G2.mem);
+      cudaFree(G2.surf);
+      cudaFree(G2.sidx);
+    }
+  }
   for (void* p : M->allocs) cudaFree(p);
   delete M;
   return SEIS_OK;
