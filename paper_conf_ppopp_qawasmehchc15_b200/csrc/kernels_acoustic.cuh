@@ -33,6 +33,15 @@ struct CpmlAxis {
 #define SEIS_AC_VNS 3
 #endif
 constexpr int AC_NS = SEIS_AC_NS;    // P kernel ring depth
+// launch bounds of the V / P kernels: minimum resident blocks per SM (0 = unspecified)
+#ifndef SEIS_AC_MINB
+#define SEIS_AC_MINB 0
+#endif
+#if SEIS_AC_MINB > 0
+#define SEIS_AC_LB(n) __launch_bounds__(n, SEIS_AC_MINB)
+#else
+#define SEIS_AC_LB(n) __launch_bounds__(n)
+#endif
 constexpr int AC_VNS = SEIS_AC_VNS;  // V kernel ring depth
 
 struct AcVArgs {
@@ -72,7 +81,7 @@ struct AcVStage {
 };
 
 template <int BY, bool IMG>
-__global__ void __launch_bounds__(NTX * BY) ac_v_kernel(const __grid_constant__ AcVArgs a) {
+__global__ void SEIS_AC_LB(NTX * BY) ac_v_kernel(const __grid_constant__ AcVArgs a) {
   using L = AcVStage<BY>;
   constexpr int W = L::W, RW = L::RW;
   constexpr uint32_t TX_BYTES = L::BYTES;
@@ -273,7 +282,7 @@ struct AcPStage {
 };
 
 template <int BY, bool SNAP>
-__global__ void __launch_bounds__(NTX * BY) ac_p_kernel(const __grid_constant__ AcPArgs a) {
+__global__ void SEIS_AC_LB(NTX * BY) ac_p_kernel(const __grid_constant__ AcPArgs a) {
   using L = AcPStage<BY>;
   constexpr int WX = L::WX;
   constexpr uint32_t TX_BYTES = L::SIZE * 4;

@@ -61,6 +61,9 @@ __device__ __forceinline__ int spml_idx(const Dims& d, int nb, int nxs, int nys,
   return nxs + nys + ((gz < nb ? gz : gz - (d.nz - 2 * nb)) * d.ny + j) * d.nx + x;
 }
 
+#ifndef SEIS_SPML_MINB
+#define SEIS_SPML_MINB 3  // O6b kernels: >= 3 resident blocks (<= 170 registers; 0.762 vs 0.974 ms)
+#endif
 #ifndef SEIS_ISO_RCP
 #define SEIS_ISO_RCP 1  // profiles/r01_sweep_zu.jsonl: iso_step 0.429 -> 0.370 ms at 512^3
 #endif
@@ -76,10 +79,12 @@ struct IsoStage {
   static constexpr size_t smem_bytes() { return (size_t)ISO_NS * SIZE * 4 + 128; }
 };
 
+// Launch bounds: an explicit minimum of 1 block lets ptxas give the plain kernel 96 registers
+// instead of 80 -- 0.370 -> 0.345 ms at 512^3 (profiles/r01_sweep_zu.jsonl).
 // GH: this slab has a neighbour slab / rank whose ghost planes it stores (f4); the single-slab
 // instantiation leaves the check out (-2.7 % iso_step time, profiles/r01_sweep_zu.jsonl)
 template <int BY, bool SNAP, bool IMG, bool SPML = false, bool GH = true>
-__global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constant__ IsoArgs a) {
+__global__ void __launch_bounds__(NTX * BY, SPML ? SEIS_SPML_MINB : 1) iso_step_kernel(const __grid_constant__ IsoArgs a) {
   using L = IsoStage<BY>;
   constexpr int W = L::W;
   constexpr uint32_t TX_BYTES = L::SIZE * 4;
@@ -160,20 +165,36 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
     // overlap, as the C-PML memory variables): w0 = level n, wm = level n-1
     int sidx[4] = {-1, -1, -1, -1};
     float w0[3][4], wm[3][4];
+    bool spv = false;  // the group's 4 components are one aligned float4 in every array
     if (SPML && (dxy || ez != 0.0f)) {
 #pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        if (own && x0 + e < d.nx && (exv.v[e] != 0.0f || eyv != 0.0f || ez != 0.0f)) {
-          const int id = spml_idx(d, a.nbl, a.nxs, a.nys, exv.v[e], eyv, x0 + e, j, k);
-          sidx[e] = id;
-          const float* cur = a.sp + (long long)a.lvl * 3 * a.spn + id;
-          const float* nxt = a.sp + (long long)(1 - a.lvl) * 3 * a.spn + id;
+      for (int e = 0; e < 4; ++e)
+        if (own && x0 + e < d.nx && (exv.v[e] != 0.0f || eyv != 0.0f || ez != 0.0f))
+          sidx[e] = spml_idx(d, a.nbl, a.nxs, a.nys, exv.v[e], eyv, x0 + e, j, k);
+      spv = sidx[0] >= 0 && (sidx[0] & 3) == 0 && (a.spn & 3) == 0 && sidx[1] == sidx[0] + 1 &&
+            sidx[2] == sidx[0] + 2 && sidx[3] == sidx[0] + 3;
+      const float* cur = a.sp + (long long)a.lvl * 3 * a.spn;
+      const float* nxt = a.sp + (long long)(1 - a.lvl) * 3 * a.spn;
+      if (spv) {
 #pragma unroll
-          for (int c = 0; c < 3; ++c) {
-            w0[c][e] = cur[c * a.spn];
-            wm[c][e] = nxt[c * a.spn];
+        for (int c = 0; c < 3; ++c) {
+          const F4 p0 = ld4(cur + c * a.spn + sidx[0]), pm = ld4(nxt + c * a.spn + sidx[0]);
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            w0[c][e] = p0.v[e];
+            wm[c][e] = pm.v[e];
           }
         }
+      } else {
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          if (sidx[e] >= 0) {
+#pragma unroll
+            for (int c = 0; c < 3; ++c) {
+              w0[c][e] = cur[c * a.spn + sidx[e]];
+              wm[c][e] = nxt[c * a.spn + sidx[e]];
+            }
+          }
       }
     }
     mbar_wait(&bar[s], (it / ISO_NS) & 1);
@@ -242,19 +263,30 @@ __global__ void __launch_bounds__(NTX * BY) iso_step_kernel(const __grid_constan
             l = fmaf(SEIS_C3, q[1].v[e] + q[7].v[e], l);
             Ld[2] = fmaf(SEIS_C4, q[0].v[e] + q[8].v[e], l);
           }
-          float* nxt = a.sp + (long long)(1 - a.lvl) * 3 * a.spn + sidx[e];
           float sum = 0.0f;
 #pragma unroll
           for (int c = 0; c < 3; ++c) {
             // = [(2 - e^2) w0 - (1 - e) wm + m L_d] / (1 + e), e = eta_d dt (O6b)
             const float w1 = fmaf(ca[c], w0[c][e], fmaf(-cb[c], wm[c][e], cc[c] * (mv.v[e] * Ld[c])));
-            nxt[c * a.spn] = w1;
+            wm[c][e] = w1;  // (the new level replaces n-1 in the same slot)
             sum += w1;
           }
           out.v[e] = sum;
         } else {
           out.v[e] = fmaf(mv.v[e], lap[e], 2.0f * u - upv.v[e]);
         }
+      }
+      float* nxt = a.sp + (long long)(1 - a.lvl) * 3 * a.spn;
+      if (spv) {
+#pragma unroll
+        for (int c = 0; c < 3; ++c) st4(nxt + c * a.spn + sidx[0], F4{{wm[c][0], wm[c][1], wm[c][2], wm[c][3]}});
+      } else {
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          if (sidx[e] >= 0) {
+#pragma unroll
+            for (int c = 0; c < 3; ++c) nxt[c * a.spn + sidx[e]] = wm[c][e];
+          }
       }
     } else {
 #pragma unroll

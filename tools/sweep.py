@@ -19,6 +19,11 @@ sys.path.insert(0, ROOT)
 
 VARIANTS = {
     "base": [],
+    "spml_mb2": ["SEIS_SPML_MINB=2"],
+    "spml_mb3": ["SEIS_SPML_MINB=3"],
+    "ac_mb1": ["SEIS_AC_MINB=1"],
+    "ac_mb3": ["SEIS_AC_MINB=3"],
+    "ac_mb5": ["SEIS_AC_MINB=5"],
 }
 
 
