@@ -187,8 +187,12 @@ seis_status seis_model_peer_import(seis_model* model, const uint8_t* lo_blob, ui
 /* ---- the hot path ---- */
 /* Seismic modeling of one shot from a zero state (Alg 1 forward phase).
  *   seis  host or device [nt][nrec] fp32, written in full: seis[n][r] = field^{n+1}(x_r) (O13).
- *         With comm != NULL every rank receives the full array (NCCL all-reduce of the
- *         rank-owned entries; exact because exactly one rank owns each receiver). */
+ *         With an NCCL communicator every rank receives the full array (NCCL all-reduce of
+ *         the rank-owned entries; exact because exactly one rank owns each receiver); with a
+ *         peer-only communicator (seis_comm_create_peer) each rank's array holds its own
+ *         receivers' columns and zeros elsewhere (the caller sums them).
+ * With peer halos (seis_model_peer_import) the call is collective over the neighbouring
+ * ranks, like every call that steps the wavefield. */
 seis_status seis_forward_model(seis_model* model, const seis_shot* shot, float* seis,
                                void* stream);
 /* Reverse-time migration of one shot.  ISO images u, ACOUSTIC p, ELASTIC the pressure
