@@ -70,6 +70,9 @@ __device__ __forceinline__ void ycol(float (*yv)[9], const float* c) {
 #ifndef SEIS_EL_SNS
 #define SEIS_EL_SNS 2
 #endif
+#ifndef SEIS_EL_MINB
+#define SEIS_EL_MINB 0  // launch-bounds minimum blocks per SM (0: 2 for BY <= 8, else 1)
+#endif
 constexpr int EL_VNS = SEIS_EL_VNS;
 constexpr int EL_SNS = SEIS_EL_SNS;
 
@@ -108,7 +111,7 @@ struct ElVStage {
 };
 
 template <int BY, bool IMG>
-__global__ void __launch_bounds__(NTX2 * BY, BY <= 8 ? 2 : 1) el_v_kernel(const __grid_constant__ ElVArgs a) {
+__global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (BY <= 8 ? 2 : 1)) el_v_kernel(const __grid_constant__ ElVArgs a) {
   using L = ElVStage<BY>;
   constexpr int WX = L::WX, T = L::T;
   constexpr uint32_t TX_BYTES = L::BYTES;
@@ -342,7 +345,7 @@ struct ElSStage {
 };
 
 template <int BY, bool SNAP>
-__global__ void __launch_bounds__(NTX2 * BY, BY <= 8 ? 2 : 1) el_s_kernel(const __grid_constant__ ElSArgs a) {
+__global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (BY <= 8 ? 2 : 1)) el_s_kernel(const __grid_constant__ ElSArgs a) {
   using L = ElSStage<BY>;
   constexpr int WX = L::WX, T = L::T, TV = L::TV, RW = L::RW;
   constexpr uint32_t TX_BYTES = L::BYTES;

@@ -19,11 +19,9 @@ sys.path.insert(0, ROOT)
 
 VARIANTS = {
     "base": [],
-    "spml_mb2": ["SEIS_SPML_MINB=2"],
-    "spml_mb3": ["SEIS_SPML_MINB=3"],
-    "ac_mb1": ["SEIS_AC_MINB=1"],
-    "ac_mb3": ["SEIS_AC_MINB=3"],
-    "ac_mb5": ["SEIS_AC_MINB=5"],
+    "e4_mb4_v2": ["SEIS_BYE=4", "SEIS_EL_MINB=4", "SEIS_EL_VNS=2"],
+    "e4_mb4_v3": ["SEIS_BYE=4", "SEIS_EL_MINB=4", "SEIS_EL_VNS=3"],
+    "e4_mb3_v3": ["SEIS_BYE=4", "SEIS_EL_MINB=3", "SEIS_EL_VNS=3"],
 }
 
 
