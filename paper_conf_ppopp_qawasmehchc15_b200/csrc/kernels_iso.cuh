@@ -18,7 +18,35 @@
 #pragma once
 #include "common.cuh"
 
+#ifndef SEIS_ISO_RCP
+#define SEIS_ISO_RCP 1  // profiles/r01_sweep_zu.jsonl: iso_step 0.429 -> 0.370 ms at 512^3
+#endif
+
 namespace seis {
+
+// Eq 1 / O3 per point, shared by the z-march kernel and the persistent small-grid kernel so
+// both contract and round identically (bitwise equal results):
+// 25-point Laplacian x h^2 of O1 from the ring pair sums xs[m], ys[m], zs[m] (m = 1..4) ...
+__device__ __forceinline__ float iso_lap(float u, const float* xs, const float* ys, const float* zs) {
+  float l = (3.0f * SEIS_C0) * u;
+  l = fmaf(SEIS_C1, (xs[0] + ys[0]) + zs[0], l);
+  l = fmaf(SEIS_C2, (xs[1] + ys[1]) + zs[1], l);
+  l = fmaf(SEIS_C3, (xs[2] + ys[2]) + zs[2], l);
+  return fmaf(SEIS_C4, (xs[3] + ys[3]) + zs[3], l);
+}
+// ... and the leapfrog update with the damped-wave layer (eta = eta dt; 0 outside)
+__device__ __forceinline__ float iso_update(float u, float up, float m, float lap, float eta) {
+  if (eta == 0.0f) return fmaf(m, lap, 2.0f * u - up);
+#if SEIS_ISO_RCP
+  // MUFU reciprocal + one Newton step (~0.5 ulp) instead of the IEEE division
+  const float den = 1.0f + eta;
+  float inv = rcp_fast(den);
+  inv = fmaf(inv, fmaf(-den, inv, 1.0f), inv);
+  return (2.0f * u - (1.0f - eta) * up + m * lap) * inv;
+#else
+  return (2.0f * u - (1.0f - eta) * up + m * lap) / (1.0f + eta);
+#endif
+}
 
 struct IsoArgs {
   CUtensorMap mun;               // u^n tile, box (64+8) x (BY+8) x 1
@@ -63,9 +91,6 @@ __device__ __forceinline__ int spml_idx(const Dims& d, int nb, int nxs, int nys,
 
 #ifndef SEIS_SPML_MINB
 #define SEIS_SPML_MINB 3  // O6b kernels: >= 3 resident blocks (<= 170 registers; 0.762 vs 0.974 ms)
-#endif
-#ifndef SEIS_ISO_RCP
-#define SEIS_ISO_RCP 1  // profiles/r01_sweep_zu.jsonl: iso_step 0.429 -> 0.370 ms at 512^3
 #endif
 #ifndef SEIS_ISO_NS
 #define SEIS_ISO_NS 3
@@ -224,16 +249,19 @@ __global__ void __launch_bounds__(NTX * BY, SPML ? SEIS_SPML_MINB : 1) iso_step_
     float lap[4];
 #pragma unroll
     for (int e = 0; e < 4; ++e) {
-      float l = (3.0f * SEIS_C0) * xv[4 + e];
-      l = fmaf(SEIS_C1, (xv[3 + e] + xv[5 + e]) + ys[0].v[e] + (q[3].v[e] + q[5].v[e]), l);
-      l = fmaf(SEIS_C2, (xv[2 + e] + xv[6 + e]) + ys[1].v[e] + (q[2].v[e] + q[6].v[e]), l);
-      l = fmaf(SEIS_C3, (xv[1 + e] + xv[7 + e]) + ys[2].v[e] + (q[1].v[e] + q[7].v[e]), l);
-      lap[e] = fmaf(SEIS_C4, (xv[0 + e] + xv[8 + e]) + ys[3].v[e] + (q[0].v[e] + q[8].v[e]), l);
+      float xs[4], yss[4], zs[4];
+#pragma unroll
+      for (int m = 0; m < 4; ++m) {
+        xs[m] = xv[3 - m + e] + xv[5 + m + e];
+        yss[m] = ys[m].v[e];
+        zs[m] = q[3 - m].v[e] + q[5 + m].v[e];
+      }
+      lap[e] = iso_lap(xv[4 + e], xs, yss, zs);
     }
     F4 out;
     if (!damp) {  // block-uniform branch
 #pragma unroll
-      for (int e = 0; e < 4; ++e) out.v[e] = fmaf(mv.v[e], lap[e], 2.0f * xv[4 + e] - upv.v[e]);
+      for (int e = 0; e < 4; ++e) out.v[e] = iso_update(xv[4 + e], upv.v[e], mv.v[e], lap[e], 0.0f);
     } else if (SPML) {
       // O6b: layer points advance u^(x), u^(y), u^(z), each damped along its own axis with the
       // 1D part L_d of the Laplacian; u^{n+1} is their sum.  Other points: Eq 1.
@@ -273,7 +301,7 @@ __global__ void __launch_bounds__(NTX * BY, SPML ? SEIS_SPML_MINB : 1) iso_step_
           }
           out.v[e] = sum;
         } else {
-          out.v[e] = fmaf(mv.v[e], lap[e], 2.0f * u - upv.v[e]);
+          out.v[e] = iso_update(u, upv.v[e], mv.v[e], lap[e], 0.0f);
         }
       }
       float* nxt = a.sp + (long long)(1 - a.lvl) * 3 * a.spn;
@@ -291,23 +319,7 @@ __global__ void __launch_bounds__(NTX * BY, SPML ? SEIS_SPML_MINB : 1) iso_step_
     } else {
 #pragma unroll
       for (int e = 0; e < 4; ++e) {
-        const float u = xv[4 + e];
-        const float eta = exy.v[e] + ez;
-        float r;
-        if (eta != 0.0f) {
-#if SEIS_ISO_RCP
-          // MUFU reciprocal + one Newton step (~0.5 ulp) instead of the IEEE division
-          const float den = 1.0f + eta;
-          float inv = rcp_fast(den);
-          inv = fmaf(inv, fmaf(-den, inv, 1.0f), inv);
-          r = (2.0f * u - (1.0f - eta) * upv.v[e] + mv.v[e] * lap[e]) * inv;
-#else
-          r = (2.0f * u - (1.0f - eta) * upv.v[e] + mv.v[e] * lap[e]) / (1.0f + eta);
-#endif
-        } else {
-          r = fmaf(mv.v[e], lap[e], 2.0f * u - upv.v[e]);
-        }
-        out.v[e] = r;
+        out.v[e] = iso_update(xv[4 + e], upv.v[e], mv.v[e], lap[e], exy.v[e] + ez);
       }
     }
     if (own) {
@@ -341,6 +353,108 @@ __global__ void __launch_bounds__(NTX * BY, SPML ? SEIS_SPML_MINB : 1) iso_step_
     });
 #pragma unroll
     for (int t = 0; t < 8; ++t) q[t] = q[t + 1];
+  }
+}
+
+}  // namespace seis
+
+// ------------------------------------------------------------------ small grids
+// Persistent ISO modeling for L2-resident grids (C1, 64^3): the whole shot is ONE cooperative
+// launch; every block owns fixed 4-point x-groups of the slab, and a grid-wide barrier
+// separates the time steps (instead of two kernel launches per step: the grid is too small to
+// hide launch gaps).  Per point it evaluates exactly the z-march kernel's expressions
+// (iso_lap, iso_update, then the source add), so the results are bitwise the same.  Receiver
+// gather of level n+1 (seis[n]) happens at the top of step n+1 (block 0 reads the input level,
+// which that step does not write) and once after the last step.
+#include <cooperative_groups.h>
+
+namespace seis {
+
+struct IsoPArgs {
+  float* u0;                       // fld[0] / fld[1]: level n is u[cur], u^{n-1} / u^{n+1} u[1-cur]
+  float* u1;
+  const float* __restrict__ m;
+  const float* __restrict__ edx;   // eta dt per axis (nullptr: no layer)
+  const float* __restrict__ edy;
+  const float* __restrict__ edz;
+  Dims d;
+  int nt, cur0;
+  long long src_o;                 // padded source index (-1: none)
+  const float* __restrict__ amp;   // device [nt]: src_scale * s[n] (the host float product)
+  float* __restrict__ seis;        // [nt][nrec_tot]
+  const long long* __restrict__ rec_off;
+  const int* __restrict__ rec_id;
+  int nrec, nrec_tot;
+};
+
+__global__ void __launch_bounds__(128) iso_persist_kernel(const __grid_constant__ IsoPArgs a) {
+  namespace cg = cooperative_groups;
+  cg::grid_group grid = cg::this_grid();
+  const Dims& d = a.d;
+  const int gx = (d.nx + 3) / 4;
+  const long long ngroups = (long long)gx * d.ny * d.nzl;
+  const long long PS = d.PS;
+  int cur = a.cur0;
+  for (int n = 0; n <= a.nt; ++n) {
+    const float* __restrict__ un = cur ? a.u1 : a.u0;
+    float* __restrict__ up = cur ? a.u0 : a.u1;
+    if (n > 0 && blockIdx.x == 0)  // receivers of level n = seis[n - 1] (gather_kernel's rule)
+      for (int r = threadIdx.x; r < a.nrec; r += blockDim.x)
+        a.seis[(long long)(n - 1) * a.nrec_tot + a.rec_id[r]] = un[a.rec_off[r]];
+    if (n == a.nt) break;
+    for (long long g = blockIdx.x * (long long)blockDim.x + threadIdx.x; g < ngroups;
+         g += (long long)gridDim.x * blockDim.x) {
+      const int x0 = (int)(g % gx) * 4;
+      const long long rest = g / gx;
+      const int j = (int)(rest % d.ny), k = (int)(rest / d.ny);
+      const long long o = d.at(x0, j, k);
+      float xv[12];
+      {
+        const F4 a0 = ld4(un + o - 4), a1 = ld4(un + o), a2 = ld4(un + o + 4);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          xv[e] = a0.v[e];
+          xv[4 + e] = a1.v[e];
+          xv[8 + e] = a2.v[e];
+        }
+      }
+      F4 yp[4], zp[4];
+#pragma unroll
+      for (int m = 1; m <= 4; ++m) {
+        const F4 ya = ld4(un + o + m * d.PX), yb = ld4(un + o - m * d.PX);
+        const F4 za = ld4(un + o - m * PS), zb = ld4(un + o + m * PS);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          yp[m - 1].v[e] = ya.v[e] + yb.v[e];
+          zp[m - 1].v[e] = za.v[e] + zb.v[e];
+        }
+      }
+      const F4 upv = ld4(up + o), mv = ldg4(a.m + o);
+      F4 out;
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        float xs[4], yss[4], zs[4];
+#pragma unroll
+        for (int m = 0; m < 4; ++m) {
+          xs[m] = xv[3 - m + e] + xv[5 + m + e];
+          yss[m] = yp[m].v[e];
+          zs[m] = zp[m].v[e];
+        }
+        const float lap = iso_lap(xv[4 + e], xs, yss, zs);
+        float eta = 0.0f;
+        if (a.edx) eta = (__ldg(a.edx + x0 + e) + __ldg(a.edy + j)) + __ldg(a.edz + k + d.z0);
+        out.v[e] = iso_update(xv[4 + e], upv.v[e], mv.v[e], lap, eta);
+      }
+      const long long rel = a.src_o - o;
+      if (rel >= 0 && rel < 4) {
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          if (rel == e) out.v[e] += a.amp[n];
+      }
+      st4_masked(up + o, out, x0, d.nx, true);
+    }
+    grid.sync();
+    cur = 1 - cur;
   }
 }
 

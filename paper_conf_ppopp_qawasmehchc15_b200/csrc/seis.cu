@@ -210,6 +210,8 @@ struct seis_model {
   size_t stage_elems = 0;
   float* scales = nullptr;  // fp16 snapshot scales + max words (seis_shot.snap_fp16)
   size_t scales_elems = 0;
+  float* pamp = nullptr;    // persistent small-grid ISO path: per-step source amplitudes
+  int pamp_n = 0;
   const float* hwav = nullptr;  // host wavelet of the current call
   int last_nt = 0;
   // shot-table cache and the CUDA graph of the last forward_model (single process)
@@ -1900,6 +1902,63 @@ seis_status ensure_stage(seis_model* M, size_t elems) {
 
 }  // namespace
 
+// Small L2-resident ISO grids: the whole shot as one cooperative launch (iso_persist_kernel).
+bool persist_ok(const seis_model* M) {
+  if (M->kind != SEIS_ISO || M->slabs.size() != 1 || (M->comm && M->nranks > 1) || prof::on) return false;
+  const Slab& S = M->slabs[0];
+  if (S.sp) return false;  // (the split-field PML keeps the z-march kernel)
+  const char* e = getenv("SEIS_NO_PERSIST");
+  const bool off = e && e[0] == '1';
+  return !off && (double)S.d.nx * S.d.ny * S.d.nzl < 4.0 * 1024 * 1024;
+}
+
+seis_status forward_persist(seis_model* M, const seis_shot* sh, float* sd, size_t ns, cudaStream_t st) {
+  Slab& S = M->slabs[0];
+  TRY(zero_state(M, st));
+  if (ns) CK(cudaMemsetAsync(sd, 0, ns * sizeof(float), st));
+  if (M->pamp_n < sh->nt) {
+    void* p = nullptr;
+    TRY(alloc_track(M, &p, (size_t)sh->nt * sizeof(float)));
+    M->pamp = (float*)p;
+    M->pamp_n = sh->nt;
+  }
+  std::vector<float> amp(sh->nt, 0.f);
+  if (S.src_o >= 0)
+    for (int n = 0; n < sh->nt; ++n) amp[n] = S.src_scale * M->hwav[n];  // as step(): float product
+  CK(cudaMemcpyAsync(M->pamp, amp.data(), amp.size() * sizeof(float), cudaMemcpyHostToDevice, st));
+  IsoPArgs a;
+  a.u0 = S.fld[0];
+  a.u1 = S.fld[1];
+  a.m = S.m;
+  a.edx = M->edx;
+  a.edy = M->edy;
+  a.edz = M->edz;
+  a.d = S.d;
+  a.nt = sh->nt;
+  a.cur0 = S.cur;
+  a.src_o = S.src_o;
+  a.amp = M->pamp;
+  a.seis = sd;
+  a.rec_off = S.d_rec_off;
+  a.rec_id = S.d_rec_id;
+  a.nrec = S.nrec_own;
+  a.nrec_tot = sh->nrec;
+  static int occ = 0, nsm = 0;
+  if (!occ) {
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, iso_persist_kernel, 128, 0));
+    CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, M->device));
+  }
+  const long long groups = (long long)((S.d.nx + 3) / 4) * S.d.ny * S.d.nzl;
+  const char* eb = getenv("SEIS_PERSIST_BPSM");  // blocks per SM (A/B; default: all that fit)
+  const int bpsm = eb ? std::max(1, std::min(atoi(eb), occ)) : occ;
+  const int blocks = (int)std::max<long long>(1, std::min<long long>((groups + 127) / 128, (long long)bpsm * nsm));
+  void* args[] = {&a};
+  CK(cudaLaunchCooperativeKernel((void*)iso_persist_kernel, dim3(blocks), dim3(128), args, 0, st));
+  ++g_launches;
+  S.cur = (S.cur + sh->nt) & 1;  // the z-march path's final level bookkeeping
+  return SEIS_OK;
+}
+
 extern "C" {
 
 // The time loop of one modeling shot (everything between the zeroed state and the
@@ -1934,7 +1993,9 @@ seis_status seis_forward_model(seis_model* M, const seis_shot* sh, float* seis, 
   // Single process: the whole shot is one CUDA graph (captured once per shot setup and
   // output buffer, replayed afterwards), so small grids are not launch-bound.
   const bool use_graph = !prof::on && !(M->comm && M->nranks > 1) && !getenv("SEIS_NO_GRAPH");
-  if (use_graph) {
+  if (persist_ok(M)) {
+    TRY(forward_persist(M, sh, sd, ns, st));
+  } else if (use_graph) {
     uint64_t key = fnv1a(sh->wavelet, (size_t)sh->nt * sizeof(float), M->shot_key);
     key = fnv1a(&sd, sizeof(sd), key);
     key = fnv1a(&sh->nt, sizeof(int32_t), key);

@@ -1,4 +1,4 @@
-"""C1 (ISO 64^3, 200 steps; L2-resident, launch-bound) under different z-chunk minimums.
+"""C1 (ISO 64^3, 200 steps; L2-resident, launch-bound): z-march path vs the persistent kernel.
 
     python tools/c1_sweep.py        # on a B200: one line per SEIS_ZCHUNK_MIN value
 """
@@ -27,8 +27,11 @@ ms = e0.elapsed_time(e1) / 20
 print(json.dumps({"ms_per_shot": round(ms, 4), "gpts_s": round(wl.npts * wl.nt / (ms * 1e-3) / 1e9, 2)}))
 '''
 
-for zmin in (8, 4, 2, 1):
-    env = dict(os.environ, SEIS_ZCHUNK_MIN=str(zmin))
+for zmin, bpsm, pers in ((2, 0, 0), (2, 1, 1), (2, 2, 1), (2, 3, 1), (2, 0, 1)):
+    env = dict(os.environ, SEIS_ZCHUNK_MIN=str(zmin), SEIS_NO_PERSIST="0" if pers else "1")
+    if bpsm:
+        env["SEIS_PERSIST_BPSM"] = str(bpsm)
     r = subprocess.run([sys.executable, "-c", ONE, ROOT], env=env, capture_output=True, text=True, timeout=600)
     out = r.stdout.strip().splitlines()[-1] if r.stdout.strip() else json.dumps({"error": r.stderr[-300:]})
-    print(json.dumps({"zchunk_min": zmin, **json.loads(out)}), flush=True)
+    print(json.dumps({"zchunk_min": zmin, "persistent": pers, "blocks_per_sm": bpsm or "max", **json.loads(out)}),
+          flush=True)
