@@ -580,9 +580,9 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
 // gives its parity / staggering): 2 launches per elastic step instead of 6.
 __global__ void fs_mirror3_kernel(float* __restrict__ f0, float* __restrict__ f1, float* __restrict__ f2, Dims d,
                                   int odd_bits, int half_bits) {
-  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  const int i0 = 4 * (blockIdx.x * blockDim.x + threadIdx.x);  // 4 x-points per thread (float4)
   const int j = blockIdx.y, t = blockIdx.z;
-  if (i >= d.nx) return;
+  if (i0 >= d.nx) return;
   float* __restrict__ f = t == 0 ? f0 : (t == 1 ? f1 : f2);
   const bool half = (half_bits >> t) & 1;
   const float sgn = ((odd_bits >> t) & 1) ? -1.0f : 1.0f;
@@ -590,7 +590,8 @@ __global__ void fs_mirror3_kernel(float* __restrict__ f0, float* __restrict__ f1
   for (int m = 0; m < 4; ++m) {
     const int src = half ? m : m + 1;
     const int dst = half ? -1 - m : -(m + 1);
-    f[d.at(i, j, dst)] = sgn * f[d.at(i, j, src)];
+    const F4 v = ld4(f + d.at(i0, j, src));  // (rows are 16-byte aligned, the x tail is padding)
+    st4_masked(f + d.at(i0, j, dst), F4{{sgn * v.v[0], sgn * v.v[1], sgn * v.v[2], sgn * v.v[3]}}, i0, d.nx, true);
   }
 }
 

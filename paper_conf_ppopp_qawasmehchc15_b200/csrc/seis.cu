@@ -1446,7 +1446,7 @@ seis_status fs_mirror(seis_model* M, std::initializer_list<int> fields, cudaStre
   }
   {
     PROF(8, st);
-    fs_mirror3_kernel<<<dim3((S.d.nx + 127) / 128, S.d.ny, t), 128, 0, st>>>(f[0], f[1], f[2], S.d, odd, half);
+    fs_mirror3_kernel<<<dim3((S.d.nx + 511) / 512, S.d.ny, t), 128, 0, st>>>(f[0], f[1], f[2], S.d, odd, half);
   }
   CKL();
   return SEIS_OK;
