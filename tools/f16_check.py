@@ -1,5 +1,7 @@
-import sys, json, numpy as np, torch
-sys.path.insert(0, "/root/repo")
+"""fp16 vs fp32 RTM snapshots on the C4 salt model at 128^3 and 256^3 (image relative L2);
+forward-modeled data, migration on the true model.  On a B200: python tools/f16_check.py"""
+import os, sys, json, numpy as np, torch
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import paper_conf_ppopp_qawasmehchc15_b200 as seis
 from paper_conf_ppopp_qawasmehchc15_b200 import inputs
 res = {}
