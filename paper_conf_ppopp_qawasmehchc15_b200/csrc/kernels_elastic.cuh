@@ -14,7 +14,7 @@
 //     sxz += (dt mu_xz/h)(Dz+ vx + Dx+ vz)             (+ psi 14,15)
 //     syz += (dt mu_yz/h)(Dz+ vy + Dy+ vz)             (+ psi 16,17)
 // psi stored times h (unscaled differences).  Free surface (O16): the top ghost
-// planes hold the mirror images (filled by fs_mirror_kernel after every
+// planes hold the mirror images (filled by fs_mirror3_kernel after every
 // exchange), the surface row uses ezz = -lam/(lam+2mu)(exx+eyy), and szz = 0 on
 // k = 0 after the source.
 //
@@ -595,17 +595,5 @@ __global__ void fs_mirror3_kernel(float* __restrict__ f0, float* __restrict__ f1
   }
 }
 
-__global__ void fs_mirror_kernel(float* __restrict__ f, Dims d, int odd, int half) {
-  const int i = blockIdx.x * blockDim.x + threadIdx.x;
-  const int j = blockIdx.y;
-  if (i >= d.nx) return;
-  const float sgn = odd ? -1.0f : 1.0f;
-#pragma unroll
-  for (int m = 0; m < 4; ++m) {
-    const int src = half ? m : m + 1;
-    const int dst = half ? -1 - m : -(m + 1);
-    f[d.at(i, j, dst)] = sgn * f[d.at(i, j, src)];
-  }
-}
 
 }  // namespace seis
