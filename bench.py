@@ -126,6 +126,17 @@ def c2_workload(n=512, nt=2000, nz=None):
     return wl
 
 
+def c2_config(wl, nz, nt, nrec, ws, args):
+    """The `config` both arms report (the reference arm times a bounded sample of it)."""
+    return {"workload": f"C2 acoustic {wl.nx}x{wl.ny}x{nz} layered, {nt} steps, C-PML nb={wl.nb}, "
+                        f"{nrec}-receiver line, 1 shot per step",
+            "grid": [wl.nx, wl.ny, nz], "nt": nt, "dt": wl.dt, "h": wl.h,
+            "parallelism": f"z-slab x{ws}" if ws > 1 else "single GPU",
+            "scaling": args.scaling if ws > 1 else None,
+            "halo": (args.halo if ws > 1 else None),
+            "l2": "inputs larger than L2 (each 512^3 field is 512 MiB > 126 MB)"}
+
+
 def psi_bytes_per_point(nx, ny, nz, nb, axes_per_dir, free_surface=False):
     """C-PML memory-variable RMW bytes per grid point (8 B per point inside a layer, per axis;
     a free-surface top has no layer)."""
@@ -242,12 +253,7 @@ def run_product(args):
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms / args.steps, 3),
            "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f32",
            "data": "synthetic (seeded layered model, Ricker source)",
-           "config": {"workload": f"C2 acoustic {wl.nx}x{wl.ny}x{nz} layered, {nt} steps, C-PML nb={wl.nb}, "
-                                  f"{shot.nrec}-receiver line, 1 shot per step",
-                      "grid": [wl.nx, wl.ny, nz], "nt": nt, "dt": wl.dt, "h": wl.h,
-                      "parallelism": f"z-slab x{ws}" if ws > 1 else "single GPU",
-                      "halo": (args.halo if ws > 1 else None),
-                      "l2": "inputs larger than L2 (each 512^3 field is 512 MiB > 126 MB)"},
+           "config": c2_config(wl, nz, nt, shot.nrec, ws, args),
            "e2e": e2e, "gpu_launches": launches, "roofline": roof}
     if rank == 0:
         out["clocks"] = clk.summary()
@@ -421,10 +427,9 @@ def run_reference(args):
     print(json.dumps({
         "impl": "reference", "metric": METRIC, "value": round(value, 5), "unit": "Gpts/s", "n_gpus": ws,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt / args.steps * 1e3, 1),
-        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f64",
         "data": "synthetic (seeded layered model, Ricker source)",
-        "config": {"workload": f"C2 acoustic {n}^3 layered, C-PML nb={wl.nb} (oracle sample)",
-                   "grid": [n, n, n], "nt_per_step": per},
+        "config": c2_config(wl, n * ws if args.scaling == "weak" else n, args.nt, wl.rec.shape[0], ws, args),
         "cpu_baseline": {"value": round(value, 5), "unit": "Gpts/s", "cores": cores, "kind": "oracle",
                          "sample": sample},
         "e2e": {"value": round(value, 5), "unit": "Gpts/s", "h2d_bytes_per_step": 0,
