@@ -19,9 +19,8 @@ sys.path.insert(0, ROOT)
 
 VARIANTS = {
     "base": [],
-    "e4_mb4_v2": ["SEIS_BYE=4", "SEIS_EL_MINB=4", "SEIS_EL_VNS=2"],
-    "e4_mb4_v3": ["SEIS_BYE=4", "SEIS_EL_MINB=4", "SEIS_EL_VNS=3"],
-    "e4_mb3_v3": ["SEIS_BYE=4", "SEIS_EL_MINB=3", "SEIS_EL_VNS=3"],
+    "ac_mb4": ["SEIS_AC_MINB=4"],
+    "ac_mb4_vns2": ["SEIS_AC_MINB=4", "SEIS_AC_VNS=2"],
 }
 
 
