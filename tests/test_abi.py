@@ -149,3 +149,27 @@ def test_memory_required_fp16_snapshots_halve_the_pool():
     m0 = seis.memory_required(g, "acoustic")
     assert seis.memory_required(g, "acoustic", sh16) - m0 == 10 * 128 * 96 * 64 * 2
     assert seis.memory_required(g, "acoustic", sh) - m0 == 10 * 128 * 96 * 64 * 4
+
+
+def test_product_path_fails_loudly_without_the_library():
+    """No CPU fallback: with the CUDA library missing, the binding raises (fresh process)."""
+    import subprocess
+    import sys
+
+    code = ("import os; os.environ['SEIS_LIBPATH'] = '/nonexistent/libseis.so'\n"
+            "import paper_conf_ppopp_qawasmehchc15_b200 as s\n"
+            "try:\n    s.lib()\nexcept RuntimeError as e:\n    print('RAISED', e)\n")
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, cwd=ROOT, timeout=120)
+    assert "RAISED" in r.stdout and "no CPU fallback" in r.stdout
+
+
+def test_product_package_never_touches_the_oracle():
+    """The oracle is test infrastructure: nothing in the product package or its CUDA sources
+    imports, includes or links it."""
+    pkg = os.path.join(ROOT, "paper_conf_ppopp_qawasmehchc15_b200")
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h")):
+                src = open(os.path.join(dirpath, f)).read()
+                assert not re.search(r"^\s*(import|from)\s+oracle\b", src, re.M), f
+                assert "oracle.h" not in src and "liboracle" not in src, f
