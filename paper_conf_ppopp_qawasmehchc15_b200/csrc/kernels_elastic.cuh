@@ -13,9 +13,9 @@
 //     sxy += (dt mu_xy/h)(Dy+ vx + Dx+ vy)             (+ psi 12,13)
 //     sxz += (dt mu_xz/h)(Dz+ vx + Dx+ vz)             (+ psi 14,15)
 //     syz += (dt mu_yz/h)(Dz+ vy + Dy+ vz)             (+ psi 16,17)
-// psi stored times h (unscaled differences).  Free surface (O16): the top ghost
-// planes hold the mirror images (filled by fs_mirror3_kernel after every
-// exchange), the surface row uses ezz = -lam/(lam+2mu)(exx+eyy), and szz = 0 on
+// psi stored times h (unscaled differences).  Free surface (O16): the planes above
+// k = 0 are the mirror images of the planes below (formed in the z-queue warm-up,
+// ldg2_fs), the surface row uses ezz = -lam/(lam+2mu)(exx+eyy), and szz = 0 on
 // k = 0 after the source.
 //
 // Both kernels are 2.5D z-marches over 64 x BY tiles with 2 x-points per thread
@@ -62,6 +62,21 @@ __device__ __forceinline__ void ycol(float (*yv)[9], const float* c) {
     yv[0][m] = a.v[0];
     yv[1][m] = a.v[1];
   }
+}
+
+// z-queue warm-up load of plane p of field f at column offset oc.  With the free surface
+// (O16), the planes above k = 0 of the top slab are the mirror images of the planes below
+// it -- integer-z fields: plane -m = sgn f(m); half-z fields: plane -1-m = sgn f(m)
+// (sgn = -1 for szz, sxz, syz) -- and they are only ever read here (every other operand of
+// the z-march is at planes >= 0), so they are formed on the fly instead of being stored by
+// a mirror kernel after every half step.
+__device__ __forceinline__ F2 ldg2_fs(const float* __restrict__ f, int p, long long PS, long long oc, bool mirror,
+                                      bool half, float sgn) {
+  if (mirror && p < 0) {
+    const F2 v = ldg2(f + (long long)((half ? -1 - p : -p) + GZ) * PS + oc);
+    return F2{{sgn * v.v[0], sgn * v.v[1]}};
+  }
+  return ldg2(f + (long long)(p + GZ) * PS + oc);
 }
 
 #ifndef SEIS_EL_VNS
@@ -172,11 +187,20 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
   const float* __restrict__ syz = a.f[ESYZ];
   const float* __restrict__ szz = a.f[ESZZ];
   F2 qxz[8], qyz[8], qzz[8];  // sxz, syz at k-4..k+3 (D-); szz at k-3..k+4 (D+)
+  if (a.fs && d.z0 == 0 && k0 < 4) {  // free-surface images above the top slab (O16)
 #pragma unroll
-  for (int t = 0; t < 7; ++t) {
-    qxz[t] = ldg2(sxz + (long long)(k0 - 4 + t + GZ) * PS + oc);
-    qyz[t] = ldg2(syz + (long long)(k0 - 4 + t + GZ) * PS + oc);
-    qzz[t] = ldg2(szz + (long long)(k0 - 3 + t + GZ) * PS + oc);
+    for (int t = 0; t < 7; ++t) {
+      qxz[t] = ldg2_fs(sxz, k0 - 4 + t, PS, oc, true, true, -1.0f);
+      qyz[t] = ldg2_fs(syz, k0 - 4 + t, PS, oc, true, true, -1.0f);
+      qzz[t] = ldg2_fs(szz, k0 - 3 + t, PS, oc, true, false, -1.0f);
+    }
+  } else {
+#pragma unroll
+    for (int t = 0; t < 7; ++t) {
+      qxz[t] = ldg2(sxz + (long long)(k0 - 4 + t + GZ) * PS + oc);
+      qyz[t] = ldg2(syz + (long long)(k0 - 4 + t + GZ) * PS + oc);
+      qzz[t] = ldg2(szz + (long long)(k0 - 3 + t + GZ) * PS + oc);
+    }
   }
   SEIS_UNROLL(SEIS_ZU_EL)
   for (int it = 0; it < np; ++it) {
@@ -402,11 +426,20 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
   const float* __restrict__ vy = a.f[EVY];
   const float* __restrict__ vz = a.f[EVZ];
   F2 qx[8], qy[8], qz[8];  // vx, vy at k-3..k+4 (D+); vz at k-4..k+3 (D-)
+  if (a.fs && d.z0 == 0 && k0 < 4) {  // free-surface images above the top slab (O16)
 #pragma unroll
-  for (int t = 0; t < 7; ++t) {
-    qx[t] = ldg2(vx + (long long)(k0 - 3 + t + GZ) * PS + oc);
-    qy[t] = ldg2(vy + (long long)(k0 - 3 + t + GZ) * PS + oc);
-    qz[t] = ldg2(vz + (long long)(k0 - 4 + t + GZ) * PS + oc);
+    for (int t = 0; t < 7; ++t) {
+      qx[t] = ldg2_fs(vx, k0 - 3 + t, PS, oc, true, false, 1.0f);
+      qy[t] = ldg2_fs(vy, k0 - 3 + t, PS, oc, true, false, 1.0f);
+      qz[t] = ldg2_fs(vz, k0 - 4 + t, PS, oc, true, true, 1.0f);
+    }
+  } else {
+#pragma unroll
+    for (int t = 0; t < 7; ++t) {
+      qx[t] = ldg2(vx + (long long)(k0 - 3 + t + GZ) * PS + oc);
+      qy[t] = ldg2(vy + (long long)(k0 - 3 + t + GZ) * PS + oc);
+      qz[t] = ldg2(vz + (long long)(k0 - 4 + t + GZ) * PS + oc);
+    }
   }
   const long long srel0 = a.src_o - oc;
   SEIS_UNROLL(SEIS_ZU_EL)
@@ -573,27 +606,6 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
   }
 }
 
-// Free-surface ghost planes above k = 0 (O16): for field f with parity `odd`
-// (1: antisymmetric, 0: symmetric) and staggering `half` (1: z-half node),
-//   integer z: ghost(-m) = +-f(m), m = 1..4;   half z: ghost(-1-m) = +-f(m), m = 0..3.
-// One launch for the three fields a phase mirrors (blockIdx.z = field t; bit t of odd / half
-// gives its parity / staggering): 2 launches per elastic step instead of 6.
-__global__ void fs_mirror3_kernel(float* __restrict__ f0, float* __restrict__ f1, float* __restrict__ f2, Dims d,
-                                  int odd_bits, int half_bits) {
-  const int i0 = 4 * (blockIdx.x * blockDim.x + threadIdx.x);  // 4 x-points per thread (float4)
-  const int j = blockIdx.y, t = blockIdx.z;
-  if (i0 >= d.nx) return;
-  float* __restrict__ f = t == 0 ? f0 : (t == 1 ? f1 : f2);
-  const bool half = (half_bits >> t) & 1;
-  const float sgn = ((odd_bits >> t) & 1) ? -1.0f : 1.0f;
-#pragma unroll
-  for (int m = 0; m < 4; ++m) {
-    const int src = half ? m : m + 1;
-    const int dst = half ? -1 - m : -(m + 1);
-    const F4 v = ld4(f + d.at(i0, j, src));  // (rows are 16-byte aligned, the x tail is padding)
-    st4_masked(f + d.at(i0, j, dst), F4{{sgn * v.v[0], sgn * v.v[1], sgn * v.v[2], sgn * v.v[3]}}, i0, d.nx, true);
-  }
-}
 
 
 }  // namespace seis

@@ -1430,27 +1430,6 @@ size_t state_elems(seis_model* M) {
   return o;
 }
 
-// Free-surface ghost planes (O16) of the slab that holds the global top.
-seis_status fs_mirror(seis_model* M, std::initializer_list<int> fields, cudaStream_t st) {
-  if (!M->g.free_surface) return SEIS_OK;
-  Slab& S = M->slabs.front();
-  if (S.d.z0 != 0) return SEIS_OK;
-  // parity / staggering per field: v even, sigma_zz/xz/yz odd; vz, sxz, syz on half z nodes
-  float* f[3] = {};
-  int odd = 0, half = 0, t = 0;
-  for (int fi : fields) {
-    f[t] = S.fld[fi];
-    if (fi == ESZZ || fi == ESXZ || fi == ESYZ) odd |= 1 << t;
-    if (fi == EVZ || fi == ESXZ || fi == ESYZ) half |= 1 << t;
-    ++t;
-  }
-  {
-    PROF(8, st);
-    fs_mirror3_kernel<<<dim3((S.d.nx + 511) / 512, S.d.ny, t), 128, 0, st>>>(f[0], f[1], f[2], S.d, odd, half);
-  }
-  CKL();
-  return SEIS_OK;
-}
 
 // ISO / ACOUSTIC: 64 x BY tiles of (16, BY) threads; ELASTIC: 32 x BYE tiles of (32, BYE)
 dim3 grid_of(const Slab& S, int tw, int by, int nch) {
@@ -1810,8 +1789,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
   };
   PostFn post_v = [&](int part, cudaStream_t ps) -> seis_status {
     if (part == 1) return SEIS_OK;
-    TRY(exchange(M, {0, 1, 2}, ps));
-    return fs_mirror(M, {EVX, EVY, EVZ}, ps);
+    return exchange(M, {0, 1, 2}, ps);  // (free-surface images: formed in el_s's z-queue warm-up)
   };
   TRY(run_phase(M, k_v, post_v, st));
   LaunchFn k_s = [&](size_t s, int ch0, int chs, int nch, cudaStream_t ks) -> seis_status {
@@ -1853,8 +1831,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
   PostFn post_s = [&](int part, cudaStream_t ps) -> seis_status {
     TRY(inject(part, ps));
     if (part == 1) return SEIS_OK;
-    TRY(exchange(M, {5, 7, 8}, ps));
-    return fs_mirror(M, {ESZZ, ESXZ, ESYZ}, ps);
+    return exchange(M, {5, 7, 8}, ps);  // (free-surface images: formed in el_v's z-queue warm-up)
   };
   return run_phase(M, k_s, post_s, st);
 }
