@@ -213,7 +213,8 @@ seis_status seis_migrate(seis_model* model, const seis_shot* shot, const float* 
  *   ELASTIC: 0..8 = vx, vy, vz, sxx, syy, szz, sxy, sxz, syz. */
 seis_status seis_get_field(const seis_model* model, int32_t which, float* dst, void* stream);
 /* Device bytes a model + one migrate call needs per process (state, coefficients,
- * C-PML slabs, snapshot pool). shot may be NULL (modeling only). */
+ * C-PML slabs, ISO split-field PML components, snapshot pool: 4 or, with snap_fp16, 2 bytes
+ * per snapshot value, and the checkpoints of ckpt_period). shot may be NULL (modeling only). */
 seis_status seis_memory_required(const seis_grid* grid, seis_kind kind, const seis_shot* shot,
                                  int32_t nranks, uint64_t* bytes);
 /* Per-kernel CUDA-event timing (profiling / bench.py).  seis_profile(1) resets the
