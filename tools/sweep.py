@@ -19,8 +19,7 @@ sys.path.insert(0, ROOT)
 
 VARIANTS = {
     "base": [],
-    "ac_mb4": ["SEIS_AC_MINB=4"],
-    "ac_mb4_vns2": ["SEIS_AC_MINB=4", "SEIS_AC_VNS=2"],
+    "el_mb1": ["SEIS_EL_MINB=1"],
 }
 
 
