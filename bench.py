@@ -11,13 +11,17 @@ Gpts/s = grid points x time steps / second (whole job over all ranks).
 
 * value:  device-timed (CUDA events on the launching stream, barrier + synchronize on
           both sides, max over ranks), inputs resident in HBM, seismogram to a device buffer.
-* e2e:    the same shots through the C ABI with HOST buffers (pinned): the wavelet and
-          receiver table are copied in and the seismogram copied out inside the timed region.
+* e2e:    the same shots through the C ABI with HOST buffers: every call copies the wavelet
+          (host [nt] fp32) to the device and the seismogram (pinned host [nt][nrec]) back,
+          inside the timed region; the receiver table is re-uploaded only when the geometry
+          changes (here: never after the first call, so its bytes are not counted).
 * roofline: dominant kernel's algorithmic bytes per launch / its average CUDA-event launch
           time (library event pairs on the launching stream, recorded over the timed region),
           against MEASURED_PEAKS.json hbm_gbs.
-* cpu_baseline: the fp64 oracle (oracle/, test infrastructure) timed on the host cores on a
-          bounded sample of the same workload (2 time steps of the full 512^3 grid).
+* cpu_baseline: the fp64 oracle (oracle/, test infrastructure) timed on the host cores
+          (child process, OMP_PROC_BIND=close, all cores) on a bounded sample of the same
+          workload: 1 untimed + 5 timed time steps of the full 512^3 grid; C1 and C3 oracle
+          timings ride along under other_configs.
 * extras (N = 1, unless --no-extras): Gpts/s of the other propagators (C1 ISO 64^3, an ISO 512^3
           sweep, C3 elastic 384^3) and RTM shots/hour (C4, 512^3 salt model, 2000 steps,
           snapshots every 20 steps in HBM).
@@ -116,13 +120,17 @@ def dist_env():
 
 
 # ---------------------------------------------------------------- workloads
-def c2_workload(n=512, nt=2000, nz=None):
+def c2_workload(n=512, nt=2000, nz=None, z0=0, nzl=None):
+    """The C2 workload on an n x n x nz grid (nz = n: the BASELINE config); with z0 / nzl only
+    that z-slab of the model is generated (each rank builds its own slab: host memory per rank
+    is bounded by the slab, not the global grid)."""
     from paper_conf_ppopp_qawasmehchc15_b200 import inputs
 
-    wl = inputs.c2(n=n, nt=nt, nb=20)
-    if nz is not None and nz != n:
-        wl.model = inputs.layered_acoustic(n, n, nz, scale=n / 512.0)
-        wl.nz = nz
+    nz = n if nz is None else nz
+    nzl = nz - z0 if nzl is None else nzl
+    wl = inputs.c2(n=n, nt=nt, nb=20, model=False)
+    wl.model = inputs.layered_acoustic(n, n, nz, scale=n / 512.0, z0=z0, nzl=nzl)
+    wl.nz = nz
     return wl
 
 
@@ -164,11 +172,11 @@ def run_product(args):
     n, nt = args.n, args.nt
     # weak scaling (default): each rank holds n^3 points; strong: the n^3 grid is split
     nz = n if args.scaling == "strong" else n * ws
-    wl = c2_workload(n=n, nt=nt, nz=nz)
     z0, nzl = seis.slab_bounds(nz, ws, rank)
+    wl = c2_workload(n=n, nt=nt, nz=nz, z0=z0, nzl=nzl)  # this rank's slab only
     grid = seis.Grid(wl.nx, wl.ny, nz, wl.h, wl.dt, nb=wl.nb, pml_R=wl.pml_R, pml_f=wl.fp)
-    model = seis.Model(grid, "acoustic", wl.model["vp"][z0:z0 + nzl], rho=wl.model["rho"][z0:z0 + nzl],
-                       comm=comm, device=local)
+    model = seis.Model(grid, "acoustic", wl.model["vp"], rho=wl.model["rho"], comm=comm, device=local)
+    del wl.model
     if ws > 1 and args.halo == "peer":
         model.enable_peer_halo()  # f4: rank faces by direct NVLink ghost stores (CUDA IPC)
     shot = seis.Shot(wl.src, wl.wavelet, wl.rec)
@@ -203,7 +211,8 @@ def run_product(args):
     pts = float(wl.nx) * wl.ny * nz  # all ranks
     value = pts * nt * args.steps / (ms * 1e-3) / 1e9
 
-    # e2e: HOST buffers through the C ABI (pinned seismogram; wavelet + receivers are host)
+    # e2e: HOST buffers through the C ABI (the wavelet is uploaded and the pinned seismogram
+    # read back by every call)
     host_seis = torch.empty((nt, shot.nrec), dtype=torch.float32).pin_memory()
     model.forward_model(shot, host_seis.numpy(), stream)
     barrier()
@@ -220,7 +229,7 @@ def run_product(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_ms = float(t.item())
     e2e = {"value": round(pts * nt * args.steps / (e2e_ms * 1e-3) / 1e9, 3), "unit": "Gpts/s",
-           "h2d_bytes_per_step": int(shot.nt * 4 + shot.nrec * 12),
+           "h2d_bytes_per_step": int(shot.nt * 4),  # the wavelet (receivers cached by geometry)
            "d2h_bytes_per_step": int(shot.nt * shot.nrec * 4)}
 
     # roofline of the dominant kernel
@@ -383,55 +392,127 @@ def run_extras(args, local):
 
 
 # ---------------------------------------------------------------- oracle arm
-def cpu_baseline(args, steps=2):
-    """The fp64 oracle (as it stands) on the host cores: `steps` time steps of the full C2 grid."""
-    import oracle
+def cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
 
-    n = args.n
-    wl = c2_workload(n=n, nt=args.nt)
-    g = oracle.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=wl.nb, pml_R=wl.pml_R, pml_f=wl.fp)
-    st = oracle.ac_state(g)
+
+def _oracle_env():
+    """OpenMP settings of every oracle timing: all host cores, threads bound close.
+    Set before liboracle (and libgomp) is loaded in this process."""
+    os.environ.setdefault("OMP_NUM_THREADS", str(os.cpu_count() or 1))
+    os.environ.setdefault("OMP_PROC_BIND", "close")
+    os.environ.setdefault("OMP_PLACES", "cores")
+    return int(os.environ["OMP_NUM_THREADS"])
+
+
+def _mem_available():
+    try:
+        with open("/proc/meminfo") as f:
+            for line in f:
+                if line.startswith("MemAvailable:"):
+                    return int(line.split()[1]) * 1024
+    except Exception:
+        pass
+    return 0
+
+
+def oracle_timing(which, n=512, nz=None, nt=2000, warm=1, steps=5):
+    """Time the fp64 oracle (as it stands) on `which` in THIS process: `warm` untimed time steps
+    (first touch of the fp64 state), then `steps` timed ones (C1: whole shots).  Returns
+    (Gpts/s, sample description).  C2 with nz > n (weak scaling config): the whole global grid
+    when its fp64 state fits in half the available host memory, else the top n^3 z-block of
+    the same model (same per-point work; stated in the sample)."""
+    import oracle
+    from paper_conf_ppopp_qawasmehchc15_b200 import inputs
+
+    if which == "C1":
+        wl = inputs.c1()
+        g = oracle.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=wl.nb)
+        run = lambda st, n0, k: oracle.iso_run(g, wl.model["vp"], st, 0, wl.nt, [wl.src], wl.wavelet[:, None],
+                                               wl.rec)
+        new = lambda: oracle.iso_state(g)
+        pts, per, what = wl.npts, wl.nt, f"C1 ISO 64^3: {{k}} whole {wl.nt}-step shot(s)"
+    elif which == "C3":
+        wl = inputs.c3(n=n * 3 // 4)
+        g = oracle.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=wl.nb, free_surface=1, pml_R=wl.pml_R, pml_f=wl.fp)
+        m = wl.model
+        run = lambda st, n0, k: oracle.el_run(g, m["vp"], m["vs"], m["rho"], st, n0, k, [wl.src],
+                                              wl.wavelet[:, None], wl.rec, component=2)
+        new = lambda: oracle.el_state(g)
+        pts, per, what = wl.npts, 1, f"C3 elastic {wl.nx}^3: {{k}} time steps of the shot on the full grid"
+    else:
+        nz = n if nz is None else nz
+        full = nz * n * n * (10 * 8 + 2 * 4) <= 0.5 * _mem_available() or nz == n
+        nzs = nz if full else n
+        wl = c2_workload(n=n, nt=nt, nz=nz, z0=0, nzl=nzs)
+        g = oracle.Grid(wl.nx, wl.ny, nzs, wl.h, wl.dt, nb=wl.nb, pml_R=wl.pml_R, pml_f=wl.fp)
+        m = wl.model
+        run = lambda st, n0, k: oracle.ac_run(g, m["vp"], m["rho"], st, n0, k, [wl.src], wl.wavelet[:, None],
+                                              wl.rec)
+        new = lambda: oracle.ac_state(g)
+        pts, per = float(n) * n * nzs, 1
+        what = (f"C2 acoustic {n}x{n}x{nz}: {{k}} time steps of the shot on the full grid" if full else
+                f"C2 acoustic {n}x{n}x{nz}: {{k}} time steps on its top {n}^3 z-block (the global grid's "
+                f"fp64 state exceeds half the host memory)")
+    st = new()
+    if warm:
+        run(st, 0, warm * per if per == 1 else per)
     t0 = time.perf_counter()
-    oracle.ac_run(g, wl.model["vp"], wl.model["rho"], st, 0, steps, [wl.src], wl.wavelet[:, None],
-                  wl.rec)
+    if per == 1:
+        run(st, warm, steps)
+    else:
+        for _ in range(steps):
+            run(new(), 0, per)
     dt = time.perf_counter() - t0
-    cores = int(os.environ.get("OMP_NUM_THREADS", os.cpu_count() or 1))
-    return {"value": round(wl.npts * steps / dt / 1e9, 5), "unit": "Gpts/s", "cores": cores,
-            "kind": "oracle",
-            "sample": f"{steps} time steps of the C2 {n}^3 acoustic shot on the full grid "
-                      f"(oracle.ac_run, fp64, OpenMP), {dt:.1f} s"}
+    return pts * per * steps / dt / 1e9, what.format(k=steps) + f", after {warm} untimed warm-up, {dt:.1f} s"
+
+
+def cpu_baseline(args):
+    """The fp64 oracle (as it stands, test infrastructure) on the host cores, in a child process
+    with OMP_NUM_THREADS = all cores and OMP_PROC_BIND=close: C2 (the headline config: 1 warm-up +
+    5 timed time steps of the full 512^3 grid), plus C1 (whole shots) and C3 (2 steps)."""
+    env = dict(os.environ, OMP_NUM_THREADS=str(os.cpu_count() or 1), OMP_PROC_BIND="close", OMP_PLACES="cores")
+    out = {}
+    for which, steps in (("C2", 5), ("C1", 3), ("C3", 2)):
+        cmd = [sys.executable, os.path.abspath(__file__), "--oracle-timing", which, "--n", str(args.n),
+               "--nt", str(args.nt), "--oracle-steps", str(steps)]
+        try:
+            r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=600)
+            out[which] = json.loads(r.stdout.strip().splitlines()[-1])
+        except Exception as e:  # pragma: no cover - reported, not fatal
+            out[which] = {"error": repr(e)[:200]}
+    c2 = out.pop("C2")
+    return {"value": c2.get("value"), "unit": "Gpts/s", "cores": int(env["OMP_NUM_THREADS"]), "kind": "oracle",
+            "sample": c2.get("sample"), "cpu_model": cpu_model(), "omp": "OMP_PROC_BIND=close, OMP_PLACES=cores",
+            "other_configs": out}
 
 
 def run_reference(args):
     ws, rank, local = dist_env()
     if rank != 0:
         return
-    import oracle
-
+    cores = _oracle_env()
     n = args.n
-    wl = c2_workload(n=n, nt=args.nt)
-    g = oracle.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=wl.nb, pml_R=wl.pml_R, pml_f=wl.fp)
-    st = oracle.ac_state(g)
+    nz = n * ws if args.scaling == "weak" else n
     per = args.ref_steps
-    for _ in range(args.warmup):
-        oracle.ac_run(g, wl.model["vp"], wl.model["rho"], st, 0, 1, [wl.src], wl.wavelet[:, None], wl.rec)
-    t0 = time.perf_counter()
-    for s in range(args.steps):
-        oracle.ac_run(g, wl.model["vp"], wl.model["rho"], st, s * per, per, [wl.src], wl.wavelet[:, None],
-                      wl.rec)
-    dt = time.perf_counter() - t0
-    value = wl.npts * per * args.steps / dt / 1e9
-    cores = int(os.environ.get("OMP_NUM_THREADS", os.cpu_count() or 1))
-    sample = (f"each step = {per} time steps of the C2 {n}^3 acoustic shot on the full grid "
-              f"(oracle.ac_run, fp64)")
+    value, sample = oracle_timing("C2", n=n, nz=nz, nt=args.nt, warm=args.warmup, steps=args.steps * per)
+    wl = c2_workload(n=n, nt=args.nt, nz=nz, z0=0, nzl=1)  # geometry for the config (one plane)
     print(json.dumps({
         "impl": "reference", "metric": METRIC, "value": round(value, 5), "unit": "Gpts/s", "n_gpus": ws,
-        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(dt / args.steps * 1e3, 1),
+        "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(float(n) * n * nz * per / (value * 1e9) * 1e3, 1),
         "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f64",
         "data": "synthetic (seeded layered model, Ricker source)",
-        "config": c2_config(wl, n * ws if args.scaling == "weak" else n, args.nt, wl.rec.shape[0], ws, args),
+        "config": c2_config(wl, nz, args.nt, wl.rec.shape[0], ws, args),
         "cpu_baseline": {"value": round(value, 5), "unit": "Gpts/s", "cores": cores, "kind": "oracle",
-                         "sample": sample},
+                         "sample": f"each step = {per} time step(s); " + sample, "cpu_model": cpu_model()},
         "e2e": {"value": round(value, 5), "unit": "Gpts/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0}}))
 
@@ -451,7 +532,14 @@ def main():
     ap.add_argument("--halo", default="nccl", choices=["nccl", "peer"],
                     help="N>1 rank-face ghost exchange: NCCL send/recv overlapped with the interior "
                          "(default) or direct peer stores from the kernels (f4)")
+    ap.add_argument("--oracle-timing", default=None, help=argparse.SUPPRESS)  # cpu_baseline child
+    ap.add_argument("--oracle-steps", type=int, default=5, help=argparse.SUPPRESS)
     args = ap.parse_args()
+    if args.oracle_timing:
+        _oracle_env()
+        v, smp = oracle_timing(args.oracle_timing, n=args.n, nt=args.nt, steps=args.oracle_steps)
+        print(json.dumps({"value": round(v, 5), "unit": "Gpts/s", "sample": smp}))
+        return
     if args.warmup < 3:
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)
     if args.impl == "reference":

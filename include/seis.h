@@ -105,14 +105,15 @@ typedef struct {
                                 segment's snapshots from its checkpoint just before they are imaged
                                 (one extra forward pass at most).  Results are bitwise identical to
                                 c = 0 (same kernels, same order of operations). */
-  int32_t snap_fp16;         /* RTM snapshot storage precision (SURVEY §8f f2's "compressed fp16
-                                snapshots"): 0 = fp32 (default); 1 = fp16 scaled per snapshot and
-                                slab by a power of two (max |S_j| near 2^15; relative rounding
-                                2^-11): half the pool (C5 1024^3: all 49 snapshots on one B200
-                                without checkpointing).  The image then differs from the fp32
-                                one by the snapshot rounding (well inside the 1e-3 image bar) and
-                                is no longer bitwise invariant under the z-slab decomposition
-                                (each slab has its own scale). */
+  int32_t snap_bits;         /* RTM snapshot storage precision (SURVEY §8f f2's compressed-snapshot
+                                alternative): 0 or 32 = fp32 (default); 24 = every snapshot value
+                                rounded to nearest-even to 24 bits of its fp32 pattern (sign, 8-bit
+                                exponent, 15 mantissa bits: relative rounding <= 2^-16), stored as
+                                a 16-bit and an 8-bit plane: 3/4 of the fp32 pool.  No scale: the
+                                stored value depends on the fp32 value only, so images stay bitwise
+                                invariant under the z-slab decomposition and checkpointing; they
+                                differ from the fp32-snapshot image by the rounding, ~1e-5
+                                relative (inside the 1e-3 image bar).  EINVAL for other values. */
 } seis_shot;
 
 /* ---- multi-GPU (one process per GPU; z-slab decomposition, §8e) ---- */
@@ -213,7 +214,7 @@ seis_status seis_migrate(seis_model* model, const seis_shot* shot, const float* 
  *   ELASTIC: 0..8 = vx, vy, vz, sxx, syy, szz, sxy, sxz, syz. */
 seis_status seis_get_field(const seis_model* model, int32_t which, float* dst, void* stream);
 /* Device bytes a model + one migrate call needs per process (state, coefficients,
- * C-PML slabs, ISO split-field PML components, snapshot pool: 4 or, with snap_fp16, 2 bytes
+ * C-PML slabs, ISO split-field PML components, snapshot pool: 4 or, with snap_bits = 24, 3 bytes
  * per snapshot value, and the checkpoints of ckpt_period). shot may be NULL (modeling only). */
 seis_status seis_memory_required(const seis_grid* grid, seis_kind kind, const seis_shot* shot,
                                  int32_t nranks, uint64_t* bytes);

@@ -58,7 +58,7 @@ class _CShot(C.Structure):
     _fields_ = [("sx", C.c_int32), ("sy", C.c_int32), ("sz", C.c_int32),
                 ("wavelet", C.POINTER(C.c_float)), ("nt", C.c_int32), ("nrec", C.c_int32),
                 ("rec", C.POINTER(C.c_int32)), ("rec_component", C.c_int32),
-                ("snap_period", C.c_int32), ("ckpt_period", C.c_int32), ("snap_fp16", C.c_int32)]
+                ("snap_period", C.c_int32), ("ckpt_period", C.c_int32), ("snap_bits", C.c_int32)]
 
 
 _lib = None
@@ -136,7 +136,7 @@ class Shot:
     rec_component: int = 2
     snap_period: int = 1
     ckpt_period: int = 0         # RTM: 0 = all snapshots in HBM; c >= 1 = checkpointed segments of c
-    snap_fp16: int = 0           # RTM: 1 = fp16 snapshots scaled by a power of two (half the pool)
+    snap_bits: int = 32          # RTM snapshot precision: 32 (fp32) or 24 (3/4 of the pool, 2^-16 rounding)
 
     def c(self):
         w = np.ascontiguousarray(self.wavelet, dtype=np.float32)
@@ -144,7 +144,7 @@ class Shot:
         cs = _CShot(int(self.src[0]), int(self.src[1]), int(self.src[2]),
                     w.ctypes.data_as(C.POINTER(C.c_float)), w.shape[0], r.shape[0],
                     r.ctypes.data_as(C.POINTER(C.c_int32)), self.rec_component, self.snap_period,
-                    self.ckpt_period, self.snap_fp16)
+                    self.ckpt_period, self.snap_bits)
         return cs, (w, r)
 
     @property
@@ -216,21 +216,34 @@ class Comm:
         return bytes(buf)
 
     @classmethod
-    def from_torch_distributed(cls, device: int):
-        """Create from an initialised torch.distributed group (broadcasts the NCCL id)."""
+    def broadcast_unique_id(cls, group=None, device: Optional[int] = None) -> bytes:
+        """Rank 0 of the torch.distributed group draws the 128-byte NCCL unique id
+        (seis_comm_unique_id); every rank returns it (broadcast over the group's backend:
+        a CUDA tensor on `device` for nccl, a CPU tensor for gloo)."""
         import torch
         import torch.distributed as dist
 
-        rank, world = dist.get_rank(), dist.get_world_size()
+        rank = dist.get_rank(group)
         uid = cls.unique_id() if rank == 0 else bytes(128)
+        on_gpu = dist.get_backend(group) == "nccl"
         t = torch.tensor(list(uid), dtype=torch.uint8,
-                         device=f"cuda:{device}" if dist.get_backend() == "nccl" else "cpu")
-        dist.broadcast(t, 0)
-        return cls(world, rank, bytes(t.cpu().tolist()), device)
+                         device=f"cuda:{device if device is not None else torch.cuda.current_device()}"
+                         if on_gpu else "cpu")
+        dist.broadcast(t, 0, group=group)
+        return bytes(t.cpu().tolist())
+
+    @classmethod
+    def from_torch_distributed(cls, device: int, group=None):
+        """Create from an initialised torch.distributed group (broadcasts the NCCL id)."""
+        import torch.distributed as dist
+
+        uid = cls.broadcast_unique_id(group, device)
+        return cls(dist.get_world_size(group), dist.get_rank(group), uid, device)
 
     def reduce_image(self, image, stream=None):
         """Sum a device image over all ranks in place (shot-parallel RTM, sum_s of P:111)."""
-        _check(lib().seis_image_reduce(self.h, _ptr(image), image.numel(), _stream(stream)))
+        n = image.numel() if hasattr(image, "numel") else int(np.asarray(image).size)
+        _check(lib().seis_image_reduce(self.h, _ptr(image), n, _stream(stream)))
         return image
 
     def close(self):

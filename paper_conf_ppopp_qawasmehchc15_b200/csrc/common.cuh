@@ -17,7 +17,6 @@
 // slab face that touches a neighbour slab are the halo planes the exchange fills.
 #pragma once
 #include <cstdint>
-#include <cuda_fp16.h>
 #include <cuda_runtime.h>
 
 namespace seis {
@@ -279,17 +278,38 @@ __device__ __forceinline__ void st2_masked(float* p, const F2& a, int x0, int nx
 }
 }  // namespace seis
 
-// ------------------------------------------------------ fp16 snapshots (f2 alternative)
-// Imaging reads S_j either as fp32 (s32) or as fp16 scaled by a power of two (s16 * *scale,
-// the scale written by the snapshot kernel of that level, kernels_aux.cuh).
+// ------------------------------------------------------ 24-bit snapshots (f2 alternative)
+// Imaging reads S_j either as fp32 (s32) or in the 24-bit format of seis_shot.snap_bits = 24:
+// the fp32 value rounded to nearest-even at bit 8 (sign, the full 8-bit exponent, 15 mantissa
+// bits: relative rounding <= 2^-16), stored as a 16-bit high plane (h16) and an 8-bit low plane
+// (l8) of the same snapshot.  The value is a pure function of the fp32 value (no scale), so
+// images stay bitwise invariant under the z-slab decomposition and checkpointing.
 namespace seis {
+__device__ __forceinline__ uint32_t snap24_round(float v) {
+  const uint32_t u = __float_as_uint(v);
+  return u + 0x7Fu + ((u >> 8) & 1u);  // round to nearest even at bit 8 (then bits 0..7 drop)
+}
 struct SnapRef {
   const float* __restrict__ s32 = nullptr;
-  const __half* __restrict__ s16 = nullptr;
-  const float* __restrict__ scale = nullptr;
+  const uint16_t* __restrict__ h16 = nullptr;
+  const uint8_t* __restrict__ l8 = nullptr;
   __device__ __forceinline__ float at(long long i) const {
-    return s16 ? __half2float(s16[i]) * __ldg(scale) : __ldg(s32 + i);
+    if (h16) return __uint_as_float(((uint32_t)__ldg(h16 + i) << 16) | ((uint32_t)__ldg(l8 + i) << 8));
+    return __ldg(s32 + i);
   }
+};
+}  // namespace seis
+
+// ------------------------------------------------------ source amplitude (O11)
+// The injected sample of step n, scale * s[n]: s is the shot's wavelet, uploaded to the device
+// once per call (so a CUDA graph of the shot does not depend on the wavelet values), scale the
+// per-node factor of O3 / O8 / O11.  One fp32 product, as the host would form it.
+namespace seis {
+struct SrcAmp {
+  const float* __restrict__ w = nullptr;  // device [nt]
+  int n = 0;
+  float scale = 0.f;
+  __device__ __forceinline__ float get() const { return __fmul_rn(scale, __ldg(w + n)); }
 };
 }  // namespace seis
 

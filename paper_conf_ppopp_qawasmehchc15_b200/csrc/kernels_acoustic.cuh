@@ -66,7 +66,7 @@ struct AcVArgs {
   int zc;
   int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   const float* __restrict__ imgS; // imaging: img += S * p (input level), or nullptr
-  SnapRef imgR;                   // the same (fp32 or fp16), what the IMG kernel reads
+  SnapRef imgR;                   // the same (fp32 or 24-bit), what the IMG kernel reads
   float* __restrict__ img;
   Ghost gh;                       // direct ghost stores of q_z (f4)
 };
@@ -269,7 +269,7 @@ struct AcPArgs {
   int zc;
   int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   long long src_o;                // padded index of the source in this slab, -1 = none
-  float src_amp;                  // dt K_s / h^3 * s[n]
+  SrcAmp src;                     // dt K_s / h^3 * s[n]
   float* __restrict__ snap;       // compact snapshot target, or nullptr
   Ghost gh;                       // direct ghost stores of p (f4)
 };
@@ -417,7 +417,7 @@ __global__ void SEIS_AC_LB(NTX * BY) ac_p_kernel(const __grid_constant__ AcPArgs
       if (rel >= 0 && rel < 4) {
 #pragma unroll
         for (int e = 0; e < 4; ++e)
-          if (rel == e) out.v[e] += a.src_amp;
+          if (rel == e) out.v[e] += a.src.get();
       }
       st4_masked(a.p + o, out, x0, d.nx, true);
       ghost_st4(a.gh, o, k, d.nzl, out, x0, d.nx);

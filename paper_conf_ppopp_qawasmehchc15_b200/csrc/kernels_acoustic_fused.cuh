@@ -60,7 +60,7 @@ struct AcFArgs {
   int zc;
   int ch0, chs;
   long long src_o;
-  float src_amp;
+  SrcAmp src;
   float* __restrict__ snap;
   const float* __restrict__ imgS;
   float* __restrict__ img;
@@ -448,7 +448,7 @@ __global__ void __launch_bounds__(NTX * BY, BY <= 16 ? 2 : 1) ac_fused_kernel(co
       if (rel >= 0 && rel < 4) {
 #pragma unroll
         for (int e = 0; e < 4; ++e)
-          if (rel == e) out.v[e] += a.src_amp;
+          if (rel == e) out.v[e] += a.src.get();
       }
       st4_masked(a.p1 + o, out, x0, d.nx, true);
       if (SNAP) st4_masked(a.snap + ((long long)k * d.ny + j) * d.nx + x0, out, x0, d.nx, (d.nx & 3) == 0);

@@ -71,44 +71,22 @@ __global__ void inject_el_kernel(float* __restrict__ sxx, float* __restrict__ sy
   }
 }
 
-// fp16 snapshots (SURVEY §8f f2 alternative, seis_shot.snap_fp16): the snapshot field
-// S = c * (f0 + f1 + f2) (ISO / ACOUSTIC: f0 with c = 1; ELASTIC pressure: -(sxx+syy+szz)/3)
-// is stored as fp16(S / 2^e) with 2^e chosen from max|S| over the slab, so the largest value
-// sits near 2^15 (fp16 max 65504): relative rounding 2^-11, no overflow, scale exact.
+// 24-bit snapshots (SURVEY §8f f2's compressed-snapshot alternative, seis_shot.snap_bits = 24):
+// the snapshot field S = f0 (ISO / ACOUSTIC) or the pressure -(sxx+syy+szz)/3 (ELASTIC, the
+// el_s SNAP epilogue's expression) rounded to 24 bits (common.cuh snap24_round) and split into
+// the high 16 bits (hi) and the next 8 bits (lo) of the fp32 pattern: 3 bytes per value.
 __device__ __forceinline__ float snap_val(const float* f0, const float* f1, const float* f2, int nf, long long o) {
   return nf == 1 ? f0[o] : -((f0[o] + f1[o]) + f2[o]) / 3.0f;
 }
-// amax (uint bits of a non-negative float) = max |S| over the slab interior
-__global__ void snap_amax_kernel(unsigned* __restrict__ amax, const float* __restrict__ f0, const float* __restrict__ f1,
-                                 const float* __restrict__ f2, int nf, Dims d) {
-  const long long n = (long long)d.nzl * d.ny * d.nx;
-  float m = 0.0f;
-  for (long long t = blockIdx.x * (long long)blockDim.x + threadIdx.x; t < n; t += (long long)gridDim.x * blockDim.x) {
-    const int i = (int)(t % d.nx);
-    const long long r = t / d.nx;
-    m = fmaxf(m, fabsf(snap_val(f0, f1, f2, nf, d.at(i, (int)(r % d.ny), (int)(r / d.ny)))));
-  }
-#pragma unroll
-  for (int s = 16; s > 0; s >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, s));
-  if ((threadIdx.x & 31) == 0) atomicMax(amax, __float_as_uint(m));
-}
-// dst[t] = fp16(S / 2^e), *scale = 2^e with 2^e >= max / 2^15 (a power of two: exact)
-__global__ void snap_f16_kernel(__half* __restrict__ dst, float* __restrict__ scale, const unsigned* __restrict__ amax,
-                                const float* __restrict__ f0, const float* __restrict__ f1,
-                                const float* __restrict__ f2, int nf, Dims d) {
-  const float mx = __uint_as_float(*amax);
-  int e = 0;
-  if (mx > 0.0f) {
-    frexpf(mx, &e);  // mx = f 2^e, f in [0.5, 1)
-    e = max(e - 15, -126);  // mx / 2^e < 2^15 (clamped: 2^-e stays finite)
-  }
-  const float sc = ldexpf(1.0f, e), inv = ldexpf(1.0f, -e);
-  if (blockIdx.x == 0 && threadIdx.x == 0) *scale = sc;
+__global__ void snap24_kernel(uint16_t* __restrict__ hi, uint8_t* __restrict__ lo, const float* __restrict__ f0,
+                              const float* __restrict__ f1, const float* __restrict__ f2, int nf, Dims d) {
   const long long n = (long long)d.nzl * d.ny * d.nx;
   for (long long t = blockIdx.x * (long long)blockDim.x + threadIdx.x; t < n; t += (long long)gridDim.x * blockDim.x) {
     const int i = (int)(t % d.nx);
     const long long r = t / d.nx;
-    dst[t] = __float2half_rn(snap_val(f0, f1, f2, nf, d.at(i, (int)(r % d.ny), (int)(r / d.ny))) * inv);
+    const uint32_t u = snap24_round(snap_val(f0, f1, f2, nf, d.at(i, (int)(r % d.ny), (int)(r / d.ny))));
+    hi[t] = (uint16_t)(u >> 16);
+    lo[t] = (uint8_t)(u >> 8);
   }
 }
 

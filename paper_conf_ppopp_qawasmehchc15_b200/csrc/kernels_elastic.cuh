@@ -110,7 +110,7 @@ struct ElVArgs {
   int zc;
   int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   const float* __restrict__ imgS;  // elastic RTM (f3): img += S * P on the input level, P = -(sxx+syy+szz)/3
-  SnapRef imgR;                    // the same (fp32 or fp16), what the IMG kernel reads
+  SnapRef imgR;                    // the same (fp32 or 24-bit), what the IMG kernel reads
   float* __restrict__ img;
   Ghost gh[3];                     // direct ghost stores of vx, vy, vz (f4)
 };
@@ -353,7 +353,7 @@ struct ElSArgs {
   int zc;
   int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   long long src_o;
-  float src_amp;   // dt (lam + 2/3 mu)_s / h^3 * s[n]
+  SrcAmp src;      // dt (lam + 2/3 mu)_s / h^3 * s[n]
   float* __restrict__ snap;  // elastic RTM (f3): snapshot of P = -(sxx+syy+szz)/3, or nullptr
   Ghost gh[3];               // direct ghost stores of szz, sxz, syz (f4)
 };
@@ -569,9 +569,10 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
         float syy = sv[1].v[e] + fmaf(l2m, eyy[e], lam * (exx[e] + ez));
         float szz = sv[2].v[e] + fmaf(l2m, ez, lam * (exx[e] + eyy[e]));
         if (rel == e) {
-          sxx -= a.src_amp;
-          syy -= a.src_amp;
-          szz -= a.src_amp;
+          const float sa = a.src.get();
+          sxx -= sa;
+          syy -= sa;
+          szz -= sa;
         }
         if (surf) szz = 0.0f;
         o6[0].v[e] = sxx;

@@ -62,10 +62,10 @@ struct IsoArgs {
   int zc;                        // z-chunk length
   int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
   long long src_o;               // padded index of the source node in this slab, -1 = none
-  float src_amp;                 // scale * s[n]
+  SrcAmp src;                    // scale * s[n]
   float* __restrict__ snap;      // compact [nzl][ny][nx] or nullptr
   const float* __restrict__ imgS;// compact snapshot S_j for imaging, or nullptr
-  SnapRef imgR;                  // the same (fp32 or fp16), what the IMG kernels read
+  SnapRef imgR;                  // the same (fp32 or 24-bit), what the IMG kernels read
   float* __restrict__ img;       // compact image (+=), or nullptr
   Ghost gh;                      // direct ghost stores of u^{n+1} (f4)
   // split-field PML (O6b, SPML kernels): components u^(x), u^(y), u^(z) of the layer points,
@@ -328,8 +328,9 @@ __global__ void __launch_bounds__(NTX * BY, SPML ? SEIS_SPML_MINB : 1) iso_step_
 #pragma unroll
         for (int e = 0; e < 4; ++e)
           if (rel == e) {
-            out.v[e] += a.src_amp;
-            if (SPML && sidx[e] >= 0) a.sp[(long long)(1 - a.lvl) * 3 * a.spn + sidx[e]] += a.src_amp;  // x component
+            const float sa = a.src.get();
+            out.v[e] += sa;
+            if (SPML && sidx[e] >= 0) a.sp[(long long)(1 - a.lvl) * 3 * a.spn + sidx[e]] += sa;  // x component
           }
       }
       st4_masked(a.up + o, out, x0, d.nx, true);

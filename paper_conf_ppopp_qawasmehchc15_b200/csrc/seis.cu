@@ -208,14 +208,19 @@ struct seis_model {
   // staging buffers
   float* stage = nullptr;
   size_t stage_elems = 0;
-  float* scales = nullptr;  // fp16 snapshot scales + max words (seis_shot.snap_fp16)
-  size_t scales_elems = 0;
   float* pamp = nullptr;    // persistent small-grid ISO path: per-step source amplitudes
   int pamp_n = 0;
   const float* hwav = nullptr;  // host wavelet of the current call
+  float* dwav = nullptr;        // its device copy (uploaded by every call, read by the source add)
+  size_t dwav_n = 0;
   int last_nt = 0;
-  // shot-table cache and the CUDA graph of the last forward_model (single process)
-  uint64_t shot_key = 0;
+  // shot-table cache and the CUDA graph of the last forward_model.  The gather tables
+  // (d_rec_off / d_rec_id, captured by the graph) and the backward-injection groups have
+  // separate keys: a migrate between two forward_model calls rebuilds only the groups, and any
+  // rebuild of the gather tables destroys the graph that holds their pointers.
+  uint64_t fwd_key = 0, bwd_key = 0;
+  uint64_t shot_key = 0;              // fwd_key of the current call (part of the graph key)
+  std::vector<int> gcur;              // S.cur of every slab after the captured shot (replay)
   cudaStream_t cap = nullptr;       // capture stream (the legacy stream cannot be captured)
   cudaGraphExec_t gexec = nullptr;
   uint64_t gkey = 0;
@@ -800,17 +805,12 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
   int dev_sms = 148;
   CK(cudaDeviceGetAttribute(&dev_sms, cudaDevAttrMultiProcessorCount, M->device));
   if (ns > 1 || M->nranks > 1) {
-    // every internal slab boundary must keep the recomputed ghost planes (8 deep) out of the
-    // absorbing layers and each slab must hold the 8 planes its neighbours read
-    const int W = g.nb > 0 ? g.nb + 1 : 0;
+    // every slab must hold the 4 planes its neighbours read as ghosts
     for (int r = 0; r < M->nranks; ++r)
       for (int s = 0; s < ns; ++s) {
         int rz0, rn, lz0, ln;
         seis_slab_bounds(g.nz, M->nranks, r, &rz0, &rn);
         seis_slab_bounds(rn, ns, s, &lz0, &ln);
-        const int z0 = rz0 + lz0;
-        (void)W;
-        (void)z0;
         if (ln < 4) return fail(SEIS_EINVAL, "z-slab of %d planes: the decomposition needs >= 4", ln);
       }
   }
@@ -1214,7 +1214,7 @@ seis_status seis_memory_required(const seis_grid* g, seis_kind kind, const seis_
             (kind == SEIS_ACOUSTIC ? 2 : 6);
     }
     ck += spml;
-    b += (double)c * nzl * (double)g->ny * g->nx * (shot->snap_fp16 == 1 ? 2.0 : 4.0) + (double)nckpt * ck;
+    b += (double)c * nzl * (double)g->ny * g->nx * (shot->snap_bits == 24 ? 3.0 : 4.0) + (double)nckpt * ck;
   }
   *bytes = (uint64_t)b;
   return SEIS_OK;
@@ -1240,6 +1240,28 @@ int spml_index_host(const seis_model* M, const Slab& S, int x, int y, int z) {
   return S.spx + S.spy + ((z < nb ? z : z - (nz - 2 * nb)) * ny + y) * nx + x;
 }
 
+// Replace a tracked device buffer by a larger one (the old one is freed, not kept until the
+// model is destroyed).  A CUDA graph holding the old pointer is destroyed with it.
+seis_status regrow(seis_model* M, float** buf, size_t* have, size_t elems) {
+  if (*have >= elems) return SEIS_OK;
+  if (*buf) {
+    if (M->gexec) {
+      cudaGraphExecDestroy(M->gexec);
+      M->gexec = nullptr;
+    }
+    CK(cudaDeviceSynchronize());  // (no queued work may still use it)
+    cudaFree(*buf);
+    M->allocs.erase(std::find(M->allocs.begin(), M->allocs.end(), (void*)*buf));
+    *buf = nullptr;
+    *have = 0;
+  }
+  void* p = nullptr;
+  TRY(alloc_track(M, &p, elems * sizeof(float)));
+  *buf = (float*)p;
+  *have = elems;
+  return SEIS_OK;
+}
+
 struct ShotTables {
   std::vector<float*> owned;  // device allocations to free
 };
@@ -1260,14 +1282,23 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
   }
   if (M->kind == SEIS_ELASTIC && (sh->rec_component < 0 || sh->rec_component > 3))
     return fail(SEIS_EINVAL, "rec_component must be 0..3");
-  M->hwav = sh->wavelet;  // source amplitudes are kernel arguments (one fused add per step)
+  M->hwav = sh->wavelet;
+  // the wavelet is copied to the device on every call: the source add reads s[n] there, so a
+  // captured shot graph does not depend on the wavelet values (P:177 injection, O11)
+  TRY(regrow(M, &M->dwav, &M->dwav_n, (size_t)sh->nt));
+  CK(cudaMemcpyAsync(M->dwav, sh->wavelet, (size_t)sh->nt * sizeof(float), cudaMemcpyHostToDevice, st));
   // receiver tables are rebuilt only when the geometry changes (CUDA graphs keep pointers)
   uint64_t key = fnv1a(&sh->sx, 3 * sizeof(int32_t));
   key = fnv1a(&sh->nrec, sizeof(int32_t), key);
   if (sh->nrec) key = fnv1a(sh->rec, (size_t)sh->nrec * 3 * sizeof(int32_t), key);
   key = fnv1a(&sh->rec_component, sizeof(int32_t), key);
-  key ^= backward_injection ? 0x9e3779b97f4a7c15ULL : 0;
-  const bool same = key == M->shot_key;
+  key = key ? key : 1;  // (0 = "no tables yet")
+  const bool fwd_same = key == M->fwd_key;
+  const bool bwd_same = !backward_injection || key == M->bwd_key;
+  if (!fwd_same && M->gexec) {  // the graph holds the gather tables about to be freed
+    cudaGraphExecDestroy(M->gexec);
+    M->gexec = nullptr;
+  }
   const double h = g.h, dt = g.dt;
   auto point_scale = [&](int x, int y, int z) -> double {
     const size_t li = ((size_t)(z - M->pz0) * g.ny + y) * g.nx + x;
@@ -1293,7 +1324,7 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
       S.src_o = S.d.at(sh->sx, sh->sy, sh->sz - z0);
       S.src_scale = (float)point_scale(sh->sx, sh->sy, sh->sz);
     }
-    if (same) continue;
+    if (fwd_same && bwd_same) continue;
     // receivers owned by this slab
     std::vector<long long> off;
     std::vector<int> rid;
@@ -1304,14 +1335,22 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
         rid.push_back(r);
       }
     }
-    S.nrec_own = (int)off.size();
-    if (S.nrec_own > 0) {
-      if (S.d_rec_off) { cudaFree(S.d_rec_off); cudaFree(S.d_rec_id); }
-      CK(dmalloc(&S.d_rec_off, off.size()));
-      CK(dmalloc(&S.d_rec_id, rid.size()));
-      CK(cudaMemcpy(S.d_rec_off, off.data(), off.size() * sizeof(long long), cudaMemcpyHostToDevice));
-      CK(cudaMemcpy(S.d_rec_id, rid.data(), rid.size() * sizeof(int), cudaMemcpyHostToDevice));
+    if (!fwd_same) {  // gather tables (forward phase)
+      if (S.d_rec_off) {
+        cudaFree(S.d_rec_off);
+        cudaFree(S.d_rec_id);
+        S.d_rec_off = nullptr;
+        S.d_rec_id = nullptr;
+      }
+      S.nrec_own = (int)off.size();
+      if (S.nrec_own > 0) {
+        CK(dmalloc(&S.d_rec_off, off.size()));
+        CK(dmalloc(&S.d_rec_id, rid.size()));
+        CK(cudaMemcpy(S.d_rec_off, off.data(), off.size() * sizeof(long long), cudaMemcpyHostToDevice));
+        CK(cudaMemcpy(S.d_rec_id, rid.data(), rid.size() * sizeof(int), cudaMemcpyHostToDevice));
+      }
     }
+    if (bwd_same) continue;
     for (auto& G2 : S.grp) {
       if (G2.off) {
         cudaFree(G2.off); cudaFree(G2.scale); cudaFree(G2.start); cudaFree(G2.mem); cudaFree(G2.surf);
@@ -1319,7 +1358,7 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
       }
       G2 = Slab::Groups{};
     }
-    if (backward_injection && S.nrec_own > 0) {
+    if (!off.empty()) {
       // merge duplicates: group receivers by node, members in receiver-index order (O12)
       std::map<long long, std::vector<int>> groups;
       for (size_t t = 0; t < off.size(); ++t) groups[off[t]].push_back(rid[t]);
@@ -1357,6 +1396,8 @@ seis_status setup_shot(seis_model* M, const seis_shot* sh, bool backward_injecti
       }
     }
   }
+  M->fwd_key = key;
+  if (backward_injection) M->bwd_key = key;
   M->shot_key = key;
   return SEIS_OK;
 }
@@ -1544,8 +1585,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.ch0 = ch0;
       a.chs = chs;
       a.src_o = with_src ? S.src_o : -1;
-      a.src_amp = 0.f;
-      if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
+      a.src = SrcAmp{M->dwav, n, S.src_scale};
       a.snap = snap ? (*snap)[s] : nullptr;
       a.imgS = imgS ? (*imgS)[s].s32 : nullptr;
       if (imgS) a.imgR = (*imgS)[s];
@@ -1627,8 +1667,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.ch0 = ch0;
       a.chs = chs;
       a.src_o = with_src ? S.src_o : -1;
-      a.src_amp = 0.f;
-      if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
+      a.src = SrcAmp{M->dwav, n, S.src_scale};
       a.snap = snap ? (*snap)[s] : nullptr;
       a.imgS = imgS ? (*imgS)[s].s32 : nullptr;
       a.img = img ? (*img)[s] : nullptr;
@@ -1723,8 +1762,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       a.ch0 = ch0;
       a.chs = chs;
       a.src_o = with_src ? S.src_o : -1;
-      a.src_amp = 0.f;
-      if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
+      a.src = SrcAmp{M->dwav, n, S.src_scale};
       a.snap = snap ? (*snap)[s] : nullptr;
       a.gh = S.gh[0];
       const dim3 gr = grid_of(S, TXV, BYP, nch), blk(NTX, BYP);
@@ -1813,8 +1851,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     a.ch0 = ch0;
     a.chs = chs;
     a.src_o = with_src ? S.src_o : -1;
-    a.src_amp = 0.f;
-    if (a.src_o >= 0) a.src_amp = S.src_scale * M->hwav[n];
+    a.src = SrcAmp{M->dwav, n, S.src_scale};
     a.snap = snap ? (*snap)[s] : nullptr;
     a.gh[0] = S.gh[ESZZ];
     a.gh[1] = S.gh[ESXZ];
@@ -1859,29 +1896,13 @@ seis_status gather(seis_model* M, const seis_shot* sh, float* seis_dev, int n, c
   return SEIS_OK;
 }
 
-seis_status ensure_scales(seis_model* M, size_t elems) {
-  if (M->scales_elems >= elems) return SEIS_OK;
-  void* p = nullptr;
-  TRY(alloc_track(M, &p, elems * sizeof(float)));
-  M->scales = (float*)p;
-  M->scales_elems = elems;
-  return SEIS_OK;
-}
-
-seis_status ensure_stage(seis_model* M, size_t elems) {
-  if (M->stage_elems >= elems) return SEIS_OK;
-  void* p = nullptr;
-  TRY(alloc_track(M, &p, elems * sizeof(float)));
-  M->stage = (float*)p;
-  M->stage_elems = elems;
-  return SEIS_OK;
-}
+seis_status ensure_stage(seis_model* M, size_t elems) { return regrow(M, &M->stage, &M->stage_elems, elems); }
 
 }  // namespace
 
 // Small L2-resident ISO grids: the whole shot as one cooperative launch (iso_persist_kernel).
 bool persist_ok(const seis_model* M) {
-  if (M->kind != SEIS_ISO || M->slabs.size() != 1 || (M->comm && M->nranks > 1) || prof::on) return false;
+  if (M->kind != SEIS_ISO || M->slabs.size() != 1 || M->comm || prof::on) return false;
   const Slab& S = M->slabs[0];
   if (S.sp) return false;  // (the split-field PML keeps the z-march kernel)
   const char* e = getenv("SEIS_NO_PERSIST");
@@ -1947,8 +1968,9 @@ static seis_status forward_loop(seis_model* M, const seis_shot* sh, float* sd, s
     TRY(step(M, n, true, nullptr, nullptr, nullptr, st));
     if (sh->nrec) TRY(gather(M, sh, sd, n, st));
   }
-  // (a peer-only communicator has no NCCL: each rank returns its own receivers' columns)
-  if (M->comm && M->comm->nccl && M->nranks > 1 && ns)
+  // (a peer-only communicator has no NCCL: each rank returns its own receivers' columns; a
+  // 1-rank NCCL communicator runs the same all-reduce, an identity)
+  if (M->comm && M->comm->nccl && ns)
     NK(ncclAllReduce(sd, sd, ns, ncclFloat, ncclSum, M->comm->nccl, st));
   return SEIS_OK;
 }
@@ -1967,14 +1989,16 @@ seis_status seis_forward_model(seis_model* M, const seis_shot* sh, float* seis, 
     TRY(ensure_stage(M, ns));
     sd = M->stage;
   }
-  // Single process: the whole shot is one CUDA graph (captured once per shot setup and
-  // output buffer, replayed afterwards), so small grids are not launch-bound.
-  const bool use_graph = !prof::on && !(M->comm && M->nranks > 1) && !getenv("SEIS_NO_GRAPH");
+  // The whole shot is one CUDA graph (captured once per receiver geometry, output buffer and
+  // step count, replayed afterwards), so small grids and thin slabs are not launch-bound.  With
+  // an NCCL communicator the graph holds the halo send/recv groups (on the side stream of the
+  // overlapped exchange) and the seismogram all-reduce: every rank captures the same sequence
+  // of NCCL calls.  Peer halos (stream memory-operation flags) and profiling run eagerly.
+  const bool use_graph = !prof::on && !M->peer && !getenv("SEIS_NO_GRAPH");
   if (persist_ok(M)) {
     TRY(forward_persist(M, sh, sd, ns, st));
   } else if (use_graph) {
-    uint64_t key = fnv1a(sh->wavelet, (size_t)sh->nt * sizeof(float), M->shot_key);
-    key = fnv1a(&sd, sizeof(sd), key);
+    uint64_t key = fnv1a(&sd, sizeof(sd), M->shot_key);  // (the wavelet is read on the device)
     key = fnv1a(&sh->nt, sizeof(int32_t), key);
     if (!M->gexec || M->gkey != key) {
       if (M->gexec) {
@@ -2000,9 +2024,12 @@ seis_status seis_forward_model(seis_model* M, const seis_shot* sh, float* seis, 
       }
       M->gkey = key;
       M->g_launches = g_launches;
+      M->gcur.clear();  // the host bookkeeping the capture ran (final level of every slab)
+      for (Slab& S : M->slabs) M->gcur.push_back(S.cur);
     }
     CK(cudaGraphLaunch(M->gexec, st));
     g_launches = M->g_launches;
+    for (size_t s = 0; s < M->slabs.size(); ++s) M->slabs[s].cur = M->gcur[s];
   } else {
     TRY(forward_loop(M, sh, sd, ns, st));
   }
@@ -2033,10 +2060,11 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
   const int nckpt = nseg > 1 ? nseg - 1 : 0;
   const size_t slab_pts = (size_t)M->pnzl * g.ny * g.nx;
   const size_t st_elems = nckpt ? state_elems(M) : 0;
-  if (sh->snap_fp16 != 0 && sh->snap_fp16 != 1) return fail(SEIS_EINVAL, "snap_fp16 must be 0 or 1");
-  const bool f16 = sh->snap_fp16 == 1;
-  if (f16 && M->ac_fused) return fail(SEIS_EUNSUPPORTED, "fp16 snapshots with the fused acoustic step");
-  const size_t esz = f16 ? 2 : 4;  // bytes per snapshot value
+  if (sh->snap_bits != 0 && sh->snap_bits != 32 && sh->snap_bits != 24)
+    return fail(SEIS_EINVAL, "snap_bits must be 0, 32 or 24");
+  const bool s24 = sh->snap_bits == 24;
+  if (s24 && M->ac_fused) return fail(SEIS_EUNSUPPORTED, "24-bit snapshots with the fused acoustic step");
+  const size_t esz = s24 ? 3 : 4;  // bytes per snapshot value
   // (pool floats of the snapshot region, 256-byte aligned so the checkpoints stay aligned)
   const size_t snap_elems = ((size_t)std::min(c, nsnap) * slab_pts * esz + 255) / 256 * 64;
   const size_t need = snap_elems + (size_t)nckpt * st_elems;
@@ -2064,35 +2092,29 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
   auto slot_of = [&](int q) { return ckpt0 + (size_t)q * st_elems; };
   std::vector<int> ckpt_cur(nckpt, 0);  // ISO: which buffer holds u^n at the checkpoint
   // pool pointers of snapshot index i (j = (i + 1) snap), which lives in segment i / c
-  auto snap_ptrs = [&](int i, std::vector<float*>& v) {  // (byte addresses for fp16)
+  // snapshot i: fp32 [slab_pts] per snapshot, or (24-bit) a uint16 plane [slab_pts] followed by
+  // a uint8 plane [slab_pts]; each slab's part starts at its z offset within the plane(s)
+  auto snap_ptrs = [&](int i, std::vector<float*>& v) {
     const size_t off = (size_t)(i % c) * slab_pts;
     for (size_t s = 0; s < M->slabs.size(); ++s)
-      v[s] = (float*)((char*)M->pool + (off + (size_t)(M->slabs[s].d.z0 - M->pz0) * g.ny * g.nx) * esz);
+      v[s] = (float*)((char*)M->pool + (off + (size_t)(M->slabs[s].d.z0 - M->pz0) * g.ny * g.nx) * (s24 ? 2 : 4));
   };
-  // fp16: one power-of-two scale per (snapshot, slab) and one max word per slab
+  auto lo_plane = [&](int i, size_t s) {  // 24-bit: the uint8 plane of slab s of snapshot i
+    return (uint8_t*)M->pool + (size_t)c * slab_pts * 2 + (size_t)(i % c) * slab_pts +
+           (size_t)(M->slabs[s].d.z0 - M->pz0) * g.ny * g.nx;
+  };
   const size_t nsl = M->slabs.size();
-  float* scales = nullptr;
-  unsigned* amax = nullptr;
-  if (f16 && nsnap > 0) {
-    TRY(ensure_scales(M, (size_t)nsnap * nsl + nsl));
-    scales = M->scales;
-    amax = (unsigned*)(M->scales + (size_t)nsnap * nsl);
-  }
-  // store snapshot i (level (i + 1) snap) of the current state as fp16
-  auto snap16 = [&](int i) -> seis_status {
+  // store snapshot i (level (i + 1) snap) of the current state in the 24-bit format
+  auto snap24 = [&](int i) -> seis_status {
     std::vector<float*> dst(nsl);
     snap_ptrs(i, dst);
-    CK(cudaMemsetAsync(amax, 0, nsl * sizeof(unsigned), st));
     for (size_t s = 0; s < nsl; ++s) {
       Slab& S = M->slabs[s];
       const float* f0 = M->kind == SEIS_ELASTIC ? S.fld[ESXX] : out_field(M, S, 0);
       const float* f1 = M->kind == SEIS_ELASTIC ? S.fld[ESYY] : f0;
       const float* f2 = M->kind == SEIS_ELASTIC ? S.fld[ESZZ] : f0;
       const int nf = M->kind == SEIS_ELASTIC ? 3 : 1;
-      snap_amax_kernel<<<4 * 148, 256, 0, st>>>(amax + s, f0, f1, f2, nf, S.d);
-      CKL();
-      snap_f16_kernel<<<8 * 148, 256, 0, st>>>((__half*)dst[s], scales + (size_t)i * nsl + s, amax + s, f0, f1, f2,
-                                              nf, S.d);
+      snap24_kernel<<<8 * 148, 256, 0, st>>>((uint16_t*)dst[s], lo_plane(i, s), f0, f1, f2, nf, S.d);
       CKL();
     }
     return SEIS_OK;
@@ -2127,9 +2149,9 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
       const int j = n + 1;
       bool take = (j % snap == 0) && j <= nt - 1;
       if (take && (j / snap - 1) / c != seg) take = false;
-      if (take && !f16) snap_ptrs(j / snap - 1, snapp);
-      TRY(step(M, n, true, take && !f16 ? &snapp : nullptr, nullptr, nullptr, st));
-      if (take && f16) TRY(snap16(j / snap - 1));
+      if (take && !s24) snap_ptrs(j / snap - 1, snapp);
+      TRY(step(M, n, true, take && !s24 ? &snapp : nullptr, nullptr, nullptr, st));
+      if (take && s24) TRY(snap24(j / snap - 1));
     }
     return SEIS_OK;
   };
@@ -2172,9 +2194,9 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
       snap_ptrs(i, tmp);
       for (size_t s = 0; s < M->slabs.size(); ++s) {
         Sp[s] = SnapRef{};
-        if (f16) {
-          Sp[s].s16 = (const __half*)tmp[s];
-          Sp[s].scale = scales + (size_t)i * nsl + s;
+        if (s24) {
+          Sp[s].h16 = (const uint16_t*)tmp[s];
+          Sp[s].l8 = lo_plane(i, s);
         } else {
           Sp[s].s32 = tmp[s];
         }

@@ -87,22 +87,25 @@ def _undulation(nx, ny, scale):
     return 10.0 * scale * np.sin(2 * np.pi * x[None, :] / L) * np.cos(2 * np.pi * y[:, None] / L)
 
 
-def layered_acoustic(nx, ny, nz, scale=None):
+def layered_acoustic(nx, ny, nz, scale=None, z0=0, nzl=None):
     """C2 recipe: interfaces at z = 40,120,220,320,420 (of 512, scaled to nz) with
     undulation 10 sin(2 pi x/256) cos(2 pi y/256) points; vp = 1500 (water, rho 1000),
-    1800, 2200, 2700, 3200, 3800; Gardner density below the water."""
+    1800, 2200, 2700, 3200, 3800; Gardner density below the water.
+    z0, nzl: generate only the planes [z0, z0 + nzl) of the nz-deep model (one rank's z-slab;
+    each plane depends on its global z only, so slabs concatenate to the whole model)."""
     s = nz / 512.0 if scale is None else scale
+    nzl = nz - z0 if nzl is None else nzl
     iface = [40, 120, 220, 320, 420]
     vps = [1500.0, 1800.0, 2200.0, 2700.0, 3200.0, 3800.0]
     und = _undulation(nx, ny, s)  # [ny][nx]
-    vp = np.empty((nz, ny, nx), dtype=np.float32)
-    rho = np.empty((nz, ny, nx), dtype=np.float32)
+    vp = np.empty((nzl, ny, nx), dtype=np.float32)
+    rho = np.empty((nzl, ny, nx), dtype=np.float32)
     table = np.asarray(vps, dtype=np.float32)
     depth = [zi * s + und for zi in iface]
-    for k in range(nz):  # plane by plane (bounded host memory at 1024^3)
+    for k in range(nzl):  # plane by plane (bounded host memory at 1024^3)
         layer = np.zeros((ny, nx), dtype=np.int32)
         for dz in depth:
-            layer += (float(k) >= dz).astype(np.int32)
+            layer += (float(z0 + k) >= dz).astype(np.int32)
         vp[k] = table[layer]
         rho[k] = gardner(vp[k])
         rho[k][layer == 0] = 1000.0
@@ -210,15 +213,16 @@ def c1(n=64, nt=200, nb=0):
                     homogeneous((n, n, n), 2000.0))
 
 
-def c2(n=512, nt=2000, nb=20):
+def c2(n=512, nt=2000, nb=20, model=True):
     """C2: acoustic layered n^3, 2000 steps of 0.8 ms, C-PML (6 faces), Ricker 10 Hz at
-    (n/2, n/2, 24 s), receiver line z = 24 s, y = n/2, x = 20 s .. n-21 s."""
+    (n/2, n/2, 24 s), receiver line z = 24 s, y = n/2, x = 20 s .. n-21 s.
+    model=False: geometry only (the caller builds the model, e.g. one z-slab per rank)."""
     s = n / 512.0
     zr = max(nb + 1, int(round(24 * s)))
     x0, x1 = int(round(20 * s)), n - 1 - int(round(20 * s))
     rec = _line_x(x0, x1, n // 2, zr)
     return Workload("C2", "acoustic", n, n, n, 10.0, 8e-4, nt, nb, 10.0, (n // 2, n // 2, zr), rec,
-                    layered_acoustic(n, n, n))
+                    layered_acoustic(n, n, n) if model else {})
 
 
 def c3(n=384, nt=1500, nb=20):

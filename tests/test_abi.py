@@ -139,15 +139,15 @@ def test_iso_split_pml_rejected_for_other_kinds():
     assert e.value.name == "SEIS_EUNSUPPORTED"
 
 
-def test_memory_required_fp16_snapshots_halve_the_pool():
+def test_memory_required_24bit_snapshots():
     import numpy as np
 
     g = seis.Grid(128, 96, 64, 10.0, 8e-4, nb=10)
     sh = seis.Shot((1, 1, 1), np.zeros(201, np.float32), np.zeros((1, 3), np.int32), snap_period=20)
-    sh16 = seis.Shot((1, 1, 1), np.zeros(201, np.float32), np.zeros((1, 3), np.int32), snap_period=20,
-                     snap_fp16=1)
+    sh24 = seis.Shot((1, 1, 1), np.zeros(201, np.float32), np.zeros((1, 3), np.int32), snap_period=20,
+                     snap_bits=24)
     m0 = seis.memory_required(g, "acoustic")
-    assert seis.memory_required(g, "acoustic", sh16) - m0 == 10 * 128 * 96 * 64 * 2
+    assert seis.memory_required(g, "acoustic", sh24) - m0 == 10 * 128 * 96 * 64 * 3
     assert seis.memory_required(g, "acoustic", sh) - m0 == 10 * 128 * 96 * 64 * 4
 
 

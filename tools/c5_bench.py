@@ -73,7 +73,7 @@ def main():
     ap.add_argument("--nt", type=int, default=1000)
     ap.add_argument("--short", type=int, default=100, help="steps of the decomposition runs")
     ap.add_argument("--out", default=None)
-    ap.add_argument("--no-fp16", action="store_true", help="skip the fp16-snapshot RTM run")
+    ap.add_argument("--no-24", action="store_true", help="skip the 24-bit-snapshot RTM run")
     a = ap.parse_args()
     dev = torch.device("cuda", 0)
     stream = torch.cuda.current_stream()
@@ -104,27 +104,34 @@ def main():
     nsnap = (wl.nt - 1) // wl.snap
     need_all = seis.memory_required(g, "acoustic", shot)
     img_bytes = npts * 4 + data.numel() * 4
-    c = 0
-    if need_all + img_bytes > 0.97 * free:
-        # smallest pool: c ~ sqrt(nsnap * checkpoint / snapshot), then the largest c that fits
+
+    def choose_c(bits):
+        """0 if every snapshot fits, else the largest checkpoint segment length that fits."""
+        if seis.memory_required(g, "acoustic", seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap,
+                                                         snap_bits=bits)) + img_bytes <= 0.95 * free:
+            return 0
         best = None
         for cc in range(1, nsnap + 1):
             need = seis.memory_required(g, "acoustic", seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap,
-                                                                 ckpt_period=cc))
+                                                                 ckpt_period=cc, snap_bits=bits))
             if need + img_bytes <= 0.95 * free:
                 best = cc if best is None else max(best, cc)
         if best is None:
             raise SystemExit("C5 RTM does not fit even with checkpointing")
-        c = best
+        return best
+
+    def recomputed(c):
+        if not c:
+            return 0, 1
+        nseg = (nsnap + c - 1) // c
+        return sum(min((s + 1) * c, nsnap) * wl.snap - s * c * wl.snap for s in range(nseg - 1)), nseg
+
+    c = choose_c(32)
     rshot = seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap, ckpt_period=c)
     mig = seis.Model(g, "acoustic", sm["vp"], rho=sm["rho"], device=0)
     img = torch.zeros((wl.nz, wl.ny, wl.nx), device=dev)
     ms = timed(lambda: mig.migrate(rshot, data, img, stream), stream, reps=1, warm=1)
-    nseg = (nsnap + c - 1) // c if c else 1
-    recompute_steps = 0
-    if c:
-        for s in range(nseg - 1):
-            recompute_steps += min((s + 1) * c, nsnap) * wl.snap - s * c * wl.snap
+    recompute_steps, nseg = recomputed(c)
     res["rtm"] = {"shots_per_hour": round(3600.0 / (ms * 1e-3), 1), "ms_per_shot": round(ms, 1),
                   "gpts_s_both_phases": round(2 * npts * wl.nt / (ms * 1e-3) / 1e9, 2),
                   "gpts_s_all_steps": round(npts * (2 * wl.nt + recompute_steps) / (ms * 1e-3) / 1e9, 2),
@@ -132,24 +139,27 @@ def main():
                   "pool_bytes": int(seis.memory_required(g, "acoustic", rshot) - seis.memory_required(g, "acoustic")),
                   "all_snapshots_would_need_bytes": int(need_all), "free_bytes_before": int(free),
                   "image_norm": float(img.norm().item())}
-    # 2b. all 49 snapshots in HBM as fp16 (seis_shot.snap_fp16, opt-in): no recomputation; the
-    # pool of 2a is reused (half the bytes per snapshot)
-    if not a.no_fp16:
-        sh16 = seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap, snap_fp16=1)
-        img16 = torch.zeros_like(img)
-        ms16 = timed(lambda: (img16.zero_(), mig.migrate(sh16, data, img16, stream)), stream, reps=1, warm=0)
+    # 2b. 24-bit snapshots (seis_shot.snap_bits = 24, opt-in): 3/4 of the pool, so fewer (or no)
+    # recomputed segments; bitwise decomposition-invariant, ~1e-5 from the fp32-snapshot image
+    if not a.no_24:
+        c24 = choose_c(24)
+        sh24 = seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap, ckpt_period=c24, snap_bits=24)
+        img24 = torch.zeros_like(img)
+        ms24 = timed(lambda: (img24.zero_(), mig.migrate(sh24, data, img24, stream)), stream, reps=1, warm=0)
         num = den = 0.0
-        # (img holds the sum of 2a's warm-up and timed calls = 2 I exactly; img16 one call)
+        # (img holds the sum of 2a's warm-up and timed calls = 2 I exactly; img24 one call)
         for z0 in range(0, wl.nz, 64):  # slab-wise norms (no 4 GiB temporary)
             ref = 0.5 * img[z0:z0 + 64]
-            num += float(torch.linalg.vector_norm(img16[z0:z0 + 64] - ref).item()) ** 2
+            num += float(torch.linalg.vector_norm(img24[z0:z0 + 64] - ref).item()) ** 2
             den += float(torch.linalg.vector_norm(ref).item()) ** 2
-        res["rtm_fp16_snapshots"] = {
-            "shots_per_hour": round(3600.0 / (ms16 * 1e-3), 1), "ms_per_shot": round(ms16, 1),
-            "gpts_s_both_phases": round(2 * npts * wl.nt / (ms16 * 1e-3) / 1e9, 2),
-            "pool_bytes": int(seis.memory_required(g, "acoustic", sh16) - seis.memory_required(g, "acoustic")),
+        r24, nseg24 = recomputed(c24)
+        res["rtm_24bit_snapshots"] = {
+            "shots_per_hour": round(3600.0 / (ms24 * 1e-3), 1), "ms_per_shot": round(ms24, 1),
+            "gpts_s_both_phases": round(2 * npts * wl.nt / (ms24 * 1e-3) / 1e9, 2),
+            "ckpt_period": c24, "segments": nseg24, "recomputed_steps": r24,
+            "pool_bytes": int(seis.memory_required(g, "acoustic", sh24) - seis.memory_required(g, "acoustic")),
             "image_rel_l2_vs_fp32": round((num / den) ** 0.5, 7)}
-        del img16
+        del img24
     mig.close()
     del mig, img
     torch.cuda.empty_cache()
