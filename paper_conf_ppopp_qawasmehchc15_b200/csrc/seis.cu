@@ -23,7 +23,7 @@
 #include "../../include/seis.h"
 #include "common.cuh"
 #include "kernels_acoustic.cuh"
-#include "kernels_acoustic_fused.cuh"
+#include "kernels_acoustic_step.cuh"
 #include "kernels_aux.cuh"
 #include "kernels_elastic.cuh"
 #include "kernels_iso.cuh"
@@ -33,6 +33,8 @@ using namespace seis;
 // ------------------------------------------------------------------ errors
 static thread_local std::string g_err;
 static thread_local long long g_launches = 0;
+static unsigned long long* g_trace = nullptr;  // SEIS_AS_TRACE builds: fused-step event buffer
+static size_t g_trace_n = 0;
 
 static seis_status fail(seis_status st, const char* fmt, ...) {
   char buf[1024];
@@ -75,7 +77,7 @@ static seis_status fail(seis_status st, const char* fmt, ...) {
 // Per-kernel CUDA-event timing (seis_profile / seis_profile_read): an event pair
 // recorded on the launching stream around every launch of a stencil / aux kernel.
 namespace prof {
-constexpr int NK = 9;
+constexpr int NK = 10;
 static bool on = false;
 static std::vector<cudaEvent_t> ev[NK];  // start, stop, start, stop, ...
 static size_t used[NK] = {};
@@ -126,10 +128,6 @@ constexpr int BYI = SEIS_BYI;  // ISO step (block 16 x BYI threads, 4 x-points e
 constexpr int BYV = SEIS_BYV;  // acoustic V (block 16 x BYV)
 constexpr int BYP = SEIS_BYP;  // acoustic P (block 16 x BYP)
 constexpr int BYE = SEIS_BYE;
-#ifndef SEIS_BYF
-#define SEIS_BYF 16
-#endif
-constexpr int BYF = SEIS_BYF;  // fused acoustic step (block 16 x BYF, 4 x-points each)  // elastic V and S (block 32 x BYE threads, 2 x-points each)
 constexpr int NPSI = 18;
 
 struct Slab {
@@ -147,8 +145,8 @@ struct Slab {
   CUtensorMap ac_qxt, ac_qyt, ac_ppc, ac_qzc, ac_kc;        // ACOUSTIC P
   CUtensorMap el_sxxt, el_sxyt, el_sxzt, el_syyt, el_syzt, el_vc[3], el_rt, el_rc;  // ELASTIC V
   CUtensorMap el_vt[3], el_sc[6], el_l2m, el_w;                           // ELASTIC S
-  CUtensorMap af_pt[2], af_qx[2], af_qy[2], af_qz[2], af_pz[2], af_rt, af_rz, af_k;  // ACOUSTIC fused
-  int cur = 0;               // ISO: fld[cur] = u^n; fused ACOUSTIC: fld[4 cur .. 4 cur + 3] = p, q
+  CUtensorMap as_pt, as_q[3], as_rt, as_rz, as_pq, as_qxn, as_qyn, as_k;  // ACOUSTIC fused step
+  int cur = 0;               // ISO: fld[cur] = u^n
   int zc = 1, nzch = 1;      // z-chunking of the stencil launches
   // shot tables
   long long src_o = -1;
@@ -228,7 +226,11 @@ struct seis_model {
   cudaStream_t xs = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   bool no_overlap = false;  // SEIS_NO_OVERLAP=1: serial exchange (A/B measurements)
-  bool ac_fused = false;    // ACOUSTIC: single-sweep fused V+P step (double-buffered state)
+  // ACOUSTIC fused step (f1, kernels_acoustic_step.cuh): one persistent launch per time step,
+  // one CTA per 64 x 32 tile, all co-resident; ntx x nty tiles, per-tile progress counters
+  bool ac_step = false;
+  int as_ntx = 0, as_nty = 0;
+  unsigned* as_cnt = nullptr;
   long long g_launches = 0;
   // f4 direct ghost stores: `direct` = the faces between the slabs of this
   // process are written by the producing kernels (no copies); `peer` = the rank faces too,
@@ -386,9 +388,9 @@ seis_status set_smem_attrs() {
   SMEM_ATTR((ac_v_kernel<BYV, true>), AcVStage<BYV>::smem_bytes());
   SMEM_ATTR((ac_p_kernel<BYP, false>), AcPStage<BYP>::smem_bytes());
   SMEM_ATTR((ac_p_kernel<BYP, true>), AcPStage<BYP>::smem_bytes());
-  SMEM_ATTR((ac_fused_kernel<BYF, false, false>), AcFStage<BYF>::smem_bytes());
-  SMEM_ATTR((ac_fused_kernel<BYF, true, false>), AcFStage<BYF>::smem_bytes());
-  SMEM_ATTR((ac_fused_kernel<BYF, false, true>), AcFStage<BYF>::smem_bytes());
+  SMEM_ATTR((ac_step_kernel<false, false>), AcSLayout::smem_bytes());
+  SMEM_ATTR((ac_step_kernel<true, false>), AcSLayout::smem_bytes());
+  SMEM_ATTR((ac_step_kernel<false, true>), AcSLayout::smem_bytes());
   SMEM_ATTR((el_v_kernel<BYE, false>), ElVStage<BYE>::smem_bytes());
   SMEM_ATTR((el_v_kernel<BYE, true>), ElVStage<BYE>::smem_bytes());
   SMEM_ATTR((el_s_kernel<BYE, false>), ElSStage<BYE>::smem_bytes());
@@ -435,8 +437,8 @@ void choose_chunks(Slab& s, int resident_per_sm, int nsm, int tw, int by, int zt
   }
 }
 
-int nfields(seis_kind k, bool fused = true) { return k == SEIS_ISO ? 2 : (k == SEIS_ACOUSTIC ? (fused ? 8 : 4) : 9); }
-int npsi_of(seis_kind k, bool fused = true) { return k == SEIS_ACOUSTIC ? (fused ? 9 : 6) : (k == SEIS_ELASTIC ? 18 : 0); }
+int nfields(seis_kind k) { return k == SEIS_ISO ? 2 : (k == SEIS_ACOUSTIC ? 4 : 9); }
+int npsi_of(seis_kind k) { return k == SEIS_ACOUSTIC ? 6 : (k == SEIS_ELASTIC ? 18 : 0); }
 // axis of each C-PML memory array: ACOUSTIC psi_p (x,y,z), psi_q (x,y,z); ELASTIC in the
 // oracle's order
 int psi_axis(seis_kind k, int t) {
@@ -585,6 +587,14 @@ seis_status seis_profile_read(int32_t kernel, double* total_ms, int64_t* launche
 }
 const char* seis_last_error(void) { return g_err.c_str(); }
 int64_t seis_last_launch_count(void) { return (int64_t)g_launches; }
+#if SEIS_AS_TRACE
+// trace builds only (tools/ac_step_trace.py): the fused step's event buffer of the last launch
+void* seis_debug_trace(uint64_t* n) {
+  cudaDeviceSynchronize();
+  *n = g_trace_n;
+  return g_trace;
+}
+#endif
 
 seis_status seis_slab_bounds(int32_t nz, int32_t nranks, int32_t rank, int32_t* z0,
                              int32_t* nz_local) {
@@ -814,20 +824,6 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
         if (ln < 4) return fail(SEIS_EINVAL, "z-slab of %d planes: the decomposition needs >= 4", ln);
       }
   }
-  // fused acoustic step (f1) with SEIS_AC_FUSED=1 -- slower than the split pair on B200 so
-  // far, kept as the measured alternative -- unless a z-slab is thinner than
-  // the 8 ghost planes of p it exchanges
-  if (kind == SEIS_ACOUSTIC) {
-    const char* e = getenv("SEIS_AC_FUSED");
-    M->ac_fused = e && e[0] == '1';
-    for (int r = 0; r < M->nranks && (ns > 1 || M->nranks > 1); ++r)
-      for (int s = 0; s < ns; ++s) {
-        int rz0, rn, lz0, ln;
-        seis_slab_bounds(g.nz, M->nranks, r, &rz0, &rn);
-        seis_slab_bounds(rn, ns, s, &lz0, &ln);
-        if (ln < 8) M->ac_fused = false;
-      }
-  }
   M->slabs.resize(ns);
   for (int s = 0; s < ns; ++s) {
     int lz0, lnz;
@@ -837,7 +833,7 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     const Dims& d = S.d;
     const size_t sp = (size_t)lnz * plane;  // slab points
     const size_t off = (size_t)lz0 * plane;
-    S.fld.resize(nfields(kind, M->ac_fused));
+    S.fld.resize(nfields(kind));
     for (auto& f : S.fld) TRY(alloc_padded(M, d, &f, st));
     // per-point coefficients (double -> fp32), compact then padded on device
     std::vector<float> hc(sp);
@@ -887,7 +883,7 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
         const int W = M->W;
         const double big = std::max((double)lnz * g.ny, std::max((double)lnz * g.nx, (double)g.ny * g.nx)) * 2.0 * W;
         if (big >= 2147483647.0) return fail(SEIS_EUNSUPPORTED, "C-PML slab of %.0f points exceeds 32-bit indexing", big);
-        const int npsi = npsi_of(kind, M->ac_fused);
+        const int npsi = npsi_of(kind);
         for (int t = 0; t < npsi; ++t) {
           const int ax = psi_axis(kind, t);
           size_t n;
@@ -918,18 +914,15 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       TRY(make_map(&S.ac_ppc, S.fld[0], d, TXV, BYP));
       TRY(make_map(&S.ac_qzc, S.fld[3], d, TXV, BYP));
       TRY(make_map(&S.ac_kc, S.kdt, d, TXV, BYP));
-      if (M->ac_fused) {
-        for (int c = 0; c < 2; ++c) {
-          TRY(make_map(&S.af_pt[c], S.fld[4 * c], d, TXV + 16, BYF + 16));
-          TRY(make_map(&S.af_qx[c], S.fld[4 * c + 1], d, TXV + 8, BYF));
-          TRY(make_map(&S.af_qy[c], S.fld[4 * c + 2], d, TXV, BYF + 8));
-          TRY(make_map(&S.af_qz[c], S.fld[4 * c + 3], d, TXV, BYF));
-          TRY(make_map(&S.af_pz[c], S.fld[4 * c], d, TXV, BYF));
-        }
-        TRY(make_map(&S.af_rt, S.rho, d, TXV + 12, BYF + 9));
-        TRY(make_map(&S.af_rz, S.rho, d, TXV, BYF));
-        TRY(make_map(&S.af_k, S.kdt, d, TXV, BYF));
-      }
+      // fused step tiles (AS_TX x AS_TY; kernels_acoustic_step.cuh)
+      TRY(make_map(&S.as_pt, S.fld[0], d, AS_TX + 8, AS_TY + 8));
+      for (int t = 0; t < 3; ++t) TRY(make_map(&S.as_q[t], S.fld[1 + t], d, AS_TX, AS_TY));
+      TRY(make_map(&S.as_rt, S.rho, d, AS_TX + 4, AS_TY + 1));
+      TRY(make_map(&S.as_rz, S.rho, d, AS_TX, AS_TY));
+      TRY(make_map(&S.as_pq, S.fld[0], d, AS_TX, AS_TY));
+      TRY(make_map(&S.as_qxn, S.fld[1], d, AS_TX + 8, AS_TY));
+      TRY(make_map(&S.as_qyn, S.fld[2], d, AS_TX, AS_TY + 8));
+      TRY(make_map(&S.as_k, S.kdt, d, AS_TX, AS_TY));
     } else {
       TRY(make_map(&S.el_sxxt, S.fld[ESXX], d, TXE + 8, BYE));
       TRY(make_map(&S.el_sxyt, S.fld[ESXY], d, TXE + 8, BYE + 8));
@@ -951,27 +944,48 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     if (kind == SEIS_ISO)
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, iso_step_kernel<BYI, false, false>, NTX * BYI,
                                                     IsoStage<BYI>::smem_bytes());
-    else if (kind == SEIS_ACOUSTIC && M->ac_fused)
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_fused_kernel<BYF, false, false>, NTX * BYF,
-                                                    AcFStage<BYF>::smem_bytes());
     else if (kind == SEIS_ACOUSTIC)
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_v_kernel<BYV, false>, NTX * BYV,
                                                     AcVStage<BYV>::smem_bytes());
     else
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, NTX2 * BYE,
                                                     ElSStage<BYE>::smem_bytes());
-    const int zex = (ns > 1 || M->nranks > 1) ? (M->ac_fused ? 8 : 4) : 0;
+    const int zex = (ns > 1 || M->nranks > 1) ? 4 : 0;
     if (kind == SEIS_ELASTIC) choose_chunks(S, occ, dev_sms, TXE, BYE, 16, zex);
     else if (kind == SEIS_ISO) choose_chunks(S, occ, dev_sms, TXV, BYI, 24, zex);
-    else choose_chunks(S, occ, dev_sms, TXV, M->ac_fused ? BYF : BYV, M->ac_fused ? 64 : 16,
-                       M->ac_fused ? 8 : zex);  // (the fused step keeps >= 8-plane chunks)
+    else choose_chunks(S, occ, dev_sms, TXV, BYV, 16, zex);
+  }
+  // f1: the fused acoustic step (kernels_acoustic_step.cuh) on a single-slab, single-process
+  // model whose tiles can all be resident at once (cooperative launch), by default when there
+  // are enough tiles to occupy half the SMs (C2 / C4: 4 x 37 = 148 tiles); SEIS_AC_STEP=1 / 0
+  // forces it on (if the tiles fit) / off.  Bitwise the split pair's results (tested).
+#ifndef AS_DEFAULT_ON
+#define AS_DEFAULT_ON 0
+#endif
+  if (kind == SEIS_ACOUSTIC && ns == 1 && !M->comm) {
+    const int ntx = (g.nx + AS_TX - 1) / AS_TX, nty = (g.ny + AS_TY - 1) / AS_TY;
+    int occ_s = 0, coop = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_s, ac_step_kernel<false, false>, AS_THREADS,
+                                                     AcSLayout::smem_bytes()));
+    CK(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, M->device));
+    const bool fits = coop && occ_s >= 1 && (long long)ntx * nty <= (long long)occ_s * dev_sms;
+    const char* e = getenv("SEIS_AC_STEP");
+    const bool want = e ? e[0] == '1' : (AS_DEFAULT_ON && 2LL * ntx * nty >= dev_sms);
+    M->ac_step = fits && want;
+    if (M->ac_step) {
+      M->as_ntx = ntx;
+      M->as_nty = nty;
+      void* p = nullptr;
+      TRY(alloc_track(M, &p, (size_t)ntx * nty * sizeof(unsigned)));
+      M->as_cnt = (unsigned*)p;
+    }
   }
   // f4: the faces between the slabs of this process by direct ghost stores of the producing
   // kernels (SEIS_GHOST_COPY=1 keeps the copy exchange, the A/B alternative).  Not for the
   // fused acoustic step, which exchanges 8 ghost planes of p.
   {
     const char* e = getenv("SEIS_GHOST_COPY");
-    M->direct = ns > 1 && !M->ac_fused && !(e && e[0] == '1');
+    M->direct = ns > 1 && !(e && e[0] == '1');
     for (int s = 0; M->direct && s < ns; ++s) {
       Slab& S = M->slabs[s];
       for (size_t f = 0; f < S.fld.size() && f < 9; ++f) {
@@ -1096,7 +1110,6 @@ seis_status seis_model_peer_export(seis_model* M, uint8_t* blob, uint64_t cap, u
   if (cap < sizeof(PeerBlob)) return fail(SEIS_EINVAL, "blob capacity %llu < %zu", (unsigned long long)cap, sizeof(PeerBlob));
   if (!M->comm || M->nranks < 2 || M->slabs.size() != 1)
     return fail(SEIS_EINVAL, "peer halo needs a multi-rank model (one slab per rank)");
-  if (M->ac_fused) return fail(SEIS_EUNSUPPORTED, "peer halo with the fused acoustic step (SEIS_AC_FUSED=1)");
   CK(cudaSetDevice(M->device));
   if (!M->flags) {
     void* f = nullptr;
@@ -1190,8 +1203,8 @@ seis_status seis_memory_required(const seis_grid* g, seis_kind kind, const seis_
   seis_slab_bounds(g->nz, nranks, 0, &z0, &nzl);
   const Dims d = make_dims(*g, 0, nzl);
   const double padded = (double)d.PS * (nzl + 2 * GZ) * 4.0;
-  // (the default split acoustic step: 4 fields, psi_p + psi_q; SEIS_AC_FUSED=1 doubles p, q, psi_p)
-  int nf = nfields(kind, false), np = kind == SEIS_ISO ? 1 : (kind == SEIS_ACOUSTIC ? 2 : 3);  // m | kdt,rho | l2m,w,rho
+  // (acoustic: 4 fields, psi_p + psi_q, split pair and fused step alike)
+  int nf = nfields(kind), np = kind == SEIS_ISO ? 1 : (kind == SEIS_ACOUSTIC ? 2 : 3);  // m | kdt,rho | l2m,w,rho
   double b = (nf + np) * padded;
   double spml = 0.0;  // ISO O6b split components (6 per layer point, compact slabs)
   if (kind == SEIS_ISO && g->iso_pml && g->nb > 0)
@@ -1411,7 +1424,7 @@ seis_status zero_state(seis_model* M, cudaStream_t st) {
     if (S.sp) CK(cudaMemsetAsync(S.sp, 0, (size_t)S.spn * 6 * sizeof(float), st));
     if (M->W > 0) {
       const int W = M->W;
-      const int npsi = npsi_of(M->kind, M->ac_fused);
+      const int npsi = npsi_of(M->kind);
       for (int t = 0; t < npsi; ++t) {
         const int ax = psi_axis(M->kind, t);
         size_t n;
@@ -1432,16 +1445,11 @@ std::vector<std::pair<float*, size_t>> state_arrays(seis_model* M) {
   std::vector<std::pair<float*, size_t>> v;
   for (Slab& S : M->slabs) {
     const size_t elems = (size_t)S.d.PS * (S.d.nzl + 2 * GZ) + 32;  // + the 128-byte alignment pad
-    // fused ACOUSTIC: only the current set (fields, psi_p) and psi_q hold state
-    const bool fz = M->ac_fused;
-    for (size_t f = 0; f < S.fld.size(); ++f)
-      if (!fz || (int)f / 4 == S.cur) v.emplace_back(S.fld[f] - 28, elems);  // base = f - 112 bytes
+    for (size_t f = 0; f < S.fld.size(); ++f) v.emplace_back(S.fld[f] - 28, elems);  // base = f - 112 bytes
     if (S.sp) v.emplace_back(S.sp, (size_t)S.spn * 6);  // ISO O6b split components
     if (M->W > 0) {
       const int W = M->W;
-      for (int t = 0; t < npsi_of(M->kind, fz); ++t) {
-        if (fz && t < 3 && S.cur != 0) continue;
-        if (fz && t >= 6 && S.cur != 1) continue;
+      for (int t = 0; t < npsi_of(M->kind); ++t) {
         const int ax = psi_axis(M->kind, t);
         size_t n;
         if (ax == 0) n = (size_t)S.d.nzl * S.d.ny * 2 * W;
@@ -1492,7 +1500,7 @@ seis_status inject_rows(seis_model* M, const float* row, int part, cudaStream_t 
                                                             G2.scale, G2.start, G2.mem, row, G2.surf, G2.n,
                                                             S.gh[ESZZ], S.d.PS, S.d.nzl);
       } else {
-        const int f = M->kind == SEIS_ISO ? S.cur : 4 * S.cur;
+        const int f = M->kind == SEIS_ISO ? S.cur : 0;
         inject_kernel<<<(G2.n + 127) / 128, 128, 0, st>>>(S.fld[f], G2.off, G2.scale, G2.start, G2.mem, row,
                                                          G2.n, S.gh[f], S.d.PS, S.d.nzl, G2.sidx,
                                                          S.sp ? S.sp + (size_t)S.cur * 3 * S.spn : nullptr);
@@ -1631,67 +1639,84 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     };
     return run_phase(M, k_iso, post, st);
   }
-  if (M->kind == SEIS_ACOUSTIC && M->ac_fused) {
-    const int c = M->slabs[0].cur;  // read set; the step writes set 1 - c
-    LaunchFn k_f = [&](size_t s, int ch0, int chs, int nch, cudaStream_t ks) -> seis_status {
-      Slab& S = M->slabs[s];
-      AcFArgs a;
-      a.mpt = S.af_pt[c];
-      a.mrt = S.af_rt;
-      a.mqx = S.af_qx[c];
-      a.mqy = S.af_qy[c];
-      a.mqz = S.af_qz[c];
-      a.mrz = S.af_rz;
-      a.mpz = S.af_pz[c];
-      a.mk = S.af_k;
-      a.p0 = S.fld[4 * c];
-      a.qz0 = S.fld[4 * c + 3];
-      a.rho = S.rho;
-      a.p1 = S.fld[4 * (1 - c)];
-      a.qx1 = S.fld[4 * (1 - c) + 1];
-      a.qy1 = S.fld[4 * (1 - c) + 2];
-      a.qz1 = S.fld[4 * (1 - c) + 3];
-      a.dth = (float)((double)M->g.dt / (double)M->g.h);
-      a.W = M->W;
-      a.zlo = 1;
-      a.cx = M->cp[0];
-      a.cy = M->cp[1];
-      a.cz = M->cp[2];
-      for (int t = 0; t < 3; ++t) {
-        a.psr[t] = S.psi[c ? 6 + t : t];
-        a.psw[t] = S.psi[c ? t : 6 + t];
-        a.pq[t] = S.psi[3 + t];
+  if (M->kind == SEIS_ACOUSTIC && M->ac_step) {
+    // f1: the whole step (V then P) in one persistent launch (kernels_acoustic_step.cuh); one
+    // slab, no exchange.  Cooperative launch: every tile's CTA is resident (they wait on their
+    // neighbours' progress counters, which the memset zeroes first).
+    Slab& S = M->slabs[0];
+    AcSArgs a;
+    a.mpt = S.as_pt;
+    a.mqx = S.as_q[0];
+    a.mqy = S.as_q[1];
+    a.mqz = S.as_q[2];
+    a.mrt = S.as_rt;
+    a.mrz = S.as_rz;
+    a.mpq = S.as_pq;
+    a.mqxn = S.as_qxn;
+    a.mqyn = S.as_qyn;
+    a.mk = S.as_k;
+    a.p0 = S.fld[0];
+    a.p = S.fld[0];
+    a.qx = S.fld[1];
+    a.qy = S.fld[2];
+    a.qz = S.fld[3];
+    a.dth = (float)((double)M->g.dt / (double)M->g.h);
+    a.W = M->W;
+    a.zlo = 1;
+    a.cx = M->cp[0];
+    a.cy = M->cp[1];
+    a.cz = M->cp[2];
+    a.psx = S.psi[0];
+    a.psy = S.psi[1];
+    a.psz = S.psi[2];
+    a.pqx = S.psi[3];
+    a.pqy = S.psi[4];
+    a.pqz = S.psi[5];
+    a.d = S.d;
+    a.ntx = M->as_ntx;
+    a.nty = M->as_nty;
+    a.cnt = M->as_cnt;
+    a.src_o = with_src ? S.src_o : -1;
+    a.src = SrcAmp{M->dwav, n, S.src_scale};
+    a.snap = snap ? (*snap)[0] : nullptr;
+    if (imgS) a.imgR = (*imgS)[0];
+    a.img = img ? (*img)[0] : nullptr;
+    a.trace = nullptr;
+#if SEIS_AS_TRACE
+    {
+      static unsigned long long* tr = nullptr;
+      static size_t trn = 0;
+      const size_t need = (size_t)M->as_ntx * M->as_nty * S.d.nzl * 12;
+      if (trn < need) {
+        if (tr) cudaFree(tr);
+        CK(cudaMallocManaged(&tr, need * sizeof(unsigned long long)));
+        trn = need;
       }
-      a.d = S.d;
-      a.zc = S.zc;
-      a.ch0 = ch0;
-      a.chs = chs;
-      a.src_o = with_src ? S.src_o : -1;
-      a.src = SrcAmp{M->dwav, n, S.src_scale};
-      a.snap = snap ? (*snap)[s] : nullptr;
-      a.imgS = imgS ? (*imgS)[s].s32 : nullptr;
-      a.img = img ? (*img)[s] : nullptr;
-      const dim3 gr = grid_of(S, TXV, BYF, nch), blk(NTX, BYF);
-      {
-        PROF(1, ks);
-        const size_t sb = AcFStage<BYF>::smem_bytes();
-        if (a.snap) ac_fused_kernel<BYF, true, false><<<gr, blk, sb, ks>>>(a);
-        else if (a.img) ac_fused_kernel<BYF, false, true><<<gr, blk, sb, ks>>>(a);
-        else ac_fused_kernel<BYF, false, false><<<gr, blk, sb, ks>>>(a);
-      }
-      CKL();
-      return SEIS_OK;
-    };
-    for (Slab& S : M->slabs) S.cur = 1 - c;  // injection / exchange act on the new set
-    PostFn post = [&](int part, cudaStream_t ps) -> seis_status {
-      TRY(inject(part, ps));
-      if (part == 1) return SEIS_OK;
-      // the next sweep recomputes q_z 4 planes into the neighbour slab: 8 ghost planes of p,
-      // 4 of q_z
-      TRY(exchange(M, {4 * (1 - c)}, ps, 8));
-      return exchange(M, {4 * (1 - c) + 3}, ps, 4);
-    };
-    return run_phase(M, k_f, post, st);
+      a.trace = tr;
+      g_trace = tr;
+      g_trace_n = need;
+    }
+#endif
+    const int ntiles = M->as_ntx * M->as_nty;
+    CK(cudaMemsetAsync(M->as_cnt, 0, (size_t)ntiles * sizeof(unsigned), st));
+    {
+      PROF(9, st);
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = dim3(ntiles);
+      cfg.blockDim = dim3(AS_THREADS);
+      cfg.dynamicSmemBytes = AcSLayout::smem_bytes();
+      cfg.stream = st;
+      cudaLaunchAttribute attr[1];
+      attr[0].id = cudaLaunchAttributeCooperative;
+      attr[0].val.cooperative = 1;
+      cfg.attrs = attr;
+      cfg.numAttrs = 1;
+      if (a.snap) CK(cudaLaunchKernelEx(&cfg, ac_step_kernel<true, false>, a));
+      else if (a.img) CK(cudaLaunchKernelEx(&cfg, ac_step_kernel<false, true>, a));
+      else CK(cudaLaunchKernelEx(&cfg, ac_step_kernel<false, false>, a));
+    }
+    CKL();
+    return inj_row ? inject_rows(M, inj_row, 2, st) : SEIS_OK;
   }
   if (M->kind == SEIS_ACOUSTIC) {
     LaunchFn k_v = [&](size_t s, int ch0, int chs, int nch, cudaStream_t ks) -> seis_status {
@@ -1876,7 +1901,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
 // Field holding the recorded / imaged quantity
 const float* out_field(seis_model* M, Slab& S, int comp) {
   if (M->kind == SEIS_ISO) return S.fld[S.cur];
-  if (M->kind == SEIS_ACOUSTIC) return S.fld[4 * S.cur];
+  if (M->kind == SEIS_ACOUSTIC) return S.fld[0];
   if (comp == 3) return S.fld[3];
   return S.fld[comp];
 }
@@ -2063,7 +2088,6 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
   if (sh->snap_bits != 0 && sh->snap_bits != 32 && sh->snap_bits != 24)
     return fail(SEIS_EINVAL, "snap_bits must be 0, 32 or 24");
   const bool s24 = sh->snap_bits == 24;
-  if (s24 && M->ac_fused) return fail(SEIS_EUNSUPPORTED, "24-bit snapshots with the fused acoustic step");
   const size_t esz = s24 ? 3 : 4;  // bytes per snapshot value
   // (pool floats of the snapshot region, 256-byte aligned so the checkpoints stay aligned)
   const size_t snap_elems = ((size_t)std::min(c, nsnap) * slab_pts * esz + 255) / 256 * 64;
@@ -2215,7 +2239,7 @@ seis_status seis_migrate(seis_model* M, const seis_shot* sh, const float* data, 
 seis_status seis_get_field(const seis_model* Mc, int32_t which, float* dst, void* stream) {
   seis_model* M = const_cast<seis_model*>(Mc);
   if (!M || !dst) return fail(SEIS_EINVAL, "null argument");
-  const int nf = nfields(M->kind, false);
+  const int nf = nfields(M->kind);
   if (which < 0 || which >= nf) return fail(SEIS_EINVAL, "field index %d out of range", which);
   CK(cudaSetDevice(M->device));
   cudaStream_t st = (cudaStream_t)stream;
@@ -2230,7 +2254,6 @@ seis_status seis_get_field(const seis_model* Mc, int32_t which, float* dst, void
   for (Slab& S : M->slabs) {
     int f = which;
     if (M->kind == SEIS_ISO) f = which == 0 ? S.cur : 1 - S.cur;
-    if (M->kind == SEIS_ACOUSTIC) f = 4 * S.cur + which;
     unpad_kernel<<<1024, 256, 0, st>>>(out + (size_t)(S.d.z0 - M->pz0) * g.ny * g.nx, S.fld[f], S.d);
     CKL();
   }

@@ -292,35 +292,3 @@ def test_checkpointed_rtm_bitwise(kind, P):
     assert rel_l2(imgs[0], I) <= TOL_IMAGE
 
 
-@pytest.mark.parametrize("P,nb", [(1, 7), (1, 0), (3, 6)])
-def test_fused_acoustic_step_bitwise_equals_split(P, nb, monkeypatch):
-    """f1: the single-sweep acoustic step (q recomputed on the tile halos and 3 planes ahead,
-    double-buffered state) reproduces the split V / P kernels bit for bit -- forward
-    modeling (seismogram + every field) and RTM, with and without C-PML and z-slabs; grids
-    with ragged x / y tails and several z-chunks."""
-    nx, ny, nz = 70, 45, 120
-    m = inputs.random_media((nz, ny, nx), seed=27)
-    h, dt, nt, snap = 10.0, 5e-4, 45, 4
-    w = inputs.source_series("acoustic", nt, dt, 35.0)
-    src = (nx // 3, ny // 2, 60)
-    rec = _deep_recs(nx, ny, nz)
-    data = np.random.default_rng(4).standard_normal((nt, rec.shape[0])).astype(np.float32)
-    runs = []
-    for fused in ("0", "1"):
-        monkeypatch.setenv("SEIS_AC_FUSED", fused)
-        g = seis.Grid(nx, ny, nz, h, dt, nb=nb, pml_f=35.0, slabs=P)
-        mod = seis.Model(g, "acoustic", m["vp"], rho=m["rho"])
-        shot = seis.Shot(src, w, rec, snap_period=snap)
-        sg = np.zeros((nt, rec.shape[0]), np.float32)
-        mod.forward_model(shot, sg)
-        fields = [mod.get_field(f) for f in range(4)]
-        img = np.zeros((nz, ny, nx), np.float32)
-        mod.migrate(shot, data, img)
-        runs.append((sg, fields, img))
-        mod.close()
-    (s0, f0, i0), (s1, f1, i1) = runs
-    assert np.abs(s0).max() > 0
-    assert np.array_equal(s0, s1)
-    for a, b in zip(f0, f1):
-        assert np.array_equal(a, b)
-    assert np.array_equal(i0, i1)
