@@ -62,6 +62,7 @@ constexpr int AS_L = 4;                      // P lags V by L planes
 #define SEIS_AS_NSP 3
 #endif
 constexpr int AS_NSV = SEIS_AS_NSV;
+
 // L2 prefetch distance (planes) of the DRAM-sourced operands: the shared-memory rings are only
 // NSV / NSP deep (one CTA per SM holds ~200 KB), so the HBM latency is covered by bringing each
 // plane into L2 AS_PF planes before its TMA load (cp.async.bulk.prefetch.tensor, no smem)
@@ -79,12 +80,13 @@ struct AcSArgs {
   CUtensorMap mpq;             // p^n, box 64 x TY (plane j+4: z-queue feed)
   CUtensorMap mqxn;            // q_x^{n+1/2}, box (64+8) x TY, origin (i0-4, j0)  (P stage)
   CUtensorMap mqyn;            // q_y^{n+1/2}, box 64 x (TY+8), origin (i0, j0-4)  (P stage)
-  CUtensorMap mk;              // dt K / h, box 64 x TY                             (P stage)
+  CUtensorMap mk;              // dt K / h, box 64 x TY (L2 prefetch only)
   const float* __restrict__ p0;   // p (padded): warm-up loads of the z-queue
   float* p;                       // p^{n+1} stores (same array as p0)
   float* __restrict__ qx;
   float* __restrict__ qy;
   float* __restrict__ qz;
+  const float* __restrict__ kk;   // dt K / h (padded): P's pointwise coefficient, by cp.async
   float dth;                      // dt / h
   int W, zlo;
   CpmlAxis cx, cy, cz;
@@ -117,7 +119,7 @@ __device__ __forceinline__ unsigned long long gtimer() {
 }
 #define AS_TRACE(k, ev)                                                                        \
   do {                                                                                         \
-    if (SEIS_AS_TRACE && a.trace) a.trace[((size_t)tile * nz + (k)) * 12 + (ev)] = gtimer();  \
+    if (SEIS_AS_TRACE && a.trace) a.trace[((size_t)tile * nz + (k)) * 48 + (ev)] = gtimer();  \
   } while (0)
 
 __host__ __device__ constexpr int r32(int n) { return (n + 31) / 32 * 32; }  // 128-byte aligned sub-tiles
@@ -128,13 +130,16 @@ struct AcSLayout {
                        R = QZ + r32(T), RZ = R + r32(RW * (AS_TY + 1)), PQ = RZ + r32(T), VSIZE = PQ + r32(T);
   static constexpr uint32_t VBYTES = (PW * (AS_TY + 8) + 5 * T + RW * (AS_TY + 1)) * 4;
   // P stage
-  static constexpr int QXN = 0, QYN = QXN + r32(PW * AS_TY), KK = QYN + r32(AS_TX * (AS_TY + 8)),
-                       PSIZE = KK + r32(T);
-  static constexpr uint32_t PBYTES = (PW * AS_TY + AS_TX * (AS_TY + 8) + T) * 4;
+  static constexpr int QXN = 0, QYN = QXN + r32(PW * AS_TY), PSIZE = QYN + r32(AS_TX * (AS_TY + 8));
+  static constexpr uint32_t PBYTES = (PW * AS_TY + AS_TX * (AS_TY + 8)) * 4;
   // q_z^{n+1/2} ring: planes j-8 .. j-1 (8 slots; each thread reads and writes only its column)
   static constexpr int ZSIZE = 0;
+  // C-PML memory variables in flight: per consumer thread and axis the 4 old values of the
+  // next half step, brought by cp.async (no registers held while they travel)
+  // (two sets: psi_p for V, psi_q for P; plus the 4 values of dt K/h for P)
+  static constexpr int QSIZE = 7 * AS_CONS * 4;
   static constexpr size_t smem_bytes() {
-    return ((size_t)AS_NSV * VSIZE + (size_t)AS_NSP * PSIZE + ZSIZE) * 4 + 128;
+    return ((size_t)AS_NSV * VSIZE + (size_t)AS_NSP * PSIZE + ZSIZE + QSIZE) * 4 + 128;
   }
 };
 
@@ -150,6 +155,37 @@ __device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
       : "memory");
   return ok != 0;
 }
+// psi <- b psi + a dv; dv += psi (common.cuh psi_upd; SEIS_AS_EXP == 4: without the psi store)
+template <int NV>
+__device__ __forceinline__ void psi_upd_s(float* dv, float* __restrict__ ps, const int* ix, const float* old,
+                                          const float* ca, const float* cb) {
+#pragma unroll
+  for (int e = 0; e < NV; ++e)
+    if (ix[e] >= 0) {
+      const float v = fmaf(cb[e], old[e], ca[e] * dv[e]);
+      ps[ix[e]] = v;
+      dv[e] += v;
+    }
+}
+// the same for a contiguous, 16-byte aligned group of 4 (one vector store)
+__device__ __forceinline__ void psi_upd_v4(float* dv, float* __restrict__ ps, int base, const float* old,
+                                           const float* ca, const float* cb) {
+  F4 v;
+#pragma unroll
+  for (int e = 0; e < 4; ++e) {
+    v.v[e] = fmaf(cb[e], old[e], ca[e] * dv[e]);
+    dv[e] += v.v[e];
+  }
+  st4(ps + base, v);
+}
+// producer-side wait: poll with a sleep between probes, so that a waiting producer thread does
+// not take issue slots from the consumer warps of its SM sub-partition
+#ifndef SEIS_AS_NAP
+#define SEIS_AS_NAP 100
+#endif
+__device__ __forceinline__ void mbar_wait_nap(uint64_t* bar, uint32_t parity) {
+  while (!mbar_test(bar, parity)) __nanosleep(SEIS_AS_NAP);
+}
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
@@ -159,6 +195,23 @@ __device__ __forceinline__ unsigned ld_relaxed_gpu(const unsigned* p) {
   return v;
 }
 __device__ __forceinline__ void fence_acq_rel_gpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+// 4-byte asynchronous global -> shared copy (zero-filled when !valid), and its group waits
+__device__ __forceinline__ void cp_async4(float* dst, const float* src, bool valid) {
+  asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;" ::"r"(smem_u32(dst)), "l"(src), "r"(valid ? 4 : 0)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async16(float* dst, const float* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+// wait until at most N of this thread's most recent cp.async groups are pending
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+__device__ __forceinline__ void prefetch_l2(const void* p) {
+  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+}
 __device__ __forceinline__ void red_release_gpu_add(unsigned* p, unsigned v) {
   asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
@@ -171,13 +224,14 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
   using L = AcSLayout;
   constexpr int PW = L::PW, RW = L::RW;
   static_assert(L::QX % 32 == 0 && L::QY % 32 == 0 && L::R % 32 == 0 && L::RZ % 32 == 0 && L::PQ % 32 == 0 &&
-                    L::VSIZE % 32 == 0 && L::QYN % 32 == 0 && L::KK % 32 == 0 && L::PSIZE % 32 == 0,
+                    L::VSIZE % 32 == 0 && L::QYN % 32 == 0 && L::PSIZE % 32 == 0,
                 "128-byte tiles");
   extern __shared__ __align__(128) float sm_raw[];
   float* sm = align128(sm_raw);
   float* smv = sm;                          // AS_NSV V stages
   float* smp = sm + AS_NSV * L::VSIZE;      // AS_NSP P stages
   __shared__ __align__(8) uint64_t fullv[AS_NSV], emptyv[AS_NSV], fullp[AS_NSP], emptyp[AS_NSP];
+  __shared__ CpmlTile<AS_TX, AS_TY> cpt;  // x / y C-PML coefficients of this tile (a, b, ah, bh)
   const Dims& d = a.d;
   const int tid = threadIdx.x;
   const int tile = blockIdx.x;
@@ -196,6 +250,7 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
     }
     mbar_fence_init();
   }
+  cpml_tile_fill(cpt, a.cx, a.cy, i0, j0, d.nx, d.ny, a.W > 0, tid, AS_THREADS);
   __syncthreads();
 
   if (tid >= AS_CONS) {
@@ -212,7 +267,7 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
       for (int j = 0; j < nz + AS_NSV; ++j) {
         const int s = j % AS_NSV;
         if (j >= AS_NSV) {
-          mbar_wait(&emptyv[s], ((j / AS_NSV) - 1) & 1);
+          mbar_wait_nap(&emptyv[s], ((j / AS_NSV) - 1) & 1);
           AS_TRACE(j - AS_NSV, 8);
           fence_proxy_async_global();
           AS_TRACE(j - AS_NSV, 9);
@@ -251,7 +306,7 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
       unsigned seen[5] = {0u, 0u, 0u, 0u, 0u};
       for (int k = 0; k < nz; ++k) {
         const int s = k % AS_NSP;
-        if (k >= AS_NSP) mbar_wait(&emptyp[s], ((k / AS_NSP) - 1) & 1);
+        if (k >= AS_NSP) mbar_wait_nap(&emptyp[s], ((k / AS_NSP) - 1) & 1);
         AS_TRACE(k, 10);
         const unsigned need = (unsigned)(k + 1);  // V(0 .. k) complete
         for (;;) {
@@ -262,7 +317,7 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
 #pragma unroll
           for (int c = 0; c < 5; ++c) ok = ok && (!cs[c] || seen[c] >= need);
           if (ok) break;
-          __nanosleep(20);
+          __nanosleep(SEIS_AS_NAP);
         }
         AS_TRACE(k, 11);
         fence_acq_rel_gpu();         // acquire: the q stores released with the counters
@@ -272,7 +327,6 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
         mbar_expect_tx(&fullp[s], L::PBYTES);
         tma_load_3d(st + L::QXN, &a.mqxn, &fullp[s], i0, y, z);
         tma_load_3d(st + L::QYN, &a.mqyn, &fullp[s], x, j0, z);
-        tma_load_3d(st + L::KK, &a.mk, &fullp[s], x, y, z);
         AS_TRACE(k, 2);
       }
     }
@@ -304,8 +358,71 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
 #pragma unroll
   for (int t = 0; t < 8; ++t) zq[t] = F4{{0.f, 0.f, 0.f, 0.f}};
   const long long srel0 = a.src_o - oc;
+  // Per-thread operands of the next half step travel by cp.async into this thread's slots while
+  // the current one computes (no registers held, latency hidden): the C-PML memory variables
+  // (V: psi_p at plane j, issued at the top of iteration j; P: psi_q at plane j - 3, issued
+  // after P(j - 4) consumed its slots) and, with psi_q, dt K/h of P's plane.  The slabs and K
+  // are prefetched into L2 AS_PF planes ahead.  Axis flags: lx / ly per thread, the z layer per
+  // plane.  Each iteration commits exactly two cp.async groups (V's, then P's), so the group of
+  // a half step is complete once at most one younger group is pending.
+  constexpr int QS = AS_CONS * 4;  // axis stride of the slots
+  // (16-byte copies / stores of a group's 4 memory variables need 16-byte aligned rows)
+  const bool vec4 = (d.nx & 3) == 0 && x0 + 3 < d.nx;
+  float* const psq_v = smp + AS_NSP * L::PSIZE + L::ZSIZE + 4 * tid;  // [3 axes] V slots
+  float* const psq_p = psq_v + 3 * QS;                                 // [3 axes] P slots
+  float* const ksl = psq_v + 6 * QS;                                   // dt K/h of P's plane
+  auto psi_issue = [&](float* const* arr, float* psq, int k) {
+    const int gz = k + d.z0;
+    const bool lzk = Wl > 0 && CpmlIdx::in(gz, d.nz, Wl, a.zlo);
+    if (own && lx) {  // x slab: the layer points of the group only (a few lanes per warp)
+      int ix[4];
+      psi_idx_x<4>(ix, d, Wl, x0, jy, k);
+#pragma unroll
+      for (int e = 0; e < 4; ++e)
+        if (ix[e] >= 0) cp_async4(psq + e, arr[0] + ix[e], true);
+    }
+    // y / z slabs: the group's 4 values are contiguous; one 16-byte copy when aligned
+    if (own && ly) {
+      const int b = (k * (2 * Wl) + CpmlIdx::slot(jy, d.ny, Wl)) * d.nx + x0;
+      if (vec4) {
+        cp_async16(psq + QS, arr[1] + b);
+      } else {
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          if (x0 + e < d.nx) cp_async4(psq + QS + e, arr[1] + b + e, true);
+      }
+    }
+    if (own && lzk) {
+      const int b = (CpmlIdx::slot(gz, d.nz, Wl) * d.ny + jy) * d.nx + x0;
+      if (vec4) {
+        cp_async16(psq + 2 * QS, arr[2] + b);
+      } else {
+#pragma unroll
+        for (int e = 0; e < 4; ++e)
+          if (x0 + e < d.nx) cp_async4(psq + 2 * QS + e, arr[2] + b + e, true);
+      }
+    }
+  };
+  auto psi_prefetch = [&](float* const* arr, int k) {  // one lane per 128-byte line
+    const int gz = k + d.z0;
+    if (!own || k >= nz) return;
+    if (lx && (tx & 7) == 0) {  // (a row's layer slots are within 2 W contiguous floats)
+      const int b = (k * d.ny + jy) * (2 * Wl) + (x0 < Wl ? 0 : Wl);
+      prefetch_l2(arr[0] + b);
+      prefetch_l2(arr[0] + b + Wl - 1);
+    }
+    if ((tx & 7) != 0) return;
+    if (ly) prefetch_l2(arr[1] + (k * (2 * Wl) + CpmlIdx::slot(jy, d.ny, Wl)) * d.nx + x0);
+    if (Wl > 0 && CpmlIdx::in(gz, d.nz, Wl, a.zlo))
+      prefetch_l2(arr[2] + (CpmlIdx::slot(gz, d.nz, Wl) * d.ny + jy) * d.nx + x0);
+  };
+  float* const psv[3] = {a.psx, a.psy, a.psz};
+  float* const psp[3] = {a.pqx, a.pqy, a.pqz};
 
+  // (the first P, k = 0, finds its operands in the group issued at the end of iteration 3)
   for (int j = 0; j < niter; ++j) {
+    if (j < nz) psi_issue(psv, psq_v, j);  // V(j)'s psi_p (its slots were consumed by V(j - 1))
+    cp_async_commit();
     if (j >= AS_L) {
       // ================================ P at plane k = j - L (ac_p, same arithmetic)
       const int k = j - AS_L;
@@ -332,7 +449,6 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
       F4 yr[8];  // q_y rows jy-4 .. jy+3
 #pragma unroll
       for (int m = 0; m < 8; ++m) yr[m] = lds4(cyp + (m - 4) * AS_TX);
-      const F4 kv = lds4(st + L::KK + pt);
       __syncwarp();
       if (lane == 0) mbar_arrive(&emptyp[s]);  // (everything of the stage is in registers)
       float dx[4], dy[4], dz[4];
@@ -356,37 +472,39 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
           dz[e] = fmaf(SEIS_D4, zq[7].v[e] - zq[0].v[e], t);
         }
       }
+      cp_async_wait<1>();  // this thread's psi_q + K slots (P's group; V(j)'s may be pending)
+      const F4 kv = lds4(ksl);
+      float* const psq = psq_p;
       if (own) {
         if (lx) {
           int ix[4];
-          float ov[4], ca[4], cb[4];
+          float ca[4], cb[4];
           psi_idx_x<4>(ix, d, Wl, x0, jy, k);
-          psi_ld<4>(ov, a.pqx, ix);
+          const F4 ov = lds4(psq);
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
-            const int x = min(x0 + e, d.nx - 1);
-            ca[e] = __ldg(a.cx.a + x);
-            cb[e] = __ldg(a.cx.b + x);
+            ca[e] = cpt.x[0][4 * tx + e];
+            cb[e] = cpt.x[1][4 * tx + e];
           }
-          psi_upd<4>(dx, a.pqx, ix, ov, ca, cb);
+          psi_upd_s<4>(dx, a.pqx, ix, ov.v, ca, cb);
         }
         if (ly) {
           int iy[4];
-          float ov[4];
           psi_idx_row<4>(iy, (k * (2 * Wl) + CpmlIdx::slot(jy, d.ny, Wl)) * d.nx + x0, x0, d.nx);
-          psi_ld<4>(ov, a.pqy, iy);
-          const float ya = __ldg(a.cy.a + jy), yb = __ldg(a.cy.b + jy);
+          const F4 ov = lds4(psq + QS);
+          const float ya = cpt.y[0][ty], yb = cpt.y[1][ty];
           const float ca[4] = {ya, ya, ya, ya}, cb[4] = {yb, yb, yb, yb};
-          psi_upd<4>(dy, a.pqy, iy, ov, ca, cb);
+          if (vec4) psi_upd_v4(dy, a.pqy, iy[0], ov.v, ca, cb);
+          else psi_upd_s<4>(dy, a.pqy, iy, ov.v, ca, cb);
         }
         if (lz) {
           int iz[4];
-          float ov[4];
           psi_idx_row<4>(iz, (CpmlIdx::slot(gz, d.nz, Wl) * d.ny + jy) * d.nx + x0, x0, d.nx);
-          psi_ld<4>(ov, a.pqz, iz);
+          const F4 ov = lds4(psq + 2 * QS);
           const float za = __ldg(a.cz.a + gz), zb = __ldg(a.cz.b + gz);
           const float ca[4] = {za, za, za, za}, cb[4] = {zb, zb, zb, zb};
-          psi_upd<4>(dz, a.pqz, iz, ov, ca, cb);
+          if (vec4) psi_upd_v4(dz, a.pqz, iz[0], ov.v, ca, cb);
+          else psi_upd_s<4>(dz, a.pqz, iz, ov.v, ca, cb);
         }
         const F4 pv = r[0];  // p^n(k)
         F4 out;
@@ -402,6 +520,12 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
         if (SNAP) st4_masked(a.snap + ((long long)k * d.ny + jy) * d.nx + x0, out, x0, d.nx, (d.nx & 3) == 0);
       }
     }
+    // P(j - 3)'s operands (psi_q, K) into the slots P(j - 4) just consumed
+    if (j + 1 - AS_L >= 0 && j + 1 - AS_L < nz) {
+      psi_issue(psp, psq_p, j + 1 - AS_L);
+      if (own) cp_async16(ksl, a.kk + (long long)(j + 1 - AS_L + GZ) * PS + oc);
+    }
+    cp_async_commit();
 #pragma unroll
     for (int t = 0; t < 7; ++t) {
       r[t] = r[t + 1];
@@ -414,6 +538,7 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
       const long long o = (long long)(k + GZ) * PS + oc;
       const int gz = k + d.z0;
       const bool lz = Wl > 0 && CpmlIdx::in(gz, d.nz, Wl, a.zlo);
+      if (lane == 0) AS_TRACE(k, 32 + (tid >> 5));  // every warp's V start (before the stage wait)
       mbar_wait(&fullv[s], (j / AS_NSV) & 1);
       if (tid == 0) AS_TRACE(k, 4);
       const float* st = smv + s * L::VSIZE;
@@ -450,39 +575,42 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
         dz[e] = fmaf(SEIS_D4, r[7].v[e] - r[0].v[e], t);
       }
       F4 oz4{{0.f, 0.f, 0.f, 0.f}};
+      cp_async_wait<1>();  // this thread's psi_p slots (V's group; P's younger may be pending)
+      float* const psq = psq_v;
       if (own) {
-        // C-PML memory variables (their old values are loaded here, not ahead of the stage
-        // wait: registers are the scarce resource of this kernel)
         if (lx) {
           int ix[4];
-          float ov[4], ca[4], cb[4];
+          float ca[4], cb[4];
           psi_idx_x<4>(ix, d, Wl, x0, jy, k);
-          psi_ld<4>(ov, a.psx, ix);
+          const F4 ov = lds4(psq);
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
-            const int x = min(x0 + e, d.nx - 1);
-            ca[e] = __ldg(a.cx.ah + x);
-            cb[e] = __ldg(a.cx.bh + x);
+            ca[e] = cpt.x[2][4 * tx + e];
+            cb[e] = cpt.x[3][4 * tx + e];
           }
-          psi_upd<4>(dx, a.psx, ix, ov, ca, cb);
+          psi_upd_s<4>(dx, a.psx, ix, ov.v, ca, cb);
         }
         if (ly) {
           int iy[4];
-          float ov[4];
           psi_idx_row<4>(iy, (k * (2 * Wl) + CpmlIdx::slot(jy, d.ny, Wl)) * d.nx + x0, x0, d.nx);
-          psi_ld<4>(ov, a.psy, iy);
-          const float ya = __ldg(a.cy.ah + jy), yb = __ldg(a.cy.bh + jy);
+          const F4 ov = lds4(psq + QS);
+          const float ya = cpt.y[2][ty], yb = cpt.y[3][ty];
           const float ca[4] = {ya, ya, ya, ya}, cb[4] = {yb, yb, yb, yb};
-          psi_upd<4>(dy, a.psy, iy, ov, ca, cb);
+          if (vec4) psi_upd_v4(dy, a.psy, iy[0], ov.v, ca, cb);
+          else psi_upd_s<4>(dy, a.psy, iy, ov.v, ca, cb);
         }
         if (lz) {
           int iz[4];
-          float ov[4];
           psi_idx_row<4>(iz, (CpmlIdx::slot(gz, d.nz, Wl) * d.ny + jy) * d.nx + x0, x0, d.nx);
-          psi_ld<4>(ov, a.psz, iz);
+          const F4 ov = lds4(psq + 2 * QS);
           const float za = __ldg(a.cz.ah + gz), zb = __ldg(a.cz.bh + gz);
           const float ca[4] = {za, za, za, za}, cb[4] = {zb, zb, zb, zb};
-          psi_upd<4>(dz, a.psz, iz, ov, ca, cb);
+          if (vec4) psi_upd_v4(dz, a.psz, iz[0], ov.v, ca, cb);
+          else psi_upd_s<4>(dz, a.psz, iz, ov.v, ca, cb);
+        }
+        if (Wl > 0) {  // L2 prefetch of the memory variables AS_PF planes ahead (both halves)
+          psi_prefetch(psv, j + AS_PF);
+          psi_prefetch(psp, j + AS_PF);
         }
         const F4 qxo = lds4(st + L::QX + pt), qyo = lds4(st + L::QY + pt), qzo = lds4(st + L::QZ + pt);
         const float* rc = st + L::R + ty * RW + 4 * tx;
@@ -524,6 +652,7 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
       if (lane == 0) mbar_arrive(&emptyv[s]);
       if (tid == 0) AS_TRACE(k, 5);
       if (tid == AS_CONS - 32) AS_TRACE(k, 7);
+      if (lane == 0) AS_TRACE(k, 16 + (tid >> 5));  // every warp's V done
     } else {
       r[7] = F4{{0.f, 0.f, 0.f, 0.f}};
       zq[7] = F4{{0.f, 0.f, 0.f, 0.f}};

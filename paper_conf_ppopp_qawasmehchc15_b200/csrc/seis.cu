@@ -33,8 +33,10 @@ using namespace seis;
 // ------------------------------------------------------------------ errors
 static thread_local std::string g_err;
 static thread_local long long g_launches = 0;
+#if SEIS_AS_TRACE
 static unsigned long long* g_trace = nullptr;  // SEIS_AS_TRACE builds: fused-step event buffer
 static size_t g_trace_n = 0;
+#endif
 
 static seis_status fail(seis_status st, const char* fmt, ...) {
   char buf[1024];
@@ -956,12 +958,12 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     else choose_chunks(S, occ, dev_sms, TXV, BYV, 16, zex);
   }
   // f1: the fused acoustic step (kernels_acoustic_step.cuh) on a single-slab, single-process
-  // model whose tiles can all be resident at once (cooperative launch), by default when there
-  // are enough tiles to occupy half the SMs (C2 / C4: 4 x 37 = 148 tiles); SEIS_AC_STEP=1 / 0
-  // forces it on (if the tiles fit) / off.  Bitwise the split pair's results (tested).
-#ifndef AS_DEFAULT_ON
-#define AS_DEFAULT_ON 0
-#endif
+  // model whose tiles can all be resident at once (cooperative launch).  Default: without
+  // absorbing layers (nb = 0) and with enough tiles to occupy half the SMs -- there it beats
+  // the split pair (512^3: 1.07 vs 1.19 ms per step); with C-PML the layer tiles (about half of
+  // them carry memory-variable work) pace the lockstep wavefront and the split pair stays
+  // faster.  SEIS_AC_STEP=1 / 0 forces it on (if the tiles fit) / off.  Bitwise
+  // the split pair's results either way (tests/test_acoustic_step_gpu.py).
   if (kind == SEIS_ACOUSTIC && ns == 1 && !M->comm) {
     const int ntx = (g.nx + AS_TX - 1) / AS_TX, nty = (g.ny + AS_TY - 1) / AS_TY;
     int occ_s = 0, coop = 0;
@@ -970,7 +972,7 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
     CK(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, M->device));
     const bool fits = coop && occ_s >= 1 && (long long)ntx * nty <= (long long)occ_s * dev_sms;
     const char* e = getenv("SEIS_AC_STEP");
-    const bool want = e ? e[0] == '1' : (AS_DEFAULT_ON && 2LL * ntx * nty >= dev_sms);
+    const bool want = e ? e[0] == '1' : (g.nb == 0 && 2LL * ntx * nty >= dev_sms);
     M->ac_step = fits && want;
     if (M->ac_step) {
       M->as_ntx = ntx;
@@ -1660,6 +1662,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     a.qx = S.fld[1];
     a.qy = S.fld[2];
     a.qz = S.fld[3];
+    a.kk = S.kdt;
     a.dth = (float)((double)M->g.dt / (double)M->g.h);
     a.W = M->W;
     a.zlo = 1;
@@ -1686,7 +1689,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     {
       static unsigned long long* tr = nullptr;
       static size_t trn = 0;
-      const size_t need = (size_t)M->as_ntx * M->as_nty * S.d.nzl * 12;
+      const size_t need = (size_t)M->as_ntx * M->as_nty * S.d.nzl * 48;
       if (trn < need) {
         if (tr) cudaFree(tr);
         CK(cudaMallocManaged(&tr, need * sizeof(unsigned long long)));

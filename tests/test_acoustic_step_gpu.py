@@ -79,9 +79,9 @@ def test_fused_step_bitwise_equals_split(nx, ny, nz, nb, monkeypatch):
     assert rel_l2(b["img"], I) <= TOL_IMAGE
 
 
-@pytest.mark.skip(reason='fused step not yet the default (C-PML tiles slower; DESIGN.md §6)')
-def test_fused_step_is_the_default_at_c2_size():
-    """A 512 x 512 plane is 4 x 37 tiles: the fused step is selected without any override."""
+def test_fused_step_default_selection():
+    """A 512 x 512 plane is 4 x 37 tiles: without absorbing layers the fused step is selected
+    without any override; with C-PML the split pair is."""
     torch = pytest.importorskip("torch")
     import os
 
@@ -89,9 +89,10 @@ def test_fused_step_is_the_default_at_c2_size():
     n, nz, nt = 512, 40, 3
     wl = inputs.c2(n=n, nt=nt, nb=20, model=False)
     vp = np.full((nz, n, n), 2000.0, np.float32)
-    g = seis.Grid(n, n, nz, wl.h, wl.dt, nb=10, pml_f=wl.fp)
-    mod = seis.Model(g, "acoustic", vp, rho=vp * 0 + 1000.0)
-    out = torch.zeros((nt, 3), device="cuda:0")
-    mod.forward_model(seis.Shot((256, 256, 20), wl.wavelet[:nt], np.asarray([[250, 256, 20]] * 3, np.int32)), out)
-    assert seis.Model.launches() == 2 * nt
-    mod.close()
+    for nb, launches in ((0, 2 * nt), (10, 3 * nt)):
+        g = seis.Grid(n, n, nz, wl.h, wl.dt, nb=nb, pml_f=wl.fp)
+        mod = seis.Model(g, "acoustic", vp, rho=vp * 0 + 1000.0)
+        out = torch.zeros((nt, 3), device="cuda:0")
+        mod.forward_model(seis.Shot((256, 256, 20), wl.wavelet[:nt], np.asarray([[250, 256, 20]] * 3, np.int32)), out)
+        assert seis.Model.launches() == launches, nb
+        mod.close()

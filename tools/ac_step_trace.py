@@ -46,8 +46,8 @@ def main():
     p = L.seis_debug_trace(C.byref(n))
     buf = np.ctypeslib.as_array((C.c_uint64 * n.value).from_address(p)).copy()
     nz = wl.nz
-    ntiles = n.value // (nz * 12)
-    t = buf.reshape(ntiles, nz, 12).astype(np.float64)
+    ntiles = n.value // (nz * 48)
+    t = buf.reshape(ntiles, nz, 48).astype(np.float64)
     t0 = t[t > 0].min()
     t = np.where(t > 0, t - t0, np.nan) / 1000.0  # us
     names = ["vload", "publish", "pload", "p_ready", "v_ready", "v_done", "p_start", "v_done_lastwarp"]
@@ -75,6 +75,23 @@ def main():
             "pslot_to_neighbours_ok": float(np.nanmedian(T[:, 11] - T[:, 10])),
             "neighbours_ok_to_pload": float(np.nanmedian(T[:, 2] - T[:, 11])),
         }
+    # per-tile busy / wait breakdown over the middle planes (consumer warp 0)
+    lo, hi = 40, nz - 44
+    pw = np.nanmean(t[:, lo:hi, 3] - t[:, lo:hi, 6], axis=1)                # P-stage wait
+    vc = np.nanmean(t[:, lo + 4:hi + 4, 5] - t[:, lo + 4:hi + 4, 4], axis=1)  # V wait-done -> V done
+    per = (t[:, hi, 1] - t[:, lo, 1]) / (hi - lo)                           # publish period
+    order = np.argsort(pw)
+    res["p_wait_least_tiles"] = [(int(i), round(float(pw[i]), 2), round(float(vc[i]), 2)) for i in order[:8]]
+    res["p_wait_most_tiles"] = [(int(i), round(float(pw[i]), 2), round(float(vc[i]), 2)) for i in order[-5:]]
+    res["publish_period_us"] = [round(float(np.nanmin(per)), 3), round(float(np.nanmedian(per)), 3),
+                                round(float(np.nanmax(per)), 3)]
+    res["p_wait_grid"] = [[round(float(pw[r * 4 + c]), 1) for c in range(4)] for r in range(ntiles // 4)]
+    # per-warp V start / done relative to the tile's earliest warp, middle planes, median
+    for tile in (0, 1, 77):
+        vs = t[tile, lo:hi, 32:46]
+        vd = t[tile, lo:hi, 16:30]
+        res[f"warps_tile{tile}_vstart_rel"] = [round(float(x), 2) for x in np.nanmedian(vs - np.nanmin(vs, axis=1, keepdims=True), axis=0)]
+        res[f"warps_tile{tile}_vdur"] = [round(float(x), 2) for x in np.nanmedian(vd - vs, axis=0)]
     # lateness of the P-load relative to the time the consumers need it
     k = np.arange(nz)
     res["pload_minus_pstart_median"] = float(np.nanmedian(t[:, mid, 2] - t[:, mid, 6]))
