@@ -26,6 +26,9 @@ constexpr int GZ = 8;    // z ghost depth: 4 for the stencil + 4 for the fused a
                          // recomputed q_z halo
 constexpr int TXW = 32;  // tile width in x = one warp
 
+// float count rounded up to 128 bytes (shared-memory sub-tile offsets; TMA destinations)
+__host__ __device__ constexpr int r32(int n) { return (n + 31) / 32 * 32; }
+
 struct Dims {
   int nx, ny, nzl;  // interior points of the slab
   int nz;           // global nz
@@ -158,6 +161,29 @@ __device__ __forceinline__ void stage_release(uint32_t* cnt, int tid, bool more,
     refill();
   }
   }
+}
+// non-blocking probe: has the phase with parity `parity` completed?
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile(
+      "{\n.reg .pred p;\n"
+      "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n"
+      "selp.u32 %0, 1, 0, p;\n}\n"
+      : "=r"(ok)
+      : "r"(smem_u32(bar)), "r"(parity)
+      : "memory");
+  return ok != 0;
+}
+// producer-side wait: poll with a sleep between probes, so that a waiting producer thread does
+// not take issue slots from the consumer warps of its SM sub-partition
+#ifndef SEIS_AS_NAP
+#define SEIS_AS_NAP 100
+#endif
+__device__ __forceinline__ void mbar_wait_nap(uint64_t* bar, uint32_t parity) {
+  while (!mbar_test(bar, parity)) __nanosleep(SEIS_AS_NAP);
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 // Fast reciprocal (MUFU.RCP, ~1 ulp; +inf -> +0) for the on-the-fly face/edge averages
 __device__ __forceinline__ float rcp_fast(float x) {

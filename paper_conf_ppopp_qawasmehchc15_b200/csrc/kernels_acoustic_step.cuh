@@ -122,7 +122,6 @@ __device__ __forceinline__ unsigned long long gtimer() {
     if (SEIS_AS_TRACE && a.trace) a.trace[((size_t)tile * nz + (k)) * 48 + (ev)] = gtimer();  \
   } while (0)
 
-__host__ __device__ constexpr int r32(int n) { return (n + 31) / 32 * 32; }  // 128-byte aligned sub-tiles
 struct AcSLayout {
   static constexpr int PW = AS_TX + 8, T = AS_TX * AS_TY, RW = AS_TX + 4;
   // V stage
@@ -143,19 +142,7 @@ struct AcSLayout {
   }
 };
 
-// non-blocking probe: has the phase with parity `parity` completed?
-__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
-  uint32_t ok;
-  asm volatile(
-      "{\n.reg .pred p;\n"
-      "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n"
-      "selp.u32 %0, 1, 0, p;\n}\n"
-      : "=r"(ok)
-      : "r"(smem_u32(bar)), "r"(parity)
-      : "memory");
-  return ok != 0;
-}
-// psi <- b psi + a dv; dv += psi (common.cuh psi_upd; SEIS_AS_EXP == 4: without the psi store)
+// psi <- b psi + a dv; dv += psi (common.cuh psi_upd)
 template <int NV>
 __device__ __forceinline__ void psi_upd_s(float* dv, float* __restrict__ ps, const int* ix, const float* old,
                                           const float* ca, const float* cb) {
@@ -177,17 +164,6 @@ __device__ __forceinline__ void psi_upd_v4(float* dv, float* __restrict__ ps, in
     dv[e] += v.v[e];
   }
   st4(ps + base, v);
-}
-// producer-side wait: poll with a sleep between probes, so that a waiting producer thread does
-// not take issue slots from the consumer warps of its SM sub-partition
-#ifndef SEIS_AS_NAP
-#define SEIS_AS_NAP 100
-#endif
-__device__ __forceinline__ void mbar_wait_nap(uint64_t* bar, uint32_t parity) {
-  while (!mbar_test(bar, parity)) __nanosleep(SEIS_AS_NAP);
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 __device__ __forceinline__ unsigned ld_relaxed_gpu(const unsigned* p) {
   unsigned v;

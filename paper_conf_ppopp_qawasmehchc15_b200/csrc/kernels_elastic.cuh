@@ -79,11 +79,28 @@ __device__ __forceinline__ F2 ldg2_fs(const float* __restrict__ f, int p, long l
   return ldg2(f + (long long)(p + GZ) * PS + oc);
 }
 
+// Warp specialization (default): one extra warp per block issues the TMA ring loads; consumer
+// warps release a stage by arriving on its "empty" mbarrier, so no block-wide barrier remains
+// in the z-march (ncu r01: 17 % of el_v's stalls were on the per-plane __syncthreads).  The
+// block is then 32 x BY consumer threads + the producer warp, one block per SM (BY = 15:
+// 16 warps, 128 registers per thread).  SEIS_EL_WS=0 restores the barrier-released ring.
+#ifndef SEIS_EL_WS
+#define SEIS_EL_WS 1
+#endif
+constexpr int EL_WS = SEIS_EL_WS;
+// (warp specialization) L2 prefetch distance of the producer, planes ahead of the ring loads
+#ifndef SEIS_EL_PF
+#define SEIS_EL_PF 0
+#endif
+constexpr int EL_PF = SEIS_EL_PF;
+#ifndef SEIS_EL_PWAIT
+#define SEIS_EL_PWAIT 1  // producer wait: 0 = test_wait + nanosleep, 1 = try_wait spin
+#endif
 #ifndef SEIS_EL_VNS
 #define SEIS_EL_VNS 3
 #endif
 #ifndef SEIS_EL_SNS
-#define SEIS_EL_SNS 2
+#define SEIS_EL_SNS (SEIS_EL_WS ? 3 : 2)
 #endif
 #ifndef SEIS_EL_MINB
 #define SEIS_EL_MINB 0  // launch-bounds minimum blocks per SM (0: 2 for BY <= 8, else 1)
@@ -118,17 +135,18 @@ struct ElVArgs {
 template <int BY>
 struct ElVStage {
   static constexpr int WX = TXE + 8, T = TXE * BY, RW = TXE + 4;
-  static constexpr int XX = 0, XY = XX + BY * WX, XZ = XY + (BY + 8) * WX, YY = XZ + BY * WX,
-                       YZ = YY + (BY + 8) * TXE, V = YZ + (BY + 8) * TXE, RZ = V + 3 * T, Q = RZ + T,
-                       R = Q + 3 * T, SIZE = R + ((RW * (BY + 1) + 31) / 32) * 32;
-  static constexpr uint32_t BYTES = (R + RW * (BY + 1)) * 4;
+  static constexpr int XX = 0, XY = XX + r32(BY * WX), XZ = XY + r32((BY + 8) * WX), YY = XZ + r32(BY * WX),
+                       YZ = YY + r32((BY + 8) * TXE), V = YZ + r32((BY + 8) * TXE), RZ = V + 3 * r32(T),
+                       Q = RZ + r32(T), R = Q + 3 * r32(T), SIZE = R + r32(RW * (BY + 1));
+  static constexpr int TS = r32(T);  // stride of the 3 v / 3 q tiles
+  static constexpr uint32_t BYTES = (2 * BY * WX + (BY + 8) * WX + 2 * (BY + 8) * TXE + 7 * T + RW * (BY + 1)) * 4;
   static constexpr size_t smem_bytes() { return (size_t)EL_VNS * SIZE * 4 + 128; }
 };
 
 template <int BY, bool IMG>
-__global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (BY <= 8 ? 2 : 1)) el_v_kernel(const __grid_constant__ ElVArgs a) {
+__global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (BY <= 8 ? 2 : 1)) el_v_kernel(const __grid_constant__ ElVArgs a) {
   using L = ElVStage<BY>;
-  constexpr int WX = L::WX, T = L::T;
+  constexpr int WX = L::WX;
   constexpr uint32_t TX_BYTES = L::BYTES;
   constexpr int RW = L::RW;
   static_assert((L::XY % 32) == 0 && (L::XZ % 32) == 0 && (L::YY % 32) == 0 && (L::V % 32) == 0 &&
@@ -137,6 +155,7 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
   extern __shared__ __align__(128) float sm_raw[];
   float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[EL_VNS];
+  __shared__ __align__(8) uint64_t ebar[EL_VNS];  // (warp specialization) stage consumed by all warps
   __shared__ uint32_t cnt[EL_VNS];
   __shared__ CpmlTile<TXE, BY> ctile;  // x / y C-PML coefficients of this tile
   const Dims& d = a.d;
@@ -162,26 +181,40 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
     tma_ld(pf, st + L::YY, &a.msyy, &bar[s], x, j0, z);
     tma_ld(pf, st + L::YZ, &a.msyz, &bar[s], x, j0, z);
 #pragma unroll
-    for (int c = 0; c < 3; ++c) tma_ld(pf, st + L::V + c * T, &a.mv[c], &bar[s], x, y, z);
+    for (int c = 0; c < 3; ++c) tma_ld(pf, st + L::V + c * L::TS, &a.mv[c], &bar[s], x, y, z);
     tma_ld(pf, st + L::R, &a.mr, &bar[s], x, y, z);
     tma_ld(pf, st + L::RZ, &a.mrz, &bar[s], x, y, z + 1);
     tma_ld(pf, st + L::Q, &a.mq[0], &bar[s], x, y, z + 3);
-    tma_ld(pf, st + L::Q + T, &a.mq[1], &bar[s], x, y, z + 3);
-    tma_ld(pf, st + L::Q + 2 * T, &a.mq[2], &bar[s], x, y, z + 4);
+    tma_ld(pf, st + L::Q + L::TS, &a.mq[1], &bar[s], x, y, z + 3);
+    tma_ld(pf, st + L::Q + 2 * L::TS, &a.mq[2], &bar[s], x, y, z + 4);
   };
   if (tid == 0) {
     for (int s = 0; s < EL_VNS; ++s) {
       mbar_init(&bar[s], 1);
+      mbar_init(&ebar[s], BY);
       cnt[s] = 0u;
     }
     mbar_fence_init();
   }
   cpml_tile_fill(ctile, a.cx, a.cy, blockIdx.x * TXE, blockIdx.y * BY, a.d.nx, a.d.ny, a.W > 0, tid,
-                 NTX2 * BY);
+                 NTX2 * (BY + EL_WS));
   __syncthreads();
-  if (tid == 0)
+  if (EL_WS && ty == BY) {  // producer warp: lane 0 refills each stage once all warps released it
+    if (tx == 0)
+      for (int it = 0; it < np; ++it) {
+        const int s = it % EL_VNS;
+        if (it >= EL_VNS) {
+          if (SEIS_EL_PWAIT) mbar_wait(&ebar[s], ((it / EL_VNS) - 1) & 1);
+          else mbar_wait_nap(&ebar[s], ((it / EL_VNS) - 1) & 1);
+        }
+        issue(s, k0 + it);
+        if (EL_PF > 0 && it + EL_PF < np) issue(s, k0 + it + EL_PF, true);  // L2 prefetch
+      }
+    return;
+  }
+  if (!EL_WS && tid == 0)
     for (int s = 0; s < EL_VNS && s < np; ++s) issue(s, k0 + s);
-  if (tid == 0)
+  if (!EL_WS && tid == 0)
     for (int t = 0; t < L2PF && EL_VNS + t < np; ++t) issue(0, k0 + EL_VNS + t, true);
   const float* __restrict__ sxz = a.f[ESXZ];
   const float* __restrict__ syz = a.f[ESYZ];
@@ -234,8 +267,8 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
     const float* st = sm + s * L::SIZE;
     const int pt = ty * TXE + 2 * tx;
     qxz[7] = lds2(st + L::Q + pt);
-    qyz[7] = lds2(st + L::Q + T + pt);
-    qzz[7] = lds2(st + L::Q + 2 * T + pt);
+    qyz[7] = lds2(st + L::Q + L::TS + pt);
+    qzz[7] = lds2(st + L::Q + 2 * L::TS + pt);
     if (own) {
       float xs[10], xy[10], xz[10], yxy[2][9], yyy[2][9], yyz[2][9];
       xrow(xs, st + L::XX + ty * WX + 2 * tx + 4);
@@ -292,7 +325,7 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
         psi_upd<2>(d5, a.psi[5], izz, oz5, ca, cb);
         psi_upd<2>(d8, a.psi[8], izz, oz8, cah, cbh);
       }
-      const F2 v0 = lds2(st + L::V + pt), v1 = lds2(st + L::V + T + pt), v2 = lds2(st + L::V + 2 * T + pt);
+      const F2 v0 = lds2(st + L::V + pt), v1 = lds2(st + L::V + L::TS + pt), v2 = lds2(st + L::V + 2 * L::TS + pt);
       // face buoyancy dt b/h = (dt/h) 2/(rho_i + rho_{i+1}), the last face clamps (O8, O9)
       const float* rc = st + L::R + ty * RW + 2 * tx;
       const F2 r0 = lds2(rc), ryn = lds2(rc + RW), rzn = lds2(st + L::RZ + pt);
@@ -326,10 +359,15 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
           }
       }
     }
-    stage_release<(SEIS_WR_EL != 0)>(&cnt[s], tid, it + EL_VNS < np, [&] {
-      issue(s, k + EL_VNS);
-      if (L2PF && it + EL_VNS + L2PF < np) issue(s, k + EL_VNS + L2PF, true);
-    });
+    if (EL_WS) {
+      __syncwarp();
+      if (tx == 0) mbar_arrive(&ebar[s]);
+    } else {
+      stage_release<(SEIS_WR_EL != 0)>(&cnt[s], tid, it + EL_VNS < np, [&] {
+        issue(s, k + EL_VNS);
+        if (L2PF && it + EL_VNS + L2PF < np) issue(s, k + EL_VNS + L2PF, true);
+      });
+    }
 #pragma unroll
     for (int t = 0; t < 7; ++t) {
       qxz[t] = qxz[t + 1];
@@ -360,24 +398,25 @@ struct ElSArgs {
 
 template <int BY>
 struct ElSStage {
-  static constexpr int WX = TXE + 8, T = TXE * BY, TV = (BY + 8) * WX, RW = TXE + 4;
+  static constexpr int WX = TXE + 8, T = TXE * BY, TV = r32((BY + 8) * WX), RW = TXE + 4, TS = r32(TXE * BY);
   static constexpr int WT = ((RW * (BY + 1) + 31) / 32) * 32;
-  static constexpr int VT = 0, S = 3 * TV, C = S + 6 * T, Q = C + T, WK = Q + 3 * T, WK1 = WK + WT,
+  static constexpr int VT = 0, S = 3 * TV, C = S + 6 * TS, Q = C + TS, WK = Q + 3 * TS, WK1 = WK + WT,
                        SIZE = WK1 + WT;
-  static constexpr uint32_t BYTES = (WK + 2 * RW * (BY + 1)) * 4;  // bytes the TMA boxes deliver
+  static constexpr uint32_t BYTES = (3 * (BY + 8) * WX + 10 * T + 2 * RW * (BY + 1)) * 4;  // what the TMA boxes deliver
   static constexpr size_t smem_bytes() { return (size_t)EL_SNS * SIZE * 4 + 128; }
 };
 
 template <int BY, bool SNAP>
-__global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (BY <= 8 ? 2 : 1)) el_s_kernel(const __grid_constant__ ElSArgs a) {
+__global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (BY <= 8 ? 2 : 1)) el_s_kernel(const __grid_constant__ ElSArgs a) {
   using L = ElSStage<BY>;
-  constexpr int WX = L::WX, T = L::T, TV = L::TV, RW = L::RW;
+  constexpr int WX = L::WX, TV = L::TV, RW = L::RW;
   constexpr uint32_t TX_BYTES = L::BYTES;
   static_assert((L::S % 32) == 0 && (L::C % 32) == 0 && (L::WK % 32) == 0 && (L::WK1 % 32) == 0,
                 "128-byte tiles");
   extern __shared__ __align__(128) float sm_raw[];
   float* sm = align128(sm_raw);
   __shared__ __align__(8) uint64_t bar[EL_SNS];
+  __shared__ __align__(8) uint64_t ebar[EL_SNS];  // (warp specialization) stage consumed by all warps
   __shared__ uint32_t cnt[EL_SNS];
   __shared__ CpmlTile<TXE, BY> ctile;  // x / y C-PML coefficients of this tile
   const Dims& d = a.d;
@@ -400,27 +439,41 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
 #pragma unroll
     for (int c = 0; c < 3; ++c) tma_ld(pf, st + L::VT + c * TV, &a.mvt[c], &bar[s], i0, j0, z);
 #pragma unroll
-    for (int c = 0; c < 6; ++c) tma_ld(pf, st + L::S + c * T, &a.ms[c], &bar[s], x, y, z);
+    for (int c = 0; c < 6; ++c) tma_ld(pf, st + L::S + c * L::TS, &a.ms[c], &bar[s], x, y, z);
     tma_ld(pf, st + L::C, &a.ml2m, &bar[s], x, y, z);
     tma_ld(pf, st + L::WK, &a.mw, &bar[s], x, y, z);
     tma_ld(pf, st + L::WK1, &a.mw, &bar[s], x, y, z + 1);
     tma_ld(pf, st + L::Q, &a.mq[0], &bar[s], x, y, z + 4);
-    tma_ld(pf, st + L::Q + T, &a.mq[1], &bar[s], x, y, z + 4);
-    tma_ld(pf, st + L::Q + 2 * T, &a.mq[2], &bar[s], x, y, z + 3);
+    tma_ld(pf, st + L::Q + L::TS, &a.mq[1], &bar[s], x, y, z + 4);
+    tma_ld(pf, st + L::Q + 2 * L::TS, &a.mq[2], &bar[s], x, y, z + 3);
   };
   if (tid == 0) {
     for (int s = 0; s < EL_SNS; ++s) {
       mbar_init(&bar[s], 1);
+      mbar_init(&ebar[s], BY);
       cnt[s] = 0u;
     }
     mbar_fence_init();
   }
   cpml_tile_fill(ctile, a.cx, a.cy, blockIdx.x * TXE, blockIdx.y * BY, a.d.nx, a.d.ny, a.W > 0, tid,
-                 NTX2 * BY);
+                 NTX2 * (BY + EL_WS));
   __syncthreads();
-  if (tid == 0)
+  if (EL_WS && ty == BY) {  // producer warp: lane 0 refills each stage once all warps released it
+    if (tx == 0)
+      for (int it = 0; it < np; ++it) {
+        const int s = it % EL_SNS;
+        if (it >= EL_SNS) {
+          if (SEIS_EL_PWAIT) mbar_wait(&ebar[s], ((it / EL_SNS) - 1) & 1);
+          else mbar_wait_nap(&ebar[s], ((it / EL_SNS) - 1) & 1);
+        }
+        issue(s, k0 + it);
+        if (EL_PF > 0 && it + EL_PF < np) issue(s, k0 + it + EL_PF, true);  // L2 prefetch
+      }
+    return;
+  }
+  if (!EL_WS && tid == 0)
     for (int s = 0; s < EL_SNS && s < np; ++s) issue(s, k0 + s);
-  if (tid == 0)
+  if (!EL_WS && tid == 0)
     for (int t = 0; t < L2PF && EL_SNS + t < np; ++t) issue(0, k0 + EL_SNS + t, true);
   const float* __restrict__ vx = a.f[EVX];
   const float* __restrict__ vy = a.f[EVY];
@@ -474,8 +527,8 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
     const float* st = sm + s * L::SIZE;
     const int pt = ty * TXE + 2 * tx;
     qx[7] = lds2(st + L::Q + pt);
-    qy[7] = lds2(st + L::Q + T + pt);
-    qz[7] = lds2(st + L::Q + 2 * T + pt);
+    qy[7] = lds2(st + L::Q + L::TS + pt);
+    qz[7] = lds2(st + L::Q + 2 * L::TS + pt);
     if (own) {
       const float* cvx = st + L::VT + (ty + 4) * WX + 2 * tx + 4;
       const float* cvy = cvx + TV;
@@ -537,7 +590,7 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
       }
       F2 sv[6];
 #pragma unroll
-      for (int c = 0; c < 6; ++c) sv[c] = lds2(st + L::S + c * T + pt);
+      for (int c = 0; c < 6; ++c) sv[c] = lds2(st + L::S + c * L::TS + pt);
       const F2 cl2m = lds2(st + L::C + pt);
       // node w = h/(dt mu) at planes k (wa) and k+1 (wb), rows j (…0) and j+1 (…1), columns
       // x0, x0+1, x0+2; neighbours past the last node clamp to it (O9)
@@ -594,10 +647,15 @@ __global__ void __launch_bounds__(NTX2 * BY, SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (
           if (x0 + e < d.nx) a.snap[cix + e] = -((o6[0].v[e] + o6[1].v[e]) + o6[2].v[e]) / 3.0f;
       }
     }
-    stage_release<(SEIS_WR_EL != 0)>(&cnt[s], tid, it + EL_SNS < np, [&] {
-      issue(s, k + EL_SNS);
-      if (L2PF && it + EL_SNS + L2PF < np) issue(s, k + EL_SNS + L2PF, true);
-    });
+    if (EL_WS) {
+      __syncwarp();
+      if (tx == 0) mbar_arrive(&ebar[s]);
+    } else {
+      stage_release<(SEIS_WR_EL != 0)>(&cnt[s], tid, it + EL_SNS < np, [&] {
+        issue(s, k + EL_SNS);
+        if (L2PF && it + EL_SNS + L2PF < np) issue(s, k + EL_SNS + L2PF, true);
+      });
+    }
 #pragma unroll
     for (int t = 0; t < 7; ++t) {
       qx[t] = qx[t + 1];

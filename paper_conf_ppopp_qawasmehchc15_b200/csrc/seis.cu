@@ -124,7 +124,7 @@ namespace {
 #define SEIS_BYP 8
 #endif
 #ifndef SEIS_BYE
-#define SEIS_BYE 8
+#define SEIS_BYE (SEIS_EL_WS ? 15 : 8)
 #endif
 constexpr int BYI = SEIS_BYI;  // ISO step (block 16 x BYI threads, 4 x-points each)
 constexpr int BYV = SEIS_BYV;  // acoustic V (block 16 x BYV)
@@ -950,7 +950,7 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_v_kernel<BYV, false>, NTX * BYV,
                                                     AcVStage<BYV>::smem_bytes());
     else
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, NTX2 * BYE,
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, NTX2 * (BYE + EL_WS),
                                                     ElSStage<BYE>::smem_bytes());
     const int zex = (ns > 1 || M->nranks > 1) ? 4 : 0;
     if (kind == SEIS_ELASTIC) choose_chunks(S, occ, dev_sms, TXE, BYE, 16, zex);
@@ -1847,8 +1847,8 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     const dim3 gr = grid_of(S, TXE, BYE, nch);
     {
       PROF(3, ks);
-      if (a.img) el_v_kernel<BYE, true><<<gr, dim3(NTX2, BYE), ElVStage<BYE>::smem_bytes(), ks>>>(a);
-      else el_v_kernel<BYE, false><<<gr, dim3(NTX2, BYE), ElVStage<BYE>::smem_bytes(), ks>>>(a);
+      if (a.img) el_v_kernel<BYE, true><<<gr, dim3(NTX2, BYE + EL_WS), ElVStage<BYE>::smem_bytes(), ks>>>(a);
+      else el_v_kernel<BYE, false><<<gr, dim3(NTX2, BYE + EL_WS), ElVStage<BYE>::smem_bytes(), ks>>>(a);
     }
     CKL();
     return SEIS_OK;
@@ -1887,8 +1887,8 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     const dim3 gr = grid_of(S, TXE, BYE, nch);
     {
       PROF(4, ks);
-      if (a.snap) el_s_kernel<BYE, true><<<gr, dim3(NTX2, BYE), ElSStage<BYE>::smem_bytes(), ks>>>(a);
-      else el_s_kernel<BYE, false><<<gr, dim3(NTX2, BYE), ElSStage<BYE>::smem_bytes(), ks>>>(a);
+      if (a.snap) el_s_kernel<BYE, true><<<gr, dim3(NTX2, BYE + EL_WS), ElSStage<BYE>::smem_bytes(), ks>>>(a);
+      else el_s_kernel<BYE, false><<<gr, dim3(NTX2, BYE + EL_WS), ElSStage<BYE>::smem_bytes(), ks>>>(a);
     }
     CKL();
     return SEIS_OK;
