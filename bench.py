@@ -24,7 +24,7 @@ Gpts/s = grid points x time steps / second (whole job over all ranks).
           timings ride along under other_configs.
 * extras (N = 1, unless --no-extras): Gpts/s of the other propagators (C1 ISO 64^3, an ISO 512^3
           sweep, C3 elastic 384^3) and RTM shots/hour (C4, 512^3 salt model, 2000 steps,
-          snapshots every 20 steps in HBM).
+          snapshots every 20 steps in HBM; C5, 1024^3, 1000 steps, checkpointed, --no-c5 skips).
 N > 1 (torchrun): weak scaling, z-slab decomposition with NCCL halo exchange; each rank
 holds 512^3 points (global nz = 512 N).  --scaling strong splits one 512^3 grid instead;
 --halo peer replaces the NCCL send/recv by direct ghost-plane stores over NVLink (f4).
@@ -388,7 +388,65 @@ def run_extras(args, local):
                          "gpts_s_both_phases": round(2 * wl.npts * wl.nt / (ms * 1e-3) / 1e9, 3),
                          "snapshots_in_hbm": (wl.nt - 1) // wl.snap, "receivers": shot.nrec}
     mig.close()
+    del mig, true, data, img, smooth, wl
+    torch.cuda.empty_cache()
+    if not args.no_c5:
+        res["C5_rtm_1024_1gpu"] = run_c5(local)
     return res
+
+
+def run_c5(local, n=1024, nt=1000):
+    """C5 (BASELINE configs[4]) on ONE B200: acoustic RTM 1024^3, 1000 steps, snapshots every
+    20 steps, 13 924-receiver carpet.  The 49 fp32 snapshots (196 GiB) do not fit in 180 GB, so
+    the migration keeps source-state checkpoints and recomputes earlier segments (f2, P:181;
+    the largest segment length that fits is chosen).  Observed data: forward modeling on the
+    true salt model; migration on its Gaussian-smoothed copy (sigma 5 points)."""
+    import torch
+
+    import paper_conf_ppopp_qawasmehchc15_b200 as seis
+    from paper_conf_ppopp_qawasmehchc15_b200 import inputs
+
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream()
+    t0 = time.perf_counter()
+    wl = inputs.c5(n=n, nt=nt)
+    build_s = time.perf_counter() - t0
+    g = seis.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=wl.nb, pml_f=wl.fp)
+    shot = seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap)
+    true = seis.Model(g, "acoustic", wl.model["vp"], rho=wl.model["rho"], device=local)
+    data = torch.empty((wl.nt, shot.nrec), device=dev)
+    fms = _timed_shots(lambda: true.forward_model(shot, data, stream), 1, stream)
+    true.close()
+    del true
+    torch.cuda.empty_cache()
+    sm = inputs.smooth_torch(wl.model, 5.0, dev)
+    del wl.model
+    free, _ = torch.cuda.mem_get_info(dev)
+    img_bytes = float(wl.npts) * 4
+    nsnap = (wl.nt - 1) // wl.snap
+    c = 0
+    if seis.memory_required(g, "acoustic", shot) + img_bytes > 0.95 * free:
+        fits = [cc for cc in range(1, nsnap + 1)
+                if seis.memory_required(g, "acoustic", seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap,
+                                                                 ckpt_period=cc)) + img_bytes <= 0.95 * free]
+        c = max(fits)
+    rshot = seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap, ckpt_period=c)
+    mig = seis.Model(g, "acoustic", sm["vp"], rho=sm["rho"], device=local)
+    del sm
+    img = torch.zeros((wl.nz, wl.ny, wl.nx), device=dev)
+    ms = _timed_shots(lambda: mig.migrate(rshot, data, img, stream), 1, stream)
+    nseg = (nsnap + c - 1) // c if c else 1
+    recomputed = sum(min((s_ + 1) * c, nsnap) * wl.snap - s_ * c * wl.snap for s_ in range(nseg - 1)) if c else 0
+    mig.close()
+    del mig, img, data
+    torch.cuda.empty_cache()
+    return {"shots_per_hour": round(3600.0 / (ms * 1e-3), 1), "ms_per_shot": round(ms, 1),
+            "gpts_s_both_phases": round(2 * wl.npts * wl.nt / (ms * 1e-3) / 1e9, 3),
+            "gpts_s_all_propagated_steps": round(wl.npts * (2 * wl.nt + recomputed) / (ms * 1e-3) / 1e9, 3),
+            "forward_gpts_s": round(wl.npts * wl.nt / (fms * 1e-3) / 1e9, 3),
+            "snapshots": nsnap, "ckpt_period": c, "segments": nseg, "recomputed_steps": recomputed,
+            "receivers": shot.nrec, "model_build_s": round(build_s, 1),
+            "note": "1 GPU; BASELINE C5 names 2/4/8 B200 (the driver's scaling run of the C2 line covers N > 1)"}
 
 
 # ---------------------------------------------------------------- oracle arm
@@ -527,6 +585,7 @@ def main():
     ap.add_argument("--nt", type=int, default=2000, help="time steps per shot (2000 = C2)")
     ap.add_argument("--ref-steps", type=int, default=1, help="oracle time steps per reference step")
     ap.add_argument("--no-extras", action="store_true")
+    ap.add_argument("--no-c5", action="store_true", help="skip the 1024^3 RTM extra (about 2 minutes)")
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
                     help="N>1: weak = n^3 per rank (default), strong = one n^3 grid split in z-slabs")
     ap.add_argument("--halo", default="nccl", choices=["nccl", "peer"],

@@ -141,6 +141,38 @@ def smooth(model, sigma):
             for k, v in model.items()}
 
 
+def smooth_torch(model, sigma, device):
+    """The same migration model as smooth() -- separable 3D Gaussian, sigma in points, 'nearest'
+    edges -- computed with torch on `device` (1024^3 grids; input preparation, not the method)."""
+    import torch
+
+    r = int(4 * sigma + 0.5)
+    x = torch.arange(-r, r + 1, dtype=torch.float32, device=device)
+    w = torch.exp(-0.5 * (x / sigma) ** 2)
+    w = (w / w.sum()).view(1, 1, -1)
+    F = torch.nn.functional
+    out_model = {}
+    for key, a in model.items():
+        t = torch.from_numpy(np.ascontiguousarray(a, dtype=np.float32)).to(device)
+        nz, ny, nx = t.shape
+        out = torch.empty_like(t)
+        for k in range(nz):  # x and y, plane by plane (small temporaries)
+            p = t[k]
+            p = F.conv1d(F.pad(p.view(ny, 1, nx), (r, r), mode="replicate"), w).view(ny, nx)
+            p = F.conv1d(F.pad(p.t().contiguous().view(nx, 1, ny), (r, r), mode="replicate"), w).view(nx, ny).t()
+            out[k] = p
+        del t
+        for j0 in range(0, ny, 64):  # z, per block of rows
+            blk = out[:, j0:j0 + 64, :].permute(1, 2, 0).contiguous()  # [yb][nx][nz]
+            yb = blk.shape[0]
+            b = F.conv1d(F.pad(blk.view(yb * nx, 1, nz), (r, r), mode="replicate"), w)
+            out[:, j0:j0 + 64, :] = b.view(yb, nx, nz).permute(2, 0, 1)
+        out_model[key] = out.cpu().numpy()
+        del out
+        torch.cuda.empty_cache()
+    return out_model
+
+
 def layered_elastic(nx, ny, nz):
     """C3 recipe: layers at z = 60, 160, 280 (of 384, scaled): (vp, vs, rho) =
     (2000,1000,2000), (2800,1600,2200), (3500,2000,2400), (4500,2600,2600)."""

@@ -39,34 +39,6 @@ def timed(fn, stream, reps=1, warm=1):
     return e0.elapsed_time(e1) / reps
 
 
-def smooth_gpu(a, sigma, dev):
-    """Migration model: separable 3D Gaussian (sigma in points, 'nearest' edges) on the GPU,
-    plane by plane so the temporaries stay small (input preparation, not the method)."""
-    r = int(4 * sigma + 0.5)
-    x = torch.arange(-r, r + 1, dtype=torch.float32, device=dev)
-    w = torch.exp(-0.5 * (x / sigma) ** 2)
-    w = (w / w.sum()).view(1, 1, -1)
-    t = torch.from_numpy(a).to(dev)
-    nz, ny, nx = t.shape
-    out = torch.empty_like(t)
-    # x and y: per z-plane
-    for k in range(nz):
-        p = t[k]
-        p = torch.nn.functional.conv1d(torch.nn.functional.pad(p.view(ny, 1, nx), (r, r), mode="replicate"), w).view(ny, nx)
-        p = torch.nn.functional.conv1d(torch.nn.functional.pad(p.t().contiguous().view(nx, 1, ny), (r, r), mode="replicate"), w).view(nx, ny).t()
-        out[k] = p
-    # z: per y-row block
-    for j0 in range(0, ny, 64):
-        blk = out[:, j0:j0 + 64, :].permute(1, 2, 0).contiguous()  # [yb][nx][nz]
-        yb = blk.shape[0]
-        b = torch.nn.functional.conv1d(torch.nn.functional.pad(blk.view(yb * nx, 1, nz), (r, r), mode="replicate"), w)
-        out[:, j0:j0 + 64, :] = b.view(yb, nx, nz).permute(2, 0, 1)
-    res = out.cpu().numpy()
-    del t, out
-    torch.cuda.empty_cache()
-    return res
-
-
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--n", type=int, default=1024)
@@ -97,7 +69,7 @@ def main():
 
     # 2. checkpointed RTM on the smoothed model
     t0 = time.time()
-    sm = {k: smooth_gpu(v, 5.0, dev) for k, v in wl.model.items()}
+    sm = inputs.smooth_torch(wl.model, 5.0, dev)
     res["smooth_s"] = round(time.time() - t0, 1)
     del wl.model
     free, total = torch.cuda.mem_get_info(dev)
