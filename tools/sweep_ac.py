@@ -1,4 +1,4 @@
-"""Acoustic-step variant sweep (fused f1 kernel tile heights / ring depth vs the split pair).
+"""Acoustic-step variant sweep: the split pair's z-chunking vs the fused persistent step (f1).
 
     python tools/sweep_ac.py build      # here: compile the variants into sweep_out/
     python tools/sweep_ac.py run        # on a B200: C2 512^3, 60 steps, per-kernel CUDA-event ms
@@ -13,18 +13,12 @@ OUT = os.path.join(ROOT, "sweep_out")
 sys.path.insert(0, ROOT)
 
 VARIANTS = {  # name: (defines, env)
-    "split": ([], {}),
-    "f16": (["SEIS_BYF=16"], {"SEIS_AC_FUSED": "1"}),
-    "f32": (["SEIS_BYF=32"], {"SEIS_AC_FUSED": "1"}),
-    "f8": (["SEIS_BYF=8"], {"SEIS_AC_FUSED": "1"}),
-    "f8_z32": (["SEIS_BYF=8"], {"SEIS_AC_FUSED": "1", "SEIS_ZCHUNK_MAX": "32"}),
-    "f8_z16": (["SEIS_BYF=8"], {"SEIS_AC_FUSED": "1", "SEIS_ZCHUNK_MAX": "16"}),
-    "f8ns3": (["SEIS_BYF=8", "SEIS_AF_NS=3"], {"SEIS_AC_FUSED": "1"}),
-    "f8ns3_z32": (["SEIS_BYF=8", "SEIS_AF_NS=3"], {"SEIS_AC_FUSED": "1", "SEIS_ZCHUNK_MAX": "32"}),
-    "f16_z32": (["SEIS_BYF=16"], {"SEIS_AC_FUSED": "1", "SEIS_ZCHUNK_MAX": "32"}),
-    "split_z128": ([], {"SEIS_ZCHUNK_MAX": "128"}),
-    "split_z64": ([], {"SEIS_ZCHUNK_MAX": "64"}),
-    "split_z32": ([], {"SEIS_ZCHUNK_MAX": "32"}),
+    "split": ([], {"SEIS_AC_STEP": "0"}),
+    "step": ([], {"SEIS_AC_STEP": "1"}),
+    "step_pf8": (["SEIS_AS_PF=8"], {"SEIS_AC_STEP": "1"}),
+    "split_z128": ([], {"SEIS_AC_STEP": "0", "SEIS_ZCHUNK_MAX": "128"}),
+    "split_z64": ([], {"SEIS_AC_STEP": "0", "SEIS_ZCHUNK_MAX": "64"}),
+    "split_z32": ([], {"SEIS_AC_STEP": "0", "SEIS_ZCHUNK_MAX": "32"}),
 }
 if os.environ.get("SWEEP_ONLY"):
     VARIANTS = {k: v for k, v in VARIANTS.items() if k in os.environ["SWEEP_ONLY"].split(",")}
