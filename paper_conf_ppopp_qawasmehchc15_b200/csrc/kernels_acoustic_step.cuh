@@ -67,9 +67,14 @@ constexpr int AS_NSV = SEIS_AS_NSV;
 // NSV / NSP deep (one CTA per SM holds ~200 KB), so the HBM latency is covered by bringing each
 // plane into L2 AS_PF planes before its TMA load (cp.async.bulk.prefetch.tensor, no smem)
 #ifndef SEIS_AS_PF
-#define SEIS_AS_PF 4
+#define SEIS_AS_PF 2
 #endif
 constexpr int AS_PF = SEIS_AS_PF;
+// per-thread L2 prefetch of the C-PML slabs (prefetch.global.L2): measured slower (1.69 ms per
+// 512^3 step with it, 1.50 without), off by default
+#ifndef SEIS_AS_PSIPF
+#define SEIS_AS_PSIPF 0
+#endif
 constexpr int AS_NSP = SEIS_AS_NSP;
 
 struct AcSArgs {
@@ -584,7 +589,7 @@ __global__ void __launch_bounds__(AS_THREADS, 1) ac_step_kernel(const __grid_con
           if (vec4) psi_upd_v4(dz, a.psz, iz[0], ov.v, ca, cb);
           else psi_upd_s<4>(dz, a.psz, iz, ov.v, ca, cb);
         }
-        if (Wl > 0) {  // L2 prefetch of the memory variables AS_PF planes ahead (both halves)
+        if (SEIS_AS_PSIPF && Wl > 0) {  // L2 prefetch of the memory variables AS_PF planes ahead
           psi_prefetch(psv, j + AS_PF);
           psi_prefetch(psp, j + AS_PF);
         }
