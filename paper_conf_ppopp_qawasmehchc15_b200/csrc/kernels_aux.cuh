@@ -29,9 +29,9 @@ __global__ void gather_kernel(float* __restrict__ seis_row, const float* __restr
   seis_row[rid[t]] = v;
 }
 
-// Backward-phase receiver injection (O15): for each distinct node u of this slab,
-//   f[off[u]] += scale[u] * sum_{r in group u, index order} data_row[r]
-// (ELASTIC is not migrated in this version.)
+// Backward-phase receiver injection (O15), ISO and ACOUSTIC: for each distinct node u of this
+// slab, f[off[u]] += scale[u] * sum_{r in group u, index order} data_row[r]
+// (ELASTIC receivers inject like the explosive source: inject_el_kernel below.)
 __global__ void inject_kernel(float* __restrict__ f, const long long* __restrict__ off,
                               const float* __restrict__ scale, const int* __restrict__ gstart,
                               const int* __restrict__ members, const float* __restrict__ data_row,
