@@ -429,7 +429,8 @@ def run_c5(local, n=1024, nt=1000):
         fits = [cc for cc in range(1, nsnap + 1)
                 if seis.memory_required(g, "acoustic", seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap,
                                                                  ckpt_period=cc)) + img_bytes <= 0.95 * free]
-        c = max(fits)
+        # fewest recomputed steps: every segment but the last is recomputed once, (nseg - 1) c
+        c = min(fits, key=lambda cc: ((nsnap + cc - 1) // cc - 1) * cc)
     rshot = seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap, ckpt_period=c)
     mig = seis.Model(g, "acoustic", sm["vp"], rho=sm["rho"], device=local)
     del sm

@@ -82,15 +82,14 @@ def main():
         if seis.memory_required(g, "acoustic", seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap,
                                                          snap_bits=bits)) + img_bytes <= 0.95 * free:
             return 0
-        best = None
-        for cc in range(1, nsnap + 1):
-            need = seis.memory_required(g, "acoustic", seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap,
-                                                                 ckpt_period=cc, snap_bits=bits))
-            if need + img_bytes <= 0.95 * free:
-                best = cc if best is None else max(best, cc)
-        if best is None:
+        fits = [cc for cc in range(1, nsnap + 1)
+                if seis.memory_required(g, "acoustic", seis.Shot(wl.src, wl.wavelet, wl.rec, snap_period=wl.snap,
+                                                                 ckpt_period=cc, snap_bits=bits)) + img_bytes
+                <= 0.95 * free]
+        if not fits:
             raise SystemExit("C5 RTM does not fit even with checkpointing")
-        return best
+        # fewest recomputed steps: every segment but the last is recomputed once, (nseg - 1) c
+        return min(fits, key=lambda cc: ((nsnap + cc - 1) // cc - 1) * cc)
 
     def recomputed(c):
         if not c:
