@@ -271,7 +271,10 @@ def run_product(args):
     torch.cuda.empty_cache()
     if rank == 0 and ws == 1:
         if not args.no_extras:
-            out["extras"] = run_extras(args, local)
+            try:
+                out["extras"] = run_extras(args, local)
+            except Exception as e:  # (reported, never fatal to the headline line)
+                out["extras"] = {"error": repr(e)[:300]}
         out["cpu_baseline"] = cpu_baseline(args)
     if ws > 1:
         dist.destroy_process_group()
@@ -391,7 +394,11 @@ def run_extras(args, local):
     del mig, true, data, img, smooth, wl
     torch.cuda.empty_cache()
     if not args.no_c5:
-        res["C5_rtm_1024_1gpu"] = run_c5(local)
+        try:
+            res["C5_rtm_1024_1gpu"] = run_c5(local)
+        except Exception as e:  # an extra must never sink the headline line
+            res["C5_rtm_1024_1gpu"] = {"error": repr(e)[:300]}
+            torch.cuda.empty_cache()
     return res
 
 
