@@ -61,6 +61,10 @@ struct IsoArgs {
   Dims d;
   int zc;                        // z-chunk length
   int ch0, chs;                  // z-chunk of blockIdx.z = ch0 + blockIdx.z * chs (boundary / interior split)
+  // Region split of the split-field PML step (O6b): 0 = every block; 1 = only blocks whose tile
+  // and z-chunk hold no layer point (the plain kernel, high occupancy); 2 = only the other
+  // blocks (the SPML kernel).  nbr = layer width (points) for the test.
+  int region, nbr;
   long long src_o;               // padded index of the source node in this slab, -1 = none
   SrcAmp src;                    // scale * s[n]
   float* __restrict__ snap;      // compact [nzl][ny][nx] or nullptr
@@ -124,6 +128,12 @@ __global__ void __launch_bounds__(NTX * BY, SPML ? SEIS_SPML_MINB : 1) iso_step_
   const int k0 = (a.ch0 + (int)blockIdx.z * a.chs) * a.zc;
   const int k1 = min(k0 + a.zc, d.nzl);
   const int np = k1 - k0;
+  if (a.region) {  // block-uniform: is this block's (tile, chunk) free of layer points?
+    const int nb = a.nbr;
+    const bool inner = i0 >= nb && min(i0 + TXV, d.nx) - 1 <= d.nx - 1 - nb && j0 >= nb &&
+                       min(j0 + BY, d.ny) - 1 <= d.ny - 1 - nb && k0 + d.z0 >= nb && k1 - 1 + d.z0 <= d.nz - 1 - nb;
+    if (inner != (a.region == 1)) return;
+  }
   const bool own = (x0 < d.nx) && (j < d.ny);
   const long long PS = d.PS;
   const long long oc = (long long)(j + G) * d.PX + (x0 + G);

@@ -1623,7 +1623,16 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
           else iso_step_kernel<BYI, false, false, SP, GH><<<gr, blk, sb, ks>>>(a);
         };
         const bool gh = a.gh.lo || a.gh.hi;
+        a.region = 0;
+        a.nbr = M->g.nb;
         if (S.sp) {
+          // O6b: the blocks without layer points run the plain kernel (96 registers, high
+          // occupancy), the others the split-field kernel; disjoint points, same arithmetic for
+          // the non-layer points of either
+          a.region = 1;
+          if (gh) go(std::false_type{}, std::true_type{});
+          else go(std::false_type{}, std::false_type{});
+          a.region = 2;
           if (gh) go(std::true_type{}, std::true_type{});
           else go(std::true_type{}, std::false_type{});
         } else if (gh) go(std::false_type{}, std::true_type{});
