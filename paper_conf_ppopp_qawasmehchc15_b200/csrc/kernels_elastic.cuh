@@ -88,6 +88,21 @@ __device__ __forceinline__ F2 ldg2_fs(const float* __restrict__ f, int p, long l
 #define SEIS_EL_WS 1
 #endif
 constexpr int EL_WS = SEIS_EL_WS;
+// C-PML memory variables by cp.async (measured and rejected, off): the old values of plane
+// k + 1 travel into per-thread shared slots (9 arrays x 2 points) while plane k computes,
+// instead of being loaded into registers before the stage wait.  Correct (parity green) but
+// el_v 0.734 vs 0.680 ms at C3 (the 4-byte cp.async issue + wait costs more than the register
+// preload hides), and el_s needs a 2-stage ring to fit the slots (0.987 vs 0.886 ms);
+// profiles/r02_el_psa_variants.log
+#ifndef SEIS_EL_PSA
+#define SEIS_EL_PSA 0
+#endif
+#ifndef SEIS_EL_VPSA
+#define SEIS_EL_VPSA SEIS_EL_PSA
+#endif
+#ifndef SEIS_EL_SPSA
+#define SEIS_EL_SPSA SEIS_EL_PSA
+#endif
 // (warp specialization) L2 prefetch distance of the producer, planes ahead of the ring loads
 #ifndef SEIS_EL_PF
 #define SEIS_EL_PF 0
@@ -140,7 +155,8 @@ struct ElVStage {
                        Q = RZ + r32(T), R = Q + 3 * r32(T), SIZE = R + r32(RW * (BY + 1));
   static constexpr int TS = r32(T);  // stride of the 3 v / 3 q tiles
   static constexpr uint32_t BYTES = (2 * BY * WX + (BY + 8) * WX + 2 * (BY + 8) * TXE + 7 * T + RW * (BY + 1)) * 4;
-  static constexpr size_t smem_bytes() { return (size_t)EL_VNS * SIZE * 4 + 128; }
+  static constexpr int PSLOT = 9 * NTX2 * BY * 2;  // per-thread C-PML slots (floats)
+  static constexpr size_t smem_bytes() { return ((size_t)EL_VNS * SIZE + (SEIS_EL_VPSA ? PSLOT : 0)) * 4 + 128; }
 };
 
 template <int BY, bool IMG>
@@ -216,6 +232,36 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
     for (int s = 0; s < EL_VNS && s < np; ++s) issue(s, k0 + s);
   if (!EL_WS && tid == 0)
     for (int t = 0; t < L2PF && EL_VNS + t < np; ++t) issue(0, k0 + EL_VNS + t, true);
+  // (C-PML by cp.async) per-thread slots of the 9 memory variables of plane kk (2 points each)
+  float* const psl = sm + EL_VNS * L::SIZE + 2 * tid;
+  constexpr int PST = NTX2 * BY * 2;  // slot stride of one array
+  auto psi_issue = [&](int kk) {
+    const int gzk = kk + d.z0;
+    int ix[2];
+    if (own && lx) {
+      psi_idx_x<2>(ix, d, W, x0, j, kk);
+#pragma unroll
+      for (int e = 0; e < 2; ++e)
+        if (ix[e] >= 0)
+          for (int t : {0, 3, 6}) cp_async4(psl + t * PST + e, a.psi[t] + ix[e], true);
+    }
+    if (own && ly) {
+      psi_idx_row<2>(ix, (kk * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0, x0, d.nx);
+#pragma unroll
+      for (int e = 0; e < 2; ++e)
+        if (ix[e] >= 0)
+          for (int t : {1, 4, 7}) cp_async4(psl + t * PST + e, a.psi[t] + ix[e], true);
+    }
+    if (own && W > 0 && CpmlIdx::in(gzk, d.nz, W, a.zlo)) {
+      psi_idx_row<2>(ix, (CpmlIdx::slot(gzk, d.nz, W) * d.ny + j) * d.nx + x0, x0, d.nx);
+#pragma unroll
+      for (int e = 0; e < 2; ++e)
+        if (ix[e] >= 0)
+          for (int t : {2, 5, 8}) cp_async4(psl + t * PST + e, a.psi[t] + ix[e], true);
+    }
+    cp_async_commit();
+  };
+  if (SEIS_EL_VPSA && W > 0 && np > 0) psi_issue(k0);
   const float* __restrict__ sxz = a.f[ESXZ];
   const float* __restrict__ syz = a.f[ESYZ];
   const float* __restrict__ szz = a.f[ESZZ];
@@ -245,19 +291,19 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
     const bool lz = W > 0 && CpmlIdx::in(gz, d.nz, W, a.zlo);
     int ixx[2], iyy[2], izz[2];  // 32-bit compact-slab indices (fewer live registers)
     float ox0[2], ox3[2], ox6[2], oy1[2], oy4[2], oy7[2], oz2[2], oz5[2], oz8[2];
-    if (own && lx) {
+    if (!SEIS_EL_VPSA && own && lx) {
       psi_idx_x<2>(ixx, d, W, x0, j, k);
       psi_ld<2>(ox0, a.psi[0], ixx);
       psi_ld<2>(ox3, a.psi[3], ixx);
       psi_ld<2>(ox6, a.psi[6], ixx);
     }
-    if (own && ly) {
+    if (!SEIS_EL_VPSA && own && ly) {
       psi_idx_row<2>(iyy, (k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0, x0, d.nx);
       psi_ld<2>(oy1, a.psi[1], iyy);
       psi_ld<2>(oy4, a.psi[4], iyy);
       psi_ld<2>(oy7, a.psi[7], iyy);
     }
-    if (own && lz) {
+    if (!SEIS_EL_VPSA && own && lz) {
       psi_idx_row<2>(izz, (CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0, x0, d.nx);
       psi_ld<2>(oz2, a.psi[2], izz);
       psi_ld<2>(oz5, a.psi[5], izz);
@@ -296,6 +342,27 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
         d6[e] = dm(xz, 4 + e);   // Dx- sxz
         d7[e] = dm(yyz[e], 4);   // Dy- syz
         d8[e] = dp(zzz, 3);      // Dz+ szz  (zzz[0..7] = k-3..k+4)
+      }
+      if (SEIS_EL_VPSA && W > 0) {  // the slots of this plane (issued one plane ahead)
+        cp_async_wait<0>();
+        if (lx) {
+          psi_idx_x<2>(ixx, d, W, x0, j, k);
+          { const F2 v = lds2(psl + 0 * PST); ox0[0] = v.v[0]; ox0[1] = v.v[1]; }
+          { const F2 v = lds2(psl + 3 * PST); ox3[0] = v.v[0]; ox3[1] = v.v[1]; }
+          { const F2 v = lds2(psl + 6 * PST); ox6[0] = v.v[0]; ox6[1] = v.v[1]; }
+        }
+        if (ly) {
+          psi_idx_row<2>(iyy, (k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0, x0, d.nx);
+          { const F2 v = lds2(psl + 1 * PST); oy1[0] = v.v[0]; oy1[1] = v.v[1]; }
+          { const F2 v = lds2(psl + 4 * PST); oy4[0] = v.v[0]; oy4[1] = v.v[1]; }
+          { const F2 v = lds2(psl + 7 * PST); oy7[0] = v.v[0]; oy7[1] = v.v[1]; }
+        }
+        if (lz) {
+          psi_idx_row<2>(izz, (CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0, x0, d.nx);
+          { const F2 v = lds2(psl + 2 * PST); oz2[0] = v.v[0]; oz2[1] = v.v[1]; }
+          { const F2 v = lds2(psl + 5 * PST); oz5[0] = v.v[0]; oz5[1] = v.v[1]; }
+          { const F2 v = lds2(psl + 8 * PST); oz8[0] = v.v[0]; oz8[1] = v.v[1]; }
+        }
       }
       if (lx) {
         float ca[2], cb[2], cah[2], cbh[2];
@@ -359,6 +426,7 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
           }
       }
     }
+    if (SEIS_EL_VPSA && W > 0 && it + 1 < np) psi_issue(k + 1);  // (own slots are consumed)
     if (EL_WS) {
       __syncwarp();
       if (tx == 0) mbar_arrive(&ebar[s]);
@@ -403,7 +471,8 @@ struct ElSStage {
   static constexpr int VT = 0, S = 3 * TV, C = S + 6 * TS, Q = C + TS, WK = Q + 3 * TS, WK1 = WK + WT,
                        SIZE = WK1 + WT;
   static constexpr uint32_t BYTES = (3 * (BY + 8) * WX + 10 * T + 2 * RW * (BY + 1)) * 4;  // what the TMA boxes deliver
-  static constexpr size_t smem_bytes() { return (size_t)EL_SNS * SIZE * 4 + 128; }
+  static constexpr int PSLOT = 9 * NTX2 * BY * 2;  // per-thread C-PML slots (floats)
+  static constexpr size_t smem_bytes() { return ((size_t)EL_SNS * SIZE + (SEIS_EL_SPSA ? PSLOT : 0)) * 4 + 128; }
 };
 
 template <int BY, bool SNAP>
@@ -475,6 +544,36 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
     for (int s = 0; s < EL_SNS && s < np; ++s) issue(s, k0 + s);
   if (!EL_WS && tid == 0)
     for (int t = 0; t < L2PF && EL_SNS + t < np; ++t) issue(0, k0 + EL_SNS + t, true);
+  // (C-PML by cp.async) per-thread slots of the 9 memory variables of plane kk (2 points each)
+  float* const psl = sm + EL_SNS * L::SIZE + 2 * tid;
+  constexpr int PST = NTX2 * BY * 2;  // slot stride of one array
+  auto psi_issue = [&](int kk) {
+    const int gzk = kk + d.z0;
+    int ix[2];
+    if (own && lx) {
+      psi_idx_x<2>(ix, d, W, x0, j, kk);
+#pragma unroll
+      for (int e = 0; e < 2; ++e)
+        if (ix[e] >= 0)
+          for (int t : {0, 4, 6}) cp_async4(psl + t * PST + e, a.psi[t] + ix[e], true);
+    }
+    if (own && ly) {
+      psi_idx_row<2>(ix, (kk * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0, x0, d.nx);
+#pragma unroll
+      for (int e = 0; e < 2; ++e)
+        if (ix[e] >= 0)
+          for (int t : {1, 3, 8}) cp_async4(psl + t * PST + e, a.psi[t] + ix[e], true);
+    }
+    if (own && W > 0 && CpmlIdx::in(gzk, d.nz, W, a.zlo)) {
+      psi_idx_row<2>(ix, (CpmlIdx::slot(gzk, d.nz, W) * d.ny + j) * d.nx + x0, x0, d.nx);
+#pragma unroll
+      for (int e = 0; e < 2; ++e)
+        if (ix[e] >= 0)
+          for (int t : {2, 5, 7}) cp_async4(psl + t * PST + e, a.psi[t] + ix[e], true);
+    }
+    cp_async_commit();
+  };
+  if (SEIS_EL_SPSA && W > 0 && np > 0) psi_issue(k0);
   const float* __restrict__ vx = a.f[EVX];
   const float* __restrict__ vy = a.f[EVY];
   const float* __restrict__ vz = a.f[EVZ];
@@ -505,19 +604,19 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
     const bool lz = W > 0 && CpmlIdx::in(gz, d.nz, W, a.zlo);
     int ixx[2], iyy[2], izz[2];  // 32-bit compact-slab indices (fewer live registers)
     float ox0[2], ox4[2], ox6[2], oy1[2], oy3[2], oy8[2], oz2[2], oz5[2], oz7[2];
-    if (own && lx) {
+    if (!SEIS_EL_SPSA && own && lx) {
       psi_idx_x<2>(ixx, d, W, x0, j, k);
       psi_ld<2>(ox0, a.psi[0], ixx);
       psi_ld<2>(ox4, a.psi[4], ixx);
       psi_ld<2>(ox6, a.psi[6], ixx);
     }
-    if (own && ly) {
+    if (!SEIS_EL_SPSA && own && ly) {
       psi_idx_row<2>(iyy, (k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0, x0, d.nx);
       psi_ld<2>(oy1, a.psi[1], iyy);
       psi_ld<2>(oy3, a.psi[3], iyy);
       psi_ld<2>(oy8, a.psi[8], iyy);
     }
-    if (own && lz) {
+    if (!SEIS_EL_SPSA && own && lz) {
       psi_idx_row<2>(izz, (CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0, x0, d.nx);
       psi_ld<2>(oz2, a.psi[2], izz);
       psi_ld<2>(oz5, a.psi[5], izz);
@@ -559,6 +658,27 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
         dxvz[e] = dp(xvz, 4 + e);  // Dx+ vz
         dzvy[e] = dp(zy, 3);       // Dz+ vy
         dyvz[e] = dp(yvz[e], 4);   // Dy+ vz
+      }
+      if (SEIS_EL_SPSA && W > 0) {  // the slots of this plane (issued one plane ahead)
+        cp_async_wait<0>();
+        if (lx) {
+          psi_idx_x<2>(ixx, d, W, x0, j, k);
+          { const F2 v = lds2(psl + 0 * PST); ox0[0] = v.v[0]; ox0[1] = v.v[1]; }
+          { const F2 v = lds2(psl + 4 * PST); ox4[0] = v.v[0]; ox4[1] = v.v[1]; }
+          { const F2 v = lds2(psl + 6 * PST); ox6[0] = v.v[0]; ox6[1] = v.v[1]; }
+        }
+        if (ly) {
+          psi_idx_row<2>(iyy, (k * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0, x0, d.nx);
+          { const F2 v = lds2(psl + 1 * PST); oy1[0] = v.v[0]; oy1[1] = v.v[1]; }
+          { const F2 v = lds2(psl + 3 * PST); oy3[0] = v.v[0]; oy3[1] = v.v[1]; }
+          { const F2 v = lds2(psl + 8 * PST); oy8[0] = v.v[0]; oy8[1] = v.v[1]; }
+        }
+        if (lz) {
+          psi_idx_row<2>(izz, (CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0, x0, d.nx);
+          { const F2 v = lds2(psl + 2 * PST); oz2[0] = v.v[0]; oz2[1] = v.v[1]; }
+          { const F2 v = lds2(psl + 5 * PST); oz5[0] = v.v[0]; oz5[1] = v.v[1]; }
+          { const F2 v = lds2(psl + 7 * PST); oz7[0] = v.v[0]; oz7[1] = v.v[1]; }
+        }
       }
       if (lx) {
         float ca[2], cb[2], cah[2], cbh[2];
@@ -647,6 +767,7 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
           if (x0 + e < d.nx) a.snap[cix + e] = -((o6[0].v[e] + o6[1].v[e]) + o6[2].v[e]) / 3.0f;
       }
     }
+    if (SEIS_EL_SPSA && W > 0 && it + 1 < np) psi_issue(k + 1);  // (own slots are consumed)
     if (EL_WS) {
       __syncwarp();
       if (tx == 0) mbar_arrive(&ebar[s]);

@@ -18,8 +18,9 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--n", type=int, default=384)
     ap.add_argument("--nt", type=int, default=100)
+    ap.add_argument("--nb", type=int, default=20)
     a = ap.parse_args()
-    wl = inputs.c3(n=a.n, nt=a.nt)
+    wl = inputs.c3(n=a.n, nt=a.nt, nb=a.nb)
     g = seis.Grid(wl.nx, wl.ny, wl.nz, wl.h, wl.dt, nb=wl.nb, free_surface=1, pml_f=wl.fp)
     m = seis.Model(g, "elastic", wl.model["vp"], vs=wl.model["vs"], rho=wl.model["rho"])
     shot = seis.Shot(wl.src, wl.wavelet, wl.rec, rec_component=2)
@@ -40,9 +41,9 @@ def main():
     seis.profile(False)
     kp = seis.profile_read()
     W = wl.nb + 1
-    psi = 8.0 * (2 * W / wl.nx + 2 * W / wl.ny + W / wl.nz) * 9 / 3.0
+    psi = 8.0 * (2 * W / wl.nx + 2 * W / wl.ny + W / wl.nz) * 9 / 3.0 if wl.nb else 0.0
     hbm = 6538.3
-    res = {"n": a.n, "nt": a.nt, "ms_per_step": round(ms / a.nt, 4), "gpts_s": round(wl.npts * a.nt / (ms * 1e-3) / 1e9, 2),
+    res = {"n": a.n, "nt": a.nt, "nb": a.nb, "ms_per_step": round(ms / a.nt, 4), "gpts_s": round(wl.npts * a.nt / (ms * 1e-3) / 1e9, 2),
            "seis_norm": float(out.norm().item())}
     for k, b in (("el_v", 52.0), ("el_s", 68.0)):
         t = kp[k][0] / kp[k][1]
