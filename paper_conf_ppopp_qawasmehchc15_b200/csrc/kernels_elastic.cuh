@@ -135,6 +135,7 @@ struct ElVArgs {
   CUtensorMap mq[3];  // z-queue feeds: sxz (k+3), syz (k+3), szz (k+4), box 64 x BY
   float* f[9];
   int W, zlo, fs;
+  int region;  // 0: every block; 1: only blocks free of C-PML points; 2: only the others
   float dth;       // dt / h (face buoyancy dt b/h = dth * 2/(rho_i + rho_{i+1}), O8/O9)
   CpmlAxis cx, cy, cz;
   float* psi[9];   // psi 0..8
@@ -146,6 +147,17 @@ struct ElVArgs {
   float* __restrict__ img;
   Ghost gh[3];                     // direct ghost stores of vx, vy, vz (f4)
 };
+
+// (region split) conservative, block-uniform: may this block's tile (TXE x BY at i0, j0) and
+// z-chunk [k0, k1) hold a C-PML point?  (A block that does runs the CP instantiation, which is
+// correct everywhere; one that does not may run either.)
+__device__ __forceinline__ bool el_block_in_layers(const Dims& d, int W, int zlo, int i0, int j0, int by, int k0,
+                                                   int k1) {
+  if (W <= 0) return false;
+  const bool inner = i0 >= W && i0 + TXE <= d.nx - W && j0 >= W && j0 + by <= d.ny - W &&
+                     (!zlo || k0 + d.z0 >= W) && k1 + d.z0 <= d.nz - W;
+  return !inner;
+}
 
 template <int BY>
 struct ElVStage {
@@ -159,7 +171,7 @@ struct ElVStage {
   static constexpr size_t smem_bytes() { return ((size_t)EL_VNS * SIZE + (SEIS_EL_VPSA ? PSLOT : 0)) * 4 + 128; }
 };
 
-template <int BY, bool IMG>
+template <int BY, bool IMG, bool CP>
 __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (BY <= 8 ? 2 : 1)) el_v_kernel(const __grid_constant__ ElVArgs a) {
   using L = ElVStage<BY>;
   constexpr int WX = L::WX;
@@ -184,7 +196,10 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
   const bool own = (x0 < d.nx) && (j < d.ny);
   const long long PS = d.PS;
   const long long oc = (long long)(j + G) * d.PX + (x0 + G);
-  const int W = a.W;
+  // (region split) CP = false: the instantiation without the C-PML code, for blocks whose
+  // tile and z-chunk hold no layer point (fewer instructions, no spills)
+  if (a.region && el_block_in_layers(d, a.W, a.zlo, i0, j0, BY, k0, k1) != (a.region == 2)) return;
+  const int W = CP ? a.W : 0;
   const bool lx = W > 0 && (x0 < W || x0 + 1 >= d.nx - W);
   const bool ly = W > 0 && CpmlIdx::in(j, d.ny, W, true);
   auto issue = [&](int s, int k, bool pf = false) {
@@ -212,7 +227,7 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
     }
     mbar_fence_init();
   }
-  cpml_tile_fill(ctile, a.cx, a.cy, blockIdx.x * TXE, blockIdx.y * BY, a.d.nx, a.d.ny, a.W > 0, tid,
+  cpml_tile_fill(ctile, a.cx, a.cy, blockIdx.x * TXE, blockIdx.y * BY, a.d.nx, a.d.ny, W > 0, tid,
                  NTX2 * (BY + EL_WS));
   __syncthreads();
   if (EL_WS && ty == BY) {  // producer warp: lane 0 refills each stage once all warps released it
@@ -453,6 +468,7 @@ struct ElSArgs {
   CUtensorMap mq[3];   // z-queue feeds: vx (k+4), vy (k+4), vz (k+3), box 64 x BY
   float* f[9];
   int W, zlo, fs;
+  int region;  // 0: every block; 1: only blocks free of C-PML points; 2: only the others
   CpmlAxis cx, cy, cz;
   float* psi[9];   // psi 9..17
   Dims d;
@@ -475,7 +491,7 @@ struct ElSStage {
   static constexpr size_t smem_bytes() { return ((size_t)EL_SNS * SIZE + (SEIS_EL_SPSA ? PSLOT : 0)) * 4 + 128; }
 };
 
-template <int BY, bool SNAP>
+template <int BY, bool SNAP, bool CP>
 __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (BY <= 8 ? 2 : 1)) el_s_kernel(const __grid_constant__ ElSArgs a) {
   using L = ElSStage<BY>;
   constexpr int WX = L::WX, TV = L::TV, RW = L::RW;
@@ -498,7 +514,10 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
   const bool own = (x0 < d.nx) && (j < d.ny);
   const long long PS = d.PS;
   const long long oc = (long long)(j + G) * d.PX + (x0 + G);
-  const int W = a.W;
+  // (region split) CP = false: the instantiation without the C-PML code, for blocks whose
+  // tile and z-chunk hold no layer point (fewer instructions, no spills)
+  if (a.region && el_block_in_layers(d, a.W, a.zlo, i0, j0, BY, k0, k1) != (a.region == 2)) return;
+  const int W = CP ? a.W : 0;
   const bool lx = W > 0 && (x0 < W || x0 + 1 >= d.nx - W);
   const bool ly = W > 0 && CpmlIdx::in(j, d.ny, W, true);
   auto issue = [&](int s, int k, bool pf = false) {
@@ -524,7 +543,7 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
     }
     mbar_fence_init();
   }
-  cpml_tile_fill(ctile, a.cx, a.cy, blockIdx.x * TXE, blockIdx.y * BY, a.d.nx, a.d.ny, a.W > 0, tid,
+  cpml_tile_fill(ctile, a.cx, a.cy, blockIdx.x * TXE, blockIdx.y * BY, a.d.nx, a.d.ny, W > 0, tid,
                  NTX2 * (BY + EL_WS));
   __syncthreads();
   if (EL_WS && ty == BY) {  // producer warp: lane 0 refills each stage once all warps released it

@@ -393,13 +393,41 @@ seis_status set_smem_attrs() {
   SMEM_ATTR((ac_step_kernel<false, false>), AcSLayout::smem_bytes());
   SMEM_ATTR((ac_step_kernel<true, false>), AcSLayout::smem_bytes());
   SMEM_ATTR((ac_step_kernel<false, true>), AcSLayout::smem_bytes());
-  SMEM_ATTR((el_v_kernel<BYE, false>), ElVStage<BYE>::smem_bytes());
-  SMEM_ATTR((el_v_kernel<BYE, true>), ElVStage<BYE>::smem_bytes());
-  SMEM_ATTR((el_s_kernel<BYE, false>), ElSStage<BYE>::smem_bytes());
-  SMEM_ATTR((el_s_kernel<BYE, true>), ElSStage<BYE>::smem_bytes());
+  SMEM_ATTR((el_v_kernel<BYE, false, true>), ElVStage<BYE>::smem_bytes());
+  SMEM_ATTR((el_v_kernel<BYE, true, true>), ElVStage<BYE>::smem_bytes());
+  SMEM_ATTR((el_s_kernel<BYE, false, true>), ElSStage<BYE>::smem_bytes());
+  SMEM_ATTR((el_s_kernel<BYE, true, true>), ElSStage<BYE>::smem_bytes());
+  SMEM_ATTR((el_v_kernel<BYE, false, false>), ElVStage<BYE>::smem_bytes());
+  SMEM_ATTR((el_v_kernel<BYE, true, false>), ElVStage<BYE>::smem_bytes());
+  SMEM_ATTR((el_s_kernel<BYE, false, false>), ElSStage<BYE>::smem_bytes());
+  SMEM_ATTR((el_s_kernel<BYE, true, false>), ElSStage<BYE>::smem_bytes());
 #undef SMEM_ATTR
   done = true;
   return SEIS_OK;
+}
+
+// Elastic instantiation choice (elastic kernels): without C-PML layers (W = 0)
+// every block runs the instantiation without the memory-variable code (fewer instructions and
+// registers, no spills: el_s 0.717 -> 0.672 ms at 384^3).  With layers one launch of the full
+// kernel: splitting by region (blocks free of layer points run the lean instantiation, the
+// others the full one; disjoint points, same arithmetic, bitwise unchanged) measured slower
+// (el_v 0.678 -> 0.701 ms at C3, profiles/r02_el_region.log) and is kept as SEIS_EL_REGION=1.
+template <class Go>
+void el_regions(int& region, int W, Go&& go) {
+  const char* e = getenv("SEIS_EL_REGION");  // (read per launch: tests flip it between models)
+  const bool split = e && e[0] == '1';
+  region = 0;
+  if (W <= 0) {
+    go(std::false_type{});
+  } else if (!split) {
+    go(std::true_type{});
+  } else {
+    region = 1;
+    go(std::false_type{});
+    region = 2;
+    go(std::true_type{});
+    ++g_launches;  // (the caller's CKL counts one)
+  }
 }
 
 // Choose the z-chunk: at most `zt` planes per chunk (short chunks keep the
@@ -950,7 +978,7 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, ac_v_kernel<BYV, false>, NTX * BYV,
                                                     AcVStage<BYV>::smem_bytes());
     else
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false>, NTX2 * (BYE + EL_WS),
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, el_s_kernel<BYE, false, true>, NTX2 * (BYE + EL_WS),
                                                     ElSStage<BYE>::smem_bytes());
     const int zex = (ns > 1 || M->nranks > 1) ? 4 : 0;
     if (kind == SEIS_ELASTIC) choose_chunks(S, occ, dev_sms, TXE, BYE, 16, zex);
@@ -1635,6 +1663,7 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
           a.region = 2;
           if (gh) go(std::true_type{}, std::true_type{});
           else go(std::true_type{}, std::false_type{});
+          ++g_launches;  // two launches (CKL counts one)
         } else if (gh) go(std::false_type{}, std::true_type{});
         else go(std::false_type{}, std::false_type{});
       }
@@ -1856,8 +1885,12 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     const dim3 gr = grid_of(S, TXE, BYE, nch);
     {
       PROF(3, ks);
-      if (a.img) el_v_kernel<BYE, true><<<gr, dim3(NTX2, BYE + EL_WS), ElVStage<BYE>::smem_bytes(), ks>>>(a);
-      else el_v_kernel<BYE, false><<<gr, dim3(NTX2, BYE + EL_WS), ElVStage<BYE>::smem_bytes(), ks>>>(a);
+      auto go = [&](auto cp) {
+        constexpr bool CP = decltype(cp)::value;
+        if (a.img) el_v_kernel<BYE, true, CP><<<gr, dim3(NTX2, BYE + EL_WS), ElVStage<BYE>::smem_bytes(), ks>>>(a);
+        else el_v_kernel<BYE, false, CP><<<gr, dim3(NTX2, BYE + EL_WS), ElVStage<BYE>::smem_bytes(), ks>>>(a);
+      };
+      el_regions(a.region, a.W, go);
     }
     CKL();
     return SEIS_OK;
@@ -1896,8 +1929,12 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
     const dim3 gr = grid_of(S, TXE, BYE, nch);
     {
       PROF(4, ks);
-      if (a.snap) el_s_kernel<BYE, true><<<gr, dim3(NTX2, BYE + EL_WS), ElSStage<BYE>::smem_bytes(), ks>>>(a);
-      else el_s_kernel<BYE, false><<<gr, dim3(NTX2, BYE + EL_WS), ElSStage<BYE>::smem_bytes(), ks>>>(a);
+      auto go = [&](auto cp) {
+        constexpr bool CP = decltype(cp)::value;
+        if (a.snap) el_s_kernel<BYE, true, CP><<<gr, dim3(NTX2, BYE + EL_WS), ElSStage<BYE>::smem_bytes(), ks>>>(a);
+        else el_s_kernel<BYE, false, CP><<<gr, dim3(NTX2, BYE + EL_WS), ElSStage<BYE>::smem_bytes(), ks>>>(a);
+      };
+      el_regions(a.region, a.W, go);
     }
     CKL();
     return SEIS_OK;
