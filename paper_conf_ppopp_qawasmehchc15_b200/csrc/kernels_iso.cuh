@@ -391,7 +391,8 @@ struct IsoPArgs {
   Dims d;
   int nt, cur0;
   long long src_o;                 // padded source index (-1: none)
-  const float* __restrict__ amp;   // device [nt]: src_scale * s[n] (the host float product)
+  const float* __restrict__ w;     // device wavelet [nt]; the amplitude is fmul_rn(src_scale, w[n])
+  float src_scale;
   float* __restrict__ seis;        // [nt][nrec_tot]
   const long long* __restrict__ rec_off;
   const int* __restrict__ rec_id;
@@ -460,12 +461,278 @@ __global__ void __launch_bounds__(128) iso_persist_kernel(const __grid_constant_
       if (rel >= 0 && rel < 4) {
 #pragma unroll
         for (int e = 0; e < 4; ++e)
-          if (rel == e) out.v[e] += a.amp[n];
+          if (rel == e) out.v[e] += __fmul_rn(a.src_scale, __ldg(a.w + n));
       }
       st4_masked(up + o, out, x0, d.nx, true);
     }
     grid.sync();
     cur = 1 - cur;
+  }
+}
+
+
+// ------------------------------------------------------------------ resident small-grid ISO
+// iso_resident_kernel<TX>: the whole shot of a small ISO grid (nx <= 128) in one cooperative
+// launch, each CTA OWNING one TX x 8 x 4 brick (TX = 64 or 128 >= nx: the whole x extent; the
+// x halo is the zero ghost) for all nt steps.  u^{n-1}, m and eta of its points stay in
+// registers, u^n of the brick + its 4-point halo (TX+8 x 16 x 12) in shared memory.
+// Halo exchange without barriers or flags-then-data round trips (the low-latency protocol of
+// NCCL's LL transport): every step the CTA writes its u^{n+1} into a per-brick exchange buffer
+// as 8-byte (value, tag) pairs, tag = base + n + 1, with 16-byte relaxed stores; a neighbour
+// polls the pairs it needs (y: 4 rows, z: the whole 4-plane brick) with relaxed 16-byte loads
+// until both tags match -- an 8-byte pair is single-copy atomic, so a matching tag proves its
+// value.  Two buffers per brick (step parity): a brick rewrites one only after consuming its
+// neighbours' next step, which they wrote after consuming this one.  The 25-point star reads
+// no corner values.  The field arrays receive the last two levels only (the final state).
+// Per point it evaluates the z-march kernel's expressions in the same order (iso_lap,
+// iso_update with eta = (eta_x + eta_y) + eta_z, then the source add fmul_rn(scale, w[n])),
+// so it is bitwise equal to it (tests/test_persist_gpu.py).  Receiver values of level n
+// (seis[n - 1]) are read from the tile centre at the top of step n and after the last step.
+#ifndef SEIS_IR_NOWAIT
+#define SEIS_IR_NOWAIT 0  // (perf-only builds: do not wait for the tags -- wrong results)
+#endif
+constexpr int IR_TY = 8, IR_TZ = 4, IR_H = IR_TY + 8, IR_D = IR_TZ + 8;
+constexpr int IR_RECMAX = 1024;  // receivers of the shot (host-checked), hence per brick
+template <int TX>
+struct IrShape {
+  static constexpr int W = TX + 8, TILE = W * IR_H * IR_D, OWN = TX * IR_TY * IR_TZ;
+  static constexpr int GPT = TX <= 64 ? 1 : 2, THREADS = OWN / 4 / GPT;  // float4 groups per thread
+  static constexpr int HALO = 3 * OWN / 2;                 // 16-byte (2-point) halo slots: z 2 x OWN/2, y 2 x OWN/4
+  static constexpr int HPT = HALO / THREADS;               // per thread (12)
+  static constexpr size_t smem() { return (size_t)(TILE + 2 * IR_RECMAX) * 4 + 128; }
+  static_assert(HPT * THREADS == HALO && (OWN / 2) % THREADS == 0 && (OWN / 4) % THREADS == 0, "slots");
+};
+__device__ __forceinline__ void st_relaxed_v4(uint4* p, uint4 v) {
+  asm volatile("st.relaxed.gpu.global.v4.u32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z),
+               "r"(v.w)
+               : "memory");
+}
+__device__ __forceinline__ uint4 ld_relaxed_v4(const uint4* p) {
+  uint4 v;
+  asm volatile("ld.relaxed.gpu.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "l"(p)
+               : "memory");
+  return v;
+}
+
+struct IsoRArgs {
+  float* u0;
+  float* u1;
+  const float* __restrict__ m;
+  const float* __restrict__ edx;   // eta dt per axis (nullptr: no layer)
+  const float* __restrict__ edy;
+  const float* __restrict__ edz;
+  Dims d;
+  int nt, cur0;                    // (the shot starts from the zero state: u^0 = u^{-1} = 0)
+  long long src_o;                 // padded source index (-1: none)
+  const float* __restrict__ w;     // device wavelet [nt]; the amplitude is fmul_rn(src_scale, w[n])
+  float src_scale;
+  float* __restrict__ seis;        // [nt][nrec_tot]
+  const long long* __restrict__ rec_off;
+  const int* __restrict__ rec_id;
+  int nrec, nrec_tot;
+  uint4* xb;                       // [bricks][2][OWN / 2] exchange pairs (value, tag) x 2
+  unsigned base;                   // tags of this shot: base + 1 .. base + nt (monotonic over shots)
+  int nby, nbz;
+  unsigned long long* trace;       // (SEIS_AS_TRACE builds) [brick][step][4] clock64 of thread 0
+};
+
+template <int TX>
+__global__ void __launch_bounds__(IrShape<TX>::THREADS, 1)
+    iso_resident_kernel(const __grid_constant__ IsoRArgs a) {
+  using S = IrShape<TX>;
+  constexpr int W = S::W, PL = W * IR_H, GPT = S::GPT, NT = S::THREADS, OWN = S::OWN;
+  extern __shared__ __align__(128) float sm_raw[];
+  float* tile = align128(sm_raw);
+  int2* rl = reinterpret_cast<int2*>(tile + S::TILE);  // (receiver, tile index)
+  __shared__ int nloc;
+  const Dims& d = a.d;
+  const int tid = threadIdx.x, b = blockIdx.x;
+  const int by = b % a.nby, bz = b / a.nby;
+  const int j0 = by * IR_TY, k0 = bz * IR_TZ;
+  if (tid == 0) nloc = 0;
+  for (int t = tid; t < S::TILE / 4; t += NT)  // u^0 = 0, and the zero x ghost
+    reinterpret_cast<float4*>(tile)[t] = make_float4(0.f, 0.f, 0.f, 0.f);
+  __syncthreads();
+  for (int r = tid; r < a.nrec; r += NT) {  // this brick's receivers
+    const long long off = a.rec_off[r];
+    const int k = (int)(off / d.PS) - GZ;
+    const long long rem = off % d.PS;
+    const int j = (int)(rem / d.PX) - G, i = (int)(rem % d.PX) - G;
+    if (j >= j0 && j < j0 + IR_TY && k >= k0 && k < k0 + IR_TZ) {
+      const int e = atomicAdd(&nloc, 1);
+      if (e < IR_RECMAX) rl[e] = make_int2(r, ((k - k0 + 4) * IR_H + (j - j0 + 4)) * W + i + 4);
+    }
+  }
+  // halo slot t (16 bytes = 2 points): source pair in the exchange buffers (both parities
+  // apart), tile destination; false: no neighbour on that side (the tile keeps the zero ghost)
+  auto slot = [&](int t, int& src, int& dst) -> bool {
+    int nb, e, rz, ry, x, row;
+    if (t < OWN / 2) {  // z-: the neighbour's whole brick -> tile planes 0..3
+      nb = bz > 0 ? b - a.nby : -1;
+      e = 2 * t;
+      rz = e / (IR_TY * TX), ry = (e / TX) % IR_TY, x = e % TX;
+      src = e / 2;
+      row = rz * IR_H + ry + 4;
+    } else if (t < OWN) {  // z+: -> tile planes 8..11
+      nb = bz + 1 < a.nbz ? b + a.nby : -1;
+      e = 2 * (t - OWN / 2);
+      rz = e / (IR_TY * TX), ry = (e / TX) % IR_TY, x = e % TX;
+      src = e / 2;
+      row = (rz + 4 + IR_TZ) * IR_H + ry + 4;
+    } else {  // y- (its rows 4..7 -> tile rows 0..3) / y+ (its rows 0..3 -> tile rows 12..15)
+      const bool lo = t < OWN + OWN / 4;
+      nb = lo ? (by > 0 ? b - 1 : -1) : (by + 1 < a.nby ? b + 1 : -1);
+      e = 2 * (t - (lo ? OWN : OWN + OWN / 4));
+      rz = e / (4 * TX), ry = (e / TX) % 4, x = e % TX;
+      src = ((rz * IR_TY + (lo ? 4 + ry : ry)) * TX + x) / 2;
+      row = (rz + 4) * IR_H + (lo ? ry : 4 + IR_TY + ry);
+    }
+    dst = row * W + 4 + x;
+    src += nb * 2 * (OWN / 2);
+    return nb >= 0;
+  };
+  long long o[GPT];
+  int cix[GPT], x0s[GPT];
+  bool own[GPT];
+  F4 upv[GPT], mv[GPT], eta[GPT];
+#pragma unroll
+  for (int q = 0; q < GPT; ++q) {
+    const int g = tid + q * NT;
+    const int x4 = g % (TX / 4), ry = (g / (TX / 4)) % IR_TY, rz = g / (TX / 4 * IR_TY);
+    const int x0 = 4 * x4, j = j0 + ry, k = k0 + rz;
+    x0s[q] = x0;
+    own[q] = x0 < d.nx && j < d.ny && k < d.nzl;
+    o[q] = d.at(x0, j, k);
+    cix[q] = ((rz + 4) * IR_H + (ry + 4)) * W + 4 + x0;
+    upv[q] = F4{{0.f, 0.f, 0.f, 0.f}};
+    mv[q] = own[q] ? ldg4(a.m + o[q]) : F4{{0.f, 0.f, 0.f, 0.f}};
+    eta[q] = F4{{0.f, 0.f, 0.f, 0.f}};
+    if (a.edx && own[q]) {
+      const F4 ex = ldg4(a.edx + x0);
+      const float ey = a.edy[j], ez = a.edz[k + d.z0];
+#pragma unroll
+      for (int e = 0; e < 4; ++e) eta[q].v[e] = (ex.v[e] + ey) + ez;
+    }
+  }
+  __syncthreads();  // (nloc)
+  const int nl = min(nloc, IR_RECMAX);
+  int cur = a.cur0;
+  for (int n = 0; n < a.nt; ++n) {
+    if (n > 0)  // receivers of level n (gather_kernel's rule: seis[n - 1])
+      for (int e = tid; e < nl; e += NT) {
+        const int2 rr = rl[e];
+        a.seis[(long long)(n - 1) * a.nrec_tot + a.rec_id[rr.x]] = tile[rr.y];
+      }
+#if SEIS_AS_TRACE
+    unsigned long long* tr = a.trace ? a.trace + ((size_t)b * a.nt + n) * 4 : nullptr;
+    if (tr && tid == 0) tr[0] = clock64();
+#endif
+    const unsigned tag = a.base + (unsigned)n + 1u;
+    const int par = (n + 1) & 1;
+    uint4* xo = a.xb + ((size_t)b * 2 + par) * (OWN / 2);
+    float* __restrict__ up = cur ? a.u0 : a.u1;  // u^{n-1} -> u^{n+1}
+    F4 out[GPT];
+#pragma unroll
+    for (int q = 0; q < GPT; ++q) {
+      const float* c = tile + cix[q];
+      float xv[12];
+      {
+        const F4 a0 = lds4(c - 4), a1 = lds4(c), a2 = lds4(c + 4);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          xv[e] = a0.v[e];
+          xv[4 + e] = a1.v[e];
+          xv[8 + e] = a2.v[e];
+        }
+      }
+      F4 ys[4], zs4[4];
+#pragma unroll
+      for (int m = 1; m <= 4; ++m) {
+        const F4 yp = lds4(c + m * W), ym = lds4(c - m * W);
+        const F4 zm = lds4(c - m * PL), zp = lds4(c + m * PL);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          ys[m - 1].v[e] = yp.v[e] + ym.v[e];
+          zs4[m - 1].v[e] = zm.v[e] + zp.v[e];
+        }
+      }
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        float xs[4], yss[4], zs[4];
+#pragma unroll
+        for (int m = 0; m < 4; ++m) {
+          xs[m] = xv[3 - m + e] + xv[5 + m + e];
+          yss[m] = ys[m].v[e];
+          zs[m] = zs4[m].v[e];
+        }
+        const float lap = iso_lap(xv[4 + e], xs, yss, zs);
+        out[q].v[e] = iso_update(xv[4 + e], upv[q].v[e], mv[q].v[e], lap, eta[q].v[e]);
+      }
+      if (own[q]) {
+        const long long rel = a.src_o - o[q];
+        if (rel >= 0 && rel < 4) {
+#pragma unroll
+          for (int e = 0; e < 4; ++e)
+            if (rel == e) out[q].v[e] += __fmul_rn(a.src_scale, __ldg(a.w + n));
+        }
+        if (n + 2 >= a.nt) st4_masked(up + o[q], out[q], x0s[q], d.nx, true);  // the final state
+      }
+      // outside the domain: the zero ghost, for the tile and the neighbours
+#pragma unroll
+      for (int e = 0; e < 4; ++e)
+        if (!own[q] || x0s[q] + e >= d.nx) out[q].v[e] = 0.f;
+      const int g = tid + q * NT;
+      st_relaxed_v4(xo + 2 * g, make_uint4(__float_as_uint(out[q].v[0]), tag, __float_as_uint(out[q].v[1]), tag));
+      st_relaxed_v4(xo + 2 * g + 1, make_uint4(__float_as_uint(out[q].v[2]), tag, __float_as_uint(out[q].v[3]), tag));
+#pragma unroll
+      for (int e = 0; e < 4; ++e) upv[q].v[e] = xv[4 + e];  // u^n: the next step's u^{n-1}
+    }
+#if SEIS_AS_TRACE
+    if (tr && tid == 0) tr[1] = clock64();
+#endif
+    __syncthreads();  // #1: the tile is consumed
+#pragma unroll
+    for (int q = 0; q < GPT; ++q)  // the brick's own u^{n+1} into the tile centre
+      *reinterpret_cast<float4*>(tile + cix[q]) = make_float4(out[q].v[0], out[q].v[1], out[q].v[2], out[q].v[3]);
+    {  // the neighbours' u^{n+1} halo pairs, in batches of HB 16-byte polls in flight
+      const uint4* xi = a.xb + (size_t)par * (OWN / 2);
+      constexpr int HB = S::HPT <= 6 ? S::HPT : S::HPT / 2;
+#pragma unroll
+      for (int h = 0; h < S::HPT; h += HB) {
+        uint4 v[HB];
+#pragma unroll
+        for (int i = 0; i < HB; ++i) {
+          int src, dst;
+          if (slot(tid + (h + i) * NT, src, dst)) v[i] = ld_relaxed_v4(xi + src);
+        }
+#pragma unroll
+        for (int i = 0; i < HB; ++i) {
+          int src, dst;
+          if (slot(tid + (h + i) * NT, src, dst)) {
+            long long spins = 0;
+            while (!SEIS_IR_NOWAIT && (v[i].y != tag || v[i].w != tag)) {
+              if (++spins > (1ll << 24)) __trap();  // (a lost neighbour: fail, do not hang)
+              v[i] = ld_relaxed_v4(xi + src);
+            }
+            *reinterpret_cast<float2*>(tile + dst) = make_float2(__uint_as_float(v[i].x), __uint_as_float(v[i].z));
+          }
+        }
+      }
+    }
+#if SEIS_AS_TRACE
+    if (tr && tid == 0) tr[2] = clock64();
+#endif
+    __syncthreads();  // #2: centre and halo of u^{n+1} are in the tile
+#if SEIS_AS_TRACE
+    if (tr && tid == 0) tr[3] = clock64();
+#endif
+    cur = 1 - cur;
+  }
+  for (int e = tid; e < nl; e += NT) {  // level nt
+    const int2 rr = rl[e];
+    a.seis[(long long)(a.nt - 1) * a.nrec_tot + a.rec_id[rr.x]] = tile[rr.y];
   }
 }
 

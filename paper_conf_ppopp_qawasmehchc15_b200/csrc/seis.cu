@@ -208,8 +208,9 @@ struct seis_model {
   // staging buffers
   float* stage = nullptr;
   size_t stage_elems = 0;
-  float* pamp = nullptr;    // persistent small-grid ISO path: per-step source amplitudes
-  int pamp_n = 0;
+  void* rxb = nullptr;      // resident small-grid ISO path: per-brick halo exchange buffers
+  size_t rxb_n = 0;         // (bytes)
+  unsigned rxb_base = 0;    // tag base (monotonic over shots: each shot uses base + 1 .. base + nt)
   const float* hwav = nullptr;  // host wavelet of the current call
   float* dwav = nullptr;        // its device copy (uploaded by every call, read by the source add)
   size_t dwav_n = 0;
@@ -281,7 +282,7 @@ uint64_t fnv1a(const void* p, size_t n, uint64_t h = 1469598103934665603ULL) {
 // cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda link).
 PFN_cuTensorMapEncodeTiled_v12000 g_encode = nullptr;
 
-seis_status make_map(CUtensorMap* m, float* base, const Dims& d, int bw, int bh) {
+seis_status make_map(CUtensorMap* m, float* base, const Dims& d, int bw, int bh, int bd = 1) {
   if (!g_encode) {
     cudaDriverEntryPointQueryResult q;
     void* fn = nullptr;
@@ -291,7 +292,7 @@ seis_status make_map(CUtensorMap* m, float* base, const Dims& d, int bw, int bh)
   }
   cuuint64_t dims[3] = {(cuuint64_t)d.PX, (cuuint64_t)d.PY, (cuuint64_t)(d.nzl + 2 * GZ)};
   cuuint64_t str[2] = {(cuuint64_t)d.PX * 4, (cuuint64_t)d.PS * 4};
-  cuuint32_t box[3] = {(cuuint32_t)bw, (cuuint32_t)bh, 1};
+  cuuint32_t box[3] = {(cuuint32_t)bw, (cuuint32_t)bh, (cuuint32_t)bd};
   cuuint32_t es[3] = {1, 1, 1};
   CUresult r = g_encode(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, base, dims, str, box, es,
                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
@@ -1974,7 +1975,8 @@ seis_status ensure_stage(seis_model* M, size_t elems) { return regrow(M, &M->sta
 
 }  // namespace
 
-// Small L2-resident ISO grids: the whole shot as one cooperative launch (iso_persist_kernel).
+// Small L2-resident ISO grids: the whole shot as one cooperative launch -- resident bricks
+// (iso_resident_kernel) where they fit, else the grid-stride kernel (iso_persist_kernel).
 bool persist_ok(const seis_model* M) {
   if (M->kind != SEIS_ISO || M->slabs.size() != 1 || M->comm || prof::on) return false;
   const Slab& S = M->slabs[0];
@@ -1988,16 +1990,6 @@ seis_status forward_persist(seis_model* M, const seis_shot* sh, float* sd, size_
   Slab& S = M->slabs[0];
   TRY(zero_state(M, st));
   if (ns) CK(cudaMemsetAsync(sd, 0, ns * sizeof(float), st));
-  if (M->pamp_n < sh->nt) {
-    void* p = nullptr;
-    TRY(alloc_track(M, &p, (size_t)sh->nt * sizeof(float)));
-    M->pamp = (float*)p;
-    M->pamp_n = sh->nt;
-  }
-  std::vector<float> amp(sh->nt, 0.f);
-  if (S.src_o >= 0)
-    for (int n = 0; n < sh->nt; ++n) amp[n] = S.src_scale * M->hwav[n];  // as step(): float product
-  CK(cudaMemcpyAsync(M->pamp, amp.data(), amp.size() * sizeof(float), cudaMemcpyHostToDevice, st));
   IsoPArgs a;
   a.u0 = S.fld[0];
   a.u1 = S.fld[1];
@@ -2009,16 +2001,97 @@ seis_status forward_persist(seis_model* M, const seis_shot* sh, float* sd, size_
   a.nt = sh->nt;
   a.cur0 = S.cur;
   a.src_o = S.src_o;
-  a.amp = M->pamp;
+  a.w = M->dwav;
+  a.src_scale = S.src_scale;
   a.seis = sd;
   a.rec_off = S.d_rec_off;
   a.rec_id = S.d_rec_id;
   a.nrec = S.nrec_own;
   a.nrec_tot = sh->nrec;
-  static int occ = 0, nsm = 0;
+  static int occ = 0, nsm = 0, rocc64 = 0, rocc128 = 0;
   if (!occ) {
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, iso_persist_kernel, 128, 0));
     CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, M->device));
+    CK(cudaFuncSetAttribute(iso_resident_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)IrShape<64>::smem()));
+    CK(cudaFuncSetAttribute(iso_resident_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)IrShape<128>::smem()));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&rocc64, iso_resident_kernel<64>, IrShape<64>::THREADS,
+                                                     IrShape<64>::smem()));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&rocc128, iso_resident_kernel<128>, IrShape<128>::THREADS,
+                                                     IrShape<128>::smem()));
+  }
+  // Resident bricks (iso_resident_kernel) when nx <= 128, every brick gets its own co-resident
+  // CTA and the receivers fit the per-brick list; else the grid-stride kernel with grid
+  // barriers.  SEIS_ISO_RESIDENT=0 forces the latter (comparison), =2 requires the former.
+  const int tx = S.d.nx <= 64 ? 64 : 128;
+  const int nby = (S.d.ny + IR_TY - 1) / IR_TY, nbz = (S.d.nzl + IR_TZ - 1) / IR_TZ;
+  const long long bricks = (long long)nby * nbz;
+  const int rocc = tx == 64 ? rocc64 : rocc128;
+  const char* er = getenv("SEIS_ISO_RESIDENT");
+  const bool fits = S.d.nx <= 128 && bricks <= (long long)rocc * nsm && sh->nrec <= IR_RECMAX;
+  if (er && er[0] == '2' && !fits)
+    return fail(SEIS_EINVAL, "resident ISO kernel: nx %d > 128, %lld bricks > %d co-resident CTAs, or %d receivers > %d",
+                S.d.nx, bricks, rocc * nsm, sh->nrec, IR_RECMAX);
+  if (!(er && er[0] == '0') && fits) {
+    const size_t xbytes = (size_t)bricks * 2 * (tx * IR_TY * IR_TZ / 2) * 16;
+    if (M->rxb_n != xbytes) {  // (a model's grid is fixed: allocated and zeroed once)
+      void* p = nullptr;
+      TRY(alloc_track(M, &p, xbytes));
+      M->rxb = p;
+      M->rxb_n = xbytes;
+      M->rxb_base = 0;
+      CK(cudaMemsetAsync(M->rxb, 0, xbytes, st));
+    }
+    IsoRArgs r;
+    r.u0 = S.fld[0];
+    r.u1 = S.fld[1];
+    r.m = S.m;
+    r.edx = M->edx;
+    r.edy = M->edy;
+    r.edz = M->edz;
+    r.d = S.d;
+    r.nt = sh->nt;
+    r.cur0 = S.cur;
+    r.src_o = S.src_o;
+    r.w = M->dwav;
+    r.src_scale = S.src_scale;
+    r.seis = sd;
+    r.rec_off = S.d_rec_off;
+    r.rec_id = S.d_rec_id;
+    r.nrec = S.nrec_own;
+    r.nrec_tot = sh->nrec;
+    r.xb = (uint4*)M->rxb;
+    r.base = M->rxb_base;
+    r.nby = nby;
+    r.nbz = nbz;
+    r.trace = nullptr;
+#if SEIS_AS_TRACE
+    {
+      static unsigned long long* tr = nullptr;
+      static size_t trn = 0;
+      const size_t need = (size_t)bricks * sh->nt * 4;
+      if (trn < need) {
+        if (tr) cudaFree(tr);
+        CK(cudaMallocManaged(&tr, need * sizeof(unsigned long long)));
+        trn = need;
+      }
+      r.trace = tr;
+      g_trace = tr;
+      g_trace_n = need;
+    }
+#endif
+    void* rargs[] = {&r};
+    if (tx == 64)
+      CK(cudaLaunchCooperativeKernel((void*)iso_resident_kernel<64>, dim3((unsigned)bricks),
+                                     dim3(IrShape<64>::THREADS), rargs, IrShape<64>::smem(), st));
+    else
+      CK(cudaLaunchCooperativeKernel((void*)iso_resident_kernel<128>, dim3((unsigned)bricks),
+                                     dim3(IrShape<128>::THREADS), rargs, IrShape<128>::smem(), st));
+    ++g_launches;
+    M->rxb_base += (unsigned)sh->nt;
+    S.cur = (S.cur + sh->nt) & 1;
+    return SEIS_OK;
   }
   const long long groups = (long long)((S.d.nx + 3) / 4) * S.d.ny * S.d.nzl;
   const char* eb = getenv("SEIS_PERSIST_BPSM");  // blocks per SM (A/B; default: all that fit)

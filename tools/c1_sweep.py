@@ -1,4 +1,4 @@
-"""C1 (ISO 64^3, 200 steps; L2-resident, launch-bound): z-march path vs the persistent kernel.
+"""C1 (ISO 64^3, 200 steps; L2-resident, launch-bound): z-march path vs the persistent kernels.
 
     python tools/c1_sweep.py        # on a B200: one line per SEIS_ZCHUNK_MIN value
 """
@@ -27,8 +27,11 @@ ms = e0.elapsed_time(e1) / 20
 print(json.dumps({"ms_per_shot": round(ms, 4), "gpts_s": round(wl.npts * wl.nt / (ms * 1e-3) / 1e9, 2)}))
 '''
 
-for zmin, bpsm, pers in ((2, 0, 0), (2, 1, 1), (2, 2, 1), (2, 3, 1), (2, 0, 1)):
-    env = dict(os.environ, SEIS_ZCHUNK_MIN=str(zmin), SEIS_NO_PERSIST="0" if pers else "1")
+# pers: 0 z-march kernels (graph), 1 grid-stride persistent kernel (grid barriers),
+# 2 resident bricks (neighbour counters, the default)
+for zmin, bpsm, pers in ((2, 0, 0), (2, 0, 1), (2, 0, 2)):
+    env = dict(os.environ, SEIS_ZCHUNK_MIN=str(zmin), SEIS_NO_PERSIST="0" if pers else "1",
+               SEIS_ISO_RESIDENT="1" if pers == 2 else "0")
     if bpsm:
         env["SEIS_PERSIST_BPSM"] = str(bpsm)
     r = subprocess.run([sys.executable, "-c", ONE, ROOT], env=env, capture_output=True, text=True, timeout=600)

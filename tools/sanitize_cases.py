@@ -5,8 +5,8 @@
     compute-sanitizer --tool racecheck python tools/sanitize_cases.py --quick
     compute-sanitizer --tool synccheck python tools/sanitize_cases.py
 
-Variants: ISO z-march (damped layer, split-field PML, 1 / 3 slabs, persistent small-grid
-kernel), acoustic split V / P (1 and 3 slabs: direct ghost stores, the copy exchange, the
+Variants: ISO z-march (damped layer, split-field PML, 1 / 3 slabs, the resident-brick and
+grid-stride persistent small-grid kernels), acoustic split V / P (1 and 3 slabs: direct ghost stores, the copy exchange, the
 serial order), the fused acoustic step (cooperative, counters), elastic V / S (free surface,
 C-PML), RTM of every kind (imaging + snapshot epilogues, fp32 and 24-bit snapshots,
 checkpointing), receiver injection / gather, host staging buffers.  Each case only checks
@@ -63,7 +63,8 @@ def main():
     s = (24, 20, 36) if a.quick else (40, 36, 70)
     # ISO
     case("iso", s, nb=4, env={"SEIS_NO_PERSIST": "1"})
-    case("iso", s, nb=4)  # persistent small-grid kernel
+    case("iso", s, nb=4)  # resident-brick small-grid kernel
+    case("iso", s, nb=4, env={"SEIS_ISO_RESIDENT": "0"})  # grid-stride small-grid kernel
     case("iso", s, nb=4, iso_pml=1)
     case("iso", s, nb=4, slabs=3, env={"SEIS_NO_PERSIST": "1"})
     # acoustic: split pair, decompositions, fused step
