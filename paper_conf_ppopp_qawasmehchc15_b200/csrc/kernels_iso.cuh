@@ -99,6 +99,12 @@ __device__ __forceinline__ int spml_idx(const Dims& d, int nb, int nxs, int nys,
 #ifndef SEIS_ISO_NS
 #define SEIS_ISO_NS 3
 #endif
+// O6b layer components by cp.async two planes ahead into per-thread shared slots, instead of
+// register loads issued one plane ahead (whose latency is the kernel's top stall): measured
+// and rejected, off -- 0.853 vs 0.739 ms at 512^3 (profiles/r02_iso_pml_variants.txt)
+#ifndef SEIS_SPML_PF
+#define SEIS_SPML_PF 0
+#endif
 constexpr int ISO_NS = SEIS_ISO_NS;
 
 template <int BY>
@@ -106,6 +112,9 @@ struct IsoStage {
   static constexpr int W = TXV + 8;
   static constexpr int U = 0, UP = (BY + 8) * W, M = UP + TXV * BY, UQ = M + TXV * BY, SIZE = UQ + TXV * BY;
   static constexpr size_t smem_bytes() { return (size_t)ISO_NS * SIZE * 4 + 128; }
+  // (SPML, SEIS_SPML_PF) + per-thread slots: 3 planes x 6 component arrays x 4 points
+  static constexpr int CSLOT = 3 * 6 * NTX * BY * 4;
+  static constexpr size_t smem_bytes_spml() { return smem_bytes() + (SEIS_SPML_PF ? (size_t)CSLOT * 4 : 0); }
 };
 
 // Launch bounds: an explicit minimum of 1 block lets ptxas give the plain kernel 96 registers
@@ -190,27 +199,71 @@ __global__ void __launch_bounds__(NTX * BY, SPML ? SEIS_SPML_MINB : 1) iso_step_
   // of such tiles take the undamped update without per-point branches (same arithmetic).
   const bool dxy = __syncthreads_or(exy.v[0] != 0.f || exy.v[1] != 0.f || exy.v[2] != 0.f || exy.v[3] != 0.f);
 
+  // (SPML, SEIS_SPML_PF) this group's component indices at plane kk (-1: not a layer point)
+  auto sp_index = [&](int kk, float ezk, int* six) {
+#pragma unroll
+    for (int e = 0; e < 4; ++e)
+      six[e] = (own && x0 + e < d.nx && (exv.v[e] != 0.0f || eyv != 0.0f || ezk != 0.0f))
+                   ? spml_idx(d, a.nbl, a.nxs, a.nys, exv.v[e], eyv, x0 + e, j, kk)
+                   : -1;
+  };
+  float* const csl = sm + ISO_NS * L::SIZE + 4 * tid;  // [plane buffer][array][thread][4]
+  constexpr int CST = NTX * BY * 4;
+  // (the caller loads eta_z of plane kk one iteration earlier: no load latency at the issue)
+  auto sp_issue = [&](int kk, int buf, float ezk) {  // cur (level n) arrays 0..2, nxt (n-1) 3..5
+    if (dxy || ezk != 0.0f) {
+      int six[4];
+      sp_index(kk, ezk, six);
+      const bool v = six[0] >= 0 && (six[0] & 3) == 0 && (a.spn & 3) == 0 && six[1] == six[0] + 1 &&
+                     six[2] == six[0] + 2 && six[3] == six[0] + 3;
+#pragma unroll
+      for (int arr = 0; arr < 6; ++arr) {
+        const float* src = a.sp + (long long)(arr < 3 ? a.lvl : 1 - a.lvl) * 3 * a.spn + (arr % 3) * a.spn;
+        float* dst = csl + (buf * 6 + arr) * CST;
+        if (v) {
+          cp_async16(dst, src + six[0]);
+        } else {
+#pragma unroll
+          for (int e = 0; e < 4; ++e)
+            if (six[e] >= 0) cp_async4(dst + e, src + six[e], true);
+        }
+      }
+    }
+    cp_async_commit();  // (one group per plane, empty or not: uniform group counting)
+  };
+  auto ez_at = [&](int kk) { return (a.edx && kk < k1) ? __ldg(a.edz + kk + d.z0) : 0.0f; };
+  float ez_pf = 0.0f;  // eta_z dt of plane k + 2 (loaded at iteration it - 1)
+  if (SPML && SEIS_SPML_PF) {
+    sp_issue(k0, 0, ez_at(k0));
+    if (np > 1) sp_issue(k0 + 1, 1, ez_at(k0 + 1));
+    else cp_async_commit();
+    ez_pf = ez_at(k0 + 2);
+  }
+
   SEIS_UNROLL(SEIS_ZU_ISO)
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
     const int s = it % ISO_NS;
     const long long o = (long long)(k + GZ) * PS + oc;
     const float ez = a.edx ? a.edz[k + d.z0] : 0.0f;
+    if (SPML && SEIS_SPML_PF) {
+      if (it + 2 < np) sp_issue(k + 2, (it + 2) % 3, ez_pf);
+      else cp_async_commit();
+      ez_pf = ez_at(k + 3);
+    }
     // (SPML) the layer components of this group are loaded before the stage wait (latency
     // overlap, as the C-PML memory variables): w0 = level n, wm = level n-1
     int sidx[4] = {-1, -1, -1, -1};
     float w0[3][4], wm[3][4];
     bool spv = false;  // the group's 4 components are one aligned float4 in every array
     if (SPML && (dxy || ez != 0.0f)) {
-#pragma unroll
-      for (int e = 0; e < 4; ++e)
-        if (own && x0 + e < d.nx && (exv.v[e] != 0.0f || eyv != 0.0f || ez != 0.0f))
-          sidx[e] = spml_idx(d, a.nbl, a.nxs, a.nys, exv.v[e], eyv, x0 + e, j, k);
+      sp_index(k, ez, sidx);
       spv = sidx[0] >= 0 && (sidx[0] & 3) == 0 && (a.spn & 3) == 0 && sidx[1] == sidx[0] + 1 &&
             sidx[2] == sidx[0] + 2 && sidx[3] == sidx[0] + 3;
       const float* cur = a.sp + (long long)a.lvl * 3 * a.spn;
       const float* nxt = a.sp + (long long)(1 - a.lvl) * 3 * a.spn;
-      if (spv) {
+      if (SEIS_SPML_PF) {  // (read after the stage wait, below)
+      } else if (spv) {
 #pragma unroll
         for (int c = 0; c < 3; ++c) {
           const F4 p0 = ld4(cur + c * a.spn + sidx[0]), pm = ld4(nxt + c * a.spn + sidx[0]);
@@ -275,6 +328,19 @@ __global__ void __launch_bounds__(NTX * BY, SPML ? SEIS_SPML_MINB : 1) iso_step_
     } else if (SPML) {
       // O6b: layer points advance u^(x), u^(y), u^(z), each damped along its own axis with the
       // 1D part L_d of the Laplacian; u^{n+1} is their sum.  Other points: Eq 1.
+      if (SEIS_SPML_PF) {  // this plane's components, copied two planes ago
+        cp_async_wait<2>();
+        const float* cs = csl + (it % 3) * 6 * CST;
+#pragma unroll
+        for (int c = 0; c < 3; ++c) {
+          const F4 p0 = lds4(cs + c * CST), pm = lds4(cs + (3 + c) * CST);
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            w0[c][e] = p0.v[e];
+            wm[c][e] = pm.v[e];
+          }
+        }
+      }
 #pragma unroll
       for (int e = 0; e < 4; ++e) {
         const float u = xv[4 + e];
@@ -365,6 +431,7 @@ __global__ void __launch_bounds__(NTX * BY, SPML ? SEIS_SPML_MINB : 1) iso_step_
 #pragma unroll
     for (int t = 0; t < 8; ++t) q[t] = q[t + 1];
   }
+  if (SPML && SEIS_SPML_PF) cp_async_wait<0>();  // (no copy into this block's shared memory outlives it)
 }
 
 }  // namespace seis

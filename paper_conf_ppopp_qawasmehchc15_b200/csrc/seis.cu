@@ -378,15 +378,15 @@ seis_status set_smem_attrs() {
   SMEM_ATTR((iso_step_kernel<BYI, false, false>), IsoStage<BYI>::smem_bytes());
   SMEM_ATTR((iso_step_kernel<BYI, true, false>), IsoStage<BYI>::smem_bytes());
   SMEM_ATTR((iso_step_kernel<BYI, false, true>), IsoStage<BYI>::smem_bytes());
-  SMEM_ATTR((iso_step_kernel<BYI, false, false, true>), IsoStage<BYI>::smem_bytes());
-  SMEM_ATTR((iso_step_kernel<BYI, true, false, true>), IsoStage<BYI>::smem_bytes());
-  SMEM_ATTR((iso_step_kernel<BYI, false, true, true>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, false, false, true>), IsoStage<BYI>::smem_bytes_spml());
+  SMEM_ATTR((iso_step_kernel<BYI, true, false, true>), IsoStage<BYI>::smem_bytes_spml());
+  SMEM_ATTR((iso_step_kernel<BYI, false, true, true>), IsoStage<BYI>::smem_bytes_spml());
   SMEM_ATTR((iso_step_kernel<BYI, false, false, false, false>), IsoStage<BYI>::smem_bytes());
   SMEM_ATTR((iso_step_kernel<BYI, true, false, false, false>), IsoStage<BYI>::smem_bytes());
   SMEM_ATTR((iso_step_kernel<BYI, false, true, false, false>), IsoStage<BYI>::smem_bytes());
-  SMEM_ATTR((iso_step_kernel<BYI, false, false, true, false>), IsoStage<BYI>::smem_bytes());
-  SMEM_ATTR((iso_step_kernel<BYI, true, false, true, false>), IsoStage<BYI>::smem_bytes());
-  SMEM_ATTR((iso_step_kernel<BYI, false, true, true, false>), IsoStage<BYI>::smem_bytes());
+  SMEM_ATTR((iso_step_kernel<BYI, false, false, true, false>), IsoStage<BYI>::smem_bytes_spml());
+  SMEM_ATTR((iso_step_kernel<BYI, true, false, true, false>), IsoStage<BYI>::smem_bytes_spml());
+  SMEM_ATTR((iso_step_kernel<BYI, false, true, true, false>), IsoStage<BYI>::smem_bytes_spml());
   SMEM_ATTR((ac_v_kernel<BYV, false>), AcVStage<BYV>::smem_bytes());
   SMEM_ATTR((ac_v_kernel<BYV, true>), AcVStage<BYV>::smem_bytes());
   SMEM_ATTR((ac_p_kernel<BYP, false>), AcPStage<BYP>::smem_bytes());
@@ -1643,10 +1643,10 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
       const dim3 gr = grid_of(S, TXV, BYI, nch), blk(NTX, BYI);
       {
         PROF(0, ks);
-        const size_t sb = IsoStage<BYI>::smem_bytes();
         // template flags: O6b split-field PML; direct ghost stores of this slab (f4)
         auto go = [&](auto spml, auto gh) {
           constexpr bool SP = decltype(spml)::value, GH = decltype(gh)::value;
+          const size_t sb = SP ? IsoStage<BYI>::smem_bytes_spml() : IsoStage<BYI>::smem_bytes();
           if (a.snap) iso_step_kernel<BYI, true, false, SP, GH><<<gr, blk, sb, ks>>>(a);
           else if (a.img) iso_step_kernel<BYI, false, true, SP, GH><<<gr, blk, sb, ks>>>(a);
           else iso_step_kernel<BYI, false, false, SP, GH><<<gr, blk, sb, ks>>>(a);
