@@ -135,7 +135,8 @@ struct ElVArgs {
   CUtensorMap mq[3];  // z-queue feeds: sxz (k+3), syz (k+3), szz (k+4), box 64 x BY
   float* f[9];
   int W, zlo, fs;
-  int region;  // 0: every block; 1: only blocks free of C-PML points; 2: only the others
+  int region;  // 0: every block; 1: only blocks free of C-PML points; 2: only the others;
+               // 3: every block, the lean body where no C-PML point is (one launch)
   float dth;       // dt / h (face buoyancy dt b/h = dth * 2/(rho_i + rho_{i+1}), O8/O9)
   CpmlAxis cx, cy, cz;
   float* psi[9];   // psi 0..8
@@ -172,7 +173,7 @@ struct ElVStage {
 };
 
 template <int BY, bool IMG, bool CP>
-__global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (BY <= 8 ? 2 : 1)) el_v_kernel(const __grid_constant__ ElVArgs a) {
+__device__ __forceinline__ void el_v_body(const ElVArgs& a) {
   using L = ElVStage<BY>;
   constexpr int WX = L::WX;
   constexpr uint32_t TX_BYTES = L::BYTES;
@@ -198,7 +199,8 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
   const long long oc = (long long)(j + G) * d.PX + (x0 + G);
   // (region split) CP = false: the instantiation without the C-PML code, for blocks whose
   // tile and z-chunk hold no layer point (fewer instructions, no spills)
-  if (a.region && el_block_in_layers(d, a.W, a.zlo, i0, j0, BY, k0, k1) != (a.region == 2)) return;
+  if ((a.region == 1 || a.region == 2) && el_block_in_layers(d, a.W, a.zlo, i0, j0, BY, k0, k1) != (a.region == 2))
+    return;
   const int W = CP ? a.W : 0;
   const bool lx = W > 0 && (x0 < W || x0 + 1 >= d.nx - W);
   const bool ly = W > 0 && CpmlIdx::in(j, d.ny, W, true);
@@ -460,6 +462,21 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
   }
 }
 
+// (region = 3) one launch, the code path chosen per block: blocks whose tile and z-chunk hold
+// no C-PML point run the body without the memory-variable code (as the lean instantiation)
+template <int BY, bool IMG, bool CP>
+__global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (BY <= 8 ? 2 : 1)) el_v_kernel(const __grid_constant__ ElVArgs a) {
+  if (CP && a.region == 3) {
+    const int k0 = (a.ch0 + (int)blockIdx.z * a.chs) * a.zc;
+    const int k1 = min(k0 + a.zc, a.d.nzl);
+    if (!el_block_in_layers(a.d, a.W, a.zlo, blockIdx.x * TXE, blockIdx.y * BY, BY, k0, k1)) {
+      el_v_body<BY, IMG, false>(a);
+      return;
+    }
+  }
+  el_v_body<BY, IMG, CP>(a);
+}
+
 struct ElSArgs {
   CUtensorMap mvt[3];  // vx, vy, vz tiles, box 72 x (BY+8)
   CUtensorMap ms[6];   // sxx, syy, szz, sxy, sxz, syz, box 64 x BY
@@ -468,7 +485,8 @@ struct ElSArgs {
   CUtensorMap mq[3];   // z-queue feeds: vx (k+4), vy (k+4), vz (k+3), box 64 x BY
   float* f[9];
   int W, zlo, fs;
-  int region;  // 0: every block; 1: only blocks free of C-PML points; 2: only the others
+  int region;  // 0: every block; 1: only blocks free of C-PML points; 2: only the others;
+               // 3: every block, the lean body where no C-PML point is (one launch)
   CpmlAxis cx, cy, cz;
   float* psi[9];   // psi 9..17
   Dims d;
@@ -492,7 +510,7 @@ struct ElSStage {
 };
 
 template <int BY, bool SNAP, bool CP>
-__global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (BY <= 8 ? 2 : 1)) el_s_kernel(const __grid_constant__ ElSArgs a) {
+__device__ __forceinline__ void el_s_body(const ElSArgs& a) {
   using L = ElSStage<BY>;
   constexpr int WX = L::WX, TV = L::TV, RW = L::RW;
   constexpr uint32_t TX_BYTES = L::BYTES;
@@ -516,7 +534,8 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
   const long long oc = (long long)(j + G) * d.PX + (x0 + G);
   // (region split) CP = false: the instantiation without the C-PML code, for blocks whose
   // tile and z-chunk hold no layer point (fewer instructions, no spills)
-  if (a.region && el_block_in_layers(d, a.W, a.zlo, i0, j0, BY, k0, k1) != (a.region == 2)) return;
+  if ((a.region == 1 || a.region == 2) && el_block_in_layers(d, a.W, a.zlo, i0, j0, BY, k0, k1) != (a.region == 2))
+    return;
   const int W = CP ? a.W : 0;
   const bool lx = W > 0 && (x0 < W || x0 + 1 >= d.nx - W);
   const bool ly = W > 0 && CpmlIdx::in(j, d.ny, W, true);
@@ -803,6 +822,21 @@ __global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL
       qz[t] = qz[t + 1];
     }
   }
+}
+
+// (region = 3) one launch, the code path chosen per block: blocks whose tile and z-chunk hold
+// no C-PML point run the body without the memory-variable code (as the lean instantiation)
+template <int BY, bool SNAP, bool CP>
+__global__ void __launch_bounds__(NTX2 *(BY + EL_WS), SEIS_EL_MINB > 0 ? SEIS_EL_MINB : (BY <= 8 ? 2 : 1)) el_s_kernel(const __grid_constant__ ElSArgs a) {
+  if (CP && a.region == 3) {
+    const int k0 = (a.ch0 + (int)blockIdx.z * a.chs) * a.zc;
+    const int k1 = min(k0 + a.zc, a.d.nzl);
+    if (!el_block_in_layers(a.d, a.W, a.zlo, blockIdx.x * TXE, blockIdx.y * BY, BY, k0, k1)) {
+      el_s_body<BY, SNAP, false>(a);
+      return;
+    }
+  }
+  el_s_body<BY, SNAP, CP>(a);
 }
 
 

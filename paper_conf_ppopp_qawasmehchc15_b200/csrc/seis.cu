@@ -407,27 +407,30 @@ seis_status set_smem_attrs() {
   return SEIS_OK;
 }
 
-// Elastic instantiation choice (elastic kernels): without C-PML layers (W = 0)
-// every block runs the instantiation without the memory-variable code (fewer instructions and
-// registers, no spills: el_s 0.717 -> 0.672 ms at 384^3).  With layers one launch of the full
-// kernel: splitting by region (blocks free of layer points run the lean instantiation, the
-// others the full one; disjoint points, same arithmetic, bitwise unchanged) measured slower
-// (el_v 0.678 -> 0.701 ms at C3, profiles/r02_el_region.log) and is kept as SEIS_EL_REGION=1.
+// Elastic code-path choice (elastic kernels): without C-PML layers (W = 0) every
+// block runs the instantiation without the memory-variable code (fewer instructions and
+// registers, no spills: el_s 0.717 -> 0.672 ms at 384^3).  With layers one launch in which
+// each block picks its body (region 3): the lean one where its tile and z-chunk hold no layer
+// point, the full one elsewhere -- disjoint points, same arithmetic, bitwise unchanged.
+// SEIS_EL_REGION=0: the full body everywhere; =1: two launches split by region (measured
+// slower: el_v 0.678 -> 0.701 ms at C3, profiles/r02_el_region.log).
 template <class Go>
 void el_regions(int& region, int W, Go&& go) {
   const char* e = getenv("SEIS_EL_REGION");  // (read per launch: tests flip it between models)
-  const bool split = e && e[0] == '1';
   region = 0;
   if (W <= 0) {
     go(std::false_type{});
-  } else if (!split) {
+  } else if (e && e[0] == '0') {
     go(std::true_type{});
-  } else {
+  } else if (e && e[0] == '1') {
     region = 1;
     go(std::false_type{});
     region = 2;
     go(std::true_type{});
     ++g_launches;  // (the caller's CKL counts one)
+  } else {
+    region = 3;
+    go(std::true_type{});
   }
 }
 
