@@ -82,6 +82,17 @@ struct CpmlIdx {
   __device__ __forceinline__ static int slot(int i, int n, int W) { return i < W ? i : i - (n - 2 * W); }
 };
 
+// Conservative, block-uniform: may the block's tile (tw x by at i0, j0) and z-chunk [k0, k1)
+// hold a C-PML point (W = layer slab width per face, zlo: the top face has one)?  A block that
+// may runs the full body (correct everywhere); one that does not may run the lean body.
+__device__ __forceinline__ bool block_in_layers(const Dims& d, int W, int zlo, int i0, int tw, int j0, int by, int k0,
+                                                int k1) {
+  if (W <= 0) return false;
+  const bool inner = i0 >= W && i0 + tw <= d.nx - W && j0 >= W && j0 + by <= d.ny - W &&
+                     (!zlo || k0 + d.z0 >= W) && k1 + d.z0 <= d.nz - W;
+  return !inner;
+}
+
 }  // namespace seis
 
 // ----------------------------------------------------------------- TMA ring

@@ -149,15 +149,10 @@ struct ElVArgs {
   Ghost gh[3];                     // direct ghost stores of vx, vy, vz (f4)
 };
 
-// (region split) conservative, block-uniform: may this block's tile (TXE x BY at i0, j0) and
-// z-chunk [k0, k1) hold a C-PML point?  (A block that does runs the CP instantiation, which is
-// correct everywhere; one that does not may run either.)
+// (region split) may this block's tile (TXE x BY) and z-chunk hold a C-PML point
 __device__ __forceinline__ bool el_block_in_layers(const Dims& d, int W, int zlo, int i0, int j0, int by, int k0,
                                                    int k1) {
-  if (W <= 0) return false;
-  const bool inner = i0 >= W && i0 + TXE <= d.nx - W && j0 >= W && j0 + by <= d.ny - W &&
-                     (!zlo || k0 + d.z0 >= W) && k1 + d.z0 <= d.nz - W;
-  return !inner;
+  return block_in_layers(d, W, zlo, i0, TXE, j0, by, k0, k1);
 }
 
 template <int BY>
