@@ -228,6 +228,10 @@ struct seis_model {
   // overlapped ghost exchange: side stream + fork / join events
   cudaStream_t xs = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  // ISO split-field PML: the plain-kernel region runs on its own stream, concurrently with the
+  // split-field region (SEIS_SPML_CONC=0: one after the other on the compute stream)
+  cudaStream_t sps = nullptr;
+  cudaEvent_t ev_spf = nullptr, ev_spj = nullptr;
   bool no_overlap = false;  // SEIS_NO_OVERLAP=1: serial exchange (A/B measurements)
   // ACOUSTIC fused step (f1, kernels_acoustic_step.cuh): one persistent launch per time step,
   // one CTA per 64 x 32 tile, all co-resident; ntx x nty tiles, per-tile progress counters
@@ -724,6 +728,9 @@ seis_status seis_model_destroy(seis_model* M) {
   if (M->gexec) cudaGraphExecDestroy(M->gexec);
   if (M->cap) cudaStreamDestroy(M->cap);
   if (M->xs) cudaStreamDestroy(M->xs);
+  if (M->sps) cudaStreamDestroy(M->sps);
+  if (M->ev_spf) cudaEventDestroy(M->ev_spf);
+  if (M->ev_spj) cudaEventDestroy(M->ev_spj);
   if (M->ev_fork) cudaEventDestroy(M->ev_fork);
   if (M->ev_join) cudaEventDestroy(M->ev_join);
   for (void* p : M->ipc_open) cudaIpcCloseMemHandle(p);
@@ -1660,13 +1667,31 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
         if (S.sp) {
           // O6b: the blocks without layer points run the plain kernel (96 registers, high
           // occupancy), the others the split-field kernel; disjoint points, same arithmetic for
-          // the non-layer points of either
-          a.region = 1;
-          if (gh) go(std::false_type{}, std::true_type{});
-          else go(std::false_type{}, std::false_type{});
+          // the non-layer points of either.  The two launches run concurrently (the plain one
+          // on a side stream) so the light blocks fill the SMs around the heavy ones.
+          static const bool conc = !(getenv("SEIS_SPML_CONC") && getenv("SEIS_SPML_CONC")[0] == '0');
+          if (conc && !M->sps) {
+            CK(cudaStreamCreateWithFlags(&M->sps, cudaStreamNonBlocking));
+            CK(cudaEventCreateWithFlags(&M->ev_spf, cudaEventDisableTiming));
+            CK(cudaEventCreateWithFlags(&M->ev_spj, cudaEventDisableTiming));
+          }
+          cudaStream_t ks2 = ks;
+          if (conc) {
+            CK(cudaEventRecord(M->ev_spf, ks));
+            CK(cudaStreamWaitEvent(M->sps, M->ev_spf, 0));
+          }
           a.region = 2;
           if (gh) go(std::true_type{}, std::true_type{});
           else go(std::true_type{}, std::false_type{});
+          a.region = 1;
+          if (conc) ks = M->sps;
+          if (gh) go(std::false_type{}, std::true_type{});
+          else go(std::false_type{}, std::false_type{});
+          ks = ks2;
+          if (conc) {
+            CK(cudaEventRecord(M->ev_spj, M->sps));
+            CK(cudaStreamWaitEvent(ks, M->ev_spj, 0));
+          }
           ++g_launches;  // two launches (CKL counts one)
         } else if (gh) go(std::false_type{}, std::true_type{});
         else go(std::false_type{}, std::false_type{});
