@@ -220,8 +220,13 @@ seis_status seis_memory_required(const seis_grid* grid, seis_kind kind, const se
                                  int32_t nranks, uint64_t* bytes);
 /* Per-kernel CUDA-event timing (profiling / bench.py).  seis_profile(1) resets the
  * counters and starts recording an event pair on the launching stream around every
- * launch; seis_profile(0) stops.  seis_profile_read synchronises on the recorded
- * events and returns the summed device time and launch count of kernel id
+ * launch (launches then run eagerly, no shot graph); seis_profile(S), S > 1, resets and
+ * keeps the forward shot's CUDA graph, with event-record nodes around the launches of
+ * every S-th time step inside it, read back after each replay (the measured path is the
+ * production one; calling seis_profile(S) again in that mode only zeroes the counters, the
+ * graph is kept); seis_profile(0) stops.  seis_profile_read synchronises on the recorded
+ * events and returns the summed device time and launch count (sampled launches in the
+ * graph-sampled mode) of kernel id
  *   0 iso_step  1 ac_v  2 ac_p  3 el_v  4 el_s  5 inject  6 gather
  *   7 halo exchange (copies / NCCL)  8 free-surface mirror.
  * Process-wide, not thread-safe; meant for single-threaded measurement runs. */

@@ -359,9 +359,11 @@ KERNEL_IDS = {"iso_step": 0, "ac_v": 1, "ac_p": 2, "el_v": 3, "el_s": 4, "inject
               "gather": 6, "exchange": 7, "fs_mirror": 8, "ac_step": 9}
 
 
-def profile(enable: bool):
-    """Start (resetting the counters) / stop per-kernel CUDA-event timing in the library."""
-    _check(lib().seis_profile(1 if enable else 0))
+def profile(enable, sample: int = 1):
+    """Start (resetting the counters) / stop per-kernel CUDA-event timing in the library.
+    sample > 1: keep the forward shot's CUDA graph and time the launches of every sample-th
+    time step through event nodes inside it (seis.h seis_profile)."""
+    _check(lib().seis_profile((sample if sample > 1 else 1) if enable else 0))
 
 
 def profile_read():

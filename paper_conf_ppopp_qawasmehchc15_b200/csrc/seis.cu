@@ -77,12 +77,21 @@ static seis_status fail(seis_status st, const char* fmt, ...) {
 
 // ------------------------------------------------------------ profiling
 // Per-kernel CUDA-event timing (seis_profile / seis_profile_read): an event pair
-// recorded on the launching stream around every launch of a stencil / aux kernel.
+// recorded on the launching stream around every launch of a stencil / aux kernel (eager
+// launches), or -- graph-sampled mode, seis_profile(S > 1) -- around the launches of every
+// S-th time step of a forward shot, as event-record nodes INSIDE the shot's CUDA graph, read
+// back after every replay (the timed path stays the production graph).
 namespace prof {
 constexpr int NK = 10;
 static bool on = false;
+static int sample = 1;          // 1: every launch, eager; S > 1: graph-sampled every S-th step
+static bool sample_now = true;  // (graph-sampled) this time step is bracketed
+static int epoch = 0;           // seis_profile resets: part of the graph key (the events are reused)
 static std::vector<cudaEvent_t> ev[NK];  // start, stop, start, stop, ...
 static size_t used[NK] = {};
+static size_t glo[NK] = {}, ghi[NK] = {};  // (graph-sampled) pairs of the current graph
+static double acc_ms[NK] = {};
+static long long acc_n[NK] = {};
 static cudaEvent_t get(int k) {
   if (used[k] == ev[k].size()) {
     cudaEvent_t e;
@@ -94,13 +103,28 @@ static cudaEvent_t get(int k) {
 struct Scope {
   int k;
   cudaStream_t st;
-  Scope(int k_, cudaStream_t s) : k(k_), st(s) {
-    if (on) cudaEventRecord(get(k), st);
+  bool rec;
+  // (External: under stream capture the record becomes an event-record NODE of the graph,
+  // replayed with it, instead of a capture-internal dependency marker)
+  Scope(int k_, cudaStream_t s) : k(k_), st(s), rec(on && sample_now) {
+    if (rec) cudaEventRecordWithFlags(get(k), st, cudaEventRecordExternal);
   }
   ~Scope() {
-    if (on) cudaEventRecord(get(k), st);
+    if (rec) cudaEventRecordWithFlags(get(k), st, cudaEventRecordExternal);
   }
 };
+// (graph-sampled) add the pairs of the replay that just completed
+static cudaError_t harvest() {
+  for (int k = 0; k < NK; ++k)
+    for (size_t p = glo[k]; p + 1 < ghi[k]; p += 2) {
+      float ms = 0.f;
+      cudaError_t e = cudaEventElapsedTime(&ms, ev[k][p], ev[k][p + 1]);
+      if (e != cudaSuccess) return e;
+      acc_ms[k] += ms;
+      ++acc_n[k];
+    }
+  return cudaSuccess;
+}
 }  // namespace prof
 #define PROF(id, st) prof::Scope prof_scope_(id, st)
 
@@ -601,16 +625,34 @@ extern "C" {
 const char* seis_version(void) { return "seis-b200 0.1 (sm_100a)"; }
 
 seis_status seis_profile(int32_t enable) {
+  const int want = enable > 1 ? enable : 1;
   if (enable) {
-    for (int k = 0; k < prof::NK; ++k) prof::used[k] = 0;
+    // the same graph-sampled mode again: zero the counters only (the shot graph and its event
+    // nodes stay valid, no recapture); anything else: reset the event lists and force new graphs
+    const bool same = prof::on && prof::sample > 1 && prof::sample == want;
+    for (int k = 0; k < prof::NK; ++k) {
+      prof::acc_ms[k] = 0.0;
+      prof::acc_n[k] = 0;
+      if (!same) prof::used[k] = prof::glo[k] = prof::ghi[k] = 0;
+    }
+    if (!same) {
+      prof::sample = want;
+      ++prof::epoch;
+    }
   }
   prof::on = enable != 0;
+  prof::sample_now = true;
   return SEIS_OK;
 }
 
 seis_status seis_profile_read(int32_t kernel, double* total_ms, int64_t* launches) {
   if (kernel < 0 || kernel >= prof::NK || !total_ms || !launches)
     return fail(SEIS_EINVAL, "seis_profile_read: bad arguments");
+  if (prof::sample > 1) {  // graph-sampled: accumulated after every replay
+    *total_ms = prof::acc_ms[kernel];
+    *launches = (int64_t)prof::acc_n[kernel];
+    return SEIS_OK;
+  }
   double t = 0.0;
   const size_t n = prof::used[kernel] / 2;
   for (size_t p = 0; p < n; ++p) {
@@ -2140,9 +2182,11 @@ static seis_status forward_loop(seis_model* M, const seis_shot* sh, float* sd, s
   TRY(zero_state(M, st));
   if (ns) CK(cudaMemsetAsync(sd, 0, ns * sizeof(float), st));
   for (int n = 0; n < sh->nt; ++n) {
+    if (prof::sample > 1) prof::sample_now = n % prof::sample == 0;
     TRY(step(M, n, true, nullptr, nullptr, nullptr, st));
     if (sh->nrec) TRY(gather(M, sh, sd, n, st));
   }
+  prof::sample_now = true;
   // (a peer-only communicator has no NCCL: each rank returns its own receivers' columns; a
   // 1-rank NCCL communicator runs the same all-reduce, an identity)
   if (M->comm && M->comm->nccl && ns)
@@ -2168,13 +2212,17 @@ seis_status seis_forward_model(seis_model* M, const seis_shot* sh, float* seis, 
   // step count, replayed afterwards), so small grids and thin slabs are not launch-bound.  With
   // an NCCL communicator the graph holds the halo send/recv groups (on the side stream of the
   // overlapped exchange) and the seismogram all-reduce: every rank captures the same sequence
-  // of NCCL calls.  Peer halos (stream memory-operation flags) and profiling run eagerly.
-  const bool use_graph = !prof::on && !M->peer && !getenv("SEIS_NO_GRAPH");
+  // of NCCL calls.  Peer halos (stream memory-operation flags) and every-launch profiling run
+  // eagerly; graph-sampled profiling (seis_profile(S > 1)) keeps the graph.
+  const bool use_graph = (!prof::on || prof::sample > 1) && !M->peer && !getenv("SEIS_NO_GRAPH");
+  const int pmode = prof::on ? prof::sample : 0;
+  const int pkey[2] = {pmode, pmode > 1 ? prof::epoch : 0};
   if (persist_ok(M)) {
     TRY(forward_persist(M, sh, sd, ns, st));
   } else if (use_graph) {
     uint64_t key = fnv1a(&sd, sizeof(sd), M->shot_key);  // (the wavelet is read on the device)
     key = fnv1a(&sh->nt, sizeof(int32_t), key);
+    key = fnv1a(pkey, sizeof(pkey), key);  // (a graph with or without profiling event nodes)
     if (!M->gexec || M->gkey != key) {
       if (M->gexec) {
         cudaGraphExecDestroy(M->gexec);
@@ -2182,8 +2230,10 @@ seis_status seis_forward_model(seis_model* M, const seis_shot* sh, float* seis, 
       }
       if (!M->cap) CK(cudaStreamCreateWithFlags(&M->cap, cudaStreamNonBlocking));
       CK(cudaStreamSynchronize(st));
+      for (int k = 0; k < prof::NK; ++k) prof::glo[k] = prof::used[k];
       CK(cudaStreamBeginCapture(M->cap, cudaStreamCaptureModeThreadLocal));
       seis_status rc = forward_loop(M, sh, sd, ns, M->cap);
+      for (int k = 0; k < prof::NK; ++k) prof::ghi[k] = prof::used[k];
       cudaGraph_t graph = nullptr;
       cudaError_t e = cudaStreamEndCapture(M->cap, &graph);
       if (rc != SEIS_OK) {
@@ -2210,6 +2260,7 @@ seis_status seis_forward_model(seis_model* M, const seis_shot* sh, float* seis, 
   }
   if (!dev && ns) CK(cudaMemcpyAsync(seis, sd, ns * sizeof(float), cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
+  if (use_graph && pmode > 1) CK(prof::harvest());  // (this replay's event nodes are complete)
   M->last_nt = sh->nt;
   return SEIS_OK;
 }
