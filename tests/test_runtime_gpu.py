@@ -91,3 +91,37 @@ def test_host_staging_buffers_regrow():
     model.forward_model(shot3, big_d)
     assert np.array_equal(big_h, big_d.cpu().numpy())
     model.close()
+
+
+def test_graph_sampled_profiling():
+    """seis_profile(S > 1) keeps the shot graph and times the launches of every S-th step by
+    event nodes inside it (bench.py's timed region): the seismogram is bitwise the unprofiled
+    one, every sampled kernel has ceil(nt / S) launches per replay with positive times, the
+    counters accumulate over replays and a repeated seis_profile(S) zeroes them only."""
+    nx, ny, nz, nt, S = 100, 40, 48, 23, 5
+    m = inputs.random_media((nz, ny, nx), seed=81)
+    w = inputs.source_series("acoustic", nt, 5e-4, 30.0)
+    rec = np.asarray([[10, 10, 10], [50, 20, 30]], np.int32)
+    mod = seis.Model(seis.Grid(nx, ny, nz, 10.0, 5e-4, nb=5, pml_f=30.0), "acoustic", m["vp"], rho=m["rho"])
+    shot = seis.Shot((50, 20, 24), w, rec)
+    ref = np.zeros((nt, 2), np.float32)
+    mod.forward_model(shot, ref)
+    try:
+        seis.profile(True, sample=S)
+        out = np.zeros((nt, 2), np.float32)
+        mod.forward_model(shot, out)  # (captures the graph with its event nodes)
+        assert np.array_equal(out, ref)
+        seis.profile(True, sample=S)  # same mode: counters zeroed, graph kept
+        for _ in range(2):
+            mod.forward_model(shot, out)
+        kp = seis.profile_read()
+        per = -(-nt // S)
+        for k in ("ac_v", "ac_p", "gather"):
+            assert kp[k][1] == 2 * per, (k, kp[k])
+            assert kp[k][0] > 0
+        assert np.array_equal(out, ref)
+    finally:
+        seis.profile(False)
+    mod.forward_model(shot, out)
+    assert np.array_equal(out, ref)
+    mod.close()
