@@ -104,13 +104,19 @@ struct Scope {
   int k;
   cudaStream_t st;
   bool rec;
-  // (External: under stream capture the record becomes an event-record NODE of the graph,
-  // replayed with it, instead of a capture-internal dependency marker)
+  // (under stream capture, the External flag makes the record an event-record NODE of the
+  // graph, replayed with it, instead of a capture-internal dependency marker; outside a
+  // capture the flag is not allowed)
+  static void record(cudaEvent_t e, cudaStream_t s) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    cudaStreamIsCapturing(s, &cs);
+    cudaEventRecordWithFlags(e, s, cs == cudaStreamCaptureStatusActive ? cudaEventRecordExternal : cudaEventRecordDefault);
+  }
   Scope(int k_, cudaStream_t s) : k(k_), st(s), rec(on && sample_now) {
-    if (rec) cudaEventRecordWithFlags(get(k), st, cudaEventRecordExternal);
+    if (rec) record(get(k), st);
   }
   ~Scope() {
-    if (rec) cudaEventRecordWithFlags(get(k), st, cudaEventRecordExternal);
+    if (rec) record(get(k), st);
   }
 };
 // (graph-sampled) add the pairs of the replay that just completed
@@ -142,7 +148,7 @@ namespace {
 #define SEIS_BYI 8
 #endif
 #ifndef SEIS_BYV
-#define SEIS_BYV 8
+#define SEIS_BYV 16  // (r02 sweep: ac_v 0.756 vs 0.762 ms at C2 with 8 rows, profiles/r02_sweep_byv.jsonl)
 #endif
 #ifndef SEIS_BYP
 #define SEIS_BYP 8

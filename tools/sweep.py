@@ -19,8 +19,14 @@ sys.path.insert(0, ROOT)
 
 VARIANTS = {
     "base": [],
-    "el_mb1": ["SEIS_EL_MINB=1"],
+    "byv16": ["SEIS_BYV=16"],
+    "byv16_vns2": ["SEIS_BYV=16", "SEIS_AC_VNS=2"],
+    "byv12": ["SEIS_BYV=12"],
+    "base2": [],
+    "byv16b": ["SEIS_BYV=16"],
 }
+if os.environ.get("SWEEP_ONLY"):
+    VARIANTS = {k: v for k, v in VARIANTS.items() if k in os.environ["SWEEP_ONLY"].split(",")}
 
 
 def build():
