@@ -408,7 +408,7 @@ __device__ __forceinline__ void el_v_body(const ElVArgs& a) {
       // face buoyancy dt b/h = (dt/h) 2/(rho_i + rho_{i+1}), the last face clamps (O8, O9)
       const float* rc = st + L::R + ty * RW + 2 * tx;
       const F2 r0 = lds2(rc), ryn = lds2(rc + RW), rzn = lds2(st + L::RZ + pt);
-      const float rx2 = rc[2];
+      const float rx2 = lds2(rc + 2).v[0];  // (8-byte load: no 2-way bank conflict)
       const bool zlast = k + d.z0 + 1 >= d.nz;
       F2 ov[3];
 #pragma unroll
@@ -750,14 +750,27 @@ __device__ __forceinline__ void el_s_body(const ElSArgs& a) {
       const float* pa = st + L::WK + ty * RW + 2 * tx;
       const float* pb = st + L::WK1 + ty * RW + 2 * tx;
       const bool ylast = j + 1 >= d.ny, zlast = gz + 1 >= d.nz;
+      // (8-byte loads of columns x0 .. x0+3: scalar loads at a 2-float lane stride were 2-way
+      // bank conflicts; the column clamp is a register select)
       float wa0[3], wa1[3], wb0[3], wb1[3];
+      {
+        const F2 a01 = lds2(pa), a23 = lds2(pa + 2), a01n = lds2(pa + RW), a23n = lds2(pa + RW + 2);
+        const F2 b01 = lds2(pb), b23 = lds2(pb + 2), b01n = lds2(pb + RW), b23n = lds2(pb + RW + 2);
+        const float ra[3] = {a01.v[0], a01.v[1], a23.v[0]}, ran[3] = {a01n.v[0], a01n.v[1], a23n.v[0]};
+        const float rb[3] = {b01.v[0], b01.v[1], b23.v[0]}, rbn[3] = {b01n.v[0], b01n.v[1], b23n.v[0]};
+        const bool in1 = x0 + 1 < d.nx, in2 = x0 + 2 < d.nx;
 #pragma unroll
-      for (int c = 0; c < 3; ++c) {
-        const int cx = (x0 + c < d.nx) ? c : (c > 0 ? c - 1 : 0);
-        wa0[c] = pa[cx];
-        wa1[c] = ylast ? wa0[c] : pa[RW + cx];
-        wb0[c] = zlast ? wa0[c] : pb[cx];
-        wb1[c] = zlast ? wa1[c] : (ylast ? wb0[c] : pb[RW + cx]);
+        for (int c = 0; c < 3; ++c) {
+          // column c, clamped to the last node: c if x0 + c < nx, else c - 1 (c = 0 always inside)
+          const float va = c == 0 ? ra[0] : c == 1 ? (in1 ? ra[1] : ra[0]) : (in2 ? ra[2] : ra[1]);
+          const float van = c == 0 ? ran[0] : c == 1 ? (in1 ? ran[1] : ran[0]) : (in2 ? ran[2] : ran[1]);
+          const float vb = c == 0 ? rb[0] : c == 1 ? (in1 ? rb[1] : rb[0]) : (in2 ? rb[2] : rb[1]);
+          const float vbn = c == 0 ? rbn[0] : c == 1 ? (in1 ? rbn[1] : rbn[0]) : (in2 ? rbn[2] : rbn[1]);
+          wa0[c] = va;
+          wa1[c] = ylast ? wa0[c] : van;
+          wb0[c] = zlast ? wa0[c] : vb;
+          wb1[c] = zlast ? wa1[c] : (ylast ? wb0[c] : vbn);
+        }
       }
       const bool surf = a.fs && gz == 0;
       const long long rel = srel0 - (long long)(k + GZ) * PS;
