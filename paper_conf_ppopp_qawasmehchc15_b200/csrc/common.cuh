@@ -379,6 +379,35 @@ struct SrcAmp {
   float scale = 0.f;
   __device__ __forceinline__ float get() const { return __fmul_rn(scale, __ldg(w + n)); }
 };
+// Where a z-marching thread adds the source: the source node has padded index
+// src_o (-1: none); the thread owns the `width` consecutive x points at padded column offset
+// oc.  The node is the thread's point e of slab-local plane k iff
+// src_o - oc - (k + GZ) PS = e in [0, width) -- at most one k since PS > width.  Resolved once
+// per thread (k = -1: never) instead of a 64-bit test per plane; the same add at the same point.
+struct SrcHit {
+  int ke = -1;  // 4 k + e (one register), -1: never
+  __device__ __forceinline__ bool at(int k) const { return (ke >> 2) == k; }
+  __device__ __forceinline__ int e() const { return ke & 3; }
+};
+__device__ __forceinline__ SrcHit src_hit(long long src_o, long long oc, long long PS, int width) {
+  SrcHit h;
+  const long long r = src_o - oc;
+  if (src_o >= 0 && r >= 0) {
+    // m = floor(r / PS) without the 64-bit division routine: a float estimate (relative error
+    // < 2^-21, so off by at most one while r / PS < 2^21 planes) and one exact correction
+    long long m = (long long)((float)r * __frcp_rn((float)PS));
+    long long e = r - m * PS;
+    if (e < 0) {
+      --m;
+      e += PS;
+    } else if (e >= PS) {
+      ++m;
+      e -= PS;
+    }
+    if (e < width && m >= GZ) h.ke = (int)(m - GZ) * 4 + (int)e;
+  }
+  return h;
+}
 }  // namespace seis
 
 // ------------------------------------------------------ direct ghost-plane stores

@@ -132,6 +132,7 @@ __global__ void SEIS_AC_LB(NTX * BY) ac_v_kernel(const __grid_constant__ AcVArgs
   for (int t = 0; t < 7; ++t) r[t] = ldg4(p + (long long)(k0 - 3 + t + GZ) * PS + oc);
   const float dth = a.dth;
 
+  const bool ghk = a.gh.lo || a.gh.hi;  // does this slab store a neighbour's ghost planes (f4)?
   SEIS_UNROLL(SEIS_ZU_AC)
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
@@ -229,10 +230,17 @@ __global__ void SEIS_AC_LB(NTX * BY) ac_v_kernel(const __grid_constant__ AcVArgs
         oy.v[e] = fmaf(by, dy[e], qyo.v[e]);
         oz.v[e] = fmaf(bz, dz[e], qzo.v[e]);
       }
-      st4_masked(a.qx + o, ox, x0, d.nx, true);
-      st4_masked(a.qy + o, oy, x0, d.nx, true);
-      st4_masked(a.qz + o, oz, x0, d.nx, true);
-      ghost_st4(a.gh, o, k, d.nzl, oz, x0, d.nx);
+      // one x-bound branch for the 3 stores; ghost tests only on a slab's 4 boundary planes
+      if (x0 + 3 < d.nx) {
+        st4(a.qx + o, ox);
+        st4(a.qy + o, oy);
+        st4(a.qz + o, oz);
+      } else {
+        st4_masked(a.qx + o, ox, x0, d.nx, false);
+        st4_masked(a.qy + o, oy, x0, d.nx, false);
+        st4_masked(a.qz + o, oz, x0, d.nx, false);
+      }
+      if (ghk && (k < 4 || k >= d.nzl - 4)) ghost_st4(a.gh, o, k, d.nzl, oz, x0, d.nx);
       if (IMG) {
         const long long cix = ((long long)k * d.ny + j) * d.nx + x0;
         F4 im;
@@ -329,13 +337,25 @@ __global__ void SEIS_AC_LB(NTX * BY) ac_p_kernel(const __grid_constant__ AcPArgs
   F4 q[8];  // q_z at k-4 .. k+3; plane k+3 arrives with stage k (TMA)
 #pragma unroll
   for (int t = 0; t < 7; ++t) q[t] = ldg4(qz + (long long)(k0 - 4 + t + GZ) * PS + oc);
-  const long long srel0 = a.src_o - oc;
+  const SrcHit sh = src_hit(a.src_o, oc, PS, 4);
 
+  const bool ghk = a.gh.lo || a.gh.hi;  // does this slab store a neighbour's ghost planes (f4)?
+  int s_ = 0;
+  uint32_t ph_ = 0u;
+  long long o_ = (long long)(k0 + GZ) * PS + oc;
   SEIS_UNROLL(SEIS_ZU_AC)
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
-    const int s = it % AC_NS;
-    const long long o = (long long)(k + GZ) * PS + oc;
+    // ring slot, its phase and the plane offset carried across iterations (no division by the
+    // ring depth or 64-bit multiply per plane)
+    const int s = s_;
+    const uint32_t ph = ph_;
+    const long long o = o_;
+    o_ += PS;
+    if (++s_ == AC_NS) {
+      s_ = 0;
+      ph_ ^= 1u;
+    }
     // C-PML: old psi values are loaded before the wait (latency overlap)
     const int gz = k + d.z0;
     const bool lz = Wl > 0 && CpmlIdx::in(gz, d.nz, Wl, a.zlo);
@@ -353,7 +373,7 @@ __global__ void SEIS_AC_LB(NTX * BY) ac_p_kernel(const __grid_constant__ AcPArgs
       psi_idx_row<4>(izz, (CpmlIdx::slot(gz, d.nz, Wl) * d.ny + j) * d.nx + x0, x0, d.nx);
       psi_ld<4>(oz, a.pqz, izz);
     }
-    mbar_wait(&bar[s], (it / AC_NS) & 1);
+    mbar_wait(&bar[s], ph);
     const float* st = sm + s * L::SIZE;
     q[7] = lds4(st + L::QQ + ty * TXV + 4 * tx);
     const float* cx = st + L::QX + ty * WX + 4 * tx + 4;      // q_x(x0, j)
@@ -413,14 +433,14 @@ __global__ void SEIS_AC_LB(NTX * BY) ac_p_kernel(const __grid_constant__ AcPArgs
       F4 out;
 #pragma unroll
       for (int e = 0; e < 4; ++e) out.v[e] = fmaf(kv.v[e], (dx[e] + dy[e]) + dz[e], pv.v[e]);
-      const long long rel = srel0 - (long long)(k + GZ) * PS;
-      if (rel >= 0 && rel < 4) {
+      if (sh.at(k)) {  // (selects: a branch per component became a local-memory array)
+        const float sa = a.src.get();
+        const int se = sh.e();
 #pragma unroll
-        for (int e = 0; e < 4; ++e)
-          if (rel == e) out.v[e] += a.src.get();
+        for (int e = 0; e < 4; ++e) out.v[e] = (se == e) ? out.v[e] + sa : out.v[e];
       }
       st4_masked(a.p + o, out, x0, d.nx, true);
-      ghost_st4(a.gh, o, k, d.nzl, out, x0, d.nx);
+      if (ghk && (k < 4 || k >= d.nzl - 4)) ghost_st4(a.gh, o, k, d.nzl, out, x0, d.nx);
       if (SNAP) st4_masked(a.snap + ((long long)k * d.ny + j) * d.nx + x0, out, x0, d.nx, (d.nx & 3) == 0);
     }
     stage_release(&cnt[s], tid, it + AC_NS < np, [&] {

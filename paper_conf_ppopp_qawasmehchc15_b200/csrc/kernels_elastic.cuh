@@ -293,6 +293,8 @@ __device__ __forceinline__ void el_v_body(const ElVArgs& a) {
       qzz[t] = ldg2(szz + (long long)(k0 - 3 + t + GZ) * PS + oc);
     }
   }
+  // does this slab store ghost planes of a neighbour (f4)?
+  const bool ghk = a.gh[0].lo || a.gh[0].hi || a.gh[1].lo || a.gh[1].hi || a.gh[2].lo || a.gh[2].hi;
   SEIS_UNROLL(SEIS_ZU_EL)
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
@@ -423,10 +425,18 @@ __device__ __forceinline__ void el_v_body(const ElVArgs& a) {
         ov[1].v[e] = fmaf(by, (d3[e] + d4[e]) + d5[e], v1.v[e]);
         ov[2].v[e] = fmaf(bz, (d6[e] + d7[e]) + d8[e], v2.v[e]);
       }
+      // one x-bound branch for the 3 stores (a branch per store cost a reconvergence pair each);
+      // the ghost-store tests only on the 4 boundary planes of a slab that has a neighbour
+      if (x0 + 1 < d.nx) {
 #pragma unroll
-      for (int c = 0; c < 3; ++c) {
-        st2_masked(a.f[EVX + c] + o, ov[c], x0, d.nx);
-        ghost_st2(a.gh[c], o, k, d.nzl, ov[c], x0, d.nx);
+        for (int c = 0; c < 3; ++c) *reinterpret_cast<float2*>(a.f[EVX + c] + o) = make_float2(ov[c].v[0], ov[c].v[1]);
+      } else {
+#pragma unroll
+        for (int c = 0; c < 3; ++c) a.f[EVX + c][o] = ov[c].v[0];
+      }
+      if (ghk && (k < 4 || k >= d.nzl - 4)) {
+#pragma unroll
+        for (int c = 0; c < 3; ++c) ghost_st2(a.gh[c], o, k, d.nzl, ov[c], x0, d.nx);
       }
       if (IMG) {
         const long long cix = ((long long)k * d.ny + j) * d.nx + x0;
@@ -626,7 +636,11 @@ __device__ __forceinline__ void el_s_body(const ElSArgs& a) {
       qz[t] = ldg2(vz + (long long)(k0 - 4 + t + GZ) * PS + oc);
     }
   }
+  // (the per-plane 64-bit source test stays here: src_hit measured slower in this kernel,
+  // el_s 0.847 vs 0.821 ms, profiles/r02_src_store_ab.log)
   const long long srel0 = a.src_o - oc;
+  // does this slab store ghost planes of a neighbour (f4)?
+  const bool ghk = a.gh[0].lo || a.gh[0].hi || a.gh[1].lo || a.gh[1].hi || a.gh[2].lo || a.gh[2].hi;
   SEIS_UNROLL(SEIS_ZU_EL)
   for (int it = 0; it < np; ++it) {
     const int k = k0 + it;
@@ -773,7 +787,6 @@ __device__ __forceinline__ void el_s_body(const ElSArgs& a) {
         }
       }
       const bool surf = a.fs && gz == 0;
-      const long long rel = srel0 - (long long)(k + GZ) * PS;
       F2 o6[6];
 #pragma unroll
       for (int e = 0; e < 2; ++e) {
@@ -787,7 +800,7 @@ __device__ __forceinline__ void el_s_body(const ElSArgs& a) {
         float sxx = sv[0].v[e] + fmaf(l2m, exx[e], lam * (eyy[e] + ez));
         float syy = sv[1].v[e] + fmaf(l2m, eyy[e], lam * (exx[e] + ez));
         float szz = sv[2].v[e] + fmaf(l2m, ez, lam * (exx[e] + eyy[e]));
-        if (rel == e) {
+        if (srel0 - (long long)(k + GZ) * PS == e) {
           const float sa = a.src.get();
           sxx -= sa;
           syy -= sa;
@@ -801,11 +814,19 @@ __device__ __forceinline__ void el_s_body(const ElSArgs& a) {
         o6[4].v[e] = fmaf(mxz, dzvx[e] + dxvz[e], sv[4].v[e]);
         o6[5].v[e] = fmaf(myz, dzvy[e] + dyvz[e], sv[5].v[e]);
       }
+      // (one x-bound branch for the 6 stores; ghost tests only on boundary planes, as el_v)
+      if (x0 + 1 < d.nx) {
 #pragma unroll
-      for (int c = 0; c < 6; ++c) st2_masked(a.f[ESXX + c] + o, o6[c], x0, d.nx);
-      ghost_st2(a.gh[0], o, k, d.nzl, o6[2], x0, d.nx);
-      ghost_st2(a.gh[1], o, k, d.nzl, o6[4], x0, d.nx);
-      ghost_st2(a.gh[2], o, k, d.nzl, o6[5], x0, d.nx);
+        for (int c = 0; c < 6; ++c) *reinterpret_cast<float2*>(a.f[ESXX + c] + o) = make_float2(o6[c].v[0], o6[c].v[1]);
+      } else {
+#pragma unroll
+        for (int c = 0; c < 6; ++c) a.f[ESXX + c][o] = o6[c].v[0];
+      }
+      if (ghk && (k < 4 || k >= d.nzl - 4)) {
+        ghost_st2(a.gh[0], o, k, d.nzl, o6[2], x0, d.nx);
+        ghost_st2(a.gh[1], o, k, d.nzl, o6[4], x0, d.nx);
+        ghost_st2(a.gh[2], o, k, d.nzl, o6[5], x0, d.nx);
+      }
       if (SNAP) {
         const long long cix = ((long long)k * d.ny + j) * d.nx + x0;
 #pragma unroll

@@ -194,7 +194,7 @@ __global__ void __launch_bounds__(NTX * BY, SPML ? SEIS_SPML_MINB : 1) iso_step_
     cby = __ldg(a.spco[1] + a.spnp[1] + j);
     ccy = __ldg(a.spco[1] + 2 * a.spnp[1] + j);
   }
-  const long long srel0 = a.src_o - oc;  // source offset relative to this column
+  const SrcHit sh = src_hit(a.src_o, oc, PS, 4);  // the source node of this column, if any
   // block-uniform: does this tile touch the x / y damping layer?  Planes outside the z layer
   // of such tiles take the undamped update without per-point branches (same arithmetic).
   const bool dxy = __syncthreads_or(exy.v[0] != 0.f || exy.v[1] != 0.f || exy.v[2] != 0.f || exy.v[3] != 0.f);
@@ -399,15 +399,14 @@ __global__ void __launch_bounds__(NTX * BY, SPML ? SEIS_SPML_MINB : 1) iso_step_
       }
     }
     if (own) {
-      const long long rel = srel0 - (long long)(k + GZ) * PS;
-      if (rel >= 0 && rel < 4) {
+      if (sh.at(k)) {  // (selects, as ac_p)
+        const float sa = a.src.get();
+        const int se = sh.e();
 #pragma unroll
-        for (int e = 0; e < 4; ++e)
-          if (rel == e) {
-            const float sa = a.src.get();
-            out.v[e] += sa;
-            if (SPML && sidx[e] >= 0) a.sp[(long long)(1 - a.lvl) * 3 * a.spn + sidx[e]] += sa;  // x component
-          }
+        for (int e = 0; e < 4; ++e) {
+          out.v[e] = (se == e) ? out.v[e] + sa : out.v[e];
+          if (SPML && se == e && sidx[e] >= 0) a.sp[(long long)(1 - a.lvl) * 3 * a.spn + sidx[e]] += sa;  // x component
+        }
       }
       st4_masked(a.up + o, out, x0, d.nx, true);
       if (GH) ghost_st4(a.gh, o, k, d.nzl, out, x0, d.nx);
