@@ -328,9 +328,16 @@ seis_status make_map(CUtensorMap* m, float* base, const Dims& d, int bw, int bh,
   cuuint64_t str[2] = {(cuuint64_t)d.PX * 4, (cuuint64_t)d.PS * 4};
   cuuint32_t box[3] = {(cuuint32_t)bw, (cuuint32_t)bh, (cuuint32_t)bd};
   cuuint32_t es[3] = {1, 1, 1};
+  // L2 sector promotion of the tile loads (SEIS_L2PROMO = 0 none, 1 64 B, 2 128 B, 3 256 B: sweeps)
+  static const int promo_env = getenv("SEIS_L2PROMO") ? atoi(getenv("SEIS_L2PROMO")) : -1;
+  const CUtensorMapL2promotion promo =
+      promo_env == 0 ? CU_TENSOR_MAP_L2_PROMOTION_NONE
+      : promo_env == 1 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B
+      : promo_env == 3 ? CU_TENSOR_MAP_L2_PROMOTION_L2_256B
+                       : CU_TENSOR_MAP_L2_PROMOTION_L2_128B;
   CUresult r = g_encode(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, base, dims, str, box, es,
-                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                        CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, promo,
+                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return fail(SEIS_ECUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
   return SEIS_OK;
 }
