@@ -357,6 +357,24 @@ def run_extras(args, local):
     res["iso_512"] = {"gpts_s": round(n ** 3 * 200 / (ms * 1e-3) / 1e9, 3), "ms_per_shot": round(ms, 3),
                       "roofline": kernel_frac("iso_step", float(n) ** 3, 16.0)}
     m.close()
+    # the same with the ISO 2-step kernel (f1, opt-in SEIS_ISO2=1 at model creation; 20 B per
+    # point per launch of two steps)
+    old = os.environ.get("SEIS_ISO2")
+    os.environ["SEIS_ISO2"] = "1"
+    try:
+        m = seis.Model(g, "iso", vp, device=local)
+    finally:
+        if old is None:
+            del os.environ["SEIS_ISO2"]
+        else:
+            os.environ["SEIS_ISO2"] = old
+    m.forward_model(shot, buf, stream)
+    ms = _timed_shots(lambda: m.forward_model(shot, buf, stream), 2, stream, prof=True)
+    seis.profile(False)
+    res["iso_512_two_step"] = {"gpts_s": round(n ** 3 * 200 / (ms * 1e-3) / 1e9, 3), "ms_per_shot": round(ms, 3),
+                               "roofline": kernel_frac("iso2", float(n) ** 3, 20.0),
+                               "note": "f1 2-step temporal blocking, opt-in (slower than the one-step kernel)"}
+    m.close()
     # the same with the split-field PML (O6b): layer points also read u^(d) at two levels and
     # write the new level (36 B per layer point)
     g = seis.Grid(n, n, n, 10.0, 1e-3, nb=20, iso_pml=1)

@@ -228,7 +228,8 @@ seis_status seis_memory_required(const seis_grid* grid, seis_kind kind, const se
  * events and returns the summed device time and launch count (sampled launches in the
  * graph-sampled mode) of kernel id
  *   0 iso_step  1 ac_v  2 ac_p  3 el_v  4 el_s  5 inject  6 gather
- *   7 halo exchange (copies / NCCL)  8 free-surface mirror.
+ *   7 halo exchange (copies / NCCL)  8 free-surface mirror  9 fused acoustic step
+ *   10 ISO 2-step kernel.
  * Process-wide, not thread-safe; meant for single-threaded measurement runs. */
 seis_status seis_profile(int32_t enable);
 seis_status seis_profile_read(int32_t kernel, double* total_ms, int64_t* launches);

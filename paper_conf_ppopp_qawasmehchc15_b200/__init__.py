@@ -356,7 +356,7 @@ class Model:
 
 
 KERNEL_IDS = {"iso_step": 0, "ac_v": 1, "ac_p": 2, "el_v": 3, "el_s": 4, "inject": 5,
-              "gather": 6, "exchange": 7, "fs_mirror": 8, "ac_step": 9}
+              "gather": 6, "exchange": 7, "fs_mirror": 8, "ac_step": 9, "iso2": 10}
 
 
 def profile(enable, sample: int = 1):

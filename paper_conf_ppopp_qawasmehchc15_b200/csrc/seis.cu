@@ -27,6 +27,7 @@
 #include "kernels_aux.cuh"
 #include "kernels_elastic.cuh"
 #include "kernels_iso.cuh"
+#include "kernels_iso2.cuh"
 
 using namespace seis;
 
@@ -82,7 +83,7 @@ static seis_status fail(seis_status st, const char* fmt, ...) {
 // S-th time step of a forward shot, as event-record nodes INSIDE the shot's CUDA graph, read
 // back after every replay (the timed path stays the production graph).
 namespace prof {
-constexpr int NK = 10;
+constexpr int NK = 11;
 static bool on = false;
 static int sample = 1;          // 1: every launch, eager; S > 1: graph-sampled every S-th step
 static bool sample_now = true;  // (graph-sampled) this time step is bracketed
@@ -173,6 +174,7 @@ struct Slab {
   // TMA descriptors of every operand tile the kernels stage:
   // "t" = tile with x/y halo, "c" = interior (centre) tile 32 x BY
   CUtensorMap iso_ut[2], iso_uc[2], iso_m;                              // ISO
+  CUtensorMap i2_t[2], i2_c[2], i2_m;  // ISO 2-step kernel: u tiles (+ halo 4), u / m interior
   CUtensorMap ac_pt, ac_qc[3], ac_rt, ac_rc, ac_pc;        // ACOUSTIC V
   CUtensorMap ac_qxt, ac_qyt, ac_ppc, ac_qzc, ac_kc;        // ACOUSTIC P
   CUtensorMap el_sxxt, el_sxyt, el_sxzt, el_syyt, el_syzt, el_vc[3], el_rt, el_rc;  // ELASTIC V
@@ -268,6 +270,9 @@ struct seis_model {
   bool ac_step = false;
   int as_ntx = 0, as_nty = 0;
   unsigned* as_cnt = nullptr;
+  bool iso2 = false;  // f1: ISO forward steps in pairs (kernels_iso2.cuh)
+  int i2_ntx = 0, i2_nty = 0;
+  unsigned* i2_cnt = nullptr;
   long long g_launches = 0;
   // f4 direct ghost stores: `direct` = the faces between the slabs of this
   // process are written by the producing kernels (no copies); `peer` = the rank faces too,
@@ -435,6 +440,8 @@ seis_status set_smem_attrs() {
   SMEM_ATTR((ac_step_kernel<false, false>), AcSLayout::smem_bytes());
   SMEM_ATTR((ac_step_kernel<true, false>), AcSLayout::smem_bytes());
   SMEM_ATTR((ac_step_kernel<false, true>), AcSLayout::smem_bytes());
+  SMEM_ATTR((iso2_kernel<false>), Iso2Layout::smem_bytes());
+  SMEM_ATTR((iso2_kernel<true>), Iso2Layout::smem_bytes());
   SMEM_ATTR((el_v_kernel<BYE, false, true>), ElVStage<BYE>::smem_bytes());
   SMEM_ATTR((el_v_kernel<BYE, true, true>), ElVStage<BYE>::smem_bytes());
   SMEM_ATTR((el_s_kernel<BYE, false, true>), ElSStage<BYE>::smem_bytes());
@@ -1074,6 +1081,36 @@ static seis_status model_create_impl(seis_model* M, const float* vp, const float
       void* p = nullptr;
       TRY(alloc_track(M, &p, (size_t)ntx * nty * sizeof(unsigned)));
       M->as_cnt = (unsigned*)p;
+    }
+  }
+  // f1: ISO 2-step temporal blocking (kernels_iso2.cuh) for forward modeling on a single-slab,
+  // single-process model without the split-field PML whose tiles are all co-resident
+  // (cooperative launch).  Opt-in (SEIS_ISO2=1): bitwise the one-step kernel's results
+  // (tests/test_iso2_gpu.py) but slower at 512^3 (0.892 ms per two steps vs 2 x 0.353 ms:
+  // 14 warps per SM with two 9-deep register queues are issue / shared-memory-latency bound,
+  // DESIGN.md §6 "ISO 2-step").
+  if (kind == SEIS_ISO && ns == 1 && !M->comm && !(g.iso_pml && g.nb > 0)) {
+    const int ntx = (g.nx + I2_TX - 1) / I2_TX, nty = (g.ny + I2_TY - 1) / I2_TY;
+    int occ2 = 0, coop = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ2, iso2_kernel<true>, I2_THREADS,
+                                                     Iso2Layout::smem_bytes()));
+    CK(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, M->device));
+    const bool fits = coop && occ2 >= 1 && (long long)ntx * nty <= (long long)occ2 * dev_sms;
+    const char* e = getenv("SEIS_ISO2");
+    M->iso2 = fits && e && e[0] == '1';
+    if (M->iso2) {
+      Slab& S = M->slabs[0];
+      const Dims& d = S.d;
+      for (int t = 0; t < 2; ++t) {
+        TRY(make_map(&S.i2_t[t], S.fld[t], d, I2_TX + 8, I2_TY + 8));
+        TRY(make_map(&S.i2_c[t], S.fld[t], d, I2_TX, I2_TY));
+      }
+      TRY(make_map(&S.i2_m, S.m, d, I2_TX, I2_TY));
+      M->i2_ntx = ntx;
+      M->i2_nty = nty;
+      void* p = nullptr;
+      TRY(alloc_track(M, &p, (size_t)ntx * nty * sizeof(unsigned)));
+      M->i2_cnt = (unsigned*)p;
     }
   }
   // f4: the faces between the slabs of this process by direct ghost stores of the producing
@@ -2031,6 +2068,51 @@ seis_status step(seis_model* M, int n, bool with_src, std::vector<float*>* snap,
   return run_phase(M, k_s, post_s, st);
 }
 
+// f1: ISO time steps n and n + 1 in one cooperative launch (kernels_iso2.cuh); u^{n+1} lands
+// in fld[1 - cur], u^{n+2} in fld[cur] (cur is unchanged, as after two single steps).
+seis_status step2(seis_model* M, int n, cudaStream_t st) {
+  Slab& S = M->slabs[0];
+  const int c = S.cur;
+  Iso2Args a;
+  a.mat = S.i2_t[c];
+  a.mbc = S.i2_c[1 - c];
+  a.mm = S.i2_m;
+  a.mac = S.i2_c[c];
+  a.mbt = S.i2_t[1 - c];
+  a.ua = S.fld[c];
+  a.ub = S.fld[1 - c];
+  a.uaw = S.fld[c];
+  a.edx = M->edx;
+  a.edy = M->edy;
+  a.edz = M->edz;
+  a.d = S.d;
+  a.ntx = M->i2_ntx;
+  a.nty = M->i2_nty;
+  a.cnt = M->i2_cnt;
+  a.src_o = S.src_o;
+  a.src1 = SrcAmp{M->dwav, n, S.src_scale};
+  a.src2 = SrcAmp{M->dwav, n + 1, S.src_scale};
+  const int ntiles = M->i2_ntx * M->i2_nty;
+  CK(cudaMemsetAsync(M->i2_cnt, 0, (size_t)ntiles * sizeof(unsigned), st));
+  {
+    PROF(10, st);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(ntiles);
+    cfg.blockDim = dim3(I2_THREADS);
+    cfg.dynamicSmemBytes = Iso2Layout::smem_bytes();
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    if (a.edx) CK(cudaLaunchKernelEx(&cfg, iso2_kernel<true>, a));
+    else CK(cudaLaunchKernelEx(&cfg, iso2_kernel<false>, a));
+  }
+  CKL();
+  return SEIS_OK;
+}
+
 // Field holding the recorded / imaged quantity
 const float* out_field(seis_model* M, Slab& S, int comp) {
   if (M->kind == SEIS_ISO) return S.fld[S.cur];
@@ -2194,10 +2276,25 @@ extern "C" {
 static seis_status forward_loop(seis_model* M, const seis_shot* sh, float* sd, size_t ns, cudaStream_t st) {
   TRY(zero_state(M, st));
   if (ns) CK(cudaMemsetAsync(sd, 0, ns * sizeof(float), st));
-  for (int n = 0; n < sh->nt; ++n) {
+  for (int n = 0; n < sh->nt;) {
+    if (M->iso2 && n + 1 < sh->nt) {  // steps n, n + 1 in one launch (f1), then both rows
+      if (prof::sample > 1) prof::sample_now = n % prof::sample == 0 || (n + 1) % prof::sample == 0;
+      TRY(step2(M, n, st));
+      if (sh->nrec) {
+        Slab& S = M->slabs[0];
+        const int c0 = S.cur;  // u^{n+1} is in fld[1 - c0], u^{n+2} in fld[c0]
+        S.cur = 1 - c0;
+        TRY(gather(M, sh, sd, n, st));
+        S.cur = c0;
+        TRY(gather(M, sh, sd, n + 1, st));
+      }
+      n += 2;
+      continue;
+    }
     if (prof::sample > 1) prof::sample_now = n % prof::sample == 0;
     TRY(step(M, n, true, nullptr, nullptr, nullptr, st));
     if (sh->nrec) TRY(gather(M, sh, sd, n, st));
+    ++n;
   }
   prof::sample_now = true;
   // (a peer-only communicator has no NCCL: each rank returns its own receivers' columns; a

@@ -33,13 +33,29 @@ def main():
     m.forward_model(shot, out)
     torch.cuda.synchronize()
     seis.profile(False)
-    kp = seis.profile_read()["iso_step"]
-    t = kp[0] / kp[1]
-    lay = 1.0 - ((n - 40) / n) ** 3
-    bpp = 16.0 + (36.0 * lay if a.pml else 0.0)
-    print(json.dumps({"n": n, "pml": a.pml, "iso_step_ms": round(t, 4), "alg_B_per_pt": round(bpp, 2),
-                      "frac": round(float(n) ** 3 * bpp / (t * 1e-3) / 1e9 / 6538.3, 4),
-                      "seis": float(out.abs().sum().item())}))
+    prof = seis.profile_read()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    m.forward_model(shot, out)
+    e1.record()
+    torch.cuda.synchronize()
+    shot_ms = e0.elapsed_time(e1)
+    res = {"n": n, "pml": a.pml, "ms_per_step": round(shot_ms / a.nt, 4),
+           "gpts_s": round(float(n) ** 3 * a.nt / (shot_ms * 1e-3) / 1e9, 2)}
+    if "iso2" in prof:  # the 2-step kernel (f1): 20 B per point per launch of two steps
+        kp = prof["iso2"]
+        t = kp[0] / kp[1]
+        res.update({"iso2_ms": round(t, 4), "alg_B_per_pt": 20.0,
+                    "frac": round(float(n) ** 3 * 20.0 / (t * 1e-3) / 1e9 / 6538.3, 4)})
+    if "iso_step" in prof:
+        kp = prof["iso_step"]
+        t = kp[0] / kp[1]
+        lay = 1.0 - ((n - 40) / n) ** 3
+        bpp = 16.0 + (36.0 * lay if a.pml else 0.0)
+        res.update({"iso_step_ms": round(t, 4), "alg_B_per_pt_step": round(bpp, 2),
+                    "frac_step": round(float(n) ** 3 * bpp / (t * 1e-3) / 1e9 / 6538.3, 4)})
+    res["seis"] = float(out.abs().sum().item())
+    print(json.dumps(res))
 
 
 if __name__ == "__main__":
