@@ -122,6 +122,44 @@ constexpr int EL_PF = SEIS_EL_PF;
 #endif
 constexpr int EL_VNS = SEIS_EL_VNS;
 constexpr int EL_SNS = SEIS_EL_SNS;
+// (C-PML body) L2 prefetch of the memory variables SEIS_EL_{V,S}PSIPF planes ahead, one lane
+// per 128-byte slab line (0 = off).  Measured at C3 (profiles/r02_el_psipf.log): el_s 0.824 ->
+// 0.812 ms at distance 2 (1: 0.814, 4: 0.934); el_v 0.650 -> 0.652 (no gain): S only.
+#ifndef SEIS_EL_VPSIPF
+#define SEIS_EL_VPSIPF 0
+#endif
+#ifndef SEIS_EL_SPSIPF
+#define SEIS_EL_SPSIPF 2
+#endif
+
+// the L2 prefetch above: arrays X of the x slab [nzl][ny][2W], Y of the y slab [nzl][2W][nx],
+// Z of the z slab [2W][ny][nx] at plane kk of this thread's row (lanes 0 / 16 of a warp row
+// cover its 64 floats; the x-slab row is 2W contiguous floats)
+template <int X0, int X1, int X2, int Y0, int Y1, int Y2, int Z0, int Z1, int Z2>
+__device__ __forceinline__ void el_psi_prefetch(float* const* psi, const Dims& d, int W, int zlo, int tx, int x0,
+                                                int j, bool lx, bool ly, int kk) {
+  if (kk >= d.nzl) return;
+  if (lx && (tx & 7) == 0) {
+    const int b = (kk * d.ny + j) * (2 * W) + (x0 < W ? 0 : W);
+    prefetch_l2(psi[X0] + b);
+    prefetch_l2(psi[X1] + b);
+    prefetch_l2(psi[X2] + b);
+  }
+  if ((tx & 15) != 0) return;
+  if (ly) {
+    const int b = (kk * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0;
+    prefetch_l2(psi[Y0] + b);
+    prefetch_l2(psi[Y1] + b);
+    prefetch_l2(psi[Y2] + b);
+  }
+  const int gz = kk + d.z0;
+  if (CpmlIdx::in(gz, d.nz, W, zlo)) {
+    const int b = (CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0;
+    prefetch_l2(psi[Z0] + b);
+    prefetch_l2(psi[Z1] + b);
+    prefetch_l2(psi[Z2] + b);
+  }
+}
 
 struct ElVArgs {
   CUtensorMap msxx;   // box 72 x BY      (x halo)
@@ -323,6 +361,8 @@ __device__ __forceinline__ void el_v_body(const ElVArgs& a) {
       psi_ld<2>(oz5, a.psi[5], izz);
       psi_ld<2>(oz8, a.psi[8], izz);
     }
+    if (SEIS_EL_VPSIPF > 0 && W > 0 && own)
+      el_psi_prefetch<0, 3, 6, 1, 4, 7, 2, 5, 8>(a.psi, d, W, a.zlo, tx, x0, j, lx, ly, k + SEIS_EL_VPSIPF);
     mbar_wait(&bar[s], (it / EL_VNS) & 1);
     const float* st = sm + s * L::SIZE;
     const int pt = ty * TXE + 2 * tx;
@@ -669,6 +709,8 @@ __device__ __forceinline__ void el_s_body(const ElSArgs& a) {
       psi_ld<2>(oz5, a.psi[5], izz);
       psi_ld<2>(oz7, a.psi[7], izz);
     }
+    if (SEIS_EL_SPSIPF > 0 && W > 0 && own)
+      el_psi_prefetch<0, 4, 6, 1, 3, 8, 2, 5, 7>(a.psi, d, W, a.zlo, tx, x0, j, lx, ly, k + SEIS_EL_SPSIPF);
     mbar_wait(&bar[s], (it / EL_SNS) & 1);
     const float* st = sm + s * L::SIZE;
     const int pt = ty * TXE + 2 * tx;
