@@ -43,6 +43,22 @@ constexpr int AC_NS = SEIS_AC_NS;    // P kernel ring depth
 #define SEIS_AC_LB(n) __launch_bounds__(n)
 #endif
 constexpr int AC_VNS = SEIS_AC_VNS;  // V kernel ring depth
+// L2 prefetch of the C-PML memory variables SEIS_AC_{V,P}PSIPF planes ahead (0 = off), one
+// lane per 128-byte slab line: x slab [nzl][ny][2W], y slab [nzl][2W][nx], z slab [2W][ny][nx]
+#ifndef SEIS_AC_VPSIPF
+#define SEIS_AC_VPSIPF 2  // ac_v 0.759 -> 0.741 ms at C2 (1: 0.745, 3: 0.743, 4: 0.746); ac_p: slower (0.553 vs 0.547), off (profiles/r02_ac_psipf.log)
+#endif
+#ifndef SEIS_AC_PPSIPF
+#define SEIS_AC_PPSIPF 0
+#endif
+__device__ __forceinline__ void ac_psi_prefetch(const float* px, const float* py, const float* pz, const Dims& d,
+                                                int W, int zlo, int tx, int x0, int j, bool lx, bool ly, int kk) {
+  if (kk >= d.nzl || (tx & 7) != 0) return;
+  if (lx) prefetch_l2(px + (kk * d.ny + j) * (2 * W) + (x0 < W ? 0 : W));
+  if (ly) prefetch_l2(py + (kk * (2 * W) + CpmlIdx::slot(j, d.ny, W)) * d.nx + x0);
+  const int gz = kk + d.z0;
+  if (CpmlIdx::in(gz, d.nz, W, zlo)) prefetch_l2(pz + (CpmlIdx::slot(gz, d.nz, W) * d.ny + j) * d.nx + x0);
+}
 
 struct AcVArgs {
   CUtensorMap mp;                 // p tile, box (64+8) x (BY+8) x 1
@@ -155,6 +171,8 @@ __global__ void SEIS_AC_LB(NTX * BY) ac_v_kernel(const __grid_constant__ AcVArgs
       psi_idx_row<4>(izz, (CpmlIdx::slot(gz, d.nz, Wl) * d.ny + j) * d.nx + x0, x0, d.nx);
       psi_ld<4>(oz, a.psz, izz);
     }
+    if (SEIS_AC_VPSIPF > 0 && Wl > 0 && own)
+      ac_psi_prefetch(a.psx, a.psy, a.psz, d, Wl, a.zlo, tx, x0, j, lx, ly, k + SEIS_AC_VPSIPF);
     mbar_wait(&bar[s], (it / AC_VNS) & 1);
     const float* st = sm + s * L::SIZE;
     r[7] = lds4(st + L::PQ + ty * TXV + 4 * tx);
@@ -373,6 +391,8 @@ __global__ void SEIS_AC_LB(NTX * BY) ac_p_kernel(const __grid_constant__ AcPArgs
       psi_idx_row<4>(izz, (CpmlIdx::slot(gz, d.nz, Wl) * d.ny + j) * d.nx + x0, x0, d.nx);
       psi_ld<4>(oz, a.pqz, izz);
     }
+    if (SEIS_AC_PPSIPF > 0 && Wl > 0 && own)
+      ac_psi_prefetch(a.pqx, a.pqy, a.pqz, d, Wl, a.zlo, tx, x0, j, lx, ly, k + SEIS_AC_PPSIPF);
     mbar_wait(&bar[s], ph);
     const float* st = sm + s * L::SIZE;
     q[7] = lds4(st + L::QQ + ty * TXV + 4 * tx);
