@@ -105,6 +105,11 @@ __device__ __forceinline__ int spml_idx(const Dims& d, int nb, int nxs, int nys,
 #ifndef SEIS_SPML_PF
 #define SEIS_SPML_PF 0
 #endif
+// (O6b) L2 prefetch of the layer components SEIS_SPML_PSIPF planes ahead (0 = off): one lane
+// per 8 (a 128-byte line of a y / z slab row), the group's first point
+#ifndef SEIS_SPML_PSIPF
+#define SEIS_SPML_PSIPF 1  // 0.715 -> 0.697 ms at 512^3 (70 % of HBM; 2: 0.697, 3: 0.699), profiles/r02_spml_psipf.log
+#endif
 constexpr int ISO_NS = SEIS_ISO_NS;
 
 template <int BY>
@@ -283,6 +288,16 @@ __global__ void __launch_bounds__(NTX * BY, SPML ? SEIS_SPML_MINB : 1) iso_step_
               wm[c][e] = nxt[c * a.spn + sidx[e]];
             }
           }
+      }
+    }
+    if (SPML && SEIS_SPML_PSIPF > 0 && own && (tx & 7) == 0 && k + SEIS_SPML_PSIPF < k1) {
+      const int kk = k + SEIS_SPML_PSIPF;
+      const float ezk = a.edx ? __ldg(a.edz + kk + d.z0) : 0.0f;
+      if (exv.v[0] != 0.0f || eyv != 0.0f || ezk != 0.0f) {
+        const int ix = spml_idx(d, a.nbl, a.nxs, a.nys, exv.v[0], eyv, x0, j, kk);
+#pragma unroll
+        for (int c = 0; c < 6; ++c)
+          prefetch_l2(a.sp + (long long)(c < 3 ? a.lvl : 1 - a.lvl) * 3 * a.spn + (c % 3) * a.spn + ix);
       }
     }
     mbar_wait(&bar[s], (it / ISO_NS) & 1);
