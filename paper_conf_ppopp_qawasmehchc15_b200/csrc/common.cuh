@@ -516,5 +516,43 @@ __device__ __forceinline__ void psi_upd(float* dv, float* __restrict__ ps, const
       dv[e] += v;
     }
 }
+// y / z slab rows: the group's NV values are contiguous (ix[e] = ix[0] + e); with the whole
+// group inside the grid and NV-aligned rows (vec: x0 + NV - 1 < nx, nx % NV == 0) one NV-wide
+// load / store instead of NV scalar ones (the same values, the same arithmetic)
+template <int NV>
+__device__ __forceinline__ void psi_ld_row(float* old, const float* __restrict__ ps, const int* ix, bool vec) {
+  static_assert(NV == 2 || NV == 4, "2- or 4-wide groups");
+  if (vec) {
+    if constexpr (NV == 4) {
+      const float4 t = *reinterpret_cast<const float4*>(ps + ix[0]);
+      old[0] = t.x;
+      old[1] = t.y;
+      old[2] = t.z;
+      old[3] = t.w;
+    } else {
+      const float2 t = *reinterpret_cast<const float2*>(ps + ix[0]);
+      old[0] = t.x;
+      old[1] = t.y;
+    }
+  } else {
+    psi_ld<NV>(old, ps, ix);
+  }
+}
+template <int NV>
+__device__ __forceinline__ void psi_upd_row(float* dv, float* __restrict__ ps, const int* ix, const float* old,
+                                            const float* ca, const float* cb, bool vec) {
+  if (vec) {
+    float v[NV];
+#pragma unroll
+    for (int e = 0; e < NV; ++e) {
+      v[e] = fmaf(cb[e], old[e], ca[e] * dv[e]);
+      dv[e] += v[e];
+    }
+    if constexpr (NV == 4) *reinterpret_cast<float4*>(ps + ix[0]) = make_float4(v[0], v[1], v[2], v[3]);
+    else *reinterpret_cast<float2*>(ps + ix[0]) = make_float2(v[0], v[1]);
+  } else {
+    psi_upd<NV>(dv, ps, ix, old, ca, cb);
+  }
+}
 
 }  // namespace seis

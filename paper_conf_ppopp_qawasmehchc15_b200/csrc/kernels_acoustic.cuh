@@ -330,6 +330,8 @@ __global__ void SEIS_AC_LB(NTX * BY) ac_p_kernel(const __grid_constant__ AcPArgs
   const int Wl = a.W;
   const bool lx = Wl > 0 && (x0 < Wl || x0 + 3 >= d.nx - Wl);
   const bool ly = Wl > 0 && CpmlIdx::in(j, d.ny, Wl, true);
+  const bool vec4 = (d.nx & 3) == 0 && x0 + 3 < d.nx;  // (y / z slab groups: one 16-byte access; in ac_p
+  // 0.5475 -> 0.545 ms at C2, in ac_v / el_v / el_s slower: profiles/r02_psi_vec_ab.log)
   auto issue = [&](int s, int k, bool pf = false) {
     float* st = sm + s * L::SIZE;
     const int z = k + GZ;
@@ -385,11 +387,11 @@ __global__ void SEIS_AC_LB(NTX * BY) ac_p_kernel(const __grid_constant__ AcPArgs
     }
     if (own && ly) {
       psi_idx_row<4>(iyy, (k * (2 * Wl) + CpmlIdx::slot(j, d.ny, Wl)) * d.nx + x0, x0, d.nx);
-      psi_ld<4>(oy, a.pqy, iyy);
+      psi_ld_row<4>(oy, a.pqy, iyy, vec4);
     }
     if (own && lz) {
       psi_idx_row<4>(izz, (CpmlIdx::slot(gz, d.nz, Wl) * d.ny + j) * d.nx + x0, x0, d.nx);
-      psi_ld<4>(oz, a.pqz, izz);
+      psi_ld_row<4>(oz, a.pqz, izz, vec4);
     }
     if (SEIS_AC_PPSIPF > 0 && Wl > 0 && own)
       ac_psi_prefetch(a.pqx, a.pqy, a.pqz, d, Wl, a.zlo, tx, x0, j, lx, ly, k + SEIS_AC_PPSIPF);
@@ -441,12 +443,12 @@ __global__ void SEIS_AC_LB(NTX * BY) ac_p_kernel(const __grid_constant__ AcPArgs
       if (ly) {
         const float ya = __ldg(a.cy.a + j), yb = __ldg(a.cy.b + j);
         const float ca[4] = {ya, ya, ya, ya}, cb[4] = {yb, yb, yb, yb};
-        psi_upd<4>(dy, a.pqy, iyy, oy, ca, cb);
+        psi_upd_row<4>(dy, a.pqy, iyy, oy, ca, cb, vec4);
       }
       if (lz) {
         const float za = __ldg(a.cz.a + gz), zb = __ldg(a.cz.b + gz);
         const float ca[4] = {za, za, za, za}, cb[4] = {zb, zb, zb, zb};
-        psi_upd<4>(dz, a.pqz, izz, oz, ca, cb);
+        psi_upd_row<4>(dz, a.pqz, izz, oz, ca, cb, vec4);
       }
       const int pt = ty * TXV + 4 * tx;
       const F4 pv = lds4(st + L::P + pt), kv = lds4(st + L::K + pt);
